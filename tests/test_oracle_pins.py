@@ -340,12 +340,12 @@ def test_injection_first_push(c1_mesh):
 def test_walk_tie_takes_lowest_index():
     """S2: on a tie for the most negative lambda the lowest local index wins.
     In tet 0 of hex 0 (path 0 -> e_x -> e_x+e_y -> 111) the closed-form
-    coordinates of f = (0.3, 0.5, 0.7) are (1-f_x, f_x-f_y, f_y-f_z, f_z) =
-    (0.7, -0.2, -0.2, 0.7): local faces 1 and 2 tie; one capped hop must cross
+    coordinates of f = (0.25, 0.5, 0.75) are (1-f_x, f_x-f_y, f_y-f_z, f_z) =
+    (0.75, -0.25, -0.25, 0.75): local faces 1 and 2 tie; one capped hop must cross
     face 1."""
     mesh = gen.kuhn_duct(2, 2, 2)
     om = oracle.Mesh.from_gen(mesh)
-    x = np.array([0.3, 0.5, 0.7])
+    x = np.array([0.25, 0.5, 0.75])
     lam = om.bary(0, x)
     assert lam[1] == lam[2] < 0
     st, fc, hops, lam2, cap = om.walk(0, x, hcap=1)
