@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""bench.py -- particle-steps/s of the fused OP-PIC particle loop on B200.
+
+One step = one pass of the whole hot path over the resident
+particle population: inject (a1) -> zero node charge (a2) -> gather E + push
+(a3, a4) -> multi-hop walk (a6, optionally DH-seeded a5) -> deposit (a7) ->
+write-back / holes (a8) -> hole fill (a9).  Default workload = config C2
+(BASELINE.json configs[1]): 48x48x72 Kuhn duct (995,328 tets), a pre-seeded
+50M-particle steady state plus 250k injected per step, fixed uniform field (the
+CG field solve is timed separately in the paper's plan and is not built yet).
+
+Contract: W untimed warm-up steps, then exactly K timed steps bracketed by a
+barrier + cuda synchronize; CUDA events on the library's stream; max over
+ranks; rank 0 prints ONE JSON line.  --impl reference times the CPU oracle
+(oracle/, single thread) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "particle-steps/sec (push+move+deposit) at 1/2/4/8 B200; % of HBM roofline"
+UNIT = "particle-steps/s"
+DEP_NAMES = {0: "atomic", 1: "atomic_warpagg", 2: "sort_segred"}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c2", choices=["c2", "c5", "c1"])
+    ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
+    ap.add_argument("--deposit", type=int, default=0, choices=[0, 1, 2])
+    ap.add_argument("--dh", action="store_true")
+    ap.add_argument("--hpass", type=int, default=4)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=0)
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------- workload
+def workload(args):
+    import gen
+    cfg = dict(gen.CONFIGS[args.config])
+    if args.n0:
+        cfg["n0"] = args.n0
+    nx, ny, nz = cfg["dims"]
+    mesh = gen.kuhn_duct(nx, ny, nz)
+    c1E = np.array(cfg["c1E"])
+    qm, dt = 1.0, cfg["dt"]
+    ef = np.tile(c1E / (qm * dt), (mesh["n_cells"], 1))
+    cluster = None
+    if cfg.get("cluster"):
+        cluster = (cfg["cluster"], gen.hot_block_cells(mesh))
+    name = {"c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
+                  "+ 250k injected/step, fixed uniform E",
+            "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
+            "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
+    return cfg, mesh, ef, qm, dt, cluster, name
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:   # noqa: BLE001
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:   # noqa: BLE001
+            self.proc = None
+        time.sleep(0.15)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:   # noqa: BLE001
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for k, nm in enumerate(names):
+                if len(r) > 4 + k and r[4 + k].lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+# ---------------------------------------------------------------- oracle legs
+def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload."""
+    import gen
+    import oracle
+    om = oracle.Mesh.from_gen(mesh)
+    om.set_field(ef)
+    P = oracle.Particles()
+    init = gen.seed_particles(mesh, n_sample, cfg["seed"], cluster=cluster)
+    P.append(init["pos"], init["vel"], init["cell"], init["id"])
+    Q = np.zeros(mesh["n_nodes"])
+    scale = n_sample / max(cfg["n0"], 1)
+    n_inj = int(round(cfg["n_inj"] * scale))
+    pushed, secs = 0, 0.0
+    for s in range(steps):
+        if n_inj:
+            b = gen.inject_batch(mesh, s, n_inj, cfg["seed"], id_base=cfg["n0"])
+            t0 = time.perf_counter()
+            P.append(b["pos"], b["vel"], b["cell"], b["id"])
+        else:
+            t0 = time.perf_counter()
+        st = oracle.step(om, P, qm * dt, dt, w, Q)
+        secs += time.perf_counter() - t0
+        pushed += st["n_before"]
+    return pushed, secs, n_inj
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    cfg, mesh, ef, qm, dt, cluster, name = workload(args)
+    w = cfg["w"]
+    n_sample = 400_000 if args.config != "c1" else cfg["n0"]
+    # warm-up steps are run and discarded, then K timed sample-steps
+    oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, max(args.warmup, 0) and 1, cluster)
+    pushed, secs, n_inj = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, args.steps, cluster)
+    v = pushed / secs
+    sample = (f"{n_sample:,} particles of the {args.config.upper()} workload "
+              f"(+{n_inj:,} injected/step), {args.steps} steps, 1 thread")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * secs / max(args.steps, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": name, "sample": sample},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def run_ours(args, rank, world):
+    import torch
+    import gen
+    import gen.cuda as gc
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+
+    if world > 1:
+        raise SystemExit("multi-GPU slab migration is not built yet (DESIGN.md §7)")
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(dev)
+    cfg, mesh, ef, qm, dt, cluster, name = workload(args)
+    w, n0, n_inj, seed = cfg["w"], cfg["n0"], cfg["n_inj"], cfg["seed"]
+    stream = torch.cuda.current_stream()
+    dm = gc.DeviceMesh(mesh)
+    total = args.warmup + args.steps
+    cap = int(n0 * 1.05) + n_inj * (total + 4) + 1024
+    sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
+                     direct_hop=args.dh, overlay_spacing=0.5, hop_budget=args.hpass)
+    init = gc.seed_particles(dm, n0, seed, cluster=cluster)
+    sim.inject(init, on_device=True)
+    torch.cuda.synchronize()
+    del init
+    batches = [gc.inject_batch(dm, s, n_inj, seed, id_base=n0) if n_inj else None
+               for s in range(total)]
+    torch.cuda.synchronize()
+
+    def one_step(s, on_device=True, readback=None):
+        if batches[s] is not None:
+            sim.inject(batches[s] if on_device else host_batches[s], on_device=on_device)
+        sim.step(dt, qm, w, stats=False, fill=True)
+        if readback is not None:
+            readback()
+
+    for s in range(args.warmup):
+        one_step(s)
+    torch.cuda.synchronize()
+    st0 = sim.last_stats()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    l0 = sim.launches()
+    sim.phase_timing(True)
+    sim.phase_times()  # reset
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(dev) as clk:
+        e0.record(stream)
+        for s in range(args.warmup, total):
+            one_step(s)
+        e1.record(stream)
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    launches = sim.launches() - l0
+    phases = sim.phase_times()
+    sim.phase_timing(False)
+    st1 = sim.last_stats()
+    pushed = st1["cum_pushed"] - st0["cum_pushed"]
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+        p = torch.tensor([pushed], device="cuda", dtype=torch.int64)
+        torch.distributed.all_reduce(p)
+        pushed = int(p.item())
+    value = pushed / (ms / 1e3)
+    n_avg = pushed / args.steps
+
+    # ---- roofline of the dominant kernel (k_push_move_deposit, pass 1)
+    peak, peak_src = load_peaks()
+    pmd_ms, pmd_cnt = phases["push_move_deposit"]
+    nc, nn = mesh["n_cells"], mesh["n_nodes"]
+    bytes_per_launch = 104.0 * n_avg + 160.0 * nc + 16.0 * nn
+    achieved = bytes_per_launch / (pmd_ms / max(pmd_cnt, 1) / 1e3) / 1e9
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tf):
+        try:
+            with open(tf) as f:
+                tj = json.load(f)
+            key = f"{args.config}_dep{args.deposit}_dh{int(args.dh)}"
+            traffic = tj.get(key)
+        except Exception:   # noqa: BLE001
+            traffic = None
+    # whole-step model bytes (SURVEY.md §8(d) B_ps)
+    f_inj = n_inj / max(n_avg, 1)
+    f_rem = (st1["cum_pushed"] and 0) or 0
+    b_ps = 104.0 + (160.0 * nc + 16.0 * nn) / max(n_avg, 1) + 60.0 * f_inj
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": name, "mesh_cells": nc, "mesh_nodes": nn,
+                   "particles_seeded": n0, "inject_per_step": n_inj,
+                   "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
+                   "walk": "DH+MH" if args.dh else "MH", "hop_budget_per_pass": args.hpass,
+                   "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n_avg * 60 / 1e9),
+                   "parallelism": f"slab{world}"},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "kernel": "k_push_move_deposit (pass 1)",
+                     "bytes_model": "104 B/particle + 160 B/cell + 16 B/node per launch",
+                     "peak_source": peak_src,
+                     "step_frac": b_ps * value / (peak * 1e9), "step_bytes_per_particle": b_ps},
+        "gpu_launches": launches,
+        "phases_ms_per_step": {k: v[0] / args.steps for k, v in phases.items() if v[1]},
+        "walk": {"hops_per_particle_last_step": st1["total_hops"] / max(st1["n_before"], 1),
+                 "max_hops_last_step": st1["max_hops"], "hop_capped": st1["n_hop_capped"],
+                 "deferred_last_step": st1["n_deferred"]},
+        "clocks": clk.summary(),
+    }
+
+    # ---- e2e: same metric through the C ABI with HOST buffers
+    if not args.no_e2e:
+        ke = args.e2e_steps or min(args.steps, 10)
+        global host_batches
+        host_batches = [None] * total
+        for s in range(args.warmup, args.warmup + ke):
+            b = batches[s]
+            if b is not None:
+                host_batches[s] = {k: b[k].cpu().pin_memory().numpy() for k in ("pos", "vel", "cell", "id")}
+        q_host = torch.empty(nn, dtype=torch.float64).pin_memory().numpy()
+        from paper_conf_icpp_lantra0m24_b200 import opp as O
+        # rewind is impossible (state advanced); e2e continues the same run
+        torch.cuda.synchronize()
+        s0 = sim.last_stats()
+        e0.record(stream)
+        for s in range(args.warmup, args.warmup + ke):
+            one_step(s, on_device=False,
+                     readback=lambda: O.opp_get_node_charge(sim.ctx, sim.node_charge, q_host))
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        s1 = sim.last_stats()
+        epushed = s1["cum_pushed"] - s0["cum_pushed"]
+        line["e2e"] = {"value": epushed / (ems / 1e3), "unit": UNIT,
+                       "h2d_bytes_per_step": n_inj * 60, "d2h_bytes_per_step": nn * 8,
+                       "steps": ke, "note": "injection arrays from pinned host memory (opp_inject "
+                       "on_device=0) + node charge read back every step (opp_get_node_charge)"}
+
+    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1)
+    if not args.no_cpu and world == 1 and rank == 0:
+        n_sample = 300_000 if args.config != "c1" else cfg["n0"]
+        pushed_c, secs, ninj_c = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, 3, cluster)
+        line["cpu_baseline"] = {"value": pushed_c / secs, "unit": UNIT, "cores": 1,
+                                "kind": "oracle",
+                                "sample": f"{n_sample:,} particles of the same workload "
+                                          f"(+{ninj_c:,} injected/step), 3 steps, 1 thread, "
+                                          f"{secs:.1f} s"}
+    sim.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        if args.impl == "ours":
+            torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", 0)))
+            dist.init_process_group("nccl")
+        else:
+            dist.init_process_group("gloo")
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+    else:
+        run_ours(args, rank, world)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

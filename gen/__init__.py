@@ -193,7 +193,9 @@ def seed_particles(mesh: dict, n: int, seed: int, drift: float = 0.25,
     s.sort(axis=1)
     b = np.stack([s[:, 0], s[:, 1] - s[:, 0], s[:, 2] - s[:, 1], 1.0 - s[:, 2]], 1)
     p = mesh["node_xyz"][mesh["c2n"][cell]]               # (n,4,3)
-    pos = np.einsum("nk,nkd->nd", b, p)
+    # explicit left-to-right sum (no BLAS / einsum reordering): the device
+    # generator (gen/gen_cuda.cu) reproduces it bit for bit
+    pos = b[:, 0:1] * p[:, 0] + b[:, 1:2] * p[:, 1] + b[:, 2:3] * p[:, 2] + b[:, 3:4] * p[:, 3]
     vel = np.stack([(2.0 * u01(seed, STREAM_VEL, idx * np.uint64(3) + np.uint64(a)) - 1.0) * spread
                     for a in range(3)], 1)
     vel[:, 2] += drift

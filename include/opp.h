@@ -1,0 +1,257 @@
+/*
+ * opp.h -- C ABI of the B200-native OP-PIC particle-loop library (libopp.so).
+ *
+ * The library implements the one data-parallel hot path of OP-PIC's
+ * unstructured-mesh PIC method (Lantra, Wright, Mudalige, ICPP '24): the
+ * per-timestep electrostatic particle loop on a tetrahedral mesh --
+ * inject, gather the cell field, leap-frog push, multi-hop / direct-hop cell
+ * walk, charge deposit to the cell's 4 nodes, hole-filling compaction, and
+ * (nranks > 1) slab migration and node-charge halo over NCCL.
+ * Citations are PAPER.md line ranges (section / figure / equation).
+ *
+ * Conventions (all entry points):
+ *  - Every function returns an opp_status (0 = OPP_OK, < 0 = error) unless
+ *    stated otherwise; on error opp_last_error() returns a thread-local
+ *    message.  A failing call leaves the context unchanged, except that an
+ *    asynchronous CUDA/NCCL failure is sticky and reported by the next call.
+ *  - Handles (opp_set, opp_map, opp_dat) are small integers valid for the
+ *    lifetime of the context that issued them.
+ *  - Host pointers passed to opp_decl_* / opp_inject(on_device = 0) are read
+ *    during the call (or, for opp_inject, before the call's stream work
+ *    completes if the memory is pinned: keep it alive until the next
+ *    synchronising call); the library copies, the caller keeps ownership.
+ *    Device pointers (on_device = 1) must be valid device memory of
+ *    params.device, ordered before the call on params.cuda_stream.
+ *  - All work is enqueued on params.cuda_stream.  Calls that return data to
+ *    the host (opp_get_*, opp_push_move_deposit with stats != NULL,
+ *    opp_fill_holes with n_after != NULL) synchronise that stream.
+ *  - Layouts: mesh dats are stored AoS ([n][dim], "dim" contiguous);
+ *    particle dats and the particle->cell map are stored SoA on the device
+ *    ([dim][capacity]) for coalesced per-component streaming.  Host-side
+ *    arrays exchanged through this ABI are always AoS [n][dim].
+ *  - One host thread per context; one context (process) per GPU.
+ */
+#ifndef OPP_H
+#define OPP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct opp_ctx_s *opp_ctx;
+typedef int32_t opp_set;
+typedef int32_t opp_map;
+typedef int32_t opp_dat;
+
+enum opp_status {
+    OPP_OK = 0,
+    OPP_ERR_ARG = -1,      /* bad handle, size, type or pointer            */
+    OPP_ERR_STATE = -2,    /* call not valid now (e.g. dats contain holes) */
+    OPP_ERR_NOMEM = -3,    /* device / host allocation failed              */
+    OPP_ERR_CAPACITY = -4, /* particle capacity exceeded, growth disabled  */
+    OPP_ERR_CUDA = -5,     /* CUDA runtime / kernel error                  */
+    OPP_ERR_NCCL = -6,     /* NCCL error, or NCCL not available            */
+    OPP_ERR_MESH = -7      /* invalid mesh: non-positive tet, bad c2c      */
+};
+
+/* opp_decl_dat types (Fig. 4: OPP_REAL ...) */
+enum opp_type { OPP_REAL = 0 /* fp64 */, OPP_INT = 1 /* int32 */, OPP_INT64 = 2 };
+
+/* Per-particle move status (Fig. 6; 1336-1340 "marked
+ * for communication" -> NEED_MIGRATE). */
+enum opp_move_status { OPP_MOVE_DONE = 0, OPP_NEED_MOVE = 1, OPP_NEED_REMOVE = 2,
+                       OPP_NEED_MIGRATE = 3 };
+
+/* Deposit race handling (§3.3 and Fig. 3):
+ * ATOMIC        one fp64 atomic add per (particle, node)              ("AT")
+ * ATOMIC_WARPAGG same-node contributions of a warp summed by shuffles
+ *                before one atomic per distinct node
+ * SORT_SEGRED   store (cell, w*lambda[4]) per particle, counting-sort by
+ *                cell, reduce per cell, then per node               ("SR")
+ * AUTO          library choice (currently ATOMIC)      */
+enum opp_deposit_mode { OPP_DEP_ATOMIC = 0, OPP_DEP_ATOMIC_WARPAGG = 1,
+                        OPP_DEP_SORT_SEGRED = 2, OPP_DEP_AUTO = 3 };
+
+typedef void *(*opp_alloc_fn)(size_t bytes, void *cuda_stream, void *user);
+typedef void (*opp_free_fn)(void *ptr, size_t bytes, void *cuda_stream, void *user);
+
+typedef struct {
+    int device;                 /* CUDA device ordinal                               */
+    void *cuda_stream;          /* cudaStream_t; NULL = the legacy default stream    */
+    int rank, nranks;           /* slab partition index / count (nranks >= 1)        */
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId, required iff nranks > 1    */
+    opp_alloc_fn alloc;         /* optional device allocator (e.g. torch's caching   */
+    opp_free_fn free;           /*  allocator); NULL = cudaMalloc / cudaFree         */
+    void *alloc_user;
+    int deposit_mode;           /* enum opp_deposit_mode                             */
+    int direct_hop;             /* 1 = seed the walk from the DH overlay (1356-1370) */
+    double overlay_spacing;     /* DH overlay cell size (mesh units); <= 0: auto     */
+    int hop_budget_per_pass;    /* H_pass: hops in the fused kernel before a particle
+                                   is deferred to the continuation pass (>= 1)      */
+    int hop_cap;                /* H_cap: hops after which the current cell is
+                                   accepted as final and counted (S4)               */
+    int allow_growth;           /* 1 = grow particle capacity x1.5 on injection     */
+} opp_init_params;
+
+/* Per-step arguments of opp_push_move_deposit. */
+typedef struct {
+    double dt;          /* time step                                                */
+    double qm;          /* charge / mass; the push uses c1 = qm * dt (one host mult) */
+    double weight;      /* macro-particle charge Q_p of Eq. 10   */
+    int zero_charge;    /* 1 = node charge := 0 before depositing                   */
+    int fill_inline;    /* 1 = also run the hole fill (opp_fill_holes) in this call */
+} opp_step_params;
+
+/* Step statistics (filled when a stats pointer is given; one D2H copy). */
+typedef struct {
+    int64_t n_before;       /* particles entering the push (incl. injected)   */
+    int64_t n_injected;     /* injected since the previous push               */
+    int64_t n_removed;      /* left through a boundary face (NEED_REMOVE)     */
+    int64_t n_after;        /* n_before - n_removed - migrated out + in        */
+    int64_t n_migrated_out, n_migrated_in;
+    int64_t total_hops;     /* sum over particles of cell hops this step      */
+    int64_t n_hop_capped;   /* walks stopped by H_cap (must be 0 on valid meshes) */
+    int64_t n_deferred;     /* particles handed to the continuation pass      */
+    int32_t max_hops;
+    int32_t migrate_rounds;
+    int64_t cum_pushed;     /* sum of n_before over every step of this set so far */
+    int64_t cum_steps;      /* number of steps of this set so far              */
+} opp_step_stats;
+
+/* Fill *p with defaults: device 0, default stream, 1 rank, cudaMalloc,
+ * OPP_DEP_ATOMIC, MH only, overlay_spacing 0 (auto = 0.5 * mean edge),
+ * H_pass = 4, H_cap = 1024, growth allowed. */
+void opp_init_params_default(opp_init_params *p);
+
+/* Create a context on params->device (nranks > 1: joins the NCCL clique). */
+int opp_init(const opp_init_params *params, opp_ctx *out);
+/* Free every device allocation and the NCCL communicator. */
+int opp_finalize(opp_ctx ctx);
+
+/* Rank 0 calls this and broadcasts the 128 bytes (e.g. via torch.distributed);
+ * returns OPP_ERR_NCCL if the library was built without NCCL. */
+int opp_get_nccl_unique_id(void *out128);
+
+/* opp_decl_set (Fig. 4 l.2-3): a mesh set of `size` elements. */
+int opp_decl_set(opp_ctx ctx, int64_t size, const char *name, opp_set *out);
+
+/* opp_decl_particle_set (Fig. 4 l.6-7): a particle set
+ * living on mesh set `cells` with n_init particles whose data follow in
+ * opp_decl_dat / opp_decl_map; `capacity` (>= n_init, 0 = auto) is the
+ * initial allocation. */
+int opp_decl_particle_set(opp_ctx ctx, const char *name, opp_set cells, int64_t n_init,
+                          int64_t capacity, opp_set *out);
+
+/* opp_decl_map (Fig. 4 l.12-15): `dim` int32
+ * entries per element of `from` pointing into `to` (-1 = none).
+ * Mesh maps: c2n (dim 4) and c2c (dim 4; c2c[c][i] = the cell across the
+ * face opposite local node c2n[c][i], -1 = domain boundary; validated,
+ * OPP_ERR_MESH otherwise).  Particle maps: p2c (dim 1, from a particle set);
+ * host may be NULL iff the set has n_init == 0.  Global
+ * cell ids when nranks > 1. */
+int opp_decl_map(opp_ctx ctx, opp_set from, opp_set to, int dim, const int32_t *host,
+                 const char *name, opp_map *out);
+
+/* opp_decl_dat (Fig. 4 l.20-30): `dim` values of
+ * `type` per element of `set`, initialised from host (AoS [n][dim]) or zero
+ * if host == NULL (NULL allowed for node/cell dats and empty particle sets). */
+int opp_decl_dat(opp_ctx ctx, opp_set set, int dim, int type, const void *host,
+                 const char *name, opp_dat *out);
+
+/* Slab partition (the user provides the rank of one set
+ * "via an opp_dat"): rank_of_cell[c] for every global cell; each rank's cells
+ * must form one contiguous global range. */
+int opp_set_partition(opp_ctx ctx, opp_set cells, const int32_t *rank_of_cell);
+
+/* opp_inject (PAPER.md:1014-1018 OPP_ITERATE_INJECTED, 1502-1508): append n
+ * particles at [N, N+n).  cols lists EVERY particle dat / the p2c map of the
+ * set (any order) and data[k] points to that column's n*dim values (AoS),
+ * host (on_device = 0, copied H2D on the stream; pinned memory makes it
+ * asynchronous) or device (on_device = 1).  Grows capacity if needed. */
+int opp_inject(opp_ctx ctx, opp_set parts, int64_t n, int ncols, const int32_t *cols,
+               const void *const *data, int on_device);
+
+/* The fused electrostatic particle loop -- one time step (PAPER.md:398-410
+ * Fig. 1 steps 2-4; CalcPosVel + Move + DepositCharge of 1586-1604):
+ *   [zero node_charge]
+ *   for every particle p (any order):
+ *     E = cell_ef[p2c[p]]                      (cell-constant, 1576-1585)
+ *     v += (qm*dt) * E ; x += v * dt           (leap-frog, 569-583)
+ *     [DH] seed cell from the overlay          (1356-1370)
+ *     walk: lambda = barycentric(x, cell); inside iff all lambda in [0,1];
+ *           else cross the face opposite argmin lambda via c2c (595-603);
+ *           -1 -> NEED_REMOVE (1508-1510); H_cap -> accept (S4)
+ *     DONE: node_charge[c2n[cell][i]] += weight * lambda_i   (Eq. 10, 637-660)
+ *     NEED_REMOVE: recorded as a hole (filled by opp_fill_holes)
+ *   nranks > 1: migrants exchanged over NCCL until no rank has any; then the
+ *   interface-node charge halo is summed (1280-1300, 1336-1354).
+ * pos, vel: particle dats dim 3 OPP_REAL; p2c: particle map dim 1;
+ * c2c, c2n: cell maps dim 4; node_pos: node dat dim 3 OPP_REAL;
+ * cell_ef: cell dat dim 3 OPP_REAL; node_charge: node dat dim 1 OPP_REAL.
+ * Between this call and opp_fill_holes the particle dats contain holes
+ * (opp_get_dat returns OPP_ERR_STATE) unless params->fill_inline.
+ * stats may be NULL (no host synchronisation). */
+int opp_push_move_deposit(opp_ctx ctx, opp_set parts, opp_dat pos, opp_dat vel, opp_map p2c,
+                          opp_map c2c, opp_map c2n, opp_dat node_pos, opp_dat cell_ef,
+                          opp_dat node_charge, const opp_step_params *params,
+                          opp_step_stats *stats);
+
+/* Statistics of the most recent opp_push_move_deposit on `parts` (and the
+ * cumulative counters); synchronises.  Lets a caller run steps with
+ * stats == NULL (no host round trip) and read the numbers afterwards. */
+int opp_get_step_stats(opp_ctx ctx, opp_set parts, opp_step_stats *stats);
+
+/* Hole filling ("shifting data from the end of the
+ * opp_dats to fill the holes"): survivors at index >= N' = N - R move into the
+ * holes below N'.  Particle order afterwards is implementation-defined.
+ * n_after may be NULL (no host synchronisation). */
+int opp_fill_holes(opp_ctx ctx, opp_set parts, int64_t *n_after);
+
+/* Copy node charge (dim 1) to host_out[n]; synchronises. */
+int opp_get_node_charge(opp_ctx ctx, opp_dat node_charge, double *host_out, int64_t n);
+
+/* Copy the first n_elems elements of any dat or map to host (AoS); for
+ * particle sets n_elems must equal the current count.  Synchronises. */
+int opp_get_dat(opp_ctx ctx, int32_t dat_or_map, void *host_out, int64_t n_elems);
+
+/* Overwrite the first n_elems elements of a dat (AoS source, host or device),
+ * e.g. the per-step cell field.  Mesh maps are static. */
+int opp_set_dat(opp_ctx ctx, opp_dat dat, const void *src, int64_t n_elems, int on_device);
+
+/* Current particle count (synchronises). */
+int opp_get_particle_count(opp_ctx ctx, opp_set parts, int64_t *n);
+
+/* Device pointer + row stride (elements) of a dat/map column, for zero-copy
+ * interop (read-only use); SoA for particle sets. */
+int opp_get_dat_device_ptr(opp_ctx ctx, int32_t dat_or_map, void **ptr, int64_t *stride);
+
+/* Phases of the step timed by opp_phase_timing (indices into ms_sum / count). */
+enum opp_phase { OPP_PH_INJECT = 0, OPP_PH_BEGIN = 1, OPP_PH_PUSH_MOVE_DEPOSIT = 2,
+                 OPP_PH_CONTINUE = 3, OPP_PH_SEGRED = 4, OPP_PH_FILL = 5, OPP_PH_MIGRATE = 6,
+                 OPP_PH_HALO = 7, OPP_N_PHASES = 8 };
+
+/* enable != 0: record CUDA events on the context stream around every phase
+ * of the following calls (negligible overhead, no host synchronisation). */
+int opp_phase_timing(opp_ctx ctx, int enable);
+
+/* Sum of the recorded device time per phase (ms_sum[OPP_N_PHASES]) and the
+ * number of recorded instances (count[OPP_N_PHASES]) since timing was
+ * enabled or last read; synchronises, then resets the records. */
+int opp_get_phase_times(opp_ctx ctx, double *ms_sum, int64_t *count);
+
+/* Number of kernels this context has launched so far (evidence counter). */
+int64_t opp_kernel_launch_count(opp_ctx ctx);
+
+/* Synchronise the context's stream; reports sticky asynchronous errors. */
+int opp_sync(opp_ctx ctx);
+
+/* Thread-local message describing the last error. */
+const char *opp_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OPP_H */

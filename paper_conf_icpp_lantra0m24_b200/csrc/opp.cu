@@ -1,0 +1,990 @@
+// opp.cu -- host side of libopp: the C ABI declared in include/opp.h.
+//
+// Owns handles, device allocations, the stream, the device-resident counters
+// and the derived mesh data (walk lines, padded cell field, DH overlay, SR
+// node->cell CSR).  Every computation of the particle loop runs in the
+// kernels of opp_kernels.cu; this file only validates arguments, sizes grids
+// and enqueues work.
+#include "opp.h"
+#include "opp_internal.h"
+#include "opp_kernels.h"
+#include "opp_comm.h"
+
+#include <algorithm>
+#include <cstdarg>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+using namespace opp;
+
+static thread_local std::string g_err;
+
+static int fail(int code, const char *fmt, ...) __attribute__((format(printf, 2, 3)));
+static int fail(int code, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CK(call)                                                                               \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess)                                                                 \
+            return fail(OPP_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,               \
+                        cudaGetErrorString(e_));                                               \
+    } while (0)
+
+#define TRY(call)                 \
+    do {                          \
+        int r_ = (call);          \
+        if (r_ != OPP_OK) return r_; \
+    } while (0)
+
+namespace {
+
+struct Col {
+    bool is_map = false;
+    int set = -1, to = -1, dim = 0, type = 0, eb = 0;
+    std::string name;
+    char *d = nullptr;          // device storage
+    size_t bytes = 0;
+    std::vector<char> host;     // mesh columns: host copy (validation, bbox)
+    uint64_t version = 0;
+};
+
+struct PSet {
+    DevCounters *dcnt = nullptr;
+    long long cap = 0;
+    long long n_ub = 0;          // upper bound of the device count
+    bool n_exact = true;
+    bool holes_pending = false;
+    bool growth = true;
+    uint32_t *holes = nullptr, *work = nullptr, *head = nullptr, *tail = nullptr;
+    int32_t *work_hops = nullptr;
+    int32_t *sr_cell = nullptr;
+    double *sr_val = nullptr;
+    char *staging = nullptr;
+    size_t staging_bytes = 0;
+    std::vector<int> cols;
+};
+
+struct Set {
+    std::string name;
+    long long size = 0;
+    bool particle = false;
+    int cells = -1;
+    int pset = -1;
+};
+
+struct MeshCache {
+    int c2c = -1, c2n = -1, node_pos = -1;
+    uint64_t vpos = ~0ull;
+    WalkLine *lines = nullptr;
+    long long nc = 0;
+    int ef = -1;
+    uint64_t vef = ~0ull;
+    double4 *efp = nullptr;
+    // overlay
+    bool ov_built = false;
+    Overlay ov{};
+    int32_t *ov_map = nullptr;
+    // SR
+    unsigned *sr_hist = nullptr, *sr_start = nullptr;
+    double *sr_sorted = nullptr, *sr_cellsum = nullptr;
+    int32_t *n2cs_ptr = nullptr, *n2cs = nullptr;
+    long long sr_cap = 0;
+};
+
+}  // namespace
+
+struct opp_ctx_s {
+    opp_init_params p{};
+    cudaStream_t s = nullptr;
+    int nsm = 148;
+    int bps = 0;                   // resident blocks / SM of the fused kernel
+    std::vector<Set> sets;
+    std::vector<Col> cols;
+    std::vector<PSet> psets;
+    MeshCache mc;
+    DevCounters *hcnt = nullptr;   // pinned mirror
+    long long launches = 0;
+    int cell_base = 0;             // global id of local cell 0 (slab partition)
+    long long cells_global = -1;
+    std::vector<int32_t> rank_of_cell;
+    opp::Comm *comm = nullptr;
+    // phase timing (opp_phase_timing)
+    bool timing = false;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    std::vector<int> ev_phase;   // phase of record k (events 2k, 2k+1)
+
+    cudaEvent_t next_event() {
+        if (ev_used == ev_pool.size()) {
+            cudaEvent_t e;
+            if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+            ev_pool.push_back(e);
+        }
+        return ev_pool[ev_used++];
+    }
+
+    void *dalloc(size_t bytes) {
+        if (bytes == 0) bytes = 16;
+        if (p.alloc) return p.alloc(bytes, (void *)s, p.alloc_user);
+        void *ptr = nullptr;
+        if (cudaMalloc(&ptr, bytes) != cudaSuccess) return nullptr;
+        return ptr;
+    }
+    void dfree(void *ptr, size_t bytes) {
+        if (!ptr) return;
+        if (p.free) p.free(ptr, bytes, (void *)s, p.alloc_user);
+        else cudaFree(ptr);
+    }
+};
+
+static int type_bytes(int t) { return t == OPP_REAL ? 8 : t == OPP_INT ? 4 : t == OPP_INT64 ? 8 : 0; }
+
+static int ctx_check(opp_ctx c) {
+    if (!c) return fail(OPP_ERR_ARG, "null context");
+    cudaError_t e = cudaSetDevice(c->p.device);
+    if (e != cudaSuccess) return fail(OPP_ERR_CUDA, "cudaSetDevice: %s", cudaGetErrorString(e));
+    return OPP_OK;
+}
+
+static int set_check(opp_ctx c, opp_set s) {
+    if (s < 0 || s >= (int)c->sets.size()) return fail(OPP_ERR_ARG, "bad set handle %d", s);
+    return OPP_OK;
+}
+
+static int col_check(opp_ctx c, int h) {
+    if (h < 0 || h >= (int)c->cols.size()) return fail(OPP_ERR_ARG, "bad dat/map handle %d", h);
+    return OPP_OK;
+}
+
+static int grid_for(opp_ctx c, long long n, int cap_mult = 8) {
+    long long g = (n + 255) / 256;
+    long long cap = (long long)c->nsm * cap_mult;
+    if (g > cap) g = cap;
+    if (g < 1) g = 1;
+    return (int)g;
+}
+
+// Records a start/end event pair around one phase when timing is enabled.
+struct PhaseScope {
+    opp_ctx c;
+    cudaEvent_t end = nullptr;
+    PhaseScope(opp_ctx c_, int phase) : c(c_) {
+        if (!c->timing) return;
+        cudaEvent_t b = c->next_event();
+        end = c->next_event();
+        if (!b || !end) { end = nullptr; return; }
+        cudaEventRecord(b, c->s);
+        c->ev_phase.push_back(phase);
+    }
+    ~PhaseScope() {
+        if (end) cudaEventRecord(end, c->s);
+    }
+};
+
+// ---------------------------------------------------------------------------
+extern "C" void opp_init_params_default(opp_init_params *p) {
+    std::memset(p, 0, sizeof *p);
+    p->device = 0;
+    p->nranks = 1;
+    p->deposit_mode = OPP_DEP_ATOMIC;
+    p->hop_budget_per_pass = 4;
+    p->hop_cap = 1024;
+    p->allow_growth = 1;
+}
+
+extern "C" const char *opp_last_error(void) { return g_err.c_str(); }
+
+extern "C" int opp_get_nccl_unique_id(void *out128) { return opp::comm_unique_id(out128, g_err); }
+
+extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
+    if (!params || !out) return fail(OPP_ERR_ARG, "null argument");
+    if (params->nranks < 1 || params->rank < 0 || params->rank >= params->nranks)
+        return fail(OPP_ERR_ARG, "bad rank/nranks %d/%d", params->rank, params->nranks);
+    if (params->hop_budget_per_pass < 1 || params->hop_cap < 0)
+        return fail(OPP_ERR_ARG, "hop_budget_per_pass must be >= 1 and hop_cap >= 0");
+    if (params->deposit_mode < 0 || params->deposit_mode > OPP_DEP_AUTO)
+        return fail(OPP_ERR_ARG, "bad deposit_mode %d", params->deposit_mode);
+    if ((params->alloc == nullptr) != (params->free == nullptr))
+        return fail(OPP_ERR_ARG, "alloc and free callbacks go together");
+    CK(cudaSetDevice(params->device));
+    opp_ctx c = new opp_ctx_s();
+    c->p = *params;
+    if (c->p.deposit_mode == OPP_DEP_AUTO) c->p.deposit_mode = OPP_DEP_ATOMIC;
+    c->s = (cudaStream_t)params->cuda_stream;
+    cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, params->device);
+    if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
+        delete c;
+        return fail(OPP_ERR_NOMEM, "cudaMallocHost");
+    }
+    if (params->nranks > 1) {
+        int r = opp::comm_init(&c->comm, params->nccl_unique_id, params->rank, params->nranks,
+                               params->device, g_err);
+        if (r != OPP_OK) {
+            cudaFreeHost(c->hcnt);
+            delete c;
+            return r;
+        }
+    }
+    *out = c;
+    return OPP_OK;
+}
+
+static void free_pset(opp_ctx c, PSet &ps) {
+    size_t cap = (size_t)ps.cap;
+    c->dfree(ps.dcnt, sizeof(DevCounters));
+    c->dfree(ps.holes, 4 * cap);
+    c->dfree(ps.work, 4 * cap);
+    c->dfree(ps.head, 4 * cap);
+    c->dfree(ps.tail, 4 * cap);
+    c->dfree(ps.work_hops, 4 * cap);
+    c->dfree(ps.sr_cell, 4 * cap);
+    c->dfree(ps.sr_val, 32 * cap);
+    c->dfree(ps.staging, ps.staging_bytes);
+    ps = PSet();
+}
+
+extern "C" int opp_finalize(opp_ctx c) {
+    if (!c) return OPP_OK;
+    cudaSetDevice(c->p.device);
+    cudaStreamSynchronize(c->s);
+    for (auto &col : c->cols) c->dfree(col.d, col.bytes);
+    for (auto &ps : c->psets) free_pset(c, ps);
+    MeshCache &m = c->mc;
+    c->dfree(m.lines, sizeof(WalkLine) * m.nc);
+    c->dfree(m.efp, sizeof(double4) * m.nc);
+    c->dfree(m.ov_map, 0);
+    c->dfree(m.sr_hist, 0);
+    c->dfree(m.sr_start, 0);
+    c->dfree(m.sr_sorted, 0);
+    c->dfree(m.sr_cellsum, 0);
+    c->dfree(m.n2cs_ptr, 0);
+    c->dfree(m.n2cs, 0);
+    if (c->comm) opp::comm_free(c->comm);
+    for (auto e : c->ev_pool) cudaEventDestroy(e);
+    cudaFreeHost(c->hcnt);
+    delete c;
+    return OPP_OK;
+}
+
+extern "C" int64_t opp_kernel_launch_count(opp_ctx c) { return c ? c->launches : -1; }
+
+extern "C" int opp_phase_timing(opp_ctx c, int enable) {
+    TRY(ctx_check(c));
+    c->timing = enable != 0;
+    return OPP_OK;
+}
+
+extern "C" int opp_get_phase_times(opp_ctx c, double *ms_sum, int64_t *count) {
+    TRY(ctx_check(c));
+    if (!ms_sum || !count) return fail(OPP_ERR_ARG, "null out");
+    CK(cudaStreamSynchronize(c->s));
+    for (int k = 0; k < OPP_N_PHASES; k++) {
+        ms_sum[k] = 0.0;
+        count[k] = 0;
+    }
+    for (size_t k = 0; k < c->ev_phase.size(); k++) {
+        float ms = 0.f;
+        CK(cudaEventElapsedTime(&ms, c->ev_pool[2 * k], c->ev_pool[2 * k + 1]));
+        ms_sum[c->ev_phase[k]] += ms;
+        count[c->ev_phase[k]]++;
+    }
+    c->ev_phase.clear();
+    c->ev_used = 0;
+    return OPP_OK;
+}
+
+extern "C" int opp_sync(opp_ctx c) {
+    TRY(ctx_check(c));
+    CK(cudaStreamSynchronize(c->s));
+    CK(cudaGetLastError());
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Declarations
+// ---------------------------------------------------------------------------
+extern "C" int opp_decl_set(opp_ctx c, int64_t size, const char *name, opp_set *out) {
+    TRY(ctx_check(c));
+    if (size < 0 || !out) return fail(OPP_ERR_ARG, "opp_decl_set: bad size or out");
+    Set s;
+    s.name = name ? name : "";
+    s.size = size;
+    c->sets.push_back(s);
+    *out = (opp_set)c->sets.size() - 1;
+    return OPP_OK;
+}
+
+static int alloc_scratch(opp_ctx c, PSet &ps, long long cap) {
+    size_t n = (size_t)cap;
+    ps.holes = (uint32_t *)c->dalloc(4 * n);
+    ps.work = (uint32_t *)c->dalloc(4 * n);
+    ps.head = (uint32_t *)c->dalloc(4 * n);
+    ps.tail = (uint32_t *)c->dalloc(4 * n);
+    ps.work_hops = (int32_t *)c->dalloc(4 * n);
+    if (!ps.holes || !ps.work || !ps.head || !ps.tail || !ps.work_hops)
+        return fail(OPP_ERR_NOMEM, "particle scratch (%lld)", cap);
+    if (c->p.deposit_mode == OPP_DEP_SORT_SEGRED) {
+        ps.sr_cell = (int32_t *)c->dalloc(4 * n);
+        ps.sr_val = (double *)c->dalloc(32 * n);
+        if (!ps.sr_cell || !ps.sr_val) return fail(OPP_ERR_NOMEM, "SR scratch");
+    }
+    return OPP_OK;
+}
+
+extern "C" int opp_decl_particle_set(opp_ctx c, const char *name, opp_set cells, int64_t n_init,
+                                     int64_t capacity, opp_set *out) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, cells));
+    if (c->sets[cells].particle) return fail(OPP_ERR_ARG, "particle set must live on a mesh set");
+    if (n_init < 0 || !out) return fail(OPP_ERR_ARG, "opp_decl_particle_set: bad n_init/out");
+    if (capacity > 0 && capacity < n_init) return fail(OPP_ERR_ARG, "capacity < n_init");
+    long long cap = std::max<long long>(std::max<long long>(n_init, capacity), 1024);
+    if (cap > 0xFFFFFFF0ll) return fail(OPP_ERR_ARG, "capacity above 2^32 indices");
+    PSet ps;
+    ps.cap = cap;
+    ps.n_ub = n_init;
+    ps.growth = c->p.allow_growth != 0 || capacity == 0;
+    ps.dcnt = (DevCounters *)c->dalloc(sizeof(DevCounters));
+    if (!ps.dcnt) return fail(OPP_ERR_NOMEM, "counters");
+    int r = alloc_scratch(c, ps, cap);
+    if (r != OPP_OK) {
+        free_pset(c, ps);
+        return r;
+    }
+    DevCounters h{};
+    h.n = (unsigned long long)n_init;
+    CK(cudaMemcpyAsync(ps.dcnt, &h, sizeof h, cudaMemcpyHostToDevice, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    Set s;
+    s.name = name ? name : "";
+    s.size = n_init;
+    s.particle = true;
+    s.cells = cells;
+    s.pset = (int)c->psets.size();
+    c->psets.push_back(ps);
+    c->sets.push_back(s);
+    *out = (opp_set)c->sets.size() - 1;
+    return OPP_OK;
+}
+
+// Upload host AoS [n][dim] into a particle column (SoA [dim][cap]).
+static int upload_particle_col(opp_ctx c, Col &col, long long cap, const void *host, long long n) {
+    if (!host || n == 0) return OPP_OK;
+    std::vector<char> tmp((size_t)n * col.eb);
+    for (int e = 0; e < col.dim; e++) {
+        const char *src = (const char *)host;
+        for (long long i = 0; i < n; i++)
+            std::memcpy(tmp.data() + (size_t)i * col.eb,
+                        src + ((size_t)i * col.dim + e) * col.eb, col.eb);
+        CK(cudaMemcpyAsync(col.d + (size_t)e * cap * col.eb, tmp.data(), (size_t)n * col.eb,
+                           cudaMemcpyHostToDevice, c->s));
+        CK(cudaStreamSynchronize(c->s));
+    }
+    return OPP_OK;
+}
+
+static int decl_col(opp_ctx c, bool is_map, opp_set set, opp_set to, int dim, int type,
+                    const void *host, const char *name, int32_t *out) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, set));
+    if (!out || dim < 1 || type_bytes(type) == 0) return fail(OPP_ERR_ARG, "bad dim/type/out");
+    Set &S = c->sets[set];
+    Col col;
+    col.is_map = is_map;
+    col.set = set;
+    col.to = to;
+    col.dim = dim;
+    col.type = type;
+    col.eb = type_bytes(type);
+    col.name = name ? name : "";
+    if (S.particle) {
+        PSet &ps = c->psets[S.pset];
+        if (ps.holes_pending || ps.n_ub != S.size)
+            return fail(OPP_ERR_STATE, "particle dats must be declared before the first step");
+        if (!host && S.size > 0)
+            return fail(OPP_ERR_ARG, "particle set has %lld initial particles: data required",
+                        (long long)S.size);
+        if ((int)ps.cols.size() >= kMaxCols) return fail(OPP_ERR_ARG, "too many particle columns");
+        col.bytes = (size_t)ps.cap * dim * col.eb;
+        col.d = (char *)c->dalloc(col.bytes);
+        if (!col.d) return fail(OPP_ERR_NOMEM, "particle dat %s", col.name.c_str());
+        int r = upload_particle_col(c, col, ps.cap, host, S.size);
+        if (r != OPP_OK) {
+            c->dfree(col.d, col.bytes);
+            return r;
+        }
+        ps.cols.push_back((int)c->cols.size());
+    } else {
+        col.bytes = (size_t)S.size * dim * col.eb;
+        col.d = (char *)c->dalloc(col.bytes);
+        if (!col.d) return fail(OPP_ERR_NOMEM, "mesh dat %s", col.name.c_str());
+        col.host.assign(col.bytes, 0);
+        if (host) std::memcpy(col.host.data(), host, col.bytes);
+        CK(cudaMemcpyAsync(col.d, col.host.data(), col.bytes, cudaMemcpyHostToDevice, c->s));
+        CK(cudaStreamSynchronize(c->s));
+    }
+    c->cols.push_back(std::move(col));
+    *out = (int32_t)c->cols.size() - 1;
+    return OPP_OK;
+}
+
+extern "C" int opp_decl_map(opp_ctx c, opp_set from, opp_set to, int dim, const int32_t *host,
+                            const char *name, opp_map *out) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, from));
+    TRY(set_check(c, to));
+    if (c->sets[to].particle) return fail(OPP_ERR_ARG, "maps point into mesh sets");
+    if (c->sets[from].particle && dim != 1) return fail(OPP_ERR_ARG, "particle maps have dim 1");
+    if (!c->sets[from].particle && !host && c->sets[from].size > 0)
+        return fail(OPP_ERR_ARG, "mesh maps are static: data required");
+    return decl_col(c, true, from, to, dim, OPP_INT, host, name, out);
+}
+
+extern "C" int opp_decl_dat(opp_ctx c, opp_set set, int dim, int type, const void *host,
+                            const char *name, opp_dat *out) {
+    return decl_col(c, false, set, -1, dim, type, host, name, out);
+}
+
+extern "C" int opp_set_partition(opp_ctx c, opp_set cells, const int32_t *rank_of_cell) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, cells));
+    if (!rank_of_cell) return fail(OPP_ERR_ARG, "rank_of_cell is NULL");
+    return opp::comm_set_partition(c->comm, c->p.rank, c->p.nranks, c->sets[cells].size,
+                                   rank_of_cell, &c->cell_base, g_err);
+}
+
+// ---------------------------------------------------------------------------
+// Particle storage management
+// ---------------------------------------------------------------------------
+static int exact_count(opp_ctx c, PSet &ps, long long *n) {
+    CK(cudaMemcpyAsync(c->hcnt, ps.dcnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    CK(cudaGetLastError());
+    ps.n_ub = (long long)c->hcnt->n;
+    ps.n_exact = true;
+    *n = ps.n_ub;
+    return OPP_OK;
+}
+
+static ColSet make_colset(opp_ctx c, PSet &ps) {
+    ColSet cs{};
+    cs.n = (int)ps.cols.size();
+    for (int j = 0; j < cs.n; j++) {
+        Col &col = c->cols[ps.cols[j]];
+        cs.c[j].ptr = col.d;
+        cs.c[j].cap = ps.cap;
+        cs.c[j].elem_bytes = col.eb;
+        cs.c[j].dim = col.dim;
+    }
+    return cs;
+}
+
+// Make room for `extra` more particles (exact count first; grow x1.5 if needed).
+static int grow(opp_ctx c, PSet &ps, long long extra) {
+    long long n;
+    TRY(exact_count(c, ps, &n));
+    const long long need = n + extra;
+    if (need <= ps.cap) return OPP_OK;
+    if (!ps.growth) return fail(OPP_ERR_CAPACITY, "capacity %lld < %lld", ps.cap, need);
+    long long ncap = std::max<long long>(need, ps.cap + ps.cap / 2);
+    if (ncap > 0xFFFFFFF0ll) return fail(OPP_ERR_CAPACITY, "capacity above 2^32 indices");
+    // allocate everything first so failure leaves the state unchanged
+    std::vector<char *> nd(ps.cols.size(), nullptr);
+    bool ok = true;
+    for (size_t j = 0; j < ps.cols.size(); j++) {
+        Col &col = c->cols[ps.cols[j]];
+        nd[j] = (char *)c->dalloc((size_t)ncap * col.dim * col.eb);
+        ok = ok && nd[j];
+    }
+    PSet tmp;
+    tmp.cap = ncap;
+    if (ok && alloc_scratch(c, tmp, ncap) != OPP_OK) ok = false;
+    if (!ok) {
+        for (size_t j = 0; j < nd.size(); j++)
+            if (nd[j]) c->dfree(nd[j], (size_t)ncap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
+        tmp.dcnt = nullptr;
+        free_pset(c, tmp);
+        return fail(OPP_ERR_NOMEM, "growing particle capacity to %lld", ncap);
+    }
+    for (size_t j = 0; j < ps.cols.size(); j++) {
+        Col &col = c->cols[ps.cols[j]];
+        if (n > 0)
+            CK(cudaMemcpy2DAsync(nd[j], (size_t)ncap * col.eb, col.d, (size_t)ps.cap * col.eb,
+                                 (size_t)n * col.eb, col.dim, cudaMemcpyDeviceToDevice, c->s));
+    }
+    CK(cudaStreamSynchronize(c->s));
+    for (size_t j = 0; j < ps.cols.size(); j++) {
+        Col &col = c->cols[ps.cols[j]];
+        c->dfree(col.d, col.bytes);
+        col.d = nd[j];
+        col.bytes = (size_t)ncap * col.dim * col.eb;
+    }
+    size_t oc = (size_t)ps.cap;
+    c->dfree(ps.holes, 4 * oc); c->dfree(ps.work, 4 * oc); c->dfree(ps.head, 4 * oc);
+    c->dfree(ps.tail, 4 * oc); c->dfree(ps.work_hops, 4 * oc);
+    c->dfree(ps.sr_cell, 4 * oc); c->dfree(ps.sr_val, 32 * oc);
+    ps.holes = tmp.holes; ps.work = tmp.work; ps.head = tmp.head; ps.tail = tmp.tail;
+    ps.work_hops = tmp.work_hops; ps.sr_cell = tmp.sr_cell; ps.sr_val = tmp.sr_val;
+    ps.cap = ncap;
+    return OPP_OK;
+}
+
+extern "C" int opp_inject(opp_ctx c, opp_set parts, int64_t n, int ncols, const int32_t *cols,
+                          const void *const *data, int on_device) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "opp_inject needs a particle set");
+    PSet &ps = c->psets[S.pset];
+    if (ps.holes_pending) return fail(OPP_ERR_STATE, "opp_fill_holes must run before injecting");
+    if (n < 0) return fail(OPP_ERR_ARG, "negative n");
+    if (n == 0) return OPP_OK;
+    if (ncols != (int)ps.cols.size() || !cols || !data)
+        return fail(OPP_ERR_ARG, "opp_inject must list every particle column (%d)",
+                    (int)ps.cols.size());
+    // order the sources by the set's column order
+    std::vector<const void *> src(ps.cols.size(), nullptr);
+    for (int k = 0; k < ncols; k++) {
+        auto it = std::find(ps.cols.begin(), ps.cols.end(), cols[k]);
+        if (it == ps.cols.end()) return fail(OPP_ERR_ARG, "column %d is not on this set", cols[k]);
+        if (!data[k]) return fail(OPP_ERR_ARG, "null data for column %d", cols[k]);
+        src[it - ps.cols.begin()] = data[k];
+    }
+    for (auto p : src)
+        if (!p) return fail(OPP_ERR_ARG, "a particle column was listed twice / missing");
+    if (ps.n_ub + n > ps.cap) TRY(grow(c, ps, n));
+    ColSet cs = make_colset(c, ps);
+    if (on_device) {
+        for (int j = 0; j < cs.n; j++) cs.src[j] = (const char *)src[j];
+    } else {
+        size_t tot = 0;
+        std::vector<size_t> off(cs.n);
+        for (int j = 0; j < cs.n; j++) {
+            off[j] = tot;
+            tot += ((size_t)n * cs.c[j].dim * cs.c[j].elem_bytes + 255) & ~(size_t)255;
+        }
+        if (tot > ps.staging_bytes) {
+            CK(cudaStreamSynchronize(c->s));
+            c->dfree(ps.staging, ps.staging_bytes);
+            ps.staging_bytes = 0;
+            ps.staging = (char *)c->dalloc(tot);
+            if (!ps.staging) return fail(OPP_ERR_NOMEM, "injection staging (%zu B)", tot);
+            ps.staging_bytes = tot;
+        }
+        for (int j = 0; j < cs.n; j++) {
+            CK(cudaMemcpyAsync(ps.staging + off[j], src[j],
+                               (size_t)n * cs.c[j].dim * cs.c[j].elem_bytes,
+                               cudaMemcpyHostToDevice, c->s));
+            cs.src[j] = ps.staging + off[j];
+        }
+    }
+    {
+        PhaseScope ph(c, OPP_PH_INJECT);
+        CK(launch_inject(cs, n, ps.dcnt, grid_for(c, n, 4), c->s));
+    }
+    c->launches++;
+    ps.n_ub += n;
+    ps.n_exact = false;
+    S.size = -1;  // device-resident count from now on
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Mesh preparation
+// ---------------------------------------------------------------------------
+static int validate_c2c(opp_ctx c, const Col &c2n, const Col &c2c, long long nc) {
+    const int32_t *cn = (const int32_t *)c2n.host.data();
+    const int32_t *cc = (const int32_t *)c2c.host.data();
+    long long base = c->cell_base;
+    for (long long e = 0; e < nc; e++) {
+        for (int i = 0; i < 4; i++) {
+            long long nb = cc[4 * e + i];
+            if (nb < 0) continue;
+            long long ln = nb - base;
+            if (ln < 0 || ln >= nc) continue;   // owned by another rank
+            int shared = 0;
+            bool opposite_in = false;
+            for (int a = 0; a < 4; a++) {
+                int v = cn[4 * ln + a];
+                if (v == cn[4 * e + i]) opposite_in = true;
+                for (int b = 0; b < 4; b++)
+                    if (b != i && cn[4 * e + b] == v) shared++;
+            }
+            if (shared != 3 || opposite_in)
+                return fail(OPP_ERR_MESH,
+                            "c2c[%lld][%d] = %lld does not share the face opposite local node %d",
+                            e + base, i, nb, i);
+        }
+    }
+    return OPP_OK;
+}
+
+static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int cell_ef) {
+    MeshCache &m = c->mc;
+    Col &cc = c->cols[c2c], &cn = c->cols[c2n], &np = c->cols[node_pos], &ef = c->cols[cell_ef];
+    long long nc = c->sets[cc.set].size;
+    if (m.c2c != c2c || m.c2n != c2n || m.node_pos != node_pos || m.vpos != np.version) {
+        TRY(validate_c2c(c, cn, cc, nc));
+        c->dfree(m.lines, sizeof(WalkLine) * m.nc);
+        c->dfree(m.efp, sizeof(double4) * m.nc);
+        m.efp = nullptr;
+        m.ef = -1;
+        m.lines = (WalkLine *)c->dalloc(sizeof(WalkLine) * std::max<long long>(nc, 1));
+        m.efp = (double4 *)c->dalloc(sizeof(double4) * std::max<long long>(nc, 1));
+        if (!m.lines || !m.efp) return fail(OPP_ERR_NOMEM, "walk lines");
+        m.nc = nc;
+        CK(cudaMemsetAsync(&ps.dcnt->err_flags, 0, sizeof(unsigned), c->s));
+        CK(launch_build_lines((const double *)np.d, (const int32_t *)cn.d, (const int32_t *)cc.d, nc,
+                              m.lines, ps.dcnt, c->s));
+        c->launches++;
+        unsigned flags = 0;
+        CK(cudaMemcpyAsync(&flags, &ps.dcnt->err_flags, sizeof flags, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        if (flags & 1u) {
+            m.c2c = -1;
+            return fail(OPP_ERR_MESH, "mesh has a tet with non-positive volume (orient c2n)");
+        }
+        m.c2c = c2c;
+        m.c2n = c2n;
+        m.node_pos = node_pos;
+        m.vpos = np.version;
+        m.ov_built = false;
+        if (m.sr_cellsum) {
+            c->dfree(m.n2cs_ptr, 0); c->dfree(m.n2cs, 0);
+            c->dfree(m.sr_hist, 0); c->dfree(m.sr_start, 0); c->dfree(m.sr_cellsum, 0);
+            m.sr_cellsum = nullptr;
+        }
+    }
+    if (m.ef != cell_ef || m.vef != ef.version) {
+        CK(launch_pack_field((const double *)ef.d, nc, m.efp, c->s));
+        c->launches++;
+        m.ef = cell_ef;
+        m.vef = ef.version;
+    }
+    if (c->p.direct_hop && !m.ov_built) {
+        // overlay box = bounding box of the nodes; spacing = given or h/2
+        const double *xyz = (const double *)np.host.data();
+        long long nn = c->sets[np.set].size;
+        double lo[3] = {1e300, 1e300, 1e300}, hi[3] = {-1e300, -1e300, -1e300};
+        for (long long i = 0; i < nn; i++)
+            for (int k = 0; k < 3; k++) {
+                lo[k] = std::min(lo[k], xyz[3 * i + k]);
+                hi[k] = std::max(hi[k], xyz[3 * i + k]);
+            }
+        double dx = c->p.overlay_spacing;
+        if (!(dx > 0)) {
+            double vol = (hi[0] - lo[0]) * (hi[1] - lo[1]) * (hi[2] - lo[2]);
+            dx = 0.5 * std::cbrt(6.0 * vol / std::max<long long>(nc, 1));
+        }
+        Overlay ov{};
+        long long tot = 1;
+        for (int k = 0; k < 3; k++) {
+            ov.x0[k] = lo[k];
+            ov.n[k] = std::max(1, (int)std::ceil((hi[k] - lo[k]) / dx));
+            tot *= ov.n[k];
+        }
+        ov.dx = dx;
+        if (tot > (1ll << 31)) return fail(OPP_ERR_ARG, "overlay too fine (%lld cells)", tot);
+        c->dfree(m.ov_map, 0);
+        m.ov_map = (int32_t *)c->dalloc(sizeof(int32_t) * tot);
+        if (!m.ov_map) return fail(OPP_ERR_NOMEM, "overlay");
+        ov.map = m.ov_map;
+        CK(launch_overlay(m.lines, (const double *)np.d, nc, c->cell_base, ov, m.ov_map, c->s));
+        c->launches += 3;
+        m.ov = ov;
+        m.ov_built = true;
+    }
+    if (c->p.deposit_mode == OPP_DEP_SORT_SEGRED && !m.sr_cellsum) {
+        long long nn = c->sets[c->cols[c2n].to].size;
+        const int32_t *h = (const int32_t *)cn.host.data();
+        std::vector<int32_t> ptr(nn + 1, 0), idx((size_t)4 * nc);
+        for (long long e = 0; e < 4 * nc; e++) ptr[h[e] + 1]++;
+        for (long long v = 0; v < nn; v++) ptr[v + 1] += ptr[v];
+        std::vector<int32_t> cur(ptr.begin(), ptr.end() - 1);
+        for (long long e = 0; e < 4 * nc; e++) idx[cur[h[e]]++] = (int32_t)e;
+        m.n2cs_ptr = (int32_t *)c->dalloc(4 * (nn + 1));
+        m.n2cs = (int32_t *)c->dalloc(4 * std::max<long long>(4 * nc, 1));
+        m.sr_hist = (unsigned *)c->dalloc(4 * (nc + 1));
+        m.sr_start = (unsigned *)c->dalloc(4 * (nc + 1));
+        m.sr_cellsum = (double *)c->dalloc(32 * std::max<long long>(nc, 1));
+        if (!m.n2cs_ptr || !m.n2cs || !m.sr_hist || !m.sr_start || !m.sr_cellsum)
+            return fail(OPP_ERR_NOMEM, "SR mesh buffers");
+        CK(cudaMemcpyAsync(m.n2cs_ptr, ptr.data(), 4 * (nn + 1), cudaMemcpyHostToDevice, c->s));
+        CK(cudaMemcpyAsync(m.n2cs, idx.data(), 4 * 4 * nc, cudaMemcpyHostToDevice, c->s));
+        CK(cudaStreamSynchronize(c->s));
+    }
+    if (c->p.deposit_mode == OPP_DEP_SORT_SEGRED && m.sr_cap < ps.cap) {
+        c->dfree(m.sr_sorted, 0);
+        m.sr_sorted = (double *)c->dalloc(32 * (size_t)ps.cap);
+        if (!m.sr_sorted) return fail(OPP_ERR_NOMEM, "SR sorted buffer");
+        m.sr_cap = ps.cap;
+    }
+    return OPP_OK;
+}
+
+static int check_col(opp_ctx c, int h, bool want_map, int set, int dim, int type, const char *what) {
+    TRY(col_check(c, h));
+    Col &col = c->cols[h];
+    if (col.is_map != want_map || (set >= 0 && col.set != set) || col.dim != dim ||
+        (!want_map && col.type != type))
+        return fail(OPP_ERR_ARG, "%s: wrong kind/set/dim/type (handle %d '%s')", what, h,
+                    col.name.c_str());
+    return OPP_OK;
+}
+
+static int do_fill(opp_ctx c, PSet &ps, int p2c) {
+    PhaseScope ph(c, OPP_PH_FILL);
+    ColSet cs = make_colset(c, ps);
+    CK(launch_fill(cs, ps.dcnt, ps.holes, (const int32_t *)c->cols[p2c].d, ps.head, ps.tail,
+                   grid_for(c, ps.n_ub, 4), c->s));
+    c->launches += 2;
+    ps.holes_pending = false;
+    return OPP_OK;
+}
+
+static int read_stats(opp_ctx c, PSet &ps, opp_step_stats *stats) {
+    CK(cudaMemcpyAsync(c->hcnt, ps.dcnt, sizeof(DevCounters), cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    CK(cudaGetLastError());
+    const DevCounters &h = *c->hcnt;
+    std::memset(stats, 0, sizeof *stats);
+    stats->n_before = (int64_t)h.n_before;
+    stats->n_injected = (int64_t)h.n_inj_last;
+    stats->n_removed = (int64_t)h.n_removed;
+    stats->n_after = (int64_t)(h.n - h.n_holes);
+    stats->n_migrated_out = (int64_t)h.n_mig_out;
+    stats->n_migrated_in = (int64_t)h.n_mig_in;
+    stats->total_hops = (int64_t)h.total_hops;
+    stats->n_hop_capped = (int64_t)h.n_capped;
+    stats->n_deferred = (int64_t)h.n_work;
+    stats->max_hops = (int32_t)h.max_hops;
+    stats->cum_pushed = (int64_t)h.cum_pushed;
+    stats->cum_steps = (int64_t)h.cum_steps;
+    if (!ps.holes_pending) {
+        ps.n_ub = (long long)h.n;
+        ps.n_exact = true;
+    }
+    return OPP_OK;
+}
+
+extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_dat vel,
+                                     opp_map p2c, opp_map c2c, opp_map c2n, opp_dat node_pos,
+                                     opp_dat cell_ef, opp_dat node_charge,
+                                     const opp_step_params *prm, opp_step_stats *stats) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    if (!prm) return fail(OPP_ERR_ARG, "null step params");
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
+    PSet &ps = c->psets[S.pset];
+    if (ps.holes_pending) return fail(OPP_ERR_STATE, "opp_fill_holes must run before the next step");
+    TRY(check_col(c, pos, false, parts, 3, OPP_REAL, "pos"));
+    TRY(check_col(c, vel, false, parts, 3, OPP_REAL, "vel"));
+    TRY(check_col(c, p2c, true, parts, 1, OPP_INT, "p2c"));
+    const int cells = S.cells;
+    TRY(check_col(c, c2c, true, cells, 4, OPP_INT, "c2c"));
+    TRY(check_col(c, c2n, true, cells, 4, OPP_INT, "c2n"));
+    if (c->cols[c2c].to != cells) return fail(OPP_ERR_ARG, "c2c must map cells to cells");
+    const int nodes = c->cols[c2n].to;
+    TRY(check_col(c, node_pos, false, nodes, 3, OPP_REAL, "node_pos"));
+    TRY(check_col(c, cell_ef, false, cells, 3, OPP_REAL, "cell_ef"));
+    TRY(check_col(c, node_charge, false, nodes, 1, OPP_REAL, "node_charge"));
+    TRY(prepare_mesh(c, ps, c2c, c2n, node_pos, cell_ef));
+
+    MeshCache &m = c->mc;
+    const long long nn = c->sets[nodes].size;
+    StepArgs a{};
+    a.pos = (double *)c->cols[pos].d;
+    a.vel = (double *)c->cols[vel].d;
+    a.p2c = (int32_t *)c->cols[p2c].d;
+    a.cap = ps.cap;
+    a.lines = m.lines;
+    a.ef = m.efp;
+    a.Q = (double *)c->cols[node_charge].d;
+    a.cnt = ps.dcnt;
+    a.holes = ps.holes;
+    a.work = ps.work;
+    a.work_hops = ps.work_hops;
+    a.sr_cell = ps.sr_cell;
+    a.sr_val = ps.sr_val;
+    a.c1 = prm->qm * prm->dt;
+    a.dt = prm->dt;
+    a.w = prm->weight;
+    a.cell_base = c->cell_base;
+    a.n_cells = (int)m.nc;
+    a.hpass = c->p.hop_budget_per_pass;
+    a.hcap = c->p.hop_cap;
+    a.ov = m.ov;
+    const int dep = c->p.deposit_mode;
+    const bool dh = c->p.direct_hop != 0;
+    const bool multi = c->p.nranks > 1;
+
+    {
+        PhaseScope ph(c, OPP_PH_BEGIN);
+        CK(launch_step_begin(a.Q, nn, ps.dcnt, prm->zero_charge, grid_for(c, nn, 2), c->s));
+    }
+    c->launches++;
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(dep, dh);
+    const int bps = c->bps;
+    const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
+                                                                       (long long)c->nsm * bps));
+    {
+        PhaseScope ph(c, OPP_PH_PUSH_MOVE_DEPOSIT);
+        CK(launch_push_move_deposit(dep, dh, multi, false, a, pgrid, c->s));
+    }
+    {
+        PhaseScope ph(c, OPP_PH_CONTINUE);
+        CK(launch_push_move_deposit(dep, dh, multi, true, a,
+                                    std::max(1, std::min(pgrid, c->nsm * 2)), c->s));
+    }
+    c->launches += 2;
+    if (multi) {
+        PhaseScope ph(c, OPP_PH_MIGRATE);
+        int r = opp::comm_migrate(c->comm, &a, c->s, g_err);
+        if (r != OPP_OK) return r;
+    }
+    if (dep == OPP_DEP_SORT_SEGRED) {
+        PhaseScope ph(c, OPP_PH_SEGRED);
+        CK(launch_sr(a, m.nc, nn, m.sr_hist, m.sr_start, m.sr_sorted, m.sr_cellsum, m.n2cs_ptr,
+                     m.n2cs, grid_for(c, ps.n_ub, 8), c->s));
+        c->launches += 5;
+    }
+    ps.holes_pending = true;
+    if (prm->fill_inline) TRY(do_fill(c, ps, p2c));
+    if (stats) TRY(read_stats(c, ps, stats));
+    return OPP_OK;
+}
+
+extern "C" int opp_get_step_stats(opp_ctx c, opp_set parts, opp_step_stats *stats) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    if (!stats) return fail(OPP_ERR_ARG, "null stats");
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
+    return read_stats(c, c->psets[S.pset], stats);
+}
+
+extern "C" int opp_fill_holes(opp_ctx c, opp_set parts, int64_t *n_after) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
+    PSet &ps = c->psets[S.pset];
+    if (ps.holes_pending) {
+        int p2c = -1;
+        for (int h : ps.cols)
+            if (c->cols[h].is_map) p2c = h;
+        if (p2c < 0) return fail(OPP_ERR_STATE, "particle set has no p2c map");
+        TRY(do_fill(c, ps, p2c));
+    }
+    if (n_after) {
+        long long n;
+        TRY(exact_count(c, ps, &n));
+        *n_after = n;
+    }
+    return OPP_OK;
+}
+
+extern "C" int opp_get_particle_count(opp_ctx c, opp_set parts, int64_t *n) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    if (!n) return fail(OPP_ERR_ARG, "null out");
+    Set &S = c->sets[parts];
+    if (!S.particle) {
+        *n = S.size;
+        return OPP_OK;
+    }
+    long long v;
+    TRY(exact_count(c, c->psets[S.pset], &v));
+    *n = c->psets[S.pset].holes_pending ? (long long)(c->hcnt->n - c->hcnt->n_holes) : v;
+    return OPP_OK;
+}
+
+extern "C" int opp_get_node_charge(opp_ctx c, opp_dat q, double *host_out, int64_t n) {
+    TRY(ctx_check(c));
+    TRY(col_check(c, q));
+    Col &col = c->cols[q];
+    if (col.is_map || col.dim != 1 || col.type != OPP_REAL || c->sets[col.set].particle)
+        return fail(OPP_ERR_ARG, "node charge is a dim-1 OPP_REAL node dat");
+    if (!host_out || n != c->sets[col.set].size) return fail(OPP_ERR_ARG, "n must equal the node count");
+    CK(cudaMemcpyAsync(host_out, col.d, sizeof(double) * n, cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    CK(cudaGetLastError());
+    return OPP_OK;
+}
+
+extern "C" int opp_get_dat(opp_ctx c, int32_t h, void *host_out, int64_t n_elems) {
+    TRY(ctx_check(c));
+    TRY(col_check(c, h));
+    if (!host_out) return fail(OPP_ERR_ARG, "null out");
+    Col &col = c->cols[h];
+    Set &S = c->sets[col.set];
+    if (!S.particle) {
+        if (n_elems < 0 || n_elems > S.size) return fail(OPP_ERR_ARG, "n_elems out of range");
+        CK(cudaMemcpyAsync(host_out, col.d, (size_t)n_elems * col.dim * col.eb,
+                           cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        return OPP_OK;
+    }
+    PSet &ps = c->psets[S.pset];
+    if (ps.holes_pending) return fail(OPP_ERR_STATE, "particle dats contain holes: opp_fill_holes first");
+    long long n;
+    TRY(exact_count(c, ps, &n));
+    if (n_elems != n) return fail(OPP_ERR_ARG, "n_elems (%lld) != particle count (%lld)",
+                                  (long long)n_elems, n);
+    std::vector<char> tmp((size_t)n * col.eb);
+    char *dst = (char *)host_out;
+    for (int e = 0; e < col.dim; e++) {
+        if (n == 0) break;
+        CK(cudaMemcpyAsync(tmp.data(), col.d + (size_t)e * ps.cap * col.eb, (size_t)n * col.eb,
+                           cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        for (long long i = 0; i < n; i++)
+            std::memcpy(dst + ((size_t)i * col.dim + e) * col.eb, tmp.data() + (size_t)i * col.eb, col.eb);
+    }
+    return OPP_OK;
+}
+
+extern "C" int opp_set_dat(opp_ctx c, opp_dat h, const void *src, int64_t n_elems, int on_device) {
+    TRY(ctx_check(c));
+    TRY(col_check(c, h));
+    if (!src) return fail(OPP_ERR_ARG, "null src");
+    Col &col = c->cols[h];
+    Set &S = c->sets[col.set];
+    if (col.is_map && !S.particle) return fail(OPP_ERR_ARG, "mesh maps are static (PAPER.md:924-926)");
+    if (S.particle) return fail(OPP_ERR_ARG, "particle dats change through opp_inject / the step");
+    if (n_elems < 0 || n_elems > S.size) return fail(OPP_ERR_ARG, "n_elems out of range");
+    size_t bytes = (size_t)n_elems * col.dim * col.eb;
+    CK(cudaMemcpyAsync(col.d, src, bytes, on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                       c->s));
+    if (on_device) {
+        CK(cudaMemcpyAsync(col.host.data(), col.d, bytes, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+    } else {
+        std::memcpy(col.host.data(), src, bytes);
+    }
+    col.version++;
+    return OPP_OK;
+}
+
+extern "C" int opp_get_dat_device_ptr(opp_ctx c, int32_t h, void **ptr, int64_t *stride) {
+    TRY(ctx_check(c));
+    TRY(col_check(c, h));
+    if (!ptr || !stride) return fail(OPP_ERR_ARG, "null out");
+    Col &col = c->cols[h];
+    Set &S = c->sets[col.set];
+    *ptr = col.d;
+    *stride = S.particle ? c->psets[S.pset].cap : col.dim;
+    return OPP_OK;
+}

@@ -1,0 +1,91 @@
+// opp_internal.h -- device data layouts shared by the host library and the
+// sm_100a kernels of libopp.  Nothing here is visible through include/opp.h.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace opp {
+
+// One 128-byte, 128-byte-aligned "walk line" per cell: everything one cell
+// visit of the walk and the deposit needs, in a single L2 line (SURVEY.md
+// §8(a)).  lambda_i = g_i . (x - p0), i = 1..3; lambda_0 = 1 - (l1+l2+l3)
+// (node-relative form: keeps absolute accuracy far from the origin).
+struct __align__(128) WalkLine {
+    double g[9];      // rows: grad lambda_1, grad lambda_2, grad lambda_3
+    double p0[3];     // local node 0
+    int32_t c2c[4];   // neighbour across the face opposite local node i (global id), -1 boundary
+    int32_t c2n[4];   // local node ids (for the deposit)
+};
+static_assert(sizeof(WalkLine) == 128, "walk line must be one 128-B line");
+
+// Device-resident counters: the particle count lives on the device so a
+// whole step can be enqueued without a host round trip.
+struct DevCounters {
+    unsigned long long n;            // committed particle count
+    unsigned long long n_before;     // count entering the last push
+    unsigned long long n_injected;   // injected since the last push
+    unsigned long long n_inj_last;   // snapshot of n_injected at the last push
+    unsigned long long n_holes;      // holes recorded by the last push (R)
+    unsigned long long n_work;       // deferred walks (continuation worklist)
+    unsigned long long n_deferred;   // snapshot of n_work for stats
+    unsigned long long total_hops;
+    unsigned long long n_capped;
+    unsigned long long n_head, n_tail;   // hole-fill pairing lists
+    unsigned long long n_removed_last;   // R of the last fill
+    unsigned long long n_removed;        // REMOVE count of the last push
+    unsigned long long n_mig_out, n_mig_in;
+    unsigned long long inj_done_blocks;  // last-block-commit ticket for k_inject
+    unsigned long long n_sr;             // SR deposit: number of stored records
+    unsigned long long cum_pushed;       // sum of n_before over all steps
+    unsigned long long cum_steps;
+    unsigned int max_hops;
+    unsigned int err_flags;              // bit 0: non-positive tet, bit 1: SR overflow
+    unsigned long long pad[11];
+};
+
+constexpr int kMaxCols = 16;
+
+// Generic particle column (a particle dat or the p2c map) for inject /
+// hole fill / growth: SoA, elem_bytes in {4, 8}, dim components of stride
+// `cap` elements each.
+struct ColDesc {
+    char *ptr;
+    long long cap;
+    int elem_bytes;
+    int dim;
+};
+struct ColSet {
+    ColDesc c[kMaxCols];
+    const char *src[kMaxCols];   // k_inject: AoS source per column
+    int n;
+};
+
+// Direct-hop overlay.
+struct Overlay {
+    double x0[3];
+    double dx;
+    int n[3];
+    const int32_t *map;   // n[0]*n[1]*n[2], -1 = no tet
+};
+
+struct StepArgs {
+    double *pos;      // SoA [3][cap]
+    double *vel;      // SoA [3][cap]
+    int32_t *p2c;     // [cap], global cell ids; -1 = hole
+    long long cap;
+    const WalkLine *lines;     // local cells
+    const double4 *ef;         // local cells, padded
+    double *Q;                 // node charge (local nodes)
+    DevCounters *cnt;
+    uint32_t *holes;           // [cap]
+    uint32_t *work;            // [cap] deferred particle indices
+    int32_t *work_hops;        // [cap]
+    int32_t *sr_cell;          // SR records (cell, 4 values)
+    double *sr_val;            // [4][cap]
+    double c1, dt, w;
+    int cell_base, n_cells;    // global id of local cell 0, local cell count
+    int hpass, hcap;
+    Overlay ov;
+};
+
+}  // namespace opp

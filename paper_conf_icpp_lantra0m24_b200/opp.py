@@ -1,0 +1,256 @@
+"""Thin ctypes binding of libopp.so (include/opp.h) -- argument marshalling only.
+
+Every entry point of the C ABI is exposed under the same name; a negative
+return code raises OppError carrying opp_last_error().  There is no fallback:
+if libopp.so is missing or cannot be loaded, importing this module raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libopp.so")
+
+OPP_OK, OPP_ERR_ARG, OPP_ERR_STATE, OPP_ERR_NOMEM, OPP_ERR_CAPACITY = 0, -1, -2, -3, -4
+OPP_ERR_CUDA, OPP_ERR_NCCL, OPP_ERR_MESH = -5, -6, -7
+OPP_REAL, OPP_INT, OPP_INT64 = 0, 1, 2
+OPP_MOVE_DONE, OPP_NEED_MOVE, OPP_NEED_REMOVE, OPP_NEED_MIGRATE = 0, 1, 2, 3
+OPP_DEP_ATOMIC, OPP_DEP_ATOMIC_WARPAGG, OPP_DEP_SORT_SEGRED, OPP_DEP_AUTO = 0, 1, 2, 3
+
+ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
+FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
+
+# Every symbol include/opp.h declares (checked by tests/test_abi.py).
+EXPORTS = (
+    "opp_init_params_default", "opp_init", "opp_finalize", "opp_get_nccl_unique_id",
+    "opp_decl_set", "opp_decl_particle_set", "opp_decl_map", "opp_decl_dat",
+    "opp_set_partition", "opp_inject", "opp_push_move_deposit", "opp_fill_holes",
+    "opp_get_node_charge", "opp_get_dat", "opp_set_dat", "opp_get_particle_count",
+    "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
+    "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats",
+)
+PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo")
+
+
+class OppError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"opp error {code}: {msg}")
+        self.code = code
+
+
+class opp_init_params(C.Structure):
+    _fields_ = [("device", C.c_int), ("cuda_stream", C.c_void_p), ("rank", C.c_int),
+                ("nranks", C.c_int), ("nccl_unique_id", C.c_void_p), ("alloc", ALLOC_FN),
+                ("free", FREE_FN), ("alloc_user", C.c_void_p), ("deposit_mode", C.c_int),
+                ("direct_hop", C.c_int), ("overlay_spacing", C.c_double),
+                ("hop_budget_per_pass", C.c_int), ("hop_cap", C.c_int),
+                ("allow_growth", C.c_int)]
+
+
+class opp_step_params(C.Structure):
+    _fields_ = [("dt", C.c_double), ("qm", C.c_double), ("weight", C.c_double),
+                ("zero_charge", C.c_int), ("fill_inline", C.c_int)]
+
+
+class opp_step_stats(C.Structure):
+    _fields_ = [("n_before", C.c_int64), ("n_injected", C.c_int64), ("n_removed", C.c_int64),
+                ("n_after", C.c_int64), ("n_migrated_out", C.c_int64),
+                ("n_migrated_in", C.c_int64), ("total_hops", C.c_int64),
+                ("n_hop_capped", C.c_int64), ("n_deferred", C.c_int64),
+                ("max_hops", C.c_int32), ("migrate_rounds", C.c_int32),
+                ("cum_pushed", C.c_int64), ("cum_steps", C.c_int64)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                          "(python -m paper_conf_icpp_lantra0m24_b200.build)")
+    lib = C.CDLL(LIB_PATH)
+    P, I, I64, I32 = C.c_void_p, C.c_int, C.c_int64, C.c_int32
+    sig = {
+        "opp_init_params_default": (None, [C.POINTER(opp_init_params)]),
+        "opp_init": (I, [C.POINTER(opp_init_params), C.POINTER(P)]),
+        "opp_finalize": (I, [P]),
+        "opp_get_nccl_unique_id": (I, [P]),
+        "opp_decl_set": (I, [P, I64, C.c_char_p, C.POINTER(I32)]),
+        "opp_decl_particle_set": (I, [P, C.c_char_p, I32, I64, I64, C.POINTER(I32)]),
+        "opp_decl_map": (I, [P, I32, I32, I, P, C.c_char_p, C.POINTER(I32)]),
+        "opp_decl_dat": (I, [P, I32, I, I, P, C.c_char_p, C.POINTER(I32)]),
+        "opp_set_partition": (I, [P, I32, P]),
+        "opp_inject": (I, [P, I32, I64, I, P, P, I]),
+        "opp_push_move_deposit": (I, [P, I32, I32, I32, I32, I32, I32, I32, I32, I32,
+                                      C.POINTER(opp_step_params), C.POINTER(opp_step_stats)]),
+        "opp_fill_holes": (I, [P, I32, C.POINTER(I64)]),
+        "opp_get_step_stats": (I, [P, I32, C.POINTER(opp_step_stats)]),
+        "opp_get_node_charge": (I, [P, I32, P, I64]),
+        "opp_get_dat": (I, [P, I32, P, I64]),
+        "opp_set_dat": (I, [P, I32, P, I64, I]),
+        "opp_get_particle_count": (I, [P, I32, C.POINTER(I64)]),
+        "opp_get_dat_device_ptr": (I, [P, I32, C.POINTER(P), C.POINTER(I64)]),
+        "opp_kernel_launch_count": (I64, [P]),
+        "opp_sync": (I, [P]),
+        "opp_phase_timing": (I, [P, I]),
+        "opp_get_phase_times": (I, [P, P, P]),
+        "opp_last_error": (C.c_char_p, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    return lib
+
+
+lib = _load()
+
+
+def _ck(rc: int) -> int:
+    if rc < 0:
+        raise OppError(rc, lib.opp_last_error().decode(errors="replace"))
+    return rc
+
+
+def _name(s) -> bytes:
+    return (s or "").encode()
+
+
+def _ptr(a):
+    """Pointer of a numpy array / torch tensor / int / None."""
+    if a is None:
+        return None
+    if isinstance(a, int):
+        return a
+    if hasattr(a, "data_ptr"):
+        return a.data_ptr()
+    return a.ctypes.data
+
+
+# ----------------------------------------------------------------- ABI mirror
+def opp_init_params_default() -> opp_init_params:
+    p = opp_init_params()
+    lib.opp_init_params_default(C.byref(p))
+    return p
+
+
+def opp_init(params: opp_init_params) -> int:
+    out = C.c_void_p()
+    _ck(lib.opp_init(C.byref(params), C.byref(out)))
+    return out.value
+
+
+def opp_finalize(ctx) -> None:
+    _ck(lib.opp_finalize(ctx))
+
+
+def opp_get_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _ck(lib.opp_get_nccl_unique_id(buf))
+    return buf.raw
+
+
+def opp_decl_set(ctx, size: int, name: str) -> int:
+    out = C.c_int32()
+    _ck(lib.opp_decl_set(ctx, int(size), _name(name), C.byref(out)))
+    return out.value
+
+
+def opp_decl_particle_set(ctx, name: str, cells: int, n_init: int = 0, capacity: int = 0) -> int:
+    out = C.c_int32()
+    _ck(lib.opp_decl_particle_set(ctx, _name(name), cells, int(n_init), int(capacity), C.byref(out)))
+    return out.value
+
+
+def opp_decl_map(ctx, frm: int, to: int, dim: int, host, name: str) -> int:
+    out = C.c_int32()
+    _ck(lib.opp_decl_map(ctx, frm, to, dim, _ptr(host), _name(name), C.byref(out)))
+    return out.value
+
+
+def opp_decl_dat(ctx, set_: int, dim: int, typ: int, host, name: str) -> int:
+    out = C.c_int32()
+    _ck(lib.opp_decl_dat(ctx, set_, dim, typ, _ptr(host), _name(name), C.byref(out)))
+    return out.value
+
+
+def opp_set_partition(ctx, cells: int, rank_of_cell) -> None:
+    _ck(lib.opp_set_partition(ctx, cells, _ptr(rank_of_cell)))
+
+
+def opp_inject(ctx, parts: int, n: int, cols, data, on_device: bool) -> None:
+    k = len(cols)
+    ca = (C.c_int32 * k)(*cols)
+    da = (C.c_void_p * k)(*[_ptr(d) for d in data])
+    _ck(lib.opp_inject(ctx, parts, int(n), k, ca, da, int(bool(on_device))))
+
+
+def opp_push_move_deposit(ctx, parts, pos, vel, p2c, c2c, c2n, node_pos, cell_ef, node_charge,
+                          params: opp_step_params, want_stats: bool = True):
+    st = opp_step_stats() if want_stats else None
+    _ck(lib.opp_push_move_deposit(ctx, parts, pos, vel, p2c, c2c, c2n, node_pos, cell_ef,
+                                  node_charge, C.byref(params), C.byref(st) if st else None))
+    return st
+
+
+def opp_get_step_stats(ctx, parts: int) -> opp_step_stats:
+    st = opp_step_stats()
+    _ck(lib.opp_get_step_stats(ctx, parts, C.byref(st)))
+    return st
+
+
+def opp_fill_holes(ctx, parts: int, want_count: bool = True):
+    if not want_count:
+        _ck(lib.opp_fill_holes(ctx, parts, None))
+        return None
+    n = C.c_int64()
+    _ck(lib.opp_fill_holes(ctx, parts, C.byref(n)))
+    return n.value
+
+
+def opp_get_node_charge(ctx, dat: int, out) -> None:
+    _ck(lib.opp_get_node_charge(ctx, dat, _ptr(out), int(out.shape[0])))
+
+
+def opp_get_dat(ctx, dat: int, out, n: int) -> None:
+    _ck(lib.opp_get_dat(ctx, dat, _ptr(out), int(n)))
+
+
+def opp_set_dat(ctx, dat: int, src, n: int, on_device: bool = False) -> None:
+    _ck(lib.opp_set_dat(ctx, dat, _ptr(src), int(n), int(bool(on_device))))
+
+
+def opp_get_particle_count(ctx, parts: int) -> int:
+    n = C.c_int64()
+    _ck(lib.opp_get_particle_count(ctx, parts, C.byref(n)))
+    return n.value
+
+
+def opp_get_dat_device_ptr(ctx, dat: int):
+    p, s = C.c_void_p(), C.c_int64()
+    _ck(lib.opp_get_dat_device_ptr(ctx, dat, C.byref(p), C.byref(s)))
+    return p.value, s.value
+
+
+def opp_kernel_launch_count(ctx) -> int:
+    return int(lib.opp_kernel_launch_count(ctx))
+
+
+def opp_sync(ctx) -> None:
+    _ck(lib.opp_sync(ctx))
+
+
+def opp_last_error() -> str:
+    return lib.opp_last_error().decode(errors="replace")
+
+
+def opp_phase_timing(ctx, enable: bool) -> None:
+    _ck(lib.opp_phase_timing(ctx, int(bool(enable))))
+
+
+def opp_get_phase_times(ctx) -> dict:
+    ms = (C.c_double * 8)()
+    cnt = (C.c_int64 * 8)()
+    _ck(lib.opp_get_phase_times(ctx, ms, cnt))
+    return {PHASES[k]: (ms[k], cnt[k]) for k in range(8)}

@@ -1,0 +1,172 @@
+"""CUDA path vs the CPU oracle, element by element (-m gpu).
+
+Config C1 (6x6x30 Kuhn duct, jittered; 100k particles + 1k injected per
+step; random per-cell field) in every deposit mode, MH and DH, H_pass in
+{1, 8}; plus edge cases (empty set, ragged sizes, everything removed, hop
+cap, capacity growth).  All calls go through the C ABI (libopp.so).
+"""
+import numpy as np
+import pytest
+
+import gen
+from parity_util import NEAR, c1_case, compare, run_oracle
+
+pytestmark = pytest.mark.gpu
+
+C1, DT, W = 0.5, 1.0, 1.0      # c1 = qm*dt with qm = 0.5, dt = 1
+
+
+def _gpu_run(mesh, ef, init, inject, steps, qm=C1, dt=DT, w=W, **kw):
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    sim = MiniFemPic(mesh, ef, **kw)
+    if init is not None and init["cell"].shape[0]:
+        sim.inject(init)
+    stats = []
+    for s in range(steps):
+        b = inject(s) if inject else None
+        if b is not None:
+            sim.inject(b)
+        stats.append(sim.step(dt, qm, w))
+    out = sim.particles()
+    Q = sim.node_charge_host()
+    launches = sim.launches()
+    sim.close()
+    return out, Q, stats, launches
+
+
+def _check(mesh, ef, init, inject, steps, hcap=1024, dh=False, **kw):
+    overlay = None
+    if dh:
+        box = mesh["box"]
+        dx = kw.get("overlay_spacing", 0.5)
+        n = [int(np.ceil((box[2 * k + 1] - box[2 * k]) / dx)) for k in range(3)]
+        overlay = ([box[0], box[2], box[4]], dx, n)
+    om, orc, Qo, ost, rem = run_oracle(mesh, ef, init, inject, steps, C1 * DT, DT, W,
+                                       hcap=hcap, use_dh=dh, overlay=overlay)
+    gout, Qg, gst, launches = _gpu_run(mesh, ef, init, inject, steps, hop_cap=hcap,
+                                        direct_hop=dh, **kw)
+    assert launches > 0
+    rep = compare(om, mesh["c2n"], orc, Qo, rem, gout, Qg, W)
+    # per-step bookkeeping agrees with the oracle exactly
+    for so, sg in zip(ost, gst):
+        assert sg["n_before"] == so["n_before"]
+        assert sg["n_removed"] == so["n_removed"]
+        assert sg["n_after"] == so["n_after"]
+        assert sg["n_hop_capped"] == so["n_capped"]
+    return rep, ost, gst
+
+
+@pytest.mark.parametrize("dep", [0, 1, 2])
+@pytest.mark.parametrize("hpass", [1, 8])
+def test_c1_parity_mh(dep, hpass):
+    mesh, ef, init, inject, steps = c1_case()
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, deposit_mode=dep, hop_budget=hpass)
+    assert rep["n_compared"] > 90_000
+    # identical arithmetic -> identical walks: hop totals match exactly
+    assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
+    assert [s["max_hops"] for s in gst] == [s["max_hops"] for s in ost]
+    if hpass == 1:
+        assert sum(s["n_deferred"] for s in gst) > 0
+
+
+@pytest.mark.parametrize("dep", [0, 1])
+def test_c1_parity_dh(dep):
+    mesh, ef, init, inject, steps = c1_case(drift=0.6, spread=0.3)
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, dh=True, deposit_mode=dep,
+                           overlay_spacing=0.5)
+    assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
+
+
+def test_c1_unjittered_uniform_field():
+    mesh, ef, init, inject, steps = c1_case(jitter=0.0, efield="uniform")
+    _check(mesh, ef, init, inject, steps)
+
+
+def test_hop_cap_counts_match():
+    mesh, ef, init, inject, steps = c1_case(n0=20_000, n_inj=0, steps=3, drift=1.5, spread=0.5)
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, hcap=2, hop_budget=1)
+    assert sum(s["n_capped"] for s in ost) > 0
+
+
+@pytest.mark.parametrize("n0", [0, 1, 31, 33, 257, 4097])
+def test_ragged_and_empty(n0):
+    mesh, ef, init, inject, steps = c1_case(n0=n0, n_inj=0, steps=3)
+    _check(mesh, ef, init, None, steps)
+
+
+def test_everything_removed():
+    mesh = gen.kuhn_duct(3, 3, 4, jitter=0.1, seed=3)
+    ef = np.zeros((mesh["n_cells"], 3))
+    init = gen.seed_particles(mesh, 5000, 9, drift=5.0, spread=0.0)   # all leave through z = 4
+    rep, ost, gst = _check(mesh, ef, init, None, 2)
+    assert gst[0]["n_after"] == 0 and gst[0]["n_removed"] == 5000
+
+
+def test_capacity_growth_through_injection():
+    mesh, ef, init, inject, steps = c1_case(n0=3000, n_inj=2500, steps=4)
+    _check(mesh, ef, init, inject, steps, capacity=1024)
+
+
+def test_stale_holes_protocol():
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh, ef, init, inject, steps = c1_case(n0=1000, n_inj=0, steps=1)
+    sim = MiniFemPic(mesh, ef)
+    sim.inject(init)
+    sim.step(DT, C1, W, fill=False)
+    with pytest.raises(O.OppError) as e:
+        sim.particles()
+    assert e.value.code == O.OPP_ERR_STATE
+    with pytest.raises(O.OppError):
+        sim.step(DT, C1, W)
+    sim.fill_holes()
+    assert sim.count() == len(sim.particles()["id"])
+    sim.close()
+
+
+def test_invalid_mesh_rejected():
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh = gen.kuhn_duct(2, 2, 2)
+    bad = dict(mesh)
+    c2n = mesh["c2n"].copy()
+    c2n[5, [2, 3]] = c2n[5, [3, 2]]      # inverted tet
+    bad["c2n"] = c2n
+    sim = MiniFemPic(bad, np.zeros((mesh["n_cells"], 3)))
+    with pytest.raises(O.OppError) as e:
+        sim.step(DT, C1, W)
+    assert e.value.code == O.OPP_ERR_MESH
+    sim.close()
+    bad2 = dict(mesh)
+    c2c = mesh["c2c"].copy()
+    c2c[[0, 1]] = c2c[[1, 0]]
+    bad2["c2c"] = c2c
+    sim = MiniFemPic(bad2, np.zeros((mesh["n_cells"], 3)))
+    with pytest.raises(O.OppError) as e:
+        sim.step(DT, C1, W)
+    assert e.value.code == O.OPP_ERR_MESH
+    sim.close()
+
+
+def test_conservation_and_bookkeeping_gpu_only():
+    """Invariants that hold at any size (P5, P6) on a larger run."""
+    mesh = gen.kuhn_duct(16, 16, 24, jitter=0.2, seed=5)
+    ef = np.tile([0.0, 0.0, 1e-3], (mesh["n_cells"], 1))
+    init = gen.seed_particles(mesh, 1_000_000, 5)
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    sim = MiniFemPic(mesh, ef)
+    sim.inject(init)
+    n = 1_000_000
+    for s in range(3):
+        b = gen.inject_batch(mesh, s, 5000, 5, id_base=10_000_000)
+        sim.inject(b)
+        st = sim.step(DT, C1, W)
+        assert st["n_before"] == n + 5000
+        n = n + 5000 - st["n_removed"]
+        assert st["n_after"] == n == sim.count()
+        Q = sim.node_charge_host()
+        assert abs(Q.sum() - W * n) <= 4 * n * 2 ** -52 * W
+        assert st["n_hop_capped"] == 0
+    out = sim.particles()
+    assert np.unique(out["id"]).size == n
+    sim.close()
