@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--deposit", type=int, default=0, choices=[0, 1, 2])
     ap.add_argument("--dh", action="store_true")
     ap.add_argument("--hpass", type=int, default=4)
+    ap.add_argument("--sort", type=int, default=0, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
@@ -52,13 +54,13 @@ def parse():
 
 
 # ---------------------------------------------------------------- workload
-def workload(args):
+def workload(args, world=1):
     import gen
     cfg = dict(gen.CONFIGS[args.config])
     if args.n0:
         cfg["n0"] = args.n0
     nx, ny, nz = cfg["dims"]
-    mesh = gen.kuhn_duct(nx, ny, nz)
+    mesh = gen.kuhn_duct(nx, ny, nz * world)
     c1E = np.array(cfg["c1E"])
     qm, dt = 1.0, cfg["dt"]
     ef = np.tile(c1E / (qm * dt), (mesh["n_cells"], 1))
@@ -190,23 +192,47 @@ def run_ours(args, rank, world):
     import gen.cuda as gc
     from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
 
-    if world > 1:
-        raise SystemExit("multi-GPU slab migration is not built yet (DESIGN.md §7)")
+    from paper_conf_icpp_lantra0m24_b200 import dist as D
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
     dev = int(os.environ.get("LOCAL_RANK", 0))
     torch.cuda.set_device(dev)
-    cfg, mesh, ef, qm, dt, cluster, name = workload(args)
+    cfg, mesh, ef, qm, dt, cluster, name = workload(args, world)
     w, n0, n_inj, seed = cfg["w"], cfg["n0"], cfg["n_inj"], cfg["seed"]
     stream = torch.cuda.current_stream()
-    dm = gc.DeviceMesh(mesh)
     total = args.warmup + args.steps
-    cap = int(n0 * 1.05) + n_inj * (total + 4) + 1024
+    base, kw = 0, {}
+    if world > 1:
+        # weak scaling: the C2 duct stacked `world` times along z, one slab
+        # (48x48x72 hex, 50M particles) per GPU; injection on rank 0's inlet
+        uid = D.broadcast_bytes(O.opp_get_nccl_unique_id() if rank == 0 else None)
+        gm = mesh
+        mesh = D.slab(gm, world, rank)
+        ef = D.local_field(ef, mesh)
+        base = mesh["cell_base"]
+        kw = dict(nranks=world, rank=rank, uid=uid, transport=0)
+        gen_mesh = dict(mesh, inlet=mesh["inlet_local"])
+        if cluster is not None:
+            cluster = (cluster[0], cluster[1][(cluster[1] >= base) & (cluster[1] < base + mesh["n_cells"])] - base)
+    else:
+        gen_mesh = mesh
+    dm = gc.DeviceMesh(gen_mesh)
+    n_inj_local = n_inj if (world == 1 or mesh["inlet"].shape[0] > 0) else 0
+    cap = int(n0 * 1.1) + n_inj_local * (total + 4) + 1024
     sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
-                     direct_hop=args.dh, overlay_spacing=0.5, hop_budget=args.hpass)
-    init = gc.seed_particles(dm, n0, seed, cluster=cluster)
+                     direct_hop=args.dh, overlay_spacing=0.5, hop_budget=args.hpass,
+                     sort_every=args.sort, tma_pipeline=not args.direct, **kw)
+    init = gc.seed_particles(dm, n0, seed + rank, cluster=cluster, id_base=rank * n0)
+    if base:
+        init["cell"] += base
     sim.inject(init, on_device=True)
     torch.cuda.synchronize()
     del init
-    batches = [gc.inject_batch(dm, s, n_inj, seed, id_base=n0) if n_inj else None
+    if args.sort:
+        # the population is born in random cell order; a sorted steady state
+        # is what periodic sorting maintains (setup, untimed)
+        sim.step(0.0, qm, w, stats=False, fill=True)      # builds mesh data, dt = 0: no motion
+        sim.sort_by_cell()
+    batches = [gc.inject_batch(dm, s, n_inj_local, seed, id_base=world * n0) if n_inj_local else None
                for s in range(total)]
     torch.cuda.synchronize()
 
@@ -241,14 +267,11 @@ def run_ours(args, rank, world):
     st1 = sim.last_stats()
     pushed = st1["cum_pushed"] - st0["cum_pushed"]
     if world > 1:
-        t = torch.tensor([ms], device="cuda")
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
-        p = torch.tensor([pushed], device="cuda", dtype=torch.int64)
-        torch.distributed.all_reduce(p)
-        pushed = int(p.item())
+        ms = D.max_over_ranks(ms)
+        pushed = D.sum_over_ranks(pushed)
+        launches = D.sum_over_ranks(launches)
     value = pushed / (ms / 1e3)
-    n_avg = pushed / args.steps
+    n_avg = pushed / args.steps / world       # per GPU
 
     # ---- roofline of the dominant kernel (k_push_move_deposit, pass 1)
     peak, peak_src = load_peaks()
@@ -268,7 +291,6 @@ def run_ours(args, rank, world):
             traffic = None
     # whole-step model bytes (SURVEY.md §8(d) B_ps)
     f_inj = n_inj / max(n_avg, 1)
-    f_rem = (st1["cum_pushed"] and 0) or 0
     b_ps = 104.0 + (160.0 * nc + 16.0 * nn) / max(n_avg, 1) + 60.0 * f_inj
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
@@ -279,8 +301,10 @@ def run_ours(args, rank, world):
                    "particles_seeded": n0, "inject_per_step": n_inj,
                    "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
                    "walk": "DH+MH" if args.dh else "MH", "hop_budget_per_pass": args.hpass,
+                   "sort_every": args.sort, "pipeline": "direct" if args.direct else "tma",
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n_avg * 60 / 1e9),
-                   "parallelism": f"slab{world}"},
+                   "parallelism": f"slab{world}",
+                   "mesh_global": f"{cfg['dims'][0]}x{cfg['dims'][1]}x{cfg['dims'][2] * world} hex"},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "kernel": "k_push_move_deposit (pass 1)",
@@ -318,8 +342,11 @@ def run_ours(args, rank, world):
         ems = e0.elapsed_time(e1)
         s1 = sim.last_stats()
         epushed = s1["cum_pushed"] - s0["cum_pushed"]
+        if world > 1:
+            ems = D.max_over_ranks(ems)
+            epushed = D.sum_over_ranks(epushed)
         line["e2e"] = {"value": epushed / (ems / 1e3), "unit": UNIT,
-                       "h2d_bytes_per_step": n_inj * 60, "d2h_bytes_per_step": nn * 8,
+                       "h2d_bytes_per_step": n_inj * 60, "d2h_bytes_per_step": nn * 8 * world,
                        "steps": ke, "note": "injection arrays from pinned host memory (opp_inject "
                        "on_device=0) + node charge read back every step (opp_get_node_charge)"}
 

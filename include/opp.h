@@ -94,6 +94,13 @@ typedef struct {
     int hop_cap;                /* H_cap: hops after which the current cell is
                                    accepted as final and counted (S4)               */
     int allow_growth;           /* 1 = grow particle capacity x1.5 on injection     */
+    int sort_every;             /* > 0: every sort_every-th step the hole fill is a
+                                   counting sort by cell (also compacts), 0 = never */
+    int tma_pipeline;           /* 1 = stream particle tiles through shared memory
+                                   with cp.async.bulk (default), 0 = direct loads   */
+    int transport;              /* nranks > 1: 0 = NCCL (one process per GPU),
+                                   1 = in-process loopback (contexts in one process,
+                                   one host thread each; testing on one GPU)        */
 } opp_init_params;
 
 /* Per-step arguments of opp_push_move_deposit. */
@@ -123,7 +130,7 @@ typedef struct {
 
 /* Fill *p with defaults: device 0, default stream, 1 rank, cudaMalloc,
  * OPP_DEP_ATOMIC, MH only, overlay_spacing 0 (auto = 0.5 * mean edge),
- * H_pass = 4, H_cap = 1024, growth allowed. */
+ * H_pass = 4, H_cap = 1024, growth allowed, no periodic sort, TMA pipeline on. */
 void opp_init_params_default(opp_init_params *p);
 
 /* Create a context on params->device (nranks > 1: joins the NCCL clique). */
@@ -162,9 +169,15 @@ int opp_decl_dat(opp_ctx ctx, opp_set set, int dim, int type, const void *host,
                  const char *name, opp_dat *out);
 
 /* Slab partition (the user provides the rank of one set
- * "via an opp_dat"): rank_of_cell[c] for every global cell; each rank's cells
- * must form one contiguous global range. */
-int opp_set_partition(opp_ctx ctx, opp_set cells, const int32_t *rank_of_cell);
+ * "via an opp_dat"; the library derives the rest).  Collective: every rank
+ * calls it.  rank_of_cell[g] for every GLOBAL cell g (n_global_cells
+ * entries); each rank's cells must form one contiguous global range, and
+ * this context's `cells` set holds exactly its range, in order (so local
+ * cell k is global cell base + k; c2c and p2c carry global ids).  node_gid
+ * gives a global id for each of this rank's `nodes` (required iff
+ * nranks > 1): nodes with equal ids on two ranks form the charge halo. */
+int opp_set_partition(opp_ctx ctx, opp_set cells, int64_t n_global_cells,
+                      const int32_t *rank_of_cell, opp_set nodes, const int64_t *node_gid);
 
 /* opp_inject (PAPER.md:1014-1018 OPP_ITERATE_INJECTED, 1502-1508): append n
  * particles at [N, N+n).  cols lists EVERY particle dat / the p2c map of the
@@ -210,6 +223,12 @@ int opp_get_step_stats(opp_ctx ctx, opp_set parts, opp_step_stats *stats);
  * n_after may be NULL (no host synchronisation). */
 int opp_fill_holes(opp_ctx ctx, opp_set parts, int64_t *n_after);
 
+/* Reorder the particle set by cell (counting sort; PAPER.md:1638-1644
+ * "particle sorting is available as an auxiliary API call").  Drops holes
+ * if a step left any (it then replaces opp_fill_holes).  Order within a cell
+ * is implementation-defined. */
+int opp_sort_by_cell(opp_ctx ctx, opp_set parts);
+
 /* Copy node charge (dim 1) to host_out[n]; synchronises. */
 int opp_get_node_charge(opp_ctx ctx, opp_dat node_charge, double *host_out, int64_t n);
 
@@ -231,7 +250,8 @@ int opp_get_dat_device_ptr(opp_ctx ctx, int32_t dat_or_map, void **ptr, int64_t 
 /* Phases of the step timed by opp_phase_timing (indices into ms_sum / count). */
 enum opp_phase { OPP_PH_INJECT = 0, OPP_PH_BEGIN = 1, OPP_PH_PUSH_MOVE_DEPOSIT = 2,
                  OPP_PH_CONTINUE = 3, OPP_PH_SEGRED = 4, OPP_PH_FILL = 5, OPP_PH_MIGRATE = 6,
-                 OPP_PH_HALO = 7, OPP_N_PHASES = 8 };
+                 OPP_PH_HALO = 7, OPP_PH_SORT_COUNT = 8, OPP_PH_SORT_MOVE = 9,
+                 OPP_N_PHASES = 10 };
 
 /* enable != 0: record CUDA events on the context stream around every phase
  * of the following calls (negligible overhead, no host synchronisation). */

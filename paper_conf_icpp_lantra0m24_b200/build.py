@@ -16,6 +16,20 @@ LIB = os.path.join(HERE, "libopp.so")
 SOURCES = ["opp.cu", "opp_kernels.cu", "opp_comm.cu"]
 HEADERS = ["opp_internal.h", "opp_kernels.h", "opp_comm.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+
+
+def _nccl_dir():
+    """torch's pip NCCL (2.28.x): the one NCCL loaded in a torch process."""
+    try:
+        import importlib.util
+        spec = importlib.util.find_spec("nvidia.nccl")
+        if spec and spec.submodule_search_locations:
+            d = list(spec.submodule_search_locations)[0]
+            if os.path.exists(os.path.join(d, "include", "nccl.h")):
+                return d
+    except Exception:   # noqa: BLE001
+        pass
+    return None
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-Wall",
          "--expt-relaxed-constexpr", "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"),
@@ -35,9 +49,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     objs = []
     os.makedirs(os.path.join(ROOT, "build"), exist_ok=True)
+    nccl = _nccl_dir()
+    extra, link = [], []
+    if nccl:
+        extra = ["-DOPP_WITH_NCCL", "-I", os.path.join(nccl, "include")]
+        link = ["-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
+                "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     for src in SOURCES:
         obj = os.path.join(ROOT, "build", src.replace(".cu", ".o"))
-        cmd = [NVCC, *ARCH, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
+        cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
@@ -45,7 +65,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         if verbose:
             sys.stderr.write(r.stderr)
         objs.append(obj)
-    cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-cudart", "static"]
+    cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-cudart", "static", *link]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

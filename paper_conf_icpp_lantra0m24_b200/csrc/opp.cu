@@ -12,6 +12,7 @@
 
 #include <algorithm>
 #include <cstdarg>
+#include <cstdlib>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -70,9 +71,14 @@ struct PSet {
     int32_t *work_hops = nullptr;
     int32_t *sr_cell = nullptr;
     double *sr_val = nullptr;
+    uint32_t *mig = nullptr;     // nranks > 1: migrants of the current round
+    int32_t *mig_cell = nullptr, *mig_hops = nullptr;
     char *staging = nullptr;
     size_t staging_bytes = 0;
     std::vector<int> cols;
+    std::vector<char *> alt;     // sort double buffers (one per column, lazily allocated)
+    long long alt_cap = 0;
+    long long steps = 0;         // pushes so far (drives sort_every)
 };
 
 struct Set {
@@ -95,8 +101,9 @@ struct MeshCache {
     bool ov_built = false;
     Overlay ov{};
     int32_t *ov_map = nullptr;
-    // SR
-    unsigned *sr_hist = nullptr, *sr_start = nullptr;
+    // per-cell counting (SR deposit and sort by cell)
+    unsigned *cell_hist = nullptr, *cell_start = nullptr;
+    unsigned long long *tile_sums = nullptr;
     double *sr_sorted = nullptr, *sr_cellsum = nullptr;
     int32_t *n2cs_ptr = nullptr, *n2cs = nullptr;
     long long sr_cap = 0;
@@ -109,6 +116,8 @@ struct opp_ctx_s {
     cudaStream_t s = nullptr;
     int nsm = 148;
     int bps = 0;                   // resident blocks / SM of the fused kernel
+    int tile_group = 8;            // OPP_TILE_GROUP: tiles per block visit (TileMap)
+    int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -201,6 +210,8 @@ extern "C" void opp_init_params_default(opp_init_params *p) {
     p->hop_budget_per_pass = 4;
     p->hop_cap = 1024;
     p->allow_growth = 1;
+    p->sort_every = 0;
+    p->tma_pipeline = 1;
 }
 
 extern "C" const char *opp_last_error(void) { return g_err.c_str(); }
@@ -223,13 +234,15 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (c->p.deposit_mode == OPP_DEP_AUTO) c->p.deposit_mode = OPP_DEP_ATOMIC;
     c->s = (cudaStream_t)params->cuda_stream;
     cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, params->device);
+    if (const char *tg = getenv("OPP_TILE_GROUP")) c->tile_group = std::max(1, atoi(tg));
+    if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         delete c;
         return fail(OPP_ERR_NOMEM, "cudaMallocHost");
     }
     if (params->nranks > 1) {
-        int r = opp::comm_init(&c->comm, params->nccl_unique_id, params->rank, params->nranks,
-                               params->device, g_err);
+        int r = opp::comm_init(&c->comm, params->transport, params->nccl_unique_id, params->rank,
+                               params->nranks, params->device, g_err);
         if (r != OPP_OK) {
             cudaFreeHost(c->hcnt);
             delete c;
@@ -250,6 +263,9 @@ static void free_pset(opp_ctx c, PSet &ps) {
     c->dfree(ps.work_hops, 4 * cap);
     c->dfree(ps.sr_cell, 4 * cap);
     c->dfree(ps.sr_val, 32 * cap);
+    c->dfree(ps.mig, 4 * cap);
+    c->dfree(ps.mig_cell, 4 * cap);
+    c->dfree(ps.mig_hops, 4 * cap);
     c->dfree(ps.staging, ps.staging_bytes);
     ps = PSet();
 }
@@ -258,14 +274,18 @@ extern "C" int opp_finalize(opp_ctx c) {
     if (!c) return OPP_OK;
     cudaSetDevice(c->p.device);
     cudaStreamSynchronize(c->s);
+    for (auto &ps : c->psets)
+        for (size_t j = 0; j < ps.alt.size(); j++)
+            c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
     for (auto &col : c->cols) c->dfree(col.d, col.bytes);
     for (auto &ps : c->psets) free_pset(c, ps);
     MeshCache &m = c->mc;
     c->dfree(m.lines, sizeof(WalkLine) * m.nc);
     c->dfree(m.efp, sizeof(double4) * m.nc);
     c->dfree(m.ov_map, 0);
-    c->dfree(m.sr_hist, 0);
-    c->dfree(m.sr_start, 0);
+    c->dfree(m.cell_hist, 0);
+    c->dfree(m.cell_start, 0);
+    c->dfree(m.tile_sums, 0);
     c->dfree(m.sr_sorted, 0);
     c->dfree(m.sr_cellsum, 0);
     c->dfree(m.n2cs_ptr, 0);
@@ -339,6 +359,12 @@ static int alloc_scratch(opp_ctx c, PSet &ps, long long cap) {
         ps.sr_val = (double *)c->dalloc(32 * n);
         if (!ps.sr_cell || !ps.sr_val) return fail(OPP_ERR_NOMEM, "SR scratch");
     }
+    if (c->p.nranks > 1) {
+        ps.mig = (uint32_t *)c->dalloc(4 * n);
+        ps.mig_cell = (int32_t *)c->dalloc(4 * n);
+        ps.mig_hops = (int32_t *)c->dalloc(4 * n);
+        if (!ps.mig || !ps.mig_cell || !ps.mig_hops) return fail(OPP_ERR_NOMEM, "migration scratch");
+    }
     return OPP_OK;
 }
 
@@ -350,6 +376,7 @@ extern "C" int opp_decl_particle_set(opp_ctx c, const char *name, opp_set cells,
     if (n_init < 0 || !out) return fail(OPP_ERR_ARG, "opp_decl_particle_set: bad n_init/out");
     if (capacity > 0 && capacity < n_init) return fail(OPP_ERR_ARG, "capacity < n_init");
     long long cap = std::max<long long>(std::max<long long>(n_init, capacity), 1024);
+    cap = (cap + 63) & ~63ll;   // 16-B aligned column segments for cp.async.bulk
     if (cap > 0xFFFFFFF0ll) return fail(OPP_ERR_ARG, "capacity above 2^32 indices");
     PSet ps;
     ps.cap = cap;
@@ -456,12 +483,31 @@ extern "C" int opp_decl_dat(opp_ctx c, opp_set set, int dim, int type, const voi
     return decl_col(c, false, set, -1, dim, type, host, name, out);
 }
 
-extern "C" int opp_set_partition(opp_ctx c, opp_set cells, const int32_t *rank_of_cell) {
+extern "C" int opp_set_partition(opp_ctx c, opp_set cells, int64_t n_global_cells,
+                                 const int32_t *rank_of_cell, opp_set nodes,
+                                 const int64_t *node_gid) {
     TRY(ctx_check(c));
     TRY(set_check(c, cells));
-    if (!rank_of_cell) return fail(OPP_ERR_ARG, "rank_of_cell is NULL");
-    return opp::comm_set_partition(c->comm, c->p.rank, c->p.nranks, c->sets[cells].size,
-                                   rank_of_cell, &c->cell_base, g_err);
+    TRY(set_check(c, nodes));
+    if (!rank_of_cell || n_global_cells < 0) return fail(OPP_ERR_ARG, "bad rank_of_cell");
+    if (c->sets[cells].particle || c->sets[nodes].particle)
+        return fail(OPP_ERR_ARG, "partition applies to mesh sets");
+    if (c->p.nranks > 1 && !node_gid) return fail(OPP_ERR_ARG, "node_gid required for nranks > 1");
+    if (c->p.nranks == 1) {
+        for (long long g = 0; g < n_global_cells; g++)
+            if (rank_of_cell[g] != 0) return fail(OPP_ERR_ARG, "single rank: rank_of_cell must be 0");
+        if (n_global_cells != c->sets[cells].size)
+            return fail(OPP_ERR_ARG, "single rank owns every cell");
+        c->cell_base = 0;
+        return OPP_OK;
+    }
+    int base = 0;
+    int r = opp::comm_set_partition(c->comm, n_global_cells, rank_of_cell, c->sets[cells].size,
+                                    c->sets[nodes].size, node_gid, &base, c->s, g_err);
+    if (r != OPP_OK) return r;
+    c->cell_base = base;
+    c->mc.c2c = -1;   // rebuild the walk lines (validation uses the base)
+    return OPP_OK;
 }
 
 // ---------------------------------------------------------------------------
@@ -498,6 +544,7 @@ static int grow(opp_ctx c, PSet &ps, long long extra) {
     if (need <= ps.cap) return OPP_OK;
     if (!ps.growth) return fail(OPP_ERR_CAPACITY, "capacity %lld < %lld", ps.cap, need);
     long long ncap = std::max<long long>(need, ps.cap + ps.cap / 2);
+    ncap = (ncap + 63) & ~63ll;
     if (ncap > 0xFFFFFFF0ll) return fail(OPP_ERR_CAPACITY, "capacity above 2^32 indices");
     // allocate everything first so failure leaves the state unchanged
     std::vector<char *> nd(ps.cols.size(), nullptr);
@@ -531,11 +578,32 @@ static int grow(opp_ctx c, PSet &ps, long long extra) {
         col.bytes = (size_t)ncap * col.dim * col.eb;
     }
     size_t oc = (size_t)ps.cap;
+    // scratch contents survive (growth can happen mid-step, during migration)
+    CK(cudaMemcpyAsync(tmp.holes, ps.holes, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+    CK(cudaMemcpyAsync(tmp.work, ps.work, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+    CK(cudaMemcpyAsync(tmp.work_hops, ps.work_hops, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+    if (ps.sr_cell) {
+        CK(cudaMemcpyAsync(tmp.sr_cell, ps.sr_cell, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+        CK(cudaMemcpy2DAsync(tmp.sr_val, 8 * (size_t)ncap, ps.sr_val, 8 * oc, 8 * oc, 4,
+                             cudaMemcpyDeviceToDevice, c->s));
+    }
+    if (ps.mig) {
+        CK(cudaMemcpyAsync(tmp.mig, ps.mig, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+        CK(cudaMemcpyAsync(tmp.mig_cell, ps.mig_cell, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+        CK(cudaMemcpyAsync(tmp.mig_hops, ps.mig_hops, 4 * oc, cudaMemcpyDeviceToDevice, c->s));
+    }
+    CK(cudaStreamSynchronize(c->s));
     c->dfree(ps.holes, 4 * oc); c->dfree(ps.work, 4 * oc); c->dfree(ps.head, 4 * oc);
     c->dfree(ps.tail, 4 * oc); c->dfree(ps.work_hops, 4 * oc);
     c->dfree(ps.sr_cell, 4 * oc); c->dfree(ps.sr_val, 32 * oc);
+    c->dfree(ps.mig, 4 * oc); c->dfree(ps.mig_cell, 4 * oc); c->dfree(ps.mig_hops, 4 * oc);
     ps.holes = tmp.holes; ps.work = tmp.work; ps.head = tmp.head; ps.tail = tmp.tail;
     ps.work_hops = tmp.work_hops; ps.sr_cell = tmp.sr_cell; ps.sr_val = tmp.sr_val;
+    ps.mig = tmp.mig; ps.mig_cell = tmp.mig_cell; ps.mig_hops = tmp.mig_hops;
+    for (size_t j = 0; j < ps.alt.size(); j++)
+        c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
+    ps.alt.clear();
+    ps.alt_cap = 0;
     ps.cap = ncap;
     return OPP_OK;
 }
@@ -661,10 +729,14 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         m.vpos = np.version;
         m.ov_built = false;
         if (m.sr_cellsum) {
-            c->dfree(m.n2cs_ptr, 0); c->dfree(m.n2cs, 0);
-            c->dfree(m.sr_hist, 0); c->dfree(m.sr_start, 0); c->dfree(m.sr_cellsum, 0);
+            c->dfree(m.n2cs_ptr, 0); c->dfree(m.n2cs, 0); c->dfree(m.sr_cellsum, 0);
             m.sr_cellsum = nullptr;
         }
+        c->dfree(m.cell_hist, 0); c->dfree(m.cell_start, 0); c->dfree(m.tile_sums, 0);
+        m.cell_hist = (unsigned *)c->dalloc(4 * (nc + 1));
+        m.cell_start = (unsigned *)c->dalloc(4 * (nc + 1));
+        m.tile_sums = (unsigned long long *)c->dalloc(8 * opp::scan_tiles(nc + 1));
+        if (!m.cell_hist || !m.cell_start || !m.tile_sums) return fail(OPP_ERR_NOMEM, "cell counters");
     }
     if (m.ef != cell_ef || m.vef != ef.version) {
         CK(launch_pack_field((const double *)ef.d, nc, m.efp, c->s));
@@ -715,10 +787,8 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         for (long long e = 0; e < 4 * nc; e++) idx[cur[h[e]]++] = (int32_t)e;
         m.n2cs_ptr = (int32_t *)c->dalloc(4 * (nn + 1));
         m.n2cs = (int32_t *)c->dalloc(4 * std::max<long long>(4 * nc, 1));
-        m.sr_hist = (unsigned *)c->dalloc(4 * (nc + 1));
-        m.sr_start = (unsigned *)c->dalloc(4 * (nc + 1));
         m.sr_cellsum = (double *)c->dalloc(32 * std::max<long long>(nc, 1));
-        if (!m.n2cs_ptr || !m.n2cs || !m.sr_hist || !m.sr_start || !m.sr_cellsum)
+        if (!m.n2cs_ptr || !m.n2cs || !m.sr_cellsum)
             return fail(OPP_ERR_NOMEM, "SR mesh buffers");
         CK(cudaMemcpyAsync(m.n2cs_ptr, ptr.data(), 4 * (nn + 1), cudaMemcpyHostToDevice, c->s));
         CK(cudaMemcpyAsync(m.n2cs, idx.data(), 4 * 4 * nc, cudaMemcpyHostToDevice, c->s));
@@ -743,13 +813,175 @@ static int check_col(opp_ctx c, int h, bool want_map, int set, int dim, int type
     return OPP_OK;
 }
 
+// Counting sort by cell into the double buffers, then swap (drops holes).
+static int do_sort(opp_ctx c, PSet &ps, int p2c) {
+    MeshCache &m = c->mc;
+    if (!m.cell_hist) return fail(OPP_ERR_STATE, "sort needs the mesh: run a step first");
+    if (ps.alt_cap != ps.cap) {
+        for (size_t j = 0; j < ps.alt.size(); j++)
+            c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
+        ps.alt.assign(ps.cols.size(), nullptr);
+        for (size_t j = 0; j < ps.cols.size(); j++) {
+            Col &col = c->cols[ps.cols[j]];
+            ps.alt[j] = (char *)c->dalloc((size_t)ps.cap * col.dim * col.eb);
+            if (!ps.alt[j]) {
+                for (size_t k = 0; k < j; k++)
+                    c->dfree(ps.alt[k], (size_t)ps.cap * c->cols[ps.cols[k]].dim * c->cols[ps.cols[k]].eb);
+                ps.alt.clear();
+                ps.alt_cap = 0;
+                return fail(OPP_ERR_NOMEM, "sort buffers");
+            }
+        }
+        ps.alt_cap = ps.cap;
+    }
+    ColSet src = make_colset(c, ps), dst = src;
+    for (int j = 0; j < dst.n; j++) dst.c[j].ptr = ps.alt[j];
+    const int32_t *pc = (const int32_t *)c->cols[p2c].d;
+    {
+        PhaseScope ph(c, OPP_PH_SORT_COUNT);
+        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.cell_hist, m.cell_start,
+                             m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
+    }
+    {
+        PhaseScope ph(c, OPP_PH_SORT_MOVE);
+        CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.cell_start, ps.head,
+                            grid_for(c, ps.n_ub, 8), c->s));
+    }
+    c->launches += 7;
+    for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
+    ps.holes_pending = false;
+    return OPP_OK;
+}
+
 static int do_fill(opp_ctx c, PSet &ps, int p2c) {
     PhaseScope ph(c, OPP_PH_FILL);
+    if (c->p.sort_every > 0 && ps.steps % c->p.sort_every == 0) return do_sort(c, ps, p2c);
     ColSet cs = make_colset(c, ps);
     CK(launch_fill(cs, ps.dcnt, ps.holes, (const int32_t *)c->cols[p2c].d, ps.head, ps.tail,
                    grid_for(c, ps.n_ub, 4), c->s));
     c->launches += 2;
     ps.holes_pending = false;
+    return OPP_OK;
+}
+
+static int p2c_of(opp_ctx c, PSet &ps) {
+    for (int h : ps.cols)
+        if (c->cols[h].is_map) return h;
+    return -1;
+}
+
+extern "C" int opp_sort_by_cell(opp_ctx c, opp_set parts) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
+    PSet &ps = c->psets[S.pset];
+    int p2c = p2c_of(c, ps);
+    if (p2c < 0) return fail(OPP_ERR_STATE, "particle set has no p2c map");
+    if (!ps.holes_pending) {
+        // no holes: the sort still needs n_holes = 0 on the device (it is)
+    }
+    PhaseScope ph(c, OPP_PH_FILL);
+    return do_sort(c, ps, p2c);
+}
+
+// Refresh the particle-side pointers of the step arguments (after growth).
+static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int p2c) {
+    a.pos = (double *)c->cols[pos].d;
+    a.vel = (double *)c->cols[vel].d;
+    a.p2c = (int32_t *)c->cols[p2c].d;
+    a.cap = ps.cap;
+    a.holes = ps.holes;
+    a.work = ps.work;
+    a.work_hops = ps.work_hops;
+    a.sr_cell = ps.sr_cell;
+    a.sr_val = ps.sr_val;
+    a.mig = ps.mig;
+    a.mig_cell = ps.mig_cell;
+    a.mig_hops = ps.mig_hops;
+}
+
+// Particle migration (Fig. 7a): after the walk, particles
+// that entered another rank's cells are packed (every column + hop count),
+// exchanged point-to-point, appended at the end of the receiver's dats and
+// walked on there; repeated until no rank has migrants.
+static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, bool dh, int p2c, int cgrid) {
+    opp::Comm *cm = c->comm;
+    const int R = cm->nranks, me = cm->rank;
+    int p2c_col = -1, rec = 0, pos = -1, vel = -1;
+    for (size_t j = 0; j < ps.cols.size(); j++) {
+        const Col &col = c->cols[ps.cols[j]];
+        if (ps.cols[j] == p2c) p2c_col = (int)j;
+        rec = (rec + col.eb - 1) & ~(col.eb - 1);    // same layout as k_mig_pack
+        rec += col.dim * col.eb;
+        if ((double *)col.d == a.pos) pos = ps.cols[j];
+        if ((double *)col.d == a.vel) vel = ps.cols[j];
+    }
+    rec += 4;                                        // hop count
+    rec = (rec + 7) & ~7;
+    std::vector<int64_t> row(R), soff(R), sbytes(R), roff(R), rbytes(R);
+    std::vector<unsigned long long> hrow(R);
+    for (int round = 0;; round++) {
+        CK(launch_mig_count(a.mig_cell, ps.dcnt, cm->rr, cm->d_counts, grid_for(c, ps.n_ub, 2), c->s));
+        CK(cudaMemcpyAsync(hrow.data(), cm->d_counts, 8 * R, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        c->launches++;
+        for (int q = 0; q < R; q++) row[q] = (int64_t)hrow[q];
+        TRY(cm->t->allgather_i64(row.data(), R, cm->counts_host.data(), c->s, g_err));
+        const int64_t *M = cm->counts_host.data();
+        int64_t total = 0, out = 0, in = 0;
+        for (int k = 0; k < R * R; k++) total += M[k];
+        if (total == 0) break;
+        for (int q = 0; q < R; q++) {
+            soff[q] = out * rec;
+            sbytes[q] = M[me * R + q] * rec;
+            out += M[me * R + q];
+            roff[q] = in * rec;
+            rbytes[q] = M[q * R + me] * rec;
+            in += M[q * R + me];
+        }
+        TRY(opp::comm_reserve(&cm->sendbuf, &cm->send_cap, (size_t)std::max<int64_t>(out, 1) * rec, g_err));
+        TRY(opp::comm_reserve(&cm->recvbuf, &cm->recv_cap, (size_t)std::max<int64_t>(in, 1) * rec, g_err));
+        std::vector<unsigned long long> cur(R);
+        for (int q = 0; q < R; q++) cur[q] = (unsigned long long)(soff[q] / rec);
+        CK(cudaMemcpyAsync(cm->d_cursor, cur.data(), 8 * R, cudaMemcpyHostToDevice, c->s));
+        ColSet cs = make_colset(c, ps);
+        CK(launch_mig_pack(cs, p2c_col, a.mig, a.mig_cell, a.mig_hops, ps.dcnt, cm->rr, cm->d_cursor,
+                           cm->sendbuf, rec, grid_for(c, out, 2), c->s));
+        c->launches++;
+        if (ps.n_ub + in > ps.cap) {
+            TRY(grow(c, ps, in));
+            refresh_args(c, ps, a, pos, vel, p2c);
+            cs = make_colset(c, ps);
+        }
+        TRY(cm->t->exchange(cm->sendbuf, soff, sbytes, cm->recvbuf, roff, rbytes, c->s, g_err));
+        CK(launch_mig_unpack(cs, cm->recvbuf, in, rec, ps.dcnt, a.work, a.work_hops,
+                             grid_for(c, in, 2), c->s));
+        ps.n_ub += in;
+        ps.n_exact = false;
+        CK(launch_push_move_deposit(dep, dh, true, true, false, a, cgrid, c->s));
+        c->launches += 2;
+        if (round > 64 * R) return fail(OPP_ERR_STATE, "migration did not terminate");
+    }
+    return OPP_OK;
+}
+
+// Node-charge halo: exchange the interface nodes'
+// partial sums with each neighbour and add them (a + b = b + a: both copies
+// of a node end bit-identical when two ranks share it).
+static int halo_sum(opp_ctx c, double *Q) {
+    opp::Comm *cm = c->comm;
+    const int R = cm->nranks;
+    CK(launch_halo_pack(Q, cm->d_halo_idx, cm->halo_n, cm->d_halo_send, c->s));
+    std::vector<int64_t> off(R), bytes(R);
+    for (int p = 0; p < R; p++) {
+        off[p] = 8 * cm->halo_off[p];
+        bytes[p] = 8 * cm->halo_cnt[p];
+    }
+    TRY(cm->t->exchange((const char *)cm->d_halo_send, off, bytes, (char *)cm->d_halo_recv, off, bytes,
+                        c->s, g_err));
+    CK(launch_halo_add(Q, cm->d_halo_idx, cm->halo_n, cm->d_halo_recv, c->s));
+    c->launches += 2;
     return OPP_OK;
 }
 
@@ -818,6 +1050,9 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.work_hops = ps.work_hops;
     a.sr_cell = ps.sr_cell;
     a.sr_val = ps.sr_val;
+    a.mig = ps.mig;
+    a.mig_cell = ps.mig_cell;
+    a.mig_hops = ps.mig_hops;
     a.c1 = prm->qm * prm->dt;
     a.dt = prm->dt;
     a.w = prm->weight;
@@ -825,42 +1060,51 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.n_cells = (int)m.nc;
     a.hpass = c->p.hop_budget_per_pass;
     a.hcap = c->p.hop_cap;
+    a.tile_group = c->tile_group;
+    a.dbg = c->dbg;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const bool dh = c->p.direct_hop != 0;
     const bool multi = c->p.nranks > 1;
+    if (multi && !c->comm->partitioned) return fail(OPP_ERR_STATE, "nranks > 1: call opp_set_partition first");
 
     {
         PhaseScope ph(c, OPP_PH_BEGIN);
         CK(launch_step_begin(a.Q, nn, ps.dcnt, prm->zero_charge, grid_for(c, nn, 2), c->s));
     }
     c->launches++;
-    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(dep, dh);
+    const bool tiled = c->p.tma_pipeline != 0;
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled);
     const int bps = c->bps;
     const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
                                                                        (long long)c->nsm * bps));
     {
         PhaseScope ph(c, OPP_PH_PUSH_MOVE_DEPOSIT);
-        CK(launch_push_move_deposit(dep, dh, multi, false, a, pgrid, c->s));
+        const int g1 = tiled ? c->nsm * bps : pgrid;
+        CK(launch_push_move_deposit(dep, dh, multi, false, tiled, a, g1, c->s));
     }
     {
         PhaseScope ph(c, OPP_PH_CONTINUE);
-        CK(launch_push_move_deposit(dep, dh, multi, true, a,
+        CK(launch_push_move_deposit(dep, dh, multi, true, false, a,
                                     std::max(1, std::min(pgrid, c->nsm * 2)), c->s));
     }
     c->launches += 2;
     if (multi) {
         PhaseScope ph(c, OPP_PH_MIGRATE);
-        int r = opp::comm_migrate(c->comm, &a, c->s, g_err);
-        if (r != OPP_OK) return r;
+        TRY(migrate_loop(c, ps, a, dep, dh, p2c, std::max(1, std::min(pgrid, c->nsm * 2))));
     }
     if (dep == OPP_DEP_SORT_SEGRED) {
         PhaseScope ph(c, OPP_PH_SEGRED);
-        CK(launch_sr(a, m.nc, nn, m.sr_hist, m.sr_start, m.sr_sorted, m.sr_cellsum, m.n2cs_ptr,
-                     m.n2cs, grid_for(c, ps.n_ub, 8), c->s));
+        CK(launch_sr(a, m.nc, nn, m.cell_hist, m.cell_start, m.tile_sums, m.sr_sorted,
+                     m.sr_cellsum, m.n2cs_ptr, m.n2cs, grid_for(c, ps.n_ub, 8), c->s));
         c->launches += 5;
     }
+    if (multi && c->comm->halo_n > 0) {
+        PhaseScope ph(c, OPP_PH_HALO);
+        TRY(halo_sum(c, a.Q));
+    }
     ps.holes_pending = true;
+    ps.steps++;
     if (prm->fill_inline) TRY(do_fill(c, ps, p2c));
     if (stats) TRY(read_stats(c, ps, stats));
     return OPP_OK;
@@ -882,9 +1126,7 @@ extern "C" int opp_fill_holes(opp_ctx c, opp_set parts, int64_t *n_after) {
     if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
     PSet &ps = c->psets[S.pset];
     if (ps.holes_pending) {
-        int p2c = -1;
-        for (int h : ps.cols)
-            if (c->cols[h].is_map) p2c = h;
+        int p2c = p2c_of(c, ps);
         if (p2c < 0) return fail(OPP_ERR_STATE, "particle set has no p2c map");
         TRY(do_fill(c, ps, p2c));
     }

@@ -38,9 +38,11 @@ struct DevCounters {
     unsigned long long n_sr;             // SR deposit: number of stored records
     unsigned long long cum_pushed;       // sum of n_before over all steps
     unsigned long long cum_steps;
+    unsigned long long n_mig;            // migrants recorded (current round)
+    unsigned long long unpack_done_blocks;
     unsigned int max_hops;
     unsigned int err_flags;              // bit 0: non-positive tet, bit 1: SR overflow
-    unsigned long long pad[11];
+    unsigned long long pad[9];
 };
 
 constexpr int kMaxCols = 16;
@@ -82,10 +84,23 @@ struct StepArgs {
     int32_t *work_hops;        // [cap]
     int32_t *sr_cell;          // SR records (cell, 4 values)
     double *sr_val;            // [4][cap]
+    uint32_t *mig;             // migrants: particle index, target global cell, hops
+    int32_t *mig_cell;
+    int32_t *mig_hops;
     double c1, dt, w;
     int cell_base, n_cells;    // global id of local cell 0, local cell count
     int hpass, hcap;
+    int tile_group;            // consecutive 256-particle tiles per block visit (>= 1)
+    int dbg;                   // diagnostics only (OPP_PMD_DEBUG): 1 stream, 2 +E, 3 +line, 4 no deposit
     Overlay ov;
+};
+
+// Slab partition: rank r owns global cells [lo[r], hi[r]).
+constexpr int kMaxRanks = 64;
+struct RankRanges {
+    int lo[kMaxRanks];
+    int hi[kMaxRanks];
+    int n;
 };
 
 }  // namespace opp

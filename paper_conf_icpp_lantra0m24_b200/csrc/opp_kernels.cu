@@ -14,13 +14,14 @@
 #include "opp_internal.h"
 #include "opp_kernels.h"
 
+#include <algorithm>
 #include <climits>
 
 namespace opp {
 
 namespace {
 
-constexpr int ST_DONE = 0, ST_MOVE = 1, ST_REMOVE = 2, ST_MIGRATE = 3;
+constexpr int ST_DONE = 0, ST_MOVE = 1, ST_REMOVE = 2, ST_MIGRATE = 3, ST_NONE = 100;
 
 __device__ __forceinline__ double mul(double a, double b) { return __dmul_rn(a, b); }
 __device__ __forceinline__ double add(double a, double b) { return __dadd_rn(a, b); }
@@ -31,16 +32,20 @@ struct Line {
     int4 cc, cn;
 };
 
+// One 128-B walk line in four 256-bit read-only loads (LDG.E.256 on sm_100:
+// half the L1 wavefronts of 16-B vector loads).
 __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, int c) {
-    const double2 *L = reinterpret_cast<const double2 *>(lines + c);
-    double2 a0 = __ldg(L + 0), a1 = __ldg(L + 1), a2 = __ldg(L + 2);
-    double2 a3 = __ldg(L + 3), a4 = __ldg(L + 4), a5 = __ldg(L + 5);
-    const int4 *I = reinterpret_cast<const int4 *>(L + 6);
+    const double *L = reinterpret_cast<const double *>(lines + c);
     Line l;
-    l.g0 = a0.x; l.g1 = a0.y; l.g2 = a1.x; l.g3 = a1.y; l.g4 = a2.x; l.g5 = a2.y;
-    l.g6 = a3.x; l.g7 = a3.y; l.g8 = a4.x; l.px = a4.y; l.py = a5.x; l.pz = a5.y;
-    l.cc = __ldg(I);
-    l.cn = __ldg(I + 1);
+    asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(l.g0), "=d"(l.g1), "=d"(l.g2), "=d"(l.g3) : "l"(L));
+    asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(l.g4), "=d"(l.g5), "=d"(l.g6), "=d"(l.g7) : "l"(L + 4));
+    asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(l.g8), "=d"(l.px), "=d"(l.py), "=d"(l.pz) : "l"(L + 8));
+    asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(l.cc.x), "=r"(l.cc.y), "=r"(l.cc.z), "=r"(l.cc.w),
+          "=r"(l.cn.x), "=r"(l.cn.y), "=r"(l.cn.z), "=r"(l.cn.w) : "l"(L + 12));
     return l;
 }
 
@@ -57,15 +62,15 @@ __device__ __forceinline__ void bary(const Line &l, double x, double y, double z
 __device__ __forceinline__ bool in01(double v) { return v >= 0.0 && v <= 1.0; }
 
 // Multi-hop walk (Fig. 6 template 1098-1124).  `cell` is a
-// global id in/out; stops when inside (DONE), at H_cap (DONE, capped), when
-// hops reaches stop_at (NEED_MOVE: deferred), across a boundary face
-// (NEED_REMOVE) or into a cell another rank owns (NEED_MIGRATE).
+// global id in/out and L its already-loaded walk line; stops when inside
+// (DONE), at H_cap (DONE, capped), when hops reaches stop_at (NEED_MOVE:
+// deferred), across a boundary face (NEED_REMOVE) or into a cell another
+// rank owns (NEED_MIGRATE).
 template <bool MULTI>
-__device__ __forceinline__ int walk(const StepArgs &a, int &cell, double x, double y, double z,
-                                    int &hops, int stop_at, double &l0, double &l1, double &l2,
-                                    double &l3, int &capped, int4 &cn) {
+__device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, double x, double y,
+                                         double z, int &hops, int stop_at, double &l0, double &l1,
+                                         double &l2, double &l3, int &capped, int4 &cn) {
     for (;;) {
-        Line L = load_line(a.lines, cell - a.cell_base);
         bary(L, x, y, z, l0, l1, l2, l3);
         cn = L.cn;
         if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) return ST_DONE;
@@ -86,6 +91,7 @@ __device__ __forceinline__ int walk(const StepArgs &a, int &cell, double x, doub
         }
         cell = nb;
         hops++;
+        L = load_line(a.lines, cell - a.cell_base);
     }
 }
 
@@ -191,39 +197,367 @@ __device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, do
 }  // namespace
 
 // ---------------------------------------------------------------------------
-// The fused push / move / deposit kernel (CalcPosVel + Move + DepositCharge,
-// PAPER.md:1586-1604, fused).  CONT = continuation pass over the worklist.
+// Per-particle body shared by the fused kernel (both its TMA-tiled and its
+// direct paths) and the continuation pass.  Must be called by full warps
+// (the deposit / append collectives use all 32 lanes); `valid` masks lanes
+// without a particle.  On return x..vz and cell hold what is written back
+// (cell = -1 for a hole).
 // ---------------------------------------------------------------------------
+struct Tally {
+    unsigned hops = 0, maxh = 0, capped = 0, removed = 0;
+};
+
+// Block b visits groups of K consecutive tiles round-robin: group g goes to
+// block g % G.  K = 1 sweeps the array as one moving window (small L2 working
+// set when storage is cell-sorted); larger K gives each SM runs of adjacent
+// cells (L1 reuse) while the window stays G*K tiles.
+struct TileMap {
+    unsigned long long ntiles, G, K, b;
+    __device__ __forceinline__ unsigned long long count() const {
+        const unsigned long long ng = (ntiles + K - 1) / K;
+        if (b >= ng) return 0;
+        const unsigned long long nb = (ng - 1 - b) / G + 1;
+        unsigned long long c = nb * K;
+        if (b + (nb - 1) * G == ng - 1) c -= ng * K - ntiles;
+        return c;
+    }
+    __device__ __forceinline__ unsigned long long tile(unsigned long long it) const {
+        return ((it / K) * G + b) * K + it % K;
+    }
+};
+
+template <int DEP, bool DH, bool CONT, bool MULTI>
+__device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
+                                         int hops, double &x, double &y, double &z, double &vx,
+                                         double &vy, double &vz, int &cell, Tally &t) {
+    int status = ST_NONE;
+    int capped = 0;
+    double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
+    int4 cn = make_int4(0, 0, 0, 0);
+    if (valid && a.dbg == 1) {   // diagnostic: stream only
+        vx = add(vx, a.c1); x = add(x, mul(vx, a.dt));
+        a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+        a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+        valid = false;
+    }
+    if (valid && a.dbg == 2) {   // diagnostic: stream + E gather
+        const double *Ep = reinterpret_cast<const double *>(a.ef + (cell - a.cell_base));
+        vx = add(vx, mul(a.c1, __ldg(Ep))); x = add(x, mul(vx, a.dt));
+        a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+        a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+        valid = false;
+    }
+    if (valid) {
+        const int lc = cell - a.cell_base;
+        Line L = load_line(a.lines, lc);            // first visit: issued with E
+        if (!CONT) {
+            // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
+            const double *Ep = reinterpret_cast<const double *>(a.ef + lc);
+            const double2 Exy = __ldg(reinterpret_cast<const double2 *>(Ep));
+            const double Ez = __ldg(Ep + 2);
+            vx = add(vx, mul(a.c1, Exy.x));
+            vy = add(vy, mul(a.c1, Exy.y));
+            vz = add(vz, mul(a.c1, Ez));
+            x = add(x, mul(vx, a.dt));
+            y = add(y, mul(vy, a.dt));
+            z = add(z, mul(vz, a.dt));
+            // position and velocity are final now: store them before the walk
+            a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+            a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+            if (DH) {
+                const int sc = dh_seed(a.ov, x, y, z, cell);
+                if (sc != cell) {
+                    cell = sc;
+                    L = load_line(a.lines, sc - a.cell_base);
+                }
+            }
+        }
+        status = walk_from<MULTI>(a, cell, L, x, y, z, hops,
+                                  a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass), l0, l1, l2, l3,
+                                  capped, cn);
+        if (a.dbg == 3 && status == ST_MOVE) status = ST_DONE;
+        if (status != ST_MOVE && status != ST_MIGRATE) {   // counted where the walk ends
+            t.hops += (unsigned)hops;
+            t.maxh = max(t.maxh, (unsigned)hops);
+            t.capped += (unsigned)capped;
+        }
+        t.removed += (status == ST_REMOVE);
+    }
+    const bool done = status == ST_DONE && a.dbg == 0;
+    if (DEP == 2) {
+        sr_store(a, done, cell, a.w, l0, l1, l2, l3);
+    } else {
+        deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+    }
+    // holes, the deferred-walk worklist, migrants
+    const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
+    unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
+    if (rem) a.holes[hs] = (uint32_t)i;
+    if (!CONT) {
+        const bool mv = status == ST_MOVE;
+        unsigned long long ws = warp_append(mv, &a.cnt->n_work);
+        if (mv) {
+            a.work[ws] = (uint32_t)i;
+            a.work_hops[ws] = hops;
+        }
+    }
+    if (MULTI) {
+        const bool mg = status == ST_MIGRATE;
+        unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
+        if (mg) {
+            a.mig[ms] = (uint32_t)i;
+            a.mig_cell[ms] = cell;
+            a.mig_hops[ms] = hops;
+        }
+    }
+    if (rem) cell = -1;
+}
+
+// ---------------------------------------------------------------------------
+// Direct-load variant: warps stride over [lo, hi) one particle per lane; the
+// next particle's state is loaded before the current one walks (a register
+// double buffer), so the HBM stream stays in flight during the latency-bound
+// walk.  Used for the continuation pass, the ragged tail of the tiled
+// kernel, and as the non-TMA variant of pass 1.
+// ---------------------------------------------------------------------------
+struct PState {
+    double x, y, z, vx, vy, vz;
+    int cell, hops;
+    unsigned long long i;
+    bool valid;
+};
+
+template <bool CONT>
+__device__ __forceinline__ void load_pstate(const StepArgs &a, unsigned long long k,
+                                            unsigned long long hi, PState &p) {
+    p.valid = k < hi;
+    p.i = k;
+    p.hops = 0;
+    p.cell = 0;
+    p.x = p.y = p.z = p.vx = p.vy = p.vz = 0.0;
+    if (p.valid) {
+        if (CONT) {
+            p.i = a.work[k];
+            p.hops = a.work_hops[k];
+        }
+        p.x = a.pos[p.i]; p.y = a.pos[a.cap + p.i]; p.z = a.pos[2 * a.cap + p.i];
+        if (!CONT) { p.vx = a.vel[p.i]; p.vy = a.vel[a.cap + p.i]; p.vz = a.vel[2 * a.cap + p.i]; }
+        p.cell = a.p2c[p.i];
+    }
+}
+
+template <int DEP, bool DH, bool CONT, bool MULTI>
+__device__ __forceinline__ void pmd_direct_range(const StepArgs &a, unsigned long long lo,
+                                                 unsigned long long hi, unsigned long long first,
+                                                 unsigned long long stride, Tally &t) {
+    unsigned long long i0 = lo + first;
+    if (i0 >= hi) return;
+    PState cur;
+    load_pstate<CONT>(a, i0 + lane_id(), hi, cur);
+    for (; i0 < hi; i0 += stride) {
+        PState nxt;
+        const bool more = i0 + stride < hi;
+        if (more) load_pstate<CONT>(a, i0 + stride + lane_id(), hi, nxt);
+        pmd_body<DEP, DH, CONT, MULTI>(a, cur.valid, cur.i, cur.hops, cur.x, cur.y, cur.z, cur.vx,
+                                       cur.vy, cur.vz, cur.cell, t);
+        if (cur.valid) a.p2c[cur.i] = cur.cell;
+        if (more) cur = nxt;
+    }
+}
+
+// Pass 1 (direct variant): every block owns one contiguous chunk of the
+// particle array, so in cell-sorted storage the walk lines a block touches
+// stay hot in its SM's L1.  Continuation: grid-stride over the worklist.
 template <int DEP, bool DH, bool CONT, bool MULTI>
 __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
-    const unsigned long long n = CONT ? *(volatile unsigned long long *)&a.cnt->n_work
-                                      : *(volatile unsigned long long *)&a.cnt->n;
+    Tally t;
+    if (CONT) {
+        const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n_work;
+        pmd_direct_range<DEP, DH, true, MULTI>(
+            a, 0, n, (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u),
+            (unsigned long long)gridDim.x * blockDim.x, t);
+    } else {
+        const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
+        const TileMap tm{(n + 255) / 256, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
+        const unsigned long long my = tm.count();
+        for (unsigned long long it = 0; it < my; it++) {
+            const unsigned long long lo = tm.tile(it) * 256;
+            pmd_direct_range<DEP, DH, false, MULTI>(a, lo, lo + 256 < n ? lo + 256 : n,
+                                                    threadIdx.x & ~31u, 256, t);
+        }
+    }
+    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
+}
+
+// ---------------------------------------------------------------------------
+// The fused push / move / deposit kernel, TMA-pipelined (CalcPosVel + Move +
+// DepositCharge of PAPER.md:1586-1604 in one pass).  Each block owns a
+// contiguous range of kTile-particle tiles (L1 locality of the walk lines in
+// cell-sorted storage).  A producer warp streams each tile's 7 SoA column
+// segments global -> shared with cp.async.bulk (complete_tx on the stage's
+// `full` mbarrier) up to kStages tiles ahead; each of the 8 consumer warps
+// copies its 32 particles out of the stage, releases it (`empty` mbarrier,
+// one arrival per warp) and then pushes / walks / deposits, storing results
+// with coalesced stores.  No block-wide barrier inside the loop: a warp whose
+// lanes walk far never stalls the others.  The ragged tail (< kTile) takes
+// the direct path.
+// ---------------------------------------------------------------------------
+constexpr int kTile = 256;
+constexpr int kConsumerWarps = kTile / 32;
+constexpr int kTiledThreads = kTile + 32;
+constexpr int kStages = 4;
+constexpr int kStageBytes = kTile * (6 * 8 + 4);
+constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)),
+                 "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+    } while (!done);
+}
+// producer-side wait: back off so the spinning lane does not steal issue slots
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) {
+    uint32_t done;
+    for (;;) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+        if (done) return;
+        __nanosleep(64);
+    }
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+struct StageView {
+    double *c[6];   // x, y, z, vx, vy, vz
+    int *cell;
+};
+__device__ __forceinline__ StageView stage_view(char *smem, int s) {
+    StageView v;
+    char *b = smem + (size_t)s * kStageBytes;
+    for (int k = 0; k < 6; k++) v.c[k] = reinterpret_cast<double *>(b + k * kTile * 8);
+    v.cell = reinterpret_cast<int *>(b + 6 * kTile * 8);
+    return v;
+}
+
+// producer: load tile `tile` into stage s
+__device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, uint64_t *full,
+                                                int s, unsigned long long tile) {
+    StageView v = stage_view(smem, s);
+    const unsigned long long base = tile * kTile;
+    mbar_expect_tx(&full[s], kStageBytes);
+    for (int k = 0; k < 3; k++) {
+        bulk_g2s(v.c[k], a.pos + k * a.cap + base, kTile * 8, &full[s]);
+        bulk_g2s(v.c[3 + k], a.vel + k * a.cap + base, kTile * 8, &full[s]);
+    }
+    bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
+}
+
+template <int DEP, bool DH, bool MULTI>
+__global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepArgs a) {
+    extern __shared__ __align__(128) char smem[];
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
+    uint64_t *empty = full + kStages;
+    const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
+    const unsigned long long ntiles = n / kTile;
+    const unsigned long long G = gridDim.x;
+    const TileMap tm{ntiles, G, (unsigned long long)a.tile_group, blockIdx.x};
+    const unsigned long long my = tm.count();
+    const int warp = threadIdx.x >> 5;
     const unsigned lane = lane_id();
-    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    unsigned my_hops = 0, my_max = 0, my_capped = 0, my_removed = 0;
-    const int stop_at = CONT ? INT_MAX : a.hpass;
-    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-         i0 < n; i0 += stride) {
-        const unsigned long long k = i0 + lane;
-        const bool valid = k < n;
-        int status = ST_REMOVE + 100;   // "no particle"
-        int cell = 0, hops = 0, capped = 0;
-        double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
-        int4 cn = make_int4(0, 0, 0, 0);
-        unsigned long long i = k;
-        if (valid) {
-            double x, y, z;
-            if (CONT) {
-                i = a.work[k];
-                hops = a.work_hops[k];
-                x = a.pos[i]; y = a.pos[a.cap + i]; z = a.pos[2 * a.cap + i];
-                cell = a.p2c[i];
-            } else {
-                x = a.pos[i]; y = a.pos[a.cap + i]; z = a.pos[2 * a.cap + i];
-                double vx = a.vel[i], vy = a.vel[a.cap + i], vz = a.vel[2 * a.cap + i];
-                cell = a.p2c[i];
-                // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
-                const double *Ep = reinterpret_cast<const double *>(a.ef + (cell - a.cell_base));
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumerWarps);
+        }
+        fence_proxy_async();
+    }
+    __syncthreads();
+    if (warp == kConsumerWarps) {
+        // producer warp: streams tiles kStages ahead of the slowest consumer
+        if (lane == 0)
+            for (unsigned long long it = 0; it < my; it++) {
+                const int s = (int)(it % kStages);
+                if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
+                issue_tile_load(a, smem, full, s, tm.tile(it));
+            }
+        return;
+    }
+    // Consumer warp: its particle stream is its 32-slot slice of every tile.
+    // Lanes are refilled independently: whenever a lane's particle finishes
+    // (DONE / REMOVE / deferred / migrating) it takes the next stream entry,
+    // so every iteration advances 32 walks by one cell visit instead of
+    // waiting for the warp's longest walk.
+    Tally t;
+    const unsigned long long total = 32ull * my;
+    unsigned long long pos = 0;
+    long long waited = -1;
+    bool active = false;
+    double x = 0, y = 0, z = 0;
+    int cell = 0, hops = 0;
+    unsigned long long i = 0;
+    Line L;
+    const unsigned lt_mask = (1u << lane) - 1u;
+    for (;;) {
+        // ---- refill idle lanes from the stream
+        const unsigned need = __ballot_sync(0xffffffffu, !active);
+        if (need && pos < total) {
+            const unsigned long long avail = total - pos;
+            const int k = (int)min((unsigned long long)__popc(need), avail);
+            const int r = __popc(need & lt_mask);
+            const bool take = !active && r < k;
+            const long long last_tile = (long long)((pos + k - 1) / 32);
+            if (last_tile > waited) {
+                mbar_wait(&full[last_tile % kStages], (uint32_t)((last_tile / kStages) & 1));
+                waited = last_tile;
+            }
+            double vx = 0, vy = 0, vz = 0;
+            if (take) {
+                const unsigned long long p = pos + r, it = p / 32;
+                const int j = warp * 32 + (int)(p % 32);
+                StageView v = stage_view(smem, (int)(it % kStages));
+                x = v.c[0][j]; y = v.c[1][j]; z = v.c[2][j];
+                vx = v.c[3][j]; vy = v.c[4][j]; vz = v.c[5][j];
+                cell = v.cell[j];
+                i = tm.tile(it) * kTile + j;
+                hops = 0;
+            }
+            __syncwarp();
+            const unsigned long long npos = pos + k;
+            if (lane == 0)
+                for (unsigned long long tt = pos / 32; tt < npos / 32; tt++)
+                    mbar_arrive(&empty[tt % kStages]);   // our slice of tile tt is read
+            pos = npos;
+            if (take) {
+                const int lc = cell - a.cell_base;
+                L = load_line(a.lines, lc);
+                const double *Ep = reinterpret_cast<const double *>(a.ef + lc);
                 const double2 Exy = __ldg(reinterpret_cast<const double2 *>(Ep));
                 const double Ez = __ldg(Ep + 2);
                 vx = add(vx, mul(a.c1, Exy.x));
@@ -234,37 +568,87 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
                 z = add(z, mul(vz, a.dt));
                 a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
                 a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-                if (DH) cell = dh_seed(a.ov, x, y, z, cell);
+                if (DH) {
+                    const int sc = dh_seed(a.ov, x, y, z, cell);
+                    if (sc != cell) {
+                        cell = sc;
+                        L = load_line(a.lines, sc - a.cell_base);
+                    }
+                }
+                active = true;
             }
-            status = walk<MULTI>(a, cell, x, y, z, hops, stop_at, l0, l1, l2, l3, capped, cn);
-            if (status != ST_MOVE) {
-                my_hops += (unsigned)hops;
-                my_max = max(my_max, (unsigned)hops);
-                my_capped += (unsigned)capped;
+        }
+        if (!__any_sync(0xffffffffu, active)) break;
+        // ---- one cell visit per active lane
+        int status = ST_NONE;
+        int capped = 0;
+        double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
+        int4 cn = make_int4(0, 0, 0, 0);
+        if (active) {
+            bary(L, x, y, z, l0, l1, l2, l3);
+            cn = L.cn;
+            if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
+                status = ST_DONE;
+            } else if (hops >= a.hcap) {
+                status = ST_DONE;
+                capped = 1;
+            } else if (hops >= a.hpass) {
+                status = ST_MOVE;
+            } else {
+                int nb = L.cc.x;
+                double m = l0;
+                if (l1 < m) { m = l1; nb = L.cc.y; }
+                if (l2 < m) { m = l2; nb = L.cc.z; }
+                if (l3 < m) { nb = L.cc.w; }
+                if (nb < 0) {
+                    status = ST_REMOVE;
+                } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
+                    cell = nb;
+                    status = ST_MIGRATE;
+                } else {
+                    cell = nb;
+                    hops++;
+                    L = load_line(a.lines, nb - a.cell_base);
+                }
             }
-            a.p2c[i] = (status == ST_REMOVE) ? -1 : cell;
-            my_removed += (status == ST_REMOVE);
         }
-        const bool done = valid && status == ST_DONE;
-        if (DEP == 2) {
-            sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-        } else {
-            deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        const bool fin = status != ST_NONE;
+        if (fin && status != ST_MOVE && status != ST_MIGRATE) {
+            t.hops += (unsigned)hops;
+            t.maxh = max(t.maxh, (unsigned)hops);
+            t.capped += (unsigned)capped;
         }
-        // holes and the deferred-walk worklist
-        const bool rem = valid && status == ST_REMOVE;
+        t.removed += (status == ST_REMOVE);
+        const bool done = status == ST_DONE;
+        if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
+        else deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
         unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
         if (rem) a.holes[hs] = (uint32_t)i;
-        if (!CONT) {
-            const bool mv = valid && status == ST_MOVE;
-            unsigned long long ws = warp_append(mv, &a.cnt->n_work);
-            if (mv) {
-                a.work[ws] = (uint32_t)i;
-                a.work_hops[ws] = hops;
+        const bool mv = status == ST_MOVE;
+        unsigned long long ws = warp_append(mv, &a.cnt->n_work);
+        if (mv) {
+            a.work[ws] = (uint32_t)i;
+            a.work_hops[ws] = hops;
+        }
+        if (MULTI) {
+            const bool mg = status == ST_MIGRATE;
+            unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
+            if (mg) {
+                a.mig[ms] = (uint32_t)i;
+                a.mig_cell[ms] = cell;
+                a.mig_hops[ms] = hops;
             }
         }
+        if (fin) {
+            a.p2c[i] = rem ? -1 : cell;
+            active = false;
+        }
     }
-    flush_stats(a.cnt, my_hops, my_max, my_capped, my_removed);
+    // ragged tail [ntiles*kTile, n): last block, consumer warps
+    if (blockIdx.x == G - 1)
+        pmd_direct_range<DEP, DH, false, MULTI>(a, ntiles * kTile, n, threadIdx.x & ~31u, kTile, t);
+    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
 // ---------------------------------------------------------------------------
@@ -286,6 +670,9 @@ __global__ void k_step_begin(double *Q, long long nn, DevCounters *c, int zero) 
         c->n_sr = 0;
         c->n_head = 0;
         c->n_tail = 0;
+        c->n_mig = 0;
+        c->n_mig_out = 0;
+        c->n_mig_in = 0;
     }
     if (zero)
         for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nn;
@@ -492,40 +879,6 @@ __global__ void k_sr_hist(const int32_t *__restrict__ sr_cell, const DevCounters
         atomicAdd(hist + sr_cell[k], 1u);
 }
 
-// Single-block exclusive scan of nc+1 counters (nc ~ 1e6: a few microseconds).
-__global__ void k_scan_1block(const unsigned *in, unsigned *out, long long n) {
-    __shared__ unsigned long long warp_sums[32];
-    __shared__ unsigned long long carry_s;
-    if (threadIdx.x == 0) carry_s = 0;
-    __syncthreads();
-    for (long long base = 0; base < n; base += blockDim.x) {
-        long long i = base + threadIdx.x;
-        unsigned long long v = i < n ? in[i] : 0;
-        unsigned long long x = v;
-        for (int off = 1; off < 32; off <<= 1) {
-            unsigned long long t = __shfl_up_sync(0xffffffffu, x, off);
-            if ((int)lane_id() >= off) x += t;
-        }
-        if (lane_id() == 31) warp_sums[threadIdx.x >> 5] = x;
-        __syncthreads();
-        if (threadIdx.x < 32) {
-            unsigned long long s = (threadIdx.x < (blockDim.x >> 5)) ? warp_sums[threadIdx.x] : 0;
-            for (int off = 1; off < 32; off <<= 1) {
-                unsigned long long t = __shfl_up_sync(0xffffffffu, s, off);
-                if ((int)threadIdx.x >= off) s += t;
-            }
-            warp_sums[threadIdx.x] = s;
-        }
-        __syncthreads();
-        unsigned long long wpre = (threadIdx.x >> 5) ? warp_sums[(threadIdx.x >> 5) - 1] : 0;
-        unsigned long long carry = carry_s;
-        if (i < n) out[i] = (unsigned)(carry + wpre + x - v);
-        __syncthreads();
-        if (threadIdx.x == blockDim.x - 1) carry_s = carry + wpre + x;
-        __syncthreads();
-    }
-}
-
 __global__ void k_sr_scatter(const int32_t *__restrict__ sr_cell, const double *__restrict__ sr_val,
                              long long cap, const DevCounters *c, unsigned *cursor,
                              double *sorted) {
@@ -567,19 +920,368 @@ __global__ void k_sr_node_gather(const int32_t *__restrict__ n2cs_ptr, const int
 }
 
 // ---------------------------------------------------------------------------
+// Multi-block exclusive scan of unsigned counts (3 phases: tile sums, scan of
+// the tile sums in one block, tile scans plus offsets).  Tile = 4096.
+// ---------------------------------------------------------------------------
+constexpr int kScanTile = 4096;   // 1024 threads x 4 elements
+
+__device__ __forceinline__ unsigned long long block_exclusive_scan(unsigned long long v,
+                                                                   unsigned long long *warp_buf,
+                                                                   unsigned long long *total) {
+    unsigned long long x = v;
+    for (int off = 1; off < 32; off <<= 1) {
+        unsigned long long t = __shfl_up_sync(0xffffffffu, x, off);
+        if ((int)lane_id() >= off) x += t;
+    }
+    const int wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    if (lane_id() == 31) warp_buf[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+        unsigned long long s = (int)lane_id() < nw ? warp_buf[lane_id()] : 0;
+        for (int off = 1; off < 32; off <<= 1) {
+            unsigned long long t = __shfl_up_sync(0xffffffffu, s, off);
+            if ((int)lane_id() >= off) s += t;
+        }
+        warp_buf[lane_id()] = s;
+    }
+    __syncthreads();
+    unsigned long long pre = wid ? warp_buf[wid - 1] : 0;
+    if (total) *total = warp_buf[nw - 1];
+    return pre + x - v;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_tiles(const unsigned *__restrict__ in, long long n,
+                                                     unsigned long long *tile_sum) {
+    __shared__ unsigned long long wb[32];
+    const long long base = (long long)blockIdx.x * kScanTile + 4 * threadIdx.x;
+    unsigned long long v = 0;
+    for (int k = 0; k < 4; k++)
+        if (base + k < n) v += in[base + k];
+    unsigned long long tot;
+    block_exclusive_scan(v, wb, &tot);
+    if (threadIdx.x == 0) tile_sum[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_top(unsigned long long *tile_sum, long long ntiles) {
+    __shared__ unsigned long long wb[32];
+    __shared__ unsigned long long carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (long long b = 0; b < ntiles; b += blockDim.x) {
+        long long i = b + threadIdx.x;
+        unsigned long long v = i < ntiles ? tile_sum[i] : 0;
+        unsigned long long tot;
+        unsigned long long ex = block_exclusive_scan(v, wb, &tot);
+        unsigned long long c = carry;
+        __syncthreads();
+        if (i < ntiles) tile_sum[i] = c + ex;
+        if (threadIdx.x == 0) carry = c + tot;
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_scan_apply(const unsigned *__restrict__ in, long long n,
+                                                     const unsigned long long *__restrict__ tile_off,
+                                                     unsigned *out) {
+    __shared__ unsigned long long wb[32];
+    const long long base = (long long)blockIdx.x * kScanTile + 4 * threadIdx.x;
+    unsigned e[4];
+    unsigned long long v = 0;
+    for (int k = 0; k < 4; k++) {
+        e[k] = base + k < n ? in[base + k] : 0u;
+        v += e[k];
+    }
+    unsigned long long ex = block_exclusive_scan(v, wb, nullptr) + tile_off[blockIdx.x];
+    for (int k = 0; k < 4; k++) {
+        if (base + k < n) out[base + k] = (unsigned)ex;
+        ex += e[k];
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Sort by cell (particle sorting as an auxiliary call;
+// here also the step's compaction): counting sort keyed by the local cell.
+// Holes (p2c = -1) are dropped, so the sorted set is also hole-free.  Runs of
+// equal cells inside a warp are aggregated into one atomic.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void run_info(int key, unsigned &heads, int &run_start, int &run_len,
+                                         bool &head) {
+    const unsigned lane = lane_id();
+    int prev = __shfl_up_sync(0xffffffffu, key, 1);
+    head = (lane == 0) || (prev != key);
+    heads = __ballot_sync(0xffffffffu, head);
+    unsigned below = heads & ((2u << lane) - 1u);      // heads at or below this lane
+    if (lane == 31) below = heads;
+    run_start = 31 - __clz(below);
+    unsigned above = heads & ~((2u << lane) - 1u);
+    if (lane == 31) above = 0;
+    int run_end = above ? (__ffs(above) - 2) : 31;
+    run_len = run_end - run_start + 1;
+}
+
+__global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
+                            unsigned *hist) {
+    const unsigned long long n = c->n;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+         i0 < n; i0 += stride) {
+        const unsigned long long i = i0 + lane_id();
+        int cell = i < n ? p2c[i] : -1;
+        int key = cell >= 0 ? cell : -2 - (int)lane_id();
+        unsigned heads;
+        int rs, rl;
+        bool head;
+        run_info(key, heads, rs, rl, head);
+        if (head && cell >= 0) atomicAdd(hist + (cell - cell_base), (unsigned)rl);
+    }
+}
+
+// Phase 1: destination slot of every particle (run heads take one atomic
+// per run of equal cells); holes get 0xffffffff.
+__global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
+                            unsigned *cursor, uint32_t *dest) {
+    const unsigned long long n = c->n;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+         i0 < n; i0 += stride) {
+        const unsigned long long i = i0 + lane_id();
+        int cell = i < n ? p2c[i] : -1;
+        int key = cell >= 0 ? cell : -2 - (int)lane_id();
+        unsigned heads;
+        int rs, rl;
+        bool head;
+        run_info(key, heads, rs, rl, head);
+        unsigned base = 0;
+        if (head && cell >= 0) base = atomicAdd(cursor + (cell - cell_base), (unsigned)rl);
+        base = __shfl_sync(0xffffffffu, base, rs);
+        if (i < n) dest[i] = cell >= 0 ? base + (lane_id() - rs) : 0xffffffffu;
+    }
+}
+
+// Phase 2: pure streaming move src[i] -> dst[dest[i]], each block a
+// contiguous chunk, kSortUnroll independent particles in flight per thread.
+constexpr int kSortUnroll = 4;
+__global__ void __launch_bounds__(256) k_sort_move(ColSet src, ColSet dst,
+                                                   const uint32_t *__restrict__ dest,
+                                                   const DevCounters *c) {
+    const unsigned long long n = c->n;
+    const unsigned long long span = (unsigned long long)blockDim.x * kSortUnroll;
+    const unsigned long long chunk = ((n + gridDim.x - 1) / gridDim.x + span - 1) / span * span;
+    const unsigned long long lo = blockIdx.x * chunk;
+    const unsigned long long hi = lo + chunk < n ? lo + chunk : n;
+    for (unsigned long long b = lo; b < hi; b += span) {
+        unsigned long long ii[kSortUnroll];
+        uint32_t dd[kSortUnroll];
+#pragma unroll
+        for (int u = 0; u < kSortUnroll; u++) {
+            ii[u] = b + (unsigned long long)u * blockDim.x + threadIdx.x;
+            dd[u] = ii[u] < hi ? __ldg(dest + ii[u]) : 0xffffffffu;
+        }
+        for (int j = 0; j < src.n; j++) {
+            const ColDesc cs = src.c[j], cd = dst.c[j];
+            for (int e = 0; e < cs.dim; e++) {
+                if (cs.elem_bytes == 8) {
+                    const long long *sp = reinterpret_cast<const long long *>(cs.ptr) + e * cs.cap;
+                    long long *dp = reinterpret_cast<long long *>(cd.ptr) + e * cd.cap;
+                    long long v[kSortUnroll];
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] != 0xffffffffu ? __ldg(sp + ii[u]) : 0;
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] != 0xffffffffu) dp[dd[u]] = v[u];
+                } else {
+                    const int *sp = reinterpret_cast<const int *>(cs.ptr) + e * cs.cap;
+                    int *dp = reinterpret_cast<int *>(cd.ptr) + e * cd.cap;
+                    int v[kSortUnroll];
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] != 0xffffffffu ? __ldg(sp + ii[u]) : 0;
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] != 0xffffffffu) dp[dd[u]] = v[u];
+                }
+            }
+        }
+    }
+}
+
+// n := number of sorted (hole-free) particles; holes consumed.
+__global__ void k_sort_commit(DevCounters *c, const unsigned *start_total) {
+    c->n_removed_last = c->n_holes;
+    c->n = *start_total;
+    c->n_holes = 0;
+}
+
+// ---------------------------------------------------------------------------
+// Particle migration between slabs (mark -> pack into one
+// buffer -> send/recv -> unpack to the end of the dats -> continue the walk).
+// A record holds every particle column (AoS bytes, the p2c slot carrying the
+// target global cell) followed by the hop count (S4: hops travel with the
+// particle).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ int owner_of(const RankRanges &rr, int cell) {
+    for (int r = 0; r < rr.n; r++)
+        if (cell >= rr.lo[r] && cell < rr.hi[r]) return r;
+    return -1;
+}
+
+__global__ void k_mig_count(const int32_t *__restrict__ mig_cell, const DevCounters *c, RankRanges rr,
+                            unsigned long long *counts) {
+    __shared__ unsigned long long sc[kMaxRanks];
+    for (int r = threadIdx.x; r < rr.n; r += blockDim.x) sc[r] = 0;
+    __syncthreads();
+    const unsigned long long m = c->n_mig;
+    for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
+         k += (unsigned long long)gridDim.x * blockDim.x) {
+        int o = owner_of(rr, mig_cell[k]);
+        if (o >= 0) atomicAdd(&sc[o], 1ull);
+    }
+    __syncthreads();
+    for (int r = threadIdx.x; r < rr.n; r += blockDim.x)
+        if (sc[r]) atomicAdd(&counts[r], sc[r]);
+}
+
+__device__ __forceinline__ void copy_elem(char *dst, const char *src, int eb) {
+    if (eb == 8) *reinterpret_cast<long long *>(dst) = *reinterpret_cast<const long long *>(src);
+    else *reinterpret_cast<int *>(dst) = *reinterpret_cast<const int *>(src);
+}
+
+__global__ void k_mig_pack(ColSet cols, int p2c_col, const uint32_t *__restrict__ mig,
+                           const int32_t *__restrict__ mig_cell, const int32_t *__restrict__ mig_hops,
+                           const DevCounters *c, RankRanges rr, unsigned long long *cursor,
+                           char *sendbuf, int rec_bytes) {
+    const unsigned long long m = c->n_mig;
+    for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
+         k += (unsigned long long)gridDim.x * blockDim.x) {
+        const int o = owner_of(rr, mig_cell[k]);
+        if (o < 0) continue;
+        const unsigned long long slot = atomicAdd(&cursor[o], 1ull);
+        char *rec = sendbuf + slot * (unsigned long long)rec_bytes;
+        const unsigned long long i = mig[k];
+        int off = 0;
+        for (int j = 0; j < cols.n; j++) {
+            const ColDesc cd = cols.c[j];
+            off = (off + cd.elem_bytes - 1) & ~(cd.elem_bytes - 1);   // natural alignment
+            for (int e = 0; e < cd.dim; e++) {
+                if (j == p2c_col) *reinterpret_cast<int *>(rec + off) = mig_cell[k];
+                else copy_elem(rec + off, cd.ptr + ((long long)e * cd.cap + (long long)i) * cd.elem_bytes,
+                               cd.elem_bytes);
+                off += cd.elem_bytes;
+            }
+        }
+        *reinterpret_cast<int *>(rec + off) = mig_hops[k];
+    }
+}
+
+// Append R received records at [N, N+R); they become the continuation
+// worklist; the last block commits N += R and resets the migrant list.
+__global__ void k_mig_unpack(ColSet cols, const char *__restrict__ recvbuf, long long R, int rec_bytes,
+                             DevCounters *c, uint32_t *work, int32_t *work_hops) {
+    __shared__ unsigned long long base_s;
+    if (threadIdx.x == 0) base_s = *(volatile unsigned long long *)&c->n;
+    __syncthreads();
+    const unsigned long long base = base_s;
+    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < R;
+         k += (long long)gridDim.x * blockDim.x) {
+        const char *rec = recvbuf + k * (long long)rec_bytes;
+        const unsigned long long i = base + k;
+        int off = 0;
+        for (int j = 0; j < cols.n; j++) {
+            const ColDesc cd = cols.c[j];
+            off = (off + cd.elem_bytes - 1) & ~(cd.elem_bytes - 1);
+            for (int e = 0; e < cd.dim; e++) {
+                copy_elem(cd.ptr + ((long long)e * cd.cap + (long long)i) * cd.elem_bytes, rec + off,
+                          cd.elem_bytes);
+                off += cd.elem_bytes;
+            }
+        }
+        work[k] = (uint32_t)i;
+        work_hops[k] = *reinterpret_cast<const int *>(rec + off);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        unsigned long long t = atomicAdd(&c->unpack_done_blocks, 1ull);
+        if (t == gridDim.x - 1) {
+            c->n = base + (unsigned long long)R;
+            c->n_work = (unsigned long long)R;
+            c->n_mig_out += c->n_mig;
+            c->n_mig = 0;
+            c->n_mig_in += (unsigned long long)R;
+            c->unpack_done_blocks = 0;
+            __threadfence();
+        }
+    }
+}
+
+// Node-charge halo: interface nodes' partial sums.
+__global__ void k_halo_pack(const double *__restrict__ Q, const int32_t *__restrict__ idx, long long m,
+                            double *out) {
+    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
+         k += (long long)gridDim.x * blockDim.x)
+        out[k] = Q[idx[k]];
+}
+
+__global__ void k_halo_add(double *Q, const int32_t *__restrict__ idx, long long m,
+                           const double *__restrict__ in) {
+    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
+         k += (long long)gridDim.x * blockDim.x)
+        atomicAdd(Q + idx[k], in[k]);
+}
+
+// ---------------------------------------------------------------------------
 // Launchers (host side of this translation unit)
 // ---------------------------------------------------------------------------
+
+long long scan_tiles(long long n) { return n > 0 ? (n + kScanTile - 1) / kScanTile : 1; }
+
+cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
+                           unsigned long long *tile_sums, cudaStream_t s) {
+    long long tiles = scan_tiles(n);
+    k_scan_tiles<<<(int)tiles, 1024, 0, s>>>(in, n, tile_sums);
+    k_scan_top<<<1, 1024, 0, s>>>(tile_sums, tiles);
+    k_scan_apply<<<(int)tiles, 1024, 0, s>>>(in, n, tile_sums, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
+                              unsigned *hist, unsigned *start, unsigned long long *tile_sums,
+                              int grid, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(hist, 0, sizeof(unsigned) * (nc + 1), s);
+    if (e != cudaSuccess) return e;
+    k_cell_hist<<<grid, 256, 0, s>>>(p2c, c, cell_base, hist);
+    return scan_exclusive(hist, start, nc + 1, tile_sums, s);
+}
+
+cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
+                             DevCounters *c, int cell_base, long long nc, unsigned *start,
+                             uint32_t *dest, int grid, cudaStream_t s) {
+    k_sort_rank<<<grid, 256, 0, s>>>(p2c, c, cell_base, start, dest);
+    k_sort_move<<<grid, 256, 0, s>>>(src, dst, dest, c);
+    k_sort_commit<<<1, 1, 0, s>>>(c, start + nc);
+    return cudaGetLastError();
+}
+
 template <int DEP, bool DH, bool CONT, bool MULTI>
-static cudaError_t launch_pmd_t(const StepArgs &a, int grid, cudaStream_t s) {
-    k_push_move_deposit<DEP, DH, CONT, MULTI><<<grid, 256, 0, s>>>(a);
+static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
+    if (!CONT && tiled) {
+        static bool attr = false;
+        if (!attr) {
+            cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI>,
+                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                 kTiledSmem);
+            if (e != cudaSuccess) return e;
+            attr = true;
+        }
+        k_push_move_deposit_tiled<DEP, DH, MULTI><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+    } else {
+        k_push_move_deposit<DEP, DH, CONT, MULTI><<<grid, 256, 0, s>>>(a);
+    }
     return cudaGetLastError();
 }
 
 template <bool CONT>
 static cudaError_t launch_pmd_c(int dep, bool dh, bool multi, const StepArgs &a, int grid,
-                                cudaStream_t s) {
+                                bool tiled, cudaStream_t s) {
 #define OPP_CASE(D, H, M) \
-    if (dep == D && dh == H && multi == M) return launch_pmd_t<D, H, CONT, M>(a, grid, s);
+    if (dep == D && dh == H && multi == M) return launch_pmd_t<D, H, CONT, M>(a, grid, tiled, s);
     OPP_CASE(0, false, false) OPP_CASE(0, true, false) OPP_CASE(1, false, false)
     OPP_CASE(1, true, false) OPP_CASE(2, false, false) OPP_CASE(2, true, false)
     OPP_CASE(0, false, true) OPP_CASE(0, true, true) OPP_CASE(1, false, true)
@@ -588,22 +1290,63 @@ static cudaError_t launch_pmd_c(int dep, bool dh, bool multi, const StepArgs &a,
     return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, const StepArgs &a,
-                                     int grid, cudaStream_t s) {
-    return cont ? launch_pmd_c<true>(dep, dh, multi, a, grid, s)
-                : launch_pmd_c<false>(dep, dh, multi, a, grid, s);
+cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, bool tiled,
+                                     const StepArgs &a, int grid, cudaStream_t s) {
+    return cont ? launch_pmd_c<true>(dep, dh, multi, a, grid, tiled, s)
+                : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
 }
 
-int pmd_blocks_per_sm(int dep, bool dh) {
+int pmd_blocks_per_sm(bool tiled) {
     int nb = 0;
     cudaError_t e;
-    if (dep == 1)
-        e = dh ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_push_move_deposit<1, true, false, false>, 256, 0)
-               : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_push_move_deposit<1, false, false, false>, 256, 0);
-    else
-        e = dh ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_push_move_deposit<0, true, false, false>, 256, 0)
-               : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_push_move_deposit<0, false, false, false>, 256, 0);
+    if (tiled) {
+        cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &nb, k_push_move_deposit_tiled<0, false, false>, kTiledThreads, kTiledSmem);
+    } else {
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &nb, k_push_move_deposit<0, false, false, false>, 256, 0);
+    }
     return (e == cudaSuccess && nb > 0) ? nb : 1;
+}
+
+cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
+                             unsigned long long *counts, int grid, cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(counts, 0, sizeof(unsigned long long) * rr.n, s);
+    if (e != cudaSuccess) return e;
+    k_mig_count<<<grid, 256, 0, s>>>(mig_cell, c, rr, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_mig_pack(const ColSet &cols, int p2c_col, const uint32_t *mig,
+                            const int32_t *mig_cell, const int32_t *mig_hops, const DevCounters *c,
+                            const RankRanges &rr, unsigned long long *cursor, char *sendbuf,
+                            int rec_bytes, int grid, cudaStream_t s) {
+    k_mig_pack<<<grid, 256, 0, s>>>(cols, p2c_col, mig, mig_cell, mig_hops, c, rr, cursor, sendbuf,
+                                    rec_bytes);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_mig_unpack(const ColSet &cols, const char *recvbuf, long long R, int rec_bytes,
+                              DevCounters *c, uint32_t *work, int32_t *work_hops, int grid,
+                              cudaStream_t s) {
+    k_mig_unpack<<<grid, 256, 0, s>>>(cols, recvbuf, R, rec_bytes, c, work, work_hops);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_halo_pack(const double *Q, const int32_t *idx, long long m, double *out,
+                             cudaStream_t s) {
+    int g = (int)std::min<long long>(1184, (m + 255) / 256);
+    k_halo_pack<<<g > 0 ? g : 1, 256, 0, s>>>(Q, idx, m, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_halo_add(double *Q, const int32_t *idx, long long m, const double *in,
+                            cudaStream_t s) {
+    int g = (int)std::min<long long>(1184, (m + 255) / 256);
+    k_halo_add<<<g > 0 ? g : 1, 256, 0, s>>>(Q, idx, m, in);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero, int grid,
@@ -653,11 +1396,13 @@ cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long n
 }
 
 cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *hist,
-                      unsigned *start, double *sorted, double *cellsum, const int32_t *n2cs_ptr,
-                      const int32_t *n2cs, int grid, cudaStream_t s) {
+                      unsigned *start, unsigned long long *tile_sums, double *sorted,
+                      double *cellsum, const int32_t *n2cs_ptr, const int32_t *n2cs, int grid,
+                      cudaStream_t s) {
     cudaMemsetAsync(hist, 0, sizeof(unsigned) * (nc + 1), s);
     k_sr_hist<<<grid, 256, 0, s>>>(a.sr_cell, a.cnt, hist);
-    k_scan_1block<<<1, 1024, 0, s>>>(hist, start, nc + 1);
+    cudaError_t e = scan_exclusive(hist, start, nc + 1, tile_sums, s);
+    if (e != cudaSuccess) return e;
     cudaMemcpyAsync(hist, start, sizeof(unsigned) * (nc + 1), cudaMemcpyDeviceToDevice, s);
     k_sr_scatter<<<grid, 256, 0, s>>>(a.sr_cell, a.sr_val, a.cap, a.cnt, hist, sorted);
     int gc = (int)((nc + 255) / 256), gn = (int)((nn + 255) / 256);

@@ -4,9 +4,9 @@
 
 namespace opp {
 
-cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, const StepArgs &a,
-                                     int grid, cudaStream_t s);
-int pmd_blocks_per_sm(int dep, bool dh);
+cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, bool tiled,
+                                     const StepArgs &a, int grid, cudaStream_t s);
+int pmd_blocks_per_sm(bool tiled);
 cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero, int grid,
                               cudaStream_t s);
 cudaError_t launch_fill(const ColSet &cols, DevCounters *c, const uint32_t *holes,
@@ -20,7 +20,32 @@ cudaError_t launch_pack_field(const double *ef, long long nc, double4 *out, cuda
 cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long nc, int cell_base,
                            const Overlay &ov, int32_t *map, cudaStream_t s);
 cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *hist,
-                      unsigned *start, double *sorted, double *cellsum, const int32_t *n2cs_ptr,
-                      const int32_t *n2cs, int grid, cudaStream_t s);
+                      unsigned *start, unsigned long long *tile_sums, double *sorted,
+                      double *cellsum, const int32_t *n2cs_ptr, const int32_t *n2cs, int grid,
+                      cudaStream_t s);
+
+long long scan_tiles(long long n);
+cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
+                           unsigned long long *tile_sums, cudaStream_t s);
+cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
+                              unsigned *hist, unsigned *start, unsigned long long *tile_sums,
+                              int grid, cudaStream_t s);
+cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
+                             DevCounters *c, int cell_base, long long nc, unsigned *start,
+                             uint32_t *dest, int grid, cudaStream_t s);
+
+cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
+                             unsigned long long *counts, int grid, cudaStream_t s);
+cudaError_t launch_mig_pack(const ColSet &cols, int p2c_col, const uint32_t *mig,
+                            const int32_t *mig_cell, const int32_t *mig_hops, const DevCounters *c,
+                            const RankRanges &rr, unsigned long long *cursor, char *sendbuf,
+                            int rec_bytes, int grid, cudaStream_t s);
+cudaError_t launch_mig_unpack(const ColSet &cols, const char *recvbuf, long long R, int rec_bytes,
+                              DevCounters *c, uint32_t *work, int32_t *work_hops, int grid,
+                              cudaStream_t s);
+cudaError_t launch_halo_pack(const double *Q, const int32_t *idx, long long m, double *out,
+                             cudaStream_t s);
+cudaError_t launch_halo_add(double *Q, const int32_t *idx, long long m, const double *in,
+                            cudaStream_t s);
 
 }  // namespace opp

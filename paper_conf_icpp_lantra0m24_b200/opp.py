@@ -28,9 +28,11 @@ EXPORTS = (
     "opp_set_partition", "opp_inject", "opp_push_move_deposit", "opp_fill_holes",
     "opp_get_node_charge", "opp_get_dat", "opp_set_dat", "opp_get_particle_count",
     "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
-    "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats",
+    "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
 )
-PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo")
+PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
+          "sort_count", "sort_move")
+# note: "fill" includes the periodic sort-by-cell when opp_init_params.sort_every > 0
 
 
 class OppError(RuntimeError):
@@ -45,7 +47,8 @@ class opp_init_params(C.Structure):
                 ("free", FREE_FN), ("alloc_user", C.c_void_p), ("deposit_mode", C.c_int),
                 ("direct_hop", C.c_int), ("overlay_spacing", C.c_double),
                 ("hop_budget_per_pass", C.c_int), ("hop_cap", C.c_int),
-                ("allow_growth", C.c_int)]
+                ("allow_growth", C.c_int), ("sort_every", C.c_int),
+                ("tma_pipeline", C.c_int), ("transport", C.c_int)]
 
 
 class opp_step_params(C.Structure):
@@ -80,12 +83,13 @@ def _load():
         "opp_decl_particle_set": (I, [P, C.c_char_p, I32, I64, I64, C.POINTER(I32)]),
         "opp_decl_map": (I, [P, I32, I32, I, P, C.c_char_p, C.POINTER(I32)]),
         "opp_decl_dat": (I, [P, I32, I, I, P, C.c_char_p, C.POINTER(I32)]),
-        "opp_set_partition": (I, [P, I32, P]),
+        "opp_set_partition": (I, [P, I32, I64, P, I32, P]),
         "opp_inject": (I, [P, I32, I64, I, P, P, I]),
         "opp_push_move_deposit": (I, [P, I32, I32, I32, I32, I32, I32, I32, I32, I32,
                                       C.POINTER(opp_step_params), C.POINTER(opp_step_stats)]),
         "opp_fill_holes": (I, [P, I32, C.POINTER(I64)]),
         "opp_get_step_stats": (I, [P, I32, C.POINTER(opp_step_stats)]),
+        "opp_sort_by_cell": (I, [P, I32]),
         "opp_get_node_charge": (I, [P, I32, P, I64]),
         "opp_get_dat": (I, [P, I32, P, I64]),
         "opp_set_dat": (I, [P, I32, P, I64, I]),
@@ -175,8 +179,9 @@ def opp_decl_dat(ctx, set_: int, dim: int, typ: int, host, name: str) -> int:
     return out.value
 
 
-def opp_set_partition(ctx, cells: int, rank_of_cell) -> None:
-    _ck(lib.opp_set_partition(ctx, cells, _ptr(rank_of_cell)))
+def opp_set_partition(ctx, cells: int, rank_of_cell, nodes: int, node_gid) -> None:
+    _ck(lib.opp_set_partition(ctx, cells, int(rank_of_cell.shape[0]), _ptr(rank_of_cell), nodes,
+                              _ptr(node_gid)))
 
 
 def opp_inject(ctx, parts: int, n: int, cols, data, on_device: bool) -> None:
@@ -207,6 +212,10 @@ def opp_fill_holes(ctx, parts: int, want_count: bool = True):
     n = C.c_int64()
     _ck(lib.opp_fill_holes(ctx, parts, C.byref(n)))
     return n.value
+
+
+def opp_sort_by_cell(ctx, parts: int) -> None:
+    _ck(lib.opp_sort_by_cell(ctx, parts))
 
 
 def opp_get_node_charge(ctx, dat: int, out) -> None:
@@ -250,7 +259,7 @@ def opp_phase_timing(ctx, enable: bool) -> None:
 
 
 def opp_get_phase_times(ctx) -> dict:
-    ms = (C.c_double * 8)()
-    cnt = (C.c_int64 * 8)()
+    ms = (C.c_double * len(PHASES))()
+    cnt = (C.c_int64 * len(PHASES))()
     _ck(lib.opp_get_phase_times(ctx, ms, cnt))
-    return {PHASES[k]: (ms[k], cnt[k]) for k in range(8)}
+    return {PHASES[k]: (ms[k], cnt[k]) for k in range(len(PHASES))}
