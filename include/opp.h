@@ -101,6 +101,10 @@ typedef struct {
     int transport;              /* nranks > 1: 0 = NCCL (one process per GPU),
                                    1 = in-process loopback (contexts in one process,
                                    one host thread each; testing on one GPU)        */
+    double sort_axis[3];        /* principal direction of motion
+                                   used as the sort-by-cell locality key: cells are
+                                   ordered by transverse bin, then along the axis;
+                                   (0,0,0) = plain cell-id order                    */
 } opp_init_params;
 
 /* Per-step arguments of opp_push_move_deposit. */

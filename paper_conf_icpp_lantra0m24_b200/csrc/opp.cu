@@ -73,8 +73,12 @@ struct PSet {
     double *sr_val = nullptr;
     uint32_t *mig = nullptr;     // nranks > 1: migrants of the current round
     int32_t *mig_cell = nullptr, *mig_hops = nullptr;
-    char *staging = nullptr;
-    size_t staging_bytes = 0;
+    // host injection: two staging slots filled on the copy stream, so the H2D
+    // copy of the next batch overlaps the current step's kernels
+    char *stg[2] = {nullptr, nullptr};
+    size_t stg_bytes[2] = {0, 0};
+    cudaEvent_t stg_free[2] = {nullptr, nullptr}, stg_ready[2] = {nullptr, nullptr};
+    int stg_next = 0;
     std::vector<int> cols;
     std::vector<char *> alt;     // sort double buffers (one per column, lazily allocated)
     long long alt_cap = 0;
@@ -101,6 +105,8 @@ struct MeshCache {
     bool ov_built = false;
     Overlay ov{};
     int32_t *ov_map = nullptr;
+    // sort locality key per cell (opp_init_params.sort_axis), NULL = cell order
+    uint32_t *sort_key = nullptr;
     // per-cell counting (SR deposit and sort by cell)
     unsigned *cell_hist = nullptr, *cell_start = nullptr;
     unsigned long long *tile_sums = nullptr;
@@ -114,10 +120,12 @@ struct MeshCache {
 struct opp_ctx_s {
     opp_init_params p{};
     cudaStream_t s = nullptr;
+    cudaStream_t cs = nullptr;     // copy stream (host injection staging)
     int nsm = 148;
     int bps = 0;                   // resident blocks / SM of the fused kernel
     int tile_group = 8;            // OPP_TILE_GROUP: tiles per block visit (TileMap)
     int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
+    int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -233,10 +241,16 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     c->p = *params;
     if (c->p.deposit_mode == OPP_DEP_AUTO) c->p.deposit_mode = OPP_DEP_ATOMIC;
     c->s = (cudaStream_t)params->cuda_stream;
+    if (cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking) != cudaSuccess) {
+        delete c;
+        return fail(OPP_ERR_CUDA, "copy stream");
+    }
     cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, params->device);
     if (const char *tg = getenv("OPP_TILE_GROUP")) c->tile_group = std::max(1, atoi(tg));
     if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
+    if (const char *rf = getenv("OPP_REFILL")) c->refill = atoi(rf);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
+        cudaStreamDestroy(c->cs);
         delete c;
         return fail(OPP_ERR_NOMEM, "cudaMallocHost");
     }
@@ -245,6 +259,7 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
                                params->nranks, params->device, g_err);
         if (r != OPP_OK) {
             cudaFreeHost(c->hcnt);
+            cudaStreamDestroy(c->cs);
             delete c;
             return r;
         }
@@ -266,7 +281,11 @@ static void free_pset(opp_ctx c, PSet &ps) {
     c->dfree(ps.mig, 4 * cap);
     c->dfree(ps.mig_cell, 4 * cap);
     c->dfree(ps.mig_hops, 4 * cap);
-    c->dfree(ps.staging, ps.staging_bytes);
+    for (int k = 0; k < 2; k++) {
+        c->dfree(ps.stg[k], ps.stg_bytes[k]);
+        if (ps.stg_free[k]) cudaEventDestroy(ps.stg_free[k]);
+        if (ps.stg_ready[k]) cudaEventDestroy(ps.stg_ready[k]);
+    }
     ps = PSet();
 }
 
@@ -286,12 +305,15 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.cell_hist, 0);
     c->dfree(m.cell_start, 0);
     c->dfree(m.tile_sums, 0);
+    c->dfree(m.sort_key, 0);
     c->dfree(m.sr_sorted, 0);
     c->dfree(m.sr_cellsum, 0);
     c->dfree(m.n2cs_ptr, 0);
     c->dfree(m.n2cs, 0);
     if (c->comm) opp::comm_free(c->comm);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
+    cudaStreamSynchronize(c->cs);
+    cudaStreamDestroy(c->cs);
     cudaFreeHost(c->hcnt);
     delete c;
     return OPP_OK;
@@ -642,20 +664,41 @@ extern "C" int opp_inject(opp_ctx c, opp_set parts, int64_t n, int ncols, const 
             off[j] = tot;
             tot += ((size_t)n * cs.c[j].dim * cs.c[j].elem_bytes + 255) & ~(size_t)255;
         }
-        if (tot > ps.staging_bytes) {
+        const int k = ps.stg_next;
+        ps.stg_next ^= 1;
+        if (!ps.stg_free[k]) {
+            CK(cudaEventCreateWithFlags(&ps.stg_free[k], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&ps.stg_ready[k], cudaEventDisableTiming));
+        }
+        if (tot > ps.stg_bytes[k]) {
             CK(cudaStreamSynchronize(c->s));
-            c->dfree(ps.staging, ps.staging_bytes);
-            ps.staging_bytes = 0;
-            ps.staging = (char *)c->dalloc(tot);
-            if (!ps.staging) return fail(OPP_ERR_NOMEM, "injection staging (%zu B)", tot);
-            ps.staging_bytes = tot;
+            CK(cudaStreamSynchronize(c->cs));
+            c->dfree(ps.stg[k], ps.stg_bytes[k]);
+            ps.stg_bytes[k] = 0;
+            ps.stg[k] = (char *)c->dalloc(tot);
+            if (!ps.stg[k]) return fail(OPP_ERR_NOMEM, "injection staging (%zu B)", tot);
+            ps.stg_bytes[k] = tot;
         }
+        // the slot's previous batch must have been consumed by its k_inject
+        CK(cudaStreamWaitEvent(c->cs, ps.stg_free[k], 0));
         for (int j = 0; j < cs.n; j++) {
-            CK(cudaMemcpyAsync(ps.staging + off[j], src[j],
+            CK(cudaMemcpyAsync(ps.stg[k] + off[j], src[j],
                                (size_t)n * cs.c[j].dim * cs.c[j].elem_bytes,
-                               cudaMemcpyHostToDevice, c->s));
-            cs.src[j] = ps.staging + off[j];
+                               cudaMemcpyHostToDevice, c->cs));
+            cs.src[j] = ps.stg[k] + off[j];
         }
+        CK(cudaEventRecord(ps.stg_ready[k], c->cs));
+        CK(cudaStreamWaitEvent(c->s, ps.stg_ready[k], 0));
+        {
+            PhaseScope ph(c, OPP_PH_INJECT);
+            CK(launch_inject(cs, n, ps.dcnt, grid_for(c, n, 4), c->s));
+        }
+        CK(cudaEventRecord(ps.stg_free[k], c->s));
+        c->launches++;
+        ps.n_ub += n;
+        ps.n_exact = false;
+        S.size = -1;
+        return OPP_OK;
     }
     {
         PhaseScope ph(c, OPP_PH_INJECT);
@@ -698,6 +741,68 @@ static int validate_c2c(opp_ctx c, const Col &c2n, const Col &c2c, long long nc)
     return OPP_OK;
 }
 
+// Locality key for the sort by cell: with a principal direction of motion d
+// (opp_init_params.sort_axis; PAPER.md:1544-1560 partitions along the same
+// direction) cells are ranked by (transverse bin across d, position along d),
+// so particles drifting along d keep their place in the sorted order and the
+// periodic re-sort moves data almost in place.  d = 0: plain cell order.
+static int build_sort_key(opp_ctx c, const Col &cn, const Col &np, long long nc) {
+    const double *d = c->p.sort_axis;
+    const double dn = std::sqrt(d[0] * d[0] + d[1] * d[1] + d[2] * d[2]);
+    if (!(dn > 0) || nc == 0) return OPP_OK;
+    double a[3] = {d[0] / dn, d[1] / dn, d[2] / dn};
+    double t[3] = {1, 0, 0};
+    if (std::fabs(a[0]) > 0.9) t[0] = 0, t[1] = 1;
+    double u[3] = {a[1] * t[2] - a[2] * t[1], a[2] * t[0] - a[0] * t[2], a[0] * t[1] - a[1] * t[0]};
+    double un = std::sqrt(u[0] * u[0] + u[1] * u[1] + u[2] * u[2]);
+    for (double &x : u) x /= un;
+    double v[3] = {a[1] * u[2] - a[2] * u[1], a[2] * u[0] - a[0] * u[2], a[0] * u[1] - a[1] * u[0]};
+    const int32_t *c2n = (const int32_t *)cn.host.data();
+    const double *xyz = (const double *)np.host.data();
+    std::vector<double> ax(nc), bu(nc), bv(nc);
+    double vol = 0;
+    for (long long e = 0; e < nc; e++) {
+        double ctr[3] = {0, 0, 0};
+        const double *p[4];
+        for (int k = 0; k < 4; k++) {
+            p[k] = xyz + 3 * (long long)c2n[4 * e + k];
+            for (int q = 0; q < 3; q++) ctr[q] += 0.25 * p[k][q];
+        }
+        double e1[3], e2[3], e3[3];
+        for (int q = 0; q < 3; q++) {
+            e1[q] = p[1][q] - p[0][q];
+            e2[q] = p[2][q] - p[0][q];
+            e3[q] = p[3][q] - p[0][q];
+        }
+        vol += std::fabs(e1[0] * (e2[1] * e3[2] - e2[2] * e3[1]) - e1[1] * (e2[0] * e3[2] - e2[2] * e3[0]) +
+                         e1[2] * (e2[0] * e3[1] - e2[1] * e3[0])) / 6.0;
+        ax[e] = ctr[0] * a[0] + ctr[1] * a[1] + ctr[2] * a[2];
+        bu[e] = ctr[0] * u[0] + ctr[1] * u[1] + ctr[2] * u[2];
+        bv[e] = ctr[0] * v[0] + ctr[1] * v[1] + ctr[2] * v[2];
+    }
+    const double h = std::cbrt(6.0 * vol / nc);   // ~ hex edge of a Kuhn-split mesh
+    std::vector<long long> ku(nc), kv(nc);
+    for (long long e = 0; e < nc; e++) {
+        ku[e] = (long long)std::floor(bu[e] / h);
+        kv[e] = (long long)std::floor(bv[e] / h);
+    }
+    std::vector<int32_t> order(nc);
+    for (long long e = 0; e < nc; e++) order[e] = (int32_t)e;
+    std::sort(order.begin(), order.end(), [&](int32_t p, int32_t q) {
+        if (kv[p] != kv[q]) return kv[p] < kv[q];
+        if (ku[p] != ku[q]) return ku[p] < ku[q];
+        if (ax[p] != ax[q]) return ax[p] < ax[q];
+        return p < q;
+    });
+    std::vector<uint32_t> key(nc);
+    for (long long r = 0; r < nc; r++) key[order[r]] = (uint32_t)r;
+    c->mc.sort_key = (uint32_t *)c->dalloc(4 * nc);
+    if (!c->mc.sort_key) return fail(OPP_ERR_NOMEM, "sort key");
+    CK(cudaMemcpyAsync(c->mc.sort_key, key.data(), 4 * nc, cudaMemcpyHostToDevice, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    return OPP_OK;
+}
+
 static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int cell_ef) {
     MeshCache &m = c->mc;
     Col &cc = c->cols[c2c], &cn = c->cols[c2n], &np = c->cols[node_pos], &ef = c->cols[cell_ef];
@@ -733,6 +838,9 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
             m.sr_cellsum = nullptr;
         }
         c->dfree(m.cell_hist, 0); c->dfree(m.cell_start, 0); c->dfree(m.tile_sums, 0);
+        c->dfree(m.sort_key, 0);
+        m.sort_key = nullptr;
+        TRY(build_sort_key(c, cn, np, nc));
         m.cell_hist = (unsigned *)c->dalloc(4 * (nc + 1));
         m.cell_start = (unsigned *)c->dalloc(4 * (nc + 1));
         m.tile_sums = (unsigned long long *)c->dalloc(8 * opp::scan_tiles(nc + 1));
@@ -839,13 +947,13 @@ static int do_sort(opp_ctx c, PSet &ps, int p2c) {
     const int32_t *pc = (const int32_t *)c->cols[p2c].d;
     {
         PhaseScope ph(c, OPP_PH_SORT_COUNT);
-        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.cell_hist, m.cell_start,
-                             m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
+        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_hist,
+                             m.cell_start, m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.cell_start, ps.head,
-                            grid_for(c, ps.n_ub, 8), c->s));
+        CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_start,
+                            ps.head, grid_for(c, ps.n_ub, 8), c->s));
     }
     c->launches += 7;
     for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
@@ -1062,6 +1170,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.hcap = c->p.hop_cap;
     a.tile_group = c->tile_group;
     a.dbg = c->dbg;
+    a.refill = c->refill;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const bool dh = c->p.direct_hop != 0;

@@ -91,6 +91,7 @@ struct StepArgs {
     int cell_base, n_cells;    // global id of local cell 0, local cell count
     int hpass, hcap;
     int tile_group;            // consecutive 256-particle tiles per block visit (>= 1)
+    int refill;                // tiled kernel: per-lane refill consumer (OPP_REFILL)
     int dbg;                   // diagnostics only (OPP_PMD_DEBUG): 1 stream, 2 +E, 3 +line, 4 no deposit
     Overlay ov;
 };

@@ -86,7 +86,8 @@ __device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, d
         if (l3 < m) { nb = L.cc.w; }
         if (nb < 0) return ST_REMOVE;
         if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
-            cell = nb;
+            cell = nb;       // the hop into the other rank's cell counts here
+            hops++;
             return ST_MIGRATE;
         }
         cell = nb;
@@ -110,9 +111,9 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 
 // Deposit of Eq. 10: Q[c2n[cell][i]] += w * lambda_i.
 // DEP 0: one fp64 reduction per (particle, node).
-// DEP 1: runs of lanes with the same cell (same 4 nodes) are summed with a
-//        segmented suffix scan (5 shuffle steps) and the run head issues the
-//        4 reductions -- "warp-level aggregation of same-cell deposits".
+// DEP 1: lanes with the same cell (same 4 nodes) are aggregated inside the
+//        warp before one set of 4 reductions per cell -- "warp-level
+//        aggregation of same-cell deposits before global atomics".
 template <int DEP>
 __device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int cell, int4 cn,
                                         double w, double l0, double l1, double l2, double l3) {
@@ -126,26 +127,42 @@ __device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int c
         }
         return;
     }
+    // Lanes depositing into the same cell (hence the same 4 nodes) are found
+    // with __match_any_sync wherever they sit in the warp; their 4 values are
+    // summed by a log-step tree over each peer group, and the group's lowest
+    // lane issues the 4 reductions.
     const unsigned lane = lane_id();
-    int key = done ? cell : -2 - (int)lane;
-    if (!done) { v0 = v1 = v2 = v3 = 0.0; }
-    int prev = __shfl_up_sync(0xffffffffu, key, 1);
-    bool head = (lane == 0) || (prev != key);
-    unsigned heads = __ballot_sync(0xffffffffu, head);
-    unsigned above = heads & ~((2u << lane) - 1u);   // heads strictly above this lane
-    if (lane == 31) above = 0;
-    int run_end = above ? (__ffs(above) - 2) : 31;
-#pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-        double t0 = __shfl_down_sync(0xffffffffu, v0, off);
-        double t1 = __shfl_down_sync(0xffffffffu, v1, off);
-        double t2 = __shfl_down_sync(0xffffffffu, v2, off);
-        double t3 = __shfl_down_sync(0xffffffffu, v3, off);
-        if ((int)lane + off <= run_end) {
+    const int key = done ? cell : -2 - (int)lane;
+    unsigned peers = __match_any_sync(0xffffffffu, key);
+    const int first = __ffs(peers) - 1;
+    if (__all_sync(0xffffffffu, peers == (1u << lane))) {   // no duplicates: plain reductions
+        if (done) {
+            atomicAdd(Q + cn.x, v0);
+            atomicAdd(Q + cn.y, v1);
+            atomicAdd(Q + cn.z, v2);
+            atomicAdd(Q + cn.w, v3);
+        }
+        return;
+    }
+    int rel = __popc(peers & ((1u << lane) - 1u));       // my rank inside the group
+    unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
+    if (lane == 31) up = 0;
+    while (__any_sync(0xffffffffu, up != 0)) {
+        const int next = up ? __ffs(up) - 1 : (int)lane;
+        const double t0 = __shfl_sync(0xffffffffu, v0, next);
+        const double t1 = __shfl_sync(0xffffffffu, v1, next);
+        const double t2 = __shfl_sync(0xffffffffu, v2, next);
+        const double t3 = __shfl_sync(0xffffffffu, v3, next);
+        if (up) {
             v0 = add(v0, t0); v1 = add(v1, t1); v2 = add(v2, t2); v3 = add(v3, t3);
         }
+        // lanes at odd group rank have been absorbed by their lower neighbour
+        const unsigned gone = __ballot_sync(0xffffffffu, (rel & 1) != 0);
+        up &= ~gone;
+        // the next surviving peer above: skip the absorbed ones
+        rel >>= 1;
     }
-    if (head && done) {
+    if (done && (int)lane == first) {
         atomicAdd(Q + cn.x, v0);
         atomicAdd(Q + cn.y, v1);
         atomicAdd(Q + cn.z, v2);
@@ -479,7 +496,7 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
-template <int DEP, bool DH, bool MULTI>
+template <int DEP, bool DH, bool MULTI, bool REFILL>
 __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
@@ -509,12 +526,34 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
             }
         return;
     }
-    // Consumer warp: its particle stream is its 32-slot slice of every tile.
+    Tally t;
+    if (!REFILL) {
+        // Consumer warp, warp-synchronous: one 32-particle slice per tile;
+        // the slice is copied to registers and the stage released at once.
+        for (unsigned long long it = 0; it < my; it++) {
+            const int s = (int)(it % kStages);
+            mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
+            StageView v = stage_view(smem, s);
+            const int j = threadIdx.x;
+            double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
+            double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
+            int cell = v.cell[j];
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            const unsigned long long i = tm.tile(it) * kTile + j;
+            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t);
+            a.p2c[i] = cell;
+        }
+        if (blockIdx.x == G - 1)
+            pmd_direct_range<DEP, DH, false, MULTI>(a, ntiles * kTile, n, threadIdx.x & ~31u, kTile, t);
+        flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
+        return;
+    }
+    // Consumer warp with per-lane refill: its particle stream is its 32-slot slice of every tile.
     // Lanes are refilled independently: whenever a lane's particle finishes
     // (DONE / REMOVE / deferred / migrating) it takes the next stream entry,
     // so every iteration advances 32 walks by one cell visit instead of
     // waiting for the warp's longest walk.
-    Tally t;
     const unsigned long long total = 32ull * my;
     unsigned long long pos = 0;
     long long waited = -1;
@@ -604,6 +643,7 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
                     status = ST_REMOVE;
                 } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
                     cell = nb;
+                    hops++;
                     status = ST_MIGRATE;
                 } else {
                     cell = nb;
@@ -1019,8 +1059,14 @@ __device__ __forceinline__ void run_info(int key, unsigned &heads, int &run_star
     run_len = run_end - run_start + 1;
 }
 
+// Sort bucket of a cell: its locality key (see opp_init_params.sort_axis) or
+// the local cell index.
+__device__ __forceinline__ unsigned bucket_of(const uint32_t *__restrict__ skey, int lc) {
+    return skey ? __ldg(skey + lc) : (unsigned)lc;
+}
+
 __global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
-                            unsigned *hist) {
+                            const uint32_t *__restrict__ skey, unsigned *hist) {
     const unsigned long long n = c->n;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
@@ -1032,14 +1078,14 @@ __global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *
         int rs, rl;
         bool head;
         run_info(key, heads, rs, rl, head);
-        if (head && cell >= 0) atomicAdd(hist + (cell - cell_base), (unsigned)rl);
+        if (head && cell >= 0) atomicAdd(hist + bucket_of(skey, cell - cell_base), (unsigned)rl);
     }
 }
 
 // Phase 1: destination slot of every particle (run heads take one atomic
 // per run of equal cells); holes get 0xffffffff.
 __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
-                            unsigned *cursor, uint32_t *dest) {
+                            const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *dest) {
     const unsigned long long n = c->n;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
@@ -1052,7 +1098,8 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
         bool head;
         run_info(key, heads, rs, rl, head);
         unsigned base = 0;
-        if (head && cell >= 0) base = atomicAdd(cursor + (cell - cell_base), (unsigned)rl);
+        if (head && cell >= 0)
+            base = atomicAdd(cursor + bucket_of(skey, cell - cell_base), (unsigned)rl);
         base = __shfl_sync(0xffffffffu, base, rs);
         if (i < n) dest[i] = cell >= 0 ? base + (lane_id() - rs) : 0xffffffffu;
     }
@@ -1242,35 +1289,41 @@ cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
 }
 
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
-                              unsigned *hist, unsigned *start, unsigned long long *tile_sums,
-                              int grid, cudaStream_t s) {
+                              const uint32_t *skey, unsigned *hist, unsigned *start,
+                              unsigned long long *tile_sums, int grid, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(hist, 0, sizeof(unsigned) * (nc + 1), s);
     if (e != cudaSuccess) return e;
-    k_cell_hist<<<grid, 256, 0, s>>>(p2c, c, cell_base, hist);
+    k_cell_hist<<<grid, 256, 0, s>>>(p2c, c, cell_base, skey, hist);
     return scan_exclusive(hist, start, nc + 1, tile_sums, s);
 }
 
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
-                             DevCounters *c, int cell_base, long long nc, unsigned *start,
-                             uint32_t *dest, int grid, cudaStream_t s) {
-    k_sort_rank<<<grid, 256, 0, s>>>(p2c, c, cell_base, start, dest);
+                             DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
+                             unsigned *start, uint32_t *dest, int grid, cudaStream_t s) {
+    k_sort_rank<<<grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest);
     k_sort_move<<<grid, 256, 0, s>>>(src, dst, dest, c);
     k_sort_commit<<<1, 1, 0, s>>>(c, start + nc);
+    return cudaGetLastError();
+}
+
+template <int DEP, bool DH, bool MULTI, bool REFILL>
+static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
     return cudaGetLastError();
 }
 
 template <int DEP, bool DH, bool CONT, bool MULTI>
 static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
     if (!CONT && tiled) {
-        static bool attr = false;
-        if (!attr) {
-            cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI>,
-                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                 kTiledSmem);
-            if (e != cudaSuccess) return e;
-            attr = true;
-        }
-        k_push_move_deposit_tiled<DEP, DH, MULTI><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+        return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
+                        : launch_tiled<DEP, DH, MULTI, false>(a, grid, s);
     } else {
         k_push_move_deposit<DEP, DH, CONT, MULTI><<<grid, 256, 0, s>>>(a);
     }
@@ -1300,10 +1353,10 @@ int pmd_blocks_per_sm(bool tiled) {
     int nb = 0;
     cudaError_t e;
     if (tiled) {
-        cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false>,
+        cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false>,
                              cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &nb, k_push_move_deposit_tiled<0, false, false>, kTiledThreads, kTiledSmem);
+            &nb, k_push_move_deposit_tiled<0, false, false, false>, kTiledThreads, kTiledSmem);
     } else {
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
             &nb, k_push_move_deposit<0, false, false, false>, 256, 0);

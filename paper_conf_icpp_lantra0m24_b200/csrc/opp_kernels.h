@@ -28,11 +28,11 @@ long long scan_tiles(long long n);
 cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
                            unsigned long long *tile_sums, cudaStream_t s);
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
-                              unsigned *hist, unsigned *start, unsigned long long *tile_sums,
-                              int grid, cudaStream_t s);
+                              const uint32_t *skey, unsigned *hist, unsigned *start,
+                              unsigned long long *tile_sums, int grid, cudaStream_t s);
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
-                             DevCounters *c, int cell_base, long long nc, unsigned *start,
-                             uint32_t *dest, int grid, cudaStream_t s);
+                             DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
+                             unsigned *start, uint32_t *dest, int grid, cudaStream_t s);
 
 cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
                              unsigned long long *counts, int grid, cudaStream_t s);

@@ -48,7 +48,8 @@ class opp_init_params(C.Structure):
                 ("direct_hop", C.c_int), ("overlay_spacing", C.c_double),
                 ("hop_budget_per_pass", C.c_int), ("hop_cap", C.c_int),
                 ("allow_growth", C.c_int), ("sort_every", C.c_int),
-                ("tma_pipeline", C.c_int), ("transport", C.c_int)]
+                ("tma_pipeline", C.c_int), ("transport", C.c_int),
+                ("sort_axis", C.c_double * 3)]
 
 
 class opp_step_params(C.Structure):

@@ -1,0 +1,12 @@
+python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -3
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -4
+run() { echo "== $OPP_TILE_GROUP $*"; timeout 300 python bench.py --steps 20 --warmup 3 --no-e2e --no-cpu "$@" 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['value']/1e9,2), round(d['ms_per_step'],3), round(d['roofline']['frac'],3), {k: round(v,3) for k,v in d['phases_ms_per_step'].items()})"; }
+export OPP_TILE_GROUP=16
+for dep in 0 1; do
+run --sort 0 --deposit $dep; run --sort 1 --axis --deposit $dep; run --sort 2 --axis --deposit $dep; run --sort 5 --axis --deposit $dep; run --sort 10 --axis --deposit $dep
+done
+run --sort 2 --axis --deposit 1 --direct
+export OPP_TILE_GROUP=1; run --sort 2 --axis --deposit 1
+export OPP_TILE_GROUP=16
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_push_move_deposit -s 6 -c 1 -o gpurun_out/prof_pmd_d3 python bench.py --steps 4 --warmup 1 --no-e2e --no-cpu --sort 2 --axis --deposit 1 > /dev/null 2>&1; echo ncu $?
+timeout 900 ncu --set full --clock-control none -k regex:k_sort_move -s 2 -c 1 -o gpurun_out/prof_sortmove_axis python bench.py --steps 12 --warmup 1 --no-e2e --no-cpu --sort 2 --axis > /dev/null 2>&1; echo ncu $?

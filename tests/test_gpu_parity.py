@@ -172,12 +172,14 @@ def test_conservation_and_bookkeeping_gpu_only():
     sim.close()
 
 
-@pytest.mark.parametrize("dep,sort_every", [(0, 1), (1, 3), (2, 2)])
-def test_c1_parity_with_periodic_sort(dep, sort_every):
+@pytest.mark.parametrize("dep,sort_every,axis", [(0, 1, 0), (1, 3, 0), (2, 2, 0), (1, 1, 1), (0, 2, 1)])
+def test_c1_parity_with_periodic_sort(dep, sort_every, axis):
     """The periodic counting sort by cell (which also compacts) changes the
-    storage order only: results keyed by id are identical."""
+    storage order only: results keyed by id are identical (plain cell-id key
+    and the locality key along the duct axis)."""
     mesh, ef, init, inject, steps = c1_case()
-    _check(mesh, ef, init, inject, steps, deposit_mode=dep, sort_every=sort_every)
+    _check(mesh, ef, init, inject, steps, deposit_mode=dep, sort_every=sort_every,
+           sort_axis=(0.0, 0.0, 1.0) if axis else (0.0, 0.0, 0.0))
 
 
 def test_sort_by_cell_orders_and_preserves():
