@@ -235,11 +235,14 @@ void orc_overlay_get(const orc_mesh *m, int32_t *out) {
 }
 
 /* DH seed: the overlay cell of x if x is inside the overlay box and the map
- * entry is a tet, otherwise the start cell (S19). */
+ * entry is a tet, otherwise the start cell (S19).  The overlay index is
+ * floor((x - x0) * (1/dx)) with 1/dx rounded once (reading S19'):
+ * the paper gives no formula; a multiply keeps the GPU seed free of a
+ * division per particle and both sides evaluate it identically. */
 static int32_t dh_seed(const orc_mesh *m, const double *x, int32_t cell) {
     int64_t g[3];
     for (int k = 0; k < 3; k++) {
-        double t = (x[k] - m->ov_x0[k]) / m->ov_dx;
+        double t = (x[k] - m->ov_x0[k]) * (1.0 / m->ov_dx);   /* reading S19': index by x * (1/dx) */
         if (!(t >= 0.0)) return cell;
         g[k] = (int64_t)floor(t);
         if (g[k] >= m->ov_n[k]) return cell;
