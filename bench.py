@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
     ap.add_argument("--deposit", type=int, default=0, choices=[0, 1, 2])
     ap.add_argument("--dh", action="store_true")
+    ap.add_argument("--ov", type=float, default=0.5, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=0, help="sort by cell every K steps (0 = never)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
@@ -220,7 +221,7 @@ def run_ours(args, rank, world):
     n_inj_local = n_inj if (world == 1 or mesh["inlet"].shape[0] > 0) else 0
     cap = int(n0 * 1.1) + n_inj_local * (total + 4) + 1024
     sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
-                     direct_hop=args.dh, overlay_spacing=0.5, hop_budget=args.hpass,
+                     direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
                      sort_every=args.sort, tma_pipeline=not args.direct,
                      sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0), **kw)
     init = gc.seed_particles(dm, n0, seed + rank, cluster=cluster, id_base=rank * n0)
@@ -302,7 +303,8 @@ def run_ours(args, rank, world):
         "config": {"workload": name, "mesh_cells": nc, "mesh_nodes": nn,
                    "particles_seeded": n0, "inject_per_step": n_inj,
                    "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
-                   "walk": "DH+MH" if args.dh else "MH", "hop_budget_per_pass": args.hpass,
+                   "walk": f"DH(overlay {args.ov} h)+MH" if args.dh else "MH",
+                   "hop_budget_per_pass": args.hpass,
                    "sort_every": args.sort, "pipeline": "direct" if args.direct else "tma",
                    "sort_key": "axis z" if args.axis else "cell id",
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n_avg * 60 / 1e9),

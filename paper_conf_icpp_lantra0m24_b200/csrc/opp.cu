@@ -875,6 +875,7 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
             tot *= ov.n[k];
         }
         ov.dx = dx;
+        ov.inv_dx = 1.0 / dx;
         if (tot > (1ll << 31)) return fail(OPP_ERR_ARG, "overlay too fine (%lld cells)", tot);
         c->dfree(m.ov_map, 0);
         m.ov_map = (int32_t *)c->dalloc(sizeof(int32_t) * tot);
@@ -953,7 +954,7 @@ static int do_sort(opp_ctx c, PSet &ps, int p2c) {
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
         CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_start,
-                            ps.head, grid_for(c, ps.n_ub, 8), c->s));
+                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), c->s));
     }
     c->launches += 7;
     for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);

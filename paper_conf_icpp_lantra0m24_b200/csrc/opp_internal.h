@@ -66,6 +66,7 @@ struct ColSet {
 struct Overlay {
     double x0[3];
     double dx;
+    double inv_dx;        // 1.0 / dx, rounded once on the host
     int n[3];
     const int32_t *map;   // n[0]*n[1]*n[2], -1 = no tet
 };

@@ -200,9 +200,10 @@ __device__ __forceinline__ void flush_stats(DevCounters *c, unsigned hops, unsig
 
 // DH seed (S19): the overlay cell's tet, else unchanged.
 __device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, double z, int cell) {
-    double t0 = __ddiv_rn(sub(x, ov.x0[0]), ov.dx);
-    double t1 = __ddiv_rn(sub(y, ov.x0[1]), ov.dx);
-    double t2 = __ddiv_rn(sub(z, ov.x0[2]), ov.dx);
+    const double inv = ov.inv_dx;
+    double t0 = mul(sub(x, ov.x0[0]), inv);
+    double t1 = mul(sub(y, ov.x0[1]), inv);
+    double t2 = mul(sub(z, ov.x0[2]), inv);
     if (!(t0 >= 0.0) || !(t1 >= 0.0) || !(t2 >= 0.0)) return cell;
     double f0 = floor(t0), f1 = floor(t1), f2 = floor(t2);
     if (f0 >= (double)ov.n[0] || f1 >= (double)ov.n[1] || f2 >= (double)ov.n[2]) return cell;
@@ -240,6 +241,20 @@ struct TileMap {
     }
     __device__ __forceinline__ unsigned long long tile(unsigned long long it) const {
         return ((it / K) * G + b) * K + it % K;
+    }
+};
+
+// Sequential walk over a block's tiles without 64-bit divisions.
+struct TileIter {
+    unsigned long long group_first, sub, K, step;   // step = G * K
+    __device__ __forceinline__ TileIter(const TileMap &m)
+        : group_first(m.b * m.K), sub(0), K(m.K), step(m.G * m.K) {}
+    __device__ __forceinline__ unsigned long long tile() const { return group_first + sub; }
+    __device__ __forceinline__ void next() {
+        if (++sub == K) {
+            sub = 0;
+            group_first += step;
+        }
     }
 };
 
@@ -397,8 +412,9 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
         const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
         const TileMap tm{(n + 255) / 256, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
         const unsigned long long my = tm.count();
-        for (unsigned long long it = 0; it < my; it++) {
-            const unsigned long long lo = tm.tile(it) * 256;
+        TileIter ti(tm);
+        for (unsigned long long it = 0; it < my; it++, ti.next()) {
+            const unsigned long long lo = ti.tile() * 256;
             pmd_direct_range<DEP, DH, false, MULTI>(a, lo, lo + 256 < n ? lo + 256 : n,
                                                     threadIdx.x & ~31u, 256, t);
         }
@@ -439,29 +455,20 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
 __device__ __forceinline__ void mbar_arrive(uint64_t *b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
+// Blocking wait on an mbarrier phase.  try_wait with a suspend-time hint
+// parks the thread in hardware until the phase completes (or the hint
+// expires), instead of spinning through the L1 data pipe.
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
     uint32_t done;
     do {
         asm volatile(
             "{\n\t.reg .pred p;\n\t"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
             "selp.u32 %0, 1, 0, p;\n\t}"
-            : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+            : "=r"(done) : "r"(smem_u32(b)), "r"(parity), "r"(1000000u) : "memory");
     } while (!done);
 }
-// producer-side wait: back off so the spinning lane does not steal issue slots
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) {
-    uint32_t done;
-    for (;;) {
-        asm volatile(
-            "{\n\t.reg .pred p;\n\t"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, p;\n\t}"
-            : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
-        if (done) return;
-        __nanosleep(64);
-    }
-}
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) { mbar_wait(b, parity); }
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -518,19 +525,22 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
     __syncthreads();
     if (warp == kConsumerWarps) {
         // producer warp: streams tiles kStages ahead of the slowest consumer
-        if (lane == 0)
-            for (unsigned long long it = 0; it < my; it++) {
+        if (lane == 0) {
+            TileIter ti(tm);
+            for (unsigned long long it = 0; it < my; it++, ti.next()) {
                 const int s = (int)(it % kStages);
                 if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
-                issue_tile_load(a, smem, full, s, tm.tile(it));
+                issue_tile_load(a, smem, full, s, ti.tile());
             }
+        }
         return;
     }
     Tally t;
     if (!REFILL) {
         // Consumer warp, warp-synchronous: one 32-particle slice per tile;
         // the slice is copied to registers and the stage released at once.
-        for (unsigned long long it = 0; it < my; it++) {
+        TileIter ti(tm);
+        for (unsigned long long it = 0; it < my; it++, ti.next()) {
             const int s = (int)(it % kStages);
             mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
             StageView v = stage_view(smem, s);
@@ -540,7 +550,7 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
             int cell = v.cell[j];
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
-            const unsigned long long i = tm.tile(it) * kTile + j;
+            const unsigned long long i = ti.tile() * kTile + j;
             pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t);
             a.p2c[i] = cell;
         }
@@ -1085,7 +1095,8 @@ __global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *
 // Phase 1: destination slot of every particle (run heads take one atomic
 // per run of equal cells); holes get 0xffffffff.
 __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
-                            const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *dest) {
+                            const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *dest,
+                            uint32_t *src_of) {
     const unsigned long long n = c->n;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
@@ -1101,28 +1112,28 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
         if (head && cell >= 0)
             base = atomicAdd(cursor + bucket_of(skey, cell - cell_base), (unsigned)rl);
         base = __shfl_sync(0xffffffffu, base, rs);
-        if (i < n) dest[i] = cell >= 0 ? base + (lane_id() - rs) : 0xffffffffu;
+        if (cell >= 0) src_of[base + (lane_id() - rs)] = (uint32_t)i;   // inverse permutation
     }
 }
 
-// Phase 2: pure streaming move src[i] -> dst[dest[i]], each block a
-// contiguous chunk, kSortUnroll independent particles in flight per thread.
+// Phase 2: gather move dst[d] = src[src_of[d]] for d in [0, total): the
+// writes stream in order (full sectors, no read-modify-write of partially
+// written sectors), the reads of nearly sorted data hit sectors that their
+// neighbours in d fetched a moment ago.
 constexpr int kSortUnroll = 4;
-__global__ void __launch_bounds__(256) k_sort_move(ColSet src, ColSet dst,
-                                                   const uint32_t *__restrict__ dest,
-                                                   const DevCounters *c) {
-    const unsigned long long n = c->n;
+__global__ void __launch_bounds__(256) k_sort_gather(ColSet src, ColSet dst,
+                                                     const uint32_t *__restrict__ src_of,
+                                                     const unsigned *__restrict__ total_p) {
+    const unsigned long long n = *total_p;
     const unsigned long long span = (unsigned long long)blockDim.x * kSortUnroll;
-    const unsigned long long chunk = ((n + gridDim.x - 1) / gridDim.x + span - 1) / span * span;
-    const unsigned long long lo = blockIdx.x * chunk;
-    const unsigned long long hi = lo + chunk < n ? lo + chunk : n;
-    for (unsigned long long b = lo; b < hi; b += span) {
-        unsigned long long ii[kSortUnroll];
-        uint32_t dd[kSortUnroll];
+    for (unsigned long long b = (unsigned long long)blockIdx.x * span; b < n;
+         b += (unsigned long long)gridDim.x * span) {
+        unsigned long long dd[kSortUnroll];
+        uint32_t ss[kSortUnroll];
 #pragma unroll
         for (int u = 0; u < kSortUnroll; u++) {
-            ii[u] = b + (unsigned long long)u * blockDim.x + threadIdx.x;
-            dd[u] = ii[u] < hi ? __ldg(dest + ii[u]) : 0xffffffffu;
+            dd[u] = b + (unsigned long long)u * blockDim.x + threadIdx.x;
+            ss[u] = dd[u] < n ? __ldg(src_of + dd[u]) : 0u;
         }
         for (int j = 0; j < src.n; j++) {
             const ColDesc cs = src.c[j], cd = dst.c[j];
@@ -1132,17 +1143,17 @@ __global__ void __launch_bounds__(256) k_sort_move(ColSet src, ColSet dst,
                     long long *dp = reinterpret_cast<long long *>(cd.ptr) + e * cd.cap;
                     long long v[kSortUnroll];
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] != 0xffffffffu ? __ldg(sp + ii[u]) : 0;
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : 0;
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] != 0xffffffffu) dp[dd[u]] = v[u];
+                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
                 } else {
                     const int *sp = reinterpret_cast<const int *>(cs.ptr) + e * cs.cap;
                     int *dp = reinterpret_cast<int *>(cd.ptr) + e * cd.cap;
                     int v[kSortUnroll];
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] != 0xffffffffu ? __ldg(sp + ii[u]) : 0;
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : 0;
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] != 0xffffffffu) dp[dd[u]] = v[u];
+                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
                 }
             }
         }
@@ -1299,9 +1310,12 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
 
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
                              DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
-                             unsigned *start, uint32_t *dest, int grid, cudaStream_t s) {
-    k_sort_rank<<<grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest);
-    k_sort_move<<<grid, 256, 0, s>>>(src, dst, dest, c);
+                             unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
+                             cudaStream_t s) {
+    // the scan left the total in start[nc]; the rank pass consumes start[] as
+    // cursors but never touches start[nc]
+    k_sort_rank<<<grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest, src_of);
+    k_sort_gather<<<grid, 256, 0, s>>>(src, dst, src_of, start + nc);
     k_sort_commit<<<1, 1, 0, s>>>(c, start + nc);
     return cudaGetLastError();
 }
