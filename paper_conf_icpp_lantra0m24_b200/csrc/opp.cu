@@ -1205,6 +1205,13 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     if (dep == OPP_DEP_SORT_SEGRED) {
         PhaseScope ph(c, OPP_PH_SEGRED);
+        if (m.sr_cap < ps.cap) {   // the set may have grown during migration
+            CK(cudaStreamSynchronize(c->s));
+            c->dfree(m.sr_sorted, 0);
+            m.sr_sorted = (double *)c->dalloc(32 * (size_t)ps.cap);
+            if (!m.sr_sorted) return fail(OPP_ERR_NOMEM, "SR sorted buffer");
+            m.sr_cap = ps.cap;
+        }
         CK(launch_sr(a, m.nc, nn, m.cell_hist, m.cell_start, m.tile_sums, m.sr_sorted,
                      m.sr_cellsum, m.n2cs_ptr, m.n2cs, grid_for(c, ps.n_ub, 8), c->s));
         c->launches += 5;

@@ -213,3 +213,32 @@ def test_c1_parity_direct_loads(dep):
     mesh, ef, init, inject, steps = c1_case()
     rep, ost, gst = _check(mesh, ef, init, inject, steps, deposit_mode=dep, tma_pipeline=False)
     assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
+
+
+@pytest.mark.parametrize("dep,dh,sort_every", [(0, True, 3), (1, True, 2), (1, False, 5)])
+def test_every_particle_inside_its_cell_many_steps(dep, dh, sort_every):
+    """Consistency at a larger size over many steps with periodic sorts and
+    injection: every stored (cell, position) pair satisfies the point-in-tet
+    test (up to rounding), charge is conserved and hop counts stay bounded."""
+    import oracle
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh = gen.kuhn_duct(16, 16, 24, jitter=0.2, seed=9)
+    ef = np.tile([0.0, 0.0, 1e-3], (mesh["n_cells"], 1))
+    sim = MiniFemPic(mesh, ef, deposit_mode=dep, direct_hop=dh, overlay_spacing=0.25,
+                     sort_every=sort_every, sort_axis=(0.0, 0.0, 1.0))
+    sim.inject(gen.seed_particles(mesh, 600_000, 9))
+    g, p0, _ = oracle.Mesh.from_gen(mesh).geometry()
+    for s in range(12):
+        sim.inject(gen.inject_batch(mesh, s, 20_000, 9, id_base=10_000_000))
+        st = sim.step(1.0, 1.0, 1.0)
+        assert st["max_hops"] <= 12, st
+        Q = sim.node_charge_host()
+        assert abs(Q.sum() - st["n_after"]) <= 1e-9 * st["n_after"]
+    out = sim.particles()
+    c = out["cell"]
+    d = out["pos"] - p0[c]
+    G = g[c].reshape(-1, 3, 3)
+    l123 = np.einsum("nij,nj->ni", G, d)
+    lam = np.concatenate([1.0 - l123.sum(1, keepdims=True), l123], 1)
+    assert lam.min() >= -1e-9 and lam.max() <= 1 + 1e-9
+    sim.close()
