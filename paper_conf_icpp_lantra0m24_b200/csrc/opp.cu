@@ -126,6 +126,7 @@ struct opp_ctx_s {
     int tile_group = 8;            // OPP_TILE_GROUP: tiles per block visit (TileMap)
     int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
     int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
+    int minb = 1;                  // OPP_MINB: register cap for 3 resident blocks / SM
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -249,6 +250,7 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (const char *tg = getenv("OPP_TILE_GROUP")) c->tile_group = std::max(1, atoi(tg));
     if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
     if (const char *rf = getenv("OPP_REFILL")) c->refill = atoi(rf);
+    if (const char *mb = getenv("OPP_MINB")) c->minb = atoi(mb);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
         delete c;
@@ -1172,6 +1174,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.tile_group = c->tile_group;
     a.dbg = c->dbg;
     a.refill = c->refill;
+    a.minb = c->minb;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const bool dh = c->p.direct_hop != 0;
@@ -1184,7 +1187,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     c->launches++;
     const bool tiled = c->p.tma_pipeline != 0;
-    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled);
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb);
     const int bps = c->bps;
     const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
                                                                        (long long)c->nsm * bps));

@@ -258,10 +258,18 @@ struct TileIter {
     }
 };
 
+__device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b);
+__device__ __forceinline__ void fence_proxy_async_fwd();
+
+// `release`: the stage mbarrier to arrive on once this warp no longer needs
+// the shared-memory copy of its particles (TMA-pipelined kernel; every lane
+// valid) -- after the push has consumed all seven loaded values, so no shared
+// load is still pending when the producer's next bulk copy overwrites it.
 template <int DEP, bool DH, bool CONT, bool MULTI>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          int hops, double &x, double &y, double &z, double &vx,
-                                         double &vy, double &vz, int &cell, Tally &t) {
+                                         double &vy, double &vz, int &cell, Tally &t,
+                                         uint64_t *release = nullptr) {
     int status = ST_NONE;
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -296,6 +304,11 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             // position and velocity are final now: store them before the walk
             a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
             a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+            if (release) {
+                fence_proxy_async_fwd();   // generic reads before the async-proxy refill
+                __syncwarp();
+                if ((threadIdx.x & 31u) == 0) mbar_arrive_fwd(release);
+            }
             if (DH) {
                 const int sc = dh_seed(a.ov, x, y, z, cell);
                 if (sc != cell) {
@@ -469,6 +482,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
     } while (!done);
 }
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) { mbar_wait(b, parity); }
+__device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b) { mbar_arrive(b); }
+__device__ __forceinline__ void fence_proxy_async_fwd() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -503,8 +520,8 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
-template <int DEP, bool DH, bool MULTI, bool REFILL>
-__global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepArgs a) {
+template <int DEP, bool DH, bool MULTI, bool REFILL, int MINB>
+__global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
     uint64_t *empty = full + kStages;
@@ -548,10 +565,8 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
             double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
             double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
             int cell = v.cell[j];
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[s]);
             const unsigned long long i = ti.tile() * kTile + j;
-            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t);
+            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t, &empty[s]);
             a.p2c[i] = cell;
         }
         if (blockIdx.x == G - 1)
@@ -597,11 +612,7 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
                 i = tm.tile(it) * kTile + j;
                 hops = 0;
             }
-            __syncwarp();
-            const unsigned long long npos = pos + k;
-            if (lane == 0)
-                for (unsigned long long tt = pos / 32; tt < npos / 32; tt++)
-                    mbar_arrive(&empty[tt % kStages]);   // our slice of tile tt is read
+            const unsigned long long pos0 = pos, npos = pos + k;
             pos = npos;
             if (take) {
                 const int lc = cell - a.cell_base;
@@ -626,6 +637,12 @@ __global__ void __launch_bounds__(kTiledThreads) k_push_move_deposit_tiled(StepA
                 }
                 active = true;
             }
+            // the push has consumed the shared copies: release fully read slices
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0)
+                for (unsigned long long tt = pos0 / 32; tt < npos / 32; tt++)
+                    mbar_arrive(&empty[tt % kStages]);
         }
         if (!__any_sync(0xffffffffu, active)) break;
         // ---- one cell visit per active lane
@@ -1320,17 +1337,23 @@ cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t
     return cudaGetLastError();
 }
 
-template <int DEP, bool DH, bool MULTI, bool REFILL>
-static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
+template <int DEP, bool DH, bool MULTI, bool REFILL, int MINB>
+static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL>,
+        cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+    k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
     return cudaGetLastError();
+}
+
+template <int DEP, bool DH, bool MULTI, bool REFILL>
+static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
+    return a.minb >= 3 ? launch_tiled_b<DEP, DH, MULTI, REFILL, 3>(a, grid, s)
+                       : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
 }
 
 template <int DEP, bool DH, bool CONT, bool MULTI>
@@ -1363,14 +1386,21 @@ cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, bo
                 : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
 }
 
-int pmd_blocks_per_sm(bool tiled) {
+int pmd_blocks_per_sm(bool tiled, int minb) {
     int nb = 0;
     cudaError_t e;
     if (tiled) {
-        cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &nb, k_push_move_deposit_tiled<0, false, false, false>, kTiledThreads, kTiledSmem);
+        if (minb >= 3) {
+            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false, 3>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &nb, k_push_move_deposit_tiled<0, false, false, false, 3>, kTiledThreads, kTiledSmem);
+        } else {
+            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false, 1>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &nb, k_push_move_deposit_tiled<0, false, false, false, 1>, kTiledThreads, kTiledSmem);
+        }
     } else {
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
             &nb, k_push_move_deposit<0, false, false, false>, 256, 0);
