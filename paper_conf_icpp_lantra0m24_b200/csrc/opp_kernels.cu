@@ -66,11 +66,29 @@ __device__ __forceinline__ bool in01(double v) { return v >= 0.0 && v <= 1.0; }
 // (DONE), at H_cap (DONE, capped), when hops reaches stop_at (NEED_MOVE:
 // deferred), across a boundary face (NEED_REMOVE) or into a cell another
 // rank owns (NEED_MIGRATE).
-template <bool MULTI>
-__device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, double x, double y,
-                                         double z, int &hops, int stop_at, double &l0, double &l1,
+// Position source for the walk: registers, or (TMA-pipelined kernel) the
+// warp's shared output buffer, re-read at every visit so the three doubles do
+// not occupy registers across the line-load latency.
+struct PosRegs {
+    double x, y, z;
+    __device__ __forceinline__ void get(double &a, double &b, double &c) const { a = x; b = y; c = z; }
+};
+struct PosSmem {
+    const double *p;   // p[0], p[32], p[64]
+    __device__ __forceinline__ void get(double &a, double &b, double &c) const {
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(a) : "r"((unsigned)__cvta_generic_to_shared(p)));
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(b) : "r"((unsigned)__cvta_generic_to_shared(p + 32)));
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(c) : "r"((unsigned)__cvta_generic_to_shared(p + 64)));
+    }
+};
+
+template <bool MULTI, typename PS>
+__device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, const PS &ps,
+                                         int &hops, int stop_at, double &l0, double &l1,
                                          double &l2, double &l3, int &capped, int4 &cn) {
     for (;;) {
+        double x, y, z;
+        ps.get(x, y, z);
         bary(L, x, y, z, l0, l1, l2, l3);
         cn = L.cn;
         if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) return ST_DONE;
@@ -246,9 +264,9 @@ struct TileMap {
 
 // Sequential walk over a block's tiles without 64-bit divisions.
 struct TileIter {
-    unsigned long long group_first, sub, K, step;   // step = G * K
+    unsigned group_first, sub, K, step;   // step = G * K; tile ids < 2^32 / kTile
     __device__ __forceinline__ TileIter(const TileMap &m)
-        : group_first(m.b * m.K), sub(0), K(m.K), step(m.G * m.K) {}
+        : group_first((unsigned)(m.b * m.K)), sub(0), K((unsigned)m.K), step((unsigned)(m.G * m.K)) {}
     __device__ __forceinline__ unsigned long long tile() const { return group_first + sub; }
     __device__ __forceinline__ void next() {
         if (++sub == K) {
@@ -257,6 +275,32 @@ struct TileIter {
         }
     }
 };
+
+// TMA-pipelined kernel geometry: tiles of kTile particles, kStages stages.
+constexpr int kTile = 256;
+constexpr int kConsumerWarps = kTile / 32;
+constexpr int kTiledThreads = kTile + 32;
+constexpr int kStages = 4;
+constexpr int kStageBytes = kTile * (6 * 8 + 4);
+constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8 + 2 * (kTile / 32) * 32 * (6 * 8 + 4);
+
+struct StageView {
+    double *c[6];   // x, y, z, vx, vy, vz
+    int *cell;
+};
+__device__ __forceinline__ StageView stage_view(char *smem, int s) {
+    StageView v;
+    char *b = smem + (size_t)s * kStageBytes;
+    for (int k = 0; k < 6; k++) v.c[k] = reinterpret_cast<double *>(b + k * kTile * 8);
+    v.cell = reinterpret_cast<int *>(b + 6 * kTile * 8);
+    return v;
+}
+
+
+// Per-warp output buffers (TMA-out): 2 x [6 x 32 doubles | 32 ints] after the
+// stages and the barriers.
+constexpr int kOutBytes = 32 * (6 * 8 + 4);
+constexpr int kOutBase = kStages * kStageBytes + 2 * kStages * 8;
 
 __device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b);
 __device__ __forceinline__ void fence_proxy_async_fwd();
@@ -269,7 +313,8 @@ template <int DEP, bool DH, bool CONT, bool MULTI>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          int hops, double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
-                                         uint64_t *release = nullptr) {
+                                         uint64_t *release = nullptr, double *sout = nullptr,
+                                         int sj = 0) {
     int status = ST_NONE;
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -302,8 +347,14 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             y = add(y, mul(vy, a.dt));
             z = add(z, mul(vz, a.dt));
             // position and velocity are final now: store them before the walk
-            a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-            a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+            // (TMA-out path: into the shared stage, bulk-stored by the warp)
+            if (sout) {   // per-warp output buffer: 6 columns of 32 doubles
+                sout[sj] = x; sout[32 + sj] = y; sout[64 + sj] = z;
+                sout[96 + sj] = vx; sout[128 + sj] = vy; sout[160 + sj] = vz;
+            } else {
+                a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+                a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+            }
             if (release) {
                 fence_proxy_async_fwd();   // generic reads before the async-proxy refill
                 __syncwarp();
@@ -317,8 +368,8 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 }
             }
         }
-        status = walk_from<MULTI>(a, cell, L, x, y, z, hops,
-                                  a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass), l0, l1, l2, l3,
+        const int stop_at = a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass);
+        status = walk_from<MULTI>(a, cell, L, PosRegs{x, y, z}, hops, stop_at, l0, l1, l2, l3,
                                   capped, cn);
         if (a.dbg == 3 && status == ST_MOVE) status = ST_DONE;
         if (status != ST_MOVE && status != ST_MIGRATE) {   // counted where the walk ends
@@ -448,13 +499,6 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
 // lanes walk far never stalls the others.  The ragged tail (< kTile) takes
 // the direct path.
 // ---------------------------------------------------------------------------
-constexpr int kTile = 256;
-constexpr int kConsumerWarps = kTile / 32;
-constexpr int kTiledThreads = kTile + 32;
-constexpr int kStages = 4;
-constexpr int kStageBytes = kTile * (6 * 8 + 4);
-constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8;
-
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
@@ -494,18 +538,19 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
-
-struct StageView {
-    double *c[6];   // x, y, z, vx, vy, vz
-    int *cell;
-};
-__device__ __forceinline__ StageView stage_view(char *smem, int s) {
-    StageView v;
-    char *b = smem + (size_t)s * kStageBytes;
-    for (int k = 0; k < 6; k++) v.c[k] = reinterpret_cast<double *>(b + k * kTile * 8);
-    v.cell = reinterpret_cast<int *>(b + 6 * kTile * 8);
-    return v;
+__device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                 ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
 }
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read1() {
+    asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
 
 // producer: load tile `tile` into stage s
 __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, uint64_t *full,
@@ -556,19 +601,57 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
     if (!REFILL) {
         // Consumer warp, warp-synchronous: one 32-particle slice per tile;
         // the slice is copied to registers and the stage released at once.
+        // Input: the warp copies its slice to registers, forces the shared
+        // loads to complete, fences the generic proxy against the producer's
+        // next bulk copy and releases the stage at once.  Output: results go
+        // to a per-warp double buffer in shared memory and leave with
+        // cp.async.bulk shared -> global (256-B / 128-B segments per column),
+        // so the LSU pipe carries no particle stores.
         TileIter ti(tm);
         for (unsigned long long it = 0; it < my; it++, ti.next()) {
             const int s = (int)(it % kStages);
+            const int ob_i = (int)(it & 1ull);
             mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
             StageView v = stage_view(smem, s);
             const int j = threadIdx.x;
             double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
             double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
             int cell = v.cell[j];
-            const unsigned long long i = ti.tile() * kTile + j;
-            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t, &empty[s]);
-            a.p2c[i] = cell;
+            const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
+                                         (unsigned long long)__double_as_longlong(y) ^
+                                         (unsigned long long)__double_as_longlong(z) ^
+                                         (unsigned long long)__double_as_longlong(vx) ^
+                                         (unsigned long long)__double_as_longlong(vy) ^
+                                         (unsigned long long)__double_as_longlong(vz) ^
+                                         (unsigned long long)(unsigned)cell;
+            asm volatile("" ::"l"(h));   // the shared loads have landed
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&empty[s]);
+                if (it >= 2) bulk_wait_read1();   // ob[ob_i]'s previous stores have read it
+            }
+            __syncwarp();
+            const unsigned long long tile = ti.tile();
+            const unsigned long long i = tile * kTile + j;
+            double *o = reinterpret_cast<double *>(smem + kOutBase +
+                                                   (size_t)(2 * warp + ob_i) * kOutBytes);
+            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t, nullptr,
+                                            o, (int)lane);
+            reinterpret_cast<int *>(o + 192)[lane] = cell;
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+                const unsigned long long g0 = tile * kTile + warp * 32;
+                for (int k = 0; k < 3; k++) {
+                    bulk_s2g(a.pos + k * a.cap + g0, o + 32 * k, 256);
+                    bulk_s2g(a.vel + k * a.cap + g0, o + 32 * (3 + k), 256);
+                }
+                bulk_s2g(a.p2c + g0, o + 192, 128);
+                bulk_commit();
+            }
         }
+        if (lane == 0) bulk_wait_all();
         if (blockIdx.x == G - 1)
             pmd_direct_range<DEP, DH, false, MULTI>(a, ntiles * kTile, n, threadIdx.x & ~31u, kTile, t);
         flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
