@@ -42,11 +42,12 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="c2", choices=["c2", "c5", "c1"])
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
-    ap.add_argument("--deposit", type=int, default=0, choices=[0, 1, 2])
+    ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
+                    help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
     ap.add_argument("--dh", action="store_true")
     ap.add_argument("--ov", type=float, default=0.5, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
-    ap.add_argument("--sort", type=int, default=0, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--sort", type=int, default=5, help="sort by cell every K steps (0 = never)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
     ap.add_argument("--axis", action="store_true", help="sort key along the duct axis (z)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -138,14 +139,21 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------- oracle legs
-def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster):
-    """Time the CPU oracle (as it stands) on a bounded sample of the workload."""
+def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster, dm=None):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload.
+    The sample's inputs come from the seeded generator (its device twin when a
+    GPU is present: bit-identical, and fast for millions of particles)."""
     import gen
     import oracle
     om = oracle.Mesh.from_gen(mesh)
     om.set_field(ef)
     P = oracle.Particles()
-    init = gen.seed_particles(mesh, n_sample, cfg["seed"], cluster=cluster)
+    if dm is not None:
+        import gen.cuda as gc
+        init = {k: v.cpu().numpy() for k, v in gc.seed_particles(dm, n_sample, cfg["seed"], cluster=cluster).items()
+                if k != "_keep"}
+    else:
+        init = gen.seed_particles(mesh, n_sample, cfg["seed"], cluster=cluster)
     P.append(init["pos"], init["vel"], init["cell"], init["id"])
     Q = np.zeros(mesh["n_nodes"])
     scale = n_sample / max(cfg["n0"], 1)
@@ -366,8 +374,8 @@ def run_ours(args, rank, world):
 
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1)
     if not args.no_cpu and world == 1 and rank == 0:
-        n_sample = 300_000 if args.config != "c1" else cfg["n0"]
-        pushed_c, secs, ninj_c = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, 3, cluster)
+        n_sample = 4_000_000 if args.config != "c1" else cfg["n0"]
+        pushed_c, secs, ninj_c = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, 3, cluster, dm=dm)
         line["cpu_baseline"] = {"value": pushed_c / secs, "unit": UNIT, "cores": 1,
                                 "kind": "oracle",
                                 "sample": f"{n_sample:,} particles of the same workload "

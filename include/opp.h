@@ -90,7 +90,8 @@ typedef struct {
     int direct_hop;             /* 1 = seed the walk from the DH overlay (1356-1370) */
     double overlay_spacing;     /* DH overlay cell size (mesh units); <= 0: auto     */
     int hop_budget_per_pass;    /* H_pass: hops in the fused kernel before a particle
-                                   is deferred to the continuation pass (>= 1)      */
+                                   is deferred to the continuation pass (>= 0;
+                                   0 = the fused kernel tests the start cell only) */
     int hop_cap;                /* H_cap: hops after which the current cell is
                                    accepted as final and counted (S4)               */
     int allow_growth;           /* 1 = grow particle capacity x1.5 on injection     */

@@ -123,7 +123,7 @@ struct opp_ctx_s {
     cudaStream_t cs = nullptr;     // copy stream (host injection staging)
     int nsm = 148;
     int bps = 0;                   // resident blocks / SM of the fused kernel
-    int tile_group = 8;            // OPP_TILE_GROUP: tiles per block visit (TileMap)
+    int tile_group = 16;           // OPP_TILE_GROUP: tiles per block visit (TileMap)
     int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
     int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
     int minb = 1;                  // OPP_MINB: register cap for 3 resident blocks / SM
@@ -231,8 +231,8 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (!params || !out) return fail(OPP_ERR_ARG, "null argument");
     if (params->nranks < 1 || params->rank < 0 || params->rank >= params->nranks)
         return fail(OPP_ERR_ARG, "bad rank/nranks %d/%d", params->rank, params->nranks);
-    if (params->hop_budget_per_pass < 1 || params->hop_cap < 0)
-        return fail(OPP_ERR_ARG, "hop_budget_per_pass must be >= 1 and hop_cap >= 0");
+    if (params->hop_budget_per_pass < 0 || params->hop_cap < 0)
+        return fail(OPP_ERR_ARG, "hop_budget_per_pass and hop_cap must be >= 0");
     if (params->deposit_mode < 0 || params->deposit_mode > OPP_DEP_AUTO)
         return fail(OPP_ERR_ARG, "bad deposit_mode %d", params->deposit_mode);
     if ((params->alloc == nullptr) != (params->free == nullptr))
@@ -1198,13 +1198,12 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     {
         PhaseScope ph(c, OPP_PH_CONTINUE);
-        CK(launch_push_move_deposit(dep, dh, multi, true, false, a,
-                                    std::max(1, std::min(pgrid, c->nsm * 2)), c->s));
+        CK(launch_push_move_deposit(dep, dh, multi, true, false, a, c->nsm * 8, c->s));
     }
     c->launches += 2;
     if (multi) {
         PhaseScope ph(c, OPP_PH_MIGRATE);
-        TRY(migrate_loop(c, ps, a, dep, dh, p2c, std::max(1, std::min(pgrid, c->nsm * 2))));
+        TRY(migrate_loop(c, ps, a, dep, dh, p2c, c->nsm * 8));
     }
     if (dep == OPP_DEP_SORT_SEGRED) {
         PhaseScope ph(c, OPP_PH_SEGRED);

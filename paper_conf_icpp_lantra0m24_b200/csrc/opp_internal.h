@@ -39,10 +39,11 @@ struct DevCounters {
     unsigned long long cum_pushed;       // sum of n_before over all steps
     unsigned long long cum_steps;
     unsigned long long n_mig;            // migrants recorded (current round)
+    unsigned long long work_cursor;      // continuation: next worklist entry to claim
     unsigned long long unpack_done_blocks;
     unsigned int max_hops;
     unsigned int err_flags;              // bit 0: non-positive tet, bit 1: SR overflow
-    unsigned long long pad[9];
+    unsigned long long pad[8];
 };
 
 constexpr int kMaxCols = 16;

@@ -527,6 +527,18 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
 }
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) { mbar_wait(b, parity); }
 __device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b) { mbar_arrive(b); }
+__device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
+    uint32_t done;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
+    return done != 0;
+}
+__device__ __forceinline__ void prefetch_l1(const void *p) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+}
 __device__ __forceinline__ void fence_proxy_async_fwd() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -802,6 +814,105 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
 }
 
 // ---------------------------------------------------------------------------
+// Continuation walk with per-lane refill: finishes the deferred walks (and
+// received migrants).  Each lane carries one particle and advances it by one
+// cell visit per iteration; a lane whose particle finished claims the next
+// worklist entry (the warp leader claims a batch with one atomic), so every
+// iteration keeps ~32 walks in flight instead of waiting for the longest walk
+// of the warp.  Small register footprint -> many resident warps to hide the
+// L2 latency of the line gathers.
+// ---------------------------------------------------------------------------
+template <int DEP, bool MULTI>
+__global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
+    const unsigned long long nw = *(volatile unsigned long long *)&a.cnt->n_work;
+    const unsigned lane = lane_id();
+    const unsigned lt = (1u << lane) - 1u;
+    Tally t;
+    bool active = false, more = true;
+    unsigned long long i = 0;
+    int cell = 0, hops = 0;
+    double x = 0, y = 0, z = 0;
+    Line L;
+    for (;;) {
+        const unsigned need = __ballot_sync(0xffffffffu, !active);
+        if (need && more) {
+            unsigned long long base = 0;
+            const unsigned k = __popc(need);
+            if (lane == 0) base = atomicAdd(&a.cnt->work_cursor, (unsigned long long)k);
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (base + k >= nw) more = false;
+            const unsigned long long q = base + __popc(need & lt);
+            if (!active && q < nw) {
+                i = a.work[q];
+                hops = a.work_hops[q];
+                x = a.pos[i]; y = a.pos[a.cap + i]; z = a.pos[2 * a.cap + i];
+                cell = a.p2c[i];
+                L = load_line(a.lines, cell - a.cell_base);
+                active = true;
+            }
+        }
+        if (!__any_sync(0xffffffffu, active)) break;
+        int status = ST_NONE, capped = 0;
+        double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
+        int4 cn = make_int4(0, 0, 0, 0);
+        if (active) {
+            bary(L, x, y, z, l0, l1, l2, l3);
+            cn = L.cn;
+            if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
+                status = ST_DONE;
+            } else if (hops >= a.hcap) {
+                status = ST_DONE;
+                capped = 1;
+            } else {
+                int nb = L.cc.x;
+                double m = l0;
+                if (l1 < m) { m = l1; nb = L.cc.y; }
+                if (l2 < m) { m = l2; nb = L.cc.z; }
+                if (l3 < m) { nb = L.cc.w; }
+                if (nb < 0) {
+                    status = ST_REMOVE;
+                } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
+                    cell = nb;
+                    hops++;
+                    status = ST_MIGRATE;
+                } else {
+                    cell = nb;
+                    hops++;
+                    L = load_line(a.lines, nb - a.cell_base);
+                }
+            }
+        }
+        const bool fin = status != ST_NONE;
+        if (fin && status != ST_MIGRATE) {
+            t.hops += (unsigned)hops;
+            t.maxh = max(t.maxh, (unsigned)hops);
+            t.capped += (unsigned)capped;
+        }
+        t.removed += (status == ST_REMOVE);
+        const bool done = status == ST_DONE;
+        if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
+        else deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
+        unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
+        if (rem) a.holes[hs] = (uint32_t)i;
+        if (MULTI) {
+            const bool mg = status == ST_MIGRATE;
+            unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
+            if (mg) {
+                a.mig[ms] = (uint32_t)i;
+                a.mig_cell[ms] = cell;
+                a.mig_hops[ms] = hops;
+            }
+        }
+        if (fin) {
+            a.p2c[i] = rem ? -1 : cell;
+            active = false;
+        }
+    }
+    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
+}
+
+// ---------------------------------------------------------------------------
 // Step prologue: zero node charge, reset the per-step counters.
 // ---------------------------------------------------------------------------
 __global__ void k_step_begin(double *Q, long long nn, DevCounters *c, int zero) {
@@ -823,6 +934,7 @@ __global__ void k_step_begin(double *Q, long long nn, DevCounters *c, int zero) 
         c->n_mig = 0;
         c->n_mig_out = 0;
         c->n_mig_in = 0;
+        c->work_cursor = 0;
     }
     if (zero)
         for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nn;
@@ -1360,6 +1472,7 @@ __global__ void k_mig_unpack(ColSet cols, const char *__restrict__ recvbuf, long
         if (t == gridDim.x - 1) {
             c->n = base + (unsigned long long)R;
             c->n_work = (unsigned long long)R;
+            c->work_cursor = 0;
             c->n_mig_out += c->n_mig;
             c->n_mig = 0;
             c->n_mig_in += (unsigned long long)R;
@@ -1444,6 +1557,8 @@ static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStr
     if (!CONT && tiled) {
         return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
                         : launch_tiled<DEP, DH, MULTI, false>(a, grid, s);
+    } else if (CONT) {
+        k_walk_refill<DEP, MULTI><<<grid, 256, 0, s>>>(a);
     } else {
         k_push_move_deposit<DEP, DH, CONT, MULTI><<<grid, 256, 0, s>>>(a);
     }

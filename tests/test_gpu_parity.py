@@ -57,7 +57,7 @@ def _check(mesh, ef, init, inject, steps, hcap=1024, dh=False, **kw):
 
 
 @pytest.mark.parametrize("dep", [0, 1, 2])
-@pytest.mark.parametrize("hpass", [1, 8])
+@pytest.mark.parametrize("hpass", [0, 1, 8])
 def test_c1_parity_mh(dep, hpass):
     mesh, ef, init, inject, steps = c1_case()
     rep, ost, gst = _check(mesh, ef, init, inject, steps, deposit_mode=dep, hop_budget=hpass)
@@ -65,7 +65,7 @@ def test_c1_parity_mh(dep, hpass):
     # identical arithmetic -> identical walks: hop totals match exactly
     assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
     assert [s["max_hops"] for s in gst] == [s["max_hops"] for s in ost]
-    if hpass == 1:
+    if hpass <= 1:
         assert sum(s["n_deferred"] for s in gst) > 0
 
 
