@@ -126,7 +126,8 @@ struct opp_ctx_s {
     int tile_group = 16;           // OPP_TILE_GROUP: tiles per block visit (TileMap)
     int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
     int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
-    int minb = 1;                  // OPP_MINB: register cap for 3 resident blocks / SM
+    int minb = 3;                  // OPP_MINB: register cap for 3 resident blocks / SM
+    int prefetch = 0;              // OPP_PREFETCH: producer-warp L1 warming
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -251,6 +252,7 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
     if (const char *rf = getenv("OPP_REFILL")) c->refill = atoi(rf);
     if (const char *mb = getenv("OPP_MINB")) c->minb = atoi(mb);
+    if (const char *pf = getenv("OPP_PREFETCH")) c->prefetch = atoi(pf);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
         delete c;
@@ -1175,6 +1177,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.dbg = c->dbg;
     a.refill = c->refill;
     a.minb = c->minb;
+    a.prefetch = c->prefetch;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const bool dh = c->p.direct_hop != 0;
@@ -1200,7 +1203,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
         PhaseScope ph(c, OPP_PH_CONTINUE);
         CK(launch_push_move_deposit(dep, dh, multi, true, false, a, c->nsm * 8, c->s));
     }
-    c->launches += 2;
+    c->launches += tiled ? 3 : 2;   // (tiled: pipelined kernel + ragged-tail kernel) + continuation
     if (multi) {
         PhaseScope ph(c, OPP_PH_MIGRATE);
         TRY(migrate_loop(c, ps, a, dep, dh, p2c, c->nsm * 8));

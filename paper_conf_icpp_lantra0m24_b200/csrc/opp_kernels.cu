@@ -282,7 +282,7 @@ constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
 constexpr int kStages = 4;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
-constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8 + 2 * (kTile / 32) * 32 * (6 * 8 + 4);
+constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8 + (kTile / 32) * 32 * (6 * 8 + 4);
 
 struct StageView {
     double *c[6];   // x, y, z, vx, vy, vz
@@ -309,7 +309,7 @@ __device__ __forceinline__ void fence_proxy_async_fwd();
 // the shared-memory copy of its particles (TMA-pipelined kernel; every lane
 // valid) -- after the push has consumed all seven loaded values, so no shared
 // load is still pending when the producer's next bulk copy overwrites it.
-template <int DEP, bool DH, bool CONT, bool MULTI>
+template <int DEP, bool DH, bool CONT, bool MULTI, bool SOUT = false>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          int hops, double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
@@ -334,7 +334,12 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     }
     if (valid) {
         const int lc = cell - a.cell_base;
-        Line L = load_line(a.lines, lc);            // first visit: issued with E
+        // First visit.  Direct paths issue the walk line together with E (one
+        // round trip).  The TMA-out path issues it after the push (through an
+        // opaque dependency on the pushed x) so the 32 line registers and the
+        // particle state are never live at once: fewer registers, more warps.
+        Line L;
+        if (!(SOUT && !CONT)) L = load_line(a.lines, lc);
         if (!CONT) {
             // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
             const double *Ep = reinterpret_cast<const double *>(a.ef + lc);
@@ -348,7 +353,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             z = add(z, mul(vz, a.dt));
             // position and velocity are final now: store them before the walk
             // (TMA-out path: into the shared stage, bulk-stored by the warp)
-            if (sout) {   // per-warp output buffer: 6 columns of 32 doubles
+            if (SOUT) {   // per-warp output buffer: 6 columns of 32 doubles
                 sout[sj] = x; sout[32 + sj] = y; sout[64 + sj] = z;
                 sout[96 + sj] = vx; sout[128 + sj] = vy; sout[160 + sj] = vz;
             } else {
@@ -364,8 +369,14 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 const int sc = dh_seed(a.ov, x, y, z, cell);
                 if (sc != cell) {
                     cell = sc;
-                    L = load_line(a.lines, sc - a.cell_base);
+                    if (!SOUT) L = load_line(a.lines, sc - a.cell_base);
                 }
+            }
+            if (SOUT) {
+                int zero;
+                asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}"
+                             : "=r"(zero) : "d"(z));
+                L = load_line(a.lines, cell - a.cell_base + zero);
             }
         }
         const int stop_at = a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass);
@@ -387,8 +398,10 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     }
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
-    unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
-    if (rem) a.holes[hs] = (uint32_t)i;
+    if (a.dbg != 6) {   // diagnostic 6: skip the hole list (timing only)
+        unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
+        if (rem) a.holes[hs] = (uint32_t)i;
+    }
     if (!CONT) {
         const bool mv = status == ST_MOVE;
         unsigned long long ws = warp_append(mv, &a.cnt->n_work);
@@ -577,6 +590,37 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
+// Producer-warp L1 warming for tile p (already issued; waits until landed).
+__device__ __forceinline__ void warm_tile(const StepArgs &a, char *smem, uint64_t *full,
+                                          unsigned long long p, unsigned lane) {
+    const int sp = (int)(p % kStages);
+    mbar_wait(&full[sp], (uint32_t)((p / kStages) & 1ull));
+    const int *cells = stage_view(smem, sp).cell + lane * (kTile / 32);
+    int prev = INT_MIN;
+    int4 cc[kTile / 32];
+    int lcs[kTile / 32];
+    int nd = 0;
+#pragma unroll
+    for (int k = 0; k < kTile / 32; k++) {
+        const int lc = cells[k] - a.cell_base;
+        if (lc == prev || (unsigned)lc >= (unsigned)a.n_cells) continue;
+        prev = lc;
+        lcs[nd] = lc;
+        cc[nd] = __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(a.lines + lc) + 12));
+        prefetch_l1(a.ef + lc);
+        nd++;
+    }
+    for (int k = 0; k < nd; k++) {
+        const int nb[4] = {cc[k].x, cc[k].y, cc[k].z, cc[k].w};
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const int ln = nb[q] - a.cell_base;
+            if (nb[q] >= 0 && (unsigned)ln < (unsigned)a.n_cells) prefetch_l1(a.lines + ln);
+        }
+        (void)lcs;
+    }
+}
+
 template <int DEP, bool DH, bool MULTI, bool REFILL, int MINB>
 __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
@@ -598,15 +642,22 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
     }
     __syncthreads();
     if (warp == kConsumerWarps) {
-        // producer warp: streams tiles kStages ahead of the slowest consumer
-        if (lane == 0) {
-            TileIter ti(tm);
-            for (unsigned long long it = 0; it < my; it++, ti.next()) {
-                const int s = (int)(it % kStages);
+        // producer warp: lane 0 streams tiles kStages ahead of the slowest
+        // consumer; then the whole warp warms the SM's L1 for the tile that
+        // landed before: the walk lines and fields of its (few, cell-sorted)
+        // start cells and the lines of their four face neighbours -- the
+        // cells the consumers' first visit and first hop will touch.
+        TileIter ti(tm);
+        for (unsigned long long it = 0; it < my; it++, ti.next()) {
+            const int s = (int)(it % kStages);
+            if (lane == 0) {
                 if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
                 issue_tile_load(a, smem, full, s, ti.tile());
             }
+            __syncwarp();
+            if (a.prefetch && it >= 1) warm_tile(a, smem, full, it - 1, lane);
         }
+        if (a.prefetch && my >= 1) warm_tile(a, smem, full, my - 1, lane);
         return;
     }
     Tally t;
@@ -622,7 +673,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
         TileIter ti(tm);
         for (unsigned long long it = 0; it < my; it++, ti.next()) {
             const int s = (int)(it % kStages);
-            const int ob_i = (int)(it & 1ull);
+            const int ob_i = 0;   // one output buffer per warp (keeps 3 blocks / SM in smem)
             mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
             StageView v = stage_view(smem, s);
             const int j = threadIdx.x;
@@ -641,15 +692,15 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&empty[s]);
-                if (it >= 2) bulk_wait_read1();   // ob[ob_i]'s previous stores have read it
+                if (it >= 1) bulk_wait_read0();   // the previous stores have read the buffer
             }
             __syncwarp();
             const unsigned long long tile = ti.tile();
             const unsigned long long i = tile * kTile + j;
             double *o = reinterpret_cast<double *>(smem + kOutBase +
-                                                   (size_t)(2 * warp + ob_i) * kOutBytes);
-            pmd_body<DEP, DH, false, MULTI>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t, nullptr,
-                                            o, (int)lane);
+                                                   (size_t)(warp + ob_i) * kOutBytes);
+            pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
+                                                  nullptr, o, (int)lane);
             reinterpret_cast<int *>(o + 192)[lane] = cell;
             fence_proxy_async();
             __syncwarp();
@@ -664,8 +715,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             }
         }
         if (lane == 0) bulk_wait_all();
-        if (blockIdx.x == G - 1)
-            pmd_direct_range<DEP, DH, false, MULTI>(a, ntiles * kTile, n, threadIdx.x & ~31u, kTile, t);
+        // the ragged tail (< kTile particles) is done by k_push_move_deposit_tail
         flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
         return;
     }
@@ -807,9 +857,18 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             active = false;
         }
     }
-    // ragged tail [ntiles*kTile, n): last block, consumer warps
-    if (blockIdx.x == G - 1)
-        pmd_direct_range<DEP, DH, false, MULTI>(a, ntiles * kTile, n, threadIdx.x & ~31u, kTile, t);
+    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
+}
+
+// Ragged tail of the TMA-pipelined pass: particles [floor(n / kTile) * kTile, n)
+// (fewer than kTile), one block, direct loads.  A separate launch so the
+// register-heavy direct path does not set the pipelined kernel's allocation.
+template <int DEP, bool DH, bool MULTI>
+__global__ void __launch_bounds__(256) k_push_move_deposit_tail(StepArgs a) {
+    const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
+    const unsigned long long lo = n / kTile * kTile;
+    Tally t;
+    pmd_direct_range<DEP, DH, false, MULTI>(a, lo, n, threadIdx.x & ~31u, 256, t);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
@@ -1543,6 +1602,7 @@ static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
         attr = true;
     }
     k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+    k_push_move_deposit_tail<DEP, DH, MULTI><<<1, 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 
