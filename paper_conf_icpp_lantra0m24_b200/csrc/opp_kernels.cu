@@ -282,7 +282,9 @@ constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
 constexpr int kStages = 4;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
-constexpr int kTiledSmem = kStages * kStageBytes + 2 * kStages * 8 + (kTile / 32) * 32 * (6 * 8 + 4);
+constexpr int kRingBytesPerWarp = 64 * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
+constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8 + (kTile / 32) * 32 * (6 * 8 + 4);
+constexpr int kTiledSmem = kRingBase + (kTile / 32) * kRingBytesPerWarp;
 
 struct StageView {
     double *c[6];   // x, y, z, vx, vy, vz
@@ -302,6 +304,51 @@ __device__ __forceinline__ StageView stage_view(char *smem, int s) {
 constexpr int kOutBytes = 32 * (6 * 8 + 4);
 constexpr int kOutBase = kStages * kStageBytes + 2 * kStages * 8;
 
+// Per-warp staging ring for appends to a global list (holes, deferred
+// walks): items are buffered in shared memory and leave 32 at a time with one
+// global atomic, instead of one single-address atomic per warp-iteration
+// (those serialise in L2 when every warp appends).
+constexpr int kRing = 64;
+struct WarpRing {
+    uint32_t *va;          // shared ring of values
+    int32_t *vb;           // optional second value (hop counts), may be null
+    unsigned head, tail;   // warp-uniform
+};
+struct Appends {
+    WarpRing holes, work;
+};
+
+__device__ __forceinline__ void ring_push(WarpRing &r, bool pred, uint32_t va, int32_t vb) {
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    if (!m) return;
+    const unsigned lane = threadIdx.x & 31u;
+    const unsigned slot = r.tail + __popc(m & ((1u << lane) - 1u));
+    if (pred) {
+        r.va[slot & (kRing - 1)] = va;
+        if (r.vb) r.vb[slot & (kRing - 1)] = vb;
+    }
+    r.tail += __popc(m);
+}
+
+__device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *counter, uint32_t *ga,
+                                           int32_t *gb, bool all) {
+    const unsigned lane = threadIdx.x & 31u;
+    while (r.tail - r.head >= 32u || (all && r.tail != r.head)) {
+        const unsigned k = min(32u, r.tail - r.head);
+        __syncwarp();
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(counter, (unsigned long long)k);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (lane < k) {
+            const unsigned sl = (r.head + lane) & (kRing - 1);
+            ga[base + lane] = r.va[sl];
+            if (gb) gb[base + lane] = r.vb[sl];
+        }
+        __syncwarp();
+        r.head += k;
+    }
+}
+
 __device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b);
 __device__ __forceinline__ void fence_proxy_async_fwd();
 
@@ -314,7 +361,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                                          int hops, double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
                                          uint64_t *release = nullptr, double *sout = nullptr,
-                                         int sj = 0) {
+                                         int sj = 0, Appends *ap = nullptr) {
     int status = ST_NONE;
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -398,16 +445,23 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     }
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
-    if (a.dbg != 6) {   // diagnostic 6: skip the hole list (timing only)
+    if (ap) {
+        ring_push(ap->holes, rem, (uint32_t)i, 0);
+        ring_flush(ap->holes, &a.cnt->n_holes, a.holes, nullptr, false);
+        if (!CONT) {
+            ring_push(ap->work, status == ST_MOVE, (uint32_t)i, hops);
+            ring_flush(ap->work, &a.cnt->n_work, a.work, a.work_hops, false);
+        }
+    } else {
         unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
         if (rem) a.holes[hs] = (uint32_t)i;
-    }
-    if (!CONT) {
-        const bool mv = status == ST_MOVE;
-        unsigned long long ws = warp_append(mv, &a.cnt->n_work);
-        if (mv) {
-            a.work[ws] = (uint32_t)i;
-            a.work_hops[ws] = hops;
+        if (!CONT) {
+            const bool mv = status == ST_MOVE;
+            unsigned long long ws = warp_append(mv, &a.cnt->n_work);
+            if (mv) {
+                a.work[ws] = (uint32_t)i;
+                a.work_hops[ws] = hops;
+            }
         }
     }
     if (MULTI) {
@@ -670,6 +724,13 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
         // to a per-warp double buffer in shared memory and leave with
         // cp.async.bulk shared -> global (256-B / 128-B segments per column),
         // so the LSU pipe carries no particle stores.
+        Appends ap;
+        {
+            char *rb = smem + kRingBase + (size_t)warp * kRingBytesPerWarp;
+            ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
+            ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
+                               reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
+        }
         TileIter ti(tm);
         for (unsigned long long it = 0; it < my; it++, ti.next()) {
             const int s = (int)(it % kStages);
@@ -700,7 +761,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             double *o = reinterpret_cast<double *>(smem + kOutBase +
                                                    (size_t)(warp + ob_i) * kOutBytes);
             pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
-                                                  nullptr, o, (int)lane);
+                                                  nullptr, o, (int)lane, &ap);
             reinterpret_cast<int *>(o + 192)[lane] = cell;
             fence_proxy_async();
             __syncwarp();
@@ -714,6 +775,8 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
                 bulk_commit();
             }
         }
+        ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
+        ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
         if (lane == 0) bulk_wait_all();
         // the ragged tail (< kTile particles) is done by k_push_move_deposit_tail
         flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
@@ -886,8 +949,20 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
     const unsigned long long nw = *(volatile unsigned long long *)&a.cnt->n_work;
     const unsigned lane = lane_id();
     const unsigned lt = (1u << lane) - 1u;
+    // Warps walk the worklist in 32-entry groups, group g = gw + k * nwarps
+    // (no shared claim counter: a single-address atomic per refill serialises
+    // in L2), so the entries in flight form one moving window of the worklist
+    // -- and of the mesh, since the list follows the cell-sorted storage.
+    const unsigned long long nwarps = (unsigned long long)gridDim.x * (blockDim.x >> 5);
+    const unsigned long long gw = (unsigned long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const unsigned long long gstep = nwarps * 32;
+    unsigned long long gstart = gw * 32;                          // current group
+    unsigned long long cur = gstart;                              // next unclaimed entry
+    unsigned long long gend = gstart + 32 < nw ? gstart + 32 : nw;
+    __shared__ uint32_t hring[8][kRing];
+    WarpRing hr{hring[threadIdx.x >> 5], nullptr, 0u, 0u};
     Tally t;
-    bool active = false, more = true;
+    bool active = false, more = gstart < nw;
     unsigned long long i = 0;
     int cell = 0, hops = 0;
     double x = 0, y = 0, z = 0;
@@ -895,13 +970,31 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
     for (;;) {
         const unsigned need = __ballot_sync(0xffffffffu, !active);
         if (need && more) {
-            unsigned long long base = 0;
-            const unsigned k = __popc(need);
-            if (lane == 0) base = atomicAdd(&a.cnt->work_cursor, (unsigned long long)k);
-            base = __shfl_sync(0xffffffffu, base, 0);
-            if (base + k >= nw) more = false;
-            const unsigned long long q = base + __popc(need & lt);
-            if (!active && q < nw) {
+            // the r-th needing lane takes the r-th unclaimed entry: first from
+            // the current group, then from the warp's next group
+            const unsigned r = __popc(need & lt), k = __popc(need);
+            const unsigned long long left = gend - cur;
+            const unsigned long long nstart = gstart + gstep;
+            const unsigned long long nend = nstart + 32 < nw ? nstart + 32 : nw;
+            unsigned long long q = ~0ull;
+            if (r < left) q = cur + r;
+            else if (nstart + (r - left) < nend) q = nstart + (r - left);
+            if (k < left) {
+                cur += k;
+            } else {
+                gstart = nstart;
+                gend = nend;
+                cur = nstart + (k - left);
+                if (gstart >= nw) {
+                    more = false;
+                } else if (cur >= gend) {
+                    gstart += gstep;
+                    cur = gstart;
+                    gend = gstart + 32 < nw ? gstart + 32 : nw;
+                    more = gstart < nw;
+                }
+            }
+            if (!active && q != ~0ull) {
                 i = a.work[q];
                 hops = a.work_hops[q];
                 x = a.pos[i]; y = a.pos[a.cap + i]; z = a.pos[2 * a.cap + i];
@@ -952,8 +1045,8 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
         if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
         else deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
         const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
-        unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
-        if (rem) a.holes[hs] = (uint32_t)i;
+        ring_push(hr, rem, (uint32_t)i, 0);
+        ring_flush(hr, &a.cnt->n_holes, a.holes, nullptr, false);
         if (MULTI) {
             const bool mg = status == ST_MIGRATE;
             unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
@@ -968,6 +1061,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
             active = false;
         }
     }
+    ring_flush(hr, &a.cnt->n_holes, a.holes, nullptr, true);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
