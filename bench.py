@@ -44,8 +44,8 @@ def parse():
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
-    ap.add_argument("--dh", action="store_true")
-    ap.add_argument("--ov", type=float, default=0.5, help="DH overlay spacing (mesh units)")
+    ap.add_argument("--mh", action="store_true", help="multi-hop only (no direct-hop seeding)")
+    ap.add_argument("--ov", type=float, default=0.25, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=5, help="sort by cell every K steps (0 = never)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
@@ -53,7 +53,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
-    return ap.parse_args()
+    args = ap.parse_args()
+    args.dh = not args.mh      # direct-hop seeding is the default
+    return args
 
 
 # ---------------------------------------------------------------- workload
