@@ -45,7 +45,9 @@ def parse():
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
     ap.add_argument("--mh", action="store_true", help="multi-hop only (no direct-hop seeding)")
-    ap.add_argument("--ov", type=float, default=0.25, help="DH overlay spacing (mesh units)")
+    ap.add_argument("--dhmode", type=int, default=1,
+                    help="1: overlay seed for every particle; 2: only for particles that left their cell")
+    ap.add_argument("--ov", type=float, default=0.125, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=5, help="sort by cell every K steps (0 = never)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
@@ -54,7 +56,7 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
     args = ap.parse_args()
-    args.dh = not args.mh      # direct-hop seeding is the default
+    args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
     return args
 
 
@@ -313,7 +315,7 @@ def run_ours(args, rank, world):
         "config": {"workload": name, "mesh_cells": nc, "mesh_nodes": nn,
                    "particles_seeded": n0, "inject_per_step": n_inj,
                    "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
-                   "walk": f"DH(overlay {args.ov} h)+MH" if args.dh else "MH",
+                   "walk": (f"DH{args.dh}(overlay {args.ov} h)+MH" if args.dh else "MH"),
                    "hop_budget_per_pass": args.hpass,
                    "sort_every": args.sort, "pipeline": "direct" if args.direct else "tma",
                    "sort_key": "axis z" if args.axis else "cell id",

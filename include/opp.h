@@ -87,7 +87,11 @@ typedef struct {
     opp_free_fn free;           /*  allocator); NULL = cudaMalloc / cudaFree         */
     void *alloc_user;
     int deposit_mode;           /* enum opp_deposit_mode                             */
-    int direct_hop;             /* 1 = seed the walk from the DH overlay (1356-1370) */
+    int direct_hop;             /* DH: 0 = multi-hop only;
+                                   1 = every particle's walk starts at the overlay
+                                   seed of its pushed position; 2 = only a particle
+                                   no longer inside its cell takes the seed
+                                   (reading S19''); else OPP_ERR_ARG    */
     double overlay_spacing;     /* DH overlay cell size (mesh units); <= 0: auto     */
     int hop_budget_per_pass;    /* H_pass: hops in the fused kernel before a particle
                                    is deferred to the continuation pass (>= 0;

@@ -184,12 +184,14 @@ class Particles:
 
 
 def step(mesh: Mesh, parts: Particles, c1: float, dt: float, w: float, Q: np.ndarray,
-         hcap: int = 1024, use_dh: bool = False, zero_charge: bool = True) -> dict:
-    """One oracle time step on an already-injected population (orc_step)."""
+         hcap: int = 1024, use_dh: int = 0, zero_charge: bool = True) -> dict:
+    """One oracle time step on an already-injected population (orc_step).
+    use_dh: 0 multi-hop only, 1 overlay seed for every particle, 2 overlay
+    seed only for particles no longer inside their cell (reading S19'')."""
     assert Q.dtype == np.float64 and Q.flags.c_contiguous and Q.shape[0] == mesh.nn
     if use_dh and mesh.overlay is None:
         raise ValueError("build_overlay first")
-    prm = _Params(float(c1), float(dt), float(w), int(hcap), int(bool(use_dh)),
+    prm = _Params(float(c1), float(dt), float(w), int(hcap), int(use_dh),
                   int(bool(zero_charge)), 0)
     st = _Stats()
     lib().orc_step(mesh.h, parts.h, C.byref(prm), _p(Q), C.byref(st))

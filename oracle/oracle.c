@@ -335,7 +335,8 @@ typedef struct {
     double dt;
     double w;       /* macro-particle weight Q_p (Eq. 10, 682-696)          */
     int32_t hcap;   /* H_cap, S4                                             */
-    int32_t use_dh; /* direct-hop seeding from the overlay                  */
+    int32_t use_dh; /* 1: overlay seed for every particle; 2: only for those
+                       that left their cell (reading S19'')                  */
     int32_t zero_charge;
     int32_t pad;
 } orc_params;
@@ -350,7 +351,8 @@ typedef struct {
  *   zero node charge; for each particle in storage order
  *     E = E[cell]                          (start-of-step cell, S6)
  *     v <- v + c1*E ; x <- x + v*dt        (leap-frog, v at half steps, S5)
- *     [DH] cell <- overlay seed(x)
+ *     [DH=1] cell <- overlay seed(x)
+ *     [DH=2] if x is not inside cell: cell <- overlay seed(x)
  *     walk -> DONE | REMOVE                (MH)
  *     DONE: Q[c2n[cell][i]] += w*lambda_i  (Eq. 10)
  *   compact: drop REMOVE particles, keep the survivors' order.
@@ -387,7 +389,16 @@ int orc_step(const orc_mesh *m, orc_parts *p, const orc_params *prm, double *Q, 
             v[k] = v[k] + prm->c1 * E[k];
             x[k] = x[k] + v[k] * prm->dt;
         }
-        if (prm->use_dh) cell = dh_seed(m, x, cell);
+        if (prm->use_dh == 1) {
+            cell = dh_seed(m, x, cell);
+        } else if (prm->use_dh == 2) {
+            /* DESIGN.md reading S19'': only a particle that is no longer in
+             * its cell takes the overlay seed ("particles are moved directly
+             * to a cell closer to the final destination") */
+            double l0[4];
+            orc_bary(m, cell, x, l0);
+            if (!inside(l0)) cell = dh_seed(m, x, cell);
+        }
         double lam[4];
         int32_t fc, hops, capped;
         int status = orc_walk(m, cell, x, 0, prm->hcap, &fc, &hops, lam, &capped);

@@ -236,6 +236,8 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
         return fail(OPP_ERR_ARG, "hop_budget_per_pass and hop_cap must be >= 0");
     if (params->deposit_mode < 0 || params->deposit_mode > OPP_DEP_AUTO)
         return fail(OPP_ERR_ARG, "bad deposit_mode %d", params->deposit_mode);
+    if (params->direct_hop < 0 || params->direct_hop > 2)
+        return fail(OPP_ERR_ARG, "bad direct_hop %d (0, 1 or 2)", params->direct_hop);
     if ((params->alloc == nullptr) != (params->free == nullptr))
         return fail(OPP_ERR_ARG, "alloc and free callbacks go together");
     CK(cudaSetDevice(params->device));
@@ -876,7 +878,8 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         for (int k = 0; k < 3; k++) {
             ov.x0[k] = lo[k];
             ov.n[k] = std::max(1, (int)std::ceil((hi[k] - lo[k]) / dx));
-            tot *= ov.n[k];
+            ov.nb[k] = (ov.n[k] + (k == 2 ? 1 : 3)) / (k == 2 ? 2 : 4);
+            tot *= ov.nb[k] * (k == 2 ? 2 : 4);
         }
         ov.dx = dx;
         ov.inv_dx = 1.0 / dx;
@@ -1018,7 +1021,7 @@ static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int
 // that entered another rank's cells are packed (every column + hop count),
 // exchanged point-to-point, appended at the end of the receiver's dats and
 // walked on there; repeated until no rank has migrants.
-static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, bool dh, int p2c, int cgrid) {
+static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p2c, int cgrid) {
     opp::Comm *cm = c->comm;
     const int R = cm->nranks, me = cm->rank;
     int p2c_col = -1, rec = 0, pos = -1, vel = -1;
@@ -1180,7 +1183,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.prefetch = c->prefetch;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
-    const bool dh = c->p.direct_hop != 0;
+    const int dh = c->p.direct_hop;
     const bool multi = c->p.nranks > 1;
     if (multi && !c->comm->partitioned) return fail(OPP_ERR_STATE, "nranks > 1: call opp_set_partition first");
 

@@ -69,7 +69,8 @@ struct Overlay {
     double dx;
     double inv_dx;        // 1.0 / dx, rounded once on the host
     int n[3];
-    const int32_t *map;   // n[0]*n[1]*n[2], -1 = no tet
+    int nb[3];            // bricks of 4x4x2 overlay cells (see ov_slot)
+    const int32_t *map;   // nb[0]*nb[1]*nb[2]*32 slots, -1 = no tet / padding
 };
 
 struct StepArgs {

@@ -49,6 +49,23 @@ __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, in
     return l;
 }
 
+// Cell field E (double4, 32-B aligned) in one 256-bit read-only load.
+__device__ __forceinline__ void load_E(const double4 *__restrict__ ef, int lc, double2 &exy,
+                                       double &ez) {
+    double pad;
+    asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+        : "=d"(exy.x), "=d"(exy.y), "=d"(ez), "=d"(pad) : "l"(ef + lc));
+}
+
+// Overlay slot of overlay cell (ix, iy, iz): 4x4x2 bricks of 32 ints (one
+// 128-B line), so the particles of one tet -- a few overlay cells in every
+// direction -- touch a few lines instead of one line per (iy, iz) row.
+__device__ __forceinline__ long long ov_slot(const Overlay &ov, int ix, int iy, int iz) {
+    const long long b = (long long)(ix >> 2) +
+                        (long long)ov.nb[0] * ((long long)(iy >> 2) + (long long)ov.nb[1] * (iz >> 1));
+    return b * 32 + (ix & 3) + 4 * (iy & 3) + 16 * (iz & 1);
+}
+
 // Barycentric coordinates, node-relative form, fixed evaluation order.
 __device__ __forceinline__ void bary(const Line &l, double x, double y, double z, double &l0,
                                      double &l1, double &l2, double &l3) {
@@ -60,6 +77,7 @@ __device__ __forceinline__ void bary(const Line &l, double x, double y, double z
 }
 
 __device__ __forceinline__ bool in01(double v) { return v >= 0.0 && v <= 1.0; }
+
 
 // Multi-hop walk (Fig. 6 template 1098-1124).  `cell` is a
 // global id in/out and L its already-loaded walk line; stops when inside
@@ -217,17 +235,37 @@ __device__ __forceinline__ void flush_stats(DevCounters *c, unsigned hops, unsig
 }
 
 // DH seed (S19): the overlay cell's tet, else unchanged.
-__device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, double z, int cell) {
+// dh_slot: the overlay slot of a position, -1 outside the overlay box.
+__device__ __forceinline__ long long dh_slot(const Overlay &ov, double x, double y, double z) {
     const double inv = ov.inv_dx;
     double t0 = mul(sub(x, ov.x0[0]), inv);
     double t1 = mul(sub(y, ov.x0[1]), inv);
     double t2 = mul(sub(z, ov.x0[2]), inv);
-    if (!(t0 >= 0.0) || !(t1 >= 0.0) || !(t2 >= 0.0)) return cell;
+    if (!(t0 >= 0.0) || !(t1 >= 0.0) || !(t2 >= 0.0)) return -1;
     double f0 = floor(t0), f1 = floor(t1), f2 = floor(t2);
-    if (f0 >= (double)ov.n[0] || f1 >= (double)ov.n[1] || f2 >= (double)ov.n[2]) return cell;
-    long long g = (long long)f0 + (long long)ov.n[0] * ((long long)f1 + (long long)ov.n[1] * (long long)f2);
+    if (f0 >= (double)ov.n[0] || f1 >= (double)ov.n[1] || f2 >= (double)ov.n[2]) return -1;
+    return ov_slot(ov, (int)f0, (int)f1, (int)f2);
+}
+
+__device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, double z, int cell) {
+    const long long g = dh_slot(ov, x, y, z);
+    if (g < 0) return cell;
     int s = __ldg(ov.map + g);
     return s >= 0 ? s : cell;
+}
+
+// DH mode 2 (reading S19''): a particle no longer inside its cell (L = its
+// line) takes the overlay seed; one still inside keeps cell and line.
+__device__ __forceinline__ void dh_if_left(const StepArgs &a, double x, double y, double z,
+                                           int &cell, Line &L) {
+    double l0, l1, l2, l3;
+    bary(L, x, y, z, l0, l1, l2, l3);
+    if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) return;
+    const int sc = dh_seed(a.ov, x, y, z, cell);
+    if (sc != cell) {
+        cell = sc;
+        L = load_line(a.lines, sc - a.cell_base);
+    }
 }
 
 }  // namespace
@@ -356,7 +394,7 @@ __device__ __forceinline__ void fence_proxy_async_fwd();
 // the shared-memory copy of its particles (TMA-pipelined kernel; every lane
 // valid) -- after the push has consumed all seven loaded values, so no shared
 // load is still pending when the producer's next bulk copy overwrites it.
-template <int DEP, bool DH, bool CONT, bool MULTI, bool SOUT = false>
+template <int DEP, int DH, bool CONT, bool MULTI, bool SOUT = false>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          int hops, double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
@@ -389,9 +427,9 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         if (!(SOUT && !CONT)) L = load_line(a.lines, lc);
         if (!CONT) {
             // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
-            const double *Ep = reinterpret_cast<const double *>(a.ef + lc);
-            const double2 Exy = __ldg(reinterpret_cast<const double2 *>(Ep));
-            const double Ez = __ldg(Ep + 2);
+            double2 Exy;
+            double Ez;
+            load_E(a.ef, lc, Exy, Ez);
             vx = add(vx, mul(a.c1, Exy.x));
             vy = add(vy, mul(a.c1, Exy.y));
             vz = add(vz, mul(a.c1, Ez));
@@ -412,7 +450,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 __syncwarp();
                 if ((threadIdx.x & 31u) == 0) mbar_arrive_fwd(release);
             }
-            if (DH) {
+            if (DH == 1) {   // seed every particle from the overlay
                 const int sc = dh_seed(a.ov, x, y, z, cell);
                 if (sc != cell) {
                     cell = sc;
@@ -425,6 +463,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                              : "=r"(zero) : "d"(z));
                 L = load_line(a.lines, cell - a.cell_base + zero);
             }
+            if (DH == 2) dh_if_left(a, x, y, z, cell, L);
         }
         const int stop_at = a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass);
         status = walk_from<MULTI>(a, cell, L, PosRegs{x, y, z}, hops, stop_at, l0, l1, l2, l3,
@@ -509,7 +548,7 @@ __device__ __forceinline__ void load_pstate(const StepArgs &a, unsigned long lon
     }
 }
 
-template <int DEP, bool DH, bool CONT, bool MULTI>
+template <int DEP, int DH, bool CONT, bool MULTI>
 __device__ __forceinline__ void pmd_direct_range(const StepArgs &a, unsigned long long lo,
                                                  unsigned long long hi, unsigned long long first,
                                                  unsigned long long stride, Tally &t) {
@@ -531,7 +570,7 @@ __device__ __forceinline__ void pmd_direct_range(const StepArgs &a, unsigned lon
 // Pass 1 (direct variant): every block owns one contiguous chunk of the
 // particle array, so in cell-sorted storage the walk lines a block touches
 // stay hot in its SM's L1.  Continuation: grid-stride over the worklist.
-template <int DEP, bool DH, bool CONT, bool MULTI>
+template <int DEP, int DH, bool CONT, bool MULTI>
 __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
     Tally t;
     if (CONT) {
@@ -675,7 +714,7 @@ __device__ __forceinline__ void warm_tile(const StepArgs &a, char *smem, uint64_
     }
 }
 
-template <int DEP, bool DH, bool MULTI, bool REFILL, int MINB>
+template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
 __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
@@ -825,9 +864,9 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             if (take) {
                 const int lc = cell - a.cell_base;
                 L = load_line(a.lines, lc);
-                const double *Ep = reinterpret_cast<const double *>(a.ef + lc);
-                const double2 Exy = __ldg(reinterpret_cast<const double2 *>(Ep));
-                const double Ez = __ldg(Ep + 2);
+                double2 Exy;
+                double Ez;
+                load_E(a.ef, lc, Exy, Ez);
                 vx = add(vx, mul(a.c1, Exy.x));
                 vy = add(vy, mul(a.c1, Exy.y));
                 vz = add(vz, mul(a.c1, Ez));
@@ -836,13 +875,14 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
                 z = add(z, mul(vz, a.dt));
                 a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
                 a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-                if (DH) {
+                if (DH == 1) {
                     const int sc = dh_seed(a.ov, x, y, z, cell);
                     if (sc != cell) {
                         cell = sc;
                         L = load_line(a.lines, sc - a.cell_base);
                     }
                 }
+                if (DH == 2) dh_if_left(a, x, y, z, cell, L);
                 active = true;
             }
             // the push has consumed the shared copies: release fully read slices
@@ -926,7 +966,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
 // Ragged tail of the TMA-pipelined pass: particles [floor(n / kTile) * kTile, n)
 // (fewer than kTile), one block, direct loads.  A separate launch so the
 // register-heavy direct path does not set the pipelined kernel's allocation.
-template <int DEP, bool DH, bool MULTI>
+template <int DEP, int DH, bool MULTI>
 __global__ void __launch_bounds__(256) k_push_move_deposit_tail(StepArgs a) {
     const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
     const unsigned long long lo = n / kTile * kTile;
@@ -1266,8 +1306,7 @@ __global__ void k_overlay_build(const WalkLine *__restrict__ lines, const double
                     double l0, l1, l2, l3;
                     bary(L, x, y, z, l0, l1, l2, l3);
                     if (l0 >= 0.0 && l1 >= 0.0 && l2 >= 0.0 && l3 >= 0.0)
-                        atomicMin(map + gx + (long long)ov.n[0] * (gy + (long long)ov.n[1] * gz),
-                                  (int)c + cell_base);
+                        atomicMin(map + ov_slot(ov, gx, gy, gz), (int)c + cell_base);
                 }
     }
 }
@@ -1686,7 +1725,7 @@ cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t
     return cudaGetLastError();
 }
 
-template <int DEP, bool DH, bool MULTI, bool REFILL, int MINB>
+template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
 static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
     static bool attr = false;
     if (!attr) {
@@ -1700,13 +1739,13 @@ static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-template <int DEP, bool DH, bool MULTI, bool REFILL>
+template <int DEP, int DH, bool MULTI, bool REFILL>
 static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
     return a.minb >= 3 ? launch_tiled_b<DEP, DH, MULTI, REFILL, 3>(a, grid, s)
                        : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
 }
 
-template <int DEP, bool DH, bool CONT, bool MULTI>
+template <int DEP, int DH, bool CONT, bool MULTI>
 static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
     if (!CONT && tiled) {
         return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
@@ -1720,19 +1759,25 @@ static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStr
 }
 
 template <bool CONT>
-static cudaError_t launch_pmd_c(int dep, bool dh, bool multi, const StepArgs &a, int grid,
+static cudaError_t launch_pmd_c(int dep, int dh, bool multi, const StepArgs &a, int grid,
                                 bool tiled, cudaStream_t s) {
+    if (CONT) dh = 0;   // the continuation resumes walks: no seeding
 #define OPP_CASE(D, H, M) \
     if (dep == D && dh == H && multi == M) return launch_pmd_t<D, H, CONT, M>(a, grid, tiled, s);
-    OPP_CASE(0, false, false) OPP_CASE(0, true, false) OPP_CASE(1, false, false)
-    OPP_CASE(1, true, false) OPP_CASE(2, false, false) OPP_CASE(2, true, false)
-    OPP_CASE(0, false, true) OPP_CASE(0, true, true) OPP_CASE(1, false, true)
-    OPP_CASE(1, true, true) OPP_CASE(2, false, true) OPP_CASE(2, true, true)
+#define OPP_CASES(H) \
+    OPP_CASE(0, H, false) OPP_CASE(1, H, false) OPP_CASE(2, H, false) \
+    OPP_CASE(0, H, true) OPP_CASE(1, H, true) OPP_CASE(2, H, true)
+    OPP_CASES(0)
+    if (!CONT) {
+        OPP_CASES(1)
+        OPP_CASES(2)
+    }
+#undef OPP_CASES
 #undef OPP_CASE
     return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_push_move_deposit(int dep, bool dh, bool multi, bool cont, bool tiled,
+cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, bool tiled,
                                      const StepArgs &a, int grid, cudaStream_t s) {
     return cont ? launch_pmd_c<true>(dep, dh, multi, a, grid, tiled, s)
                 : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
@@ -1743,19 +1788,19 @@ int pmd_blocks_per_sm(bool tiled, int minb) {
     cudaError_t e;
     if (tiled) {
         if (minb >= 3) {
-            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false, 3>,
+            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, 3>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &nb, k_push_move_deposit_tiled<0, false, false, false, 3>, kTiledThreads, kTiledSmem);
+                &nb, k_push_move_deposit_tiled<0, 0, false, false, 3>, kTiledThreads, kTiledSmem);
         } else {
-            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, false, false, false, 1>,
+            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, 1>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &nb, k_push_move_deposit_tiled<0, false, false, false, 1>, kTiledThreads, kTiledSmem);
+                &nb, k_push_move_deposit_tiled<0, 0, false, false, 1>, kTiledThreads, kTiledSmem);
         }
     } else {
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &nb, k_push_move_deposit<0, false, false, false>, 256, 0);
+            &nb, k_push_move_deposit<0, 0, false, false>, 256, 0);
     }
     return (e == cudaSuccess && nb > 0) ? nb : 1;
 }
@@ -1836,7 +1881,7 @@ cudaError_t launch_pack_field(const double *ef, long long nc, double4 *out, cuda
 
 cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long nc, int cell_base,
                            const Overlay &ov, int32_t *map, cudaStream_t s) {
-    long long tot = (long long)ov.n[0] * ov.n[1] * ov.n[2];
+    long long tot = (long long)ov.nb[0] * ov.nb[1] * ov.nb[2] * 32;   // bricks incl. padding
     int g1 = (int)((tot + 255) / 256), g2 = (int)((nc + 255) / 256);
     k_overlay_init<<<g1 > 0 ? g1 : 1, 256, 0, s>>>(map, tot);
     k_overlay_build<<<g2 > 0 ? g2 : 1, 256, 0, s>>>(lines, xyz, nc, cell_base, ov, map);

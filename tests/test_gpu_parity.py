@@ -69,10 +69,10 @@ def test_c1_parity_mh(dep, hpass):
         assert sum(s["n_deferred"] for s in gst) > 0
 
 
-@pytest.mark.parametrize("dep", [0, 1])
-def test_c1_parity_dh(dep):
+@pytest.mark.parametrize("dep,mode", [(0, 1), (1, 1), (0, 2), (1, 2), (2, 2)])
+def test_c1_parity_dh(dep, mode):
     mesh, ef, init, inject, steps = c1_case(drift=0.6, spread=0.3)
-    rep, ost, gst = _check(mesh, ef, init, inject, steps, dh=True, deposit_mode=dep,
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, dh=mode, deposit_mode=dep,
                            overlay_spacing=0.5)
     assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
 
@@ -215,7 +215,7 @@ def test_c1_parity_direct_loads(dep):
     assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
 
 
-@pytest.mark.parametrize("dep,dh,sort_every", [(0, True, 3), (1, True, 2), (1, False, 5)])
+@pytest.mark.parametrize("dep,dh,sort_every", [(0, 1, 3), (1, 1, 2), (1, 0, 5), (1, 2, 5)])
 def test_every_particle_inside_its_cell_many_steps(dep, dh, sort_every):
     """Consistency at a larger size over many steps with periodic sorts and
     injection: every stored (cell, position) pair satisfies the point-in-tet

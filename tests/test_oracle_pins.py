@@ -297,7 +297,7 @@ def test_direct_hop_equals_multi_hop(c1_mesh_jit):
     p = gen.seed_particles(m, 5000, seed=12, drift=0.6, spread=0.3)
     ef = np.zeros((m["n_cells"], 3))
     res = {}
-    for dh in (False, True):
+    for dh in (0, 1, 2):
         om = oracle.Mesh.from_gen(m)
         om.set_field(ef)
         om.build_overlay([0.0, 0.0, 0.0], 0.5, [12, 12, 60])
@@ -306,12 +306,43 @@ def test_direct_hop_equals_multi_hop(c1_mesh_jit):
         Q = np.zeros(m["n_nodes"])
         st = oracle.step(om, P, 1.0, 1.0, 1.0, Q, use_dh=dh)
         res[dh] = (P.get(), Q, st)
-    a, b = res[False][0], res[True][0]
-    np.testing.assert_array_equal(a["id"], b["id"])
-    ok = np.minimum(a["margin"], b["margin"]) > 1e-10
-    np.testing.assert_array_equal(a["cell"][ok], b["cell"][ok])
-    assert res[True][2]["total_hops"] < res[False][2]["total_hops"]
-    np.testing.assert_allclose(res[False][1], res[True][1], rtol=1e-12, atol=1e-12)
+    a = res[0][0]
+    for dh in (1, 2):
+        b = res[dh][0]
+        np.testing.assert_array_equal(a["id"], b["id"])
+        ok = np.minimum(a["margin"], b["margin"]) > 1e-10
+        np.testing.assert_array_equal(a["cell"][ok], b["cell"][ok])
+        assert res[dh][2]["total_hops"] < res[0][2]["total_hops"]
+        np.testing.assert_allclose(res[0][1], res[dh][1], rtol=1e-12, atol=1e-12)
+    # mode 2 consults the overlay only for particles that left their cell, so
+    # it never takes more hops than multi-hop alone on any particle that stays
+    assert res[2][2]["total_hops"] <= res[0][2]["total_hops"]
+
+
+def test_direct_hop_mode2_stayers_take_no_hop(c1_mesh_jit):
+    """DH mode 2 (reading S19''): a particle still inside its cell after the
+    push keeps it with zero hops, even where the overlay would seed another
+    tet (centre of the overlay cell in a neighbour)."""
+    m = c1_mesh_jit
+    g, p0, _ = oracle.Mesh.from_gen(m).geometry()
+    # particles at rest at tet centroids: they stay where they are
+    cells = np.arange(0, m["n_cells"], 7, dtype=np.int32)
+    xyz = m["node_xyz"][m["c2n"][cells]].mean(axis=1)
+    ef = np.zeros((m["n_cells"], 3))
+    om = oracle.Mesh.from_gen(m)
+    om.set_field(ef)
+    om.build_overlay([0.0, 0.0, 0.0], 1.0, [3, 2, 15])   # coarse: seeds often wrong
+    P = oracle.Particles()
+    P.append(xyz, np.zeros_like(xyz), cells, np.arange(cells.size, dtype=np.int64))
+    Q = np.zeros(m["n_nodes"])
+    st = oracle.step(om, P, 1.0, 1.0, 1.0, Q, use_dh=2)
+    assert st["total_hops"] == 0
+    np.testing.assert_array_equal(P.get()["cell"], cells)
+    P1 = oracle.Particles()
+    P1.append(xyz, np.zeros_like(xyz), cells, np.arange(cells.size, dtype=np.int64))
+    st1 = oracle.step(om, P1, 1.0, 1.0, 1.0, np.zeros(m["n_nodes"]), use_dh=1)
+    assert st1["total_hops"] > 0          # mode 1 re-walks from the (coarse) seed
+    np.testing.assert_array_equal(P1.get()["cell"], cells)
 
 
 # ---------------------------------------------------------------- P10 injection
