@@ -127,6 +127,8 @@ struct opp_ctx_s {
     int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
     int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
     int minb = 3;                  // OPP_MINB: register cap for 3 resident blocks / SM
+    int sort_hgrid = 8;            // OPP_SORT_HGRID / OPP_SORT_RGRID: blocks per SM of the
+    int sort_rgrid = 8;            //   sort histogram / rank kernels
     int prefetch = 0;              // OPP_PREFETCH: producer-warp L1 warming
     std::vector<Set> sets;
     std::vector<Col> cols;
@@ -254,6 +256,8 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
     if (const char *rf = getenv("OPP_REFILL")) c->refill = atoi(rf);
     if (const char *mb = getenv("OPP_MINB")) c->minb = atoi(mb);
+    if (const char *e = getenv("OPP_SORT_HGRID")) c->sort_hgrid = atoi(e);
+    if (const char *e = getenv("OPP_SORT_RGRID")) c->sort_rgrid = atoi(e);
     if (const char *pf = getenv("OPP_PREFETCH")) c->prefetch = atoi(pf);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
@@ -956,12 +960,13 @@ static int do_sort(opp_ctx c, PSet &ps, int p2c) {
     {
         PhaseScope ph(c, OPP_PH_SORT_COUNT);
         CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_hist,
-                             m.cell_start, m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
+                             m.cell_start, m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
         CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_start,
-                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), c->s));
+                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), grid_for(c, ps.n_ub, c->sort_rgrid),
+                            c->s));
     }
     c->launches += 7;
     for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);

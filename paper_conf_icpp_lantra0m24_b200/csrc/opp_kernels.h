@@ -33,7 +33,7 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
                              DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
                              unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
-                             cudaStream_t s);
+                             int rank_grid, cudaStream_t s);
 
 cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
                              unsigned long long *counts, int grid, cudaStream_t s);
