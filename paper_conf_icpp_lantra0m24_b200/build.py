@@ -12,7 +12,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libopp.so")
+LIB = os.environ.get("OPP_LIB_OUT", os.path.join(HERE, "libopp.so"))
 SOURCES = ["opp.cu", "opp_kernels.cu", "opp_comm.cu"]
 HEADERS = ["opp_internal.h", "opp_kernels.h", "opp_comm.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -33,7 +33,7 @@ def _nccl_dir():
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-Wall",
          "--expt-relaxed-constexpr", "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"),
-         "-I", CSRC]
+         "-I", CSRC] + os.environ.get("OPP_NVCC_EXTRA", "").split()
 
 
 def _stale() -> bool:

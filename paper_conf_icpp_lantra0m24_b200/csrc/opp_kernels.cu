@@ -242,9 +242,12 @@ __device__ __forceinline__ long long dh_slot(const Overlay &ov, double x, double
     double t1 = mul(sub(y, ov.x0[1]), inv);
     double t2 = mul(sub(z, ov.x0[2]), inv);
     if (!(t0 >= 0.0) || !(t1 >= 0.0) || !(t2 >= 0.0)) return -1;
-    double f0 = floor(t0), f1 = floor(t1), f2 = floor(t2);
-    if (f0 >= (double)ov.n[0] || f1 >= (double)ov.n[1] || f2 >= (double)ov.n[2]) return -1;
-    return ov_slot(ov, (int)f0, (int)f1, (int)f2);
+    // floor(t) for t >= 0 as one saturating fp64 -> int conversion each (the
+    // conversion unit is the slow part of this lookup; no FRND + I2F pair);
+    // t >= 2^31 saturates to INT_MAX and fails the range test like floor(t).
+    const int f0 = __double2int_rd(t0), f1 = __double2int_rd(t1), f2 = __double2int_rd(t2);
+    if (f0 >= ov.n[0] || f1 >= ov.n[1] || f2 >= ov.n[2]) return -1;
+    return ov_slot(ov, f0, f1, f2);
 }
 
 __device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, double z, int cell) {
@@ -318,7 +321,14 @@ struct TileIter {
 constexpr int kTile = 256;
 constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
-constexpr int kStages = 4;
+#ifndef OPP_STAGES
+#define OPP_STAGES 2   // measured on C2: 2 stages leave more of the L1/shared array to
+                       // L1 for the walk lines (pmd 1.91 -> 1.87 ms vs 4 stages)
+#endif
+#ifndef OPP_MINB_HI
+#define OPP_MINB_HI 3   // resident blocks per SM the register budget is cut for
+#endif
+constexpr int kStages = OPP_STAGES;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
 constexpr int kRingBytesPerWarp = 64 * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
 constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8 + (kTile / 32) * 32 * (6 * 8 + 4);
@@ -427,6 +437,18 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         if (!(SOUT && !CONT)) L = load_line(a.lines, lc);
         if (!CONT) {
             // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
+            // DH: the overlay entry of the drift-only position x + v dt is
+            // fetched together with E; it is used only when the pushed
+            // position lies in the same overlay cell (all but ~|c1 E dt| / dx
+            // of the particles), so the seed is exactly that of the pushed
+            // position and the lookup leaves the dependent chain.
+            long long spec_slot = -1;
+            int spec_val = -1;
+            if (DH == 1) {
+                spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
+                                    add(z, mul(vz, a.dt)));
+                spec_val = __ldg(a.ov.map + (spec_slot >= 0 ? spec_slot : 0));
+            }
             double2 Exy;
             double Ez;
             load_E(a.ef, lc, Exy, Ez);
@@ -451,7 +473,10 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 if ((threadIdx.x & 31u) == 0) mbar_arrive_fwd(release);
             }
             if (DH == 1) {   // seed every particle from the overlay
-                const int sc = dh_seed(a.ov, x, y, z, cell);
+                const long long g = dh_slot(a.ov, x, y, z);
+                int v = g == spec_slot ? spec_val : (g >= 0 ? __ldg(a.ov.map + g) : -1);
+                if (g < 0) v = -1;
+                int sc = v >= 0 ? v : cell;
                 if (sc != cell) {
                     cell = sc;
                     if (!SOUT) L = load_line(a.lines, sc - a.cell_base);
@@ -1759,6 +1784,13 @@ static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
         cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
         if (e != cudaSuccess) return e;
+        // shared-memory carveout (percent of the unified L1/shared array);
+        // what the stages do not take is L1 for the walk lines (OPP_CARVEOUT)
+        if (const char *cv = getenv("OPP_CARVEOUT")) {
+            e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB>,
+                                     cudaFuncAttributePreferredSharedMemoryCarveout, atoi(cv));
+            if (e != cudaSuccess) return e;
+        }
         attr = true;
     }
     k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
@@ -1768,7 +1800,7 @@ static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
 
 template <int DEP, int DH, bool MULTI, bool REFILL>
 static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
-    return a.minb >= 3 ? launch_tiled_b<DEP, DH, MULTI, REFILL, 3>(a, grid, s)
+    return a.minb >= 3 ? launch_tiled_b<DEP, DH, MULTI, REFILL, OPP_MINB_HI>(a, grid, s)
                        : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
 }
 
@@ -1815,10 +1847,10 @@ int pmd_blocks_per_sm(bool tiled, int minb) {
     cudaError_t e;
     if (tiled) {
         if (minb >= 3) {
-            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, 3>,
+            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &nb, k_push_move_deposit_tiled<0, 0, false, false, 3>, kTiledThreads, kTiledSmem);
+                &nb, k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>, kTiledThreads, kTiledSmem);
         } else {
             cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, 1>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
