@@ -233,6 +233,30 @@ def inject_batch(mesh: dict, step: int, n_inj: int, seed: int, v_inj: float = 0.
     }
 
 
+def duct_bc(mesh: dict, wall=None, inlet=None, outlet=None, node_xyz=None):
+    """Dirichlet boundary data for the field solve (an input, like the mesh):
+    returns (mask int32[nn], value fp64[nn]).  A None value leaves that
+    boundary homogeneous-Neumann.  Side walls are x in {0, X} or y in {0, Y};
+    the inlet is z = 0, the outlet z = Z (Mini-FEM-PIC, PAPER.md:1495-1500:
+    "the outer wall is fixed at a higher potential"; reading F3:
+    a node on both a wall and the inlet/outlet takes the wall value).
+    Boundary nodes of a Kuhn duct sit exactly on the box (jitter moves
+    interior nodes only), so the tests are exact comparisons."""
+    xyz = mesh["node_xyz"] if node_xyz is None else node_xyz
+    x0, x1, y0, y1, z0, z1 = mesh["box"]
+    nn = xyz.shape[0]
+    mask = np.zeros(nn, dtype=np.int32)
+    val = np.zeros(nn, dtype=np.float64)
+    for v, sel in ((inlet, xyz[:, 2] == z0), (outlet, xyz[:, 2] == z1),
+                   (wall, (xyz[:, 0] == x0) | (xyz[:, 0] == x1) | (xyz[:, 1] == y0) | (xyz[:, 1] == y1))):
+        if v is None:
+            continue
+        vv = np.broadcast_to(np.asarray(v, dtype=np.float64), (nn,)) if np.ndim(v) else np.full(nn, float(v))
+        mask[sel] = 1
+        val[sel] = vv[sel]
+    return mask, val
+
+
 def hot_block_cells(mesh: dict, lo=(18, 18, 30), size=(12, 12, 12)) -> np.ndarray:
     """Cells of the hex block [lo, lo+size) (config C5's clustered region)."""
     nx, ny = mesh["nx"], mesh["ny"]
