@@ -6,8 +6,10 @@ particle population: inject (a1) -> zero node charge (a2) -> gather E + push
 (a3, a4) -> multi-hop walk (a6, optionally DH-seeded a5) -> deposit (a7) ->
 write-back / holes (a8) -> hole fill (a9).  Default workload = config C2
 (BASELINE.json configs[1]): 48x48x72 Kuhn duct (995,328 tets), a pre-seeded
-50M-particle steady state plus 250k injected per step, fixed uniform field (the
-CG field solve is timed separately in the paper's plan and is not built yet).
+50M-particle steady state plus 250k injected per step; every step first solves
+the field (P1 FEM Poisson by the persistent CG kernel, Fig. 1 step 1) from the
+previous step's charge.  The field solve is timed separately (SURVEY.md §8(d):
+"value" counts the particle loop; "field" and "value_incl_field" report it).
 
 Contract: W untimed warm-up steps, then exactly K timed steps bracketed by a
 barrier + cuda synchronize; CUDA events on the library's stream; max over
@@ -55,8 +57,16 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
+    ap.add_argument("--field", type=int, default=-1,
+                    help="solve the field (CG) every step: 1 on, 0 off (fixed uniform E); "
+                         "default: on for c2, off otherwise")
+    ap.add_argument("--rhs", type=float, default=2e-7, help="field solve: b = rhs * node charge")
+    ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
+    ap.add_argument("--cg-tol", type=float, default=1e-10)
     args = ap.parse_args()
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
+    if args.field < 0:   # the CG is single-GPU: multi-GPU runs keep the fixed field
+        args.field = 1 if (args.config == "c2" and int(os.environ.get("WORLD_SIZE", "1")) == 1) else 0
     return args
 
 
@@ -75,7 +85,8 @@ def workload(args, world=1):
     if cfg.get("cluster"):
         cluster = (cfg["cluster"], gen.hot_block_cells(mesh))
     name = {"c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
-                  "+ 250k injected/step, fixed uniform E",
+                  "+ 250k injected/step, " + ("CG Poisson field solve every step" if args.field
+                                              else "fixed uniform E"),
             "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
             "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
     return cfg, mesh, ef, qm, dt, cluster, name
@@ -229,6 +240,10 @@ def run_ours(args, rank, world):
             cluster = (cluster[0], cluster[1][(cluster[1] >= base) & (cluster[1] < base + mesh["n_cells"])] - base)
     else:
         gen_mesh = mesh
+    if args.field and world > 1:
+        raise SystemExit("--field 1 is single-GPU only (the CG is not slab-partitioned)")
+    if args.field:
+        ef = np.zeros_like(ef)
     dm = gc.DeviceMesh(gen_mesh)
     n_inj_local = n_inj if (world == 1 or mesh["inlet"].shape[0] > 0) else 0
     cap = int(n0 * 1.1) + n_inj_local * (total + 4) + 1024
@@ -236,6 +251,9 @@ def run_ours(args, rank, world):
                      direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
                      sort_every=args.sort, tma_pipeline=not args.direct,
                      sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0), **kw)
+    if args.field:
+        fmask, fval = gen.duct_bc(mesh, wall=args.wall, inlet=0.0)
+        sim.field_init(fmask, fval)
     init = gc.seed_particles(dm, n0, seed + rank, cluster=cluster, id_base=rank * n0)
     if base:
         init["cell"] += base
@@ -251,7 +269,12 @@ def run_ours(args, rank, world):
                for s in range(total)]
     torch.cuda.synchronize()
 
+    def field():
+        if args.field:
+            sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=True, stats=False)
+
     def one_step(s, on_device=True, readback=None):
+        field()
         if batches[s] is not None:
             sim.inject(batches[s] if on_device else host_batches[s], on_device=on_device)
         sim.step(dt, qm, w, stats=False, fill=True)
@@ -285,7 +308,8 @@ def run_ours(args, rank, world):
         ms = D.max_over_ranks(ms)
         pushed = D.sum_over_ranks(pushed)
         launches = D.sum_over_ranks(launches)
-    value = pushed / (ms / 1e3)
+    field_ms = phases["field"][0] if args.field else 0.0
+    value = pushed / ((ms - field_ms) / 1e3)  # the particle loop; field apart
     n_avg = pushed / args.steps / world       # per GPU
 
     # ---- roofline of the dominant kernel (k_push_move_deposit, pass 1)
@@ -335,6 +359,15 @@ def run_ours(args, rank, world):
                  "deferred_last_step": st1["n_deferred"]},
         "clocks": clk.summary(),
     }
+    if args.field:
+        fst = sim.field_stats()
+        line["field"] = {"ms_per_step": field_ms / args.steps, "cg_iterations_last": fst["iterations"],
+                         "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
+                         "rhs_scale": args.rhs, "wall_potential": args.wall,
+                         "solver": "Jacobi-PCG, one persistent cooperative kernel, warm start",
+                         "note": "value excludes the field solve (timed separately, SURVEY.md "
+                                 "§8(d)); value_incl_field counts it"}
+        line["value_incl_field"] = pushed / (ms / 1e3)
 
     # ---- e2e: same metric through the C ABI with HOST buffers
     if not args.no_e2e:
@@ -357,7 +390,10 @@ def run_ours(args, rank, world):
         s_lo, s_hi = args.warmup, args.warmup + ke
         if host_batches[s_lo] is not None:
             sim.inject(host_batches[s_lo], on_device=False)
+        sim.phase_timing(args.field)
+        sim.phase_times()
         for s in range(s_lo, s_hi):
+            field()
             sim.step(dt, qm, w, stats=False, fill=True)
             if s + 1 < s_hi and host_batches[s + 1] is not None:
                 sim.inject(host_batches[s + 1], on_device=False)
@@ -365,6 +401,9 @@ def run_ours(args, rank, world):
         e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
+        if args.field:
+            ems -= sim.phase_times()["field"][0]
+        sim.phase_timing(False)
         s1 = sim.last_stats()
         epushed = s1["cum_pushed"] - s0["cum_pushed"]
         if world > 1:

@@ -260,7 +260,7 @@ int opp_get_dat_device_ptr(opp_ctx ctx, int32_t dat_or_map, void **ptr, int64_t 
 enum opp_phase { OPP_PH_INJECT = 0, OPP_PH_BEGIN = 1, OPP_PH_PUSH_MOVE_DEPOSIT = 2,
                  OPP_PH_CONTINUE = 3, OPP_PH_SEGRED = 4, OPP_PH_FILL = 5, OPP_PH_MIGRATE = 6,
                  OPP_PH_HALO = 7, OPP_PH_SORT_COUNT = 8, OPP_PH_SORT_MOVE = 9,
-                 OPP_N_PHASES = 10 };
+                 OPP_PH_FIELD = 10, OPP_N_PHASES = 11 };
 
 /* enable != 0: record CUDA events on the context stream around every phase
  * of the following calls (negligible overhead, no host synchronisation). */
@@ -273,6 +273,59 @@ int opp_get_phase_times(opp_ctx ctx, double *ms_sum, int64_t *count);
 
 /* Number of kernels this context has launched so far (evidence counter). */
 int64_t opp_kernel_launch_count(opp_ctx ctx);
+
+/* ---------------------------------------------------------------------------
+ * Field solve: step 1 of the PIC loop (Fig. 1, Gauss' law
+ * Eq. 1) by the finite-element method on the tetrahedral mesh.
+ * Mini-FEM-PIC's ComputeJMatrix / ComputeF1Vector / linear solve /
+ * ComputeElectricField (Fig. 6) in the
+ * linear form north_star names ("a plain GPU conjugate-gradient on the FEM
+ * Poisson system"; the Boltzmann-electron Newton solve is out of scope):
+ *   K phi = b,  K_ij = sum_e V_e grad(lambda_i) . grad(lambda_j)   (P1 Laplacian)
+ *   b = rhs_scale * node_charge    (the consistent P1 load of the deposited
+ *                                   point charges, Eq. 10; F2)
+ *   phi = dirichlet_value on Dirichlet nodes; homogeneous Neumann elsewhere
+ *   E_c = -sum_i phi[c2n[c][i]] grad(lambda_i)   (cell-constant, 1576-1585)
+ * One rank only (nranks > 1: OPP_ERR_STATE).
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    double rhs_scale;   /* b = rhs_scale * node_charge (q / eps0 per unit weight)       */
+    double tol;         /* stop when ||r||_2 <= tol * ||b_F - K_FD phi_D||_2 (>= 0)      */
+    int max_iter;       /* iteration cap (>= 0)                                          */
+    int warm_start;     /* 1: free nodes start from node_potential's current values     */
+    int precond;        /* 0: plain CG; 1: Jacobi (diagonal) preconditioned CG          */
+} opp_field_params;
+
+typedef struct {
+    int32_t iterations; /* CG iterations of the last solve                              */
+    int32_t converged;  /* 1 if the tolerance was met (0: max_iter reached)             */
+    double rel_residual;/* ||r||_2 / ||b_F - K_FD phi_D||_2 (recursive residual)         */
+    double rhs_norm;    /* ||b_F - K_FD phi_D||_2                                        */
+} opp_field_stats;
+
+/* Build the P1 system on the mesh of c2n (cells -> nodes, dim 4) with node
+ * coordinates node_pos (dim 3 OPP_REAL): the sparsity (sliced ELLPACK, 32
+ * rows per slice), the stiffness values (assembled on the device in a fixed
+ * order: deterministic) and the Dirichlet data.  dirichlet_mask[n] != 0 marks
+ * node n Dirichlet with value dirichlet_value[n] (host arrays of the node
+ * count; copied).  Maps are static: call again to rebuild.
+ * Errors: OPP_ERR_ARG (handles, NULL), OPP_ERR_MESH (c2n out of range),
+ * OPP_ERR_NOMEM, OPP_ERR_STATE (nranks > 1).  Synchronises. */
+int opp_field_init(opp_ctx ctx, opp_map c2n, opp_dat node_pos, const int32_t *dirichlet_mask,
+                   const double *dirichlet_value);
+
+/* Solve for node_potential (node dat dim 1 OPP_REAL; in: warm start if
+ * params->warm_start, out: phi) from node_charge (node dat dim 1 OPP_REAL,
+ * e.g. after opp_push_move_deposit), then write cell_ef (cell dat dim 3
+ * OPP_REAL; -1 = skip) = -grad(phi) per cell, which the next
+ * opp_push_move_deposit gathers.  One persistent cooperative kernel runs the
+ * whole CG; enqueued on the stream; stats may be NULL (no synchronisation;
+ * read them later with opp_get_field_stats). */
+int opp_field_solve(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential, opp_dat cell_ef,
+                    const opp_field_params *params, opp_field_stats *stats);
+
+/* Statistics of the last opp_field_solve; synchronises. */
+int opp_get_field_stats(opp_ctx ctx, opp_field_stats *stats);
 
 /* Synchronise the context's stream; reports sticky asynchronous errors. */
 int opp_sync(opp_ctx ctx);

@@ -9,6 +9,7 @@
 #include "opp_internal.h"
 #include "opp_kernels.h"
 #include "opp_comm.h"
+#include "opp_field.h"
 
 #include <algorithm>
 #include <cstdarg>
@@ -115,6 +116,19 @@ struct MeshCache {
     long long sr_cap = 0;
 };
 
+// Field solve state (opp_field_init / opp_field_solve).
+struct FieldState {
+    bool ready = false;
+    int c2n = -1, node_pos = -1;
+    long long nn = 0, nc = 0;
+    FieldMat K;
+    int32_t *n2c_ptr = nullptr, *n2c = nullptr;
+    double *vec = nullptr;          // r, u, w, p, s: 5 * nn
+    double *part = nullptr;         // 3 * part_cap block partials
+    long long part_cap = 0;
+    CgState *st = nullptr;
+};
+
 }  // namespace
 
 struct opp_ctx_s {
@@ -134,6 +148,7 @@ struct opp_ctx_s {
     std::vector<Col> cols;
     std::vector<PSet> psets;
     MeshCache mc;
+    FieldState fs;
     DevCounters *hcnt = nullptr;   // pinned mirror
     long long launches = 0;
     int cell_base = 0;             // global id of local cell 0 (slab partition)
@@ -299,6 +314,15 @@ static void free_pset(opp_ctx c, PSet &ps) {
     ps = PSet();
 }
 
+static void free_field(opp_ctx c) {
+    FieldState &f = c->fs;
+    c->dfree(f.K.slice_off, 0); c->dfree(f.K.col, 0); c->dfree(f.K.val, 0);
+    c->dfree(f.K.dinv, 0); c->dfree(f.K.dmask, 0); c->dfree(f.K.dval, 0);
+    c->dfree(f.n2c_ptr, 0); c->dfree(f.n2c, 0); c->dfree(f.vec, 0); c->dfree(f.part, 0);
+    c->dfree(f.st, 0);
+    f = FieldState();
+}
+
 extern "C" int opp_finalize(opp_ctx c) {
     if (!c) return OPP_OK;
     cudaSetDevice(c->p.device);
@@ -320,6 +344,7 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.sr_cellsum, 0);
     c->dfree(m.n2cs_ptr, 0);
     c->dfree(m.n2cs, 0);
+    free_field(c);
     if (c->comm) opp::comm_free(c->comm);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     cudaStreamSynchronize(c->cs);
@@ -1358,5 +1383,182 @@ extern "C" int opp_get_dat_device_ptr(opp_ctx c, int32_t h, void **ptr, int64_t 
     Set &S = c->sets[col.set];
     *ptr = col.d;
     *stride = S.particle ? c->psets[S.pset].cap : col.dim;
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Field solve
+// ---------------------------------------------------------------------------
+extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const int32_t *dirichlet_mask,
+                              const double *dirichlet_value) {
+    TRY(ctx_check(c));
+    if (c->p.nranks > 1)
+        return fail(OPP_ERR_STATE, "field solve: one rank only (slab-partitioned CG not built)");
+    TRY(col_check(c, c2n));
+    const Col &cn = c->cols[c2n];
+    if (!cn.is_map || cn.dim != 4 || c->sets[cn.set].particle)
+        return fail(OPP_ERR_ARG, "c2n must be a dim-4 cell->node map");
+    const int nodes = cn.to;
+    TRY(check_col(c, node_pos, false, nodes, 3, OPP_REAL, "node_pos"));
+    if (!dirichlet_mask || !dirichlet_value) return fail(OPP_ERR_ARG, "null Dirichlet data");
+    const long long nc = c->sets[cn.set].size, nn = c->sets[nodes].size;
+    const int32_t *h = (const int32_t *)cn.host.data();
+    for (long long e = 0; e < 4 * nc; e++)
+        if (h[e] < 0 || h[e] >= nn) return fail(OPP_ERR_MESH, "c2n entry out of range");
+    // node -> cell CSR (cells in increasing order: the assembly's fixed order)
+    std::vector<int32_t> ptr(nn + 1, 0), n2c((size_t)4 * nc);
+    for (long long e = 0; e < 4 * nc; e++) ptr[h[e] + 1]++;
+    for (long long v = 0; v < nn; v++) ptr[v + 1] += ptr[v];
+    {
+        std::vector<int32_t> cur(ptr.begin(), ptr.end() - 1);
+        for (long long e = 0; e < 4 * nc; e++) n2c[cur[h[e]]++] = (int32_t)(e / 4);
+    }
+    // sparsity: row i = sorted unique nodes of i's cells; SELL-32 slices
+    const long long nsl = (nn + kSell - 1) / kSell;
+    std::vector<std::vector<int32_t>> rows(nn);
+    for (long long i = 0; i < nn; i++) {
+        auto &r = rows[i];
+        for (int e = ptr[i]; e < ptr[i + 1]; e++)
+            for (int k = 0; k < 4; k++) r.push_back(h[4ll * n2c[e] + k]);
+        if (r.empty()) r.push_back((int32_t)i);   // isolated node: identity row
+        std::sort(r.begin(), r.end());
+        r.erase(std::unique(r.begin(), r.end()), r.end());
+    }
+    std::vector<int64_t> soff(nsl + 1, 0);
+    for (long long s = 0; s < nsl; s++) {
+        size_t W = 0;
+        for (long long i = s * kSell; i < std::min<long long>(nn, (s + 1) * kSell); i++)
+            W = std::max(W, rows[i].size());
+        soff[s + 1] = soff[s] + (int64_t)W * kSell;
+    }
+    const long long nnz = soff[nsl];
+    std::vector<int32_t> col((size_t)nnz);
+    for (long long s = 0; s < nsl; s++) {
+        long long W = (soff[s + 1] - soff[s]) / kSell;
+        for (int l = 0; l < kSell; l++) {
+            long long i = s * kSell + l;
+            for (long long k = 0; k < W; k++) {
+                int32_t v = (i < nn && k < (long long)rows[i].size()) ? rows[i][k]
+                                                                      : (int32_t)std::min(i, nn - 1);
+                col[soff[s] + kSell * k + l] = v;
+            }
+        }
+    }
+    std::vector<int32_t> dm(dirichlet_mask, dirichlet_mask + nn);
+    std::vector<double> dv(nn);
+    for (long long i = 0; i < nn; i++) {
+        dm[i] = dm[i] != 0;
+        dv[i] = dm[i] ? dirichlet_value[i] : 0.0;
+    }
+    CK(cudaStreamSynchronize(c->s));
+    free_field(c);
+    FieldState &f = c->fs;
+    f.nn = nn;
+    f.nc = nc;
+    f.K.nn = nn;
+    f.K.nslices = nsl;
+    f.K.nnz_pad = nnz;
+    f.K.slice_off = (int64_t *)c->dalloc(8 * (nsl + 1));
+    f.K.col = (int32_t *)c->dalloc(4 * std::max<long long>(nnz, 1));
+    f.K.val = (double *)c->dalloc(8 * std::max<long long>(nnz, 1));
+    f.K.dinv = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
+    f.K.dmask = (int32_t *)c->dalloc(4 * std::max<long long>(nn, 1));
+    f.K.dval = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
+    f.n2c_ptr = (int32_t *)c->dalloc(4 * (nn + 1));
+    f.n2c = (int32_t *)c->dalloc(4 * std::max<long long>(4 * nc, 1));
+    f.vec = (double *)c->dalloc(8 * 5 * std::max<long long>(nn, 1));
+    f.part_cap = (long long)c->nsm * 8;
+    f.part = (double *)c->dalloc(8 * 3 * f.part_cap);
+    f.st = (CgState *)c->dalloc(sizeof(CgState));
+    if (!f.K.slice_off || !f.K.col || !f.K.val || !f.K.dinv || !f.K.dmask || !f.K.dval ||
+        !f.n2c_ptr || !f.n2c || !f.vec || !f.part || !f.st) {
+        free_field(c);
+        return fail(OPP_ERR_NOMEM, "field solve buffers");
+    }
+    CK(cudaMemcpyAsync(f.K.slice_off, soff.data(), 8 * (nsl + 1), cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemcpyAsync(f.K.col, col.data(), 4 * nnz, cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemcpyAsync(f.K.dmask, dm.data(), 4 * nn, cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemcpyAsync(f.K.dval, dv.data(), 8 * nn, cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemcpyAsync(f.n2c_ptr, ptr.data(), 4 * (nn + 1), cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemcpyAsync(f.n2c, n2c.data(), 4 * 4 * nc, cudaMemcpyHostToDevice, c->s));
+    CK(cudaMemsetAsync(f.st, 0, sizeof(CgState), c->s));
+    CK(launch_field_assemble((const double *)c->cols[node_pos].d, (const int32_t *)cn.d, f.n2c_ptr,
+                             f.n2c, f.K, c->s));
+    c->launches++;
+    CK(cudaStreamSynchronize(c->s));   // host vectors above go out of scope
+    f.c2n = c2n;
+    f.node_pos = node_pos;
+    f.ready = true;
+    return OPP_OK;
+}
+
+extern "C" int opp_get_field_stats(opp_ctx c, opp_field_stats *stats) {
+    TRY(ctx_check(c));
+    if (!stats) return fail(OPP_ERR_ARG, "null stats");
+    FieldState &f = c->fs;
+    if (!f.ready) return fail(OPP_ERR_STATE, "opp_field_init first");
+    CgState st{};
+    CK(cudaMemcpyAsync(&st, f.st, sizeof st, cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    stats->iterations = st.iterations;
+    stats->converged = st.converged;
+    stats->rel_residual = st.rr0 > 0 ? std::sqrt(st.rr / st.rr0) : 0.0;
+    stats->rhs_norm = std::sqrt(st.rr0);
+    return OPP_OK;
+}
+
+extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_potential, opp_dat cell_ef,
+                               const opp_field_params *prm, opp_field_stats *stats) {
+    TRY(ctx_check(c));
+    FieldState &f = c->fs;
+    if (!f.ready) return fail(OPP_ERR_STATE, "opp_field_init first");
+    if (!prm) return fail(OPP_ERR_ARG, "null field params");
+    if (!(prm->tol >= 0.0) || prm->max_iter < 0) return fail(OPP_ERR_ARG, "tol >= 0, max_iter >= 0");
+    const Col &cn = c->cols[f.c2n];
+    const int nodes = cn.to, cells = cn.set;
+    TRY(check_col(c, node_charge, false, nodes, 1, OPP_REAL, "node_charge"));
+    TRY(check_col(c, node_potential, false, nodes, 1, OPP_REAL, "node_potential"));
+    if (cell_ef >= 0) TRY(check_col(c, cell_ef, false, cells, 3, OPP_REAL, "cell_ef"));
+    CgArgs a{};
+    a.K = f.K;
+    a.Q = (const double *)c->cols[node_charge].d;
+    a.x = (double *)c->cols[node_potential].d;
+    const long long nn = f.nn;
+    a.r = f.vec;
+    a.u = f.vec + nn;
+    a.w = f.vec + 2 * nn;
+    a.p = f.vec + 3 * nn;
+    a.s = f.vec + 4 * nn;
+    a.part = f.part;
+    a.st = f.st;
+    a.rhs_scale = prm->rhs_scale;
+    a.tol = prm->tol;
+    a.max_iter = prm->max_iter;
+    a.warm = prm->warm_start != 0;
+    a.precond = prm->precond != 0;
+    if (const char *e = getenv("OPP_CG_DBG")) a.dbg = atoi(e);
+    {
+        PhaseScope ph(c, OPP_PH_FIELD);
+        int grid = 0;
+        if (nn > 0) {
+            int bps = 4;
+            if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
+            bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
+            CK(launch_cg(a, c->nsm, bps, c->s, &grid));
+            c->launches++;
+        }
+        if (cell_ef >= 0) {
+            Col &ef = c->cols[cell_ef];
+            MeshCache &m = c->mc;
+            const bool packed = m.efp && m.ef == cell_ef && m.nc == f.nc;
+            CK(launch_efield((const double *)c->cols[f.node_pos].d, (const int32_t *)cn.d, a.x, f.nc,
+                             (double *)ef.d, packed ? m.efp : nullptr, c->s));
+            c->launches++;
+            ef.version++;
+            if (packed) m.vef = ef.version;
+        }
+    }
+    c->cols[node_potential].version++;
+    if (stats) return opp_get_field_stats(c, stats);
     return OPP_OK;
 }

@@ -1,0 +1,363 @@
+// opp_field.cu -- sm_100a kernels of the electrostatic field solve (internal).
+//
+// The field solve is step 1 of the PIC loop (Fig. 1; Gauss'
+// law, Eq. 1) solved by the finite-element method on the tetrahedral mesh
+// (PAPER.md:469-479).  Mini-FEM-PIC's routines ComputeJMatrix /
+// ComputeF1Vector / linear solve / ComputeElectricField (PAPER.md:1604-1612,
+// Fig. 6) become, in the linear case north_star names
+// ("a plain GPU conjugate-gradient on the FEM Poisson system"):
+//   k_field_assemble   K_ij = sum_e V_e grad(l_i).grad(l_j), Dirichlet rows
+//                      -> identity; one thread per row walks the node's cells
+//                      in a fixed order (deterministic, no atomics)
+//   k_cg               one persistent cooperative launch runs the whole
+//                      (Jacobi-)preconditioned CG in the Chronopoulos-Gear
+//                      form: one fused SpMV + 3-dot pass and one vector-update
+//                      pass per iteration, two grid barriers, every block
+//                      reduces the block partials in the same order (same
+//                      alpha/beta everywhere, run-to-run deterministic)
+//   k_efield           E_c = -sum_i phi[c2n[c][i]] grad(l_i), written to the
+//                      cell dat and straight into the padded field the
+//                      particle kernels gather (no separate pack)
+// At C2 (175,273 nodes) K is ~2.6M padded entries = 31 MB: the matrix and the
+// six work vectors (8.4 MB) stay in the 126 MB L2 across iterations, so an
+// iteration is bound by L2 latency and the two grid barriers, not HBM.
+#include <cooperative_groups.h>
+
+#include "opp_field.h"
+
+namespace cg = cooperative_groups;
+
+namespace opp {
+
+namespace {
+
+constexpr int kCgThreads = 256;
+constexpr int kCgWarps = kCgThreads / 32;
+
+// Gradients of the 4 barycentric coordinates and the volume of a tet
+// (Cramer's rule on M = [p1-p0, p2-p0, p3-p0]).
+__device__ __forceinline__ void tet_grads(const double *__restrict__ xyz, int4 n, double g[4][3],
+                                          double *vol) {
+    double p0[3], a[3], b[3], c[3];
+    for (int k = 0; k < 3; k++) {
+        p0[k] = xyz[3ll * n.x + k];
+        a[k] = xyz[3ll * n.y + k] - p0[k];
+        b[k] = xyz[3ll * n.z + k] - p0[k];
+        c[k] = xyz[3ll * n.w + k] - p0[k];
+    }
+    double bxc[3] = {b[1] * c[2] - b[2] * c[1], b[2] * c[0] - b[0] * c[2], b[0] * c[1] - b[1] * c[0]};
+    double cxa[3] = {c[1] * a[2] - c[2] * a[1], c[2] * a[0] - c[0] * a[2], c[0] * a[1] - c[1] * a[0]};
+    double axb[3] = {a[1] * b[2] - a[2] * b[1], a[2] * b[0] - a[0] * b[2], a[0] * b[1] - a[1] * b[0]};
+    double det = a[0] * bxc[0] + a[1] * bxc[1] + a[2] * bxc[2];
+    double id = 1.0 / det;
+    for (int k = 0; k < 3; k++) {
+        g[1][k] = bxc[k] * id;
+        g[2][k] = cxa[k] * id;
+        g[3][k] = axb[k] * id;
+        g[0][k] = -(g[1][k] + g[2][k] + g[3][k]);
+    }
+    *vol = det / 6.0;
+}
+
+__global__ void k_field_assemble(const double *__restrict__ xyz, const int32_t *__restrict__ c2n,
+                                 const int32_t *__restrict__ n2c_ptr,
+                                 const int32_t *__restrict__ n2c, FieldMat K) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    long long sl = i / kSell;
+    int lane = (int)(i % kSell);
+    long long off = K.slice_off[sl];
+    int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+    for (int k = 0; k < W; k++) K.val[off + (long long)kSell * k + lane] = 0.0;
+    if (K.dmask[i]) {
+        for (int k = 0; k < W; k++)
+            if (K.col[off + (long long)kSell * k + lane] == (int32_t)i) {
+                K.val[off + (long long)kSell * k + lane] = 1.0;
+                break;
+            }
+        K.dinv[i] = 1.0;
+        return;
+    }
+    double diag = 0.0;
+    for (int e = n2c_ptr[i]; e < n2c_ptr[i + 1]; e++) {
+        int cell = n2c[e];
+        int4 n = reinterpret_cast<const int4 *>(c2n)[cell];
+        int nl[4] = {n.x, n.y, n.z, n.w};
+        double g[4][3], V;
+        tet_grads(xyz, n, g, &V);
+        int li = 0;
+        while (nl[li] != (int)i) li++;
+        for (int lj = 0; lj < 4; lj++) {
+            double kij = V * (g[li][0] * g[lj][0] + g[li][1] * g[lj][1] + g[li][2] * g[lj][2]);
+            for (int k = 0; k < W; k++) {
+                long long q = off + (long long)kSell * k + lane;
+                if (K.col[q] == nl[lj]) {
+                    K.val[q] += kij;
+                    break;
+                }
+            }
+            if (lj == li) diag += kij;
+        }
+    }
+    K.dinv[i] = 1.0 / diag;
+}
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Block-reduce NV partial sums and publish them as part[k * gridDim.x + block].
+template <int NV>
+__device__ __forceinline__ void block_publish(double (&v)[NV], double *part, double *sm) {
+    int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < NV; k++) v[k] = warp_sum(v[k]);
+    if (lane == 0)
+#pragma unroll
+        for (int k = 0; k < NV; k++) sm[k * kCgWarps + wid] = v[k];
+    __syncthreads();
+    if (threadIdx.x < NV) {
+        double t = 0.0;
+        for (int w = 0; w < kCgWarps; w++) t += sm[threadIdx.x * kCgWarps + w];
+        part[threadIdx.x * gridDim.x + blockIdx.x] = t;
+    }
+    __syncthreads();
+}
+
+// After a grid barrier: every block sums the published partials in the same
+// order, so all blocks hold bit-identical totals.
+template <int NV>
+__device__ __forceinline__ void block_total(const double *part, double *sm, double (&out)[NV]) {
+    int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    double v[NV];
+#pragma unroll
+    for (int k = 0; k < NV; k++) {
+        v[k] = 0.0;
+        for (int b = threadIdx.x; b < (int)gridDim.x; b += kCgThreads)
+            v[k] += __ldcg(part + k * gridDim.x + b);
+        v[k] = warp_sum(v[k]);
+    }
+    if (lane == 0)
+#pragma unroll
+        for (int k = 0; k < NV; k++) sm[k * kCgWarps + wid] = v[k];
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < NV; k++) {
+        double t = 0.0;
+        for (int w = 0; w < kCgWarps; w++) t += sm[k * kCgWarps + w];
+        out[k] = t;
+    }
+    __syncthreads();
+}
+
+// y_row = sum_k val * v[col]  (lane = row of the slice).  Entries go in
+// chunks of kChunk: all column indices and values of a chunk are loaded,
+// then all gathers of v are issued, then the products are summed -- two
+// dependent L2 round trips per chunk instead of two per entry (a P1 Kuhn
+// row has <= 15 entries: one chunk).
+constexpr int kChunk = 16;
+__device__ __forceinline__ double sell_row(const FieldMat &K, long long sl, int lane,
+                                           const double *v) {
+    long long off = __ldg(K.slice_off + sl);
+    int W = (int)((__ldg(K.slice_off + sl + 1) - off) / kSell);
+    const int32_t *cp = K.col + off + lane;
+    const double *vp = K.val + off + lane;
+    double acc = 0.0;
+    for (int k0 = 0; k0 < W; k0 += kChunk) {
+        int c[kChunk];
+        double m[kChunk], xv[kChunk];
+#pragma unroll
+        for (int j = 0; j < kChunk; j++) {
+            const bool in = k0 + j < W;
+            c[j] = in ? __ldg(cp + kSell * (k0 + j)) : 0;
+            m[j] = in ? __ldg(vp + kSell * (k0 + j)) : 0.0;
+        }
+#pragma unroll
+        for (int j = 0; j < kChunk; j++) xv[j] = k0 + j < W ? __ldcg(v + c[j]) : 0.0;
+#pragma unroll
+        for (int j = 0; j < kChunk; j++) acc += m[j] * xv[j];
+    }
+    return acc;
+}
+
+__global__ void __launch_bounds__(kCgThreads) k_cg(CgArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ double sm[4 * kCgWarps];
+    const FieldMat &K = a.K;
+    const long long nn = K.nn;
+    const int lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long TW = ((long long)gridDim.x * blockDim.x) >> 5;
+
+    // ---- x0: Dirichlet values on D, warm start or 0 on F
+    for (long long sl = gw; sl < K.nslices; sl += TW) {
+        long long i = sl * kSell + lane;
+        if (i >= nn) continue;
+        double xi = K.dmask[i] ? K.dval[i] : (a.warm ? a.x[i] : 0.0);
+        a.x[i] = xi;
+    }
+    grid.sync();
+    // ---- r0 = b - K x0 (free rows), lifted rhs b_F - K_FD phi_D, u0 = M^-1 r0
+    {
+        double v[1] = {0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double ri = 0.0, bi = 0.0;
+            if (!K.dmask[i]) {
+                long long off = K.slice_off[sl];
+                int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+                double ax = 0.0, ad = 0.0;
+                for (int k = 0; k < W; k++) {
+                    long long q = off + (long long)kSell * k + lane;
+                    int c = K.col[q];
+                    double t = K.val[q] * __ldcg(a.x + c);
+                    ax += t;
+                    if (K.dmask[c]) ad += t;
+                }
+                double b = a.rhs_scale * a.Q[i];
+                ri = b - ax;
+                bi = b - ad;
+            }
+            a.r[i] = ri;
+            a.u[i] = a.precond ? ri * K.dinv[i] : ri;
+            a.p[i] = 0.0;
+            a.s[i] = 0.0;
+            v[0] += bi * bi;
+        }
+        block_publish<1>(v, a.part, sm);
+    }
+    grid.sync();
+    double rr0;
+    {
+        double t[1];
+        block_total<1>(a.part, sm, t);
+        rr0 = t[0];
+    }
+    grid.sync();   // partials are reused below
+    // ---- w0 = K u0 and the first dots
+    {
+        double v[3] = {0.0, 0.0, 0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double wi = sell_row(K, sl, lane, a.u);
+            double ri = a.r[i], ui = a.u[i];
+            a.w[i] = wi;
+            v[0] += ri * ui;
+            v[1] += wi * ui;
+            v[2] += ri * ri;
+        }
+        block_publish<3>(v, a.part, sm);
+    }
+    grid.sync();
+    double gamma_old = 0.0, alpha = 0.0, beta = 0.0;
+    const double stop = a.tol * a.tol * rr0;
+    int it = 0;
+    double rho = 0.0;
+    for (;;) {
+        double t[3];
+        block_total<3>(a.part, sm, t);
+        double gamma = t[0], delta = t[1];
+        rho = t[2];
+        if (rho <= stop || it >= a.max_iter) break;
+        if (it == 0) {
+            beta = 0.0;
+            alpha = gamma / delta;
+        } else {
+            beta = gamma / gamma_old;
+            alpha = gamma / (delta - beta * gamma / alpha);
+        }
+        gamma_old = gamma;
+        // phase A (row-local): p = u + beta p; s = w + beta s; x += alpha p;
+        // r -= alpha s; u = M^-1 r
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double pi = a.u[i] + beta * a.p[i];
+            double si = a.w[i] + beta * a.s[i];
+            a.p[i] = pi;
+            a.s[i] = si;
+            a.x[i] += alpha * pi;
+            double ri = a.r[i] - alpha * si;
+            a.r[i] = ri;
+            a.u[i] = a.precond ? ri * K.dinv[i] : ri;
+        }
+        if (a.dbg != 2) grid.sync();
+        // phase B: w = K u, dots (r,u), (w,u), (r,r)
+        double v[3] = {0.0, 0.0, 0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double wi = a.dbg == 1 ? a.u[i] : sell_row(K, sl, lane, a.u);
+            double ri = a.r[i], ui = a.u[i];
+            a.w[i] = wi;
+            v[0] += ri * ui;
+            v[1] += wi * ui;
+            v[2] += ri * ri;
+        }
+        block_publish<3>(v, a.part, sm);
+        if (a.dbg != 2) grid.sync();
+        it++;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.st->iterations = it;
+        a.st->converged = rho <= stop;
+        a.st->rr0 = rr0;
+        a.st->rr = rho;
+    }
+}
+
+__global__ void k_efield(const double *__restrict__ xyz, const int32_t *__restrict__ c2n,
+                         const double *__restrict__ phi, long long nc, double *__restrict__ ef,
+                         double4 *__restrict__ efp) {
+    long long c = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    int4 n = reinterpret_cast<const int4 *>(c2n)[c];
+    double g[4][3], V;
+    tet_grads(xyz, n, g, &V);
+    double f[4] = {phi[n.x], phi[n.y], phi[n.z], phi[n.w]};
+    double E[3];
+    for (int k = 0; k < 3; k++)
+        E[k] = -(f[0] * g[0][k] + f[1] * g[1][k] + f[2] * g[2][k] + f[3] * g[3][k]);
+    ef[3 * c + 0] = E[0];
+    ef[3 * c + 1] = E[1];
+    ef[3 * c + 2] = E[2];
+    if (efp) efp[c] = make_double4(E[0], E[1], E[2], 0.0);
+}
+
+}  // namespace
+
+cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const int32_t *n2c_ptr,
+                                  const int32_t *n2c, const FieldMat &K, cudaStream_t s) {
+    if (K.nn == 0) return cudaSuccess;
+    k_field_assemble<<<(unsigned)((K.nn + 255) / 256), 256, 0, s>>>(xyz, c2n, n2c_ptr, n2c, K);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out) {
+    int occ = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_cg, kCgThreads, 0);
+    if (e != cudaSuccess) return e;
+    int bps = occ < max_bps ? occ : max_bps;
+    if (bps < 1) return cudaErrorCooperativeLaunchTooLarge;
+    long long want = (a.K.nslices + kCgWarps - 1) / kCgWarps;   // one slice per warp at most
+    int grid = nsm * bps;
+    if (want < grid) grid = (int)(want > 0 ? want : 1);
+    CgArgs args = a;
+    void *params[] = {&args};
+    e = cudaLaunchCooperativeKernel((const void *)k_cg, dim3(grid), dim3(kCgThreads), params, 0, s);
+    if (grid_out) *grid_out = grid;
+    return e;
+}
+
+cudaError_t launch_efield(const double *xyz, const int32_t *c2n, const double *phi, long long nc,
+                          double *ef, double4 *efp, cudaStream_t s) {
+    if (nc == 0) return cudaSuccess;
+    k_efield<<<(unsigned)((nc + 255) / 256), 256, 0, s>>>(xyz, c2n, phi, nc, ef, efp);
+    return cudaGetLastError();
+}
+
+}  // namespace opp

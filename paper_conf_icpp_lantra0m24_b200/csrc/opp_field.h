@@ -1,0 +1,61 @@
+// opp_field.h -- the electrostatic field solve of libopp (internal): P1 FEM
+// Poisson matrix in sliced-ELLPACK form, a persistent cooperative CG kernel and
+// the cell-field kernel (Fig. 1
+// step 1, 469-479, 1044-1068, 1604-1612).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace opp {
+
+constexpr int kSell = 32;   // rows per slice (one warp, lane = row)
+
+// K stored as SELL-32: slice s holds rows [32 s, 32 s + 32); its width
+// W_s = max nnz of those rows; entry k of row 32 s + l is at
+// slice_off[s] + 32 k + l (column-major inside the slice: a warp's 32 lanes
+// read 32 consecutive values).  Padding: col = the row itself, val = 0.
+// Dirichlet rows are identity rows; free rows keep their Dirichlet columns
+// (needed once, for the lifted initial residual).
+struct FieldMat {
+    long long nn = 0, nslices = 0, nnz_pad = 0;
+    int64_t *slice_off = nullptr;   // [nslices + 1]
+    int32_t *col = nullptr;         // [nnz_pad]
+    double *val = nullptr;          // [nnz_pad]
+    double *dinv = nullptr;         // [nn] Jacobi: 1 / K_ii (1 on Dirichlet rows)
+    int32_t *dmask = nullptr;       // [nn] 1 = Dirichlet node
+    double *dval = nullptr;         // [nn] Dirichlet values (0 on free nodes)
+};
+
+// Device-side solver state (read back by opp_get_field_stats).
+struct CgState {
+    int iterations;
+    int converged;
+    double rr0;          // ||b_F - K_FD phi_D||^2 (the stopping reference)
+    double rr;           // ||r||^2 at exit (recursive residual)
+    double pad[5];
+};
+
+struct CgArgs {
+    FieldMat K;
+    const double *Q;     // node charge
+    double *x;           // node potential (in: warm start, out: solution)
+    double *r, *u, *w, *p, *s;   // work vectors [nn]
+    double *part;        // [3 * grid] block partial sums
+    CgState *st;
+    double rhs_scale, tol;
+    int max_iter, warm, precond;
+    int dbg;             // diagnostics (OPP_CG_DBG): 1 = no SpMV in the loop, 2 = no grid barriers
+};
+
+// Per-row assembly from the node->cell CSR (deterministic order, no atomics).
+cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const int32_t *n2c_ptr,
+                                  const int32_t *n2c, const FieldMat &K, cudaStream_t s);
+// One cooperative launch runs the whole CG solve (grid = nsm x min(occupancy,
+// max_bps) blocks, fewer if the matrix has fewer slices); returns the grid used.
+cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out);
+// E_c = -sum_i phi[c2n[c][i]] grad(lambda_i) -> ef (AoS [nc][3]) and, if
+// non-NULL, the padded copy the particle kernels read.
+cudaError_t launch_efield(const double *xyz, const int32_t *c2n, const double *phi, long long nc,
+                          double *ef, double4 *efp, cudaStream_t s);
+
+}  // namespace opp

@@ -29,9 +29,10 @@ EXPORTS = (
     "opp_get_node_charge", "opp_get_dat", "opp_set_dat", "opp_get_particle_count",
     "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
+    "opp_field_init", "opp_field_solve", "opp_get_field_stats",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
-          "sort_count", "sort_move")
+          "sort_count", "sort_move", "field")
 # note: "fill" includes the periodic sort-by-cell when opp_init_params.sort_every > 0
 
 
@@ -69,6 +70,19 @@ class opp_step_stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class opp_field_params(C.Structure):
+    _fields_ = [("rhs_scale", C.c_double), ("tol", C.c_double), ("max_iter", C.c_int),
+                ("warm_start", C.c_int), ("precond", C.c_int)]
+
+
+class opp_field_stats(C.Structure):
+    _fields_ = [("iterations", C.c_int32), ("converged", C.c_int32),
+                ("rel_residual", C.c_double), ("rhs_norm", C.c_double)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
@@ -101,6 +115,10 @@ def _load():
         "opp_phase_timing": (I, [P, I]),
         "opp_get_phase_times": (I, [P, P, P]),
         "opp_last_error": (C.c_char_p, []),
+        "opp_field_init": (I, [P, I32, I32, P, P]),
+        "opp_field_solve": (I, [P, I32, I32, I32, C.POINTER(opp_field_params),
+                                C.POINTER(opp_field_stats)]),
+        "opp_get_field_stats": (I, [P, C.POINTER(opp_field_stats)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -264,3 +282,24 @@ def opp_get_phase_times(ctx) -> dict:
     cnt = (C.c_int64 * len(PHASES))()
     _ck(lib.opp_get_phase_times(ctx, ms, cnt))
     return {PHASES[k]: (ms[k], cnt[k]) for k in range(len(PHASES))}
+
+
+def opp_field_init(ctx, c2n: int, node_pos: int, dirichlet_mask, dirichlet_value) -> None:
+    import numpy as np
+    m = np.ascontiguousarray(dirichlet_mask, dtype=np.int32)
+    v = np.ascontiguousarray(dirichlet_value, dtype=np.float64)
+    _ck(lib.opp_field_init(ctx, c2n, node_pos, _ptr(m), _ptr(v)))
+
+
+def opp_field_solve(ctx, node_charge: int, node_potential: int, cell_ef: int,
+                    params: opp_field_params, want_stats: bool = True):
+    st = opp_field_stats() if want_stats else None
+    _ck(lib.opp_field_solve(ctx, node_charge, node_potential, cell_ef, C.byref(params),
+                            C.byref(st) if st else None))
+    return st
+
+
+def opp_get_field_stats(ctx) -> opp_field_stats:
+    st = opp_field_stats()
+    _ck(lib.opp_get_field_stats(ctx, C.byref(st)))
+    return st
