@@ -65,8 +65,8 @@ def parse():
     ap.add_argument("--cg-tol", type=float, default=1e-10)
     args = ap.parse_args()
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
-    if args.field < 0:   # the CG is single-GPU: multi-GPU runs keep the fixed field
-        args.field = 1 if (args.config == "c2" and int(os.environ.get("WORLD_SIZE", "1")) == 1) else 0
+    if args.field < 0:
+        args.field = 1 if args.config == "c2" else 0
     return args
 
 
@@ -240,8 +240,6 @@ def run_ours(args, rank, world):
             cluster = (cluster[0], cluster[1][(cluster[1] >= base) & (cluster[1] < base + mesh["n_cells"])] - base)
     else:
         gen_mesh = mesh
-    if args.field and world > 1:
-        raise SystemExit("--field 1 is single-GPU only (the CG is not slab-partitioned)")
     if args.field:
         ef = np.zeros_like(ef)
     dm = gc.DeviceMesh(gen_mesh)
@@ -364,7 +362,9 @@ def run_ours(args, rank, world):
         line["field"] = {"ms_per_step": field_ms / args.steps, "cg_iterations_last": fst["iterations"],
                          "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
                          "rhs_scale": args.rhs, "wall_potential": args.wall,
-                         "solver": "Jacobi-PCG, one persistent cooperative kernel, warm start",
+                         "solver": ("Jacobi-PCG, one persistent cooperative kernel, warm start"
+                                    if world == 1 else "Jacobi-PCG over slabs (node halo + "
+                                    "cross-rank dots, host-driven), warm start"),
                          "note": "value excludes the field solve (timed separately, SURVEY.md "
                                  "§8(d)); value_incl_field counts it"}
         line["value_incl_field"] = pushed / (ms / 1e3)

@@ -286,7 +286,10 @@ int64_t opp_kernel_launch_count(opp_ctx ctx);
  *                                   point charges, Eq. 10; F2)
  *   phi = dirichlet_value on Dirichlet nodes; homogeneous Neumann elsewhere
  *   E_c = -sum_i phi[c2n[c][i]] grad(lambda_i)   (cell-constant, 1576-1585)
- * One rank only (nranks > 1: OPP_ERR_STATE).
+ * nranks > 1: every rank assembles its slab's cells; interface rows are
+ * completed by the node halo exchange of the charge halo (opp_set_partition)
+ * and dot products count each node once, reduced across ranks in rank order
+ * (a host-driven iteration; one rank runs one persistent kernel).
  * ------------------------------------------------------------------------- */
 typedef struct {
     double rhs_scale;   /* b = rhs_scale * node_charge (q / eps0 per unit weight)       */
@@ -309,8 +312,10 @@ typedef struct {
  * order: deterministic) and the Dirichlet data.  dirichlet_mask[n] != 0 marks
  * node n Dirichlet with value dirichlet_value[n] (host arrays of the node
  * count; copied).  Maps are static: call again to rebuild.
- * Errors: OPP_ERR_ARG (handles, NULL), OPP_ERR_MESH (c2n out of range),
- * OPP_ERR_NOMEM, OPP_ERR_STATE (nranks > 1).  Synchronises. */
+ * nranks > 1: collective, after opp_set_partition (node data are this rank's
+ * nodes).  Errors: OPP_ERR_ARG (handles, NULL), OPP_ERR_MESH (c2n out of
+ * range), OPP_ERR_NOMEM, OPP_ERR_STATE (nranks > 1 before the partition).
+ * Synchronises. */
 int opp_field_init(opp_ctx ctx, opp_map c2n, opp_dat node_pos, const int32_t *dirichlet_mask,
                    const double *dirichlet_value);
 
@@ -318,9 +323,10 @@ int opp_field_init(opp_ctx ctx, opp_map c2n, opp_dat node_pos, const int32_t *di
  * params->warm_start, out: phi) from node_charge (node dat dim 1 OPP_REAL,
  * e.g. after opp_push_move_deposit), then write cell_ef (cell dat dim 3
  * OPP_REAL; -1 = skip) = -grad(phi) per cell, which the next
- * opp_push_move_deposit gathers.  One persistent cooperative kernel runs the
- * whole CG; enqueued on the stream; stats may be NULL (no synchronisation;
- * read them later with opp_get_field_stats). */
+ * opp_push_move_deposit gathers.  One rank: one persistent cooperative kernel
+ * runs the whole CG, enqueued on the stream; stats may be NULL (no
+ * synchronisation; read them later with opp_get_field_stats).  nranks > 1:
+ * collective, synchronises once per iteration. */
 int opp_field_solve(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential, opp_dat cell_ef,
                     const opp_field_params *params, opp_field_stats *stats);
 

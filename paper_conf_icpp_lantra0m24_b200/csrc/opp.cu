@@ -127,6 +127,12 @@ struct FieldState {
     double *part = nullptr;         // 3 * part_cap block partials
     long long part_cap = 0;
     CgState *st = nullptr;
+    // host-driven CG (nranks > 1 or OPP_CG_HOSTLOOP): owner weights of the
+    // dot products (1 on the lowest rank holding a node), y / yd / beff
+    // vectors, the reduced dots, and the host-kept stats of the last solve
+    double *own = nullptr, *hvec = nullptr, *dots = nullptr;
+    bool host_stats = false;
+    opp_field_stats hst{};
 };
 
 }  // namespace
@@ -320,6 +326,7 @@ static void free_field(opp_ctx c) {
     c->dfree(f.K.dinv, 0); c->dfree(f.K.dmask, 0); c->dfree(f.K.dval, 0);
     c->dfree(f.n2c_ptr, 0); c->dfree(f.n2c, 0); c->dfree(f.vec, 0); c->dfree(f.part, 0);
     c->dfree(f.st, 0);
+    c->dfree(f.own, 0); c->dfree(f.hvec, 0); c->dfree(f.dots, 0);
     f = FieldState();
 }
 
@@ -1392,8 +1399,9 @@ extern "C" int opp_get_dat_device_ptr(opp_ctx c, int32_t h, void **ptr, int64_t 
 extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const int32_t *dirichlet_mask,
                               const double *dirichlet_value) {
     TRY(ctx_check(c));
-    if (c->p.nranks > 1)
-        return fail(OPP_ERR_STATE, "field solve: one rank only (slab-partitioned CG not built)");
+    const bool multi = c->p.nranks > 1;
+    if (multi && !c->comm->partitioned)
+        return fail(OPP_ERR_STATE, "nranks > 1: call opp_set_partition before opp_field_init");
     TRY(col_check(c, c2n));
     const Col &cn = c->cols[c2n];
     if (!cn.is_map || cn.dim != 4 || c->sets[cn.set].particle)
@@ -1470,8 +1478,11 @@ extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const in
     f.part_cap = (long long)c->nsm * 8;
     f.part = (double *)c->dalloc(8 * 3 * f.part_cap);
     f.st = (CgState *)c->dalloc(sizeof(CgState));
+    f.own = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
+    f.hvec = (double *)c->dalloc(8 * 3 * std::max<long long>(nn, 1));
+    f.dots = (double *)c->dalloc(8 * 4);
     if (!f.K.slice_off || !f.K.col || !f.K.val || !f.K.dinv || !f.K.dmask || !f.K.dval ||
-        !f.n2c_ptr || !f.n2c || !f.vec || !f.part || !f.st) {
+        !f.n2c_ptr || !f.n2c || !f.vec || !f.part || !f.st || !f.own || !f.hvec || !f.dots) {
         free_field(c);
         return fail(OPP_ERR_NOMEM, "field solve buffers");
     }
@@ -1485,6 +1496,24 @@ extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const in
     CK(launch_field_assemble((const double *)c->cols[node_pos].d, (const int32_t *)cn.d, f.n2c_ptr,
                              f.n2c, f.K, c->s));
     c->launches++;
+    // dot-product owner weights: a node shared with a lower rank is counted there
+    std::vector<double> own(nn, 1.0);
+    if (multi && c->comm->halo_n > 0) {
+        opp::Comm *cm = c->comm;
+        std::vector<int32_t> hidx(cm->halo_n);
+        CK(cudaMemcpyAsync(hidx.data(), cm->d_halo_idx, 4 * cm->halo_n, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        for (int p = 0; p < c->p.rank; p++)
+            for (int64_t k = 0; k < cm->halo_cnt[p]; k++) own[hidx[cm->halo_off[p] + k]] = 0.0;
+    }
+    CK(cudaMemcpyAsync(f.own, own.data(), 8 * nn, cudaMemcpyHostToDevice, c->s));
+    if (multi && c->comm->halo_n > 0) {
+        // Jacobi: the diagonal of the assembled (summed over ranks) matrix
+        CK(launch_diag(f.K, f.hvec, c->s));
+        TRY(halo_sum(c, f.hvec));
+        CK(launch_dinv(f.K, f.hvec, c->s));
+        c->launches += 2;
+    }
     CK(cudaStreamSynchronize(c->s));   // host vectors above go out of scope
     f.c2n = c2n;
     f.node_pos = node_pos;
@@ -1497,6 +1526,11 @@ extern "C" int opp_get_field_stats(opp_ctx c, opp_field_stats *stats) {
     if (!stats) return fail(OPP_ERR_ARG, "null stats");
     FieldState &f = c->fs;
     if (!f.ready) return fail(OPP_ERR_STATE, "opp_field_init first");
+    if (f.host_stats) {
+        CK(cudaStreamSynchronize(c->s));
+        *stats = f.hst;
+        return OPP_OK;
+    }
     CgState st{};
     CK(cudaMemcpyAsync(&st, f.st, sizeof st, cudaMemcpyDeviceToHost, c->s));
     CK(cudaStreamSynchronize(c->s));
@@ -1504,6 +1538,93 @@ extern "C" int opp_get_field_stats(opp_ctx c, opp_field_stats *stats) {
     stats->converged = st.converged;
     stats->rel_residual = st.rr0 > 0 ? std::sqrt(st.rr / st.rr0) : 0.0;
     stats->rhs_norm = std::sqrt(st.rr0);
+    return OPP_OK;
+}
+
+// Sum of n doubles (device) over all ranks, in rank order (identical on every
+// rank): the reduction of the host-driven CG's dot products.
+static int allreduce_dots(opp_ctx c, const double *dev, int n, double *out) {
+    double mine[4];
+    CK(cudaMemcpyAsync(mine, dev, 8 * n, cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    if (c->p.nranks == 1) {
+        for (int k = 0; k < n; k++) out[k] = mine[k];
+        return OPP_OK;
+    }
+    const int R = c->p.nranks;
+    std::vector<int64_t> all((size_t)n * R);
+    int64_t bits[4];
+    std::memcpy(bits, mine, 8 * n);
+    TRY(c->comm->t->allgather_i64(bits, n, all.data(), c->s, g_err));
+    for (int k = 0; k < n; k++) {
+        double t = 0.0;
+        for (int r = 0; r < R; r++) {
+            double v;
+            std::memcpy(&v, &all[(size_t)r * n + k], 8);
+            t += v;
+        }
+        out[k] = t;
+    }
+    return OPP_OK;
+}
+
+// The same Chronopoulos-Gear (P)CG as k_cg, one kernel per phase: local SpMV
+// rows of interface nodes are completed by the node halo exchange (the
+// charge halo's plan), dots count each node once (owner weights) and are
+// reduced across ranks in rank order; alpha, beta on the host.
+static int field_solve_hostloop(opp_ctx c, CgArgs &a) {
+    FieldState &f = c->fs;
+    const FieldMat &K = f.K;
+    const long long nn = f.nn;
+    const bool multi = c->p.nranks > 1 && c->comm->halo_n > 0;
+    double *y = f.hvec, *yd = f.hvec + nn, *beff = f.hvec + 2 * nn;
+    const int nblk = (int)std::min<long long>(f.part_cap, std::max<long long>(1, (nn + 255) / 256));
+    CK(launch_cg_x0(K, a.x, a.warm, c->s));
+    CK(launch_spmv(K, a.x, y, yd, c->nsm, c->s));
+    c->launches += 2;
+    if (multi) {
+        TRY(halo_sum(c, y));
+        TRY(halo_sum(c, yd));
+    }
+    CK(launch_cg_r0(K, a.Q, a.rhs_scale, y, yd, a.r, a.u, a.p, a.s, beff, a.precond, c->s));
+    const double *va[3], *vb[3];
+    va[0] = beff; vb[0] = beff;
+    CK(launch_dots(nn, f.own, 1, va, vb, f.part, nblk, f.dots, c->s));
+    c->launches += 3;
+    double rr0;
+    TRY(allreduce_dots(c, f.dots, 1, &rr0));
+    const double stop = a.tol * a.tol * rr0;
+    va[0] = a.r; vb[0] = a.u;
+    va[1] = a.w; vb[1] = a.u;
+    va[2] = a.r; vb[2] = a.r;
+    double gamma_old = 0.0, alpha = 0.0, beta = 0.0, rho = 0.0;
+    int it = 0;
+    for (bool first = true;; first = false) {
+        if (!first) CK(launch_cg_update(K, alpha, beta, a.x, a.r, a.u, a.w, a.p, a.s, a.precond, c->s));
+        CK(launch_spmv(K, a.u, a.w, nullptr, c->nsm, c->s));
+        if (multi) TRY(halo_sum(c, a.w));
+        CK(launch_dots(nn, f.own, 3, va, vb, f.part, nblk, f.dots, c->s));
+        c->launches += first ? 3 : 4;
+        if (!first) it++;
+        double t[3];
+        TRY(allreduce_dots(c, f.dots, 3, t));
+        const double gamma = t[0], delta = t[1];
+        rho = t[2];
+        if (rho <= stop || it >= a.max_iter) break;
+        if (it == 0) {
+            beta = 0.0;
+            alpha = gamma / delta;
+        } else {
+            beta = gamma / gamma_old;
+            alpha = gamma / (delta - beta * gamma / alpha);
+        }
+        gamma_old = gamma;
+    }
+    f.host_stats = true;
+    f.hst.iterations = it;
+    f.hst.converged = rho <= stop;
+    f.hst.rel_residual = rr0 > 0 ? std::sqrt(rho / rr0) : 0.0;
+    f.hst.rhs_norm = std::sqrt(rr0);
     return OPP_OK;
 }
 
@@ -1540,8 +1661,12 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     {
         PhaseScope ph(c, OPP_PH_FIELD);
         int grid = 0;
-        if (nn > 0) {
-            int bps = 4;
+        const char *hl = getenv("OPP_CG_HOSTLOOP");
+        f.host_stats = false;
+        if (nn > 0 && (c->p.nranks > 1 || (hl && atoi(hl)))) {
+            TRY(field_solve_hostloop(c, a));
+        } else if (nn > 0) {
+            int bps = 2;
             if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
             bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
             CK(launch_cg(a, c->nsm, bps, c->s, &grid));

@@ -127,18 +127,22 @@ __device__ __forceinline__ void block_publish(double (&v)[NV], double *part, dou
 }
 
 // After a grid barrier: every block sums the published partials in the same
-// order, so all blocks hold bit-identical totals.
+// order, so all blocks hold bit-identical totals.  The grid has at most
+// 2 * kCgThreads blocks (launch_cg), so every thread issues its (at most 2 *
+// NV) loads at once: one L2 round trip, not one per partial.
 template <int NV>
 __device__ __forceinline__ void block_total(const double *part, double *sm, double (&out)[NV]) {
     int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    double v[NV];
+    const int G = (int)gridDim.x;
+    const int b0 = threadIdx.x, b1 = threadIdx.x + kCgThreads;
+    double t0[NV], t1[NV], v[NV];
 #pragma unroll
     for (int k = 0; k < NV; k++) {
-        v[k] = 0.0;
-        for (int b = threadIdx.x; b < (int)gridDim.x; b += kCgThreads)
-            v[k] += __ldcg(part + k * gridDim.x + b);
-        v[k] = warp_sum(v[k]);
+        t0[k] = b0 < G ? __ldcg(part + k * G + b0) : 0.0;
+        t1[k] = b1 < G ? __ldcg(part + k * G + b1) : 0.0;
     }
+#pragma unroll
+    for (int k = 0; k < NV; k++) v[k] = warp_sum(t0[k] + t1[k]);
     if (lane == 0)
 #pragma unroll
         for (int k = 0; k < NV; k++) sm[k * kCgWarps + wid] = v[k];
@@ -345,6 +349,7 @@ cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int
     if (bps < 1) return cudaErrorCooperativeLaunchTooLarge;
     long long want = (a.K.nslices + kCgWarps - 1) / kCgWarps;   // one slice per warp at most
     int grid = nsm * bps;
+    if (grid > 2 * kCgThreads) grid = 2 * kCgThreads;   // block_total reads <= 2 partials per thread
     if (want < grid) grid = (int)(want > 0 ? want : 1);
     CgArgs args = a;
     void *params[] = {&args};
@@ -357,6 +362,192 @@ cudaError_t launch_efield(const double *xyz, const int32_t *c2n, const double *p
                           double *ef, double4 *efp, cudaStream_t s) {
     if (nc == 0) return cudaSuccess;
     k_efield<<<(unsigned)((nc + 255) / 256), 256, 0, s>>>(xyz, c2n, phi, nc, ef, efp);
+    return cudaGetLastError();
+}
+
+}  // namespace opp
+
+// ---------------------------------------------------------------------------
+// Host-driven CG kernels (multi-rank slabs; see opp_field.h)
+// ---------------------------------------------------------------------------
+namespace opp {
+namespace {
+
+__global__ void k_cg_x0(FieldMat K, double *x, int warm) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    x[i] = K.dmask[i] ? K.dval[i] : (warm ? x[i] : 0.0);
+}
+
+__global__ void k_spmv(FieldMat K, const double *__restrict__ v, double *__restrict__ y,
+                       double *__restrict__ yd) {
+    const int lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long TW = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long sl = gw; sl < K.nslices; sl += TW) {
+        long long i = sl * kSell + lane;
+        if (i >= K.nn) continue;
+        if (!yd) {
+            y[i] = sell_row(K, sl, lane, v);
+            continue;
+        }
+        long long off = K.slice_off[sl];
+        int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+        double ax = 0.0, ad = 0.0;
+        for (int k = 0; k < W; k++) {
+            long long q = off + (long long)kSell * k + lane;
+            int c = K.col[q];
+            double t = K.val[q] * v[c];
+            ax += t;
+            if (K.dmask[c]) ad += t;
+        }
+        y[i] = ax;
+        yd[i] = ad;
+    }
+}
+
+__global__ void k_cg_r0(FieldMat K, const double *__restrict__ Q, double rhs_scale,
+                        const double *__restrict__ y, const double *__restrict__ yd, double *r,
+                        double *u, double *p, double *sv, double *beff, int precond) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    double ri = 0.0, bi = 0.0;
+    if (!K.dmask[i]) {
+        double b = rhs_scale * Q[i];
+        ri = b - y[i];
+        bi = b - yd[i];
+    }
+    r[i] = ri;
+    beff[i] = bi;
+    u[i] = precond ? ri * K.dinv[i] : ri;
+    p[i] = 0.0;
+    sv[i] = 0.0;
+}
+
+constexpr int kDotThreads = 256;
+struct DotArgs {
+    const double *a[4];
+    const double *b[4];
+};
+
+template <int NV>
+__global__ void __launch_bounds__(kDotThreads) k_dots_part(long long n, const double *__restrict__ own,
+                                                           DotArgs d, double *part) {
+    __shared__ double sm[4 * kCgWarps];
+    double v[NV];
+#pragma unroll
+    for (int k = 0; k < NV; k++) v[k] = 0.0;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x) {
+        const double o = own ? own[i] : 1.0;
+#pragma unroll
+        for (int k = 0; k < NV; k++) v[k] += o * d.a[k][i] * d.b[k][i];
+    }
+    block_publish<NV>(v, part, sm);
+}
+
+__global__ void k_dots_final(const double *__restrict__ part, int nblk, int nv, double *out) {
+    // one warp per value, fixed order: deterministic
+    const int k = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (k >= nv) return;
+    double t = 0.0;
+    for (int b = lane; b < nblk; b += 32) t += part[k * nblk + b];
+    t = warp_sum(t);
+    if (lane == 0) out[k] = t;
+}
+
+__global__ void k_cg_update(FieldMat K, double alpha, double beta, double *x, double *r, double *u,
+                            const double *__restrict__ w, double *p, double *sv, int precond) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    double pi = u[i] + beta * p[i];
+    double si = w[i] + beta * sv[i];
+    p[i] = pi;
+    sv[i] = si;
+    x[i] += alpha * pi;
+    double ri = r[i] - alpha * si;
+    r[i] = ri;
+    u[i] = precond ? ri * K.dinv[i] : ri;
+}
+
+__global__ void k_diag(FieldMat K, double *diag) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    long long sl = i / kSell;
+    int lane = (int)(i % kSell);
+    long long off = K.slice_off[sl];
+    int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+    double d = 0.0;
+    for (int k = 0; k < W; k++)
+        if (K.col[off + (long long)kSell * k + lane] == (int32_t)i) {
+            d = K.val[off + (long long)kSell * k + lane];
+            break;
+        }
+    diag[i] = d;
+}
+
+__global__ void k_dinv(FieldMat K, const double *__restrict__ diag) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn) return;
+    K.dinv[i] = K.dmask[i] ? 1.0 : 1.0 / diag[i];
+}
+
+inline unsigned blocks_for(long long n) { return (unsigned)((n + 255) / 256 > 0 ? (n + 255) / 256 : 1); }
+
+}  // namespace
+
+cudaError_t launch_cg_x0(const FieldMat &K, double *x, int warm, cudaStream_t s) {
+    k_cg_x0<<<blocks_for(K.nn), 256, 0, s>>>(K, x, warm);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_spmv(const FieldMat &K, const double *v, double *y, double *yd, int nsm,
+                        cudaStream_t s) {
+    long long warps = K.nslices;
+    long long blocks = (warps + 7) / 8;
+    if (blocks > 4ll * nsm) blocks = 4ll * nsm;
+    k_spmv<<<(unsigned)(blocks > 0 ? blocks : 1), 256, 0, s>>>(K, v, y, yd);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cg_r0(const FieldMat &K, const double *Q, double rhs_scale, const double *y,
+                         const double *yd, double *r, double *u, double *p, double *sv,
+                         double *beff, int precond, cudaStream_t s) {
+    k_cg_r0<<<blocks_for(K.nn), 256, 0, s>>>(K, Q, rhs_scale, y, yd, r, u, p, sv, beff, precond);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dots(long long n, const double *own, int nv, const double *const *va,
+                        const double *const *vb, double *part, int nblk, double *out,
+                        cudaStream_t s) {
+    DotArgs d{};
+    for (int k = 0; k < nv; k++) {
+        d.a[k] = va[k];
+        d.b[k] = vb[k];
+    }
+    switch (nv) {
+    case 1: k_dots_part<1><<<nblk, kDotThreads, 0, s>>>(n, own, d, part); break;
+    case 3: k_dots_part<3><<<nblk, kDotThreads, 0, s>>>(n, own, d, part); break;
+    default: return cudaErrorInvalidValue;
+    }
+    k_dots_final<<<1, 32 * nv, 0, s>>>(part, nblk, nv, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cg_update(const FieldMat &K, double alpha, double beta, double *x, double *r,
+                             double *u, const double *w, double *p, double *sv, int precond,
+                             cudaStream_t s) {
+    k_cg_update<<<blocks_for(K.nn), 256, 0, s>>>(K, alpha, beta, x, r, u, w, p, sv, precond);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_diag(const FieldMat &K, double *diag, cudaStream_t s) {
+    k_diag<<<blocks_for(K.nn), 256, 0, s>>>(K, diag);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dinv(const FieldMat &K, const double *diag, cudaStream_t s) {
+    k_dinv<<<blocks_for(K.nn), 256, 0, s>>>(K, diag);
     return cudaGetLastError();
 }
 

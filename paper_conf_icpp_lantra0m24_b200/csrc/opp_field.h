@@ -59,3 +59,27 @@ cudaError_t launch_efield(const double *xyz, const int32_t *c2n, const double *p
                           double *ef, double4 *efp, cudaStream_t s);
 
 }  // namespace opp
+
+// ---- host-driven CG (nranks > 1, or OPP_CG_HOSTLOOP=1): one kernel per
+// phase, the partial SpMV rows of interface nodes completed by the charge
+// halo exchange, dot products over owned nodes reduced across ranks.
+namespace opp {
+cudaError_t launch_cg_x0(const FieldMat &K, double *x, int warm, cudaStream_t s);
+// y = K v over all local rows; yd (may be NULL) = the Dirichlet-column part.
+cudaError_t launch_spmv(const FieldMat &K, const double *v, double *y, double *yd, int nsm,
+                        cudaStream_t s);
+// r = b - y, beff = b - yd on free rows (0 on Dirichlet rows), u = M^-1 r, p = s = 0.
+cudaError_t launch_cg_r0(const FieldMat &K, const double *Q, double rhs_scale, const double *y,
+                         const double *yd, double *r, double *u, double *p, double *sv,
+                         double *beff, int precond, cudaStream_t s);
+// out[k] = sum_i own[i] * a_k[i] * b_k[i], k < nv (deterministic two-pass sum).
+cudaError_t launch_dots(long long n, const double *own, int nv, const double *const *va,
+                        const double *const *vb, double *part, int nblk, double *out,
+                        cudaStream_t s);
+cudaError_t launch_cg_update(const FieldMat &K, double alpha, double beta, double *x, double *r,
+                             double *u, const double *w, double *p, double *sv, int precond,
+                             cudaStream_t s);
+// diag[i] = K_ii (local partial on interface rows); then dinv from the summed diag.
+cudaError_t launch_diag(const FieldMat &K, double *diag, cudaStream_t s);
+cudaError_t launch_dinv(const FieldMat &K, const double *diag, cudaStream_t s);
+}  // namespace opp

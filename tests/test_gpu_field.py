@@ -30,9 +30,12 @@ def _set_charge(sim, Q):
     O.opp_set_dat(sim.ctx, sim.node_charge, np.ascontiguousarray(Q, np.float64), sim.nn)
 
 
+@pytest.mark.parametrize("hostloop", ["0", "1"])
 @pytest.mark.parametrize("precond", [0, 1])
 @pytest.mark.parametrize("dims,jit", [((6, 6, 30), 0.2), ((5, 3, 7), 0.1), ((1, 1, 1), 0.0)])
-def test_field_solve_matches_direct_solve(dims, jit, precond):
+def test_field_solve_matches_direct_solve(dims, jit, precond, hostloop, monkeypatch):
+    """hostloop 1: the host-driven CG (the multi-rank solver) on one rank."""
+    monkeypatch.setenv("OPP_CG_HOSTLOOP", hostloop)
     mesh = gen.kuhn_duct(*dims, jitter=jit, seed=4)
     xyz, c2n = mesh["node_xyz"], mesh["c2n"]
     rng = np.random.default_rng(1)

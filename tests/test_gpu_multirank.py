@@ -77,3 +77,63 @@ def test_loopback_multi_slab_crossing_and_sort():
     om, orc, Qo, ost, rem = run_oracle(mesh, ef, init, inject, steps, QM * DT, DT, W)
     parts, Qg, stats = _run_ranks(mesh, ef, init, inject, steps, 4, sort_every=2, deposit_mode=1)
     compare(om, mesh["c2n"], orc, Qo, rem, parts, Qg, W)
+
+
+@pytest.mark.parametrize("R", [2, 3])
+def test_loopback_field_solve_equals_single_domain(R):
+    """Slab-partitioned CG (host-driven, node halo + cross-rank dots) on R
+    contexts: the merged potential equals the single-domain direct solve
+    within the CG bound, interface copies agree, and each rank's cell field
+    is -grad(phi) of its potential."""
+    import torch
+    from oracle import field as F
+    from paper_conf_icpp_lantra0m24_b200 import dist
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh = gen.kuhn_duct(5, 4, 12, jitter=0.15, seed=8)
+    rng = np.random.default_rng(3)
+    Qg = rng.uniform(0.0, 4.0, mesh["n_nodes"])
+    mask, val = gen.duct_bc(mesh, wall=0.03, inlet=0.0)
+    rhs_scale, tol = 0.01, 1e-12
+    K = F.stiffness(mesh["node_xyz"], mesh["c2n"])
+    phi_ref = F.solve(K, F.load_vector(Qg, rhs_scale), mask, val)
+    uid = os.urandom(128)
+    streams = [torch.cuda.Stream() for _ in range(R)]
+    out, errs = [None] * R, []
+
+    def worker(r):
+        try:
+            sl = dist.slab(mesh, R, r)
+            sim = MiniFemPic(sl, np.zeros((sl["n_cells"], 3)), nranks=R, rank=r, uid=uid,
+                             transport=1, torch_alloc=False, stream=streams[r].cuda_stream)
+            gid = sl["node_gid"]
+            sim.field_init(mask[gid], val[gid])
+            O.opp_set_dat(sim.ctx, sim.node_charge, np.ascontiguousarray(Qg[gid]), sim.nn)
+            st = sim.field_solve(rhs_scale, tol=tol, warm_start=False)
+            out[r] = (gid, sim.potential_host(), sim.field_host(), st, sl)
+            sim.close()
+        except Exception as e:   # noqa: BLE001
+            errs.append((r, e))
+            raise
+
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(R)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not errs, errs
+    phi = np.full(mesh["n_nodes"], np.nan)
+    its = {o[3]["iterations"] for o in out}
+    assert len(its) == 1 and all(o[3]["converged"] == 1 for o in out)   # one global CG
+    for gid, ph, E, st, sl in out:
+        seen = ~np.isnan(phi[gid])
+        np.testing.assert_array_equal(phi[gid][seen], ph[seen])     # interface copies agree
+        phi[gid] = ph
+        Eo = F.efield(sl["node_xyz"], sl["c2n"], ph)
+        np.testing.assert_allclose(E, Eo, rtol=0, atol=1e-13 * max(np.abs(Eo).max(), 1e-3))
+    assert not np.isnan(phi).any()
+    free = mask == 0
+    lam_min = np.linalg.eigvalsh(K[free][:, free].toarray())[0]
+    b = F.load_vector(Qg, rhs_scale)
+    rhs = b[free] - K[free][:, ~free] @ val[~free]
+    assert np.linalg.norm(phi - phi_ref) <= 2 * tol * np.linalg.norm(rhs) / lam_min + 1e-14
