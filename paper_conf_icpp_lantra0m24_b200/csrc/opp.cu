@@ -150,6 +150,7 @@ struct opp_ctx_s {
     int sort_hgrid = 8;            // OPP_SORT_HGRID / OPP_SORT_RGRID: blocks per SM of the
     int sort_rgrid = 8;            //   sort histogram / rank kernels
     int prefetch = 0;              // OPP_PREFETCH: producer-warp L1 warming
+    int pairs = 0;                 // OPP_PAIRS: pair-per-lane tiled kernel (DH 0 / 1)
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -280,6 +281,7 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (const char *e = getenv("OPP_SORT_HGRID")) c->sort_hgrid = atoi(e);
     if (const char *e = getenv("OPP_SORT_RGRID")) c->sort_rgrid = atoi(e);
     if (const char *pf = getenv("OPP_PREFETCH")) c->prefetch = atoi(pf);
+    if (const char *pp = getenv("OPP_PAIRS")) c->pairs = atoi(pp);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
         delete c;
@@ -1218,6 +1220,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.refill = c->refill;
     a.minb = c->minb;
     a.prefetch = c->prefetch;
+    a.pairs = c->pairs && c->p.direct_hop != 2;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const int dh = c->p.direct_hop;
@@ -1230,7 +1233,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     c->launches++;
     const bool tiled = c->p.tma_pipeline != 0;
-    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb);
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb, a.pairs != 0);
     const int bps = c->bps;
     const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
                                                                        (long long)c->nsm * bps));

@@ -97,6 +97,7 @@ struct StepArgs {
     int refill;                // tiled kernel: per-lane refill consumer (OPP_REFILL)
     int minb;                  // tiled kernel: min resident blocks per SM (OPP_MINB: 1 or 3)
     int prefetch;              // tiled kernel: producer-warp L1 warming (OPP_PREFETCH, default 1)
+    int pairs;                 // tiled kernel: two adjacent particles per lane (OPP_PAIRS; DH 0/1)
     int dbg;                   // diagnostics only (OPP_PMD_DEBUG): 1 stream, 2 +E, 3 +line, 4 no deposit
     Overlay ov;
 };

@@ -150,36 +150,31 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 // DEP 1: lanes with the same cell (same 4 nodes) are aggregated inside the
 //        warp before one set of 4 reductions per cell -- "warp-level
 //        aggregation of same-cell deposits before global atomics".
-template <int DEP>
-__device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int cell, int4 cn,
-                                        double w, double l0, double l1, double l2, double l3) {
-    double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
-    if (DEP == 0) {
-        if (done) {
-            atomicAdd(Q + cn.x, v0);
-            atomicAdd(Q + cn.y, v1);
-            atomicAdd(Q + cn.z, v2);
-            atomicAdd(Q + cn.w, v3);
-        }
-        return;
-    }
-    // Lanes depositing into the same cell (hence the same 4 nodes) are found
-    // with __match_any_sync wherever they sit in the warp; their 4 values are
-    // summed by a log-step tree over each peer group, and the group's lowest
-    // lane issues the 4 reductions.
+//
+// Lanes with the same key are found with __match_any_sync wherever they sit
+// in the warp.  A lane alone with its cell reduces straight to Q.  Each
+// group of >= 2 lanes (in cell-sorted storage: the one or two cells a warp's
+// slice covers, while the few particles that hopped are mostly alone) is
+// summed by a full-warp reduce-scatter -- xor 16 halves the 4 values, xor 8
+// halves them again, xor 4/2/1 finish -- 12 shuffles and 6 adds per group;
+// lanes 0, 8, 16, 24 then hold the group's 4 sums and issue one reduction
+// each.  With more than kMaxRsGroups groups a log-step tree over each group
+// (lowest lane issues the 4 reductions) is cheaper.
+constexpr int kMaxRsGroups = 3;
+
+__device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0, double v1,
+                                     double v2, double v3) {
+    atomicAdd(Q + cn.x, v0);
+    atomicAdd(Q + cn.y, v1);
+    atomicAdd(Q + cn.z, v2);
+    atomicAdd(Q + cn.w, v3);
+}
+
+// Log-step tree over every peer group of the lanes with `act` set.
+__device__ __forceinline__ void deposit_tree(double *__restrict__ Q, bool act, unsigned peers,
+                                             int4 cn, double v0, double v1, double v2, double v3) {
     const unsigned lane = lane_id();
-    const int key = done ? cell : -2 - (int)lane;
-    unsigned peers = __match_any_sync(0xffffffffu, key);
     const int first = __ffs(peers) - 1;
-    if (__all_sync(0xffffffffu, peers == (1u << lane))) {   // no duplicates: plain reductions
-        if (done) {
-            atomicAdd(Q + cn.x, v0);
-            atomicAdd(Q + cn.y, v1);
-            atomicAdd(Q + cn.z, v2);
-            atomicAdd(Q + cn.w, v3);
-        }
-        return;
-    }
     int rel = __popc(peers & ((1u << lane) - 1u));       // my rank inside the group
     unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
     if (lane == 31) up = 0;
@@ -195,15 +190,61 @@ __device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int c
         // lanes at odd group rank have been absorbed by their lower neighbour
         const unsigned gone = __ballot_sync(0xffffffffu, (rel & 1) != 0);
         up &= ~gone;
-        // the next surviving peer above: skip the absorbed ones
         rel >>= 1;
     }
-    if (done && (int)lane == first) {
-        atomicAdd(Q + cn.x, v0);
-        atomicAdd(Q + cn.y, v1);
-        atomicAdd(Q + cn.z, v2);
-        atomicAdd(Q + cn.w, v3);
+    if (act && (int)lane == first) red4(Q, cn, v0, v1, v2, v3);
+}
+
+// Warp-aggregated deposit of (key, cn, v0..v3) for the lanes with `done`
+// (key: the cell; lanes with equal keys have equal cn).
+__device__ __forceinline__ void deposit_agg(double *__restrict__ Q, bool done, int key, int4 cn,
+                                            double v0, double v1, double v2, double v3) {
+    const unsigned FULL = 0xffffffffu;
+    const unsigned lane = lane_id();
+    const unsigned peers = __match_any_sync(FULL, done ? key : -2 - (int)lane);
+    const bool single = peers == (1u << lane);
+    if (done && single) red4(Q, cn, v0, v1, v2, v3);
+    unsigned lead = __ballot_sync(FULL, done && !single && (int)lane == __ffs(peers) - 1);
+    if (!lead) return;
+    if (__popc(lead) > kMaxRsGroups) {
+        deposit_tree(Q, done && !single, peers, cn, v0, v1, v2, v3);
+        return;
     }
+    const bool h16 = (lane & 16u) != 0, h8 = (lane & 8u) != 0;
+    do {
+        const int L = __ffs(lead) - 1;
+        lead &= lead - 1u;
+        const unsigned gm = __shfl_sync(FULL, peers, L);
+        const bool in = done && ((gm >> lane) & 1u);
+        const double a0 = in ? v0 : 0.0, a1 = in ? v1 : 0.0, a2 = in ? v2 : 0.0, a3 = in ? v3 : 0.0;
+        double k0 = h16 ? a2 : a0, k1 = h16 ? a3 : a1;    // the pair this lane keeps
+        const double s0 = h16 ? a0 : a2, s1 = h16 ? a1 : a3;
+        k0 = add(k0, __shfl_xor_sync(FULL, s0, 16));
+        k1 = add(k1, __shfl_xor_sync(FULL, s1, 16));
+        double t = h8 ? k1 : k0;
+        t = add(t, __shfl_xor_sync(FULL, h8 ? k0 : k1, 8));
+        t = add(t, __shfl_xor_sync(FULL, t, 4));
+        t = add(t, __shfl_xor_sync(FULL, t, 2));
+        t = add(t, __shfl_xor_sync(FULL, t, 1));
+        // lane 8q holds the sum of value q = 2*h16 + h8
+        const int n0 = __shfl_sync(FULL, cn.x, L), n1 = __shfl_sync(FULL, cn.y, L);
+        const int n2 = __shfl_sync(FULL, cn.z, L), n3 = __shfl_sync(FULL, cn.w, L);
+        if ((lane & 7u) == 0) {
+            const int node = h16 ? (h8 ? n3 : n2) : (h8 ? n1 : n0);
+            atomicAdd(Q + node, t);
+        }
+    } while (lead);
+}
+
+template <int DEP>
+__device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int cell, int4 cn,
+                                        double w, double l0, double l1, double l2, double l3) {
+    double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
+    if (DEP == 0) {
+        if (done) red4(Q, cn, v0, v1, v2, v3);
+        return;
+    }
+    deposit_agg(Q, done, cell, cn, v0, v1, v2, v3);
 }
 
 // SR deposit, phase 1: store (cell, w*lambda[4]) records.
@@ -400,6 +441,17 @@ __device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *coun
 __device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b);
 __device__ __forceinline__ void fence_proxy_async_fwd();
 
+// Gathers of the NEXT slice issued one slice ahead by the TMA-pipelined
+// consumer (OPP_PREFETCH_NEXT): the cell field and the speculative overlay
+// entry only depend on the streamed state, so they leave the per-slice
+// dependent chain (their latency hides behind the current slice's walk).
+struct Pre {
+    long long slot;
+    int val;
+    double2 Exy;
+    double Ez;
+};
+
 // `release`: the stage mbarrier to arrive on once this warp no longer needs
 // the shared-memory copy of its particles (TMA-pipelined kernel; every lane
 // valid) -- after the push has consumed all seven loaded values, so no shared
@@ -409,7 +461,8 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                                          int hops, double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
                                          uint64_t *release = nullptr, double *sout = nullptr,
-                                         int sj = 0, Appends *ap = nullptr) {
+                                         int sj = 0, Appends *ap = nullptr,
+                                         const Pre *pre = nullptr) {
     int status = ST_NONE;
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -444,14 +497,21 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             // position and the lookup leaves the dependent chain.
             long long spec_slot = -1;
             int spec_val = -1;
-            if (DH == 1) {
-                spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
-                                    add(z, mul(vz, a.dt)));
-                spec_val = __ldg(a.ov.map + (spec_slot >= 0 ? spec_slot : 0));
-            }
             double2 Exy;
             double Ez;
-            load_E(a.ef, lc, Exy, Ez);
+            if (pre) {
+                spec_slot = pre->slot;
+                spec_val = pre->val;
+                Exy = pre->Exy;
+                Ez = pre->Ez;
+            } else {
+                if (DH == 1) {
+                    spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
+                                        add(z, mul(vz, a.dt)));
+                    spec_val = __ldg(a.ov.map + (spec_slot >= 0 ? spec_slot : 0));
+                }
+                load_E(a.ef, lc, Exy, Ez);
+            }
             vx = add(vx, mul(a.c1, Exy.x));
             vy = add(vy, mul(a.c1, Exy.y));
             vz = add(vz, mul(a.c1, Ez));
@@ -739,8 +799,14 @@ __device__ __forceinline__ void warm_tile(const StepArgs &a, char *smem, uint64_
     }
 }
 
+#ifndef OPP_PRE
+#define OPP_PRE 0   // 1: issue the next slice's E / overlay gathers one slice ahead
+                    // (C2: pmd 1.98 vs 1.94 ms -- the extra stage reads cost more L1
+                    // data-pipe wavefronts than the hidden latency saves)
+#endif
 template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
 __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
+    constexpr bool PRE = OPP_PRE != 0;
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
     uint64_t *empty = full + kStages;
@@ -796,6 +862,8 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
                                reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
         }
         TileIter ti(tm);
+        Pre cur{-1, -1, make_double2(0.0, 0.0), 0.0};
+        bool have_cur = false;
         for (unsigned long long it = 0; it < my; it++, ti.next()) {
             const int s = (int)(it % kStages);
             const int ob_i = 0;   // one output buffer per warp (keeps 3 blocks / SM in smem)
@@ -805,6 +873,28 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
             double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
             int cell = v.cell[j];
+            Pre nxt;
+            bool have_nxt = false;
+            if (PRE && it + 1 < my) {
+                const int s1 = (int)((it + 1) % kStages);
+                const bool landed = __all_sync(0xffffffffu,
+                                               mbar_test(&full[s1], (uint32_t)(((it + 1) / kStages) & 1ull)));
+                if (landed) {
+                    StageView v1 = stage_view(smem, s1);
+                    const double x1 = v1.c[0][j], y1 = v1.c[1][j], z1 = v1.c[2][j];
+                    const double vx1 = v1.c[3][j], vy1 = v1.c[4][j], vz1 = v1.c[5][j];
+                    const int c1 = v1.cell[j];
+                    nxt.slot = -1;
+                    nxt.val = -1;
+                    if (DH == 1) {
+                        nxt.slot = dh_slot(a.ov, add(x1, mul(vx1, a.dt)), add(y1, mul(vy1, a.dt)),
+                                           add(z1, mul(vz1, a.dt)));
+                        nxt.val = __ldg(a.ov.map + (nxt.slot >= 0 ? nxt.slot : 0));
+                    }
+                    load_E(a.ef, c1 - a.cell_base, nxt.Exy, nxt.Ez);
+                    have_nxt = true;
+                }
+            }
             const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
                                          (unsigned long long)__double_as_longlong(y) ^
                                          (unsigned long long)__double_as_longlong(z) ^
@@ -825,7 +915,12 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             double *o = reinterpret_cast<double *>(smem + kOutBase +
                                                    (size_t)(warp + ob_i) * kOutBytes);
             pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
-                                                  nullptr, o, (int)lane, &ap);
+                                                  nullptr, o, (int)lane, &ap,
+                                                  (PRE && have_cur) ? &cur : nullptr);
+            if (PRE) {
+                cur = nxt;
+                have_cur = have_nxt;
+            }
             reinterpret_cast<int *>(o + 192)[lane] = cell;
             fence_proxy_async();
             __syncwarp();
@@ -985,6 +1080,256 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             active = false;
         }
     }
+    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
+}
+
+// ---------------------------------------------------------------------------
+// Pair-per-lane variant of the TMA-pipelined pass (StepArgs.pairs; DH 0 / 1).
+// Same producer warp and bulk-copy pipeline, but 4 consumer warps per tile,
+// each lane carrying two ADJACENT particles (2l, 2l+1 of its warp's 64).  In
+// cell-sorted storage the two usually share their start cell and their
+// final cell, so one E gather and one 128-B walk line serve both (the L1
+// data pipe that returns gathered bytes to registers is the busiest unit of
+// the one-per-lane kernel: every lane receives its own copy of the line),
+// their deposits merge in registers before the warp aggregation, and the
+// per-warp pipeline bookkeeping (barrier waits, fences, bulk stores, ring
+// flushes) is paid once per 64 particles.  Walks that leave the shared line
+// (hops, a different seed cell) take the general walk with their own loads.
+// ---------------------------------------------------------------------------
+constexpr int kPairWarps = kTile / 64;
+constexpr int kPairThreads = kPairWarps * 32 + 32;
+constexpr int kPairOutBytes = 64 * (6 * 8 + 4);
+constexpr int kPairOutBase = kStages * kStageBytes + 2 * kStages * 8;
+constexpr int kPairRingBase = kPairOutBase + kPairWarps * kPairOutBytes;
+constexpr int kPairSmem = kPairRingBase + kPairWarps * kRingBytesPerWarp;
+
+__device__ __forceinline__ bool inside4(double l0, double l1, double l2, double l3) {
+    return in01(l0) & in01(l1) & in01(l2) & in01(l3);
+}
+
+// Walk from `cell` (its line loaded here: an L1 hit in sorted storage).
+template <bool MULTI>
+__device__ __forceinline__ int walk_cell(const StepArgs &a, int &cell, double x, double y, double z,
+                                         int &hops, double &l0, double &l1, double &l2, double &l3,
+                                         int &capped, int4 &cn) {
+    Line L = load_line(a.lines, cell - a.cell_base);
+    return walk_from<MULTI>(a, cell, L, PosRegs{x, y, z}, hops, a.hpass, l0, l1, l2, l3, capped, cn);
+}
+
+__device__ __forceinline__ void tally(Tally &t, int st, int hops, int capped) {
+    if (st != ST_MOVE && st != ST_MIGRATE) {
+        t.hops += (unsigned)hops;
+        t.maxh = max(t.maxh, (unsigned)hops);
+        t.capped += (unsigned)capped;
+    }
+    t.removed += (st == ST_REMOVE);
+}
+
+// DH seed of a pushed position given the speculative lookup (see pmd_body).
+__device__ __forceinline__ int dh_seed_spec(const Overlay &ov, double x, double y, double z, int cell,
+                                            long long spec_slot, int spec_val) {
+    const long long g = dh_slot(ov, x, y, z);
+    int v = g == spec_slot ? spec_val : (g >= 0 ? __ldg(ov.map + g) : -1);
+    if (g < 0) v = -1;
+    return v >= 0 ? v : cell;
+}
+
+template <int DEP, int DH, bool MULTI>
+__device__ __forceinline__ void pair_body(const StepArgs &a, unsigned long long ia, double2 X,
+                                          double2 Y, double2 Z, double2 VX, double2 VY, double2 VZ,
+                                          int2 C, Tally &t, double *o, unsigned lane, Appends &ap) {
+    const unsigned FULL = 0xffffffffu;
+    const int ca = C.x, cb = C.y;
+    long long spa = -1, spb = -1;
+    int sva = -1, svb = -1;
+    if (DH == 1) {   // speculative overlay entries of the drift-only positions (see pmd_body)
+        spa = dh_slot(a.ov, add(X.x, mul(VX.x, a.dt)), add(Y.x, mul(VY.x, a.dt)), add(Z.x, mul(VZ.x, a.dt)));
+        spb = dh_slot(a.ov, add(X.y, mul(VX.y, a.dt)), add(Y.y, mul(VY.y, a.dt)), add(Z.y, mul(VZ.y, a.dt)));
+        sva = __ldg(a.ov.map + (spa >= 0 ? spa : 0));
+        svb = spb == spa ? sva : __ldg(a.ov.map + (spb >= 0 ? spb : 0));
+    }
+    // gather the cell-constant field (one load when the pair shares its cell), push
+    double2 Ea, Eb;
+    double Eaz, Ebz;
+    load_E(a.ef, ca - a.cell_base, Ea, Eaz);
+    if (cb != ca) {
+        load_E(a.ef, cb - a.cell_base, Eb, Ebz);
+    } else {
+        Eb = Ea;
+        Ebz = Eaz;
+    }
+    VX.x = add(VX.x, mul(a.c1, Ea.x)); VY.x = add(VY.x, mul(a.c1, Ea.y)); VZ.x = add(VZ.x, mul(a.c1, Eaz));
+    VX.y = add(VX.y, mul(a.c1, Eb.x)); VY.y = add(VY.y, mul(a.c1, Eb.y)); VZ.y = add(VZ.y, mul(a.c1, Ebz));
+    X.x = add(X.x, mul(VX.x, a.dt)); Y.x = add(Y.x, mul(VY.x, a.dt)); Z.x = add(Z.x, mul(VZ.x, a.dt));
+    X.y = add(X.y, mul(VX.y, a.dt)); Y.y = add(Y.y, mul(VY.y, a.dt)); Z.y = add(Z.y, mul(VZ.y, a.dt));
+    {
+        double2 *o2 = reinterpret_cast<double2 *>(o) + lane;   // column k: o + 64 k
+        o2[0] = X; o2[32] = Y; o2[64] = Z; o2[96] = VX; o2[128] = VY; o2[160] = VZ;
+    }
+    int sa = ca, sb = cb;
+    if (DH == 1) {
+        sa = dh_seed_spec(a.ov, X.x, Y.x, Z.x, ca, spa, sva);
+        sb = dh_seed_spec(a.ov, X.y, Y.y, Z.y, cb, spb, svb);
+    }
+    // the shared line: issued after the push (opaque dependency on z) so the
+    // line registers and the velocities are never live together
+    int zero;
+    asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}" : "=r"(zero) : "d"(Z.y));
+    int cellA = sa, cellB = sb;
+    double la0, la1, la2, la3, lb0 = 0, lb1 = 0, lb2 = 0, lb3 = 0;
+    int4 cna, cnb;
+    bool ina, inb = false;
+    const bool sameb = sb == sa;
+    {
+        const Line L = load_line(a.lines, sa - a.cell_base + zero);
+        bary(L, X.x, Y.x, Z.x, la0, la1, la2, la3);
+        ina = inside4(la0, la1, la2, la3);
+        cna = L.cn;
+        cnb = L.cn;
+        if (sameb) {
+            bary(L, X.y, Y.y, Z.y, lb0, lb1, lb2, lb3);
+            inb = inside4(lb0, lb1, lb2, lb3);
+        }
+    }
+    int hA = 0, hB = 0, capA = 0, capB = 0;
+    int stA = ST_DONE, stB = ST_DONE;
+    if (!ina) stA = walk_cell<MULTI>(a, cellA, X.x, Y.x, Z.x, hA, la0, la1, la2, la3, capA, cna);
+    if (!inb) stB = walk_cell<MULTI>(a, cellB, X.y, Y.y, Z.y, hB, lb0, lb1, lb2, lb3, capB, cnb);
+    tally(t, stA, hA, capA);
+    tally(t, stB, hB, capB);
+    // deposit (Eq. 10)
+    const bool dA = stA == ST_DONE, dB = stB == ST_DONE;
+    if (DEP == 2) {
+        sr_store(a, dA, cellA, a.w, la0, la1, la2, la3);
+        sr_store(a, dB, cellB, a.w, lb0, lb1, lb2, lb3);
+    } else {
+        double va0 = mul(a.w, la0), va1 = mul(a.w, la1), va2 = mul(a.w, la2), va3 = mul(a.w, la3);
+        const double vb0 = mul(a.w, lb0), vb1 = mul(a.w, lb1), vb2 = mul(a.w, lb2), vb3 = mul(a.w, lb3);
+        if (DEP == 0) {
+            if (dA) red4(a.Q, cna, va0, va1, va2, va3);
+            if (dB) red4(a.Q, cnb, vb0, vb1, vb2, vb3);
+        } else {
+            const bool merge = dA && dB && cellA == cellB;
+            if (merge) {
+                va0 = add(va0, vb0); va1 = add(va1, vb1); va2 = add(va2, vb2); va3 = add(va3, vb3);
+            }
+            const bool eA = dA || dB, eB = dA && dB && !merge;
+            // entry A: the merged pair, or whichever particle deposits
+            const bool useB = !dA && dB;
+            deposit_agg(a.Q, eA, useB ? cellB : cellA, useB ? cnb : cna, useB ? vb0 : va0,
+                        useB ? vb1 : va1, useB ? vb2 : va2, useB ? vb3 : va3);
+            if (__any_sync(FULL, eB)) deposit_agg(a.Q, eB, cellB, cnb, vb0, vb1, vb2, vb3);
+        }
+    }
+    // holes, deferred walks, migrants
+    const bool remA = stA == ST_REMOVE || stA == ST_MIGRATE;
+    const bool remB = stB == ST_REMOVE || stB == ST_MIGRATE;
+    ring_push(ap.holes, remA, (uint32_t)ia, 0);
+    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
+    ring_push(ap.holes, remB, (uint32_t)(ia + 1), 0);
+    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
+    ring_push(ap.work, stA == ST_MOVE, (uint32_t)ia, hA);
+    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
+    ring_push(ap.work, stB == ST_MOVE, (uint32_t)(ia + 1), hB);
+    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
+    if (MULTI) {
+        const bool mA = stA == ST_MIGRATE, mB = stB == ST_MIGRATE;
+        unsigned long long ms = warp_append(mA, &a.cnt->n_mig);
+        if (mA) { a.mig[ms] = (uint32_t)ia; a.mig_cell[ms] = cellA; a.mig_hops[ms] = hA; }
+        ms = warp_append(mB, &a.cnt->n_mig);
+        if (mB) { a.mig[ms] = (uint32_t)(ia + 1); a.mig_cell[ms] = cellB; a.mig_hops[ms] = hB; }
+    }
+    reinterpret_cast<int2 *>(o + 384)[lane] = make_int2(remA ? -1 : cellA, remB ? -1 : cellB);
+}
+
+#ifndef OPP_PAIR_MINB
+#define OPP_PAIR_MINB 4   // resident blocks per SM the pair kernel's registers are cut for
+#endif
+template <int DEP, int DH, bool MULTI>
+__global__ void __launch_bounds__(kPairThreads, OPP_PAIR_MINB) k_pmd_pairs(StepArgs a) {
+    extern __shared__ __align__(128) char smem[];
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
+    uint64_t *empty = full + kStages;
+    const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
+    const unsigned long long ntiles = n / kTile;
+    const TileMap tm{ntiles, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
+    const unsigned long long my = tm.count();
+    const int warp = threadIdx.x >> 5;
+    const unsigned lane = lane_id();
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kPairWarps);
+        }
+        fence_proxy_async();
+    }
+    __syncthreads();
+    if (warp == kPairWarps) {   // producer warp (lane 0): stream tiles kStages ahead
+        if (lane == 0) {
+            TileIter ti(tm);
+            for (unsigned long long it = 0; it < my; it++, ti.next()) {
+                const int s = (int)(it % kStages);
+                if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
+                issue_tile_load(a, smem, full, s, ti.tile());
+            }
+        }
+        return;
+    }
+    Appends ap;
+    {
+        char *rb = smem + kPairRingBase + (size_t)warp * kRingBytesPerWarp;
+        ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
+        ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
+                           reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
+    }
+    Tally t;
+    double *o = reinterpret_cast<double *>(smem + kPairOutBase + (size_t)warp * kPairOutBytes);
+    TileIter ti(tm);
+    for (unsigned long long it = 0; it < my; it++, ti.next()) {
+        const int s = (int)(it % kStages);
+        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
+        StageView v = stage_view(smem, s);
+        const int j = 64 * warp + 2 * (int)lane;
+        const double2 X = *reinterpret_cast<const double2 *>(v.c[0] + j);
+        const double2 Y = *reinterpret_cast<const double2 *>(v.c[1] + j);
+        const double2 Z = *reinterpret_cast<const double2 *>(v.c[2] + j);
+        const double2 VX = *reinterpret_cast<const double2 *>(v.c[3] + j);
+        const double2 VY = *reinterpret_cast<const double2 *>(v.c[4] + j);
+        const double2 VZ = *reinterpret_cast<const double2 *>(v.c[5] + j);
+        const int2 C = *reinterpret_cast<const int2 *>(v.cell + j);
+        unsigned long long h = 0;
+        h ^= (unsigned long long)__double_as_longlong(X.x) ^ (unsigned long long)__double_as_longlong(X.y);
+        h ^= (unsigned long long)__double_as_longlong(Y.x) ^ (unsigned long long)__double_as_longlong(Y.y);
+        h ^= (unsigned long long)__double_as_longlong(Z.x) ^ (unsigned long long)__double_as_longlong(Z.y);
+        h ^= (unsigned long long)__double_as_longlong(VX.x) ^ (unsigned long long)__double_as_longlong(VX.y);
+        h ^= (unsigned long long)__double_as_longlong(VY.x) ^ (unsigned long long)__double_as_longlong(VY.y);
+        h ^= (unsigned long long)__double_as_longlong(VZ.x) ^ (unsigned long long)__double_as_longlong(VZ.y);
+        h ^= (unsigned long long)(unsigned)C.x ^ (unsigned long long)(unsigned)C.y;
+        asm volatile("" ::"l"(h));   // the shared loads have landed
+        fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(&empty[s]);
+            if (it >= 1) bulk_wait_read0();   // the previous stores have read the buffer
+        }
+        __syncwarp();
+        const unsigned long long tile = ti.tile();
+        pair_body<DEP, DH, MULTI>(a, tile * kTile + j, X, Y, Z, VX, VY, VZ, C, t, o, lane, ap);
+        fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+            const unsigned long long g0 = tile * kTile + 64 * warp;
+            for (int k = 0; k < 3; k++) {
+                bulk_s2g(a.pos + k * a.cap + g0, o + 64 * k, 512);
+                bulk_s2g(a.vel + k * a.cap + g0, o + 64 * (3 + k), 512);
+            }
+            bulk_s2g(a.p2c + g0, o + 384, 256);
+            bulk_commit();
+        }
+    }
+    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
+    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
+    if (lane == 0) bulk_wait_all();
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
@@ -1804,8 +2149,25 @@ static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
                        : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
 }
 
+template <int DEP, int DH, bool MULTI>
+static cudaError_t launch_pairs(const StepArgs &a, int grid, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_pmd_pairs<DEP, DH, MULTI>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kPairSmem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    k_pmd_pairs<DEP, DH, MULTI><<<grid, kPairThreads, kPairSmem, s>>>(a);
+    k_push_move_deposit_tail<DEP, DH, MULTI><<<1, 256, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
 template <int DEP, int DH, bool CONT, bool MULTI>
 static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
+    if (!CONT && tiled && a.pairs && DH != 2) {
+        return launch_pairs<DEP, DH == 2 ? 0 : DH, MULTI>(a, grid, s);
+    }
     if (!CONT && tiled) {
         return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
                         : launch_tiled<DEP, DH, MULTI, false>(a, grid, s);
@@ -1842,10 +2204,15 @@ cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, boo
                 : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
 }
 
-int pmd_blocks_per_sm(bool tiled, int minb) {
+int pmd_blocks_per_sm(bool tiled, int minb, bool pairs) {
     int nb = 0;
     cudaError_t e;
-    if (tiled) {
+    if (tiled && pairs) {
+        cudaFuncSetAttribute(k_pmd_pairs<0, 0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             kPairSmem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_pmd_pairs<0, 0, false>,
+                                                          kPairThreads, kPairSmem);
+    } else if (tiled) {
         if (minb >= 3) {
             cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);

@@ -6,7 +6,7 @@ namespace opp {
 
 cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, bool tiled,
                                      const StepArgs &a, int grid, cudaStream_t s);
-int pmd_blocks_per_sm(bool tiled, int minb);
+int pmd_blocks_per_sm(bool tiled, int minb, bool pairs);
 cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero, int grid,
                               cudaStream_t s);
 cudaError_t launch_fill(const ColSet &cols, DevCounters *c, const uint32_t *holes,
