@@ -51,7 +51,7 @@ def parse():
                     help="1: overlay seed for every particle; 2: only for particles that left their cell")
     ap.add_argument("--ov", type=float, default=0.125, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
-    ap.add_argument("--sort", type=int, default=5, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--sort", type=int, default=10, help="sort by cell every K steps (0 = never)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
     ap.add_argument("--axis", action="store_true", help="sort key along the duct axis (z)")
     ap.add_argument("--no-e2e", action="store_true")

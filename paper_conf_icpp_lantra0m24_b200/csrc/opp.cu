@@ -84,6 +84,7 @@ struct PSet {
     std::vector<char *> alt;     // sort double buffers (one per column, lazily allocated)
     long long alt_cap = 0;
     long long steps = 0;         // pushes so far (drives sort_every)
+    bool fused_sort = false;     // this step's move already wrote the particles sorted
 };
 
 struct Set {
@@ -106,6 +107,8 @@ struct MeshCache {
     bool ov_built = false;
     Overlay ov{};
     int32_t *ov_map = nullptr;
+    int16_t *ov_off = nullptr;    // compact overlay (Overlay.compact)
+    int32_t *ov_base = nullptr;
     // sort locality key per cell (opp_init_params.sort_axis), NULL = cell order
     uint32_t *sort_key = nullptr;
     // per-cell counting (SR deposit and sort by cell)
@@ -150,7 +153,8 @@ struct opp_ctx_s {
     int sort_hgrid = 8;            // OPP_SORT_HGRID / OPP_SORT_RGRID: blocks per SM of the
     int sort_rgrid = 8;            //   sort histogram / rank kernels
     int prefetch = 0;              // OPP_PREFETCH: producer-warp L1 warming
-    int pairs = 0;                 // OPP_PAIRS: pair-per-lane tiled kernel (DH 0 / 1)
+    int fuse_sort = 0;             // OPP_FUSE_SORT=1: sort steps write the move's output sorted
+                                   //   (C2: slower -- 2.71 vs 2.42 ms/step: scattered writes)
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -281,7 +285,7 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     if (const char *e = getenv("OPP_SORT_HGRID")) c->sort_hgrid = atoi(e);
     if (const char *e = getenv("OPP_SORT_RGRID")) c->sort_rgrid = atoi(e);
     if (const char *pf = getenv("OPP_PREFETCH")) c->prefetch = atoi(pf);
-    if (const char *pp = getenv("OPP_PAIRS")) c->pairs = atoi(pp);
+    if (const char *fs = getenv("OPP_FUSE_SORT")) c->fuse_sort = atoi(fs);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
         delete c;
@@ -345,6 +349,8 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.lines, sizeof(WalkLine) * m.nc);
     c->dfree(m.efp, sizeof(double4) * m.nc);
     c->dfree(m.ov_map, 0);
+    c->dfree(m.ov_off, 0);
+    c->dfree(m.ov_base, 0);
     c->dfree(m.cell_hist, 0);
     c->dfree(m.cell_start, 0);
     c->dfree(m.tile_sums, 0);
@@ -928,6 +934,42 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         ov.map = m.ov_map;
         CK(launch_overlay(m.lines, (const double *)np.d, nc, c->cell_base, ov, m.ov_map, c->s));
         c->launches += 3;
+        // compact form (int16 offsets per 4x4x4 brick) when every brick fits
+        c->dfree(m.ov_off, 0);
+        c->dfree(m.ov_base, 0);
+        m.ov_off = nullptr;
+        m.ov_base = nullptr;
+        ov.compact = 0;
+        const char *ce = getenv("OPP_OV_COMPACT");
+        if (!ce || atoi(ce)) {
+            long long nbt = 1;
+            for (int k = 0; k < 3; k++) {
+                ov.nbc[k] = (ov.n[k] + 3) / 4;
+                nbt *= ov.nbc[k];
+            }
+            m.ov_off = (int16_t *)c->dalloc(2 * 64 * nbt);
+            m.ov_base = (int32_t *)c->dalloc(4 * nbt);
+            if (!m.ov_off || !m.ov_base) return fail(OPP_ERR_NOMEM, "compact overlay");
+            unsigned *flag = (unsigned *)m.tile_sums;   // scratch word (rebuilt before any scan)
+            CK(launch_overlay_compact(m.ov_map, ov, m.ov_off, m.ov_base, flag, c->s));
+            c->launches++;
+            unsigned over = 1;
+            CK(cudaMemcpyAsync(&over, flag, sizeof over, cudaMemcpyDeviceToHost, c->s));
+            CK(cudaStreamSynchronize(c->s));
+            if (!over) {
+                ov.compact = 1;
+                ov.off = m.ov_off;
+                ov.base = m.ov_base;
+                c->dfree(m.ov_map, 0);   // the int32 form is no longer needed
+                m.ov_map = nullptr;
+                ov.map = nullptr;
+            } else {
+                c->dfree(m.ov_off, 0);
+                c->dfree(m.ov_base, 0);
+                m.ov_off = nullptr;
+                m.ov_base = nullptr;
+            }
+        }
         m.ov = ov;
         m.ov_built = true;
     }
@@ -968,9 +1010,7 @@ static int check_col(opp_ctx c, int h, bool want_map, int set, int dim, int type
 }
 
 // Counting sort by cell into the double buffers, then swap (drops holes).
-static int do_sort(opp_ctx c, PSet &ps, int p2c) {
-    MeshCache &m = c->mc;
-    if (!m.cell_hist) return fail(OPP_ERR_STATE, "sort needs the mesh: run a step first");
+static int ensure_alt(opp_ctx c, PSet &ps) {
     if (ps.alt_cap != ps.cap) {
         for (size_t j = 0; j < ps.alt.size(); j++)
             c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
@@ -988,6 +1028,13 @@ static int do_sort(opp_ctx c, PSet &ps, int p2c) {
         }
         ps.alt_cap = ps.cap;
     }
+    return OPP_OK;
+}
+
+static int do_sort(opp_ctx c, PSet &ps, int p2c) {
+    MeshCache &m = c->mc;
+    if (!m.cell_hist) return fail(OPP_ERR_STATE, "sort needs the mesh: run a step first");
+    TRY(ensure_alt(c, ps));
     ColSet src = make_colset(c, ps), dst = src;
     for (int j = 0; j < dst.n; j++) dst.c[j].ptr = ps.alt[j];
     const int32_t *pc = (const int32_t *)c->cols[p2c].d;
@@ -1010,7 +1057,9 @@ static int do_sort(opp_ctx c, PSet &ps, int p2c) {
 
 static int do_fill(opp_ctx c, PSet &ps, int p2c) {
     PhaseScope ph(c, OPP_PH_FILL);
-    if (c->p.sort_every > 0 && ps.steps % c->p.sort_every == 0) return do_sort(c, ps, p2c);
+    if (c->p.sort_every > 0 && ps.steps % c->p.sort_every == 0 && !ps.fused_sort)
+        return do_sort(c, ps, p2c);
+    ps.fused_sort = false;
     ColSet cs = make_colset(c, ps);
     CK(launch_fill(cs, ps.dcnt, ps.holes, (const int32_t *)c->cols[p2c].d, ps.head, ps.tail,
                    grid_for(c, ps.n_ub, 4), c->s));
@@ -1045,6 +1094,10 @@ static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int
     a.pos = (double *)c->cols[pos].d;
     a.vel = (double *)c->cols[vel].d;
     a.p2c = (int32_t *)c->cols[p2c].d;
+    a.pos_out = a.pos;
+    a.vel_out = a.vel;
+    a.p2c_out = a.p2c;
+    a.dest = nullptr;
     a.cap = ps.cap;
     a.holes = ps.holes;
     a.work = ps.work;
@@ -1165,6 +1218,51 @@ static int read_stats(opp_ctx c, PSet &ps, opp_step_stats *stats) {
     return OPP_OK;
 }
 
+// Sort fused into the move (a sort step, opp_init_params.sort_every): the
+// counting sort's rank pass runs on the START cells before the move, and the
+// move writes every particle straight to its sorted position in the second
+// buffers (the columns it does not touch, e.g. ids, are scattered here); the
+// buffers are swapped after the move.  Saves the sort's separate read +
+// write of every particle (the auxiliary sort).
+static int fused_sort_prepass(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int p2c) {
+    MeshCache &m = c->mc;
+    TRY(ensure_alt(c, ps));
+    int jp = -1, jv = -1, jc = -1;
+    ColSet src{}, dst{};
+    for (size_t j = 0; j < ps.cols.size(); j++) {
+        const int h = ps.cols[j];
+        if (h == pos) jp = (int)j;
+        else if (h == vel) jv = (int)j;
+        else if (h == p2c) jc = (int)j;
+        else {
+            const Col &col = c->cols[h];
+            src.c[src.n] = ColDesc{col.d, ps.cap, col.eb, col.dim};
+            dst.c[dst.n] = ColDesc{ps.alt[j], ps.cap, col.eb, col.dim};
+            src.n++;
+            dst.n++;
+        }
+    }
+    if (jp < 0 || jv < 0 || jc < 0) return fail(OPP_ERR_STATE, "fused sort: columns not found");
+    const int32_t *pc = (const int32_t *)c->cols[p2c].d;
+    {
+        PhaseScope ph(c, OPP_PH_SORT_COUNT);
+        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_hist, m.cell_start,
+                             m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
+        CK(launch_sort_rank(pc, ps.dcnt, c->cell_base, m.sort_key, m.cell_start, ps.head, ps.tail,
+                            grid_for(c, ps.n_ub, c->sort_rgrid), c->s));
+    }
+    {
+        PhaseScope ph(c, OPP_PH_SORT_MOVE);
+        CK(launch_scatter_cols(src, dst, ps.head, ps.dcnt, grid_for(c, ps.n_ub, 8), c->s));
+    }
+    c->launches += 6;
+    a.pos_out = (double *)ps.alt[jp];
+    a.vel_out = (double *)ps.alt[jv];
+    a.p2c_out = (int32_t *)ps.alt[jc];
+    a.dest = ps.head;
+    return OPP_OK;
+}
+
 extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_dat vel,
                                      opp_map p2c, opp_map c2c, opp_map c2n, opp_dat node_pos,
                                      opp_dat cell_ef, opp_dat node_charge,
@@ -1195,6 +1293,10 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.pos = (double *)c->cols[pos].d;
     a.vel = (double *)c->cols[vel].d;
     a.p2c = (int32_t *)c->cols[p2c].d;
+    a.pos_out = a.pos;
+    a.vel_out = a.vel;
+    a.p2c_out = a.p2c;
+    a.dest = nullptr;
     a.cap = ps.cap;
     a.lines = m.lines;
     a.ef = m.efp;
@@ -1220,7 +1322,6 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.refill = c->refill;
     a.minb = c->minb;
     a.prefetch = c->prefetch;
-    a.pairs = c->pairs && c->p.direct_hop != 2;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const int dh = c->p.direct_hop;
@@ -1233,14 +1334,22 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     c->launches++;
     const bool tiled = c->p.tma_pipeline != 0;
-    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb, a.pairs != 0);
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb);
     const int bps = c->bps;
     const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
                                                                        (long long)c->nsm * bps));
+    const bool fuse = c->fuse_sort && c->p.sort_every > 0 && (ps.steps + 1) % c->p.sort_every == 0 &&
+                      m.cell_hist && !c->refill && !c->dbg;
+    if (fuse) TRY(fused_sort_prepass(c, ps, a, pos, vel, p2c));
     {
         PhaseScope ph(c, OPP_PH_PUSH_MOVE_DEPOSIT);
         const int g1 = tiled ? c->nsm * bps : pgrid;
         CK(launch_push_move_deposit(dep, dh, multi, false, tiled, a, g1, c->s));
+    }
+    if (fuse) {   // the sorted copies become the particle set
+        for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
+        refresh_args(c, ps, a, pos, vel, p2c);
+        ps.fused_sort = true;
     }
     {
         PhaseScope ph(c, OPP_PH_CONTINUE);

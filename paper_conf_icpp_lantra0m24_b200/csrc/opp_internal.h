@@ -69,8 +69,17 @@ struct Overlay {
     double dx;
     double inv_dx;        // 1.0 / dx, rounded once on the host
     int n[3];
-    int nb[3];            // bricks of 4x4x2 overlay cells (see ov_slot)
+    int nb[3];            // bricks of 4x4x2 overlay cells (see ov_slot32)
     const int32_t *map;   // nb[0]*nb[1]*nb[2]*32 slots, -1 = no tet / padding
+    // compact form (used when every 4x4x4 brick's tets lie within 32767 ids
+    // of the brick's lowest): one 128-B line of 64 int16 offsets per brick +
+    // an int32 base per brick -- twice the overlay cells per line, so the
+    // lookups of a warp (particles of one or two tets) touch about half the
+    // lines.  -32768 = no tet.
+    int compact;
+    int nbc[3];           // bricks of 4x4x4 overlay cells
+    const int16_t *off;   // nbc[0]*nbc[1]*nbc[2]*64
+    const int32_t *base;  // nbc[0]*nbc[1]*nbc[2]
 };
 
 struct StepArgs {
@@ -90,6 +99,14 @@ struct StepArgs {
     uint32_t *mig;             // migrants: particle index, target global cell, hops
     int32_t *mig_cell;
     int32_t *mig_hops;
+    // sort fused into the move (sort steps, opp_init_params.sort_every): the
+    // particle with index i is written to position dest[i] of the *_out
+    // columns (the sort's second buffers, counting-sorted by start cell) and
+    // recorded (holes, deferred walks, migrants) under that position.
+    // Otherwise dest == NULL and the *_out columns are the inputs (in place).
+    double *pos_out, *vel_out;
+    int32_t *p2c_out;
+    const uint32_t *dest;
     double c1, dt, w;
     int cell_base, n_cells;    // global id of local cell 0, local cell count
     int hpass, hcap;
@@ -97,7 +114,6 @@ struct StepArgs {
     int refill;                // tiled kernel: per-lane refill consumer (OPP_REFILL)
     int minb;                  // tiled kernel: min resident blocks per SM (OPP_MINB: 1 or 3)
     int prefetch;              // tiled kernel: producer-warp L1 warming (OPP_PREFETCH, default 1)
-    int pairs;                 // tiled kernel: two adjacent particles per lane (OPP_PAIRS; DH 0/1)
     int dbg;                   // diagnostics only (OPP_PMD_DEBUG): 1 stream, 2 +E, 3 +line, 4 no deposit
     Overlay ov;
 };

@@ -60,10 +60,29 @@ __device__ __forceinline__ void load_E(const double4 *__restrict__ ef, int lc, d
 // Overlay slot of overlay cell (ix, iy, iz): 4x4x2 bricks of 32 ints (one
 // 128-B line), so the particles of one tet -- a few overlay cells in every
 // direction -- touch a few lines instead of one line per (iy, iz) row.
-__device__ __forceinline__ long long ov_slot(const Overlay &ov, int ix, int iy, int iz) {
+__device__ __forceinline__ long long ov_slot32(const Overlay &ov, int ix, int iy, int iz) {
     const long long b = (long long)(ix >> 2) +
                         (long long)ov.nb[0] * ((long long)(iy >> 2) + (long long)ov.nb[1] * (iz >> 1));
     return b * 32 + (ix & 3) + 4 * (iy & 3) + 16 * (iz & 1);
+}
+
+__device__ __forceinline__ long long ov_slot16(const Overlay &ov, int ix, int iy, int iz) {
+    const unsigned b = (unsigned)(ix >> 2) +
+                       (unsigned)ov.nbc[0] * ((unsigned)(iy >> 2) + (unsigned)ov.nbc[1] * (unsigned)(iz >> 2));
+    return (long long)b * 64 + (ix & 3) + 4 * (iy & 3) + 16 * (iz & 3);
+}
+
+// Slot of overlay cell (ix, iy, iz) in the active layout, and its tet.
+__device__ __forceinline__ long long ov_slot(const Overlay &ov, int ix, int iy, int iz) {
+    return ov.compact ? ov_slot16(ov, ix, iy, iz) : ov_slot32(ov, ix, iy, iz);
+}
+__device__ __forceinline__ int ov_value(const Overlay &ov, long long slot) {
+    if (ov.compact) {   // the two loads are independent: one round trip
+        const int o = __ldg(ov.off + slot);
+        const int b = __ldg(ov.base + (slot >> 6));
+        return o == -32768 ? -1 : b + o;
+    }
+    return __ldg(ov.map + slot);
 }
 
 // Barycentric coordinates, node-relative form, fixed evaluation order.
@@ -294,7 +313,7 @@ __device__ __forceinline__ long long dh_slot(const Overlay &ov, double x, double
 __device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, double z, int cell) {
     const long long g = dh_slot(ov, x, y, z);
     if (g < 0) return cell;
-    int s = __ldg(ov.map + g);
+    int s = ov_value(ov, g);
     return s >= 0 ? s : cell;
 }
 
@@ -467,6 +486,8 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
     int4 cn = make_int4(0, 0, 0, 0);
+    // output position: i (in place), or dest[i] on a sort-fused step
+    const unsigned long long o = (!CONT && a.dest && valid) ? (unsigned long long)__ldg(a.dest + i) : i;
     if (valid && a.dbg == 1) {   // diagnostic: stream only
         vx = add(vx, a.c1); x = add(x, mul(vx, a.dt));
         a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
@@ -508,7 +529,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 if (DH == 1) {
                     spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
                                         add(z, mul(vz, a.dt)));
-                    spec_val = __ldg(a.ov.map + (spec_slot >= 0 ? spec_slot : 0));
+                    spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
                 }
                 load_E(a.ef, lc, Exy, Ez);
             }
@@ -524,8 +545,8 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 sout[sj] = x; sout[32 + sj] = y; sout[64 + sj] = z;
                 sout[96 + sj] = vx; sout[128 + sj] = vy; sout[160 + sj] = vz;
             } else {
-                a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-                a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+                a.pos_out[o] = x; a.pos_out[a.cap + o] = y; a.pos_out[2 * a.cap + o] = z;
+                a.vel_out[o] = vx; a.vel_out[a.cap + o] = vy; a.vel_out[2 * a.cap + o] = vz;
             }
             if (release) {
                 fence_proxy_async_fwd();   // generic reads before the async-proxy refill
@@ -534,7 +555,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             }
             if (DH == 1) {   // seed every particle from the overlay
                 const long long g = dh_slot(a.ov, x, y, z);
-                int v = g == spec_slot ? spec_val : (g >= 0 ? __ldg(a.ov.map + g) : -1);
+                int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
                 if (g < 0) v = -1;
                 int sc = v >= 0 ? v : cell;
                 if (sc != cell) {
@@ -570,20 +591,20 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
     if (ap) {
-        ring_push(ap->holes, rem, (uint32_t)i, 0);
+        ring_push(ap->holes, rem, (uint32_t)o, 0);
         ring_flush(ap->holes, &a.cnt->n_holes, a.holes, nullptr, false);
         if (!CONT) {
-            ring_push(ap->work, status == ST_MOVE, (uint32_t)i, hops);
+            ring_push(ap->work, status == ST_MOVE, (uint32_t)o, hops);
             ring_flush(ap->work, &a.cnt->n_work, a.work, a.work_hops, false);
         }
     } else {
         unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
-        if (rem) a.holes[hs] = (uint32_t)i;
+        if (rem) a.holes[hs] = (uint32_t)o;
         if (!CONT) {
             const bool mv = status == ST_MOVE;
             unsigned long long ws = warp_append(mv, &a.cnt->n_work);
             if (mv) {
-                a.work[ws] = (uint32_t)i;
+                a.work[ws] = (uint32_t)o;
                 a.work_hops[ws] = hops;
             }
         }
@@ -592,7 +613,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         const bool mg = status == ST_MIGRATE;
         unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
         if (mg) {
-            a.mig[ms] = (uint32_t)i;
+            a.mig[ms] = (uint32_t)o;
             a.mig_cell[ms] = cell;
             a.mig_hops[ms] = hops;
         }
@@ -647,7 +668,7 @@ __device__ __forceinline__ void pmd_direct_range(const StepArgs &a, unsigned lon
         if (more) load_pstate<CONT>(a, i0 + stride + lane_id(), hi, nxt);
         pmd_body<DEP, DH, CONT, MULTI>(a, cur.valid, cur.i, cur.hops, cur.x, cur.y, cur.z, cur.vx,
                                        cur.vy, cur.vz, cur.cell, t);
-        if (cur.valid) a.p2c[cur.i] = cur.cell;
+        if (cur.valid) a.p2c_out[(!CONT && a.dest) ? (unsigned long long)__ldg(a.dest + cur.i) : cur.i] = cur.cell;
         if (more) cur = nxt;
     }
 }
@@ -889,7 +910,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
                     if (DH == 1) {
                         nxt.slot = dh_slot(a.ov, add(x1, mul(vx1, a.dt)), add(y1, mul(vy1, a.dt)),
                                            add(z1, mul(vz1, a.dt)));
-                        nxt.val = __ldg(a.ov.map + (nxt.slot >= 0 ? nxt.slot : 0));
+                        nxt.val = ov_value(a.ov, nxt.slot >= 0 ? nxt.slot : 0);
                     }
                     load_E(a.ef, c1 - a.cell_base, nxt.Exy, nxt.Ez);
                     have_nxt = true;
@@ -920,6 +941,13 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             if (PRE) {
                 cur = nxt;
                 have_cur = have_nxt;
+            }
+            if (a.dest) {   // sort-fused step: each lane stores at its sorted position
+                const unsigned long long od = __ldg(a.dest + i);
+                a.pos_out[od] = x; a.pos_out[a.cap + od] = y; a.pos_out[2 * a.cap + od] = z;
+                a.vel_out[od] = vx; a.vel_out[a.cap + od] = vy; a.vel_out[2 * a.cap + od] = vz;
+                a.p2c_out[od] = cell;
+                continue;
             }
             reinterpret_cast<int *>(o + 192)[lane] = cell;
             fence_proxy_async();
@@ -1080,256 +1108,6 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             active = false;
         }
     }
-    flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
-}
-
-// ---------------------------------------------------------------------------
-// Pair-per-lane variant of the TMA-pipelined pass (StepArgs.pairs; DH 0 / 1).
-// Same producer warp and bulk-copy pipeline, but 4 consumer warps per tile,
-// each lane carrying two ADJACENT particles (2l, 2l+1 of its warp's 64).  In
-// cell-sorted storage the two usually share their start cell and their
-// final cell, so one E gather and one 128-B walk line serve both (the L1
-// data pipe that returns gathered bytes to registers is the busiest unit of
-// the one-per-lane kernel: every lane receives its own copy of the line),
-// their deposits merge in registers before the warp aggregation, and the
-// per-warp pipeline bookkeeping (barrier waits, fences, bulk stores, ring
-// flushes) is paid once per 64 particles.  Walks that leave the shared line
-// (hops, a different seed cell) take the general walk with their own loads.
-// ---------------------------------------------------------------------------
-constexpr int kPairWarps = kTile / 64;
-constexpr int kPairThreads = kPairWarps * 32 + 32;
-constexpr int kPairOutBytes = 64 * (6 * 8 + 4);
-constexpr int kPairOutBase = kStages * kStageBytes + 2 * kStages * 8;
-constexpr int kPairRingBase = kPairOutBase + kPairWarps * kPairOutBytes;
-constexpr int kPairSmem = kPairRingBase + kPairWarps * kRingBytesPerWarp;
-
-__device__ __forceinline__ bool inside4(double l0, double l1, double l2, double l3) {
-    return in01(l0) & in01(l1) & in01(l2) & in01(l3);
-}
-
-// Walk from `cell` (its line loaded here: an L1 hit in sorted storage).
-template <bool MULTI>
-__device__ __forceinline__ int walk_cell(const StepArgs &a, int &cell, double x, double y, double z,
-                                         int &hops, double &l0, double &l1, double &l2, double &l3,
-                                         int &capped, int4 &cn) {
-    Line L = load_line(a.lines, cell - a.cell_base);
-    return walk_from<MULTI>(a, cell, L, PosRegs{x, y, z}, hops, a.hpass, l0, l1, l2, l3, capped, cn);
-}
-
-__device__ __forceinline__ void tally(Tally &t, int st, int hops, int capped) {
-    if (st != ST_MOVE && st != ST_MIGRATE) {
-        t.hops += (unsigned)hops;
-        t.maxh = max(t.maxh, (unsigned)hops);
-        t.capped += (unsigned)capped;
-    }
-    t.removed += (st == ST_REMOVE);
-}
-
-// DH seed of a pushed position given the speculative lookup (see pmd_body).
-__device__ __forceinline__ int dh_seed_spec(const Overlay &ov, double x, double y, double z, int cell,
-                                            long long spec_slot, int spec_val) {
-    const long long g = dh_slot(ov, x, y, z);
-    int v = g == spec_slot ? spec_val : (g >= 0 ? __ldg(ov.map + g) : -1);
-    if (g < 0) v = -1;
-    return v >= 0 ? v : cell;
-}
-
-template <int DEP, int DH, bool MULTI>
-__device__ __forceinline__ void pair_body(const StepArgs &a, unsigned long long ia, double2 X,
-                                          double2 Y, double2 Z, double2 VX, double2 VY, double2 VZ,
-                                          int2 C, Tally &t, double *o, unsigned lane, Appends &ap) {
-    const unsigned FULL = 0xffffffffu;
-    const int ca = C.x, cb = C.y;
-    long long spa = -1, spb = -1;
-    int sva = -1, svb = -1;
-    if (DH == 1) {   // speculative overlay entries of the drift-only positions (see pmd_body)
-        spa = dh_slot(a.ov, add(X.x, mul(VX.x, a.dt)), add(Y.x, mul(VY.x, a.dt)), add(Z.x, mul(VZ.x, a.dt)));
-        spb = dh_slot(a.ov, add(X.y, mul(VX.y, a.dt)), add(Y.y, mul(VY.y, a.dt)), add(Z.y, mul(VZ.y, a.dt)));
-        sva = __ldg(a.ov.map + (spa >= 0 ? spa : 0));
-        svb = spb == spa ? sva : __ldg(a.ov.map + (spb >= 0 ? spb : 0));
-    }
-    // gather the cell-constant field (one load when the pair shares its cell), push
-    double2 Ea, Eb;
-    double Eaz, Ebz;
-    load_E(a.ef, ca - a.cell_base, Ea, Eaz);
-    if (cb != ca) {
-        load_E(a.ef, cb - a.cell_base, Eb, Ebz);
-    } else {
-        Eb = Ea;
-        Ebz = Eaz;
-    }
-    VX.x = add(VX.x, mul(a.c1, Ea.x)); VY.x = add(VY.x, mul(a.c1, Ea.y)); VZ.x = add(VZ.x, mul(a.c1, Eaz));
-    VX.y = add(VX.y, mul(a.c1, Eb.x)); VY.y = add(VY.y, mul(a.c1, Eb.y)); VZ.y = add(VZ.y, mul(a.c1, Ebz));
-    X.x = add(X.x, mul(VX.x, a.dt)); Y.x = add(Y.x, mul(VY.x, a.dt)); Z.x = add(Z.x, mul(VZ.x, a.dt));
-    X.y = add(X.y, mul(VX.y, a.dt)); Y.y = add(Y.y, mul(VY.y, a.dt)); Z.y = add(Z.y, mul(VZ.y, a.dt));
-    {
-        double2 *o2 = reinterpret_cast<double2 *>(o) + lane;   // column k: o + 64 k
-        o2[0] = X; o2[32] = Y; o2[64] = Z; o2[96] = VX; o2[128] = VY; o2[160] = VZ;
-    }
-    int sa = ca, sb = cb;
-    if (DH == 1) {
-        sa = dh_seed_spec(a.ov, X.x, Y.x, Z.x, ca, spa, sva);
-        sb = dh_seed_spec(a.ov, X.y, Y.y, Z.y, cb, spb, svb);
-    }
-    // the shared line: issued after the push (opaque dependency on z) so the
-    // line registers and the velocities are never live together
-    int zero;
-    asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}" : "=r"(zero) : "d"(Z.y));
-    int cellA = sa, cellB = sb;
-    double la0, la1, la2, la3, lb0 = 0, lb1 = 0, lb2 = 0, lb3 = 0;
-    int4 cna, cnb;
-    bool ina, inb = false;
-    const bool sameb = sb == sa;
-    {
-        const Line L = load_line(a.lines, sa - a.cell_base + zero);
-        bary(L, X.x, Y.x, Z.x, la0, la1, la2, la3);
-        ina = inside4(la0, la1, la2, la3);
-        cna = L.cn;
-        cnb = L.cn;
-        if (sameb) {
-            bary(L, X.y, Y.y, Z.y, lb0, lb1, lb2, lb3);
-            inb = inside4(lb0, lb1, lb2, lb3);
-        }
-    }
-    int hA = 0, hB = 0, capA = 0, capB = 0;
-    int stA = ST_DONE, stB = ST_DONE;
-    if (!ina) stA = walk_cell<MULTI>(a, cellA, X.x, Y.x, Z.x, hA, la0, la1, la2, la3, capA, cna);
-    if (!inb) stB = walk_cell<MULTI>(a, cellB, X.y, Y.y, Z.y, hB, lb0, lb1, lb2, lb3, capB, cnb);
-    tally(t, stA, hA, capA);
-    tally(t, stB, hB, capB);
-    // deposit (Eq. 10)
-    const bool dA = stA == ST_DONE, dB = stB == ST_DONE;
-    if (DEP == 2) {
-        sr_store(a, dA, cellA, a.w, la0, la1, la2, la3);
-        sr_store(a, dB, cellB, a.w, lb0, lb1, lb2, lb3);
-    } else {
-        double va0 = mul(a.w, la0), va1 = mul(a.w, la1), va2 = mul(a.w, la2), va3 = mul(a.w, la3);
-        const double vb0 = mul(a.w, lb0), vb1 = mul(a.w, lb1), vb2 = mul(a.w, lb2), vb3 = mul(a.w, lb3);
-        if (DEP == 0) {
-            if (dA) red4(a.Q, cna, va0, va1, va2, va3);
-            if (dB) red4(a.Q, cnb, vb0, vb1, vb2, vb3);
-        } else {
-            const bool merge = dA && dB && cellA == cellB;
-            if (merge) {
-                va0 = add(va0, vb0); va1 = add(va1, vb1); va2 = add(va2, vb2); va3 = add(va3, vb3);
-            }
-            const bool eA = dA || dB, eB = dA && dB && !merge;
-            // entry A: the merged pair, or whichever particle deposits
-            const bool useB = !dA && dB;
-            deposit_agg(a.Q, eA, useB ? cellB : cellA, useB ? cnb : cna, useB ? vb0 : va0,
-                        useB ? vb1 : va1, useB ? vb2 : va2, useB ? vb3 : va3);
-            if (__any_sync(FULL, eB)) deposit_agg(a.Q, eB, cellB, cnb, vb0, vb1, vb2, vb3);
-        }
-    }
-    // holes, deferred walks, migrants
-    const bool remA = stA == ST_REMOVE || stA == ST_MIGRATE;
-    const bool remB = stB == ST_REMOVE || stB == ST_MIGRATE;
-    ring_push(ap.holes, remA, (uint32_t)ia, 0);
-    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
-    ring_push(ap.holes, remB, (uint32_t)(ia + 1), 0);
-    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
-    ring_push(ap.work, stA == ST_MOVE, (uint32_t)ia, hA);
-    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
-    ring_push(ap.work, stB == ST_MOVE, (uint32_t)(ia + 1), hB);
-    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
-    if (MULTI) {
-        const bool mA = stA == ST_MIGRATE, mB = stB == ST_MIGRATE;
-        unsigned long long ms = warp_append(mA, &a.cnt->n_mig);
-        if (mA) { a.mig[ms] = (uint32_t)ia; a.mig_cell[ms] = cellA; a.mig_hops[ms] = hA; }
-        ms = warp_append(mB, &a.cnt->n_mig);
-        if (mB) { a.mig[ms] = (uint32_t)(ia + 1); a.mig_cell[ms] = cellB; a.mig_hops[ms] = hB; }
-    }
-    reinterpret_cast<int2 *>(o + 384)[lane] = make_int2(remA ? -1 : cellA, remB ? -1 : cellB);
-}
-
-#ifndef OPP_PAIR_MINB
-#define OPP_PAIR_MINB 4   // resident blocks per SM the pair kernel's registers are cut for
-#endif
-template <int DEP, int DH, bool MULTI>
-__global__ void __launch_bounds__(kPairThreads, OPP_PAIR_MINB) k_pmd_pairs(StepArgs a) {
-    extern __shared__ __align__(128) char smem[];
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
-    uint64_t *empty = full + kStages;
-    const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
-    const unsigned long long ntiles = n / kTile;
-    const TileMap tm{ntiles, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
-    const unsigned long long my = tm.count();
-    const int warp = threadIdx.x >> 5;
-    const unsigned lane = lane_id();
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < kStages; s++) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], kPairWarps);
-        }
-        fence_proxy_async();
-    }
-    __syncthreads();
-    if (warp == kPairWarps) {   // producer warp (lane 0): stream tiles kStages ahead
-        if (lane == 0) {
-            TileIter ti(tm);
-            for (unsigned long long it = 0; it < my; it++, ti.next()) {
-                const int s = (int)(it % kStages);
-                if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
-                issue_tile_load(a, smem, full, s, ti.tile());
-            }
-        }
-        return;
-    }
-    Appends ap;
-    {
-        char *rb = smem + kPairRingBase + (size_t)warp * kRingBytesPerWarp;
-        ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
-        ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
-                           reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
-    }
-    Tally t;
-    double *o = reinterpret_cast<double *>(smem + kPairOutBase + (size_t)warp * kPairOutBytes);
-    TileIter ti(tm);
-    for (unsigned long long it = 0; it < my; it++, ti.next()) {
-        const int s = (int)(it % kStages);
-        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
-        StageView v = stage_view(smem, s);
-        const int j = 64 * warp + 2 * (int)lane;
-        const double2 X = *reinterpret_cast<const double2 *>(v.c[0] + j);
-        const double2 Y = *reinterpret_cast<const double2 *>(v.c[1] + j);
-        const double2 Z = *reinterpret_cast<const double2 *>(v.c[2] + j);
-        const double2 VX = *reinterpret_cast<const double2 *>(v.c[3] + j);
-        const double2 VY = *reinterpret_cast<const double2 *>(v.c[4] + j);
-        const double2 VZ = *reinterpret_cast<const double2 *>(v.c[5] + j);
-        const int2 C = *reinterpret_cast<const int2 *>(v.cell + j);
-        unsigned long long h = 0;
-        h ^= (unsigned long long)__double_as_longlong(X.x) ^ (unsigned long long)__double_as_longlong(X.y);
-        h ^= (unsigned long long)__double_as_longlong(Y.x) ^ (unsigned long long)__double_as_longlong(Y.y);
-        h ^= (unsigned long long)__double_as_longlong(Z.x) ^ (unsigned long long)__double_as_longlong(Z.y);
-        h ^= (unsigned long long)__double_as_longlong(VX.x) ^ (unsigned long long)__double_as_longlong(VX.y);
-        h ^= (unsigned long long)__double_as_longlong(VY.x) ^ (unsigned long long)__double_as_longlong(VY.y);
-        h ^= (unsigned long long)__double_as_longlong(VZ.x) ^ (unsigned long long)__double_as_longlong(VZ.y);
-        h ^= (unsigned long long)(unsigned)C.x ^ (unsigned long long)(unsigned)C.y;
-        asm volatile("" ::"l"(h));   // the shared loads have landed
-        fence_proxy_async();
-        __syncwarp();
-        if (lane == 0) {
-            mbar_arrive(&empty[s]);
-            if (it >= 1) bulk_wait_read0();   // the previous stores have read the buffer
-        }
-        __syncwarp();
-        const unsigned long long tile = ti.tile();
-        pair_body<DEP, DH, MULTI>(a, tile * kTile + j, X, Y, Z, VX, VY, VZ, C, t, o, lane, ap);
-        fence_proxy_async();
-        __syncwarp();
-        if (lane == 0) {
-            const unsigned long long g0 = tile * kTile + 64 * warp;
-            for (int k = 0; k < 3; k++) {
-                bulk_s2g(a.pos + k * a.cap + g0, o + 64 * k, 512);
-                bulk_s2g(a.vel + k * a.cap + g0, o + 64 * (3 + k), 512);
-            }
-            bulk_s2g(a.p2c + g0, o + 384, 256);
-            bulk_commit();
-        }
-    }
-    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
-    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
-    if (lane == 0) bulk_wait_all();
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
@@ -1676,7 +1454,7 @@ __global__ void k_overlay_build(const WalkLine *__restrict__ lines, const double
                     double l0, l1, l2, l3;
                     bary(L, x, y, z, l0, l1, l2, l3);
                     if (l0 >= 0.0 && l1 >= 0.0 && l2 >= 0.0 && l3 >= 0.0)
-                        atomicMin(map + ov_slot(ov, gx, gy, gz), (int)c + cell_base);
+                        atomicMin(map + ov_slot32(ov, gx, gy, gz), (int)c + cell_base);
                 }
     }
 }
@@ -1886,7 +1664,10 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
         if (head && cell >= 0)
             base = atomicAdd(cursor + bucket_of(skey, cell - cell_base), (unsigned)rl);
         base = __shfl_sync(0xffffffffu, base, rs);
-        if (cell >= 0) src_of[base + (lane_id() - rs)] = (uint32_t)i;   // inverse permutation
+        if (cell >= 0) {
+            src_of[base + (lane_id() - rs)] = (uint32_t)i;   // inverse permutation
+            if (dest) dest[i] = base + (lane_id() - rs);      // forward (sort fused into the move)
+        }
     }
 }
 
@@ -1932,6 +1713,29 @@ __global__ void __launch_bounds__(256) k_sort_gather(ColSet src, ColSet dst,
 #pragma unroll
                     for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
                 }
+            }
+        }
+    }
+}
+
+// Sort-fused step: the columns the move does not write (ids, user dats)
+// follow their particles, dst[dest[i]] = src[i] for i < n.
+__global__ void __launch_bounds__(256) k_scatter_cols(ColSet src, ColSet dst,
+                                                      const uint32_t *__restrict__ dest,
+                                                      const DevCounters *c) {
+    const unsigned long long n = c->n;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+        const unsigned long long d = __ldg(dest + i);
+        for (int j = 0; j < src.n; j++) {
+            const ColDesc cs = src.c[j], cd = dst.c[j];
+            for (int e = 0; e < cs.dim; e++) {
+                if (cs.elem_bytes == 8)
+                    reinterpret_cast<long long *>(cd.ptr)[e * cd.cap + d] =
+                        __ldg(reinterpret_cast<const long long *>(cs.ptr) + e * cs.cap + i);
+                else
+                    reinterpret_cast<int *>(cd.ptr)[e * cd.cap + d] =
+                        __ldg(reinterpret_cast<const int *>(cs.ptr) + e * cs.cap + i);
             }
         }
     }
@@ -2086,6 +1890,20 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
     return scan_exclusive(hist, start, nc + 1, tile_sums, s);
 }
 
+cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
+                             unsigned *start, uint32_t *dest, uint32_t *src_of, int rank_grid,
+                             cudaStream_t s) {
+    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest, src_of);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_scatter_cols(const ColSet &src, const ColSet &dst, const uint32_t *dest,
+                                const DevCounters *c, int grid, cudaStream_t s) {
+    if (src.n == 0) return cudaSuccess;
+    k_scatter_cols<<<grid, 256, 0, s>>>(src, dst, dest, c);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
                              DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
                              unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
@@ -2093,7 +1911,7 @@ cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t
     // the scan left the total in start[nc]; the rank pass consumes start[] as
     // cursors but never touches start[nc].  One thread per particle: every
     // warp waits on its cursor atomics once, so the round trips overlap.
-    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest, src_of);
+    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, nullptr, src_of);
     // column passes: each pass moves a group of components so that the
     // source window it re-reads stays resident in L2 (OPP_SORT_PASSES)
     int nu = 0;
@@ -2149,25 +1967,8 @@ static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
                        : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
 }
 
-template <int DEP, int DH, bool MULTI>
-static cudaError_t launch_pairs(const StepArgs &a, int grid, cudaStream_t s) {
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_pmd_pairs<DEP, DH, MULTI>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kPairSmem);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
-    k_pmd_pairs<DEP, DH, MULTI><<<grid, kPairThreads, kPairSmem, s>>>(a);
-    k_push_move_deposit_tail<DEP, DH, MULTI><<<1, 256, 0, s>>>(a);
-    return cudaGetLastError();
-}
-
 template <int DEP, int DH, bool CONT, bool MULTI>
 static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
-    if (!CONT && tiled && a.pairs && DH != 2) {
-        return launch_pairs<DEP, DH == 2 ? 0 : DH, MULTI>(a, grid, s);
-    }
     if (!CONT && tiled) {
         return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
                         : launch_tiled<DEP, DH, MULTI, false>(a, grid, s);
@@ -2204,15 +2005,10 @@ cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, boo
                 : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
 }
 
-int pmd_blocks_per_sm(bool tiled, int minb, bool pairs) {
+int pmd_blocks_per_sm(bool tiled, int minb) {
     int nb = 0;
     cudaError_t e;
-    if (tiled && pairs) {
-        cudaFuncSetAttribute(k_pmd_pairs<0, 0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             kPairSmem);
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_pmd_pairs<0, 0, false>,
-                                                          kPairThreads, kPairSmem);
-    } else if (tiled) {
+    if (tiled) {
         if (minb >= 3) {
             cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
@@ -2302,6 +2098,46 @@ cudaError_t launch_pack_field(const double *ef, long long nc, double4 *out, cuda
     int grid = (int)((nc + 255) / 256);
     if (grid < 1) grid = 1;
     k_pack_field<<<grid, 256, 0, s>>>(ef, nc, out);
+    return cudaGetLastError();
+}
+
+// Compact overlay: per 4x4x4 brick, base = the lowest tet id, offsets int16;
+// *overflow set if some brick spans more than 32767 ids (then the int32 map
+// stays in use).
+__global__ void k_overlay_compact(const int32_t *__restrict__ map, Overlay ov, int16_t *off,
+                                  int32_t *base, unsigned *overflow) {
+    const long long nbt = (long long)ov.nbc[0] * ov.nbc[1] * ov.nbc[2];
+    for (long long b = (long long)blockIdx.x * blockDim.x + threadIdx.x; b < nbt;
+         b += (long long)gridDim.x * blockDim.x) {
+        const int bx = (int)(b % ov.nbc[0]), by = (int)((b / ov.nbc[0]) % ov.nbc[1]),
+                  bz = (int)(b / ((long long)ov.nbc[0] * ov.nbc[1]));
+        int v[64];
+        int lo = INT_MAX, hi = -1;
+        for (int e = 0; e < 64; e++) {
+            const int ix = 4 * bx + (e & 3), iy = 4 * by + ((e >> 2) & 3), iz = 4 * bz + (e >> 4);
+            int t = -1;
+            if (ix < ov.n[0] && iy < ov.n[1] && iz < ov.n[2]) t = map[ov_slot32(ov, ix, iy, iz)];
+            v[e] = t;
+            if (t >= 0) {
+                lo = min(lo, t);
+                hi = max(hi, t);
+            }
+        }
+        if (hi >= 0 && hi - lo > 32767) atomicOr(overflow, 1u);
+        const int bs = hi >= 0 ? lo : 0;
+        base[b] = bs;
+        for (int e = 0; e < 64; e++) off[b * 64 + e] = (int16_t)(v[e] >= 0 ? v[e] - bs : -32768);
+    }
+}
+
+cudaError_t launch_overlay_compact(const int32_t *map, const Overlay &ov, int16_t *off, int32_t *base,
+                                   unsigned *overflow, cudaStream_t s) {
+    const long long nbt = (long long)ov.nbc[0] * ov.nbc[1] * ov.nbc[2];
+    cudaError_t e = cudaMemsetAsync(overflow, 0, sizeof(unsigned), s);
+    if (e != cudaSuccess) return e;
+    long long g = (nbt + 127) / 128;
+    k_overlay_compact<<<(unsigned)(g > 0 ? (g < 65535 ? g : 65535) : 1), 128, 0, s>>>(map, ov, off, base,
+                                                                                  overflow);
     return cudaGetLastError();
 }
 

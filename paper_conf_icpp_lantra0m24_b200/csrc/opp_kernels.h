@@ -6,7 +6,7 @@ namespace opp {
 
 cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, bool tiled,
                                      const StepArgs &a, int grid, cudaStream_t s);
-int pmd_blocks_per_sm(bool tiled, int minb, bool pairs);
+int pmd_blocks_per_sm(bool tiled, int minb);
 cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero, int grid,
                               cudaStream_t s);
 cudaError_t launch_fill(const ColSet &cols, DevCounters *c, const uint32_t *holes,
@@ -19,6 +19,8 @@ cudaError_t launch_build_lines(const double *xyz, const int32_t *c2n, const int3
 cudaError_t launch_pack_field(const double *ef, long long nc, double4 *out, cudaStream_t s);
 cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long nc, int cell_base,
                            const Overlay &ov, int32_t *map, cudaStream_t s);
+cudaError_t launch_overlay_compact(const int32_t *map, const Overlay &ov, int16_t *off, int32_t *base,
+                                   unsigned *overflow, cudaStream_t s);
 cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *hist,
                       unsigned *start, unsigned long long *tile_sums, double *sorted,
                       double *cellsum, const int32_t *n2cs_ptr, const int32_t *n2cs, int grid,
@@ -30,6 +32,11 @@ cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
                               unsigned long long *tile_sums, int grid, cudaStream_t s);
+cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
+                             unsigned *start, uint32_t *dest, uint32_t *src_of, int rank_grid,
+                             cudaStream_t s);
+cudaError_t launch_scatter_cols(const ColSet &src, const ColSet &dst, const uint32_t *dest,
+                                const DevCounters *c, int grid, cudaStream_t s);
 cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
                              DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
                              unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
