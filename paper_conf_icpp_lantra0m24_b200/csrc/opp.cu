@@ -1586,9 +1586,9 @@ extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const in
     f.K.dval = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
     f.n2c_ptr = (int32_t *)c->dalloc(4 * (nn + 1));
     f.n2c = (int32_t *)c->dalloc(4 * std::max<long long>(4 * nc, 1));
-    f.vec = (double *)c->dalloc(8 * 5 * std::max<long long>(nn, 1));
+    f.vec = (double *)c->dalloc(8 * 9 * std::max<long long>(nn, 1));
     f.part_cap = (long long)c->nsm * 8;
-    f.part = (double *)c->dalloc(8 * 3 * f.part_cap);
+    f.part = (double *)c->dalloc(8 * 7 * f.part_cap);   // k_pcg: 1 + 2 x 3 partials per block
     f.st = (CgState *)c->dalloc(sizeof(CgState));
     f.own = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
     f.hvec = (double *)c->dalloc(8 * 3 * std::max<long long>(nn, 1));
@@ -1762,6 +1762,12 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     a.w = f.vec + 2 * nn;
     a.p = f.vec + 3 * nn;
     a.s = f.vec + 4 * nn;
+    a.m0 = f.vec + 5 * nn;
+    a.m1 = f.vec + 6 * nn;
+    a.z = f.vec + 7 * nn;
+    a.q = f.vec + 8 * nn;
+    a.pipelined = 1;
+    if (const char *e = getenv("OPP_CG_PIPE")) a.pipelined = atoi(e);
     a.part = f.part;
     a.st = f.st;
     a.rhs_scale = prm->rhs_scale;

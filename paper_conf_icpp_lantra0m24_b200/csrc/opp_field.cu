@@ -314,6 +314,140 @@ __global__ void __launch_bounds__(kCgThreads) k_cg(CgArgs a) {
     }
 }
 
+// Pipelined (P)CG (Ghysels & Vanroose): the three dot products of an
+// iteration are reduced while the SpMV of the next runs, so an iteration is
+// ONE phase -- SpMV n = K m, then the row-local recurrences -- and one grid
+// barrier.  m = M^-1 w is double-buffered by iteration parity (rows of m
+// are read by their neighbours' SpMV while their owners write the next m),
+// and so are the block partials.  Same stopping rule as k_cg.
+__global__ void __launch_bounds__(kCgThreads) k_pcg(CgArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ double sm[4 * kCgWarps];
+    const FieldMat &K = a.K;
+    const long long nn = K.nn;
+    const int lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long TW = ((long long)gridDim.x * blockDim.x) >> 5;
+    const int G = (int)gridDim.x;
+    double *part0 = a.part;                 // ||b_eff||^2 partials
+    double *partR[2] = {a.part + G, a.part + 4 * G};   // (r,u), (w,u), (r,r) by parity
+
+    for (long long sl = gw; sl < K.nslices; sl += TW) {
+        long long i = sl * kSell + lane;
+        if (i >= nn) continue;
+        a.x[i] = K.dmask[i] ? K.dval[i] : (a.warm ? a.x[i] : 0.0);
+    }
+    grid.sync();
+    {   // r0 = b - K x0, lifted rhs, u0 = M^-1 r0
+        double v[1] = {0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double ri = 0.0, bi = 0.0;
+            if (!K.dmask[i]) {
+                long long off = K.slice_off[sl];
+                int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+                double ax = 0.0, ad = 0.0;
+                for (int k = 0; k < W; k++) {
+                    long long q = off + (long long)kSell * k + lane;
+                    int c = K.col[q];
+                    double t = K.val[q] * __ldcg(a.x + c);
+                    ax += t;
+                    if (K.dmask[c]) ad += t;
+                }
+                double b = a.rhs_scale * a.Q[i];
+                ri = b - ax;
+                bi = b - ad;
+            }
+            a.r[i] = ri;
+            a.u[i] = a.precond ? ri * K.dinv[i] : ri;
+            a.p[i] = 0.0;
+            a.s[i] = 0.0;
+            a.q[i] = 0.0;
+            a.z[i] = 0.0;
+            v[0] += bi * bi;
+        }
+        block_publish<1>(v, part0, sm);
+    }
+    grid.sync();
+    {   // w0 = K u0, m0 = M^-1 w0, first dots
+        double v[3] = {0.0, 0.0, 0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double wi = sell_row(K, sl, lane, a.u);
+            double ri = a.r[i], ui = a.u[i];
+            a.w[i] = wi;
+            a.m0[i] = a.precond ? wi * K.dinv[i] : wi;
+            v[0] += ri * ui;
+            v[1] += wi * ui;
+            v[2] += ri * ri;
+        }
+        block_publish<3>(v, partR[0], sm);
+    }
+    grid.sync();
+    double rr0;
+    {
+        double t[1];
+        block_total<1>(part0, sm, t);
+        rr0 = t[0];
+    }
+    const double stop = a.tol * a.tol * rr0;
+    double gamma_old = 0.0, alpha = 0.0, beta = 0.0, rho = 0.0;
+    int it = 0;
+    for (;;) {
+        double t[3];
+        block_total<3>(partR[it & 1], sm, t);
+        const double gamma = t[0], delta = t[1];
+        rho = t[2];
+        if (rho <= stop || it >= a.max_iter) break;
+        if (it == 0) {
+            beta = 0.0;
+            alpha = gamma / delta;
+        } else {
+            beta = gamma / gamma_old;
+            alpha = gamma / (delta - beta * gamma / alpha);
+        }
+        gamma_old = gamma;
+        const double *mc = (it & 1) ? a.m1 : a.m0;
+        double *mn = (it & 1) ? a.m0 : a.m1;
+        double v[3] = {0.0, 0.0, 0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            const double ni = sell_row(K, sl, lane, mc);
+            const double zi = ni + beta * a.z[i];
+            const double qi = mc[i] + beta * a.q[i];
+            const double si = a.w[i] + beta * a.s[i];
+            const double pi = a.u[i] + beta * a.p[i];
+            a.z[i] = zi;
+            a.q[i] = qi;
+            a.s[i] = si;
+            a.p[i] = pi;
+            a.x[i] += alpha * pi;
+            const double ri = a.r[i] - alpha * si;
+            const double ui = a.u[i] - alpha * qi;
+            const double wi = a.w[i] - alpha * zi;
+            a.r[i] = ri;
+            a.u[i] = ui;
+            a.w[i] = wi;
+            mn[i] = a.precond ? wi * K.dinv[i] : wi;
+            v[0] += ri * ui;
+            v[1] += wi * ui;
+            v[2] += ri * ri;
+        }
+        block_publish<3>(v, partR[(it + 1) & 1], sm);
+        grid.sync();
+        it++;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.st->iterations = it;
+        a.st->converged = rho <= stop;
+        a.st->rr0 = rr0;
+        a.st->rr = rho;
+    }
+}
+
 __global__ void k_efield(const double *__restrict__ xyz, const int32_t *__restrict__ c2n,
                          const double *__restrict__ phi, long long nc, double *__restrict__ ef,
                          double4 *__restrict__ efp) {
@@ -343,7 +477,8 @@ cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const i
 
 cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out) {
     int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_cg, kCgThreads, 0);
+    const void *fn = a.pipelined ? (const void *)k_pcg : (const void *)k_cg;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kCgThreads, 0);
     if (e != cudaSuccess) return e;
     int bps = occ < max_bps ? occ : max_bps;
     if (bps < 1) return cudaErrorCooperativeLaunchTooLarge;
@@ -353,7 +488,7 @@ cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int
     if (want < grid) grid = (int)(want > 0 ? want : 1);
     CgArgs args = a;
     void *params[] = {&args};
-    e = cudaLaunchCooperativeKernel((const void *)k_cg, dim3(grid), dim3(kCgThreads), params, 0, s);
+    e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kCgThreads), params, 0, s);
     if (grid_out) *grid_out = grid;
     return e;
 }

@@ -40,11 +40,13 @@ struct CgArgs {
     const double *Q;     // node charge
     double *x;           // node potential (in: warm start, out: solution)
     double *r, *u, *w, *p, *s;   // work vectors [nn]
+    double *m0, *m1, *z, *q;     // pipelined CG (k_pcg): M^-1 w (two buffers), z, q
     double *part;        // [3 * grid] block partial sums
     CgState *st;
     double rhs_scale, tol;
     int max_iter, warm, precond;
     int dbg;             // diagnostics (OPP_CG_DBG): 1 = no SpMV in the loop, 2 = no grid barriers
+    int pipelined;       // 1: k_pcg (one grid barrier per iteration), 0: k_cg
 };
 
 // Per-row assembly from the node->cell CSR (deterministic order, no atomics).

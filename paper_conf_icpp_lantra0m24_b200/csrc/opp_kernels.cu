@@ -391,7 +391,15 @@ constexpr int kTiledThreads = kTile + 32;
 constexpr int kStages = OPP_STAGES;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
 constexpr int kRingBytesPerWarp = 64 * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
-constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8 + (kTile / 32) * 32 * (6 * 8 + 4);
+#ifndef OPP_TMA_OUT
+// 0: results leave as coalesced per-lane stores (C2: pmd 1.99 vs 2.06 ms --
+// staging the stores in shared memory cost L1 data-pipe wavefronts twice,
+// the shared stores and the bulk copy's reads); 1: per-warp shared buffer +
+// cp.async.bulk shared -> global
+#define OPP_TMA_OUT 0
+#endif
+constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8 +
+                          (OPP_TMA_OUT ? (kTile / 32) * 32 * (6 * 8 + 4) : 0);
 constexpr int kTiledSmem = kRingBase + (kTile / 32) * kRingBytesPerWarp;
 
 struct StageView {
@@ -541,7 +549,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             z = add(z, mul(vz, a.dt));
             // position and velocity are final now: store them before the walk
             // (TMA-out path: into the shared stage, bulk-stored by the warp)
-            if (SOUT) {   // per-warp output buffer: 6 columns of 32 doubles
+            if (SOUT && sout) {   // per-warp output buffer: 6 columns of 32 doubles
                 sout[sj] = x; sout[32 + sj] = y; sout[64 + sj] = z;
                 sout[96 + sj] = vx; sout[128 + sj] = vy; sout[160 + sj] = vz;
             } else {
@@ -828,6 +836,7 @@ __device__ __forceinline__ void warm_tile(const StepArgs &a, char *smem, uint64_
 template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
 __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
     constexpr bool PRE = OPP_PRE != 0;
+    constexpr bool TMA_OUT = OPP_TMA_OUT != 0;
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
     uint64_t *empty = full + kStages;
@@ -935,18 +944,18 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             const unsigned long long i = tile * kTile + j;
             double *o = reinterpret_cast<double *>(smem + kOutBase +
                                                    (size_t)(warp + ob_i) * kOutBytes);
+            // results leave through the shared buffer + bulk stores (TMA_OUT),
+            // or (sort-fused step / OPP_TMA_OUT=0) as coalesced per-lane stores
+            double *obuf = (TMA_OUT && !a.dest) ? o : nullptr;
             pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
-                                                  nullptr, o, (int)lane, &ap,
+                                                  nullptr, obuf, (int)lane, &ap,
                                                   (PRE && have_cur) ? &cur : nullptr);
             if (PRE) {
                 cur = nxt;
                 have_cur = have_nxt;
             }
-            if (a.dest) {   // sort-fused step: each lane stores at its sorted position
-                const unsigned long long od = __ldg(a.dest + i);
-                a.pos_out[od] = x; a.pos_out[a.cap + od] = y; a.pos_out[2 * a.cap + od] = z;
-                a.vel_out[od] = vx; a.vel_out[a.cap + od] = vy; a.vel_out[2 * a.cap + od] = vz;
-                a.p2c_out[od] = cell;
+            if (!obuf) {
+                a.p2c_out[a.dest ? (unsigned long long)__ldg(a.dest + i) : i] = cell;
                 continue;
             }
             reinterpret_cast<int *>(o + 192)[lane] = cell;
