@@ -32,8 +32,19 @@ struct Line {
     int4 cc, cn;
 };
 
-// One 128-B walk line in four 256-bit read-only loads (LDG.E.256 on sm_100:
-// half the L1 wavefronts of 16-B vector loads).
+#ifndef OPP_LAZY_LINE
+// 1: a visit loads only the 96 B lambda needs (gradients, p0: three 256-bit
+// loads); the neighbour ids (c2c) are loaded by the lanes that hop and the
+// node ids (c2n) by the lanes that issue the deposit reductions.  An L1 load
+// costs ~8 SM cycles per 256-bit warp instruction and distinct line even for
+// one active lane (scripts/micro/wf_cost.cu), so the fourth sector of every
+// visit was a quarter of the walk's L1 data-pipe time.
+#define OPP_LAZY_LINE 1
+#endif
+constexpr bool kLazyLine = OPP_LAZY_LINE != 0;
+
+// One 128-B walk line: four 256-bit read-only loads (LDG.E.256), or the first
+// three (lazy: the c2c / c2n sector is read on demand, below).
 __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, int c) {
     const double *L = reinterpret_cast<const double *>(lines + c);
     Line l;
@@ -43,10 +54,27 @@ __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, in
         : "=d"(l.g4), "=d"(l.g5), "=d"(l.g6), "=d"(l.g7) : "l"(L + 4));
     asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
         : "=d"(l.g8), "=d"(l.px), "=d"(l.py), "=d"(l.pz) : "l"(L + 8));
-    asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-        : "=r"(l.cc.x), "=r"(l.cc.y), "=r"(l.cc.z), "=r"(l.cc.w),
-          "=r"(l.cn.x), "=r"(l.cn.y), "=r"(l.cn.z), "=r"(l.cn.w) : "l"(L + 12));
+    if (!kLazyLine) {
+        asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+            : "=r"(l.cc.x), "=r"(l.cc.y), "=r"(l.cc.z), "=r"(l.cc.w),
+              "=r"(l.cn.x), "=r"(l.cn.y), "=r"(l.cn.z), "=r"(l.cn.w) : "l"(L + 12));
+    }
     return l;
+}
+
+// c2c of local cell c (walk line bytes 96..111) and c2n (112..127).
+__device__ __forceinline__ int4 line_c2c(const WalkLine *__restrict__ lines, int c) {
+    return __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(lines + c) + 12));
+}
+__device__ __forceinline__ int4 line_c2n(const WalkLine *__restrict__ lines, int c) {
+    return __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(lines + c) + 14));
+}
+__device__ __forceinline__ int line_node(const WalkLine *__restrict__ lines, int c, int q) {
+    return __ldg(reinterpret_cast<const int *>(reinterpret_cast<const double *>(lines + c) + 14) + q);
+}
+// the neighbours of the cell whose line L is (lc: its local index)
+__device__ __forceinline__ int4 cc_of(const WalkLine *__restrict__ lines, const Line &L, int lc) {
+    return kLazyLine ? line_c2c(lines, lc) : L.cc;
 }
 
 // Cell field E (double4, 32-B aligned) in one 256-bit read-only load.
@@ -134,11 +162,12 @@ __device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, c
             return ST_DONE;
         }
         if (hops >= stop_at) return ST_MOVE;
-        int nb = L.cc.x;
+        const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
+        int nb = cc.x;
         double m = l0;
-        if (l1 < m) { m = l1; nb = L.cc.y; }
-        if (l2 < m) { m = l2; nb = L.cc.z; }
-        if (l3 < m) { nb = L.cc.w; }
+        if (l1 < m) { m = l1; nb = cc.y; }
+        if (l2 < m) { m = l2; nb = cc.z; }
+        if (l3 < m) { nb = cc.w; }
         if (nb < 0) return ST_REMOVE;
         if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
             cell = nb;       // the hop into the other rank's cell counts here
@@ -181,6 +210,20 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 // (lowest lane issues the 4 reductions) is cheaper.
 constexpr int kMaxRsGroups = 3;
 
+// Node ids of the depositing cell: from the walk line already in registers,
+// or (lazy line) loaded by the lanes that issue the reductions only.
+struct CnSrc {
+    const WalkLine *lines;
+    int base;   // cell_base: key - base is the local cell
+    __device__ __forceinline__ int4 get(int key, int4 cn) const {
+        return kLazyLine ? line_c2n(lines, key - base) : cn;
+    }
+    __device__ __forceinline__ int node(int key, int4 cn, int q) const {
+        if (kLazyLine) return line_node(lines, key - base, q);
+        return q == 0 ? cn.x : q == 1 ? cn.y : q == 2 ? cn.z : cn.w;
+    }
+};
+
 __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0, double v1,
                                      double v2, double v3) {
     atomicAdd(Q + cn.x, v0);
@@ -191,12 +234,15 @@ __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0,
 
 // Log-step tree over every peer group of the lanes with `act` set.
 __device__ __forceinline__ void deposit_tree(double *__restrict__ Q, bool act, unsigned peers,
-                                             int4 cn, double v0, double v1, double v2, double v3) {
+                                             const CnSrc &cs, int key, int4 cn, double v0,
+                                             double v1, double v2, double v3) {
     const unsigned lane = lane_id();
     const int first = __ffs(peers) - 1;
     int rel = __popc(peers & ((1u << lane) - 1u));       // my rank inside the group
     unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
     if (lane == 31) up = 0;
+    // the lowest lane of each group fetches the node ids while the tree runs
+    if (act && (int)lane == first) cn = cs.get(key, cn);
     while (__any_sync(0xffffffffu, up != 0)) {
         const int next = up ? __ffs(up) - 1 : (int)lane;
         const double t0 = __shfl_sync(0xffffffffu, v0, next);
@@ -216,17 +262,18 @@ __device__ __forceinline__ void deposit_tree(double *__restrict__ Q, bool act, u
 
 // Warp-aggregated deposit of (key, cn, v0..v3) for the lanes with `done`
 // (key: the cell; lanes with equal keys have equal cn).
-__device__ __forceinline__ void deposit_agg(double *__restrict__ Q, bool done, int key, int4 cn,
-                                            double v0, double v1, double v2, double v3) {
+__device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const CnSrc &cs, bool done,
+                                            int key, int4 cn, double v0, double v1, double v2,
+                                            double v3) {
     const unsigned FULL = 0xffffffffu;
     const unsigned lane = lane_id();
     const unsigned peers = __match_any_sync(FULL, done ? key : -2 - (int)lane);
     const bool single = peers == (1u << lane);
-    if (done && single) red4(Q, cn, v0, v1, v2, v3);
+    if (done && single) red4(Q, cs.get(key, cn), v0, v1, v2, v3);
     unsigned lead = __ballot_sync(FULL, done && !single && (int)lane == __ffs(peers) - 1);
     if (!lead) return;
     if (__popc(lead) > kMaxRsGroups) {
-        deposit_tree(Q, done && !single, peers, cn, v0, v1, v2, v3);
+        deposit_tree(Q, done && !single, peers, cs, key, cn, v0, v1, v2, v3);
         return;
     }
     const bool h16 = (lane & 16u) != 0, h8 = (lane & 8u) != 0;
@@ -246,24 +293,31 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, bool done, i
         t = add(t, __shfl_xor_sync(FULL, t, 2));
         t = add(t, __shfl_xor_sync(FULL, t, 1));
         // lane 8q holds the sum of value q = 2*h16 + h8
-        const int n0 = __shfl_sync(FULL, cn.x, L), n1 = __shfl_sync(FULL, cn.y, L);
-        const int n2 = __shfl_sync(FULL, cn.z, L), n3 = __shfl_sync(FULL, cn.w, L);
-        if ((lane & 7u) == 0) {
-            const int node = h16 ? (h8 ? n3 : n2) : (h8 ? n1 : n0);
-            atomicAdd(Q + node, t);
+        const int q = 2 * (int)h16 + (int)h8;
+        if (kLazyLine) {
+            const int kL = __shfl_sync(FULL, key, L);
+            if ((lane & 7u) == 0) atomicAdd(Q + cs.node(kL, cn, q), t);
+        } else {
+            const int n0 = __shfl_sync(FULL, cn.x, L), n1 = __shfl_sync(FULL, cn.y, L);
+            const int n2 = __shfl_sync(FULL, cn.z, L), n3 = __shfl_sync(FULL, cn.w, L);
+            if ((lane & 7u) == 0) {
+                const int node = h16 ? (h8 ? n3 : n2) : (h8 ? n1 : n0);
+                atomicAdd(Q + node, t);
+            }
         }
     } while (lead);
 }
 
 template <int DEP>
-__device__ __forceinline__ void deposit(double *__restrict__ Q, bool done, int cell, int4 cn,
-                                        double w, double l0, double l1, double l2, double l3) {
+__device__ __forceinline__ void deposit(double *__restrict__ Q, const CnSrc &cs, bool done,
+                                        int cell, int4 cn, double w, double l0, double l1,
+                                        double l2, double l3) {
     double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
     if (DEP == 0) {
-        if (done) red4(Q, cn, v0, v1, v2, v3);
+        if (done) red4(Q, cs.get(cell, cn), v0, v1, v2, v3);
         return;
     }
-    deposit_agg(Q, done, cell, cn, v0, v1, v2, v3);
+    deposit_agg(Q, cs, done, cell, cn, v0, v1, v2, v3);
 }
 
 // SR deposit, phase 1: store (cell, w*lambda[4]) records.
@@ -594,7 +648,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     if (DEP == 2) {
         sr_store(a, done, cell, a.w, l0, l1, l2, l3);
     } else {
-        deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
     }
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
@@ -1066,11 +1120,12 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             } else if (hops >= a.hpass) {
                 status = ST_MOVE;
             } else {
-                int nb = L.cc.x;
+                const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
+                int nb = cc.x;
                 double m = l0;
-                if (l1 < m) { m = l1; nb = L.cc.y; }
-                if (l2 < m) { m = l2; nb = L.cc.z; }
-                if (l3 < m) { nb = L.cc.w; }
+                if (l1 < m) { m = l1; nb = cc.y; }
+                if (l2 < m) { m = l2; nb = cc.z; }
+                if (l3 < m) { nb = cc.w; }
                 if (nb < 0) {
                     status = ST_REMOVE;
                 } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
@@ -1093,7 +1148,7 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
         t.removed += (status == ST_REMOVE);
         const bool done = status == ST_DONE;
         if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-        else deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        else deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
         const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
         unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
         if (rem) a.holes[hs] = (uint32_t)i;
@@ -1213,11 +1268,12 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
                 status = ST_DONE;
                 capped = 1;
             } else {
-                int nb = L.cc.x;
+                const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
+                int nb = cc.x;
                 double m = l0;
-                if (l1 < m) { m = l1; nb = L.cc.y; }
-                if (l2 < m) { m = l2; nb = L.cc.z; }
-                if (l3 < m) { nb = L.cc.w; }
+                if (l1 < m) { m = l1; nb = cc.y; }
+                if (l2 < m) { m = l2; nb = cc.z; }
+                if (l3 < m) { nb = cc.w; }
                 if (nb < 0) {
                     status = ST_REMOVE;
                 } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
@@ -1240,7 +1296,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
         t.removed += (status == ST_REMOVE);
         const bool done = status == ST_DONE;
         if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-        else deposit<DEP>(a.Q, done, cell, cn, a.w, l0, l1, l2, l3);
+        else deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
         const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
         ring_push(hr, rem, (uint32_t)i, 0);
         ring_flush(hr, &a.cnt->n_holes, a.holes, nullptr, false);
@@ -1438,8 +1494,9 @@ __global__ void k_overlay_build(const WalkLine *__restrict__ lines, const double
                                 long long nc, int cell_base, Overlay ov, int32_t *map) {
     for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
          c += (long long)gridDim.x * blockDim.x) {
-        Line L = load_line(lines, (int)c);
-        int nodes[4] = {L.cn.x, L.cn.y, L.cn.z, L.cn.w};
+        const Line L = load_line(lines, (int)c);
+        const int4 cn = line_c2n(lines, (int)c);
+        int nodes[4] = {cn.x, cn.y, cn.z, cn.w};
         double lo[3], hi[3];
         for (int k = 0; k < 3; k++) {
             lo[k] = hi[k] = xyz[3 * (long long)nodes[0] + k];
