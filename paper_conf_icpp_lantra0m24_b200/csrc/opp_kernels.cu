@@ -77,9 +77,19 @@ __device__ __forceinline__ int4 cc_of(const WalkLine *__restrict__ lines, const 
     return kLazyLine ? line_c2c(lines, lc) : L.cc;
 }
 
-// Cell field E (double4, 32-B aligned) in one 256-bit read-only load.
+// Cell field E (double4, 32-B aligned): one 256-bit read-only load, or
+// (OPP_E_NARROW) a 128-bit + a 64-bit load of just the 24 B used.
+#ifndef OPP_E_NARROW
+#define OPP_E_NARROW 0
+#endif
 __device__ __forceinline__ void load_E(const double4 *__restrict__ ef, int lc, double2 &exy,
                                        double &ez) {
+    if (OPP_E_NARROW) {
+        const double *p = reinterpret_cast<const double *>(ef + lc);
+        exy = __ldg(reinterpret_cast<const double2 *>(p));
+        ez = __ldg(p + 2);
+        return;
+    }
     double pad;
     asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
         : "=d"(exy.x), "=d"(exy.y), "=d"(ez), "=d"(pad) : "l"(ef + lc));
@@ -208,7 +218,10 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 // lanes 0, 8, 16, 24 then hold the group's 4 sums and issue one reduction
 // each.  With more than kMaxRsGroups groups a log-step tree over each group
 // (lowest lane issues the 4 reductions) is cheaper.
-constexpr int kMaxRsGroups = 3;
+#ifndef OPP_RS_GROUPS
+#define OPP_RS_GROUPS 0   // C2: 0 (always the tree) 1.894 ms, 3: 1.912, 8: 2.35
+#endif
+constexpr int kMaxRsGroups = OPP_RS_GROUPS;
 
 // Node ids of the depositing cell: from the walk line already in registers,
 // or (lazy line) loaded by the lanes that issue the reductions only.
