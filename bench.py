@@ -42,7 +42,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c2", "c5", "c1"])
+    ap.add_argument("--config", default="c2", choices=["c2", "c5", "c1", "c3"])
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
@@ -63,6 +63,7 @@ def parse():
     ap.add_argument("--rhs", type=float, default=2e-7, help="field solve: b = rhs * node charge")
     ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
     ap.add_argument("--cg-tol", type=float, default=1e-10)
+    ap.add_argument("--ppc", type=int, default=750, help="c3: particles per cell (750 = 72M, 1500 = 144M)")
     args = ap.parse_args()
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
     if args.field < 0:
@@ -208,6 +209,168 @@ def run_reference(args, rank, world):
                              "sample": sample},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- config C3
+C3 = dict(dims=(40, 40, 60), seed=20240814, v0=0.2, pert=0.01, vth=0.01, qdt_2mc=0.05,
+          cdt_2h=(1.0, 1.0, 1.0), e_amp=1e-2, b0=0.5, b_amp=1e-2, kcap=16)
+C3_NAME = ("C3 CabanaPIC-style two-stream: 40x40x60 periodic hex (96,000 cells) declared through "
+           "c2c, {ppc} particles/cell, Boris push + face-crossing move + Eq. 11 current deposit "
+           "(Move_Deposit), fixed fields")
+
+
+def c3_inputs(args):
+    import gen.em as ge
+    nx, ny, nz = C3["dims"]
+    e, b = ge.em_fields(nx, ny, nz, C3["seed"], e_amp=C3["e_amp"], b0=C3["b0"], b_amp=C3["b_amp"])
+    return nx, ny, nz, ge.periodic_hex(nx, ny, nz), e, b
+
+
+def run_reference_c3(args, rank, world):
+    if rank != 0:
+        return
+    import gen.em as ge
+    import oracle.em as OE
+    nx, ny, nz, c2c, e, b = c3_inputs(args)
+    interp = OE.interpolate(nx, ny, nz, e, b)
+    # bounded sample: the first `ppc_s` particles of every cell of a z-range
+    ppc_s = 16
+    p = ge.two_stream(nx, ny, nz, ppc_s, C3["seed"], v0=C3["v0"], pert=C3["pert"], vth=C3["vth"])
+    prm = OE.params(C3["qdt_2mc"], C3["cdt_2h"], 1.0, C3["kcap"])
+    acc = np.zeros((nx * ny * nz, 12))
+    off, u, w, cell = p["off"], p["u"], p["w"], p["cell"]
+    OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)   # warm-up step
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)
+    secs = time.perf_counter() - t0
+    v = p["n"] * args.steps / secs
+    sample = f"{p['n']:,} particles ({ppc_s}/cell) of the C3 workload, {args.steps} steps, 1 thread"
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / max(args.steps, 1),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": C3_NAME.format(ppc=args.ppc), "sample": sample},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_ours_c3(args, rank, world):
+    """C3: one step = Move_Deposit over the whole resident population (the
+    accumulator is zeroed between steps outside the timed kernel's model).
+    N > 1: independent replicas (the periodic two-stream box is not
+    partitioned in this round: DESIGN.md §10)."""
+    import torch
+    import gen.cuda as gc
+    from paper_conf_icpp_lantra0m24_b200.em_app import CabanaPicEM
+    from paper_conf_icpp_lantra0m24_b200 import dist as D
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(dev)
+    nx, ny, nz, c2c, e, b = c3_inputs(args)
+    nc = nx * ny * nz
+    sim = CabanaPicEM(nx, ny, nz, c2c, e, b, C3["qdt_2mc"], C3["cdt_2h"], 1.0, C3["kcap"],
+                      deposit_mode=1 if args.deposit != 0 else 0, device=dev)
+    d = gc.em_two_stream(nx, ny, nz, args.ppc, C3["seed"] + rank, v0=C3["v0"], pert=C3["pert"],
+                         vth=C3["vth"])
+    sim.set_particles(d["off"], d["u"], d["w"], d["cell"])
+    del d
+    n = sim.n
+    stream = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        sim.step()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    l0 = sim.launches()
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    O.opp_phase_timing(sim.ctx, True)
+    O.opp_get_phase_times(sim.ctx)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(dev) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            sim.step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    launches = sim.launches() - l0
+    ph = O.opp_get_phase_times(sim.ctx)
+    O.opp_phase_timing(sim.ctx, False)
+    st = sim.step(want_stats=True)
+    pushed = n * args.steps
+    if world > 1:
+        ms = D.max_over_ranks(ms)
+        pushed = D.sum_over_ranks(pushed)
+        launches = D.sum_over_ranks(launches)
+    value = pushed / (ms / 1e3)
+    peak, peak_src = load_peaks()
+    k_ms, k_cnt = ph["em_move_deposit"]
+    # algorithmic bytes per launch: particle state in (off, u, w, cell = 60 B) and
+    # out (off, u, cell = 52 B); per cell the interpolator (144 B), c2c (24 B)
+    # and the accumulator read-modify-write (2 x 96 B)
+    bpl = 112.0 * n + (144.0 + 24.0 + 192.0) * nc
+    achieved = bpl / (k_ms / max(k_cnt, 1) / 1e3) / 1e9
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": C3_NAME.format(ppc=args.ppc), "mesh_cells": nc, "particles": n,
+                   "ppc": args.ppc, "deposit": "atomic_warpagg" if args.deposit != 0 else "atomic",
+                   "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n * 60 / 1e9),
+                   "parallelism": f"replicas{world}" if world > 1 else "single"},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": None, "kernel": "k_em_move_deposit",
+                     "bytes_model": "112 B/particle + 360 B/cell per launch", "peak_source": peak_src},
+        "gpu_launches": launches,
+        "phases_ms_per_step": {k: v[0] / args.steps for k, v in ph.items() if v[1]},
+        "move": {"crossings_per_particle": st["n_crossings"] / max(n, 1),
+                 "max_crossings": st["max_crossings"], "capped": st["n_capped"]},
+        "clocks": clk.summary(),
+    }
+    if not args.no_e2e:
+        # e2e through the public API: the step's fields arrive from pinned host
+        # memory (H2D), Interpolate + Move_Deposit run, the accumulator is read back
+        ke = args.e2e_steps or min(args.steps, 10)
+        eh = torch.from_numpy(e).pin_memory()
+        bh = torch.from_numpy(b).pin_memory()
+        acc_h = torch.empty((nc, 12), dtype=torch.float64).pin_memory()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(ke):
+            sim.e.copy_(eh, non_blocking=True)
+            sim.b.copy_(bh, non_blocking=True)
+            sim.interpolate()
+            sim.step()
+            acc_h.copy_(sim.acc, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        ep = n * ke
+        if world > 1:
+            ems = D.max_over_ranks(ems)
+            ep = D.sum_over_ranks(ep)
+        line["e2e"] = {"value": ep / (ems / 1e3), "unit": UNIT,
+                       "h2d_bytes_per_step": int(e.nbytes + b.nbytes), "d2h_bytes_per_step": nc * 96,
+                       "steps": ke, "note": "edge E and face B from pinned host memory every step, "
+                       "opp_em_interpolate + opp_em_move_deposit, accumulator read back"}
+    if not args.no_cpu and world == 1 and rank == 0:
+        import gen.em as ge
+        import oracle.em as OE
+        interp = OE.interpolate(nx, ny, nz, e, b)
+        p = ge.two_stream(nx, ny, nz, 16, C3["seed"], v0=C3["v0"], pert=C3["pert"], vth=C3["vth"])
+        acc = np.zeros((nc, 12))
+        prm = OE.params(C3["qdt_2mc"], C3["cdt_2h"], 1.0, C3["kcap"])
+        t0 = time.perf_counter()
+        for _ in range(2):
+            OE.move_deposit(prm, p["off"], p["u"], p["w"], p["cell"], interp, c2c, acc)
+        secs = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": 2 * p["n"] / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": f"{p['n']:,} particles (16/cell) of the C3 workload, 2 steps, "
+                                          f"1 thread, {secs:.1f} s"}
+    sim.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------- our arm
@@ -441,7 +604,9 @@ def main():
             dist.init_process_group("nccl")
         else:
             dist.init_process_group("gloo")
-    if args.impl == "reference":
+    if args.config == "c3":
+        (run_reference_c3 if args.impl == "reference" else run_ours_c3)(args, rank, world)
+    elif args.impl == "reference":
         run_reference(args, rank, world)
     else:
         run_ours(args, rank, world)

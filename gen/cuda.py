@@ -32,6 +32,8 @@ def lib():
         P, L, U, D = C.c_void_p, C.c_longlong, C.c_ulonglong, C.c_double
         _lib.gen_seed_particles.argtypes = [P, P, L, L, U, D, D, L, P, L, D, P, P, P, P, P]
         _lib.gen_inject_batch.argtypes = [P, P, L, L, L, U, D, L, P, P, P, P, P]
+        I = C.c_int
+        _lib.gen_em_two_stream.argtypes = [I, I, I, I, U, D, D, D, P, P, P, P, P, P]
     return _lib
 
 
@@ -86,4 +88,26 @@ def inject_batch(dm: DeviceMesh, step: int, n_inj: int, seed: int, v_inj=0.25, i
                                 o["cell"].data_ptr(), o["id"].data_ptr(), s)
     if rc:
         raise RuntimeError(f"gen_inject_batch: cuda error {rc}")
+    return o
+
+
+def em_two_stream(nx: int, ny: int, nz: int, ppc: int, seed: int, v0: float = 0.2,
+                  pert: float = 0.01, vth: float = 0.01, w: float = 1.0, device="cuda",
+                  stream=None) -> dict:
+    """Device twin of gen.em.two_stream (SoA torch tensors off[3][n], u[3][n], w, cell)."""
+    import torch
+    from .em import pert_table
+    n = nx * ny * nz * ppc
+    tab = torch.from_numpy(pert_table(nz, v0, pert)).to(device)
+    o = {"off": torch.empty((3, n), dtype=torch.float64, device=device),
+         "u": torch.empty((3, n), dtype=torch.float64, device=device),
+         "w": torch.empty(n, dtype=torch.float64, device=device),
+         "cell": torch.empty(n, dtype=torch.int32, device=device), "n": n}
+    s = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+    rc = lib().gen_em_two_stream(nx, ny, nz, ppc, seed, v0, vth, w, tab.data_ptr(),
+                                 o["off"].data_ptr(), o["u"].data_ptr(), o["w"].data_ptr(),
+                                 o["cell"].data_ptr(), s)
+    if rc:
+        raise RuntimeError(f"gen_em_two_stream: cuda error {rc}")
+    o["_keep"] = tab
     return o

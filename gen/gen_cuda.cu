@@ -113,6 +113,31 @@ Keys keys(unsigned long long seed) {
     return Keys{key_of(seed, 0), key_of(seed, 1), key_of(seed, 2), key_of(seed, 3), key_of(seed, 4)};
 }
 
+// Two-stream population of gen.em.two_stream (config C3): particle p in cell
+// p / ppc, offsets 2 u - 1, beams +-v0 along z (even / odd p) plus the
+// per-plane perturbation table, thermal spread vth (2 u - 1).  SoA outputs.
+__global__ void k_em_two_stream(long long n, int ppc, long long nxy, unsigned long long ko0,
+                                unsigned long long ko1, unsigned long long ko2,
+                                unsigned long long ku0, unsigned long long ku1,
+                                unsigned long long ku2, double v0, double vth, double w,
+                                const double *__restrict__ tab, double *off, double *u,
+                                double *wout, int *cell) {
+    for (long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x; p < n;
+         p += (long long)gridDim.x * blockDim.x) {
+        const long long c = p / ppc;
+        const unsigned long long i = (unsigned long long)p;
+        off[p] = ds(dm(2.0, u01(ko0, i)), 1.0);
+        off[n + p] = ds(dm(2.0, u01(ko1, i)), 1.0);
+        off[2 * n + p] = ds(dm(2.0, u01(ko2, i)), 1.0);
+        const double sgn = (p % 2 == 0) ? 1.0 : -1.0;
+        u[p] = dm(vth, ds(dm(2.0, u01(ku0, i)), 1.0));
+        u[n + p] = dm(vth, ds(dm(2.0, u01(ku1, i)), 1.0));
+        u[2 * n + p] = da(da(dm(sgn, v0), tab[c / nxy]), dm(vth, ds(dm(2.0, u01(ku2, i)), 1.0)));
+        wout[p] = w;
+        cell[p] = (int)c;
+    }
+}
+
 }  // namespace
 
 extern "C" int gen_seed_particles(const double *xyz, const int *c2n, long long nc, long long n,
@@ -137,5 +162,18 @@ extern "C" int gen_inject_batch(const double *xyz, const long long *inlet, long 
     if (g > 148 * 16) g = 148 * 16;
     k_inject<<<(int)g, 256, 0, (cudaStream_t)stream>>>(xyz, inlet, nf, step, n_inj, keys(seed),
                                                        v_inj, id_base, pos, vel, cell, id);
+    return (int)cudaGetLastError();
+}
+
+extern "C" int gen_em_two_stream(int nx, int ny, int nz, int ppc, unsigned long long seed,
+                                 double v0, double vth, double w, const double *tab, double *off,
+                                 double *u, double *wout, int *cell, void *stream) {
+    const long long n = (long long)nx * ny * nz * ppc;
+    if (n <= 0) return 0;
+    long long g = (n + 255) / 256;
+    if (g > 148 * 16) g = 148 * 16;
+    k_em_two_stream<<<(int)g, 256, 0, (cudaStream_t)stream>>>(
+        n, ppc, (long long)nx * ny, key_of(seed, 10), key_of(seed, 11), key_of(seed, 12),
+        key_of(seed, 13), key_of(seed, 14), key_of(seed, 15), v0, vth, w, tab, off, u, wout, cell);
     return (int)cudaGetLastError();
 }

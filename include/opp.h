@@ -260,7 +260,7 @@ int opp_get_dat_device_ptr(opp_ctx ctx, int32_t dat_or_map, void **ptr, int64_t 
 enum opp_phase { OPP_PH_INJECT = 0, OPP_PH_BEGIN = 1, OPP_PH_PUSH_MOVE_DEPOSIT = 2,
                  OPP_PH_CONTINUE = 3, OPP_PH_SEGRED = 4, OPP_PH_FILL = 5, OPP_PH_MIGRATE = 6,
                  OPP_PH_HALO = 7, OPP_PH_SORT_COUNT = 8, OPP_PH_SORT_MOVE = 9,
-                 OPP_PH_FIELD = 10, OPP_N_PHASES = 11 };
+                 OPP_PH_FIELD = 10, OPP_PH_EM_MOVE_DEPOSIT = 11, OPP_N_PHASES = 12 };
 
 /* enable != 0: record CUDA events on the context stream around every phase
  * of the following calls (negligible overhead, no host synchronisation). */
@@ -332,6 +332,68 @@ int opp_field_solve(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential, op
 
 /* Statistics of the last opp_field_solve; synchronises. */
 int opp_get_field_stats(opp_ctx ctx, opp_field_stats *stats);
+
+/* ---------------------------------------------------------------------------
+ * CabanaPIC-style electromagnetic particle loop (config C3; SURVEY.md §8(f)
+ * NEXT-2): hex cells of a periodic nx*ny*nz grid declared as an unstructured
+ * mesh through their cell-to-cell map.
+ * All pointers are DEVICE pointers owned by the caller; calls are enqueued on
+ * the context stream (no synchronisation unless stated).  Readings E1-E9 of
+ * DESIGN.md §10 define what the paper leaves open.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    double qdt_2mc;    /* q dt / (2 m c): E and B enter the push scaled by it            */
+    double cdt_2h[3];  /* 2 c dt / h_a: offset units per unit u / gamma, per axis         */
+    double qsp;        /* charge per unit weight (Q_p = qsp * w, Eq. 11)                  */
+    int kcap;          /* face crossings allowed per particle and step (>= 0); at the cap
+                          the particle stops on the face, inside its cell                 */
+    int deposit_mode;  /* OPP_DEP_ATOMIC (12 fp64 reductions per segment) or
+                          OPP_DEP_ATOMIC_WARPAGG (lanes sharing a cell summed in the warp) */
+} opp_em_params;
+
+typedef struct {
+    int64_t n_crossings;   /* face crossings in the last opp_em_move_deposit             */
+    int64_t n_capped;      /* particles stopped by kcap                                  */
+    int32_t max_crossings;
+    int32_t pad;
+} opp_em_stats;
+
+/* Interpolate: from edge E and face B of the periodic
+ * grid to per-cell interpolators.  e[3][nc]: E_a on the cell's edge along a
+ * at the (-,-) corner of its transverse offsets ((a+1)%3, (a+2)%3); the other
+ * three edges of the cell are those of its transverse neighbours.  b[3][nc]:
+ * B_a on the cell's face at offset -1 along a.  interp[nc][18]: ex, dexdy,
+ * dexdz, d2exdydz, ey, deydz, deydx, d2eydzdx, ez, dezdx, dezdy, d2ezdxdy,
+ * bx, dbxdx, by, dbydy, bz, dbzdz, so that E_a = f0 + s f1 + t (f2 + s f3)
+ * with (s, t) the transverse offsets and B_a = f + x_a df.  Cell id =
+ * i + nx (j + ny k).  Errors: OPP_ERR_ARG (sizes < 1, NULL). */
+int opp_em_interpolate(opp_ctx ctx, int nx, int ny, int nz, const double *e, const double *b,
+                       double *interp);
+
+/* Move_Deposit: for particles [0, n) -- SoA columns of
+ * row stride `stride` (elements): off[3][stride] offsets in [-1, 1]^3 of the
+ * particle in its cell, u[3][stride] momenta gamma v / c, w[stride] weights,
+ * cell[stride] -- interpolate E, B from interp[cell] (layout above), Boris-push
+ * u (relativistic, exact rotation with t = qdt_2mc B / gamma), then move the
+ * particle along its streak d_a = cdt_2h[a] u_a / gamma through the faces it
+ * crosses, in order (first face hit; ties -> lowest axis; landing exactly on
+ * a face is inside), the next cell from c2c[cell][f] (f = -x,+x,-y,+y,-z,+z;
+ * n_cells rows), and add to acc[cell][12] the Eq. 11 current of every segment
+ * (PAPER.md:637-680): for the edges along axis a, acc[4a + k] += Q_p *
+ * integral of (1 + sb b)(1 + sc c)/4 d(offset_a) along the segment, edge k =
+ * (sb, sc) in the order (-,-), (+,-), (-,+), (+,+) over the transverse
+ * offsets (b, c) = ((a+1)%3, (a+2)%3).  off, u, cell are updated in place.
+ * cell values must lie in [0, n_cells) and c2c must map into it (not
+ * checked: out-of-range ids are undefined behaviour).  stats may be NULL (no
+ * synchronisation); otherwise the call synchronises and fills it.
+ * Errors: OPP_ERR_ARG (NULL, n < 0, stride < n, kcap < 0, bad mode). */
+int opp_em_move_deposit(opp_ctx ctx, int64_t n, int64_t stride, double *off, double *u,
+                        const double *w, int32_t *cell, const double *interp,
+                        const int32_t *c2c, int64_t n_cells, double *acc,
+                        const opp_em_params *params, opp_em_stats *stats);
+
+/* Statistics of the last opp_em_move_deposit; synchronises. */
+int opp_em_get_stats(opp_ctx ctx, opp_em_stats *stats);
 
 /* Synchronise the context's stream; reports sticky asynchronous errors. */
 int opp_sync(opp_ctx ctx);

@@ -10,6 +10,7 @@
 #include "opp_kernels.h"
 #include "opp_comm.h"
 #include "opp_field.h"
+#include "opp_em.h"
 
 #include <algorithm>
 #include <cstdarg>
@@ -160,6 +161,7 @@ struct opp_ctx_s {
     std::vector<PSet> psets;
     MeshCache mc;
     FieldState fs;
+    opp::EmCounters *em_cnt = nullptr;   // opp_em_move_deposit statistics (device)
     DevCounters *hcnt = nullptr;   // pinned mirror
     long long launches = 0;
     int cell_base = 0;             // global id of local cell 0 (slab partition)
@@ -360,6 +362,7 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.n2cs_ptr, 0);
     c->dfree(m.n2cs, 0);
     free_field(c);
+    c->dfree(c->em_cnt, sizeof(opp::EmCounters));
     if (c->comm) opp::comm_free(c->comm);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     cudaStreamSynchronize(c->cs);
@@ -1737,6 +1740,76 @@ static int field_solve_hostloop(opp_ctx c, CgArgs &a) {
     f.hst.converged = rho <= stop;
     f.hst.rel_residual = rr0 > 0 ? std::sqrt(rho / rr0) : 0.0;
     f.hst.rhs_norm = std::sqrt(rr0);
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// CabanaPIC-style EM loop (config C3): thin marshalling around opp_em.cu.
+// ---------------------------------------------------------------------------
+extern "C" int opp_em_interpolate(opp_ctx c, int nx, int ny, int nz, const double *e,
+                                  const double *b, double *interp) {
+    TRY(ctx_check(c));
+    if (nx < 1 || ny < 1 || nz < 1) return fail(OPP_ERR_ARG, "nx, ny, nz >= 1");
+    if (!e || !b || !interp) return fail(OPP_ERR_ARG, "null field pointer");
+    CK(opp::launch_em_interpolate(nx, ny, nz, e, b, interp, c->s));
+    c->launches += 1;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_get_stats(opp_ctx c, opp_em_stats *st) {
+    TRY(ctx_check(c));
+    if (!st) return fail(OPP_ERR_ARG, "null stats");
+    std::memset(st, 0, sizeof *st);
+    if (!c->em_cnt) return OPP_OK;
+    opp::EmCounters h{};
+    CK(cudaMemcpyAsync(&h, c->em_cnt, sizeof h, cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    st->n_crossings = (int64_t)h.n_crossings;
+    st->n_capped = (int64_t)h.n_capped;
+    st->max_crossings = (int32_t)h.max_crossings;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_move_deposit(opp_ctx c, int64_t n, int64_t stride, double *off, double *u,
+                                   const double *w, int32_t *cell, const double *interp,
+                                   const int32_t *c2c, int64_t n_cells, double *acc,
+                                   const opp_em_params *prm, opp_em_stats *stats) {
+    TRY(ctx_check(c));
+    if (!prm) return fail(OPP_ERR_ARG, "null params");
+    if (n < 0 || stride < n || n_cells < 1) return fail(OPP_ERR_ARG, "n >= 0, stride >= n, n_cells >= 1");
+    if (n > 0 && (!off || !u || !w || !cell)) return fail(OPP_ERR_ARG, "null particle column");
+    if (!interp || !c2c || !acc) return fail(OPP_ERR_ARG, "null mesh array");
+    if (prm->kcap < 0) return fail(OPP_ERR_ARG, "kcap >= 0");
+    if (prm->deposit_mode != OPP_DEP_ATOMIC && prm->deposit_mode != OPP_DEP_ATOMIC_WARPAGG)
+        return fail(OPP_ERR_ARG, "deposit_mode: OPP_DEP_ATOMIC or OPP_DEP_ATOMIC_WARPAGG");
+    if (!c->em_cnt) {
+        c->em_cnt = (opp::EmCounters *)c->dalloc(sizeof(opp::EmCounters));
+        if (!c->em_cnt) return fail(OPP_ERR_NOMEM, "em counters");
+    }
+    CK(cudaMemsetAsync(c->em_cnt, 0, sizeof(opp::EmCounters), c->s));
+    opp::EmArgs a{};
+    a.n = n;
+    a.cap = stride;
+    a.off = off;
+    a.u = u;
+    a.w = w;
+    a.cell = cell;
+    a.interp = interp;
+    a.c2c = c2c;
+    a.nc = n_cells;
+    a.acc = acc;
+    a.qdt_2mc = prm->qdt_2mc;
+    for (int k = 0; k < 3; k++) a.cdt[k] = prm->cdt_2h[k];
+    a.qsp = prm->qsp;
+    a.kcap = prm->kcap;
+    a.dep = prm->deposit_mode == OPP_DEP_ATOMIC_WARPAGG ? 1 : 0;
+    a.cnt = c->em_cnt;
+    if (n > 0) {
+        PhaseScope ph(c, OPP_PH_EM_MOVE_DEPOSIT);
+        CK(opp::launch_em_move_deposit(a, c->nsm, c->s));
+        c->launches += 1;
+    }
+    if (stats) return opp_em_get_stats(c, stats);
     return OPP_OK;
 }
 

@@ -1,0 +1,330 @@
+// opp_em.cu -- sm_100a kernels of the CabanaPIC-style electromagnetic loop
+// (config C3).
+//
+// k_em_move_deposit is the paper's Move_Deposit routine ("calculating new
+// positions and velocities, moving to the correct final cell, and depositing
+// current into an accumulator in a single routine"), one
+// particle per lane:
+//   1. gather the cell's 18-double interpolator (nine 128-bit loads) and
+//      evaluate E (bilinear) and B (linear) at the particle's offsets;
+//   2. relativistic Boris push of u = gamma v / c (Eqs. 7-9 with B);
+//   3. streak d = (2 c dt / h) u / gamma in offset units;
+//   4. walk the straight path through the faces it crosses, in order, the next
+//      cell read from the c2c map, depositing for every
+//      segment the Eq. 11 current of the cell's 12 edges
+//      in closed form: Q da/4 [(1 + sb mb)(1 + sc mc) + sb sc db dc / 12];
+//   5. warp-aggregated accumulation: the lanes depositing into one cell are
+//      summed by a 16-value reduce-scatter over the warp (16 shuffles of
+//      doubles) and leave as one 12-lane reduction instruction -- in
+//      cell-sorted storage (~750 particles per cell) nearly every warp's
+//      first segments share one cell.
+// Arithmetic that decides a result (push, streak, face times, positions) uses
+// explicit round-to-nearest intrinsics, in the oracle's evaluation order
+// (oracle/em.c), so cells and offsets match it bit for bit.
+#include "opp_em.h"
+
+#include <algorithm>
+
+namespace opp {
+namespace {
+
+__device__ __forceinline__ double mul(double a, double b) { return __dmul_rn(a, b); }
+__device__ __forceinline__ double add(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ double sub(double a, double b) { return __dsub_rn(a, b); }
+__device__ __forceinline__ double dvd(double a, double b) { return __ddiv_rn(a, b); }
+
+// ---------------------------------------------------------------------------
+// Interpolate: edge E / face B on the periodic grid ->
+// per-cell interpolator (bilinear E_a in the two transverse offsets, linear
+// B_a).  Same layouts and evaluation order as the oracle's em_interpolate.
+// ---------------------------------------------------------------------------
+__global__ void k_em_interpolate(int nx, int ny, int nz, const double *__restrict__ e,
+                                 const double *__restrict__ b, double *__restrict__ interp) {
+    const long long nc = (long long)nx * ny * nz;
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+         c += (long long)gridDim.x * blockDim.x) {
+        const int i = (int)(c % nx), j = (int)((c / nx) % ny), k = (int)(c / ((long long)nx * ny));
+        const int ip = (i + 1) % nx, jp = (j + 1) % ny, kp = (k + 1) % nz;
+        auto id = [&](int I, int J, int K) { return I + (long long)nx * (J + (long long)ny * K); };
+        double v[3][4];
+        v[0][0] = e[id(i, j, k)];           v[0][1] = e[id(i, jp, k)];
+        v[0][2] = e[id(i, j, kp)];          v[0][3] = e[id(i, jp, kp)];
+        v[1][0] = e[nc + id(i, j, k)];      v[1][1] = e[nc + id(i, j, kp)];
+        v[1][2] = e[nc + id(ip, j, k)];     v[1][3] = e[nc + id(ip, j, kp)];
+        v[2][0] = e[2 * nc + id(i, j, k)];  v[2][1] = e[2 * nc + id(ip, j, k)];
+        v[2][2] = e[2 * nc + id(i, jp, k)]; v[2][3] = e[2 * nc + id(ip, jp, k)];
+        double *f = interp + kEmNI * c;
+#pragma unroll
+        for (int a = 0; a < 3; a++) {
+            const double *q = v[a];
+            f[4 * a + 0] = dvd(add(add(q[0], q[1]), add(q[2], q[3])), 4.0);
+            f[4 * a + 1] = dvd(add(sub(q[1], q[0]), sub(q[3], q[2])), 4.0);
+            f[4 * a + 2] = dvd(add(sub(q[2], q[0]), sub(q[3], q[1])), 4.0);
+            f[4 * a + 3] = dvd(sub(sub(q[3], q[2]), sub(q[1], q[0])), 4.0);
+        }
+        const double b0x = b[id(i, j, k)], b1x = b[id(ip, j, k)];
+        const double b0y = b[nc + id(i, j, k)], b1y = b[nc + id(i, jp, k)];
+        const double b0z = b[2 * nc + id(i, j, k)], b1z = b[2 * nc + id(i, j, kp)];
+        f[12] = dvd(add(b0x, b1x), 2.0); f[13] = dvd(sub(b1x, b0x), 2.0);
+        f[14] = dvd(add(b0y, b1y), 2.0); f[15] = dvd(sub(b1y, b0y), 2.0);
+        f[16] = dvd(add(b0z, b1z), 2.0); f[17] = dvd(sub(b1z, b0z), 2.0);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Move_Deposit
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ double2 ldnc2(const double *p) {
+    double2 v;
+    asm("ld.global.nc.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+    return v;
+}
+
+// Eq. 11 of one straight segment p -> q in offset units, charge Q, closed
+// form: edge k = (sb, sc) along axis a, transverse offsets (b, c) =
+// ((a+1)%3, (a+2)%3), order (-,-), (+,-), (-,+), (+,+).
+__device__ __forceinline__ void seg_current(const double p[3], const double q[3], double Q,
+                                            double v[kEmNA]) {
+    double d[3], m[3];
+#pragma unroll
+    for (int a = 0; a < 3; a++) {
+        d[a] = sub(q[a], p[a]);
+        m[a] = mul(0.5, add(p[a], q[a]));
+    }
+#pragma unroll
+    for (int a = 0; a < 3; a++) {
+        const int b = (a + 1) % 3, c = (a + 2) % 3;
+        const double A = mul(mul(Q, d[a]), 0.25);
+        const double cr = dvd(mul(d[b], d[c]), 12.0);
+        const double bm = sub(1.0, m[b]), bp = add(1.0, m[b]);
+        const double cm = sub(1.0, m[c]), cp = add(1.0, m[c]);
+        v[4 * a + 0] = mul(A, add(mul(bm, cm), cr));
+        v[4 * a + 1] = mul(A, sub(mul(bp, cm), cr));
+        v[4 * a + 2] = mul(A, sub(mul(bm, cp), cr));
+        v[4 * a + 3] = mul(A, add(mul(bp, cp), cr));
+    }
+}
+
+// Sum the 12 values of every lane in `grp` (lanes outside contribute 0) by a
+// reduce-scatter over 16 slots (xor 16, 8, 4, 2 halve the slots, xor 1
+// completes): even lanes 2s (s < 12) then hold slot s and issue one
+// reduction each -- one 12-lane instruction on 96 contiguous bytes.
+__device__ __forceinline__ void rs_deposit(double *__restrict__ acc_cell, bool in,
+                                           const double v[kEmNA]) {
+    const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    double s8[8];
+    const bool h16 = lane & 16u;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const double lo = in ? v[i] : 0.0;
+        const double hi = (in && i + 8 < kEmNA) ? v[i + 8] : 0.0;
+        const double keep = h16 ? hi : lo, send = h16 ? lo : hi;
+        s8[i] = add(keep, __shfl_xor_sync(FULL, send, 16));
+    }
+    double s4[4];
+    const bool h8 = lane & 8u;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const double keep = h8 ? s8[i + 4] : s8[i], send = h8 ? s8[i] : s8[i + 4];
+        s4[i] = add(keep, __shfl_xor_sync(FULL, send, 8));
+    }
+    double s2[2];
+    const bool h4 = lane & 4u;
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+        const double keep = h4 ? s4[i + 2] : s4[i], send = h4 ? s4[i] : s4[i + 2];
+        s2[i] = add(keep, __shfl_xor_sync(FULL, send, 4));
+    }
+    const bool h2 = lane & 2u;
+    double t = add(h2 ? s2[1] : s2[0], __shfl_xor_sync(FULL, h2 ? s2[0] : s2[1], 2));
+    t = add(t, __shfl_xor_sync(FULL, t, 1));
+    const int slot = (h16 ? 8 : 0) + (h8 ? 4 : 0) + (h4 ? 2 : 0) + (h2 ? 1 : 0);
+    if (!(lane & 1u) && slot < kEmNA) atomicAdd(acc_cell + slot, t);
+}
+
+// Deposit one segment per lane (lanes with has = false contribute nothing).
+// DEP 1: lanes are grouped by cell (match_any); up to kEmMaxGroups groups go
+// through the reduce-scatter one after another, more fall back to per-lane
+// reductions.  DEP 0: 12 reductions per lane.
+constexpr int kEmMaxGroups = 3;
+
+template <int DEP>
+__device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, int key,
+                                           const double v[kEmNA]) {
+    const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    if (DEP == 1) {
+        const unsigned peers = __match_any_sync(FULL, has ? key : -1 - (int)lane);
+        unsigned lead = __ballot_sync(FULL, has && (int)lane == __ffs(peers) - 1);
+        if (!lead) return;
+        if (__popc(lead) <= kEmMaxGroups) {
+            do {
+                const int L = __ffs(lead) - 1;
+                lead &= lead - 1u;
+                const int kL = __shfl_sync(FULL, key, L);
+                rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, v);
+            } while (lead);
+            return;
+        }
+    }
+    if (has) {
+        double *a = acc + (long long)kEmNA * key;
+#pragma unroll
+        for (int s = 0; s < kEmNA; s++) atomicAdd(a + s, v[s]);
+    }
+}
+
+template <int DEP>
+__global__ void __launch_bounds__(256) k_em_move_deposit(EmArgs a) {
+    const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
+    const long long gw = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    unsigned long long ncross = 0, ncap = 0;
+    unsigned maxk = 0;
+    for (long long base = gw * 32; base < a.n; base += nwarps * 32) {
+        const long long i = base + lane;
+        const bool valid = i < a.n;
+        int c = 0;
+        double p[3] = {0, 0, 0}, uu[3] = {0, 0, 0}, w = 0;
+        if (valid) {
+            c = a.cell[i];
+            p[0] = a.off[i]; p[1] = a.off[a.cap + i]; p[2] = a.off[2 * a.cap + i];
+            uu[0] = a.u[i]; uu[1] = a.u[a.cap + i]; uu[2] = a.u[2 * a.cap + i];
+            w = a.w[i];
+        }
+        double d[3] = {0, 0, 0};
+        double Q = 0;
+        if (valid) {
+            // 1. interpolate E, B at the offsets (oracle em_fields order)
+            const double *f = a.interp + (long long)kEmNI * c;
+            double F[kEmNI];
+#pragma unroll
+            for (int k = 0; k < kEmNI / 2; k++) {
+                const double2 t = ldnc2(f + 2 * k);
+                F[2 * k] = t.x;
+                F[2 * k + 1] = t.y;
+            }
+            const double x = p[0], y = p[1], z = p[2];
+            const double Ex = add(add(F[0], mul(y, F[1])), mul(z, add(F[2], mul(y, F[3]))));
+            const double Ey = add(add(F[4], mul(z, F[5])), mul(x, add(F[6], mul(z, F[7]))));
+            const double Ez = add(add(F[8], mul(x, F[9])), mul(y, add(F[10], mul(x, F[11]))));
+            const double Bx = add(F[12], mul(x, F[13]));
+            const double By = add(F[14], mul(y, F[15]));
+            const double Bz = add(F[16], mul(z, F[17]));
+            // 2. Boris (oracle em_boris order)
+            const double q2 = a.qdt_2mc;
+            const double h0 = mul(q2, Ex), h1 = mul(q2, Ey), h2 = mul(q2, Ez);
+            double m0 = add(uu[0], h0), m1 = add(uu[1], h1), m2 = add(uu[2], h2);
+            const double gam = __dsqrt_rn(add(1.0, add(add(mul(m0, m0), mul(m1, m1)), mul(m2, m2))));
+            const double r = dvd(q2, gam);
+            const double t0 = mul(r, Bx), t1 = mul(r, By), t2 = mul(r, Bz);
+            const double tt = add(add(mul(t0, t0), mul(t1, t1)), mul(t2, t2));
+            const double p0 = add(m0, sub(mul(m1, t2), mul(m2, t1)));
+            const double p1 = add(m1, sub(mul(m2, t0), mul(m0, t2)));
+            const double p2 = add(m2, sub(mul(m0, t1), mul(m1, t0)));
+            const double sc = dvd(2.0, add(1.0, tt));
+            const double s0 = mul(sc, t0), s1 = mul(sc, t1), s2 = mul(sc, t2);
+            m0 = add(m0, sub(mul(p1, s2), mul(p2, s1)));
+            m1 = add(m1, sub(mul(p2, s0), mul(p0, s2)));
+            m2 = add(m2, sub(mul(p0, s1), mul(p1, s0)));
+            uu[0] = add(m0, h0); uu[1] = add(m1, h1); uu[2] = add(m2, h2);
+            // 3. streak in offset units
+            const double rg = dvd(1.0, __dsqrt_rn(add(1.0, add(add(mul(uu[0], uu[0]), mul(uu[1], uu[1])),
+                                                                 mul(uu[2], uu[2])))));
+            d[0] = mul(a.cdt[0], mul(uu[0], rg));
+            d[1] = mul(a.cdt[1], mul(uu[1], rg));
+            d[2] = mul(a.cdt[2], mul(uu[2], rg));
+            Q = mul(a.qsp, w);
+            a.u[i] = uu[0]; a.u[a.cap + i] = uu[1]; a.u[2 * a.cap + i] = uu[2];
+        }
+        // 4. move through the faces crossed; one segment per lane per round,
+        //    deposited warp-aggregated (rounds continue while any lane moves)
+        bool moving = valid;
+        int k = 0;
+        bool capped = false;
+        while (__any_sync(FULL, moving)) {
+            double v[kEmNA];
+            int face = -1;
+            double q[3] = {p[0], p[1], p[2]};
+            if (moving) {
+                double t = 1.0;
+#pragma unroll
+                for (int ax = 0; ax < 3; ax++) {
+                    if (d[ax] > 0.0) {
+                        const double ta = dvd(sub(1.0, p[ax]), d[ax]);
+                        if (ta < t) { t = ta; face = 2 * ax + 1; }
+                    } else if (d[ax] < 0.0) {
+                        const double ta = dvd(sub(-1.0, p[ax]), d[ax]);
+                        if (ta < t) { t = ta; face = 2 * ax; }
+                    }
+                }
+#pragma unroll
+                for (int ax = 0; ax < 3; ax++) q[ax] = add(p[ax], mul(t, d[ax]));
+                if (face >= 0) q[face >> 1] = (face & 1) ? 1.0 : -1.0;
+                seg_current(p, q, Q, v);
+            } else {
+#pragma unroll
+                for (int s = 0; s < kEmNA; s++) v[s] = 0.0;
+            }
+            em_deposit<DEP>(a.acc, moving, c, v);
+            if (moving) {
+                if (face < 0) {
+                    p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
+                    moving = false;
+                } else if (k >= a.kcap) {
+                    p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
+                    capped = true;
+                    moving = false;
+                } else {
+#pragma unroll
+                    for (int ax = 0; ax < 3; ax++) {
+                        d[ax] = sub(d[ax], sub(q[ax], p[ax]));
+                        p[ax] = q[ax];
+                    }
+                    p[face >> 1] = -p[face >> 1];
+                    c = __ldg(a.c2c + 6 * (long long)c + face);
+                    k++;
+                }
+            }
+        }
+        if (valid) {
+            a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
+            a.cell[i] = c;
+            ncross += (unsigned)k;
+            ncap += capped;
+            maxk = max(maxk, (unsigned)k);
+        }
+    }
+    const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
+    const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
+    const unsigned mk = __reduce_max_sync(FULL, maxk);
+    if (lane == 0) {
+        if (sc) atomicAdd(&a.cnt->n_crossings, (unsigned long long)sc);
+        if (scap) atomicAdd(&a.cnt->n_capped, (unsigned long long)scap);
+        if (mk) atomicMax(&a.cnt->max_crossings, mk);
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
+                                  double *interp, cudaStream_t s) {
+    const long long nc = (long long)nx * ny * nz;
+    const int grid = (int)std::min<long long>((nc + 255) / 256, 4096);
+    k_em_interpolate<<<grid > 0 ? grid : 1, 256, 0, s>>>(nx, ny, nz, e, b, interp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
+    int per = 0;
+    if (a.dep == 1)
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<1>, 256, 0);
+    else
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<0>, 256, 0);
+    const long long need = (a.n + 255) / 256;
+    const long long grid = std::max(1LL, std::min<long long>(need, (long long)nsm * std::max(per, 1)));
+    if (a.dep == 1) k_em_move_deposit<1><<<(int)grid, 256, 0, s>>>(a);
+    else k_em_move_deposit<0><<<(int)grid, 256, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+}  // namespace opp

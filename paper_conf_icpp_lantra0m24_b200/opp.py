@@ -30,9 +30,10 @@ EXPORTS = (
     "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
     "opp_field_init", "opp_field_solve", "opp_get_field_stats",
+    "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
-          "sort_count", "sort_move", "field")
+          "sort_count", "sort_move", "field", "em_move_deposit")
 # note: "fill" includes the periodic sort-by-cell when opp_init_params.sort_every > 0
 
 
@@ -83,6 +84,19 @@ class opp_field_stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class opp_em_params(C.Structure):
+    _fields_ = [("qdt_2mc", C.c_double), ("cdt_2h", C.c_double * 3), ("qsp", C.c_double),
+                ("kcap", C.c_int), ("deposit_mode", C.c_int)]
+
+
+class opp_em_stats(C.Structure):
+    _fields_ = [("n_crossings", C.c_int64), ("n_capped", C.c_int64),
+                ("max_crossings", C.c_int32), ("pad", C.c_int32)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_ if k != "pad"}
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
@@ -119,6 +133,10 @@ def _load():
         "opp_field_solve": (I, [P, I32, I32, I32, C.POINTER(opp_field_params),
                                 C.POINTER(opp_field_stats)]),
         "opp_get_field_stats": (I, [P, C.POINTER(opp_field_stats)]),
+        "opp_em_interpolate": (I, [P, I, I, I, P, P, P]),
+        "opp_em_move_deposit": (I, [P, I64, I64, P, P, P, P, P, P, I64, P,
+                                    C.POINTER(opp_em_params), C.POINTER(opp_em_stats)]),
+        "opp_em_get_stats": (I, [P, C.POINTER(opp_em_stats)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -302,4 +320,30 @@ def opp_field_solve(ctx, node_charge: int, node_potential: int, cell_ef: int,
 def opp_get_field_stats(ctx) -> opp_field_stats:
     st = opp_field_stats()
     _ck(lib.opp_get_field_stats(ctx, C.byref(st)))
+    return st
+
+
+def opp_em_params_make(qdt_2mc: float, cdt_2h, qsp: float, kcap: int = 16,
+                       deposit_mode: int = OPP_DEP_ATOMIC_WARPAGG) -> opp_em_params:
+    return opp_em_params(qdt_2mc, (C.c_double * 3)(*cdt_2h), qsp, kcap, deposit_mode)
+
+
+def opp_em_interpolate(ctx, nx: int, ny: int, nz: int, e, b, interp) -> None:
+    """Device tensors: e[3][nc], b[3][nc] -> interp[nc][18]."""
+    _ck(lib.opp_em_interpolate(ctx, nx, ny, nz, _ptr(e), _ptr(b), _ptr(interp)))
+
+
+def opp_em_move_deposit(ctx, n: int, stride: int, off, u, w, cell, interp, c2c, n_cells: int, acc,
+                        params: opp_em_params, want_stats: bool = True):
+    """Device tensors (SoA columns of row stride `stride`); returns stats or None."""
+    st = opp_em_stats() if want_stats else None
+    _ck(lib.opp_em_move_deposit(ctx, int(n), int(stride), _ptr(off), _ptr(u), _ptr(w), _ptr(cell),
+                                _ptr(interp), _ptr(c2c), int(n_cells), _ptr(acc), C.byref(params),
+                                C.byref(st) if st else None))
+    return st
+
+
+def opp_em_get_stats(ctx) -> opp_em_stats:
+    st = opp_em_stats()
+    _ck(lib.opp_em_get_stats(ctx, C.byref(st)))
     return st

@@ -21,3 +21,12 @@ def test_seed_and_inject_bit_identical():
         b = gc.inject_batch(dm, s, 5001, 77, id_base=9)
         for k in ("pos", "vel", "cell", "id"):
             np.testing.assert_array_equal(a[k], b[k].cpu().numpy())
+
+
+def test_em_two_stream_bit_identical():
+    import gen.cuda as gc
+    import gen.em as ge
+    a = ge.two_stream(5, 4, 6, 37, 91, v0=0.3, vth=0.02)
+    b = gc.em_two_stream(5, 4, 6, 37, 91, v0=0.3, vth=0.02)
+    for k in ("off", "u", "w", "cell"):
+        np.testing.assert_array_equal(a[k], b[k].cpu().numpy())
