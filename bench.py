@@ -64,6 +64,7 @@ def parse():
     ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
     ap.add_argument("--cg-tol", type=float, default=1e-10)
     ap.add_argument("--ppc", type=int, default=750, help="c3: particles per cell (750 = 72M, 1500 = 144M)")
+    ap.add_argument("--em-sort", type=int, default=0, help="c3: sort particles by cell every K steps (0 = never)")
     args = ap.parse_args()
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
     if args.field < 0:
@@ -276,8 +277,16 @@ def run_ours_c3(args, rank, world):
     del d
     n = sim.n
     stream = torch.cuda.current_stream()
+    nstep = [0]
+
+    def em_step(stats=False):
+        if args.em_sort and nstep[0] % args.em_sort == 0:
+            sim.sort_by_cell()
+        nstep[0] += 1
+        return sim.step(want_stats=stats)
+
     for _ in range(args.warmup):
-        sim.step()
+        em_step()
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
@@ -290,14 +299,14 @@ def run_ours_c3(args, rank, world):
     with ClockSampler(dev) as clk:
         e0.record(stream)
         for _ in range(args.steps):
-            sim.step()
+            em_step()
         e1.record(stream)
         torch.cuda.synchronize()
     ms = e0.elapsed_time(e1)
     launches = sim.launches() - l0
     ph = O.opp_get_phase_times(sim.ctx)
     O.opp_phase_timing(sim.ctx, False)
-    st = sim.step(want_stats=True)
+    st = em_step(stats=True)
     pushed = n * args.steps
     if world > 1:
         ms = D.max_over_ranks(ms)
@@ -317,6 +326,7 @@ def run_ours_c3(args, rank, world):
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": C3_NAME.format(ppc=args.ppc), "mesh_cells": nc, "particles": n,
                    "ppc": args.ppc, "deposit": "atomic_warpagg" if args.deposit != 0 else "atomic",
+                   "sort_every": args.em_sort,
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n * 60 / 1e9),
                    "parallelism": f"replicas{world}" if world > 1 else "single"},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -341,7 +351,7 @@ def run_ours_c3(args, rank, world):
             sim.e.copy_(eh, non_blocking=True)
             sim.b.copy_(bh, non_blocking=True)
             sim.interpolate()
-            sim.step()
+            em_step()
             acc_h.copy_(sim.acc, non_blocking=True)
         e1.record(stream)
         torch.cuda.synchronize()

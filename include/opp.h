@@ -392,6 +392,18 @@ int opp_em_move_deposit(opp_ctx ctx, int64_t n, int64_t stride, double *off, dou
                         const int32_t *c2c, int64_t n_cells, double *acc,
                         const opp_em_params *params, opp_em_stats *stats);
 
+/* Counting sort of the EM particles by cell (the auxiliary sort of
+ * PAPER.md:1638-1644 applied to Move_Deposit: lanes of a warp then share a cell,
+ * so the warp-aggregated current deposit sums one group): the n particles of
+ * the input columns (row stride `stride`) are written, grouped by ascending
+ * cell, to the output columns (same stride; must not alias the inputs).  The
+ * order inside a cell is unspecified (any order is a correct sort).  Enqueued,
+ * no synchronisation.  Errors: OPP_ERR_ARG (NULL, n < 0, stride < n),
+ * OPP_ERR_NOMEM (scratch: 4 B per particle + 8 B per cell). */
+int opp_em_sort_by_cell(opp_ctx ctx, int64_t n, int64_t stride, const double *off, const double *u,
+                        const double *w, const int32_t *cell, int64_t n_cells, double *off_out,
+                        double *u_out, double *w_out, int32_t *cell_out);
+
 /* Statistics of the last opp_em_move_deposit; synchronises. */
 int opp_em_get_stats(opp_ctx ctx, opp_em_stats *stats);
 

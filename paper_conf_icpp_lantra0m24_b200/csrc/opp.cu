@@ -162,6 +162,14 @@ struct opp_ctx_s {
     MeshCache mc;
     FieldState fs;
     opp::EmCounters *em_cnt = nullptr;   // opp_em_move_deposit statistics (device)
+    struct {                             // opp_em_sort_by_cell scratch
+        unsigned *hist = nullptr, *start = nullptr;
+        unsigned long long *tile_sums = nullptr;
+        uint32_t *src_of = nullptr;
+        DevCounters *dc = nullptr;
+        long long nc = 0, n = 0;
+        unsigned long long n_host = 0;
+    } em_sort;
     DevCounters *hcnt = nullptr;   // pinned mirror
     long long launches = 0;
     int cell_base = 0;             // global id of local cell 0 (slab partition)
@@ -363,6 +371,11 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.n2cs, 0);
     free_field(c);
     c->dfree(c->em_cnt, sizeof(opp::EmCounters));
+    c->dfree(c->em_sort.hist, 0);
+    c->dfree(c->em_sort.start, 0);
+    c->dfree(c->em_sort.tile_sums, 0);
+    c->dfree(c->em_sort.src_of, 0);
+    c->dfree(c->em_sort.dc, 0);
     if (c->comm) opp::comm_free(c->comm);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     cudaStreamSynchronize(c->cs);
@@ -1767,6 +1780,63 @@ extern "C" int opp_em_get_stats(opp_ctx c, opp_em_stats *st) {
     st->n_crossings = (int64_t)h.n_crossings;
     st->n_capped = (int64_t)h.n_capped;
     st->max_crossings = (int32_t)h.max_crossings;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_sort_by_cell(opp_ctx c, int64_t n, int64_t stride, const double *off,
+                                   const double *u, const double *w, const int32_t *cell,
+                                   int64_t n_cells, double *off_out, double *u_out, double *w_out,
+                                   int32_t *cell_out) {
+    TRY(ctx_check(c));
+    if (n < 0 || stride < n || n_cells < 1) return fail(OPP_ERR_ARG, "n >= 0, stride >= n, n_cells >= 1");
+    if (n > (int64_t)UINT32_MAX) return fail(OPP_ERR_ARG, "n < 2^32");
+    if (!off || !u || !w || !cell || !off_out || !u_out || !w_out || !cell_out)
+        return fail(OPP_ERR_ARG, "null column");
+    if (n == 0) return OPP_OK;
+    auto &es = c->em_sort;
+    if (es.nc < n_cells) {
+        c->dfree(es.hist, 0);
+        c->dfree(es.start, 0);
+        c->dfree(es.tile_sums, 0);
+        es.hist = (unsigned *)c->dalloc(4 * (n_cells + 1));
+        es.start = (unsigned *)c->dalloc(4 * (n_cells + 1));
+        es.tile_sums = (unsigned long long *)c->dalloc(8 * opp::scan_tiles(n_cells + 1));
+        if (!es.hist || !es.start || !es.tile_sums) return fail(OPP_ERR_NOMEM, "em sort scratch");
+        es.nc = n_cells;
+    }
+    if (es.n < n) {
+        c->dfree(es.src_of, 0);
+        es.src_of = (uint32_t *)c->dalloc(4 * (size_t)n);
+        if (!es.src_of) return fail(OPP_ERR_NOMEM, "em sort scratch");
+        es.n = n;
+    }
+    if (!es.dc) {
+        es.dc = (DevCounters *)c->dalloc(sizeof(DevCounters));
+        if (!es.dc) return fail(OPP_ERR_NOMEM, "em sort counters");
+        CK(cudaMemsetAsync(es.dc, 0, sizeof(DevCounters), c->s));
+    }
+    es.n_host = (unsigned long long)n;
+    CK(cudaMemcpyAsync(&es.dc->n, &es.n_host, sizeof(unsigned long long), cudaMemcpyHostToDevice, c->s));
+    ColSet src{}, dst{};
+    const void *in[4] = {off, u, w, cell};
+    void *out[4] = {off_out, u_out, w_out, cell_out};
+    const int dims[4] = {3, 3, 1, 1}, ebs[4] = {8, 8, 8, 4};
+    for (int j = 0; j < 4; j++) {
+        src.c[j] = ColDesc{(char *)in[j], stride, ebs[j], dims[j]};
+        dst.c[j] = ColDesc{(char *)out[j], stride, ebs[j], dims[j]};
+    }
+    src.n = dst.n = 4;
+    {
+        PhaseScope ph(c, OPP_PH_SORT_COUNT);
+        CK(launch_sort_count(cell, es.dc, 0, n_cells, nullptr, es.hist, es.start, es.tile_sums,
+                             grid_for(c, n, c->sort_hgrid), c->s));
+    }
+    {
+        PhaseScope ph(c, OPP_PH_SORT_MOVE);
+        CK(launch_sort_move(src, dst, cell, es.dc, 0, n_cells, nullptr, es.start, nullptr, es.src_of,
+                            grid_for(c, n, 8), grid_for(c, n, c->sort_rgrid), c->s));
+    }
+    c->launches += 7;
     return OPP_OK;
 }
 

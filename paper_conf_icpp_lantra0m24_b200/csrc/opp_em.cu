@@ -95,7 +95,7 @@ __device__ __forceinline__ void seg_current(const double p[3], const double q[3]
     for (int a = 0; a < 3; a++) {
         const int b = (a + 1) % 3, c = (a + 2) % 3;
         const double A = mul(mul(Q, d[a]), 0.25);
-        const double cr = dvd(mul(d[b], d[c]), 12.0);
+        const double cr = mul(mul(d[b], d[c]), 1.0 / 12.0);
         const double bm = sub(1.0, m[b]), bp = add(1.0, m[b]);
         const double cm = sub(1.0, m[c]), cp = add(1.0, m[c]);
         v[4 * a + 0] = mul(A, add(mul(bm, cm), cr));
@@ -143,33 +143,69 @@ __device__ __forceinline__ void rs_deposit(double *__restrict__ acc_cell, bool i
 }
 
 // Deposit one segment per lane (lanes with has = false contribute nothing).
-// DEP 1: lanes are grouped by cell (match_any); up to kEmMaxGroups groups go
-// through the reduce-scatter one after another, more fall back to per-lane
-// reductions.  DEP 0: 12 reductions per lane.
-constexpr int kEmMaxGroups = 3;
-
+// DEP 1: lanes are grouped by cell (match_any).  One group (a cell-uniform
+// warp): the reduce-scatter above.  Several groups (the two beams of a
+// two-stream population drift apart, so a warp's lanes spread over a few
+// cells): a log-step tree sums each group's 12 values into its lowest lane,
+// then the (group, slot) pairs are dealt out 32 per pass -- lane j takes pair
+// 32 r + j: its group's leader and slot -- so each reduction instruction
+// covers up to 32 pairs (consecutive slots of a cell are adjacent doubles).
+// DEP 0: 12 reductions per lane.
 template <int DEP>
 __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, int key,
-                                           const double v[kEmNA]) {
+                                           const double vin[kEmNA]) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
-    if (DEP == 1) {
-        const unsigned peers = __match_any_sync(FULL, has ? key : -1 - (int)lane);
-        unsigned lead = __ballot_sync(FULL, has && (int)lane == __ffs(peers) - 1);
-        if (!lead) return;
-        if (__popc(lead) <= kEmMaxGroups) {
-            do {
-                const int L = __ffs(lead) - 1;
-                lead &= lead - 1u;
-                const int kL = __shfl_sync(FULL, key, L);
-                rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, v);
-            } while (lead);
-            return;
-        }
-    }
-    if (has) {
-        double *a = acc + (long long)kEmNA * key;
+    if (DEP == 0) {
+        if (has) {
+            double *a = acc + (long long)kEmNA * key;
 #pragma unroll
-        for (int s = 0; s < kEmNA; s++) atomicAdd(a + s, v[s]);
+            for (int s = 0; s < kEmNA; s++) atomicAdd(a + s, vin[s]);
+        }
+        return;
+    }
+    const unsigned peers = __match_any_sync(FULL, has ? key : -1 - (int)lane);
+    const unsigned lead = __ballot_sync(FULL, has && (int)lane == __ffs(peers) - 1);
+    if (!lead) return;
+    const int G = __popc(lead);
+    if (G == 1) {
+        const int L = __ffs(lead) - 1;
+        const int kL = __shfl_sync(FULL, key, L);
+        rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, vin);
+        return;
+    }
+    double v[kEmNA];
+#pragma unroll
+    for (int s = 0; s < kEmNA; s++) v[s] = has ? vin[s] : 0.0;
+    // tree: each round a lane absorbs the next still-present lane of its group
+    int rel = __popc(peers & ((1u << lane) - 1u));
+    unsigned up = has ? (peers & ~((2u << lane) - 1u)) : 0u;
+    if (lane == 31) up = 0;
+    while (__any_sync(FULL, up != 0)) {
+        const int nx = up ? __ffs(up) - 1 : (int)lane;
+#pragma unroll
+        for (int s = 0; s < kEmNA; s++) {
+            const double t = __shfl_sync(FULL, v[s], nx);
+            if (up) v[s] = add(v[s], t);
+        }
+        const unsigned gone = __ballot_sync(FULL, (rel & 1) != 0);
+        up &= ~gone;
+        rel >>= 1;
+    }
+    // deal the G x 12 (leader, slot) pairs over the lanes, 32 per pass
+    const int P = G * kEmNA;
+    for (int base = 0; base < P; base += 32) {
+        const int pr = base + (int)lane;
+        const bool act = pr < P;
+        const int g = act ? pr / kEmNA : 0, sl = act ? pr - g * kEmNA : 0;
+        const int L = (int)__fns(lead, 0, g + 1);
+        double val = 0.0;
+#pragma unroll
+        for (int s = 0; s < kEmNA; s++) {
+            const double t = __shfl_sync(FULL, v[s], L);
+            if (s == sl) val = t;
+        }
+        const int kL = __shfl_sync(FULL, key, L);
+        if (act) atomicAdd(acc + (long long)kEmNA * kL + sl, val);
     }
 }
 
@@ -259,7 +295,13 @@ __global__ void __launch_bounds__(256) k_em_move_deposit(EmArgs a) {
                 }
 #pragma unroll
                 for (int ax = 0; ax < 3; ax++) q[ax] = add(p[ax], mul(t, d[ax]));
-                if (face >= 0) q[face >> 1] = (face & 1) ? 1.0 : -1.0;
+                if (face >= 0) {
+                    const double fv = (face & 1) ? 1.0 : -1.0;
+                    const int fa = face >> 1;
+                    q[0] = fa == 0 ? fv : q[0];
+                    q[1] = fa == 1 ? fv : q[1];
+                    q[2] = fa == 2 ? fv : q[2];
+                }
                 seg_current(p, q, Q, v);
             } else {
 #pragma unroll
@@ -280,7 +322,10 @@ __global__ void __launch_bounds__(256) k_em_move_deposit(EmArgs a) {
                         d[ax] = sub(d[ax], sub(q[ax], p[ax]));
                         p[ax] = q[ax];
                     }
-                    p[face >> 1] = -p[face >> 1];
+                    const int fa = face >> 1;
+                    p[0] = fa == 0 ? -p[0] : p[0];
+                    p[1] = fa == 1 ? -p[1] : p[1];
+                    p[2] = fa == 2 ? -p[2] : p[2];
                     c = __ldg(a.c2c + 6 * (long long)c + face);
                     k++;
                 }

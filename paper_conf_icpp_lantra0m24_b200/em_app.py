@@ -60,6 +60,18 @@ class CabanaPicEM:
                                    self.interp, self.c2c, self.nc, self.acc, self.params, want_stats)
         return st.as_dict() if st is not None else None
 
+    def sort_by_cell(self) -> None:
+        """Group the particles by cell (opp_em_sort_by_cell into spare columns, then swap)."""
+        t = self.torch
+        if getattr(self, "_alt", None) is None or self._alt[3].shape[0] != self.n:
+            self._alt = (t.empty_like(self.off), t.empty_like(self.u), t.empty_like(self.w),
+                         t.empty_like(self.cell))
+        ao, au, aw, ac = self._alt
+        O.opp_em_sort_by_cell(self.ctx, self.n, self.n, self.off, self.u, self.w, self.cell, self.nc,
+                              ao, au, aw, ac)
+        self._alt = (self.off, self.u, self.w, self.cell)
+        self.off, self.u, self.w, self.cell = ao, au, aw, ac
+
     def zero_acc(self) -> None:
         self.acc.zero_()
 

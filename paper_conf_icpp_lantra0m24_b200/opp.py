@@ -30,7 +30,7 @@ EXPORTS = (
     "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
     "opp_field_init", "opp_field_solve", "opp_get_field_stats",
-    "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats",
+    "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats", "opp_em_sort_by_cell",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
           "sort_count", "sort_move", "field", "em_move_deposit")
@@ -137,6 +137,7 @@ def _load():
         "opp_em_move_deposit": (I, [P, I64, I64, P, P, P, P, P, P, I64, P,
                                     C.POINTER(opp_em_params), C.POINTER(opp_em_stats)]),
         "opp_em_get_stats": (I, [P, C.POINTER(opp_em_stats)]),
+        "opp_em_sort_by_cell": (I, [P, I64, I64, P, P, P, P, I64, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -347,3 +348,10 @@ def opp_em_get_stats(ctx) -> opp_em_stats:
     st = opp_em_stats()
     _ck(lib.opp_em_get_stats(ctx, C.byref(st)))
     return st
+
+
+def opp_em_sort_by_cell(ctx, n: int, stride: int, off, u, w, cell, n_cells: int, off_out, u_out,
+                        w_out, cell_out) -> None:
+    _ck(lib.opp_em_sort_by_cell(ctx, int(n), int(stride), _ptr(off), _ptr(u), _ptr(w), _ptr(cell),
+                                int(n_cells), _ptr(off_out), _ptr(u_out), _ptr(w_out),
+                                _ptr(cell_out)))
