@@ -256,6 +256,14 @@ def run_reference_c3(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def c3_traffic(args):
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            return json.load(f).get(f"c3_dep{1 if args.deposit != 0 else 0}")
+    except Exception:   # noqa: BLE001
+        return None
+
+
 def run_ours_c3(args, rank, world):
     """C3: one step = Move_Deposit over the whole resident population (the
     accumulator is zeroed between steps outside the timed kernel's model).
@@ -330,7 +338,7 @@ def run_ours_c3(args, rank, world):
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n * 60 / 1e9),
                    "parallelism": f"replicas{world}" if world > 1 else "single"},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": None, "kernel": "k_em_move_deposit",
+                     "frac": achieved / peak, "traffic": c3_traffic(args), "kernel": "k_em_move_deposit",
                      "bytes_model": "112 B/particle + 360 B/cell per launch", "peak_source": peak_src},
         "gpu_launches": launches,
         "phases_ms_per_step": {k: v[0] / args.steps for k, v in ph.items() if v[1]},
