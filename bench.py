@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--ov", type=float, default=0.125, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=10, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--shuffle", type=int, default=0,
+                    help="randomly shuffle the particles every K steps (the paper's GPU policy; use with --sort 0)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
     ap.add_argument("--axis", action="store_true", help="sort key along the duct axis (z)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -457,6 +459,8 @@ def run_ours(args, rank, world):
         if batches[s] is not None:
             sim.inject(batches[s] if on_device else host_batches[s], on_device=on_device)
         sim.step(dt, qm, w, stats=False, fill=True)
+        if args.shuffle and s % args.shuffle == 0:
+            sim.shuffle(seed + 7919 * s)
         if readback is not None:
             readback()
 
@@ -520,7 +524,8 @@ def run_ours(args, rank, world):
                    "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
                    "walk": (f"DH{args.dh}(overlay {args.ov} h)+MH" if args.dh else "MH"),
                    "hop_budget_per_pass": args.hpass,
-                   "sort_every": args.sort, "pipeline": "direct" if args.direct else "tma",
+                   "sort_every": args.sort, "shuffle_every": args.shuffle,
+                   "pipeline": "direct" if args.direct else "tma",
                    "sort_key": "axis z" if args.axis else "cell id",
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n_avg * 60 / 1e9),
                    "parallelism": f"slab{world}",

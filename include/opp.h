@@ -238,6 +238,16 @@ int opp_fill_holes(opp_ctx ctx, opp_set parts, int64_t *n_after);
  * is implementation-defined. */
 int opp_sort_by_cell(opp_ctx ctx, opp_set parts);
 
+/* Random shuffle of the particle set -- the paper's "periodic shuffling"
+ * (on its GPUs shuffling + hole fill beat sorting, since
+ * it spreads same-cell particles and their atomics apart).  Every particle
+ * draws a bucket from a counter-based hash of (index, seed); a counting sort
+ * by bucket moves all columns (holes are dropped, like opp_sort_by_cell).
+ * The permutation depends on seed and on the atomic order inside a bucket;
+ * results of later steps are unchanged up to the deposit's summation order.
+ * Call between steps.  Errors as opp_sort_by_cell. */
+int opp_shuffle(opp_ctx ctx, opp_set parts, uint64_t seed);
+
 /* Copy node charge (dim 1) to host_out[n]; synchronises. */
 int opp_get_node_charge(opp_ctx ctx, opp_dat node_charge, double *host_out, int64_t n);
 

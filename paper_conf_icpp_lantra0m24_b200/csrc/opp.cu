@@ -1105,6 +1105,40 @@ extern "C" int opp_sort_by_cell(opp_ctx c, opp_set parts) {
     return do_sort(c, ps, p2c);
 }
 
+extern "C" int opp_shuffle(opp_ctx c, opp_set parts, uint64_t seed) {
+    TRY(ctx_check(c));
+    TRY(set_check(c, parts));
+    Set &S = c->sets[parts];
+    if (!S.particle) return fail(OPP_ERR_ARG, "not a particle set");
+    PSet &ps = c->psets[S.pset];
+    const int p2c = p2c_of(c, ps);
+    if (p2c < 0) return fail(OPP_ERR_STATE, "particle set has no p2c map");
+    MeshCache &m = c->mc;
+    if (!m.cell_hist) return fail(OPP_ERR_STATE, "shuffle needs the mesh: run a step first");
+    TRY(ensure_alt(c, ps));
+    PhaseScope ph(c, OPP_PH_FILL);
+    ColSet src = make_colset(c, ps), dst = src;
+    for (int j = 0; j < dst.n; j++) dst.c[j].ptr = ps.alt[j];
+    int32_t *keys = (int32_t *)ps.work;   // the continuation worklist is free between steps
+    CK(opp::launch_shuffle_keys((const int32_t *)c->cols[p2c].d, ps.dcnt, (unsigned long long)seed,
+                                m.nc, c->cell_base, keys, grid_for(c, ps.n_ub, 8), c->s));
+    {
+        PhaseScope ph2(c, OPP_PH_SORT_COUNT);
+        CK(launch_sort_count(keys, ps.dcnt, c->cell_base, m.nc, nullptr, m.cell_hist, m.cell_start,
+                             m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
+    }
+    {
+        PhaseScope ph2(c, OPP_PH_SORT_MOVE);
+        CK(launch_sort_move(src, dst, keys, ps.dcnt, c->cell_base, m.nc, nullptr, m.cell_start,
+                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), grid_for(c, ps.n_ub, c->sort_rgrid),
+                            c->s));
+    }
+    c->launches += 8;
+    for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
+    ps.holes_pending = false;
+    return OPP_OK;
+}
+
 // Refresh the particle-side pointers of the step arguments (after growth).
 static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int p2c) {
     a.pos = (double *)c->cols[pos].d;

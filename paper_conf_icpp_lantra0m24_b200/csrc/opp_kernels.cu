@@ -1960,6 +1960,30 @@ cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
     return cudaGetLastError();
 }
 
+// Shuffle keys (opp_shuffle): bucket = hash(index, seed) mod nc (+ cell_base,
+// so the cell-keyed counting sort can consume them), -1 for holes.
+__global__ void k_shuffle_keys(const int32_t *__restrict__ p2c, const DevCounters *c,
+                               unsigned long long seed, long long nb, int cell_base,
+                               int32_t *__restrict__ keys) {
+    const unsigned long long n = c->n;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (unsigned long long)gridDim.x * blockDim.x) {
+        unsigned long long z = seed + (i + 1ull) * 0x9E3779B97F4A7C15ull;
+        z ^= z >> 30;
+        z *= 0xBF58476D1CE4E5B9ull;
+        z ^= z >> 27;
+        z *= 0x94D049BB133111EBull;
+        z ^= z >> 31;
+        keys[i] = p2c[i] < 0 ? -1 : cell_base + (int32_t)(z % (unsigned long long)nb);
+    }
+}
+
+cudaError_t launch_shuffle_keys(const int32_t *p2c, const DevCounters *c, unsigned long long seed,
+                                long long nb, int cell_base, int32_t *keys, int grid, cudaStream_t s) {
+    k_shuffle_keys<<<grid, 256, 0, s>>>(p2c, c, seed, nb, cell_base, keys);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
                               unsigned long long *tile_sums, int grid, cudaStream_t s) {

@@ -29,6 +29,8 @@ cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *h
 long long scan_tiles(long long n);
 cudaError_t scan_exclusive(const unsigned *in, unsigned *out, long long n,
                            unsigned long long *tile_sums, cudaStream_t s);
+cudaError_t launch_shuffle_keys(const int32_t *p2c, const DevCounters *c, unsigned long long seed,
+                                long long nb, int cell_base, int32_t *keys, int grid, cudaStream_t s);
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
                               unsigned long long *tile_sums, int grid, cudaStream_t s);

@@ -31,6 +31,7 @@ EXPORTS = (
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
     "opp_field_init", "opp_field_solve", "opp_get_field_stats",
     "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats", "opp_em_sort_by_cell",
+    "opp_shuffle",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
           "sort_count", "sort_move", "field", "em_move_deposit")
@@ -119,6 +120,7 @@ def _load():
         "opp_fill_holes": (I, [P, I32, C.POINTER(I64)]),
         "opp_get_step_stats": (I, [P, I32, C.POINTER(opp_step_stats)]),
         "opp_sort_by_cell": (I, [P, I32]),
+        "opp_shuffle": (I, [P, I32, C.c_uint64]),
         "opp_get_node_charge": (I, [P, I32, P, I64]),
         "opp_get_dat": (I, [P, I32, P, I64]),
         "opp_set_dat": (I, [P, I32, P, I64, I]),
@@ -254,6 +256,10 @@ def opp_fill_holes(ctx, parts: int, want_count: bool = True):
 
 def opp_sort_by_cell(ctx, parts: int) -> None:
     _ck(lib.opp_sort_by_cell(ctx, parts))
+
+
+def opp_shuffle(ctx, parts: int, seed: int) -> None:
+    _ck(lib.opp_shuffle(ctx, parts, int(seed) & 0xFFFFFFFFFFFFFFFF))
 
 
 def opp_get_node_charge(ctx, dat: int, out) -> None:

@@ -18,6 +18,7 @@ C1, DT, W = 0.5, 1.0, 1.0      # c1 = qm*dt with qm = 0.5, dt = 1
 
 def _gpu_run(mesh, ef, init, inject, steps, qm=C1, dt=DT, w=W, **kw):
     from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    shuffle_every = kw.pop("shuffle_every", 0)
     sim = MiniFemPic(mesh, ef, **kw)
     if init is not None and init["cell"].shape[0]:
         sim.inject(init)
@@ -27,6 +28,8 @@ def _gpu_run(mesh, ef, init, inject, steps, qm=C1, dt=DT, w=W, **kw):
         if b is not None:
             sim.inject(b)
         stats.append(sim.step(dt, qm, w))
+        if shuffle_every and (s + 1) % shuffle_every == 0:
+            sim.shuffle(1000 + s)
     out = sim.particles()
     Q = sim.node_charge_host()
     launches = sim.launches()
@@ -245,4 +248,32 @@ def test_every_particle_inside_its_cell_many_steps(dep, dh, sort_every):
     l123 = np.einsum("nij,nj->ni", G, d)
     lam = np.concatenate([1.0 - l123.sum(1, keepdims=True), l123], 1)
     assert lam.min() >= -1e-9 and lam.max() <= 1 + 1e-9
+    sim.close()
+
+
+@pytest.mark.parametrize("dep,shuffle_every", [(1, 1), (0, 2), (2, 1)])
+def test_c1_parity_with_periodic_shuffle(dep, shuffle_every):
+    """opp_shuffle (the paper's periodic shuffling) between
+    steps permutes storage only: compared by id, results equal the oracle's."""
+    mesh, ef, init, inject, steps = c1_case()
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, deposit_mode=dep,
+                           shuffle_every=shuffle_every)
+    assert rep["n_compared"] > 90_000
+
+
+def test_shuffle_permutes_and_preserves():
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh, ef, init, inject, steps = c1_case()
+    sim = MiniFemPic(mesh, ef)
+    sim.inject(init)
+    sim.step(DT, C1, W)
+    before = sim.particles()
+    sim.shuffle(7)
+    raw = sim.particles(sort_by_id=False)
+    after = sim.particles()
+    for k in before:
+        assert np.array_equal(before[k], after[k])
+    # storage order is no longer the id order nor cell-sorted
+    assert not np.all(np.diff(raw["id"]) > 0)
+    assert not np.all(np.diff(raw["cell"]) >= 0)
     sim.close()
