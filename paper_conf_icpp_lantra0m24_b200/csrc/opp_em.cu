@@ -143,14 +143,25 @@ __device__ __forceinline__ void rs_deposit(double *__restrict__ acc_cell, bool i
 }
 
 // Deposit one segment per lane (lanes with has = false contribute nothing).
-// DEP 1: lanes are grouped by cell (match_any).  One group (a cell-uniform
-// warp): the reduce-scatter above.  Several groups (the two beams of a
+// DEP 1: at most OPP_EM_DIRECT active lanes (the later move rounds: only the
+// particles still crossing faces) reduce directly -- an fp64 reduction costs
+// the L1 ~2 cycles per lane, cheaper than any warp-wide shuffle reduction of
+// 12 values.  Otherwise lanes are grouped by cell (match_any).  Up to
+// OPP_EM_RS_MAX groups: one reduce-scatter (above) per group.  More groups (the two beams of a
 // two-stream population drift apart, so a warp's lanes spread over a few
 // cells): a log-step tree sums each group's 12 values into its lowest lane,
 // then the (group, slot) pairs are dealt out 32 per pass -- lane j takes pair
 // 32 r + j: its group's leader and slot -- so each reduction instruction
 // covers up to 32 pairs (consecutive slots of a cell are adjacent doubles).
 // DEP 0: 12 reductions per lane.
+#ifndef OPP_EM_DIRECT
+#define OPP_EM_DIRECT 8   // active lanes at or below which segments reduce directly
+                          // (C3: 0 -> 8 lanes: 5.38 -> 4.80 ms; 12, 16: same)
+#endif
+#ifndef OPP_EM_RS_MAX
+#define OPP_EM_RS_MAX 3   // cells per warp at or below which each gets a reduce-scatter
+                          // (C3: 1, 2, 3 within 1%; 6: 8% slower)
+#endif
 template <int DEP>
 __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, int key,
                                            const double vin[kEmNA]) {
@@ -163,14 +174,27 @@ __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, i
         }
         return;
     }
+    const unsigned act = __ballot_sync(FULL, has);
+    if (!act) return;
+    if (__popc(act) <= OPP_EM_DIRECT) {   // a few lanes (later move rounds): direct reductions
+        if (has) {
+            double *a = acc + (long long)kEmNA * key;
+#pragma unroll
+            for (int s = 0; s < kEmNA; s++) atomicAdd(a + s, vin[s]);
+        }
+        return;
+    }
     const unsigned peers = __match_any_sync(FULL, has ? key : -1 - (int)lane);
     const unsigned lead = __ballot_sync(FULL, has && (int)lane == __ffs(peers) - 1);
-    if (!lead) return;
     const int G = __popc(lead);
-    if (G == 1) {
-        const int L = __ffs(lead) - 1;
-        const int kL = __shfl_sync(FULL, key, L);
-        rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, vin);
+    if (G <= OPP_EM_RS_MAX) {   // one reduce-scatter per cell
+        unsigned l = lead;
+        do {
+            const int L = __ffs(l) - 1;
+            l &= l - 1u;
+            const int kL = __shfl_sync(FULL, key, L);
+            rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, vin);
+        } while (l);
         return;
     }
     double v[kEmNA];
