@@ -22,17 +22,17 @@ static const char *names[] = {"ldg.256", "ldg.128", "ldg.64", "ldg.32", "ldg.16"
 // distinct: number of distinct addresses in the warp; spread: bytes between them
 template <int MODE>
 __global__ void __launch_bounds__(256) k(const char *__restrict__ src, double *out, int iters,
-                                         int distinct, int spread, int active = 32) {
+                                         int distinct, int spread, int active = 32, int contig = 0) {
     __shared__ __align__(32) double sm[1024];
     for (int i = threadIdx.x; i < 1024; i += blockDim.x) sm[i] = i;
     __syncthreads();
     const int lane = threadIdx.x & 31;
-    const int grp = lane % distinct;
+    const int grp = contig ? lane / (32 / distinct) : lane % distinct;
     const long long woff = (long long)(threadIdx.x >> 5) * 4096;   // 32 KB per window, shared by all SMs: L1-resident
     const char *p = src + woff + (long long)grp * spread;
     double acc = 0;
     unsigned acci = 0;
-    double *dst = out + 1024 + grp * (spread / 8) + (blockIdx.x % 16) * 4096;
+    double *dst = out + 1024 + grp * (spread / 8) + (long long)(blockIdx.x * 8 + (threadIdx.x >> 5)) * 4096;   // per-warp region: no inter-warp contention
 #pragma unroll 1
     for (int it = 0; it < iters; it++) {
         // 8 independent instructions per iteration, consumed after all issued
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(256) k(const char *__restrict__ src, double *o
             } else if (MODE == SHFL64) {
                 r[k] = __shfl_sync(0xffffffffu, acc + (double)k, grp);
             } else if (MODE == RED64) {
-                asm volatile("red.global.add.f64 [%0], %1;" :: "l"(dst + k * 16384), "d"(1.0) : "memory");
+                asm volatile("red.global.add.f64 [%0], %1;" :: "l"(dst + k * 512), "d"(1.0) : "memory");
             }
         }
 #pragma unroll
@@ -94,13 +94,13 @@ __global__ void __launch_bounds__(256) k(const char *__restrict__ src, double *o
 }
 
 template <int MODE>
-static float run(const char *src, double *out, int iters, int d, int spread, int active = 32) {
+static float run(const char *src, double *out, int iters, int d, int spread, int active = 32, int contig = 0) {
     cudaEvent_t e0, e1;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
     k<MODE><<<148 * 4, 256>>>(src, out, 8, d, spread);   // warm
     cudaEventRecord(e0);
-    k<MODE><<<148 * 4, 256>>>(src, out, iters, d, spread, active);
+    k<MODE><<<148 * 4, 256>>>(src, out, iters, d, spread, active, contig);
     cudaEventRecord(e1);
     cudaEventSynchronize(e1);
     float ms;
@@ -113,14 +113,29 @@ int main() {
     double *out;
     cudaMalloc(&src, 64 << 20);
     cudaMemset(src, 0, 64 << 20);
-    cudaMalloc(&out, 8 * (1024 + 16 * 4096 + 8 * 16384 + 64 * 1024));
-    cudaMemset(out, 0, 8 * (1024 + 16 * 4096 + 8 * 16384 + 64 * 1024));
+    const size_t ob = 8ull * (1024 + 148 * 4 * 8 * 4096ull + 64 * 1024);
+    cudaMalloc(&out, ob);
+    cudaMemset(out, 0, ob);
     int clk_khz = 0;
     cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, 0);
     const int iters = 1024;
     const double winstr_per_sm = 4.0 * 8 * iters * 8;
     printf("mode distinct spread_B cycles_per_warp_instr (SM clock %d MHz)\n", clk_khz / 1000);
 
+
+    printf("contiguous lane groups (lanes 0..32/d-1 share line 0, ...), spread 128\n");
+    for (int d : {1, 2, 4, 8}) {
+        auto cyc = [&](float t) { return (double)t * 1e-3 * clk_khz * 1e3 / winstr_per_sm; };
+        printf("d=%d contig: ldg.256 %6.2f ldg.64 %6.2f lds.128 %6.2f | interleaved: ldg.256 %6.2f\n", d,
+               cyc(run<G256>(src, out, iters, d, 128, 32, 1)), cyc(run<G64>(src, out, iters, d, 128, 32, 1)),
+               cyc(run<S128>(src, out, iters, d, 128, 32, 1)), cyc(run<G256>(src, out, iters, d, 128, 32, 0)));
+    }
+    printf("red.f64, per-warp region (no contention): active lanes x distinct lines\n");
+    for (int act : {1, 4, 8, 16, 32}) {
+        auto cyc = [&](float t) { return (double)t * 1e-3 * clk_khz * 1e3 / winstr_per_sm; };
+        printf("active=%2d d=1 %7.2f  d=32(sp128) %7.2f  d=32(sp8) %7.2f\n", act, cyc(run<RED64>(src, out, 256, 1, 128, act)) * 4,
+               cyc(run<RED64>(src, out, 256, 32, 128, act)) * 4, cyc(run<RED64>(src, out, 256, 32, 8, act)) * 4);
+    }
     printf("partial warps: active lanes, each on its own line (spread 128) or all on one line\n");
     for (int act : {1, 2, 4, 8, 16}) {
         for (int d : {1, 32}) {
