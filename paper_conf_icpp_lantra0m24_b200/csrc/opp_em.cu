@@ -307,14 +307,14 @@ __global__ void __launch_bounds__(256) k_em_move_deposit(EmArgs a) {
             double q[3] = {p[0], p[1], p[2]};
             if (moving) {
                 double t = 1.0;
+                // one division site per axis (the oracle's two branches differ only
+                // in the numerator): divergent lanes would otherwise run both
 #pragma unroll
                 for (int ax = 0; ax < 3; ax++) {
-                    if (d[ax] > 0.0) {
-                        const double ta = dvd(sub(1.0, p[ax]), d[ax]);
-                        if (ta < t) { t = ta; face = 2 * ax + 1; }
-                    } else if (d[ax] < 0.0) {
-                        const double ta = dvd(sub(-1.0, p[ax]), d[ax]);
-                        if (ta < t) { t = ta; face = 2 * ax; }
+                    const bool pos = d[ax] > 0.0;
+                    if (d[ax] != 0.0) {
+                        const double ta = dvd(sub(pos ? 1.0 : -1.0, p[ax]), d[ax]);
+                        if (ta < t) { t = ta; face = 2 * ax + (pos ? 1 : 0); }
                     }
                 }
 #pragma unroll
