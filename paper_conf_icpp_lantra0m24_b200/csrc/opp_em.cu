@@ -233,8 +233,11 @@ __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, i
     }
 }
 
+#ifndef OPP_EM_MINB
+#define OPP_EM_MINB 3   // resident blocks per SM (80 registers); 4 spills and measured slower
+#endif
 template <int DEP>
-__global__ void __launch_bounds__(256) k_em_move_deposit(EmArgs a) {
+__global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
     const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
     const long long gw = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
