@@ -222,6 +222,9 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 #define OPP_RS_GROUPS 0   // C2: 0 (always the tree) 1.894 ms, 3: 1.912, 8: 2.35
 #endif
 constexpr int kMaxRsGroups = OPP_RS_GROUPS;
+#ifndef OPP_DEP_MERGE
+#define OPP_DEP_MERGE 1   // singles through the tree too: C2 pass 1 1.901 -> 1.849 ms, C5 2.80 -> 2.71
+#endif
 
 // Node ids of the depositing cell: from the walk line already in registers,
 // or (lazy line) loaded by the lanes that issue the reductions only.
@@ -282,6 +285,13 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const CnSrc 
     const unsigned lane = lane_id();
     const unsigned peers = __match_any_sync(FULL, done ? key : -2 - (int)lane);
     const bool single = peers == (1u << lane);
+    if (OPP_DEP_MERGE && kMaxRsGroups == 0) {
+        // singles ride through the tree as groups of one, so every cell's
+        // four reductions leave in the same four instructions (the fixed
+        // cost of a reduction instruction is paid once, not twice)
+        if (__any_sync(FULL, done)) deposit_tree(Q, done, peers, cs, key, cn, v0, v1, v2, v3);
+        return;
+    }
     if (done && single) red4(Q, cs.get(key, cn), v0, v1, v2, v3);
     unsigned lead = __ballot_sync(FULL, done && !single && (int)lane == __ffs(peers) - 1);
     if (!lead) return;
