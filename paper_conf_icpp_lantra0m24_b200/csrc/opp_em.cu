@@ -162,9 +162,15 @@ __device__ __forceinline__ void rs_deposit(double *__restrict__ acc_cell, bool i
 #define OPP_EM_RS_MAX 3   // cells per warp at or below which each gets a reduce-scatter
                           // (C3: 1, 2, 3 within 1%; 6: 8% slower)
 #endif
+#ifndef OPP_EM_SMEM_SUM
+#define OPP_EM_SMEM_SUM 1   // > OPP_EM_RS_MAX cells per warp: transpose through shared memory
+                            // (C3: 4.50 -> 4.16 ms vs the shuffle tree + deal)
+#endif
+constexpr int kEmBufLd = 33;   // row stride (doubles) of the per-warp transpose buffer
+
 template <int DEP>
 __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, int key,
-                                           const double vin[kEmNA]) {
+                                           const double vin[kEmNA], double *__restrict__ buf) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
     if (DEP == 0) {
         if (has) {
@@ -195,6 +201,38 @@ __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, i
             const int kL = __shfl_sync(FULL, key, L);
             rs_deposit(acc + (long long)kEmNA * kL, has && key == kL, vin);
         } while (l);
+        return;
+    }
+    if (OPP_EM_SMEM_SUM) {
+        // transpose: buf[slot][lane]; then lane j sums (cell g, slot s) pair
+        // 32 r + j over the members of cell g -- about 12 G x (32 / G) / 32 =
+        // 12 iterations for any number of cells, where shuffle reductions cost
+        // a full warp pass per cell
+        if (has) {
+#pragma unroll
+            for (int s = 0; s < kEmNA; s++) buf[s * kEmBufLd + lane] = vin[s];
+        }
+        __syncwarp();
+        const int P = G * kEmNA;
+        for (int base = 0; base < P; base += 32) {
+            const int pr = base + (int)lane;
+            const bool act = pr < P;
+            const int g = act ? pr / kEmNA : 0, sl = act ? pr - g * kEmNA : 0;
+            const int L = (int)__fns(lead, 0, g + 1);
+            unsigned m = __shfl_sync(FULL, peers, L);
+            const int kL = __shfl_sync(FULL, key, L);
+            if (act) {
+                const double *row = buf + sl * kEmBufLd;
+                double sum = 0.0;
+                while (m) {
+                    const int k = __ffs(m) - 1;
+                    m &= m - 1u;
+                    sum = add(sum, row[k]);
+                }
+                atomicAdd(acc + (long long)kEmNA * kL + sl, sum);
+            }
+        }
+        __syncwarp();
         return;
     }
     double v[kEmNA];
@@ -239,6 +277,8 @@ __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, i
 template <int DEP>
 __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    __shared__ double em_buf[OPP_EM_SMEM_SUM ? 8 : 1][OPP_EM_SMEM_SUM ? kEmNA * kEmBufLd : 1];
+    double *wbuf = em_buf[OPP_EM_SMEM_SUM ? (threadIdx.x >> 5) : 0];
     const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
     const long long gw = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     unsigned long long ncross = 0, ncap = 0;
@@ -334,7 +374,7 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
 #pragma unroll
                 for (int s = 0; s < kEmNA; s++) v[s] = 0.0;
             }
-            em_deposit<DEP>(a.acc, moving, c, v);
+            em_deposit<DEP>(a.acc, moving, c, v, wbuf);
             if (moving) {
                 if (face < 0) {
                     p[0] = q[0]; p[1] = q[1]; p[2] = q[2];

@@ -277,3 +277,18 @@ def test_shuffle_permutes_and_preserves():
     assert not np.all(np.diff(raw["id"]) > 0)
     assert not np.all(np.diff(raw["cell"]) >= 0)
     sim.close()
+
+
+@pytest.mark.parametrize("dep,sort_every", [(0, 0), (1, 0), (1, 2), (2, 0)])
+def test_c5_style_clustered_parity(dep, sort_every):
+    """C5's shape at C1 size: 90% of 100k particles in a 2x2x3-hex block
+    (72 tets, ~1,250 particles per hot tet): the deposit under heavy
+    same-cell contention (plain fp64 atomics, warp-aggregated, sort +
+    segmented reduction), sorted and unsorted storage."""
+    mesh = gen.kuhn_duct(6, 6, 30, jitter=0.2, seed=20240816)
+    rng = np.random.default_rng(16)
+    ef = rng.uniform(-2e-3, 2e-3, (mesh["n_cells"], 3))
+    hot = gen.hot_block_cells(mesh, lo=(2, 2, 10), size=(2, 2, 3))
+    init = gen.seed_particles(mesh, 100_000, 20240816, cluster=(0.9, hot))
+    rep, ost, gst = _check(mesh, ef, init, None, 4, deposit_mode=dep, sort_every=sort_every)
+    assert rep["n_compared"] > 95_000
