@@ -467,7 +467,12 @@ constexpr int kTiledThreads = kTile + 32;
 #endif
 constexpr int kStages = OPP_STAGES;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
-constexpr int kRingBytesPerWarp = 64 * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
+constexpr int kRingBytesPerWarp = 64 * 12 + 128;   // holes ring (4 B) + work ring (4 B + 4 B hops) + lane permutation (32 x 4 B)
+#ifndef OPP_SEED_PERM
+#define OPP_SEED_PERM 0   // 1: regroup a warp's lanes by seed cell before the first walk-line load
+                          // (C2: parity green, pass 1 1.844 -> 1.884 ms: the shuffles cost more than
+                          // the cheaper line loads save -- off)
+#endif
 #ifndef OPP_TMA_OUT
 // 0: results leave as coalesced per-lane stores (C2: pmd 1.99 vs 2.06 ms --
 // staging the stores in shared memory cost L1 data-pipe wavefronts twice,
@@ -566,13 +571,13 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                                          double &vy, double &vz, int &cell, Tally &t,
                                          uint64_t *release = nullptr, double *sout = nullptr,
                                          int sj = 0, Appends *ap = nullptr,
-                                         const Pre *pre = nullptr) {
+                                         const Pre *pre = nullptr, int *perm = nullptr) {
     int status = ST_NONE;
     int capped = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
     int4 cn = make_int4(0, 0, 0, 0);
     // output position: i (in place), or dest[i] on a sort-fused step
-    const unsigned long long o = (!CONT && a.dest && valid) ? (unsigned long long)__ldg(a.dest + i) : i;
+    unsigned long long o = (!CONT && a.dest && valid) ? (unsigned long long)__ldg(a.dest + i) : i;
     if (valid && a.dbg == 1) {   // diagnostic: stream only
         vx = add(vx, a.c1); x = add(x, mul(vx, a.dt));
         a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
@@ -648,6 +653,33 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                     if (!SOUT) L = load_line(a.lines, sc - a.cell_base);
                 }
             }
+            if (SOUT && DH == 1 && perm) {
+                // regroup the warp's particles by seed cell (contiguous lanes share
+                // a cell): a 256-bit load costs the L1 ~2 cycles per distinct line
+                // per 8-lane quarter, so interleaved seeds (~6 per warp) cost ~27
+                // cycles per walk-line load and grouped ones ~17.  Position, cell
+                // and output slot move; v is already stored.
+                const unsigned FULL = 0xffffffffu, ln = threadIdx.x & 31u;
+                const unsigned peers = __match_any_sync(FULL, cell);
+                const int leader = __ffs(peers) - 1;
+                const int sz = (int)ln == leader ? __popc(peers) : 0;
+                int incl = sz;
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const int tq = __shfl_up_sync(FULL, incl, d);
+                    if ((int)ln >= d) incl += tq;
+                }
+                const int dest = __shfl_sync(FULL, incl - sz, leader) + __popc(peers & ((1u << ln) - 1u));
+                perm[dest] = (int)ln;
+                __syncwarp();
+                const int src = perm[ln];
+                __syncwarp();
+                x = __shfl_sync(FULL, x, src);
+                y = __shfl_sync(FULL, y, src);
+                z = __shfl_sync(FULL, z, src);
+                cell = __shfl_sync(FULL, cell, src);
+                o = __shfl_sync(FULL, o, src);
+            }
             if (SOUT) {
                 int zero;
                 asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}"
@@ -704,6 +736,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         }
     }
     if (rem) cell = -1;
+    if (perm) a.p2c_out[o] = cell;   // regrouped lanes store their own particle's cell
 }
 
 // ---------------------------------------------------------------------------
@@ -1024,15 +1057,18 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
             // results leave through the shared buffer + bulk stores (TMA_OUT),
             // or (sort-fused step / OPP_TMA_OUT=0) as coalesced per-lane stores
             double *obuf = (TMA_OUT && !a.dest) ? o : nullptr;
+            int *perm = (OPP_SEED_PERM && DH == 1 && !obuf)
+                             ? reinterpret_cast<int *>(smem + kRingBase + (size_t)warp * kRingBytesPerWarp + 64 * 12)
+                             : nullptr;
             pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
                                                   nullptr, obuf, (int)lane, &ap,
-                                                  (PRE && have_cur) ? &cur : nullptr);
+                                                  (PRE && have_cur) ? &cur : nullptr, perm);
             if (PRE) {
                 cur = nxt;
                 have_cur = have_nxt;
             }
             if (!obuf) {
-                a.p2c_out[a.dest ? (unsigned long long)__ldg(a.dest + i) : i] = cell;
+                if (!perm) a.p2c_out[a.dest ? (unsigned long long)__ldg(a.dest + i) : i] = cell;
                 continue;
             }
             reinterpret_cast<int *>(o + 192)[lane] = cell;
