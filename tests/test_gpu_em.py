@@ -211,3 +211,37 @@ def test_em_sorted_steps_parity():
     np.testing.assert_allclose(bb[0], a[0], rtol=1e-12, atol=1e-15)
     np.testing.assert_allclose(bb[1], a[1], rtol=1e-12, atol=1e-15)
     assert np.abs(g["acc"] - acc).max() <= 1e-10 * np.abs(acc).max()
+
+
+def test_em_face_start_and_rest_edge_cases():
+    """Particles starting exactly on a face and moving out (zero-length first
+    segment, immediate crossing), on a face moving in, at rest (d = 0), and on
+    an edge / corner (two or three faces hit at t = 0: lowest axis first)."""
+    nx, ny, nz = 3, 3, 3
+    e, b = G.em_fields(nx, ny, nz, 2)
+    e[:] = 0.0
+    b[:] = 0.0
+    cases_off = [(1.0, 0.2, -0.3), (-1.0, 0.5, 0.5), (0.3, 1.0, 0.0), (0.1, 0.1, -1.0),
+                 (1.0, 1.0, 0.0), (1.0, 1.0, 1.0), (-1.0, -1.0, -1.0), (0.0, 0.0, 0.0),
+                 (1.0, 0.0, 0.0), (0.5, -0.5, 0.25)]
+    cases_u = [(0.3, 0.0, 0.0), (-0.2, 0.1, 0.0), (0.0, 0.4, 0.1), (0.0, 0.0, -0.5),
+               (0.2, 0.2, 0.0), (0.1, 0.1, 0.1), (-0.3, -0.3, -0.3), (0.0, 0.0, 0.0),
+               (-0.3, 0.0, 0.0), (0.0, 0.0, 0.0)]
+    n = len(cases_off)
+    off = np.ascontiguousarray(np.array(cases_off).T)
+    u = np.ascontiguousarray(np.array(cases_u).T)
+    w = np.linspace(0.5, 1.5, n)
+    cell = np.arange(n, dtype=np.int32) % (nx * ny * nz)
+    interp = OE.interpolate(nx, ny, nz, e, b)
+    c2c = G.periodic_hex(nx, ny, nz)
+    acc = np.zeros((nx * ny * nz, 12))
+    prm = OE.params(0.05, [1.0, 1.0, 1.0], 1.0, 16)
+    o_off, o_u, o_cell = off.copy(), u.copy(), cell.copy()
+    ost = [OE.move_deposit(prm, o_off, o_u, w, o_cell, interp, c2c, acc) for _ in range(2)]
+    sim = _app(nx, ny, nz, e, b, 0.05, [1.0, 1.0, 1.0])
+    sim.set_particles(off, u, w, cell)
+    gst = [sim.step(want_stats=True) for _ in range(2)]
+    g = sim.state()
+    sim.close()
+    _check((o_off, o_u, o_cell, acc, ost), g, gst)
+    assert ost[0]["n_crossings"] >= 6
