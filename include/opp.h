@@ -414,6 +414,29 @@ int opp_em_sort_by_cell(opp_ctx ctx, int64_t n, int64_t stride, const double *of
                         const double *w, const int32_t *cell, int64_t n_cells, double *off_out,
                         double *u_out, double *w_out, int32_t *cell_out);
 
+/* Field side of the EM loop ("the accumulator data is
+ * processed in the AccumulateCurrent routine to obtain the current density
+ * necessary for field solving.  Field solving follows a kernel based
+ * leap-frog approach, with AdvanceE and AdvanceB"), normalised units
+ * (c = eps0 = 1), Yee staggering matching opp_em_interpolate's layout: E_a and
+ * J_a on the cell's edge along a at the (-,-) corner of its transverse
+ * offsets, B_a on its face at offset -1; neighbours read through
+ * c2c[n_cells][6]; h[3] the cell sizes; all arrays [3][n_cells] device
+ * memory.  Enqueued, no synchronisation.  Errors: OPP_ERR_ARG (NULL,
+ * n_cells < 1, h or dt not positive).
+ *
+ * AccumulateCurrent: J_a(edge) = (sum of the 4 adjacent cells' accumulator
+ * entries for that edge) / (2 dt h_b h_c) -- with it the discrete continuity
+ * equation (and so Gauss's law) holds exactly for the Eq. 11 deposit. */
+int opp_em_accumulate_current(opp_ctx ctx, const double *acc, const int32_t *c2c, int64_t n_cells,
+                              const double *h, double dt, double *J);
+/* AdvanceB: B -= frac_dt * curl E (the leap-frog's half steps). */
+int opp_em_advance_b(opp_ctx ctx, const double *e, double *b, const int32_t *c2c, int64_t n_cells,
+                     const double *h, double frac_dt);
+/* AdvanceE: E += dt * (curl B - J). */
+int opp_em_advance_e(opp_ctx ctx, double *e, const double *b, const double *J, const int32_t *c2c,
+                     int64_t n_cells, const double *h, double dt);
+
 /* Statistics of the last opp_em_move_deposit; synchronises. */
 int opp_em_get_stats(opp_ctx ctx, opp_em_stats *stats);
 

@@ -1817,6 +1817,45 @@ extern "C" int opp_em_get_stats(opp_ctx c, opp_em_stats *st) {
     return OPP_OK;
 }
 
+static int em_field_check(const void *a, const void *b, const void *c2c, int64_t nc, const double *h,
+                          double dt) {
+    if (!a || !b || !c2c || !h) return fail(OPP_ERR_ARG, "null array");
+    if (nc < 1) return fail(OPP_ERR_ARG, "n_cells >= 1");
+    if (!(h[0] > 0.0 && h[1] > 0.0 && h[2] > 0.0) || !(dt > 0.0)) return fail(OPP_ERR_ARG, "h, dt > 0");
+    return OPP_OK;
+}
+
+extern "C" int opp_em_accumulate_current(opp_ctx c, const double *acc, const int32_t *c2c,
+                                         int64_t n_cells, const double *h, double dt, double *J) {
+    TRY(ctx_check(c));
+    TRY(em_field_check(acc, J, c2c, n_cells, h, dt));
+    PhaseScope ph(c, OPP_PH_FIELD);
+    CK(opp::launch_em_accumulate_current(acc, c2c, n_cells, h, dt, J, c->s));
+    c->launches += 1;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_advance_b(opp_ctx c, const double *e, double *b, const int32_t *c2c,
+                                int64_t n_cells, const double *h, double frac_dt) {
+    TRY(ctx_check(c));
+    TRY(em_field_check(e, b, c2c, n_cells, h, frac_dt));
+    PhaseScope ph(c, OPP_PH_FIELD);
+    CK(opp::launch_em_advance_b(e, b, c2c, n_cells, h, frac_dt, c->s));
+    c->launches += 1;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_advance_e(opp_ctx c, double *e, const double *b, const double *J,
+                                const int32_t *c2c, int64_t n_cells, const double *h, double dt) {
+    TRY(ctx_check(c));
+    TRY(em_field_check(e, b, c2c, n_cells, h, dt));
+    if (!J) return fail(OPP_ERR_ARG, "null J");
+    PhaseScope ph(c, OPP_PH_FIELD);
+    CK(opp::launch_em_advance_e(e, b, J, c2c, n_cells, h, dt, c->s));
+    c->launches += 1;
+    return OPP_OK;
+}
+
 extern "C" int opp_em_sort_by_cell(opp_ctx c, int64_t n, int64_t stride, const double *off,
                                    const double *u, const double *w, const int32_t *cell,
                                    int64_t n_cells, double *off_out, double *u_out, double *w_out,

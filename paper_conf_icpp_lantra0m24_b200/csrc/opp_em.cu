@@ -416,7 +416,98 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
     }
 }
 
+// ---------------------------------------------------------------------------
+// Field side: AccumulateCurrent, AdvanceB, AdvanceE on the
+// Yee-staggered periodic grid, neighbours read through c2c (f = -x,+x,-y,+y,
+// -z,+z).  One thread per cell; the oracle's operation order (oracle/em_field.py)
+// so results are bit-identical.  E_a / J_a live on the cell's edge along a at
+// the (-,-) corner of its transverse offsets, B_a on its face at offset -1.
+// ---------------------------------------------------------------------------
+__global__ void k_em_accumulate_current(const double *__restrict__ acc,
+                                        const int32_t *__restrict__ c2c, long long nc, double sx,
+                                        double sy, double sz, double *__restrict__ J) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+         c += (long long)gridDim.x * blockDim.x) {
+        const int *nb = c2c + 6 * c;
+        const int xm = nb[0], ym = nb[2], zm = nb[4];
+        const int ymzm = __ldg(c2c + 6 * (long long)ym + 4);   // (j-1, k-1)
+        const int xmzm = __ldg(c2c + 6 * (long long)xm + 4);   // (i-1, k-1)
+        const int xmym = __ldg(c2c + 6 * (long long)xm + 2);   // (i-1, j-1)
+        const double *A = acc;
+        // x edge: cells (i,j,k) (-,-), (i,j-1,k) (+,-), (i,j,k-1) (-,+), (i,j-1,k-1) (+,+)
+        double jx = add(add(add(A[kEmNA * c + 0], A[kEmNA * (long long)ym + 1]),
+                            A[kEmNA * (long long)zm + 2]), A[kEmNA * (long long)ymzm + 3]);
+        // y edge (transverse z, x): (i,j,k), (i,j,k-1), (i-1,j,k), (i-1,j,k-1)
+        double jy = add(add(add(A[kEmNA * c + 4], A[kEmNA * (long long)zm + 5]),
+                            A[kEmNA * (long long)xm + 6]), A[kEmNA * (long long)xmzm + 7]);
+        // z edge (transverse x, y): (i,j,k), (i-1,j,k), (i,j-1,k), (i-1,j-1,k)
+        double jz = add(add(add(A[kEmNA * c + 8], A[kEmNA * (long long)xm + 9]),
+                            A[kEmNA * (long long)ym + 10]), A[kEmNA * (long long)xmym + 11]);
+        J[c] = dvd(jx, sx);
+        J[nc + c] = dvd(jy, sy);
+        J[2 * nc + c] = dvd(jz, sz);
+    }
+}
+
+__global__ void k_em_advance_b(const double *__restrict__ e, double *__restrict__ b,
+                               const int32_t *__restrict__ c2c, long long nc, double hx, double hy,
+                               double hz, double fdt) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+         c += (long long)gridDim.x * blockDim.x) {
+        const int *nb = c2c + 6 * c;
+        const long long xp = nb[1], yp = nb[3], zp = nb[5];
+        const double ex = e[c], ey = e[nc + c], ez = e[2 * nc + c];
+        const double cx = sub(dvd(sub(e[2 * nc + yp], ez), hy), dvd(sub(e[nc + zp], ey), hz));
+        const double cy = sub(dvd(sub(e[zp], ex), hz), dvd(sub(e[2 * nc + xp], ez), hx));
+        const double cz = sub(dvd(sub(e[nc + xp], ey), hx), dvd(sub(e[yp], ex), hy));
+        b[c] = sub(b[c], mul(fdt, cx));
+        b[nc + c] = sub(b[nc + c], mul(fdt, cy));
+        b[2 * nc + c] = sub(b[2 * nc + c], mul(fdt, cz));
+    }
+}
+
+__global__ void k_em_advance_e(double *__restrict__ e, const double *__restrict__ b,
+                               const double *__restrict__ J, const int32_t *__restrict__ c2c,
+                               long long nc, double hx, double hy, double hz, double dt) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+         c += (long long)gridDim.x * blockDim.x) {
+        const int *nb = c2c + 6 * c;
+        const long long xm = nb[0], ym = nb[2], zm = nb[4];
+        const double bx = b[c], by = b[nc + c], bz = b[2 * nc + c];
+        const double cx = sub(dvd(sub(bz, b[2 * nc + ym]), hy), dvd(sub(by, b[nc + zm]), hz));
+        const double cy = sub(dvd(sub(bx, b[zm]), hz), dvd(sub(bz, b[2 * nc + xm]), hx));
+        const double cz = sub(dvd(sub(by, b[nc + xm]), hx), dvd(sub(bx, b[ym]), hy));
+        e[c] = add(e[c], mul(dt, sub(cx, J[c])));
+        e[nc + c] = add(e[nc + c], mul(dt, sub(cy, J[nc + c])));
+        e[2 * nc + c] = add(e[2 * nc + c], mul(dt, sub(cz, J[2 * nc + c])));
+    }
+}
+
 }  // namespace
+
+cudaError_t launch_em_accumulate_current(const double *acc, const int32_t *c2c, long long nc,
+                                         const double h[3], double dt, double *J, cudaStream_t s) {
+    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
+    // scale 2 dt h_b h_c, formed as the oracle forms it: (2.0 * dt) * h_b * h_c
+    const double sx = 2.0 * dt * h[1] * h[2], sy = 2.0 * dt * h[2] * h[0], sz = 2.0 * dt * h[0] * h[1];
+    k_em_accumulate_current<<<grid, 256, 0, s>>>(acc, c2c, nc, sx, sy, sz, J);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_advance_b(const double *e, double *b, const int32_t *c2c, long long nc,
+                                const double h[3], double fdt, cudaStream_t s) {
+    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
+    k_em_advance_b<<<grid, 256, 0, s>>>(e, b, c2c, nc, h[0], h[1], h[2], fdt);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_advance_e(double *e, const double *b, const double *J, const int32_t *c2c,
+                                long long nc, const double h[3], double dt, cudaStream_t s) {
+    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
+    k_em_advance_e<<<grid, 256, 0, s>>>(e, b, J, c2c, nc, h[0], h[1], h[2], dt);
+    return cudaGetLastError();
+}
+
 
 cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
                                   double *interp, cudaStream_t s) {

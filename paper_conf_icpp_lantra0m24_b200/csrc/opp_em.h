@@ -33,5 +33,11 @@ struct EmArgs {
 cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
                                   double *interp, cudaStream_t s);
 cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s);
+cudaError_t launch_em_accumulate_current(const double *acc, const int32_t *c2c, long long nc,
+                                         const double h[3], double dt, double *J, cudaStream_t s);
+cudaError_t launch_em_advance_b(const double *e, double *b, const int32_t *c2c, long long nc,
+                                const double h[3], double fdt, cudaStream_t s);
+cudaError_t launch_em_advance_e(double *e, const double *b, const double *J, const int32_t *c2c,
+                                long long nc, const double h[3], double dt, cudaStream_t s);
 
 }  // namespace opp

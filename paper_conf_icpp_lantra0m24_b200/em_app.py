@@ -5,8 +5,8 @@ map; per step the application runs the
 library's Move_Deposit on device-resident SoA particle
 columns.  This module only marshals arguments: Interpolate and Move_Deposit
 run in libopp's CUDA kernels (csrc/opp_em.cu); PyTorch holds the device
-memory and the stream.  AccumulateCurrent / AdvanceE / AdvanceB (the field
-leap-frog) are outside the particle loop and not built.
+memory and the stream.  ``field_step`` runs the field side (AccumulateCurrent,
+AdvanceB / AdvanceE leap-frog, Interpolate) in the library's kernels too.
 """
 from __future__ import annotations
 
@@ -71,6 +71,19 @@ class CabanaPicEM:
                               ao, au, aw, ac)
         self._alt = (self.off, self.u, self.w, self.cell)
         self.off, self.u, self.w, self.cell = ao, au, aw, ac
+
+    def field_step(self, dt: float, h=(1.0, 1.0, 1.0)) -> None:
+        """AccumulateCurrent -> AdvanceB(dt/2) -> AdvanceE(dt) -> AdvanceB(dt/2) ->
+        Interpolate, then the accumulator is cleared for the next Move_Deposit."""
+        c = self.ctx
+        if getattr(self, "J", None) is None:
+            self.J = self.torch.empty_like(self.e)
+        O.opp_em_accumulate_current(c, self.acc, self.c2c, self.nc, h, dt, self.J)
+        O.opp_em_advance_b(c, self.e, self.b, self.c2c, self.nc, h, dt / 2)
+        O.opp_em_advance_e(c, self.e, self.b, self.J, self.c2c, self.nc, h, dt)
+        O.opp_em_advance_b(c, self.e, self.b, self.c2c, self.nc, h, dt / 2)
+        self.interpolate()
+        self.acc.zero_()
 
     def zero_acc(self) -> None:
         self.acc.zero_()

@@ -31,7 +31,7 @@ EXPORTS = (
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
     "opp_field_init", "opp_field_solve", "opp_get_field_stats",
     "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats", "opp_em_sort_by_cell",
-    "opp_shuffle",
+    "opp_shuffle", "opp_em_accumulate_current", "opp_em_advance_b", "opp_em_advance_e",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
           "sort_count", "sort_move", "field", "em_move_deposit")
@@ -140,6 +140,9 @@ def _load():
                                     C.POINTER(opp_em_params), C.POINTER(opp_em_stats)]),
         "opp_em_get_stats": (I, [P, C.POINTER(opp_em_stats)]),
         "opp_em_sort_by_cell": (I, [P, I64, I64, P, P, P, P, I64, P, P, P, P]),
+        "opp_em_accumulate_current": (I, [P, P, P, I64, P, C.c_double, P]),
+        "opp_em_advance_b": (I, [P, P, P, P, I64, P, C.c_double]),
+        "opp_em_advance_e": (I, [P, P, P, P, P, I64, P, C.c_double]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -361,3 +364,19 @@ def opp_em_sort_by_cell(ctx, n: int, stride: int, off, u, w, cell, n_cells: int,
     _ck(lib.opp_em_sort_by_cell(ctx, int(n), int(stride), _ptr(off), _ptr(u), _ptr(w), _ptr(cell),
                                 int(n_cells), _ptr(off_out), _ptr(u_out), _ptr(w_out),
                                 _ptr(cell_out)))
+
+
+def _h3(h):
+    return (C.c_double * 3)(*[float(x) for x in h])
+
+
+def opp_em_accumulate_current(ctx, acc, c2c, n_cells: int, h, dt: float, J) -> None:
+    _ck(lib.opp_em_accumulate_current(ctx, _ptr(acc), _ptr(c2c), int(n_cells), _h3(h), float(dt), _ptr(J)))
+
+
+def opp_em_advance_b(ctx, e, b, c2c, n_cells: int, h, frac_dt: float) -> None:
+    _ck(lib.opp_em_advance_b(ctx, _ptr(e), _ptr(b), _ptr(c2c), int(n_cells), _h3(h), float(frac_dt)))
+
+
+def opp_em_advance_e(ctx, e, b, J, c2c, n_cells: int, h, dt: float) -> None:
+    _ck(lib.opp_em_advance_e(ctx, _ptr(e), _ptr(b), _ptr(J), _ptr(c2c), int(n_cells), _h3(h), float(dt)))

@@ -245,3 +245,105 @@ def test_em_face_start_and_rest_edge_cases():
     sim.close()
     _check((o_off, o_u, o_cell, acc, ost), g, gst)
     assert ost[0]["n_crossings"] >= 6
+
+
+def test_em_field_kernels_bit_exact():
+    """AccumulateCurrent / AdvanceB / AdvanceE (C ABI) equal oracle/em_field.py bit for bit."""
+    import oracle.em_field as F
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    nx, ny, nz, h, dt = 5, 4, 6, (1.0, 0.8, 1.25), 0.3
+    rng = np.random.default_rng(9)
+    nc = nx * ny * nz
+    e0, b0 = rng.uniform(-1, 1, (3, nc)), rng.uniform(-1, 1, (3, nc))
+    acc = rng.uniform(-1, 1, (nc, 12))
+    sim = _app(nx, ny, nz, e0, b0, 0.05, [1, 1, 1])
+    dev = sim.dev
+    ta = torch.from_numpy(acc).to(dev)
+    J = torch.empty((3, nc), dtype=torch.float64, device=dev)
+    O.opp_em_accumulate_current(sim.ctx, ta, sim.c2c, nc, h, dt, J)
+    Jo = F.accumulate_current(acc, nx, ny, nz, h, dt)
+    assert np.array_equal(J.cpu().numpy(), Jo)
+    O.opp_em_advance_b(sim.ctx, sim.e, sim.b, sim.c2c, nc, h, dt / 2)
+    eo, bo = e0.copy(), b0.copy()
+    F.advance_b(eo, bo, nx, ny, nz, h, dt / 2)
+    assert np.array_equal(sim.b.cpu().numpy(), bo)
+    O.opp_em_advance_e(sim.ctx, sim.e, sim.b, J, sim.c2c, nc, h, dt)
+    F.advance_e(eo, bo, Jo, nx, ny, nz, h, dt)
+    assert np.array_equal(sim.e.cpu().numpy(), eo)
+    with pytest.raises(O.OppError):
+        O.opp_em_advance_e(sim.ctx, sim.e, sim.b, J, sim.c2c, nc, (1.0, 0.0, 1.0), dt)
+    sim.close()
+
+
+def test_em_full_pic_loop_vs_oracle():
+    """Move_Deposit + AccumulateCurrent + AdvanceB/E/B + Interpolate, 4 steps,
+    GPU against the oracle loop: fields within 1e-12, particles within
+    1e-10 relative (the reduction order of the deposit perturbs the fields at
+    the 1e-16 level and the next pushes through them)."""
+    import oracle.em_field as F
+    nx, ny, nz, ppc, seed = 4, 4, 5, 30, 21
+    h, dt, qdt, cdt = (1.0, 1.0, 1.0), 0.5, 0.05, [1.0, 1.0, 1.0]
+    e, b = G.em_fields(nx, ny, nz, seed, e_amp=0.05, b0=0.4, b_amp=0.05)
+    p = _inputs(nx, ny, nz, ppc, seed, False, v0=0.4, vth=0.05)
+    c2c = G.periodic_hex(nx, ny, nz)
+    o_off, o_u, o_cell = p["off"].copy(), p["u"].copy(), p["cell"].copy()
+    eo, bo = e.copy(), b.copy()
+    prm = OE.params(qdt, cdt, 1.0, 16)
+    sim = _app(nx, ny, nz, e, b, qdt, cdt)
+    sim.set_particles(p["off"], p["u"], p["w"], p["cell"])
+    g0 = F.div_e(eo, nx, ny, nz, h) - F.node_charge_density(o_off, o_cell, p["w"], 1.0, nx, ny, nz, h)
+    for _ in range(4):
+        acc = np.zeros((nx * ny * nz, 12))
+        OE.move_deposit(prm, o_off, o_u, p["w"], o_cell, OE.interpolate(nx, ny, nz, eo, bo), c2c, acc)
+        J = F.accumulate_current(acc, nx, ny, nz, h, dt)
+        F.advance_b(eo, bo, nx, ny, nz, h, dt / 2)
+        F.advance_e(eo, bo, J, nx, ny, nz, h, dt)
+        F.advance_b(eo, bo, nx, ny, nz, h, dt / 2)
+        sim.step()
+        sim.field_step(dt, h)
+    g = sim.state()
+    ge, gb = sim.e.cpu().numpy(), sim.b.cpu().numpy()
+    sim.close()
+    np.testing.assert_allclose(ge, eo, rtol=0, atol=1e-12)
+    np.testing.assert_allclose(gb, bo, rtol=0, atol=1e-12)
+    assert np.array_equal(g["cell"], o_cell)
+    np.testing.assert_allclose(g["off"], o_off, rtol=1e-10, atol=1e-13)
+    np.testing.assert_allclose(g["u"], o_u, rtol=1e-10, atol=1e-13)
+    # Gauss's law held on the GPU run too
+    g1 = F.div_e(ge, nx, ny, nz, h) - F.node_charge_density(g["off"], g["cell"], p["w"], 1.0, nx, ny, nz, h)
+    np.testing.assert_allclose(g1, g0, rtol=0, atol=1e-11)
+
+
+def test_em_full_size_gauss_law():
+    """C3 at full size through one full PIC step (Move_Deposit + field side):
+    div E - rho at every node is unchanged (continuity of the Eq. 11 deposit +
+    the AccumulateCurrent scale + AdvanceE), and div B stays 0."""
+    import gen.cuda as GC
+    from paper_conf_icpp_lantra0m24_b200.em_app import CabanaPicEM
+    nx, ny, nz, ppc, seed = 40, 40, 60, 750, 20240814
+    h, dt = (1.0, 1.0, 1.0), 0.5
+    e, b = G.em_fields(nx, ny, nz, seed, e_amp=1e-2, b0=0.5, b_amp=1e-2)
+    sim = CabanaPicEM(nx, ny, nz, G.periodic_hex(nx, ny, nz), e, b, 0.05, [1.0, 1.0, 1.0])
+    d = GC.em_two_stream(nx, ny, nz, ppc, seed)
+    sim.set_particles(d["off"], d["u"], d["w"], d["cell"])
+    nc = nx * ny * nz
+
+    def div_e(ev):
+        E = ev.view(3, nz, ny, nx)
+        return ((E[0] - torch.roll(E[0], 1, 2)) + (E[1] - torch.roll(E[1], 1, 1)) +
+                (E[2] - torch.roll(E[2], 1, 0))).reshape(-1)
+
+    def div_b(bv):
+        B = bv.view(3, nz, ny, nx)
+        return ((torch.roll(B[0], -1, 2) - B[0]) + (torch.roll(B[1], -1, 1) - B[1]) +
+                (torch.roll(B[2], -1, 0) - B[2])).reshape(-1)
+    rho0 = _node_weights_t(sim.off, sim.cell, sim.w, nx, ny, nz)
+    g0 = div_e(sim.e) - rho0
+    db0 = div_b(sim.b)
+    sim.step()
+    sim.field_step(dt, h)
+    rho1 = _node_weights_t(sim.off, sim.cell, sim.w, nx, ny, nz)
+    g1 = div_e(sim.e) - rho1
+    assert (g1 - g0).abs().max().item() <= 1e-9
+    assert (div_b(sim.b) - db0).abs().max().item() <= 1e-12
+    sim.close()
