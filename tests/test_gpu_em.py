@@ -347,3 +347,39 @@ def test_em_full_size_gauss_law():
     assert (g1 - g0).abs().max().item() <= 1e-9
     assert (div_b(sim.b) - db0).abs().max().item() <= 1e-12
     sim.close()
+
+
+def test_em_two_stream_growth_rate_gpu():
+    """The cold two-stream instability through the product path (Move_Deposit +
+    field side kernels, C ABI) grows at the textbook rate omega_b / 2 within
+    10% -- the setup of tests/test_oracle_em_twostream.py at 4x the particles."""
+    nx, ny, nz, ppc = 1, 1, 16, 4096
+    h, dt, qdt = (1.0, 1.0, 1.0), 0.5, 0.05
+    k = 2 * np.pi / nz
+    v0 = 0.1
+    wb = 2 * k * v0 / np.sqrt(3.0)
+    qsp = 2 * wb ** 2 / ((2 * qdt / dt) * ppc)
+    n = nz * ppc
+    half = ppc // 2
+    cell = np.repeat(np.arange(nz, dtype=np.int32), ppc)
+    j = np.tile(np.arange(ppc), nz)
+    offz = -1.0 + (2.0 * (j // 2) + 1.0) / half
+    off = np.stack([np.zeros(n), np.zeros(n), offz])
+    zpos = cell + (offz + 1.0) / 2.0
+    u = np.zeros((3, n))
+    u[2] = np.where(j % 2 == 0, 1.0, -1.0) * v0 + 1e-5 * v0 * np.sin(k * zpos)
+    from paper_conf_icpp_lantra0m24_b200.em_app import CabanaPicEM
+    sim = CabanaPicEM(nx, ny, nz, G.periodic_hex(nx, ny, nz), np.zeros((3, nz)), np.zeros((3, nz)),
+                      qdt, [2 * dt / h[0]] * 3, qsp)
+    sim.set_particles(off, u, np.ones(n), cell)
+    steps, amps = 760, []
+    for _ in range(steps):
+        sim.step()
+        sim.field_step(dt, h)
+        amps.append(sim.e[2].clone())
+    ez = torch.stack(amps).cpu().numpy()
+    sim.close()
+    a = np.abs(np.fft.rfft(ez, axis=1)[:, 1])
+    t = dt * (np.arange(steps) + 1)
+    gamma = np.polyfit(t[450:750], np.log(a[450:750]), 1)[0]
+    assert abs(gamma - wb / 2) <= 0.10 * wb / 2, (gamma, wb / 2)
