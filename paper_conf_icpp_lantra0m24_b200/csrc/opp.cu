@@ -162,6 +162,10 @@ struct opp_ctx_s {
     MeshCache mc;
     FieldState fs;
     opp::EmCounters *em_cnt = nullptr;   // opp_em_move_deposit statistics (device)
+    uint32_t *em_work = nullptr;         // deferred face crossers (continuation worklist)
+    long long em_work_cap = 0;
+    int em_defer = 0;                    // OPP_EM_DEFER=1: face crossers finish in a continuation pass
+                                         // (C3: 4.16 -> 5.17 ms, parity green: off)
     struct {                             // opp_em_sort_by_cell scratch
         unsigned *hist = nullptr, *start = nullptr;
         unsigned long long *tile_sums = nullptr;
@@ -371,6 +375,7 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.n2cs, 0);
     free_field(c);
     c->dfree(c->em_cnt, sizeof(opp::EmCounters));
+    c->dfree(c->em_work, 0);
     c->dfree(c->em_sort.hist, 0);
     c->dfree(c->em_sort.start, 0);
     c->dfree(c->em_sort.tile_sums, 0);
@@ -1947,10 +1952,19 @@ extern "C" int opp_em_move_deposit(opp_ctx c, int64_t n, int64_t stride, double 
     a.kcap = prm->kcap;
     a.dep = prm->deposit_mode == OPP_DEP_ATOMIC_WARPAGG ? 1 : 0;
     a.cnt = c->em_cnt;
+    if (const char *ed = getenv("OPP_EM_DEFER")) c->em_defer = atoi(ed);
+    if (c->em_defer && n > c->em_work_cap) {
+        c->dfree(c->em_work, 0);
+        c->em_work = (uint32_t *)c->dalloc(4 * (size_t)n);
+        if (!c->em_work) return fail(OPP_ERR_NOMEM, "em worklist");
+        c->em_work_cap = n;
+    }
+    a.work = c->em_defer ? c->em_work : nullptr;
+    if (n > (long long)UINT32_MAX) a.work = nullptr;
     if (n > 0) {
         PhaseScope ph(c, OPP_PH_EM_MOVE_DEPOSIT);
         CK(opp::launch_em_move_deposit(a, c->nsm, c->s));
-        c->launches += 1;
+        c->launches += (a.work && a.kcap > 0) ? 2 : 1;
     }
     if (stats) return opp_em_get_stats(c, stats);
     return OPP_OK;

@@ -271,10 +271,62 @@ __device__ __forceinline__ void em_deposit(double *__restrict__ acc, bool has, i
     }
 }
 
+// Face hit by the streak d from p (first along the path; t = 1 ends inside)
+// and the segment's end point q (exactly on the face when one is hit).
+__device__ __forceinline__ int em_face(const double p[3], const double d[3], double q[3]) {
+    double t = 1.0;
+    int face = -1;
+    // one division site per axis (the oracle's two branches differ only in
+    // the numerator): divergent lanes would otherwise run both
+#pragma unroll
+    for (int ax = 0; ax < 3; ax++) {
+        const bool pos = d[ax] > 0.0;
+        if (d[ax] != 0.0) {
+            const double ta = dvd(sub(pos ? 1.0 : -1.0, p[ax]), d[ax]);
+            if (ta < t) { t = ta; face = 2 * ax + (pos ? 1 : 0); }
+        }
+    }
+#pragma unroll
+    for (int ax = 0; ax < 3; ax++) q[ax] = add(p[ax], mul(t, d[ax]));
+    if (face >= 0) {
+        const double fv = (face & 1) ? 1.0 : -1.0;
+        const int fa = face >> 1;
+        q[0] = fa == 0 ? fv : q[0];
+        q[1] = fa == 1 ? fv : q[1];
+        q[2] = fa == 2 ? fv : q[2];
+    }
+    return face;
+}
+
+// Cross `face`: the rest of the streak continues from the face point in the
+// neighbour, with the offset along the face axis flipped.
+__device__ __forceinline__ void em_cross(double p[3], double d[3], const double q[3], int face,
+                                         int &c, const int32_t *__restrict__ c2c) {
+#pragma unroll
+    for (int ax = 0; ax < 3; ax++) {
+        d[ax] = sub(d[ax], sub(q[ax], p[ax]));
+        p[ax] = q[ax];
+    }
+    const int fa = face >> 1;
+    p[0] = fa == 0 ? -p[0] : p[0];
+    p[1] = fa == 1 ? -p[1] : p[1];
+    p[2] = fa == 2 ? -p[2] : p[2];
+    c = __ldg(c2c + 6 * (long long)c + face);
+}
+
+// Streak of the (already pushed) momentum u, offset units.
+__device__ __forceinline__ void em_streak(const EmArgs &a, const double uu[3], double d[3]) {
+    const double rg = dvd(1.0, __dsqrt_rn(add(1.0, add(add(mul(uu[0], uu[0]), mul(uu[1], uu[1])),
+                                                         mul(uu[2], uu[2])))));
+    d[0] = mul(a.cdt[0], mul(uu[0], rg));
+    d[1] = mul(a.cdt[1], mul(uu[1], rg));
+    d[2] = mul(a.cdt[2], mul(uu[2], rg));
+}
+
 #ifndef OPP_EM_MINB
 #define OPP_EM_MINB 3   // resident blocks per SM (80 registers); 4 spills and measured slower
 #endif
-template <int DEP>
+template <int DEP, bool DEFER>
 __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
     __shared__ double em_buf[OPP_EM_SMEM_SUM ? 8 : 1][OPP_EM_SMEM_SUM ? kEmNA * kEmBufLd : 1];
@@ -331,44 +383,25 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
             m2 = add(m2, sub(mul(p0, s1), mul(p1, s0)));
             uu[0] = add(m0, h0); uu[1] = add(m1, h1); uu[2] = add(m2, h2);
             // 3. streak in offset units
-            const double rg = dvd(1.0, __dsqrt_rn(add(1.0, add(add(mul(uu[0], uu[0]), mul(uu[1], uu[1])),
-                                                                 mul(uu[2], uu[2])))));
-            d[0] = mul(a.cdt[0], mul(uu[0], rg));
-            d[1] = mul(a.cdt[1], mul(uu[1], rg));
-            d[2] = mul(a.cdt[2], mul(uu[2], rg));
+            em_streak(a, uu, d);
             Q = mul(a.qsp, w);
             a.u[i] = uu[0]; a.u[a.cap + i] = uu[1]; a.u[2 * a.cap + i] = uu[2];
         }
         // 4. move through the faces crossed; one segment per lane per round,
-        //    deposited warp-aggregated (rounds continue while any lane moves)
+        //    deposited warp-aggregated (rounds continue while any lane moves).
+        //    DEFER: only the first round runs here; particles that cross a face
+        //    (~10% per step on C3) go to a worklist that k_em_move_continue
+        //    finishes in full warps (a later round with a few active lanes
+        //    costs a whole warp pass of the move)
         bool moving = valid;
         int k = 0;
-        bool capped = false;
+        bool capped = false, deferred = false;
         while (__any_sync(FULL, moving)) {
             double v[kEmNA];
             int face = -1;
             double q[3] = {p[0], p[1], p[2]};
             if (moving) {
-                double t = 1.0;
-                // one division site per axis (the oracle's two branches differ only
-                // in the numerator): divergent lanes would otherwise run both
-#pragma unroll
-                for (int ax = 0; ax < 3; ax++) {
-                    const bool pos = d[ax] > 0.0;
-                    if (d[ax] != 0.0) {
-                        const double ta = dvd(sub(pos ? 1.0 : -1.0, p[ax]), d[ax]);
-                        if (ta < t) { t = ta; face = 2 * ax + (pos ? 1 : 0); }
-                    }
-                }
-#pragma unroll
-                for (int ax = 0; ax < 3; ax++) q[ax] = add(p[ax], mul(t, d[ax]));
-                if (face >= 0) {
-                    const double fv = (face & 1) ? 1.0 : -1.0;
-                    const int fa = face >> 1;
-                    q[0] = fa == 0 ? fv : q[0];
-                    q[1] = fa == 1 ? fv : q[1];
-                    q[2] = fa == 2 ? fv : q[2];
-                }
+                face = em_face(p, d, q);
                 seg_current(p, q, Q, v);
             } else {
 #pragma unroll
@@ -383,28 +416,90 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                     p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
                     capped = true;
                     moving = false;
+                } else if (DEFER) {
+                    deferred = true;
+                    moving = false;
                 } else {
-#pragma unroll
-                    for (int ax = 0; ax < 3; ax++) {
-                        d[ax] = sub(d[ax], sub(q[ax], p[ax]));
-                        p[ax] = q[ax];
-                    }
-                    const int fa = face >> 1;
-                    p[0] = fa == 0 ? -p[0] : p[0];
-                    p[1] = fa == 1 ? -p[1] : p[1];
-                    p[2] = fa == 2 ? -p[2] : p[2];
-                    c = __ldg(a.c2c + 6 * (long long)c + face);
+                    em_cross(p, d, q, face, c, a.c2c);
                     k++;
                 }
             }
         }
-        if (valid) {
+        if (DEFER) {
+            const unsigned m = __ballot_sync(FULL, deferred);
+            if (m) {
+                unsigned long long base = 0;
+                if (lane == (unsigned)(__ffs(m) - 1)) base = atomicAdd(&a.cnt->n_work, (unsigned long long)__popc(m));
+                base = __shfl_sync(FULL, base, __ffs(m) - 1);
+                if (deferred) a.work[base + __popc(m & ((1u << lane) - 1u))] = (uint32_t)i;
+            }
+        }
+        if (valid && !deferred) {
             a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
             a.cell[i] = c;
             ncross += (unsigned)k;
             ncap += capped;
             maxk = max(maxk, (unsigned)k);
         }
+    }
+    const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
+    const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
+    const unsigned mk = __reduce_max_sync(FULL, maxk);
+    if (lane == 0) {
+        if (sc) atomicAdd(&a.cnt->n_crossings, (unsigned long long)sc);
+        if (scap) atomicAdd(&a.cnt->n_capped, (unsigned long long)scap);
+        if (mk) atomicMax(&a.cnt->max_crossings, mk);
+    }
+}
+
+// Continuation of the deferred particles: one particle per lane, lanes fully
+// independent (the deposit reduces directly: the particles are few and in
+// scattered cells).  The first round is recomputed bit for bit from the
+// stored state (offsets not yet written, u already pushed) and not deposited
+// again; the later rounds are deposited.
+__global__ void __launch_bounds__(256) k_em_move_continue(EmArgs a) {
+    const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    const unsigned long long nw = *(volatile unsigned long long *)&a.cnt->n_work;
+    unsigned long long ncross = 0, ncap = 0;
+    unsigned maxk = 0;
+    for (unsigned long long w = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; w < nw;
+         w += (unsigned long long)gridDim.x * blockDim.x) {
+        const long long i = a.work[w];
+        int c = a.cell[i];
+        double p[3] = {a.off[i], a.off[a.cap + i], a.off[2 * a.cap + i]};
+        const double uu[3] = {a.u[i], a.u[a.cap + i], a.u[2 * a.cap + i]};
+        const double Q = mul(a.qsp, a.w[i]);
+        double d[3];
+        em_streak(a, uu, d);
+        double q[3];
+        int face = em_face(p, d, q);   // round 1 (deposited by the first pass): crosses
+        em_cross(p, d, q, face, c, a.c2c);
+        int k = 1;
+        bool capped = false;
+        for (;;) {
+            double v[kEmNA];
+            face = em_face(p, d, q);
+            seg_current(p, q, Q, v);
+            double *acc = a.acc + (long long)kEmNA * c;
+#pragma unroll
+            for (int s = 0; s < kEmNA; s++) atomicAdd(acc + s, v[s]);
+            if (face < 0) {
+                p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
+                break;
+            }
+            if (k >= a.kcap) {
+                p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
+                capped = true;
+                break;
+            }
+            em_cross(p, d, q, face, c, a.c2c);
+            k++;
+        }
+        a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
+        a.cell[i] = c;
+        ncross += (unsigned)k;
+        ncap += capped;
+        maxk = max(maxk, (unsigned)k);
     }
     const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
     const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
@@ -518,15 +613,22 @@ cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const
 }
 
 cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
+    const bool defer = a.work != nullptr && a.kcap > 0;
     int per = 0;
     if (a.dep == 1)
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<1>, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<1, false>, 256, 0);
     else
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<0>, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<0, false>, 256, 0);
     const long long need = (a.n + 255) / 256;
     const long long grid = std::max(1LL, std::min<long long>(need, (long long)nsm * std::max(per, 1)));
-    if (a.dep == 1) k_em_move_deposit<1><<<(int)grid, 256, 0, s>>>(a);
-    else k_em_move_deposit<0><<<(int)grid, 256, 0, s>>>(a);
+    if (a.dep == 1) {
+        if (defer) k_em_move_deposit<1, true><<<(int)grid, 256, 0, s>>>(a);
+        else k_em_move_deposit<1, false><<<(int)grid, 256, 0, s>>>(a);
+    } else {
+        if (defer) k_em_move_deposit<0, true><<<(int)grid, 256, 0, s>>>(a);
+        else k_em_move_deposit<0, false><<<(int)grid, 256, 0, s>>>(a);
+    }
+    if (defer) k_em_move_continue<<<(int)std::min<long long>(grid, (long long)nsm * 8), 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 

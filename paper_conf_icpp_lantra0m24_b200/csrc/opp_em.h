@@ -13,6 +13,7 @@ constexpr int kEmNA = 12;   // accumulator doubles per cell (jx[4], jy[4], jz[4]
 struct EmCounters {
     unsigned long long n_crossings, n_capped;
     unsigned max_crossings, pad;
+    unsigned long long n_work;   // particles deferred to the continuation pass
 };
 
 struct EmArgs {
@@ -28,6 +29,7 @@ struct EmArgs {
     int kcap;
     int dep;                   // 0: 12 reductions per segment and lane; 1: warp-aggregated
     EmCounters *cnt;
+    uint32_t *work;            // deferred particles (face crossers), capacity >= n; null: no deferral
 };
 
 cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
