@@ -323,14 +323,107 @@ __device__ __forceinline__ void em_streak(const EmArgs &a, const double uu[3], d
     d[2] = mul(a.cdt[2], mul(uu[2], rg));
 }
 
+// Per-warp queue of particles still crossing faces (OPP_EM_QUEUE): their later
+// move rounds run in batches of 32, so a round never runs for a handful of
+// lanes (a round costs the warp the same ~250 instructions for 2 lanes as
+// for 32).  Ring of kEmQ slots in shared memory: position, remaining streak,
+// cell, crossings so far, particle index.
+constexpr int kEmQ = 64;
+struct EmQueue {
+    double *p[3], *d[3];
+    int *c, *k, *i;
+    unsigned head, tail;   // warp-uniform
+    __device__ __forceinline__ unsigned count() const { return tail - head; }
+    __device__ __forceinline__ void push(bool pred, const double pp[3], const double dd[3], int cc,
+                                         int kk, int ii) {
+        const unsigned m = __ballot_sync(0xffffffffu, pred);
+        if (!m) return;
+        const unsigned lane = threadIdx.x & 31u;
+        if (pred) {
+            const unsigned sl = (tail + __popc(m & ((1u << lane) - 1u))) & (kEmQ - 1);
+            p[0][sl] = pp[0]; p[1][sl] = pp[1]; p[2][sl] = pp[2];
+            d[0][sl] = dd[0]; d[1][sl] = dd[1]; d[2][sl] = dd[2];
+            c[sl] = cc; k[sl] = kk; i[sl] = ii;
+        }
+        tail += __popc(m);
+        __syncwarp();
+    }
+};
+constexpr int kEmQBytes = kEmQ * (6 * 8 + 3 * 4);                  // per warp
+constexpr int kEmBufBytes = kEmNA * kEmBufLd * 8;                   // per warp
+#ifndef OPP_EM_QUEUE
+#define OPP_EM_QUEUE 1   // C3: 4.16 -> 3.77 ms with direct reductions for the queued rounds
+#endif
+#ifndef OPP_EM_QDEP
+#define OPP_EM_QDEP 0    // 1: warp-aggregated deposits for queued rounds (scattered cells: 4.56 ms)
+#endif
+
 #ifndef OPP_EM_MINB
 #define OPP_EM_MINB 3   // resident blocks per SM (80 registers); 4 spills and measured slower
 #endif
-template <int DEP, bool DEFER>
+// One move round for up to 32 queued particles (lane j takes entry head + j).
+template <int DEP>
+__device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, double *wbuf,
+                                               unsigned long long &ncross, unsigned long long &ncap,
+                                               unsigned &maxk) {
+    const unsigned lane = threadIdx.x & 31u;
+    const unsigned take = min(32u, qs.count());
+    const bool has = lane < take;
+    double p[3] = {0, 0, 0}, d[3] = {0, 0, 0};
+    int c = 0, k = 0, i = 0;
+    if (has) {
+        const unsigned sl = (qs.head + lane) & (kEmQ - 1);
+        p[0] = qs.p[0][sl]; p[1] = qs.p[1][sl]; p[2] = qs.p[2][sl];
+        d[0] = qs.d[0][sl]; d[1] = qs.d[1][sl]; d[2] = qs.d[2][sl];
+        c = qs.c[sl]; k = qs.k[sl]; i = qs.i[sl];
+    }
+    __syncwarp();
+    qs.head += take;
+    double v[kEmNA], q[3] = {p[0], p[1], p[2]};
+    int face = -1;
+    if (has) {
+        face = em_face(p, d, q);
+        seg_current(p, q, mul(a.qsp, __ldg(a.w + i)), v);
+    } else {
+#pragma unroll
+        for (int s = 0; s < kEmNA; s++) v[s] = 0.0;
+    }
+    // queued particles sit in scattered cells: direct reductions (OPP_EM_QDEP=1: warp-aggregated)
+    em_deposit<OPP_EM_QDEP ? DEP : 0>(a.acc, has, c, v, wbuf);
+    bool again = false, capped = false;
+    if (has) {
+        if (face >= 0 && k < a.kcap) {
+            em_cross(p, d, q, face, c, a.c2c);
+            k++;
+            again = true;
+        } else {
+            capped = face >= 0;
+            a.off[i] = q[0]; a.off[a.cap + i] = q[1]; a.off[2 * a.cap + i] = q[2];
+            a.cell[i] = c;
+            ncross += (unsigned)k;
+            ncap += capped;
+            maxk = max(maxk, (unsigned)k);
+        }
+    }
+    qs.push(again, p, d, c, k, i);
+}
+
+template <int DEP, bool DEFER, bool QUEUE>
 __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
-    __shared__ double em_buf[OPP_EM_SMEM_SUM ? 8 : 1][OPP_EM_SMEM_SUM ? kEmNA * kEmBufLd : 1];
-    double *wbuf = em_buf[OPP_EM_SMEM_SUM ? (threadIdx.x >> 5) : 0];
+    extern __shared__ __align__(16) char em_dyn[];   // per warp: transpose buffer, then the queue
+    char *wbase = em_dyn + (size_t)(threadIdx.x >> 5) * (kEmBufBytes + (QUEUE ? kEmQBytes : 0));
+    double *wbuf = reinterpret_cast<double *>(wbase);
+    EmQueue qs{};
+    if (QUEUE) {
+        char *qb = wbase + kEmBufBytes;
+        for (int a_ = 0; a_ < 3; a_++) qs.p[a_] = reinterpret_cast<double *>(qb + a_ * kEmQ * 8);
+        for (int a_ = 0; a_ < 3; a_++) qs.d[a_] = reinterpret_cast<double *>(qb + (3 + a_) * kEmQ * 8);
+        qs.c = reinterpret_cast<int *>(qb + 6 * kEmQ * 8);
+        qs.k = qs.c + kEmQ;
+        qs.i = qs.k + kEmQ;
+        qs.head = qs.tail = 0;
+    }
     const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
     const long long gw = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     unsigned long long ncross = 0, ncap = 0;
@@ -395,7 +488,7 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
         //    costs a whole warp pass of the move)
         bool moving = valid;
         int k = 0;
-        bool capped = false, deferred = false;
+        bool capped = false, deferred = false, queued = false;
         while (__any_sync(FULL, moving)) {
             double v[kEmNA];
             int face = -1;
@@ -419,6 +512,11 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                 } else if (DEFER) {
                     deferred = true;
                     moving = false;
+                } else if (QUEUE) {
+                    em_cross(p, d, q, face, c, a.c2c);
+                    k++;
+                    queued = true;
+                    moving = false;
                 } else {
                     em_cross(p, d, q, face, c, a.c2c);
                     k++;
@@ -434,14 +532,20 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                 if (deferred) a.work[base + __popc(m & ((1u << lane) - 1u))] = (uint32_t)i;
             }
         }
-        if (valid && !deferred) {
+        if (valid && !deferred && !queued) {
             a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
             a.cell[i] = c;
             ncross += (unsigned)k;
             ncap += capped;
             maxk = max(maxk, (unsigned)k);
         }
+        if (QUEUE) {
+            qs.push(queued, p, d, c, k, (int)i);
+            while (qs.count() >= 32) em_queue_round<DEP>(a, qs, wbuf, ncross, ncap, maxk);
+        }
     }
+    if (QUEUE)
+        while (qs.count() > 0) em_queue_round<DEP>(a, qs, wbuf, ncross, ncap, maxk);
     const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
     const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
     const unsigned mk = __reduce_max_sync(FULL, maxk);
@@ -612,22 +716,37 @@ cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const
     return cudaGetLastError();
 }
 
-cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
-    const bool defer = a.work != nullptr && a.kcap > 0;
+template <int DEP, bool DEFER, bool QUEUE>
+static cudaError_t em_launch(const EmArgs &a, int nsm, cudaStream_t s, long long *grid_out) {
+    const int smem = 8 * (kEmBufBytes + (QUEUE ? kEmQBytes : 0));
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_em_move_deposit<DEP, DEFER, QUEUE>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
     int per = 0;
-    if (a.dep == 1)
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<1, false>, 256, 0);
-    else
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<0, false>, 256, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<DEP, DEFER, QUEUE>, 256, smem);
     const long long need = (a.n + 255) / 256;
     const long long grid = std::max(1LL, std::min<long long>(need, (long long)nsm * std::max(per, 1)));
-    if (a.dep == 1) {
-        if (defer) k_em_move_deposit<1, true><<<(int)grid, 256, 0, s>>>(a);
-        else k_em_move_deposit<1, false><<<(int)grid, 256, 0, s>>>(a);
-    } else {
-        if (defer) k_em_move_deposit<0, true><<<(int)grid, 256, 0, s>>>(a);
-        else k_em_move_deposit<0, false><<<(int)grid, 256, 0, s>>>(a);
-    }
+    k_em_move_deposit<DEP, DEFER, QUEUE><<<(int)grid, 256, smem, s>>>(a);
+    *grid_out = grid;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
+    const bool defer = a.work != nullptr && a.kcap > 0;
+    const bool queue = !defer && OPP_EM_QUEUE && a.kcap > 0 && a.n < (1LL << 31);
+    long long grid = 1;
+    cudaError_t e;
+    if (a.dep == 1)
+        e = defer ? em_launch<1, true, false>(a, nsm, s, &grid)
+                  : queue ? em_launch<1, false, true>(a, nsm, s, &grid) : em_launch<1, false, false>(a, nsm, s, &grid);
+    else
+        e = defer ? em_launch<0, true, false>(a, nsm, s, &grid)
+                  : queue ? em_launch<0, false, true>(a, nsm, s, &grid) : em_launch<0, false, false>(a, nsm, s, &grid);
+    if (e != cudaSuccess) return e;
     if (defer) k_em_move_continue<<<(int)std::min<long long>(grid, (long long)nsm * 8), 256, 0, s>>>(a);
     return cudaGetLastError();
 }
