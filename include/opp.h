@@ -344,6 +344,53 @@ int opp_field_solve(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential, op
 int opp_get_field_stats(opp_ctx ctx, opp_field_stats *stats);
 
 /* ---------------------------------------------------------------------------
+ * Boltzmann-electron field solve: the nonlinear
+ * Poisson problem Mini-FEM-PIC solves by Newton's method with
+ * ComputeF1Vector, ComputeJMatrix and a linear solver (PETSc KSP in the
+ * paper; §4.1.1).  The paper names the routines only;
+ * DESIGN.md §11 readings B1-B4 fix the formulas (normalised units):
+ *   F_n(phi) = (K phi)_n - rhs_scale Q_n + ne_coef m_n exp((phi_n - phi0) / te)
+ *   on free nodes (Dirichlet nodes hold dirichlet_value), m_n the lumped P1
+ *   mass (sum over the node's cells of |V_e| / 4);
+ *   J = K + diag(ne_coef m_n / te exp((phi_n - phi0) / te));
+ *   Newton: J_FF delta_F = -F_F (Jacobi-)preconditioned CG to cg_tol relative
+ *   to ||F_F||, phi_F += delta_F; start phi_F = phi0 (or the warm start);
+ *   stop when ||F_F||_2 <= max(newton_tol ||F_F(phi_start)||_2, newton_atol)
+ *   or after max_newton steps.
+ * Needs opp_field_init (same matrix, Dirichlet data and n2c).  One rank only
+ * (OPP_ERR_STATE when nranks > 1).  node_charge / node_potential / cell_ef
+ * as in opp_field_solve.  The loop is host-driven: one ||F|| read-back per
+ * Newton step (synchronises).  Errors: OPP_ERR_ARG (te <= 0, ne_coef < 0,
+ * tolerances < 0, max_newton / cg_max_iter < 0, NULL params), OPP_ERR_STATE,
+ * OPP_ERR_NOMEM, OPP_ERR_CUDA.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+    double rhs_scale;   /* ion load b = rhs_scale * node_charge                          */
+    double ne_coef;     /* electron term coefficient (n0 e / eps0 in solver units), >= 0 */
+    double phi0;        /* reference potential (electron density = n0 at phi0)          */
+    double te;          /* electron temperature in potential units (kTe / e), > 0       */
+    double newton_tol;  /* relative stopping tolerance on ||F_F||_2 (>= 0)              */
+    double newton_atol; /* absolute stopping tolerance on ||F_F||_2 (>= 0)              */
+    double cg_tol;      /* inner CG: ||r|| <= cg_tol * ||F_F|| (>= 0)                    */
+    int max_newton;     /* Newton step cap (>= 0)                                        */
+    int cg_max_iter;    /* inner CG iteration cap per Newton step (>= 0)                 */
+    int warm_start;     /* 1: free nodes start from node_potential's values; 0: phi0     */
+    int precond;        /* inner CG: 0 plain, 1 Jacobi (J's diagonal)                    */
+} opp_boltzmann_params;
+
+typedef struct {
+    int32_t newton_steps;   /* Newton steps taken                                        */
+    int32_t converged;      /* 1 if the stopping rule was met                            */
+    int64_t cg_iterations;  /* inner CG iterations summed over the steps                 */
+    double res_norm;        /* ||F_F(phi)||_2 at exit                                    */
+    double res0_norm;       /* ||F_F(phi_start)||_2                                      */
+} opp_boltzmann_stats;
+
+int opp_field_solve_boltzmann(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential,
+                              opp_dat cell_ef, const opp_boltzmann_params *params,
+                              opp_boltzmann_stats *stats);
+
+/* ---------------------------------------------------------------------------
  * CabanaPIC-style electromagnetic particle loop (config C3; SURVEY.md §8(f)
  * NEXT-2): hex cells of a periodic nx*ny*nz grid declared as an unstructured
  * mesh through their cell-to-cell map.

@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.environ.get("OPP_LIB_OUT", os.path.join(HERE, "libopp.so"))
-SOURCES = ["opp.cu", "opp_kernels.cu", "opp_comm.cu", "opp_field.cu", "opp_em.cu"]
+SOURCES = ["opp.cu", "opp_kernels.cu", "opp_comm.cu", "opp_field.cu", "opp_em.cu", "opp_boltz.cu"]
 HEADERS = ["opp_internal.h", "opp_kernels.h", "opp_comm.h", "opp_field.h", "opp_em.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 

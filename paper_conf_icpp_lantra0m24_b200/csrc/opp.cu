@@ -137,6 +137,14 @@ struct FieldState {
     double *own = nullptr, *hvec = nullptr, *dots = nullptr;
     bool host_stats = false;
     opp_field_stats hst{};
+    // Boltzmann-electron Newton solve (allocated on first use): lumped mass,
+    // Jacobian values / Jacobi diagonal, zero Dirichlet data, the CG load -F,
+    // the Newton update, block partials of ||F||^2 and the norm (+ pinned copy)
+    double *bz_m = nullptr, *bz_jval = nullptr, *bz_jdinv = nullptr, *bz_zero = nullptr;
+    double *bz_rhs = nullptr, *bz_delta = nullptr, *bz_part = nullptr, *bz_norm = nullptr;
+    double *bz_host = nullptr;
+    int bz_nblk = 0;
+    opp_boltzmann_stats bst{};
 };
 
 }  // namespace
@@ -347,6 +355,9 @@ static void free_field(opp_ctx c) {
     c->dfree(f.n2c_ptr, 0); c->dfree(f.n2c, 0); c->dfree(f.vec, 0); c->dfree(f.part, 0);
     c->dfree(f.st, 0);
     c->dfree(f.own, 0); c->dfree(f.hvec, 0); c->dfree(f.dots, 0);
+    c->dfree(f.bz_m, 0); c->dfree(f.bz_jval, 0); c->dfree(f.bz_jdinv, 0); c->dfree(f.bz_zero, 0);
+    c->dfree(f.bz_rhs, 0); c->dfree(f.bz_delta, 0); c->dfree(f.bz_part, 0); c->dfree(f.bz_norm, 0);
+    if (f.bz_host) cudaFreeHost(f.bz_host);
     f = FieldState();
 }
 
@@ -2033,5 +2044,146 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     }
     c->cols[node_potential].version++;
     if (stats) return opp_get_field_stats(c, stats);
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Boltzmann-electron field solve (
+// DESIGN.md §11 readings B1-B4): Newton on F(phi) with the fused
+// ComputeF1Vector + ComputeJMatrix pass (k_newton_eval) and the persistent
+// CG kernel on the Jacobian.  Host-driven: one ||F|| read-back per step.
+// ---------------------------------------------------------------------------
+static int boltz_alloc(opp_ctx c) {
+    FieldState &f = c->fs;
+    if (f.bz_m) return OPP_OK;
+    const long long nn = std::max<long long>(f.nn, 1), nnz = std::max<long long>(f.K.nnz_pad, 1);
+    f.bz_nblk = newton_eval_blocks(f.K, c->nsm);
+    f.bz_m = (double *)c->dalloc(8 * nn);
+    f.bz_jval = (double *)c->dalloc(8 * nnz);
+    f.bz_jdinv = (double *)c->dalloc(8 * nn);
+    f.bz_zero = (double *)c->dalloc(8 * nn);
+    f.bz_rhs = (double *)c->dalloc(8 * nn);
+    f.bz_delta = (double *)c->dalloc(8 * nn);
+    f.bz_part = (double *)c->dalloc(8 * (size_t)f.bz_nblk);
+    f.bz_norm = (double *)c->dalloc(8 * 2);
+    if (cudaMallocHost(&f.bz_host, 64) != cudaSuccess) f.bz_host = nullptr;
+    if (!f.bz_m || !f.bz_jval || !f.bz_jdinv || !f.bz_zero || !f.bz_rhs || !f.bz_delta ||
+        !f.bz_part || !f.bz_norm || !f.bz_host) {
+        c->dfree(f.bz_m, 0); c->dfree(f.bz_jval, 0); c->dfree(f.bz_jdinv, 0); c->dfree(f.bz_zero, 0);
+        c->dfree(f.bz_rhs, 0); c->dfree(f.bz_delta, 0); c->dfree(f.bz_part, 0); c->dfree(f.bz_norm, 0);
+        if (f.bz_host) cudaFreeHost(f.bz_host);
+        f.bz_m = f.bz_jval = f.bz_jdinv = f.bz_zero = f.bz_rhs = f.bz_delta = f.bz_part = nullptr;
+        f.bz_norm = f.bz_host = nullptr;
+        return fail(OPP_ERR_NOMEM, "Boltzmann solve buffers");
+    }
+    CK(cudaMemsetAsync(f.bz_zero, 0, 8 * nn, c->s));
+    const Col &cn = c->cols[f.c2n];
+    CK(launch_lumped_mass((const double *)c->cols[f.node_pos].d, (const int32_t *)cn.d, f.n2c_ptr,
+                          f.n2c, f.nn, f.bz_m, c->s));
+    c->launches++;
+    return OPP_OK;
+}
+
+extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat node_potential,
+                                         opp_dat cell_ef, const opp_boltzmann_params *prm,
+                                         opp_boltzmann_stats *stats) {
+    TRY(ctx_check(c));
+    FieldState &f = c->fs;
+    if (!f.ready) return fail(OPP_ERR_STATE, "opp_field_init first");
+    if (c->p.nranks > 1) return fail(OPP_ERR_STATE, "the Boltzmann solve runs on one rank only");
+    if (!prm) return fail(OPP_ERR_ARG, "null Boltzmann params");
+    if (!(prm->te > 0.0) || !(prm->ne_coef >= 0.0) || !(prm->newton_tol >= 0.0) ||
+        !(prm->newton_atol >= 0.0) || !(prm->cg_tol >= 0.0) || prm->max_newton < 0 ||
+        prm->cg_max_iter < 0 || !std::isfinite(prm->phi0) || !std::isfinite(prm->rhs_scale))
+        return fail(OPP_ERR_ARG, "te > 0, ne_coef >= 0, tolerances >= 0, caps >= 0, finite phi0");
+    const Col &cn = c->cols[f.c2n];
+    const int nodes = cn.to, cells = cn.set;
+    TRY(check_col(c, node_charge, false, nodes, 1, OPP_REAL, "node_charge"));
+    TRY(check_col(c, node_potential, false, nodes, 1, OPP_REAL, "node_potential"));
+    if (cell_ef >= 0) TRY(check_col(c, cell_ef, false, cells, 3, OPP_REAL, "cell_ef"));
+    TRY(boltz_alloc(c));
+    const long long nn = f.nn;
+    double *phi = (double *)c->cols[node_potential].d;
+    const double *Q = (const double *)c->cols[node_charge].d;
+    opp_boltzmann_stats bs{};
+    {
+        PhaseScope ph(c, OPP_PH_FIELD);
+        if (nn > 0) {
+            CK(launch_newton_start(f.K, phi, prm->phi0, prm->warm_start != 0, c->s));
+            c->launches++;
+            NewtonCoef co{prm->rhs_scale, prm->ne_coef, prm->phi0, 1.0 / prm->te};
+            FieldMat J = f.K;
+            J.val = f.bz_jval;
+            J.dinv = f.bz_jdinv;
+            J.dval = f.bz_zero;
+            CgArgs a{};
+            a.K = J;
+            a.Q = f.bz_rhs;
+            a.x = f.bz_delta;
+            a.r = f.vec;
+            a.u = f.vec + nn;
+            a.w = f.vec + 2 * nn;
+            a.p = f.vec + 3 * nn;
+            a.s = f.vec + 4 * nn;
+            a.m0 = f.vec + 5 * nn;
+            a.m1 = f.vec + 6 * nn;
+            a.z = f.vec + 7 * nn;
+            a.q = f.vec + 8 * nn;
+            a.pipelined = 1;
+            a.part = f.part;
+            a.st = f.st;
+            a.rhs_scale = 1.0;
+            a.tol = prm->cg_tol;
+            a.max_iter = prm->cg_max_iter;
+            a.warm = 0;
+            a.precond = prm->precond != 0;
+            int bps = 2;
+            if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
+            bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
+            double thr = 0.0;
+            for (int k = 0;; k++) {
+                CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, phi, f.bz_m, co, f.bz_rhs,
+                                      f.bz_part, f.bz_nblk, f.bz_norm, c->s));
+                c->launches += 2;
+                CK(cudaMemcpyAsync(f.bz_host, f.bz_norm, 8, cudaMemcpyDeviceToHost, c->s));
+                if (k > 0) CK(cudaMemcpyAsync(f.bz_host + 1, f.st, sizeof(int), cudaMemcpyDeviceToHost, c->s));
+                CK(cudaStreamSynchronize(c->s));
+                const double fn = std::sqrt(f.bz_host[0]);
+                if (k > 0) {
+                    int it;
+                    memcpy(&it, f.bz_host + 1, sizeof(int));
+                    bs.cg_iterations += it;
+                }
+                if (!std::isfinite(fn)) return fail(OPP_ERR_STATE, "Newton diverged (||F|| not finite)");
+                if (k == 0) {
+                    bs.res0_norm = fn;
+                    thr = std::max(prm->newton_tol * fn, prm->newton_atol);
+                }
+                bs.res_norm = fn;
+                bs.newton_steps = k;
+                if (fn <= thr) { bs.converged = 1; break; }
+                if (k >= prm->max_newton) break;
+                int grid = 0;
+                CK(launch_cg(a, c->nsm, bps, c->s, &grid));
+                CK(launch_newton_update(f.K, phi, f.bz_delta, c->s));
+                c->launches += 2;
+            }
+        } else {
+            bs.converged = 1;
+        }
+        if (cell_ef >= 0) {
+            Col &ef = c->cols[cell_ef];
+            MeshCache &m = c->mc;
+            const bool packed = m.efp && m.ef == cell_ef && m.nc == f.nc;
+            CK(launch_efield((const double *)c->cols[f.node_pos].d, (const int32_t *)cn.d, phi, f.nc,
+                             (double *)ef.d, packed ? m.efp : nullptr, c->s));
+            c->launches++;
+            ef.version++;
+            if (packed) m.vef = ef.version;
+        }
+    }
+    c->cols[node_potential].version++;
+    f.bst = bs;
+    if (stats) *stats = bs;
     return OPP_OK;
 }

@@ -85,3 +85,26 @@ cudaError_t launch_cg_update(const FieldMat &K, double alpha, double beta, doubl
 cudaError_t launch_diag(const FieldMat &K, double *diag, cudaStream_t s);
 cudaError_t launch_dinv(const FieldMat &K, const double *diag, cudaStream_t s);
 }  // namespace opp
+
+// ---- Boltzmann-electron Newton solve (opp_boltz.cu; SURVEY.md §8(f) NEXT-4,
+// DESIGN.md §11 readings B1-B4)
+namespace opp {
+struct NewtonCoef {
+    double rhs_scale, ne, phi0, inv_te;
+};
+// m_n = sum over the node's cells of |V_e| / 4 (lumped P1 mass)
+cudaError_t launch_lumped_mass(const double *xyz, const int32_t *c2n, const int32_t *n2c_ptr,
+                               const int32_t *n2c, long long nn, double *m, cudaStream_t s);
+// blocks of k_newton_eval (= the partial count launch_newton_eval reduces)
+int newton_eval_blocks(const FieldMat &K, int nsm);
+// One pass over K: rhsv = -F(phi) (0 on Dirichlet rows), jval / jdinv = the
+// Jacobian's values and Jacobi inverse diagonal, *norm2 = ||F||^2 (fixed order).
+cudaError_t launch_newton_eval(const FieldMat &K, double *jval, double *jdinv, const double *Q,
+                               const double *phi, const double *m, const NewtonCoef &co,
+                               double *rhsv, double *part, int nblk, double *norm2,
+                               cudaStream_t s);
+cudaError_t launch_newton_start(const FieldMat &K, double *phi, double phi0, int warm,
+                                cudaStream_t s);
+cudaError_t launch_newton_update(const FieldMat &K, double *phi, const double *delta,
+                                 cudaStream_t s);
+}  // namespace opp

@@ -29,7 +29,7 @@ EXPORTS = (
     "opp_get_node_charge", "opp_get_dat", "opp_set_dat", "opp_get_particle_count",
     "opp_get_dat_device_ptr", "opp_kernel_launch_count", "opp_sync", "opp_last_error",
     "opp_phase_timing", "opp_get_phase_times", "opp_get_step_stats", "opp_sort_by_cell",
-    "opp_field_init", "opp_field_solve", "opp_get_field_stats",
+    "opp_field_init", "opp_field_solve", "opp_get_field_stats", "opp_field_solve_boltzmann",
     "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats", "opp_em_sort_by_cell",
     "opp_shuffle", "opp_em_accumulate_current", "opp_em_advance_b", "opp_em_advance_e",
 )
@@ -75,6 +75,22 @@ class opp_step_stats(C.Structure):
 class opp_field_params(C.Structure):
     _fields_ = [("rhs_scale", C.c_double), ("tol", C.c_double), ("max_iter", C.c_int),
                 ("warm_start", C.c_int), ("precond", C.c_int)]
+
+
+class opp_boltzmann_params(C.Structure):
+    _fields_ = [("rhs_scale", C.c_double), ("ne_coef", C.c_double), ("phi0", C.c_double),
+                ("te", C.c_double), ("newton_tol", C.c_double), ("newton_atol", C.c_double),
+                ("cg_tol", C.c_double), ("max_newton", C.c_int), ("cg_max_iter", C.c_int),
+                ("warm_start", C.c_int), ("precond", C.c_int)]
+
+
+class opp_boltzmann_stats(C.Structure):
+    _fields_ = [("newton_steps", C.c_int32), ("converged", C.c_int32),
+                ("cg_iterations", C.c_int64), ("res_norm", C.c_double),
+                ("res0_norm", C.c_double)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 class opp_field_stats(C.Structure):
@@ -135,6 +151,8 @@ def _load():
         "opp_field_solve": (I, [P, I32, I32, I32, C.POINTER(opp_field_params),
                                 C.POINTER(opp_field_stats)]),
         "opp_get_field_stats": (I, [P, C.POINTER(opp_field_stats)]),
+        "opp_field_solve_boltzmann": (I, [P, I32, I32, I32, C.POINTER(opp_boltzmann_params),
+                                          C.POINTER(opp_boltzmann_stats)]),
         "opp_em_interpolate": (I, [P, I, I, I, P, P, P]),
         "opp_em_move_deposit": (I, [P, I64, I64, P, P, P, P, P, P, I64, P,
                                     C.POINTER(opp_em_params), C.POINTER(opp_em_stats)]),
@@ -324,6 +342,14 @@ def opp_field_solve(ctx, node_charge: int, node_potential: int, cell_ef: int,
     st = opp_field_stats() if want_stats else None
     _ck(lib.opp_field_solve(ctx, node_charge, node_potential, cell_ef, C.byref(params),
                             C.byref(st) if st else None))
+    return st
+
+
+def opp_field_solve_boltzmann(ctx, node_charge: int, node_potential: int, cell_ef: int,
+                              params: opp_boltzmann_params) -> opp_boltzmann_stats:
+    st = opp_boltzmann_stats()
+    _ck(lib.opp_field_solve_boltzmann(ctx, node_charge, node_potential, cell_ef,
+                                      C.byref(params), C.byref(st)))
     return st
 
 

@@ -1,0 +1,156 @@
+"""CUDA Boltzmann-electron Newton field solve vs its oracle (oracle/boltzmann.py), -m gpu.
+
+The GPU runs the fused ComputeF1Vector + ComputeJMatrix pass and the
+persistent CG on the Jacobian (opp_field_solve_boltzmann through the C ABI);
+the oracle runs exact Newton steps (sparse direct solves) from the same
+start.  Both stop on the same rule (reading B4); the GPU's inner CG stops at
+cg_tol relative to ||F||, so the two potentials agree to the order of
+newton_tol * ||F_0|| / lambda_min(J) -- the bound the tolerances below follow
+(DESIGN.md §11).  The GPU answer's own residual is evaluated independently
+by the oracle's residual_vector.
+"""
+import time
+
+import numpy as np
+import pytest
+
+import gen
+from oracle import boltzmann as B
+from oracle import field as F
+
+pytestmark = pytest.mark.gpu
+
+
+def _sim(mesh):
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    return MiniFemPic(mesh, np.zeros((mesh["n_cells"], 3)))
+
+
+def _set(sim, handle, arr):
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    O.opp_set_dat(sim.ctx, handle, np.ascontiguousarray(arr, np.float64), sim.nn)
+
+
+def _solve_both(mesh, Q, mask, val, rhs_scale, ne, phi0, te, precond=1, newton_tol=1e-10):
+    xyz, c2n = mesh["node_xyz"], mesh["c2n"]
+    K = F.stiffness(xyz, c2n)
+    M = B.lumped_mass(xyz, c2n)
+    phi_o, k_o, hist = B.newton(K, Q, M, mask, val, rhs_scale, ne, phi0, te, tol=newton_tol)
+    sim = _sim(mesh)
+    sim.field_init(mask, val)
+    _set(sim, sim.node_charge, Q)
+    st = sim.field_solve_boltzmann(rhs_scale, ne, phi0, te, newton_tol=newton_tol, cg_tol=1e-13,
+                                   precond=bool(precond))
+    phi = sim.potential_host()
+    E = sim.field_host()
+    launches = sim.launches()
+    sim.close()
+    assert launches > 0
+    Fg = B.residual_vector(K, Q, M, phi, mask, rhs_scale, ne, phi0, te)
+    return dict(K=K, M=M, phi_o=phi_o, k_o=k_o, hist=hist, st=st, phi=phi, E=E, Fg=Fg)
+
+
+@pytest.mark.parametrize("precond", [0, 1])
+@pytest.mark.parametrize("dims,jit", [((6, 6, 30), 0.2), ((5, 3, 7), 0.1), ((1, 1, 1), 0.0)])
+def test_boltzmann_matches_newton_oracle(dims, jit, precond):
+    mesh = gen.kuhn_duct(*dims, jitter=jit, seed=9)
+    rng = np.random.default_rng(4)
+    Q = rng.uniform(0.0, 2.0, mesh["n_nodes"])          # deposited ion charge per node
+    mask, val = gen.duct_bc(mesh, wall=3.0, inlet=0.0)
+    r = _solve_both(mesh, Q, mask, val, rhs_scale=0.5, ne=0.8, phi0=0.0, te=1.5, precond=precond)
+    st, phi, phi_o = r["st"], r["phi"], r["phi_o"]
+    assert st["converged"] == 1
+    assert abs(st["newton_steps"] - r["k_o"]) <= 1
+    assert st["res0_norm"] == pytest.approx(r["hist"][0], rel=1e-12)
+    assert np.linalg.norm(r["Fg"]) <= 10 * 1e-10 * r["hist"][0]
+    free = mask == 0
+    np.testing.assert_array_equal(phi[~free], val[~free])
+    scale = np.abs(phi_o).max()
+    assert np.abs(phi - phi_o).max() <= 1e-8 * scale
+    Eo = F.efield(mesh["node_xyz"], mesh["c2n"], phi_o)
+    assert np.abs(r["E"] - Eo).max() <= 1e-7 * max(np.abs(Eo).max(), 1.0)
+
+
+def test_boltzmann_zero_electron_term_is_linear_solve():
+    mesh = gen.kuhn_duct(4, 3, 6, jitter=0.2, seed=5)
+    Q = np.random.default_rng(2).uniform(0, 3, mesh["n_nodes"])
+    mask, val = gen.duct_bc(mesh, wall=0.3, inlet=0.0)
+    r = _solve_both(mesh, Q, mask, val, rhs_scale=0.02, ne=0.0, phi0=0.0, te=1.0)
+    ref = F.solve(r["K"], F.load_vector(Q, 0.02), mask, val)
+    assert r["st"]["newton_steps"] == 1
+    assert np.abs(r["phi"] - ref).max() <= 1e-9 * np.abs(ref).max()
+
+
+def test_boltzmann_debye_sheath_closed_form():
+    """Small-amplitude sheath through the GPU path: the discrete Debye profile."""
+    nz, lam, te = 60, 5.0, 1.0
+    mesh = gen.kuhn_duct(2, 2, nz)
+    ne = te / lam ** 2
+    A = 1e-6
+    M = B.lumped_mass(mesh["node_xyz"], mesh["c2n"])
+    mask, val = gen.duct_bc(mesh, inlet=A, outlet=0.0)
+    sim = _sim(mesh)
+    sim.field_init(mask, val)
+    _set(sim, sim.node_charge, ne * M)                   # uniform ion background
+    # ||F_0|| ~ 1e-6 here, its rounding floor ~1e-17: stop on the absolute rule
+    st = sim.field_solve_boltzmann(1.0, ne, 0.0, te, newton_tol=0.0, newton_atol=1e-15,
+                                   cg_tol=1e-14)
+    phi = sim.potential_host()
+    sim.close()
+    z = mesh["node_xyz"][:, 2]
+    th = np.arccosh(1.0 + 1.0 / (2.0 * lam ** 2))
+    ex = A * np.sinh((nz - z) * th) / np.sinh(nz * th)
+    assert st["converged"] == 1
+    assert np.abs(phi - ex).max() <= 1e-5 * A
+
+
+def test_boltzmann_warm_start_and_errors():
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    mesh = gen.kuhn_duct(3, 3, 6, jitter=0.1, seed=1)
+    Q = np.random.default_rng(3).uniform(0, 1, mesh["n_nodes"])
+    mask, val = gen.duct_bc(mesh, wall=2.0)
+    sim = _sim(mesh)
+    with pytest.raises(O.OppError):                      # before opp_field_init
+        sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0)
+    sim.field_init(mask, val)
+    _set(sim, sim.node_charge, Q)
+    with pytest.raises(O.OppError):
+        sim.field_solve_boltzmann(1.0, 1.0, 0.0, 0.0)    # te must be > 0
+    with pytest.raises(O.OppError):
+        sim.field_solve_boltzmann(1.0, -1.0, 0.0, 1.0)   # ne_coef >= 0
+    st = sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0, newton_atol=1e-9)
+    assert st["converged"] == 1 and st["newton_steps"] >= 2
+    st2 = sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0, newton_atol=1e-9, warm_start=True)
+    assert st2["converged"] == 1 and st2["newton_steps"] == 0 and st2["cg_iterations"] == 0
+    st3 = sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0, max_newton=1)
+    assert st3["newton_steps"] == 1 and st3["converged"] == 0
+    sim.close()
+
+
+def test_boltzmann_full_size_c2_residual():
+    """C2 mesh (48x48x72 hex, 175,273 nodes): the oracle checks the GPU answer's
+    residual and the max principle bounds; time of the solve printed."""
+    mesh = gen.kuhn_duct(48, 48, 72, jitter=0.2, seed=2)
+    xyz, c2n = mesh["node_xyz"], mesh["c2n"]
+    nn = mesh["n_nodes"]
+    M = B.lumped_mass(xyz, c2n)
+    # ions: quasi-uniform background with a 20% random modulation
+    Q = M * (1.0 + 0.2 * np.random.default_rng(8).uniform(-1, 1, nn))
+    mask, val = gen.duct_bc(mesh, wall=4.0, inlet=0.0)
+    sim = _sim(mesh)
+    sim.field_init(mask, val)
+    _set(sim, sim.node_charge, Q)
+    sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0)       # warm-up (allocations, mass)
+    t = time.perf_counter()
+    st = sim.field_solve_boltzmann(1.0, 1.0, 0.0, 1.0, newton_tol=1e-10, cg_tol=1e-12)
+    dt = time.perf_counter() - t
+    phi = sim.potential_host()
+    sim.close()
+    K = F.stiffness(xyz, c2n)
+    Fg = B.residual_vector(K, Q, M, phi, mask, 1.0, 1.0, 0.0, 1.0)
+    print(f"C2 Boltzmann solve: {dt * 1e3:.1f} ms, {st}")
+    assert st["converged"] == 1
+    assert np.linalg.norm(Fg) <= 10 * 1e-10 * st["res0_norm"]
+    # ion density in [0.8, 1.2] n0 -> the free potential lies between the
+    # quasi-neutral levels te ln 0.8 and the wall potential
+    assert phi.min() >= np.log(0.8) - 1e-9 and phi.max() <= 4.0 + 1e-9
