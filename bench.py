@@ -65,6 +65,13 @@ def parse():
     ap.add_argument("--rhs", type=float, default=2e-7, help="field solve: b = rhs * node charge")
     ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
     ap.add_argument("--cg-tol", type=float, default=1e-10)
+    ap.add_argument("--field-model", choices=("linear", "boltzmann"), default="linear",
+                    help="field solve: linear Poisson CG (north_star) or the Boltzmann-electron "
+                         "Newton solve (PAPER.md:1604-1612, DESIGN.md §11; one GPU)")
+    ap.add_argument("--te", type=float, default=0.01, help="boltzmann: electron temperature (potential units)")
+    ap.add_argument("--ne", type=float, default=-1.0,
+                    help="boltzmann: electron coefficient (default: the mean ion load per volume, "
+                         "rhs * w * n0 / duct volume, so electrons balance ions at phi0 = 0)")
     ap.add_argument("--ppc", type=int, default=750, help="c3: particles per cell (750 = 72M, 1500 = 144M)")
     ap.add_argument("--em-sort", type=int, default=0, help="c3: sort particles by cell every K steps (0 = never)")
     args = ap.parse_args()
@@ -89,7 +96,9 @@ def workload(args, world=1):
     if cfg.get("cluster"):
         cluster = (cfg["cluster"], gen.hot_block_cells(mesh))
     name = {"c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
-                  "+ 250k injected/step, " + ("CG Poisson field solve every step" if args.field
+                  "+ 250k injected/step, " + (("Boltzmann-electron Newton field solve every step"
+                                               if args.field_model == "boltzmann" else
+                                               "CG Poisson field solve every step") if args.field
                                               else "fixed uniform E"),
             "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
             "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
@@ -468,8 +477,20 @@ def run_ours(args, rank, world):
                for s in range(total)]
     torch.cuda.synchronize()
 
+    boltz = args.field and args.field_model == "boltzmann"
+    if boltz and world > 1:
+        raise SystemExit("--field-model boltzmann runs on one GPU (DESIGN.md §11)")
+    if boltz and args.ne < 0:
+        x0, x1, y0, y1, z0, z1 = mesh["box"]
+        args.ne = args.rhs * w * n0 / ((x1 - x0) * (y1 - y0) * (z1 - z0))
+    bz_last = {}
+
     def field():
-        if args.field:
+        if boltz:
+            bz_last.update(sim.field_solve_boltzmann(args.rhs, args.ne, 0.0, args.te,
+                                                     newton_tol=args.cg_tol, cg_tol=1e-6,
+                                                     warm_start=True))
+        elif args.field:
             sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=True, stats=False)
 
     def one_step(s, on_device=True, readback=None):
@@ -561,7 +582,17 @@ def run_ours(args, rank, world):
                  "deferred_last_step": st1["n_deferred"]},
         "clocks": clk.summary(),
     }
-    if args.field:
+    if boltz:
+        line["field"] = {"ms_per_step": field_ms / args.steps, "model": "boltzmann",
+                         "last_solve": bz_last, "newton_tol": args.cg_tol, "inner_cg_tol": 1e-6,
+                         "ne_coef": args.ne, "te": args.te, "rhs_scale": args.rhs,
+                         "wall_potential": args.wall,
+                         "solver": "Newton: fused F/J pass + Jacobi-PCG persistent kernel, warm start, "
+                                   "host-driven (one ||F|| read-back per Newton step)",
+                         "note": "value excludes the field solve (timed separately, SURVEY.md "
+                                 "§8(d)); value_incl_field counts it"}
+        line["value_incl_field"] = pushed / (ms / 1e3)
+    elif args.field:
         fst = sim.field_stats()
         line["field"] = {"ms_per_step": field_ms / args.steps, "cg_iterations_last": fst["iterations"],
                          "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
