@@ -65,6 +65,8 @@ def parse():
     ap.add_argument("--rhs", type=float, default=2e-7, help="field solve: b = rhs * node charge")
     ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
     ap.add_argument("--cg-tol", type=float, default=1e-10)
+    ap.add_argument("--cg-warm", type=int, default=2,
+                    help="linear field solve start: 1 = last solution, 2 = extrapolated from the last two")
     ap.add_argument("--field-model", choices=("linear", "boltzmann"), default="linear",
                     help="field solve: linear Poisson CG (north_star) or the Boltzmann-electron "
                          "Newton solve (PAPER.md:1604-1612, DESIGN.md §11; one GPU)")
@@ -491,7 +493,7 @@ def run_ours(args, rank, world):
                                                      newton_tol=args.cg_tol, cg_tol=1e-6,
                                                      warm_start=True))
         elif args.field:
-            sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=True, stats=False)
+            sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=args.cg_warm, stats=False)
 
     def one_step(s, on_device=True, readback=None):
         field()
@@ -597,7 +599,7 @@ def run_ours(args, rank, world):
         line["field"] = {"ms_per_step": field_ms / args.steps, "cg_iterations_last": fst["iterations"],
                          "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
                          "rhs_scale": args.rhs, "wall_potential": args.wall,
-                         "solver": ("Jacobi-PCG, one persistent cooperative kernel, warm start"
+                         "solver": ("Jacobi-PCG, one persistent cooperative kernel, warm start " + ("extrapolated from the last two solutions" if args.cg_warm == 2 else "from the last solution")
                                     if world == 1 else "Jacobi-PCG over slabs (node halo + "
                                     "cross-rank dots, host-driven), warm start"),
                          "note": "value excludes the field solve (timed separately, SURVEY.md "

@@ -305,7 +305,10 @@ typedef struct {
     double rhs_scale;   /* b = rhs_scale * node_charge (q / eps0 per unit weight)       */
     double tol;         /* stop when ||r||_2 <= tol * ||b_F - K_FD phi_D||_2 (>= 0)      */
     int max_iter;       /* iteration cap (>= 0)                                          */
-    int warm_start;     /* 1: free nodes start from node_potential's current values     */
+    int warm_start;     /* 1: free nodes start from node_potential's current values;
+                           2: from 2 phi_{n-1} - phi_{n-2}, the linear extrapolation of the
+                           last two solutions of warm-start-2 solves into this dat (the
+                           first such solve starts like 1); 0: from 0                   */
     int precond;        /* 0: plain CG; 1: Jacobi (diagonal) preconditioned CG          */
 } opp_field_params;
 

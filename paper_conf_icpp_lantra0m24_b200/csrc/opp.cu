@@ -144,6 +144,9 @@ struct FieldState {
     double *bz_rhs = nullptr, *bz_delta = nullptr, *bz_part = nullptr, *bz_norm = nullptr;
     double *bz_host = nullptr;
     int bz_nblk = 0;
+    // warm_start 2: the solution before the last one (-1: no history yet)
+    double *xprev = nullptr;
+    int xprev_dat = -1;
     opp_boltzmann_stats bst{};
 };
 
@@ -358,6 +361,7 @@ static void free_field(opp_ctx c) {
     c->dfree(f.bz_m, 0); c->dfree(f.bz_jval, 0); c->dfree(f.bz_jdinv, 0); c->dfree(f.bz_zero, 0);
     c->dfree(f.bz_rhs, 0); c->dfree(f.bz_delta, 0); c->dfree(f.bz_part, 0); c->dfree(f.bz_norm, 0);
     if (f.bz_host) cudaFreeHost(f.bz_host);
+    c->dfree(f.xprev, 0);
     f = FieldState();
 }
 
@@ -2016,6 +2020,18 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     a.max_iter = prm->max_iter;
     a.warm = prm->warm_start != 0;
     a.precond = prm->precond != 0;
+    if (prm->warm_start == 2 && nn > 0) {
+        // extrapolate from the last two solutions into this potential dat
+        if (!f.xprev) {
+            f.xprev = (double *)c->dalloc(8 * nn);
+            if (!f.xprev) return fail(OPP_ERR_NOMEM, "field extrapolation buffer");
+        }
+        if (f.xprev_dat != node_potential)
+            CK(cudaMemcpyAsync(f.xprev, a.x, 8 * nn, cudaMemcpyDeviceToDevice, c->s));
+        CK(launch_extrapolate(f.K, a.x, f.xprev, c->s));
+        c->launches++;
+        f.xprev_dat = node_potential;
+    }
     if (const char *e = getenv("OPP_CG_DBG")) a.dbg = atoi(e);
     {
         PhaseScope ph(c, OPP_PH_FIELD);

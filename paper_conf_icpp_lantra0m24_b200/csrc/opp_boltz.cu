@@ -131,6 +131,16 @@ __global__ void k_newton_update(FieldMat K, double *phi, const double *__restric
     if (!K.dmask[i]) phi[i] += delta[i];
 }
 
+// warm_start 2 of opp_field_solve: x0 = 2 x_{n-1} - x_{n-2} on free rows,
+// then xprev = x_{n-1} (linear extrapolation of the last two solutions)
+__global__ void k_extrapolate(FieldMat K, double *x, double *xprev) {
+    long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= K.nn || K.dmask[i]) return;
+    const double xc = x[i];
+    x[i] = 2.0 * xc - xprev[i];
+    xprev[i] = xc;
+}
+
 inline unsigned blocks_of(long long n) { return (unsigned)((n + kBzThreads - 1) / kBzThreads); }
 
 }  // namespace
@@ -168,6 +178,12 @@ cudaError_t launch_newton_update(const FieldMat &K, double *phi, const double *d
                                  cudaStream_t s) {
     if (K.nn <= 0) return cudaSuccess;
     k_newton_update<<<blocks_of(K.nn), kBzThreads, 0, s>>>(K, phi, delta);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_extrapolate(const FieldMat &K, double *x, double *xprev, cudaStream_t s) {
+    if (K.nn <= 0) return cudaSuccess;
+    k_extrapolate<<<blocks_of(K.nn), kBzThreads, 0, s>>>(K, x, xprev);
     return cudaGetLastError();
 }
 

@@ -105,6 +105,8 @@ cudaError_t launch_newton_eval(const FieldMat &K, double *jval, double *jdinv, c
                                cudaStream_t s);
 cudaError_t launch_newton_start(const FieldMat &K, double *phi, double phi0, int warm,
                                 cudaStream_t s);
+// free rows: x <- 2 x - xprev, xprev <- old x (warm_start 2 of opp_field_solve)
+cudaError_t launch_extrapolate(const FieldMat &K, double *x, double *xprev, cudaStream_t s);
 cudaError_t launch_newton_update(const FieldMat &K, double *phi, const double *delta,
                                  cudaStream_t s);
 }  // namespace opp

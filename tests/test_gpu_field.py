@@ -161,3 +161,32 @@ def test_pic_loop_with_field_solve_replay():
     sim.close()
     rep = compare(om, c2n, P.get(), Qo, removed, gout, Qg, w, v_ref=0.2371)
     assert rep["n_compared"] > 0.9 * n_inj * steps
+
+
+def test_field_extrapolated_warm_start():
+    """warm_start 2 (x0 = 2 phi_{n-1} - phi_{n-2}) changes the start only: every
+    solve of a drifting charge sequence still meets the CG bound against the
+    direct solve."""
+    mesh = gen.kuhn_duct(6, 6, 12, jitter=0.2, seed=6)
+    xyz, c2n = mesh["node_xyz"], mesh["c2n"]
+    mask, val = gen.duct_bc(mesh, wall=0.05, inlet=0.0)
+    K = F.stiffness(xyz, c2n)
+    rng = np.random.default_rng(3)
+    base, drift = rng.uniform(0, 5, mesh["n_nodes"]), rng.uniform(-1, 1, mesh["n_nodes"])
+    sim = _sim(mesh)
+    sim.field_init(mask, val)
+    its = []
+    for n in range(5):
+        Q = base + 0.1 * n * drift
+        _set_charge(sim, Q)
+        st = sim.field_solve(0.01, tol=1e-11, max_iter=5000, warm_start=2)
+        phi = sim.potential_host()
+        ref = F.solve(K, F.load_vector(Q, 0.01), mask, val)
+        assert st["converged"] == 1
+        assert F.residual(K, F.load_vector(Q, 0.01), mask, val, phi) <= 2e-11
+        assert np.abs(phi - ref).max() <= 1e-8 * np.abs(ref).max()
+        its.append(st["iterations"])
+    sim.close()
+    # a charge drifting linearly is extrapolated exactly: the later solves start
+    # at the answer (up to the previous solves' tolerance)
+    assert its[-1] < its[0]
