@@ -70,6 +70,8 @@ def parse():
     ap.add_argument("--field-model", choices=("linear", "boltzmann"), default="linear",
                     help="field solve: linear Poisson CG (north_star) or the Boltzmann-electron "
                          "Newton solve (PAPER.md:1604-1612, DESIGN.md §11; one GPU)")
+    ap.add_argument("--newton-cg-tol", type=float, default=1e-6,
+                    help="boltzmann: inner CG tolerance relative to ||F|| per Newton step")
     ap.add_argument("--te", type=float, default=0.01, help="boltzmann: electron temperature (potential units)")
     ap.add_argument("--ne", type=float, default=-1.0,
                     help="boltzmann: electron coefficient (default: the mean ion load per volume, "
@@ -490,7 +492,7 @@ def run_ours(args, rank, world):
     def field():
         if boltz:
             bz_last.update(sim.field_solve_boltzmann(args.rhs, args.ne, 0.0, args.te,
-                                                     newton_tol=args.cg_tol, cg_tol=1e-6,
+                                                     newton_tol=args.cg_tol, cg_tol=args.newton_cg_tol,
                                                      warm_start=True))
         elif args.field:
             sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=args.cg_warm, stats=False)
@@ -586,7 +588,7 @@ def run_ours(args, rank, world):
     }
     if boltz:
         line["field"] = {"ms_per_step": field_ms / args.steps, "model": "boltzmann",
-                         "last_solve": bz_last, "newton_tol": args.cg_tol, "inner_cg_tol": 1e-6,
+                         "last_solve": bz_last, "newton_tol": args.cg_tol, "inner_cg_tol": args.newton_cg_tol,
                          "ne_coef": args.ne, "te": args.te, "rhs_scale": args.rhs,
                          "wall_potential": args.wall,
                          "solver": "Newton: fused F/J pass + Jacobi-PCG persistent kernel, warm start, "
