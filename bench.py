@@ -493,7 +493,7 @@ def run_ours(args, rank, world):
         if boltz:
             bz_last.update(sim.field_solve_boltzmann(args.rhs, args.ne, 0.0, args.te,
                                                      newton_tol=args.cg_tol, cg_tol=args.newton_cg_tol,
-                                                     warm_start=True))
+                                                     warm_start=args.cg_warm))
         elif args.field:
             sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=args.cg_warm, stats=False)
 

@@ -358,8 +358,9 @@ int opp_get_field_stats(opp_ctx ctx, opp_field_stats *stats);
  *   J = K + diag(ne_coef m_n / te exp((phi_n - phi0) / te));
  *   Newton: J_FF delta_F = -F_F (Jacobi-)preconditioned CG to cg_tol relative
  *   to ||F_F||, phi_F += delta_F; start phi_F = phi0 (or the warm start);
- *   stop when ||F_F||_2 <= max(newton_tol ||F_F(phi_start)||_2, newton_atol)
- *   or after max_newton steps.
+ *   stop when ||F_F||_2 <= max(newton_tol ||F_F(phi_cold)||_2, newton_atol)
+ *   or after max_newton steps, phi_cold = the cold start (phi0 on free
+ *   nodes): a reference independent of the warm start.
  * Needs opp_field_init (same matrix, Dirichlet data and n2c).  One rank only
  * (OPP_ERR_STATE when nranks > 1).  node_charge / node_potential / cell_ef
  * as in opp_field_solve.  The loop is host-driven: one ||F|| read-back per
@@ -374,10 +375,14 @@ typedef struct {
     double te;          /* electron temperature in potential units (kTe / e), > 0       */
     double newton_tol;  /* relative stopping tolerance on ||F_F||_2 (>= 0)              */
     double newton_atol; /* absolute stopping tolerance on ||F_F||_2 (>= 0)              */
-    double cg_tol;      /* inner CG: ||r|| <= cg_tol * ||F_F|| (>= 0)                    */
+    double cg_tol;      /* inner CG: ||r|| <= cg_tol * ||F_F|| (>= 0); once ||F_F|| <= 1e-3
+                           of the reference (the linear regime) the step solves only
+                           as tightly as the stop needs: min(cg_tol, thr / (2 ||F_F||)) */
     int max_newton;     /* Newton step cap (>= 0)                                        */
     int cg_max_iter;    /* inner CG iteration cap per Newton step (>= 0)                 */
-    int warm_start;     /* 1: free nodes start from node_potential's values; 0: phi0     */
+    int warm_start;     /* 1: free nodes start from node_potential's values; 2: from the
+                           extrapolation of the last two warm-start-2 solutions (shared
+                           with opp_field_solve); 0: phi0                              */
     int precond;        /* inner CG: 0 plain, 1 Jacobi (J's diagonal)                    */
 } opp_boltzmann_params;
 
@@ -387,6 +392,7 @@ typedef struct {
     int64_t cg_iterations;  /* inner CG iterations summed over the steps                 */
     double res_norm;        /* ||F_F(phi)||_2 at exit                                    */
     double res0_norm;       /* ||F_F(phi_start)||_2                                      */
+    double ref_norm;        /* ||F_F(phi_cold)||_2, the stopping reference               */
 } opp_boltzmann_stats;
 
 int opp_field_solve_boltzmann(opp_ctx ctx, opp_dat node_charge, opp_dat node_potential,

@@ -24,7 +24,9 @@ DESIGN.md §11 fix them (normalised units):
   B3  Newton: J = K + diag(ne_coef * m_n / te * exp((phi_n - phi0) / te)),
       J_FF delta_F = -F_F, delta_D = 0, phi <- phi + delta
   B4  start: phi_F = phi0 (or the caller's warm start), phi_D = dval_D;
-      stop when ||F_F(phi_k)||_2 <= max(tol * ||F_F(phi_start)||_2, atol),
+      stop when ||F_F(phi_k)||_2 <= max(tol * ||F_F(phi_cold)||_2, atol), with
+      phi_cold the cold start (phi0 on free nodes, dval_D): a reference that
+      does not depend on the warm start (as the linear CG's ||b_eff||);
       or after max_newton steps.
 Here each Newton step is solved exactly (sparse direct solve); the product
 solves it by Jacobi-preconditioned CG to a tolerance the caller sets.
@@ -80,11 +82,13 @@ def newton(K: sp.csr_matrix, Q: np.ndarray, m: np.ndarray, dmask: np.ndarray, dv
     Returns (phi, newton_steps, [||F_F(phi_k)||_2 for k = 0..steps])."""
     D = np.asarray(dmask, bool)
     Fr = ~D
-    phi = np.full(K.shape[0], float(phi0)) if phi_start is None else np.array(phi_start, np.float64)
+    cold = np.full(K.shape[0], float(phi0))
+    cold[D] = np.asarray(dval, np.float64)[D]
+    f0 = float(np.linalg.norm(residual_vector(K, Q, m, cold, D, rhs_scale, ne_coef, phi0, te)))
+    phi = cold.copy() if phi_start is None else np.array(phi_start, np.float64)
     phi[D] = np.asarray(dval, np.float64)[D]
     F = residual_vector(K, Q, m, phi, D, rhs_scale, ne_coef, phi0, te)
     hist = [float(np.linalg.norm(F))]
-    f0 = hist[0]
     k = 0
     while k < max_newton and hist[-1] > max(tol * f0, atol):
         J = jacobian(K, m, phi, ne_coef, phi0, te)

@@ -2125,9 +2125,30 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
     {
         PhaseScope ph(c, OPP_PH_FIELD);
         if (nn > 0) {
+            NewtonCoef co{prm->rhs_scale, prm->ne_coef, prm->phi0, 1.0 / prm->te};
+            // reading B4: the stopping reference is ||F_F|| at the cold start
+            // (phi0 on free nodes), whatever the start; a warm start evaluates
+            // it once on a scratch vector (the Newton update buffer)
+            double ref = -1.0;
+            if (prm->warm_start == 2) {
+                if (!f.xprev) {
+                    f.xprev = (double *)c->dalloc(8 * nn);
+                    if (!f.xprev) return fail(OPP_ERR_NOMEM, "field extrapolation buffer");
+                }
+                if (f.xprev_dat != node_potential)
+                    CK(cudaMemcpyAsync(f.xprev, phi, 8 * nn, cudaMemcpyDeviceToDevice, c->s));
+                CK(launch_extrapolate(f.K, phi, f.xprev, c->s));
+                c->launches++;
+                f.xprev_dat = node_potential;
+            }
+            if (prm->warm_start != 0) {
+                CK(launch_newton_start(f.K, f.bz_delta, prm->phi0, 0, c->s));
+                CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, f.bz_delta, f.bz_m, co,
+                                      f.bz_rhs, f.bz_part, f.bz_nblk, f.bz_norm + 1, c->s));
+                c->launches += 3;
+            }
             CK(launch_newton_start(f.K, phi, prm->phi0, prm->warm_start != 0, c->s));
             c->launches++;
-            NewtonCoef co{prm->rhs_scale, prm->ne_coef, prm->phi0, 1.0 / prm->te};
             FieldMat J = f.K;
             J.val = f.bz_jval;
             J.dinv = f.bz_jdinv;
@@ -2161,24 +2182,31 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
                 CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, phi, f.bz_m, co, f.bz_rhs,
                                       f.bz_part, f.bz_nblk, f.bz_norm, c->s));
                 c->launches += 2;
-                CK(cudaMemcpyAsync(f.bz_host, f.bz_norm, 8, cudaMemcpyDeviceToHost, c->s));
-                if (k > 0) CK(cudaMemcpyAsync(f.bz_host + 1, f.st, sizeof(int), cudaMemcpyDeviceToHost, c->s));
+                CK(cudaMemcpyAsync(f.bz_host, f.bz_norm, 16, cudaMemcpyDeviceToHost, c->s));
+                if (k > 0) CK(cudaMemcpyAsync(f.bz_host + 2, f.st, sizeof(int), cudaMemcpyDeviceToHost, c->s));
                 CK(cudaStreamSynchronize(c->s));
                 const double fn = std::sqrt(f.bz_host[0]);
                 if (k > 0) {
                     int it;
-                    memcpy(&it, f.bz_host + 1, sizeof(int));
+                    memcpy(&it, f.bz_host + 2, sizeof(int));
                     bs.cg_iterations += it;
                 }
                 if (!std::isfinite(fn)) return fail(OPP_ERR_STATE, "Newton diverged (||F|| not finite)");
                 if (k == 0) {
+                    ref = prm->warm_start != 0 ? std::sqrt(f.bz_host[1]) : fn;
                     bs.res0_norm = fn;
-                    thr = std::max(prm->newton_tol * fn, prm->newton_atol);
+                    bs.ref_norm = ref;
+                    thr = std::max(prm->newton_tol * ref, prm->newton_atol);
                 }
                 bs.res_norm = fn;
                 bs.newton_steps = k;
                 if (fn <= thr) { bs.converged = 1; break; }
                 if (k >= prm->max_newton) break;
+                // inner tolerance: cg_tol; near the solution (||F|| <= 1e-3 of
+                // the reference: the linear regime) only as tight as this step
+                // needs to meet the stop, r <= thr / 2
+                a.tol = prm->cg_tol;
+                if (fn <= 1e-3 * ref) a.tol = std::min(a.tol, std::max(0.5 * thr / fn, 1e-15));
                 int grid = 0;
                 CK(launch_cg(a, c->nsm, bps, c->s, &grid));
                 CK(launch_newton_update(f.K, phi, f.bz_delta, c->s));

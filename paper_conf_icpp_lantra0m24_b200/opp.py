@@ -87,7 +87,7 @@ class opp_boltzmann_params(C.Structure):
 class opp_boltzmann_stats(C.Structure):
     _fields_ = [("newton_steps", C.c_int32), ("converged", C.c_int32),
                 ("cg_iterations", C.c_int64), ("res_norm", C.c_double),
-                ("res0_norm", C.c_double)]
+                ("res0_norm", C.c_double), ("ref_norm", C.c_double)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

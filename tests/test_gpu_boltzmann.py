@@ -62,6 +62,7 @@ def test_boltzmann_matches_newton_oracle(dims, jit, precond):
     assert st["converged"] == 1
     assert abs(st["newton_steps"] - r["k_o"]) <= 1
     assert st["res0_norm"] == pytest.approx(r["hist"][0], rel=1e-12)
+    assert st["ref_norm"] == pytest.approx(r["hist"][0], rel=1e-12)   # cold start: same
     assert np.linalg.norm(r["Fg"]) <= 10 * 1e-10 * r["hist"][0]
     free = mask == 0
     np.testing.assert_array_equal(phi[~free], val[~free])
@@ -154,3 +155,31 @@ def test_boltzmann_full_size_c2_residual():
     # ion density in [0.8, 1.2] n0 -> the free potential lies between the
     # quasi-neutral levels te ln 0.8 and the wall potential
     assert phi.min() >= np.log(0.8) - 1e-9 and phi.max() <= 4.0 + 1e-9
+
+
+@pytest.mark.parametrize("warm", [1, 2])
+def test_boltzmann_warm_start_matches_oracle(warm):
+    """Reading B4 through the GPU path: a perturbed warm start stops against the
+    cold-start reference and lands on the oracle's answer from that start
+    (warm 2: the first extrapolated solve starts like warm 1)."""
+    mesh = gen.kuhn_duct(5, 4, 9, jitter=0.2, seed=4)
+    xyz, c2n = mesh["node_xyz"], mesh["c2n"]
+    Q = np.random.default_rng(6).uniform(0, 2, mesh["n_nodes"])
+    mask, val = gen.duct_bc(mesh, wall=3.0, inlet=0.0)
+    K, M = F.stiffness(xyz, c2n), B.lumped_mass(xyz, c2n)
+    args = (K, Q, M, mask, val, 0.5, 0.8, 0.0, 1.5)
+    phi_c, _, hist_c = B.newton(*args, tol=1e-10)
+    pert = phi_c + 0.05 * np.random.default_rng(7).uniform(-1, 1, phi_c.size)
+    phi_o, k_o, hist = B.newton(*args, tol=1e-10, phi_start=pert)
+    sim = _sim(mesh)
+    sim.field_init(mask, val)
+    _set(sim, sim.node_charge, Q)
+    _set(sim, sim.node_potential, pert)
+    st = sim.field_solve_boltzmann(0.5, 0.8, 0.0, 1.5, newton_tol=1e-10, cg_tol=1e-13,
+                                   warm_start=warm)
+    phi = sim.potential_host()
+    sim.close()
+    assert st["converged"] == 1 and abs(st["newton_steps"] - k_o) <= 1
+    assert st["ref_norm"] == pytest.approx(hist_c[0], rel=1e-12)
+    assert st["res0_norm"] == pytest.approx(hist[0], rel=1e-9)
+    assert np.abs(phi - phi_o).max() <= 1e-8 * np.abs(phi_o).max()

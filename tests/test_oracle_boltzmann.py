@@ -111,3 +111,21 @@ def test_nonlinear_sheath_first_integral_and_quadratic_newton():
             if h[i] < 0.05 * h[0] and h[i + 1] > 1e-12 * h[0]]   # above the rounding floor
     assert tail and max(tail) <= 5.0
     assert h[-1] <= 1e-12 * h[0]
+
+
+def test_warm_start_reference_is_the_cold_start():
+    """Reading B4: the stopping reference is ||F(phi_cold)||, whatever the start:
+    a start at the answer takes no step, a perturbed start reaches the same
+    answer (to the tolerance)."""
+    m, K, M = _sys(4, 4, 8, jitter=0.2, seed=4)
+    Q = np.random.default_rng(6).uniform(0, 2, m["n_nodes"])
+    mask, val = gen.duct_bc(m, wall=3.0, inlet=0.0)
+    args = (K, Q, M, mask, val, 0.5, 0.8, 0.0, 1.5)
+    phi, k, hist = B.newton(*args, tol=1e-10)
+    assert k >= 3
+    _, k0, _ = B.newton(*args, tol=1e-10, phi_start=phi)
+    assert k0 == 0
+    pert = phi + 0.05 * np.random.default_rng(7).uniform(-1, 1, phi.size)
+    phi2, k2, hist2 = B.newton(*args, tol=1e-10, phi_start=pert)
+    assert 1 <= k2 <= k
+    assert np.abs(phi2 - phi).max() <= 1e-9 * np.abs(phi).max()
