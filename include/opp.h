@@ -361,10 +361,14 @@ int opp_get_field_stats(opp_ctx ctx, opp_field_stats *stats);
  *   stop when ||F_F||_2 <= max(newton_tol ||F_F(phi_cold)||_2, newton_atol)
  *   or after max_newton steps, phi_cold = the cold start (phi0 on free
  *   nodes): a reference independent of the warm start.
- * Needs opp_field_init (same matrix, Dirichlet data and n2c).  One rank only
- * (OPP_ERR_STATE when nranks > 1).  node_charge / node_potential / cell_ef
- * as in opp_field_solve.  The loop is host-driven: one ||F|| read-back per
- * Newton step (synchronises).  Errors: OPP_ERR_ARG (te <= 0, ne_coef < 0,
+ * Needs opp_field_init (same matrix, Dirichlet data and n2c).  node_charge /
+ * node_potential / cell_ef as in opp_field_solve.  The loop is host-driven:
+ * one ||F|| read-back per Newton step (synchronises).  nranks > 1 (slabs,
+ * collective): K phi of interface rows is completed by the node halo, the
+ * lumped mass likewise, the electron diagonal enters the Jacobian on the
+ * owning rank's copy only, norms count each node once and are reduced across
+ * ranks, and each Newton step runs the host-driven slab CG of
+ * opp_field_solve.  Errors: OPP_ERR_ARG (te <= 0, ne_coef < 0,
  * tolerances < 0, max_newton / cg_max_iter < 0, NULL params), OPP_ERR_STATE,
  * OPP_ERR_NOMEM, OPP_ERR_CUDA.
  * ------------------------------------------------------------------------- */

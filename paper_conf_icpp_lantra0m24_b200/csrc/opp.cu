@@ -1756,7 +1756,7 @@ static int allreduce_dots(opp_ctx c, const double *dev, int n, double *out) {
 // reduced across ranks in rank order; alpha, beta on the host.
 static int field_solve_hostloop(opp_ctx c, CgArgs &a) {
     FieldState &f = c->fs;
-    const FieldMat &K = f.K;
+    const FieldMat &K = a.K;       // f.K (linear solve) or the Newton Jacobian
     const long long nn = f.nn;
     const bool multi = c->p.nranks > 1 && c->comm->halo_n > 0;
     double *y = f.hvec, *yd = f.hvec + nn, *beff = f.hvec + 2 * nn;
@@ -2097,6 +2097,8 @@ static int boltz_alloc(opp_ctx c) {
     CK(launch_lumped_mass((const double *)c->cols[f.node_pos].d, (const int32_t *)cn.d, f.n2c_ptr,
                           f.n2c, f.nn, f.bz_m, c->s));
     c->launches++;
+    // slabs: interface nodes' masses summed over the ranks sharing them
+    if (c->p.nranks > 1 && c->comm->halo_n > 0) TRY(halo_sum(c, f.bz_m));
     return OPP_OK;
 }
 
@@ -2106,7 +2108,6 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
     TRY(ctx_check(c));
     FieldState &f = c->fs;
     if (!f.ready) return fail(OPP_ERR_STATE, "opp_field_init first");
-    if (c->p.nranks > 1) return fail(OPP_ERR_STATE, "the Boltzmann solve runs on one rank only");
     if (!prm) return fail(OPP_ERR_ARG, "null Boltzmann params");
     if (!(prm->te > 0.0) || !(prm->ne_coef >= 0.0) || !(prm->newton_tol >= 0.0) ||
         !(prm->newton_atol >= 0.0) || !(prm->cg_tol >= 0.0) || prm->max_newton < 0 ||
@@ -2119,18 +2120,45 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
     if (cell_ef >= 0) TRY(check_col(c, cell_ef, false, cells, 3, OPP_REAL, "cell_ef"));
     TRY(boltz_alloc(c));
     const long long nn = f.nn;
+    // slabs (nranks > 1): K phi through the partial SpMV + node halo, the
+    // electron diagonal on the owning rank's copy, own-weighted norms reduced
+    // across ranks, the host-driven CG of the linear solve on the Jacobian
+    const bool multi = c->p.nranks > 1;
+    const bool halo = multi && c->comm->halo_n > 0;
     double *phi = (double *)c->cols[node_potential].d;
     const double *Q = (const double *)c->cols[node_charge].d;
+    const NewtonCoef co{prm->rhs_scale, prm->ne_coef, prm->phi0, 1.0 / prm->te};
+    const int dblk = (int)std::min<long long>(f.part_cap, std::max<long long>(1, (nn + 255) / 256));
+    // F(v) -> f.bz_rhs (= -F), J(v) -> f.bz_jval / f.bz_jdinv; returns ||F_F||_2 (synchronises)
+    auto eval = [&](const double *v, double *norm) -> int {
+        double n2 = 0.0;
+        if (!multi) {
+            CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, v, f.bz_m, co, f.bz_rhs, f.bz_part,
+                                  f.bz_nblk, f.bz_norm, c->s));
+            c->launches += 2;
+            CK(cudaMemcpyAsync(f.bz_host, f.bz_norm, 8, cudaMemcpyDeviceToHost, c->s));
+            CK(cudaStreamSynchronize(c->s));
+            n2 = f.bz_host[0];
+        } else {
+            double *y = f.hvec;
+            CK(launch_spmv(f.K, v, y, nullptr, c->nsm, c->s));
+            c->launches++;
+            if (halo) TRY(halo_sum(c, y));
+            CK(launch_newton_eval_y(f.K, y, f.own, f.bz_jval, f.bz_jdinv, Q, v, f.bz_m, co, f.bz_rhs,
+                                    f.bz_nblk, c->s));
+            const double *va[1] = {f.bz_rhs}, *vb[1] = {f.bz_rhs};
+            CK(launch_dots(nn, f.own, 1, va, vb, f.part, dblk, f.dots, c->s));
+            c->launches += 3;
+            TRY(allreduce_dots(c, f.dots, 1, &n2));
+        }
+        *norm = std::sqrt(n2);
+        return OPP_OK;
+    };
     opp_boltzmann_stats bs{};
     {
         PhaseScope ph(c, OPP_PH_FIELD);
-        if (nn > 0) {
-            NewtonCoef co{prm->rhs_scale, prm->ne_coef, prm->phi0, 1.0 / prm->te};
-            // reading B4: the stopping reference is ||F_F|| at the cold start
-            // (phi0 on free nodes), whatever the start; a warm start evaluates
-            // it once on a scratch vector (the Newton update buffer)
-            double ref = -1.0;
-            if (prm->warm_start == 2) {
+        if (nn > 0 || multi) {
+            if (prm->warm_start == 2 && nn > 0) {
                 if (!f.xprev) {
                     f.xprev = (double *)c->dalloc(8 * nn);
                     if (!f.xprev) return fail(OPP_ERR_NOMEM, "field extrapolation buffer");
@@ -2141,11 +2169,14 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
                 c->launches++;
                 f.xprev_dat = node_potential;
             }
+            // reading B4: the stopping reference is ||F_F|| at the cold start
+            // (phi0 on free nodes), whatever the start; a warm start evaluates
+            // it once on a scratch vector (the Newton update buffer)
+            double ref = 0.0;
             if (prm->warm_start != 0) {
                 CK(launch_newton_start(f.K, f.bz_delta, prm->phi0, 0, c->s));
-                CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, f.bz_delta, f.bz_m, co,
-                                      f.bz_rhs, f.bz_part, f.bz_nblk, f.bz_norm + 1, c->s));
-                c->launches += 3;
+                c->launches++;
+                TRY(eval(f.bz_delta, &ref));
             }
             CK(launch_newton_start(f.K, phi, prm->phi0, prm->warm_start != 0, c->s));
             c->launches++;
@@ -2170,7 +2201,6 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
             a.part = f.part;
             a.st = f.st;
             a.rhs_scale = 1.0;
-            a.tol = prm->cg_tol;
             a.max_iter = prm->cg_max_iter;
             a.warm = 0;
             a.precond = prm->precond != 0;
@@ -2178,22 +2208,20 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
             if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
             bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
             double thr = 0.0;
+            bool pending_it = false;   // single rank: CG iterations still on the device
             for (int k = 0;; k++) {
-                CK(launch_newton_eval(f.K, f.bz_jval, f.bz_jdinv, Q, phi, f.bz_m, co, f.bz_rhs,
-                                      f.bz_part, f.bz_nblk, f.bz_norm, c->s));
-                c->launches += 2;
-                CK(cudaMemcpyAsync(f.bz_host, f.bz_norm, 16, cudaMemcpyDeviceToHost, c->s));
-                if (k > 0) CK(cudaMemcpyAsync(f.bz_host + 2, f.st, sizeof(int), cudaMemcpyDeviceToHost, c->s));
-                CK(cudaStreamSynchronize(c->s));
-                const double fn = std::sqrt(f.bz_host[0]);
-                if (k > 0) {
-                    int it;
-                    memcpy(&it, f.bz_host + 2, sizeof(int));
-                    bs.cg_iterations += it;
+                double fn = 0.0;
+                TRY(eval(phi, &fn));
+                if (pending_it) {
+                    CgState st;
+                    CK(cudaMemcpyAsync(&st, f.st, sizeof(CgState), cudaMemcpyDeviceToHost, c->s));
+                    CK(cudaStreamSynchronize(c->s));
+                    bs.cg_iterations += st.iterations;
+                    pending_it = false;
                 }
                 if (!std::isfinite(fn)) return fail(OPP_ERR_STATE, "Newton diverged (||F|| not finite)");
                 if (k == 0) {
-                    ref = prm->warm_start != 0 ? std::sqrt(f.bz_host[1]) : fn;
+                    if (prm->warm_start == 0) ref = fn;
                     bs.res0_norm = fn;
                     bs.ref_norm = ref;
                     thr = std::max(prm->newton_tol * ref, prm->newton_atol);
@@ -2207,10 +2235,17 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
                 // needs to meet the stop, r <= thr / 2
                 a.tol = prm->cg_tol;
                 if (fn <= 1e-3 * ref) a.tol = std::min(a.tol, std::max(0.5 * thr / fn, 1e-15));
-                int grid = 0;
-                CK(launch_cg(a, c->nsm, bps, c->s, &grid));
+                if (!multi) {
+                    int grid = 0;
+                    CK(launch_cg(a, c->nsm, bps, c->s, &grid));
+                    c->launches++;
+                    pending_it = true;
+                } else {
+                    TRY(field_solve_hostloop(c, a));
+                    bs.cg_iterations += f.hst.iterations;
+                }
                 CK(launch_newton_update(f.K, phi, f.bz_delta, c->s));
-                c->launches += 2;
+                c->launches++;
             }
         } else {
             bs.converged = 1;

@@ -111,6 +111,45 @@ __global__ void __launch_bounds__(kBzThreads)
     }
 }
 
+// Multi-rank form (slab partition): y = K phi with the interface rows already
+// summed over ranks (halo), K.dinv = 1 / the summed diagonal.  The electron
+// diagonal is added to the Jacobian values on the owning rank only (own[i] =
+// 1), so the halo-summed SpMV of the CG applies K + diag(d) exactly once.
+__global__ void __launch_bounds__(kBzThreads)
+    k_newton_eval_y(FieldMat K, const double *__restrict__ y, const double *__restrict__ own,
+                    double *__restrict__ jval, double *__restrict__ jdinv,
+                    const double *__restrict__ Q, const double *__restrict__ phi,
+                    const double *__restrict__ m, NewtonCoef co, double *__restrict__ rhsv) {
+    const int lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long TW = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long sl = gw; sl < K.nslices; sl += TW) {
+        const long long i = sl * kSell + lane;
+        const long long off = K.slice_off[sl];
+        const int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+        const bool row = i < K.nn;
+        int kd = -1;
+        for (int k = 0; k < W; k++) {
+            const long long q = off + (long long)kSell * k + lane;
+            const int c = K.col[q];
+            if (kd < 0 && c == (int)i) kd = k;
+            jval[q] = K.val[q];
+        }
+        if (!row) continue;
+        double F = 0.0;
+        if (!K.dmask[i]) {
+            const double e = exp((phi[i] - co.phi0) * co.inv_te);
+            const double d = co.ne * m[i] * e * co.inv_te;
+            F = y[i] - co.rhs_scale * Q[i] + co.ne * m[i] * e;
+            if (kd >= 0 && own[i] > 0.0) jval[off + (long long)kSell * kd + lane] += d;
+            jdinv[i] = 1.0 / (1.0 / K.dinv[i] + d);
+        } else {
+            jdinv[i] = 1.0;
+        }
+        rhsv[i] = -F;
+    }
+}
+
 __global__ void k_sum_final(const double *__restrict__ part, int nblk, double *out) {
     const int lane = threadIdx.x;
     double t = 0.0;
@@ -164,6 +203,14 @@ cudaError_t launch_newton_eval(const FieldMat &K, double *jval, double *jdinv, c
                                cudaStream_t s) {
     k_newton_eval<<<nblk, kBzThreads, 0, s>>>(K, jval, jdinv, Q, phi, m, co, rhsv, part);
     k_sum_final<<<1, 32, 0, s>>>(part, nblk, norm2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_newton_eval_y(const FieldMat &K, const double *y, const double *own,
+                                 double *jval, double *jdinv, const double *Q, const double *phi,
+                                 const double *m, const NewtonCoef &co, double *rhsv, int nblk,
+                                 cudaStream_t s) {
+    k_newton_eval_y<<<nblk, kBzThreads, 0, s>>>(K, y, own, jval, jdinv, Q, phi, m, co, rhsv);
     return cudaGetLastError();
 }
 

@@ -103,6 +103,12 @@ cudaError_t launch_newton_eval(const FieldMat &K, double *jval, double *jdinv, c
                                const double *phi, const double *m, const NewtonCoef &co,
                                double *rhsv, double *part, int nblk, double *norm2,
                                cudaStream_t s);
+// Multi-rank form: y = the halo-summed K phi; the electron diagonal goes into
+// the Jacobian values where own[i] > 0 only; no norm (own-weighted dots follow).
+cudaError_t launch_newton_eval_y(const FieldMat &K, const double *y, const double *own,
+                                 double *jval, double *jdinv, const double *Q, const double *phi,
+                                 const double *m, const NewtonCoef &co, double *rhsv, int nblk,
+                                 cudaStream_t s);
 cudaError_t launch_newton_start(const FieldMat &K, double *phi, double phi0, int warm,
                                 cudaStream_t s);
 // free rows: x <- 2 x - xprev, xprev <- old x (warm_start 2 of opp_field_solve)

@@ -137,3 +137,61 @@ def test_loopback_field_solve_equals_single_domain(R):
     b = F.load_vector(Qg, rhs_scale)
     rhs = b[free] - K[free][:, ~free] @ val[~free]
     assert np.linalg.norm(phi - phi_ref) <= 2 * tol * np.linalg.norm(rhs) / lam_min + 1e-14
+
+
+@pytest.mark.parametrize("R", [2, 3])
+def test_loopback_boltzmann_equals_single_domain(R):
+    """Boltzmann-electron Newton solve on R slabs (halo-completed K phi and
+    lumped mass, electron diagonal on the owning copy, cross-rank norms, the
+    slab CG per Newton step): the merged potential equals the single-domain
+    Newton oracle, interface copies agree, one global Newton iteration."""
+    import torch
+    from oracle import boltzmann as B
+    from oracle import field as F
+    from paper_conf_icpp_lantra0m24_b200 import dist
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh = gen.kuhn_duct(5, 4, 12, jitter=0.15, seed=8)
+    Qg = np.random.default_rng(3).uniform(0.0, 2.0, mesh["n_nodes"])
+    mask, val = gen.duct_bc(mesh, wall=3.0, inlet=0.0)
+    prm = (0.5, 0.8, 0.0, 1.5)                  # rhs_scale, ne_coef, phi0, te
+    K = F.stiffness(mesh["node_xyz"], mesh["c2n"])
+    M = B.lumped_mass(mesh["node_xyz"], mesh["c2n"])
+    phi_o, k_o, hist = B.newton(K, Qg, M, mask, val, *prm, tol=1e-10)
+    uid = os.urandom(128)
+    streams = [torch.cuda.Stream() for _ in range(R)]
+    out, errs = [None] * R, []
+
+    def worker(r):
+        try:
+            sl = dist.slab(mesh, R, r)
+            sim = MiniFemPic(sl, np.zeros((sl["n_cells"], 3)), nranks=R, rank=r, uid=uid,
+                             transport=1, torch_alloc=False, stream=streams[r].cuda_stream)
+            gid = sl["node_gid"]
+            sim.field_init(mask[gid], val[gid])
+            O.opp_set_dat(sim.ctx, sim.node_charge, np.ascontiguousarray(Qg[gid]), sim.nn)
+            st = sim.field_solve_boltzmann(*prm, newton_tol=1e-10, cg_tol=1e-13)
+            out[r] = (gid, sim.potential_host(), st)
+            sim.close()
+        except Exception as e:   # noqa: BLE001
+            errs.append((r, e))
+            raise
+
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(R)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not errs, errs
+    steps = {o[2]["newton_steps"] for o in out}
+    assert len(steps) == 1 and all(o[2]["converged"] == 1 for o in out)
+    assert abs(steps.pop() - k_o) <= 1
+    for o in out:
+        assert o[2]["ref_norm"] == pytest.approx(hist[0], rel=1e-12)
+    phi = np.full(mesh["n_nodes"], np.nan)
+    for gid, ph, st in out:
+        seen = ~np.isnan(phi[gid])
+        np.testing.assert_array_equal(phi[gid][seen], ph[seen])     # interface copies agree
+        phi[gid] = ph
+    assert not np.isnan(phi).any()
+    assert np.abs(phi - phi_o).max() <= 1e-8 * np.abs(phi_o).max()
