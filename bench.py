@@ -69,7 +69,7 @@ def parse():
                     help="linear field solve start: 1 = last solution, 2 = extrapolated from the last two")
     ap.add_argument("--field-model", choices=("linear", "boltzmann"), default="linear",
                     help="field solve: linear Poisson CG (north_star) or the Boltzmann-electron "
-                         "Newton solve (PAPER.md:1604-1612, DESIGN.md §11; one GPU)")
+                         "Newton solve (PAPER.md:1604-1612, DESIGN.md §11)")
     ap.add_argument("--newton-cg-tol", type=float, default=1e-6,
                     help="boltzmann: inner CG tolerance relative to ||F|| per Newton step")
     ap.add_argument("--te", type=float, default=0.01, help="boltzmann: electron temperature (potential units)")
@@ -482,8 +482,6 @@ def run_ours(args, rank, world):
     torch.cuda.synchronize()
 
     boltz = args.field and args.field_model == "boltzmann"
-    if boltz and world > 1:
-        raise SystemExit("--field-model boltzmann runs on one GPU (DESIGN.md §11)")
     if boltz and args.ne < 0:
         x0, x1, y0, y1, z0, z1 = mesh["box"]
         args.ne = args.rhs * w * n0 / ((x1 - x0) * (y1 - y0) * (z1 - z0))
@@ -591,7 +589,11 @@ def run_ours(args, rank, world):
                          "last_solve": bz_last, "newton_tol": args.cg_tol, "inner_cg_tol": args.newton_cg_tol,
                          "ne_coef": args.ne, "te": args.te, "rhs_scale": args.rhs,
                          "wall_potential": args.wall,
-                         "solver": "Newton: fused F/J pass + Jacobi-PCG persistent kernel, warm start, "
+                         "solver": ("Newton: fused F/J pass + Jacobi-PCG persistent kernel, "
+                                    if world == 1 else "Newton over slabs: halo-completed F, "
+                                    "host-driven slab Jacobi-PCG, ") +
+                                   ("warm start extrapolated from the last two solutions, "
+                                    if args.cg_warm == 2 else "warm start, ") +
                                    "host-driven (one ||F|| read-back per Newton step)",
                          "note": "value excludes the field solve (timed separately, SURVEY.md "
                                  "§8(d)); value_incl_field counts it"}
