@@ -448,6 +448,184 @@ __global__ void __launch_bounds__(kCgThreads) k_pcg(CgArgs a) {
     }
 }
 
+// k_pcg with the row-local vectors (x, r, u, w, p, s, q, z, M^-1 w and the
+// Jacobi diagonal) of a thread's R rows held in shared memory for the whole
+// solve (10 R doubles per thread, [vector][slot][thread]: conflict-free):
+// an iteration reads the matrix and gathers the SpMV input from L2 and writes
+// only the next SpMV input (8 B per row) instead of 15 vector elements.
+// Needs ceil(nslices / warps) <= R (launch_cg picks R; else k_pcg).
+template <int R>
+__global__ void __launch_bounds__(kCgThreads) k_pcg_reg(CgArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ double sm[4 * kCgWarps];
+    const FieldMat &K = a.K;
+    const long long nn = K.nn;
+    const int lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long TW = ((long long)gridDim.x * blockDim.x) >> 5;
+    const int G = (int)gridDim.x;
+    double *part0 = a.part;                 // ||b_eff||^2 partials
+    double *partR[2] = {a.part + G, a.part + 4 * G};   // (r,u), (w,u), (r,r) by parity
+
+    for (long long sl = gw; sl < K.nslices; sl += TW) {
+        long long i = sl * kSell + lane;
+        if (i >= nn) continue;
+        a.x[i] = K.dmask[i] ? K.dval[i] : (a.warm ? a.x[i] : 0.0);
+    }
+    grid.sync();
+    {   // r0 = b - K x0, lifted rhs, u0 = M^-1 r0
+        double v[1] = {0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double ri = 0.0, bi = 0.0;
+            if (!K.dmask[i]) {
+                long long off = K.slice_off[sl];
+                int W = (int)((K.slice_off[sl + 1] - off) / kSell);
+                double ax = 0.0, ad = 0.0;
+                for (int k = 0; k < W; k++) {
+                    long long q = off + (long long)kSell * k + lane;
+                    int c = K.col[q];
+                    double t = K.val[q] * __ldcg(a.x + c);
+                    ax += t;
+                    if (K.dmask[c]) ad += t;
+                }
+                double b = a.rhs_scale * a.Q[i];
+                ri = b - ax;
+                bi = b - ad;
+            }
+            a.r[i] = ri;
+            a.u[i] = a.precond ? ri * K.dinv[i] : ri;
+            a.p[i] = 0.0;
+            a.s[i] = 0.0;
+            a.q[i] = 0.0;
+            a.z[i] = 0.0;
+            v[0] += bi * bi;
+        }
+        block_publish<1>(v, part0, sm);
+    }
+    grid.sync();
+    {   // w0 = K u0, m0 = M^-1 w0, first dots
+        double v[3] = {0.0, 0.0, 0.0};
+        for (long long sl = gw; sl < K.nslices; sl += TW) {
+            long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            double wi = sell_row(K, sl, lane, a.u);
+            double ri = a.r[i], ui = a.u[i];
+            a.w[i] = wi;
+            a.m0[i] = a.precond ? wi * K.dinv[i] : wi;
+            v[0] += ri * ui;
+            v[1] += wi * ui;
+            v[2] += ri * ri;
+        }
+        block_publish<3>(v, partR[0], sm);
+    }
+    grid.sync();
+    double rr0;
+    {
+        double t[1];
+        block_total<1>(part0, sm, t);
+        rr0 = t[0];
+    }
+    const double stop = a.tol * a.tol * rr0;
+    // the row-local vectors live in dynamic shared memory, [vector][row slot][thread]
+    extern __shared__ double vsm[];
+#define VS(k, j) vsm[((k) * R + (j)) * kCgThreads + threadIdx.x]
+#define xr(j) VS(0, j)
+#define rr_(j) VS(1, j)
+#define ur(j) VS(2, j)
+#define wr(j) VS(3, j)
+#define pr(j) VS(4, j)
+#define sr(j) VS(5, j)
+#define qr(j) VS(6, j)
+#define zr(j) VS(7, j)
+#define mr(j) VS(8, j)
+#define dr(j) VS(9, j)
+#pragma unroll
+    for (int j = 0; j < R; j++) {
+        const long long sl = gw + (long long)j * TW;
+        const long long i = sl * kSell + lane;
+        const bool ok = sl < K.nslices && i < nn;
+        xr(j) = ok ? a.x[i] : 0.0;
+        rr_(j) = ok ? a.r[i] : 0.0;
+        ur(j) = ok ? a.u[i] : 0.0;
+        wr(j) = ok ? a.w[i] : 0.0;
+        mr(j) = ok ? a.m0[i] : 0.0;
+        dr(j) = ok ? (a.precond ? K.dinv[i] : 1.0) : 0.0;
+        pr(j) = 0.0;
+        sr(j) = 0.0;
+        qr(j) = 0.0;
+        zr(j) = 0.0;
+    }
+    double gamma_old = 0.0, alpha = 0.0, beta = 0.0, rho = 0.0;
+    int it = 0;
+    for (;;) {
+        double t[3];
+        block_total<3>(partR[it & 1], sm, t);
+        const double gamma = t[0], delta = t[1];
+        rho = t[2];
+        if (rho <= stop || it >= a.max_iter) break;
+        if (it == 0) {
+            beta = 0.0;
+            alpha = gamma / delta;
+        } else {
+            beta = gamma / gamma_old;
+            alpha = gamma / (delta - beta * gamma / alpha);
+        }
+        gamma_old = gamma;
+        const double *mc = (it & 1) ? a.m1 : a.m0;
+        double *mn = (it & 1) ? a.m0 : a.m1;
+        double v[3] = {0.0, 0.0, 0.0};
+#pragma unroll
+        for (int j = 0; j < R; j++) {
+            const long long sl = gw + (long long)j * TW;
+            if (sl >= K.nslices) continue;
+            const long long i = sl * kSell + lane;
+            if (i >= nn) continue;
+            const double ni = sell_row(K, sl, lane, mc);
+            zr(j) = ni + beta * zr(j);
+            qr(j) = mr(j) + beta * qr(j);
+            sr(j) = wr(j) + beta * sr(j);
+            pr(j) = ur(j) + beta * pr(j);
+            xr(j) += alpha * pr(j);
+            rr_(j) -= alpha * sr(j);
+            ur(j) -= alpha * qr(j);
+            wr(j) -= alpha * zr(j);
+            mr(j) = wr(j) * dr(j);
+            mn[i] = mr(j);
+            v[0] += rr_(j) * ur(j);
+            v[1] += wr(j) * ur(j);
+            v[2] += rr_(j) * rr_(j);
+        }
+        block_publish<3>(v, partR[(it + 1) & 1], sm);
+        grid.sync();
+        it++;
+    }
+#pragma unroll
+    for (int j = 0; j < R; j++) {
+        const long long sl = gw + (long long)j * TW;
+        const long long i = sl * kSell + lane;
+        if (sl < K.nslices && i < nn) a.x[i] = xr(j);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.st->iterations = it;
+        a.st->converged = rho <= stop;
+        a.st->rr0 = rr0;
+        a.st->rr = rho;
+    }
+#undef xr
+#undef rr_
+#undef ur
+#undef wr
+#undef pr
+#undef sr
+#undef qr
+#undef zr
+#undef mr
+#undef dr
+#undef VS
+}
+
 __global__ void k_efield(const double *__restrict__ xyz, const int32_t *__restrict__ c2n,
                          const double *__restrict__ phi, long long nc, double *__restrict__ ef,
                          double4 *__restrict__ efp) {
@@ -478,7 +656,38 @@ cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const i
 cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out) {
     int occ = 0;
     const void *fn = a.pipelined ? (const void *)k_pcg : (const void *)k_cg;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kCgThreads, 0);
+    // OPP_CG_REG (default 1): k_pcg_reg<R>, the smallest R (<= 4) for which
+    // every thread's rows fit its R shared-memory slots at the grid it gets
+    static const int use_reg = [] {
+        const char *e = getenv("OPP_CG_REG");
+        return e ? atoi(e) : 1;
+    }();
+    size_t dsm = 0;
+    if (a.pipelined && use_reg) {
+        const void *regk[4] = {(const void *)k_pcg_reg<1>, (const void *)k_pcg_reg<2>,
+                               (const void *)k_pcg_reg<3>, (const void *)k_pcg_reg<4>};
+        for (int R = 1; R <= 4; R++) {
+            const size_t smem = (size_t)10 * R * kCgThreads * sizeof(double);
+            if (cudaFuncSetAttribute(regk[R - 1], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)smem) != cudaSuccess)
+                break;
+            int occ0 = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ0, regk[R - 1], kCgThreads, smem) !=
+                    cudaSuccess || occ0 < 1)
+                break;
+            int g = nsm * (occ0 < max_bps ? occ0 : max_bps);
+            if (g > 2 * kCgThreads) g = 2 * kCgThreads;
+            long long want0 = (a.K.nslices + kCgWarps - 1) / kCgWarps;
+            if (want0 < g) g = (int)(want0 > 0 ? want0 : 1);
+            const long long tw = (long long)g * kCgWarps;
+            if ((a.K.nslices + tw - 1) / tw <= R) {
+                fn = regk[R - 1];
+                dsm = smem;
+                break;
+            }
+        }
+    }
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kCgThreads, dsm);
     if (e != cudaSuccess) return e;
     int bps = occ < max_bps ? occ : max_bps;
     if (bps < 1) return cudaErrorCooperativeLaunchTooLarge;
@@ -488,7 +697,7 @@ cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int
     if (want < grid) grid = (int)(want > 0 ? want : 1);
     CgArgs args = a;
     void *params[] = {&args};
-    e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kCgThreads), params, 0, s);
+    e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kCgThreads), params, dsm, s);
     if (grid_out) *grid_out = grid;
     return e;
 }
