@@ -656,7 +656,7 @@ cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const i
 cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out) {
     int occ = 0;
     const void *fn = a.pipelined ? (const void *)k_pcg : (const void *)k_cg;
-    // OPP_CG_REG (default 1): k_pcg_reg<R>, the smallest R (<= 4) for which
+    // OPP_CG_REG (default 1): k_pcg_reg<R>, the smallest R (<= 6) for which
     // every thread's rows fit its R shared-memory slots at the grid it gets
     static const int use_reg = [] {
         const char *e = getenv("OPP_CG_REG");
@@ -664,9 +664,10 @@ cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int
     }();
     size_t dsm = 0;
     if (a.pipelined && use_reg) {
-        const void *regk[4] = {(const void *)k_pcg_reg<1>, (const void *)k_pcg_reg<2>,
-                               (const void *)k_pcg_reg<3>, (const void *)k_pcg_reg<4>};
-        for (int R = 1; R <= 4; R++) {
+        const void *regk[6] = {(const void *)k_pcg_reg<1>, (const void *)k_pcg_reg<2>,
+                               (const void *)k_pcg_reg<3>, (const void *)k_pcg_reg<4>,
+                               (const void *)k_pcg_reg<5>, (const void *)k_pcg_reg<6>};
+        for (int R = 1; R <= 6; R++) {
             const size_t smem = (size_t)10 * R * kCgThreads * sizeof(double);
             if (cudaFuncSetAttribute(regk[R - 1], cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)smem) != cudaSuccess)
