@@ -290,7 +290,8 @@ int64_t opp_kernel_launch_count(opp_ctx ctx);
  * Mini-FEM-PIC's ComputeJMatrix / ComputeF1Vector / linear solve /
  * ComputeElectricField (Fig. 6) in the
  * linear form north_star names ("a plain GPU conjugate-gradient on the FEM
- * Poisson system"; the Boltzmann-electron Newton solve is out of scope):
+ * Poisson system"; the Boltzmann-electron Newton solve is
+ * opp_field_solve_boltzmann below):
  *   K phi = b,  K_ij = sum_e V_e grad(lambda_i) . grad(lambda_j)   (P1 Laplacian)
  *   b = rhs_scale * node_charge    (the consistent P1 load of the deposited
  *                                   point charges, Eq. 10; F2)

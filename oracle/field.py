@@ -19,7 +19,8 @@ Passages followed (PAPER.md line ranges; section / figure / equation):
                                              at a higher potential")
 Readings (F1-F5): linear Poisson  -div(grad phi) = rho/eps
 (north_star: "a plain GPU conjugate-gradient on the FEM Poisson system", in
-place of the paper's Boltzmann-electron Newton solve, NEXT-4); the load
+place of the paper's Boltzmann-electron Newton solve, NEXT-4, whose oracle is
+oracle/boltzmann.py); the load
 vector is the consistent P1 load of the deposited point charges,
 b_n = rhs_scale * Q_n with Q_n = w * sum_p lambda_n(x_p) (S7); Dirichlet
 nodes take given values, every other boundary is homogeneous Neumann;
