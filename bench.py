@@ -3,24 +3,38 @@
 
 One step = one pass of the whole hot path over the resident
 particle population: inject (a1) -> zero node charge (a2) -> gather E + push
-(a3, a4) -> multi-hop walk (a6, optionally DH-seeded a5) -> deposit (a7) ->
-write-back / holes (a8) -> hole fill (a9).  Default workload = config C2
-(BASELINE.json configs[1]): 48x48x72 Kuhn duct (995,328 tets), a pre-seeded
-50M-particle steady state plus 250k injected per step; every step first solves
-the field (P1 FEM Poisson by the persistent CG kernel, Fig. 1 step 1) from the
-previous step's charge.  The field solve is timed separately (SURVEY.md §8(d):
-"value" counts the particle loop; "field" and "value_incl_field" report it).
+(a3, a4) -> multi-hop walk (a6, DH-seeded a5) -> deposit (a7) -> write-back /
+holes (a8) -> hole fill (a9) -> (N > 1) migration rounds (a10) and the
+node-charge halo (a11).
 
-Contract: W untimed warm-up steps, then exactly K timed steps bracketed by a
-barrier + cuda synchronize; CUDA events on the library's stream; max over
-ranks; rank 0 prints ONE JSON line.  --impl reference times the CPU oracle
-(oracle/, single thread) on a bounded sample of the same workload.
+Default workload = config C4 (BASELINE.json configs[3], the metric's
+"at 1/2/4/8 B200" configuration): per GPU a 40x40x72-hex Kuhn slab (691,200
+tets) holding 1e9 particles, global duct 40x40x(72 N), contiguous z-slabs,
+3.5M particles injected per step on rank 0, fixed uniform E (weak scaling:
+per-GPU work fixed).  --config c2 is BASELINE.json's "1xB200" config (the
+48x48x72 duct, 50M particles + 250k/step, CG Poisson solve every step timed
+apart), c5 the clustered deposit stress, c3 the CabanaPIC-style EM loop.
+
+Launch: `python bench.py --gpus N` starts N ranks itself (torch.distributed.run,
+one process per GPU, NCCL) when run outside torchrun; under torchrun
+WORLD_SIZE must equal --gpus.  `--gpus N --loopback` runs N slabs as N
+contexts on ONE GPU (the in-process transport: a protocol check, not a
+scaling number; reports n_gpus 1 and ranks N).
+
+Contract: W untimed warm-up steps, then K timed steps bracketed by a barrier +
+cuda synchronize, repeated --reps times (median reported, min shown; each
+repetition times exactly K steps); CUDA events on the library's stream; max
+over ranks; rank 0 prints ONE JSON line.  --impl reference times the CPU
+oracle (oracle/, single thread, pinned core) on a bounded sample of the same
+workload.
 """
 from __future__ import annotations
 
 import argparse
+import hashlib
 import json
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -36,14 +50,18 @@ UNIT = "particle-steps/s"
 DEP_NAMES = {0: "atomic", 1: "atomic_warpagg", 2: "sort_segred"}
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--reps", type=int, default=3,
+                    help="timed repetitions of the K steps (median reported, min shown)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c2", "c5", "c1", "c3"])
-    ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count")
+    ap.add_argument("--config", default="c4", choices=["c4", "c2", "c5", "c1", "c3"])
+    ap.add_argument("--loopback", action="store_true",
+                    help="with --gpus N: N slabs as N contexts on one GPU (in-process transport)")
+    ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count (per rank)")
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
     ap.add_argument("--mh", action="store_true", help="multi-hop only (no direct-hop seeding)")
@@ -61,7 +79,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=0)
     ap.add_argument("--field", type=int, default=-1,
                     help="solve the field (CG) every step: 1 on, 0 off (fixed uniform E); "
-                         "default: on for c2, off otherwise")
+                         "default: on for c2 and c3, off otherwise")
     ap.add_argument("--rhs", type=float, default=2e-7, help="field solve: b = rhs * node charge")
     ap.add_argument("--wall", type=float, default=0.02, help="field solve: side-wall potential")
     ap.add_argument("--cg-tol", type=float, default=1e-10)
@@ -74,41 +92,19 @@ def parse():
                     help="boltzmann: inner CG tolerance relative to ||F|| per Newton step")
     ap.add_argument("--te", type=float, default=0.01, help="boltzmann: electron temperature (potential units)")
     ap.add_argument("--ne", type=float, default=-1.0,
-                    help="boltzmann: electron coefficient (default: the mean ion load per volume, "
-                         "rhs * w * n0 / duct volume, so electrons balance ions at phi0 = 0)")
+                    help="boltzmann: electron coefficient (default: the mean ion load per volume)")
     ap.add_argument("--ppc", type=int, default=750, help="c3: particles per cell (750 = 72M, 1500 = 144M)")
     ap.add_argument("--em-sort", type=int, default=0, help="c3: sort particles by cell every K steps (0 = never)")
-    args = ap.parse_args()
+    args = ap.parse_args(argv)
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
     if args.field < 0:
         args.field = 1 if args.config in ("c2", "c3") else 0
+    if args.config in ("c4", "c5") and args.field:
+        raise SystemExit("c4 / c5 run with a fixed uniform field (SURVEY.md §8(d))")
     return args
 
 
-# ---------------------------------------------------------------- workload
-def workload(args, world=1):
-    import gen
-    cfg = dict(gen.CONFIGS[args.config])
-    if args.n0:
-        cfg["n0"] = args.n0
-    nx, ny, nz = cfg["dims"]
-    mesh = gen.kuhn_duct(nx, ny, nz * world)
-    c1E = np.array(cfg["c1E"])
-    qm, dt = 1.0, cfg["dt"]
-    ef = np.tile(c1E / (qm * dt), (mesh["n_cells"], 1))
-    cluster = None
-    if cfg.get("cluster"):
-        cluster = (cfg["cluster"], gen.hot_block_cells(mesh))
-    name = {"c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
-                  "+ 250k injected/step, " + (("Boltzmann-electron Newton field solve every step"
-                                               if args.field_model == "boltzmann" else
-                                               "CG Poisson field solve every step") if args.field
-                                              else "fixed uniform E"),
-            "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
-            "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
-    return cfg, mesh, ef, qm, dt, cluster, name
-
-
+# ---------------------------------------------------------------- helpers
 def load_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -116,6 +112,70 @@ def load_peaks():
         return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:   # noqa: BLE001
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def src_hash() -> str:
+    """Hash of the library sources: a stored ncu traffic figure is only
+    reported for the kernels it was captured from."""
+    h = hashlib.sha256()
+    d = os.path.join(ROOT, "paper_conf_icpp_lantra0m24_b200", "csrc")
+    for f in sorted(os.listdir(d)):
+        if f.endswith((".cu", ".h")):
+            with open(os.path.join(d, f), "rb") as fh:
+                h.update(f.encode() + fh.read())
+    return h.hexdigest()[:16]
+
+
+def traffic_for(key: str):
+    """dram bytes per launch of the dominant kernel from this source tree's
+    ncu --set full capture (profiles/ncu_traffic.json, written by
+    scripts/ncu_summary.py traffic); null when the capture is of other code."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            e = json.load(f).get(key)
+    except Exception:   # noqa: BLE001
+        return None, "no capture"
+    if not isinstance(e, dict):
+        return None, "no capture"
+    if e.get("src_hash") != src_hash():
+        return None, f"capture {e.get('capture')} is of other kernel sources (stale)"
+    return e.get("bytes"), e.get("capture")
+
+
+def opp_env():
+    return {k: v for k, v in os.environ.items() if k.startswith("OPP_")}
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:   # noqa: BLE001
+        pass
+    return "unknown"
+
+
+class pinned_core:
+    """Pin the calling thread to one host core while the oracle runs."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = sorted(self.prev)[0]
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.prev)
+
+
+def cpu_meta(core=None) -> dict:
+    import oracle
+    d = {"cpu": cpu_model(), "threads": 1, **oracle.build_info()}
+    if core is not None:
+        d["pinned_core"] = core
+    return d
 
 
 class ClockSampler:
@@ -170,11 +230,79 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(self.rows)}
 
 
+# ---------------------------------------------------------------- rank groups
+class Group:
+    """The ranks this process drives: one (torchrun / N = 1) or all N
+    (loopback threads).  Barrier + max / sum reductions over every rank."""
+
+    def __init__(self, world: int, mode: str):
+        self.world, self.mode = world, mode      # mode: "single", "dist" (process group), "loopback"
+        self._bar = threading.Barrier(world) if mode == "loopback" else None
+        self._vals = {}
+        self._lock = threading.Lock()
+
+    def barrier(self):
+        if self.mode == "dist":
+            import torch.distributed as dist
+            dist.barrier()
+        elif self.mode == "loopback":
+            self._bar.wait()
+
+    def _reduce(self, tag, v, op):
+        if self.mode == "single":
+            return v
+        if self.mode == "dist":
+            from paper_conf_icpp_lantra0m24_b200 import dist as D
+            return D.max_over_ranks(v) if op == "max" else D.sum_over_ranks(v)
+        with self._lock:
+            self._vals.setdefault(tag, []).append(v)
+        self._bar.wait()
+        vals = self._vals[tag]
+        r = max(vals) if op == "max" else sum(vals)
+        self._bar.wait()
+        with self._lock:
+            self._vals.pop(tag, None)
+        return r
+
+    def max(self, tag, v):
+        return self._reduce(tag, v, "max")
+
+    def sum(self, tag, v):
+        return self._reduce(tag, v, "sum")
+
+
+# ---------------------------------------------------------------- workload
+def workload(args, world=1):
+    import gen
+    cfg = dict(gen.CONFIGS[args.config])
+    if args.n0:
+        cfg["n0"] = args.n0
+    nx, ny, nz = cfg["dims"]
+    mesh = gen.kuhn_duct(nx, ny, nz * world)
+    c1E = np.array(cfg["c1E"])
+    qm, dt = 1.0, cfg["dt"]
+    ef = np.tile(c1E / (qm * dt), (mesh["n_cells"], 1))
+    cluster = None
+    if cfg.get("cluster"):
+        cluster = (cfg["cluster"], gen.hot_block_cells(mesh))
+    field = ("Boltzmann-electron Newton field solve every step" if args.field_model == "boltzmann"
+             else "CG Poisson field solve every step") if args.field else "fixed uniform E"
+    name = {"c4": f"C4 Mini-FEM-PIC weak scaling: per GPU a 40x40x72-hex Kuhn slab (691,200 tets) "
+                  f"with {cfg['n0']:,} particles, global duct 40x40x{72 * world}, "
+                  f"{cfg['n_inj']:,} injected/step on rank 0, {field}",
+            "c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
+                  "+ 250k injected/step, " + field,
+            "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
+            "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
+    return cfg, mesh, ef, qm, dt, cluster, name
+
+
 # ---------------------------------------------------------------- oracle legs
 def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster, dm=None):
-    """Time the CPU oracle (as it stands) on a bounded sample of the workload.
-    The sample's inputs come from the seeded generator (its device twin when a
-    GPU is present: bit-identical, and fast for millions of particles)."""
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload,
+    pinned to one host core.  The sample's inputs come from the seeded
+    generator (its device twin when a GPU is present: bit-identical, and fast
+    for millions of particles)."""
     import gen
     import oracle
     om = oracle.Mesh.from_gen(mesh)
@@ -191,17 +319,18 @@ def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster, dm=None):
     scale = n_sample / max(cfg["n0"], 1)
     n_inj = int(round(cfg["n_inj"] * scale))
     pushed, secs = 0, 0.0
-    for s in range(steps):
-        if n_inj:
-            b = gen.inject_batch(mesh, s, n_inj, cfg["seed"], id_base=cfg["n0"])
-            t0 = time.perf_counter()
-            P.append(b["pos"], b["vel"], b["cell"], b["id"])
-        else:
-            t0 = time.perf_counter()
-        st = oracle.step(om, P, qm * dt, dt, w, Q)
-        secs += time.perf_counter() - t0
-        pushed += st["n_before"]
-    return pushed, secs, n_inj
+    with pinned_core() as pc:
+        for s in range(steps):
+            if n_inj:
+                b = gen.inject_batch(mesh, s, n_inj, cfg["seed"], id_base=cfg["n0"])
+                t0 = time.perf_counter()
+                P.append(b["pos"], b["vel"], b["cell"], b["id"])
+            else:
+                t0 = time.perf_counter()
+            st = oracle.step(om, P, qm * dt, dt, w, Q)
+            secs += time.perf_counter() - t0
+            pushed += st["n_before"]
+    return pushed, secs, n_inj, pc.core
 
 
 def run_reference(args, rank, world):
@@ -211,18 +340,20 @@ def run_reference(args, rank, world):
     w = cfg["w"]
     n_sample = 400_000 if args.config != "c1" else cfg["n0"]
     # warm-up steps are run and discarded, then K timed sample-steps
-    oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, max(args.warmup, 0) and 1, cluster)
-    pushed, secs, n_inj = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, args.steps, cluster)
+    if args.warmup > 0:
+        oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, args.warmup, cluster)
+    pushed, secs, n_inj, core = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, args.steps, cluster)
     v = pushed / secs
     sample = (f"{n_sample:,} particles of the {args.config.upper()} workload "
-              f"(+{n_inj:,} injected/step), {args.steps} steps, 1 thread")
+              f"(+{n_inj:,} injected/step), {args.steps} steps, 1 thread; the GPU arm runs "
+              f"{cfg['n0']:,} per rank (different cache behaviour)")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * secs / max(args.steps, 1), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": name, "sample": sample},
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, **cpu_meta(core)},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -252,17 +383,19 @@ def run_reference_c3(args, rank, world):
     import oracle.em as OE
     nx, ny, nz, c2c, e, b = c3_inputs(args)
     interp = OE.interpolate(nx, ny, nz, e, b)
-    # bounded sample: the first `ppc_s` particles of every cell of a z-range
+    # bounded sample: the first `ppc_s` particles of every cell
     ppc_s = 16
     p = ge.two_stream(nx, ny, nz, ppc_s, C3["seed"], v0=C3["v0"], pert=C3["pert"], vth=C3["vth"])
     prm = OE.params(C3["qdt_2mc"], C3["cdt_2h"], C3["qsp"], C3["kcap"])
     acc = np.zeros((nx * ny * nz, 12))
     off, u, w, cell = p["off"], p["u"], p["w"], p["cell"]
-    OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)   # warm-up step
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)
-    secs = time.perf_counter() - t0
+    with pinned_core() as pc:
+        for _ in range(max(args.warmup, 0)):
+            OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            OE.move_deposit(prm, off, u, w, cell, interp, c2c, acc)
+        secs = time.perf_counter() - t0
     v = p["n"] * args.steps / secs
     sample = f"{p['n']:,} particles ({ppc_s}/cell) of the C3 workload, {args.steps} steps, 1 thread"
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
@@ -270,28 +403,22 @@ def run_reference_c3(args, rank, world):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": {"workload": C3_NAME.format(ppc=args.ppc, fields=", fixed fields"),
                                             "sample": sample},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             **cpu_meta(pc.core)},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
-
-
-def c3_traffic(args):
-    try:
-        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-            return json.load(f).get(f"c3_dep{1 if args.deposit != 0 else 0}")
-    except Exception:   # noqa: BLE001
-        return None
 
 
 def run_ours_c3(args, rank, world):
     """C3: one step = Move_Deposit over the whole resident population (the
     accumulator is zeroed between steps outside the timed kernel's model).
     N > 1: independent replicas (the periodic two-stream box is not
-    partitioned in this round: DESIGN.md §10)."""
+    partitioned: DESIGN.md §10)."""
     import torch
     import gen.cuda as gc
     from paper_conf_icpp_lantra0m24_b200.em_app import CabanaPicEM
     from paper_conf_icpp_lantra0m24_b200 import dist as D
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
     dev = int(os.environ.get("LOCAL_RANK", 0))
     torch.cuda.set_device(dev)
     nx, ny, nz, c2c, e, b = c3_inputs(args)
@@ -305,7 +432,6 @@ def run_ours_c3(args, rank, world):
     n = sim.n
     stream = torch.cuda.current_stream()
     nstep = [0]
-
     em_field = args.field != 0      # c3 default: the field side runs every step
 
     def em_step(stats=False):
@@ -321,33 +447,40 @@ def run_ours_c3(args, rank, world):
 
     for _ in range(args.warmup):
         em_step()
-    torch.cuda.synchronize()
-    if world > 1:
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
-    l0 = sim.launches()
-    from paper_conf_icpp_lantra0m24_b200 import opp as O
-    O.opp_phase_timing(sim.ctx, True)
-    O.opp_get_phase_times(sim.ctx)
+    reps = []
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(dev) as clk:
-        e0.record(stream)
-        for _ in range(args.steps):
-            em_step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1)
-    launches = sim.launches() - l0
-    ph = O.opp_get_phase_times(sim.ctx)
-    O.opp_phase_timing(sim.ctx, False)
+        for _ in range(max(args.reps, 1)):
+            torch.cuda.synchronize()
+            if world > 1:
+                torch.distributed.barrier()
+            torch.cuda.synchronize()
+            l0 = sim.launches()
+            O.opp_phase_timing(sim.ctx, True)
+            O.opp_get_phase_times(sim.ctx)
+            e0.record(stream)
+            for _ in range(args.steps):
+                em_step()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1)
+            launches = sim.launches() - l0
+            ph = O.opp_get_phase_times(sim.ctx)
+            O.opp_phase_timing(sim.ctx, False)
+            pushed = n * args.steps
+            field_ms = ph["field"][0] if em_field else 0.0
+            if world > 1:
+                ms = D.max_over_ranks(ms)
+                field_ms = D.max_over_ranks(field_ms)
+                pushed = D.sum_over_ranks(pushed)
+                launches = D.sum_over_ranks(launches)
+            reps.append(dict(ms=ms, field_ms=field_ms, pushed=pushed, launches=launches, ph=ph,
+                             value=pushed / ((ms - field_ms) / 1e3)))
     st = em_step(stats=True)
-    pushed = n * args.steps
-    field_ms = ph["field"][0] if em_field else 0.0
-    if world > 1:
-        ms = D.max_over_ranks(ms)
-        pushed = D.sum_over_ranks(pushed)
-        launches = D.sum_over_ranks(launches)
-    value = pushed / ((ms - field_ms) / 1e3)   # the particle loop; the field side apart (as C2)
+    order = sorted(range(len(reps)), key=lambda k: reps[k]["value"])
+    med = reps[order[len(order) // 2]]
+    ms, field_ms, pushed, launches, ph = med["ms"], med["field_ms"], med["pushed"], med["launches"], med["ph"]
+    value = med["value"]          # the particle loop; the field side apart (as C2)
     peak, peak_src = load_peaks()
     k_ms, k_cnt = ph["em_move_deposit"]
     # algorithmic bytes per launch: particle state in (off, u, w, cell = 60 B) and
@@ -355,6 +488,7 @@ def run_ours_c3(args, rank, world):
     # and the accumulator read-modify-write (2 x 96 B)
     bpl = 112.0 * n + (144.0 + 24.0 + 192.0) * nc
     achieved = bpl / (k_ms / max(k_cnt, 1) / 1e3) / 1e9
+    tb, tsrc = traffic_for(f"c3_dep{1 if args.deposit != 0 else 0}")
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
@@ -366,8 +500,11 @@ def run_ours_c3(args, rank, world):
                    "sort_every": args.em_sort,
                    "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n * 60 / 1e9),
                    "parallelism": f"replicas{world}" if world > 1 else "single"},
+        "reps": {"values": [r["value"] for r in reps], "median": value,
+                 "min": min(r["value"] for r in reps)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": c3_traffic(args), "kernel": "k_em_move_deposit",
+                     "frac": achieved / peak, "traffic": tb, "traffic_source": tsrc,
+                     "kernel": "k_em_move_deposit",
                      "bytes_model": "112 B/particle + 360 B/cell per launch", "peak_source": peak_src},
         "gpu_launches": launches,
         "phases_ms_per_step": {k: v[0] / args.steps for k, v in ph.items() if v[1]},
@@ -378,6 +515,7 @@ def run_ours_c3(args, rank, world):
         "move": {"crossings_per_particle": st["n_crossings"] / max(n, 1),
                  "max_crossings": st["max_crossings"], "capped": st["n_capped"]},
         "clocks": clk.summary(),
+        "env": opp_env(),
     }
     if not args.no_e2e:
         # e2e through the public API: the step's fields arrive from pinned host
@@ -442,268 +580,401 @@ def run_ours_c3(args, rank, world):
         p = ge.two_stream(nx, ny, nz, 16, C3["seed"], v0=C3["v0"], pert=C3["pert"], vth=C3["vth"])
         acc = np.zeros((nc, 12))
         prm = OE.params(C3["qdt_2mc"], C3["cdt_2h"], C3["qsp"], C3["kcap"])
-        t0 = time.perf_counter()
-        for _ in range(2):
-            OE.move_deposit(prm, p["off"], p["u"], p["w"], p["cell"], interp, c2c, acc)
-        secs = time.perf_counter() - t0
+        with pinned_core() as pc:
+            t0 = time.perf_counter()
+            for _ in range(2):
+                OE.move_deposit(prm, p["off"], p["u"], p["w"], p["cell"], interp, c2c, acc)
+            secs = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": 2 * p["n"] / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"{p['n']:,} particles (16/cell) of the C3 workload, 2 steps, "
-                                          f"1 thread, {secs:.1f} s"}
+                                          f"1 thread, {secs:.1f} s", **cpu_meta(pc.core)}
     sim.close()
     if rank == 0:
         print(json.dumps(line), flush=True)
 
 
-# ---------------------------------------------------------------- our arm
-def run_ours(args, rank, world):
+# ---------------------------------------------------------------- our arm (electrostatic)
+class EsRank:
+    """One rank of the electrostatic particle loop: its slab (or the whole
+    duct), its libopp context, its seeded population and its injection
+    batches, all resident on the device before any timed step."""
+
+    def __init__(self, args, cfg, gmesh, gef, world, rank, stream, transport=0, uid=None,
+                 cluster=None):
+        import torch
+        import gen
+        import gen.cuda as gc
+        from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+        from paper_conf_icpp_lantra0m24_b200 import dist as D
+        self.args, self.cfg, self.rank, self.world = args, cfg, rank, world
+        self.stream = stream
+        w, n0, n_inj, seed = cfg["w"], cfg["n0"], cfg["n_inj"], cfg["seed"]
+        base, kw = 0, {}
+        mesh, ef = gmesh, gef
+        if world > 1:
+            mesh = D.slab(gmesh, world, rank)
+            ef = D.local_field(gef, mesh)
+            base = mesh["cell_base"]
+            kw = dict(nranks=world, rank=rank, uid=uid, transport=transport)
+            gen_mesh = dict(mesh, inlet=mesh["inlet_local"])
+            if cluster is not None:
+                cluster = (cluster[0], cluster[1][(cluster[1] >= base) & (cluster[1] < base + mesh["n_cells"])] - base)
+        else:
+            gen_mesh = mesh
+        if args.field:
+            ef = np.zeros_like(ef)
+        self.mesh, self.base = mesh, base
+        dm = gc.DeviceMesh(gen_mesh)
+        self.dm = dm
+        self.n_inj = n_inj if (world == 1 or mesh["inlet"].shape[0] > 0) else 0
+        total = args.warmup + max(args.reps, 1) * args.steps
+        self.total = total
+        # capacity: the seeded population + a 4% margin for the flow imbalance
+        # between ranks + two steps of injection (injection precedes the push)
+        cap = int(n0 * 1.04) + 2 * self.n_inj + 4096
+        self.sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
+                              direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
+                              sort_every=args.sort, tma_pipeline=not args.direct,
+                              sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0),
+                              torch_alloc=transport == 0, device=stream.device.index, **kw)
+        sim = self.sim
+        if args.field:
+            fmask, fval = gen.duct_bc(mesh, wall=args.wall, inlet=0.0)
+            sim.field_init(fmask, fval)
+        # seed in chunks (C4: 1e9 particles; a chunk is 60 B per particle of
+        # temporary device memory), generated on the device, bit-identical to
+        # generating the population at once
+        chunk = 50_000_000
+        with torch.cuda.stream(stream):
+            for first in range(0, n0, chunk):
+                m = min(chunk, n0 - first)
+                init = gc.seed_particles(dm, m, seed + rank, cluster=cluster, id_base=rank * n0, first=first,
+                                         stream=stream.cuda_stream)
+                if base:
+                    init["cell"] += base
+                sim.inject(init, on_device=True)
+                stream.synchronize()
+                del init
+            if args.sort:
+                # the population is born in random cell order; a sorted steady
+                # state is what periodic sorting maintains (setup, untimed)
+                sim.step(0.0, 1.0, w, stats=False, fill=True)   # builds mesh data; dt = 0: no motion
+                sim.sort_by_cell()
+            self.batches = [gc.inject_batch(dm, s, self.n_inj, seed, id_base=world * n0,
+                                            stream=stream.cuda_stream) if self.n_inj else None
+                            for s in range(total)]
+        stream.synchronize()
+        self.host_batches = None
+        self.bz_last = {}
+
+    def field(self):
+        a = self.args
+        if a.field and a.field_model == "boltzmann":
+            self.bz_last.update(self.sim.field_solve_boltzmann(a.rhs, a.ne, 0.0, a.te, newton_tol=a.cg_tol,
+                                                               cg_tol=a.newton_cg_tol, warm_start=a.cg_warm))
+        elif a.field:
+            self.sim.field_solve(a.rhs, tol=a.cg_tol, warm_start=a.cg_warm, stats=False)
+
+    def one_step(self, s, on_device=True):
+        sim, a = self.sim, self.args
+        self.field()
+        b = self.batches[s] if on_device else self.host_batches[s]
+        if b is not None:
+            sim.inject(b, on_device=on_device)
+        sim.step(self.cfg["dt"], 1.0, self.cfg["w"], stats=False, fill=True)
+        if a.shuffle and s % a.shuffle == 0:
+            sim.shuffle(self.cfg["seed"] + 7919 * s)
+
+
+def es_rank_main(args, rank, world, group, cfg, gmesh, gef, cluster, uid, transport, res):
+    """Everything one rank does: setup, warm-up, the timed repetitions, the
+    e2e leg.  Per-rank results go to res[rank] (rank 0's dict carries the
+    reduced values)."""
     import torch
-    import gen
-    import gen.cuda as gc
-    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
-
-    from paper_conf_icpp_lantra0m24_b200 import dist as D
     from paper_conf_icpp_lantra0m24_b200 import opp as O
-    dev = int(os.environ.get("LOCAL_RANK", 0))
+    dev = int(os.environ.get("LOCAL_RANK", 0)) if transport == 0 else 0
     torch.cuda.set_device(dev)
-    cfg, mesh, ef, qm, dt, cluster, name = workload(args, world)
-    w, n0, n_inj, seed = cfg["w"], cfg["n0"], cfg["n_inj"], cfg["seed"]
-    stream = torch.cuda.current_stream()
-    total = args.warmup + args.steps
-    base, kw = 0, {}
-    if world > 1:
-        # weak scaling: the C2 duct stacked `world` times along z, one slab
-        # (48x48x72 hex, 50M particles) per GPU; injection on rank 0's inlet
-        uid = D.broadcast_bytes(O.opp_get_nccl_unique_id() if rank == 0 else None)
-        gm = mesh
-        mesh = D.slab(gm, world, rank)
-        ef = D.local_field(ef, mesh)
-        base = mesh["cell_base"]
-        kw = dict(nranks=world, rank=rank, uid=uid, transport=0)
-        gen_mesh = dict(mesh, inlet=mesh["inlet_local"])
-        if cluster is not None:
-            cluster = (cluster[0], cluster[1][(cluster[1] >= base) & (cluster[1] < base + mesh["n_cells"])] - base)
-    else:
-        gen_mesh = mesh
-    if args.field:
-        ef = np.zeros_like(ef)
-    dm = gc.DeviceMesh(gen_mesh)
-    n_inj_local = n_inj if (world == 1 or mesh["inlet"].shape[0] > 0) else 0
-    cap = int(n0 * 1.1) + n_inj_local * (total + 4) + 1024
-    sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
-                     direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
-                     sort_every=args.sort, tma_pipeline=not args.direct,
-                     sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0), **kw)
-    if args.field:
-        fmask, fval = gen.duct_bc(mesh, wall=args.wall, inlet=0.0)
-        sim.field_init(fmask, fval)
-    init = gc.seed_particles(dm, n0, seed + rank, cluster=cluster, id_base=rank * n0)
-    if base:
-        init["cell"] += base
-    sim.inject(init, on_device=True)
-    torch.cuda.synchronize()
-    del init
-    if args.sort:
-        # the population is born in random cell order; a sorted steady state
-        # is what periodic sorting maintains (setup, untimed)
-        sim.step(0.0, qm, w, stats=False, fill=True)      # builds mesh data, dt = 0: no motion
-        sim.sort_by_cell()
-    batches = [gc.inject_batch(dm, s, n_inj_local, seed, id_base=world * n0) if n_inj_local else None
-               for s in range(total)]
-    torch.cuda.synchronize()
-
-    boltz = args.field and args.field_model == "boltzmann"
-    if boltz and args.ne < 0:
-        x0, x1, y0, y1, z0, z1 = mesh["box"]
-        args.ne = args.rhs * w * n0 / ((x1 - x0) * (y1 - y0) * (z1 - z0))
-    bz_last = {}
-
-    def field():
-        if boltz:
-            bz_last.update(sim.field_solve_boltzmann(args.rhs, args.ne, 0.0, args.te,
-                                                     newton_tol=args.cg_tol, cg_tol=args.newton_cg_tol,
-                                                     warm_start=args.cg_warm))
-        elif args.field:
-            sim.field_solve(args.rhs, tol=args.cg_tol, warm_start=args.cg_warm, stats=False)
-
-    def one_step(s, on_device=True, readback=None):
-        field()
-        if batches[s] is not None:
-            sim.inject(batches[s] if on_device else host_batches[s], on_device=on_device)
-        sim.step(dt, qm, w, stats=False, fill=True)
-        if args.shuffle and s % args.shuffle == 0:
-            sim.shuffle(seed + 7919 * s)
-        if readback is not None:
-            readback()
-
-    for s in range(args.warmup):
-        one_step(s)
-    torch.cuda.synchronize()
-    st0 = sim.last_stats()
-    if world > 1:
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
-    l0 = sim.launches()
-    sim.phase_timing(True)
-    sim.phase_times()  # reset
+    stream = torch.cuda.Stream(device=dev)
+    R = EsRank(args, cfg, gmesh, gef, world, rank, stream, transport=transport, uid=uid, cluster=cluster)
+    sim = R.sim
+    if args.field and args.field_model == "boltzmann" and args.ne < 0:
+        x0, x1, y0, y1, z0, z1 = gmesh["box"]
+        args.ne = args.rhs * cfg["w"] * cfg["n0"] * world / ((x1 - x0) * (y1 - y0) * (z1 - z0))
+    with torch.cuda.stream(stream):
+        for s in range(args.warmup):
+            R.one_step(s)
+    stream.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    reps = []
+    s_next = args.warmup
     with ClockSampler(dev) as clk:
-        e0.record(stream)
-        for s in range(args.warmup, total):
-            one_step(s)
-        e1.record(stream)
-        torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1)
-    launches = sim.launches() - l0
-    phases = sim.phase_times()
-    sim.phase_timing(False)
-    st1 = sim.last_stats()
-    pushed = st1["cum_pushed"] - st0["cum_pushed"]
-    if world > 1:
-        ms = D.max_over_ranks(ms)
-        pushed = D.sum_over_ranks(pushed)
-        launches = D.sum_over_ranks(launches)
-    field_ms = phases["field"][0] if args.field else 0.0
-    value = pushed / ((ms - field_ms) / 1e3)  # the particle loop; field apart
-    n_avg = pushed / args.steps / world       # per GPU
-
-    # ---- roofline of the dominant kernel (k_push_move_deposit, pass 1)
-    peak, peak_src = load_peaks()
-    pmd_ms, pmd_cnt = phases["push_move_deposit"]
-    nc, nn = mesh["n_cells"], mesh["n_nodes"]
-    bytes_per_launch = 104.0 * n_avg + 160.0 * nc + 16.0 * nn
-    achieved = bytes_per_launch / (pmd_ms / max(pmd_cnt, 1) / 1e3) / 1e9
-    traffic = None
-    tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tf):
-        try:
-            with open(tf) as f:
-                tj = json.load(f)
-            key = f"{args.config}_dep{args.deposit}_dh{int(args.dh)}"
-            traffic = tj.get(key)
-        except Exception:   # noqa: BLE001
-            traffic = None
-    # whole-step model bytes (SURVEY.md §8(d) B_ps)
-    f_inj = n_inj / max(n_avg, 1)
-    b_ps = 104.0 + (160.0 * nc + 16.0 * nn) / max(n_avg, 1) + 60.0 * f_inj
-    line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic",
-        "config": {"workload": name, "mesh_cells": nc, "mesh_nodes": nn,
-                   "particles_seeded": n0, "inject_per_step": n_inj,
-                   "avg_particles_per_step": n_avg, "deposit": DEP_NAMES[args.deposit],
-                   "walk": (f"DH{args.dh}(overlay {args.ov} h)+MH" if args.dh else "MH"),
-                   "hop_budget_per_pass": args.hpass,
-                   "sort_every": args.sort, "shuffle_every": args.shuffle,
-                   "pipeline": "direct" if args.direct else "tma",
-                   "sort_key": "axis z" if args.axis else "cell id",
-                   "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n_avg * 60 / 1e9),
-                   "parallelism": f"slab{world}",
-                   "mesh_global": f"{cfg['dims'][0]}x{cfg['dims'][1]}x{cfg['dims'][2] * world} hex"},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic,
-                     "kernel": "k_push_move_deposit (pass 1)",
-                     "bytes_model": "104 B/particle + 160 B/cell + 16 B/node per launch",
-                     "peak_source": peak_src,
-                     "step_frac": b_ps * value / (peak * 1e9), "step_bytes_per_particle": b_ps},
-        "gpu_launches": launches,
-        "phases_ms_per_step": {k: v[0] / args.steps for k, v in phases.items() if v[1]},
-        "walk": {"hops_per_particle_last_step": st1["total_hops"] / max(st1["n_before"], 1),
-                 "max_hops_last_step": st1["max_hops"], "hop_capped": st1["n_hop_capped"],
-                 "deferred_last_step": st1["n_deferred"]},
-        "clocks": clk.summary(),
-    }
-    if boltz:
-        line["field"] = {"ms_per_step": field_ms / args.steps, "model": "boltzmann",
-                         "last_solve": bz_last, "newton_tol": args.cg_tol, "inner_cg_tol": args.newton_cg_tol,
-                         "ne_coef": args.ne, "te": args.te, "rhs_scale": args.rhs,
-                         "wall_potential": args.wall,
-                         "solver": ("Newton: fused F/J pass + Jacobi-PCG persistent kernel, "
-                                    if world == 1 else "Newton over slabs: halo-completed F, "
-                                    "host-driven slab Jacobi-PCG, ") +
-                                   ("warm start extrapolated from the last two solutions, "
-                                    if args.cg_warm == 2 else "warm start, ") +
-                                   "host-driven (one ||F|| read-back per Newton step)",
-                         "note": "value excludes the field solve (timed separately, SURVEY.md "
-                                 "§8(d)); value_incl_field counts it"}
-        line["value_incl_field"] = pushed / (ms / 1e3)
-    elif args.field:
-        fst = sim.field_stats()
-        line["field"] = {"ms_per_step": field_ms / args.steps, "cg_iterations_last": fst["iterations"],
-                         "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
-                         "rhs_scale": args.rhs, "wall_potential": args.wall,
-                         "solver": ("Jacobi-PCG, one persistent cooperative kernel, warm start " + ("extrapolated from the last two solutions" if args.cg_warm == 2 else "from the last solution")
-                                    if world == 1 else "Jacobi-PCG over slabs (node halo + "
-                                    "cross-rank dots, host-driven), warm start"),
-                         "note": "value excludes the field solve (timed separately, SURVEY.md "
-                                 "§8(d)); value_incl_field counts it"}
-        line["value_incl_field"] = pushed / (ms / 1e3)
-
+        for rep in range(max(args.reps, 1)):
+            st0 = sim.last_stats()
+            group.barrier()
+            torch.cuda.synchronize()
+            l0 = sim.launches()
+            sim.phase_timing(True)
+            sim.phase_times()  # reset
+            with torch.cuda.stream(stream):
+                e0.record(stream)
+                for s in range(s_next, s_next + args.steps):
+                    R.one_step(s)
+                e1.record(stream)
+            torch.cuda.synchronize()
+            group.barrier()
+            s_next += args.steps
+            ms = e0.elapsed_time(e1)
+            launches = sim.launches() - l0
+            phases = sim.phase_times()
+            sim.phase_timing(False)
+            st1 = sim.last_stats()
+            pushed = st1["cum_pushed"] - st0["cum_pushed"]
+            field_ms = phases["field"][0] if args.field else 0.0
+            ms_max = group.max(f"ms{rep}", ms)
+            loop_ms_max = group.max(f"lms{rep}", ms - field_ms)
+            pushed_sum = group.sum(f"p{rep}", pushed)
+            launches_sum = group.sum(f"l{rep}", launches)
+            pmd_ms_max = group.max(f"pmd{rep}", phases["push_move_deposit"][0])
+            reps.append(dict(ms=ms_max, loop_ms=loop_ms_max, field_ms=field_ms, pushed=pushed_sum,
+                             launches=launches_sum, phases=phases, pmd_ms=pmd_ms_max,
+                             pushed_local=pushed, value=pushed_sum / (loop_ms_max / 1e3), st=st1))
+    out = dict(reps=reps, clocks=clk.summary(), mesh=R.mesh, n_inj=R.n_inj, bz=R.bz_last)
+    if args.field == 1 and args.field_model == "linear":
+        out["fst"] = sim.field_stats()
     # ---- e2e: same metric through the C ABI with HOST buffers
     if not args.no_e2e:
         ke = args.e2e_steps or min(args.steps, 10)
-        global host_batches
-        host_batches = [None] * total
-        for s in range(args.warmup, args.warmup + ke):
-            b = batches[s]
+        lo = args.warmup   # the device batches of these steps were consumed; host copies of them
+        R.host_batches = [None] * R.total
+        for s in range(lo, lo + ke):
+            b = R.batches[s]
             if b is not None:
-                host_batches[s] = {k: b[k].cpu().pin_memory().numpy() for k in ("pos", "vel", "cell", "id")}
-        q_host = torch.empty(nn, dtype=torch.float64).pin_memory().numpy()
-        from paper_conf_icpp_lantra0m24_b200 import opp as O
+                R.host_batches[s] = {k: b[k].cpu().pin_memory().numpy() for k in ("pos", "vel", "cell", "id")}
+        q_host = torch.empty(R.mesh["n_nodes"], dtype=torch.float64).pin_memory().numpy()
         # rewind is impossible (state advanced); e2e continues the same run
         torch.cuda.synchronize()
         s0 = sim.last_stats()
-        e0.record(stream)
-        # a user's pipelined loop through the public API: inject the next
-        # step's batch (H2D on the library's copy stream) while this step
-        # computes, then read this step's node charge back
-        s_lo, s_hi = args.warmup, args.warmup + ke
-        if host_batches[s_lo] is not None:
-            sim.inject(host_batches[s_lo], on_device=False)
-        sim.phase_timing(args.field)
-        sim.phase_times()
-        for s in range(s_lo, s_hi):
-            field()
-            sim.step(dt, qm, w, stats=False, fill=True)
-            if s + 1 < s_hi and host_batches[s + 1] is not None:
-                sim.inject(host_batches[s + 1], on_device=False)
-            O.opp_get_node_charge(sim.ctx, sim.node_charge, q_host)
-        e1.record(stream)
+        group.barrier()
+        with torch.cuda.stream(stream):
+            e0.record(stream)
+            # a user's pipelined loop through the public API: inject the next
+            # step's batch (H2D on the library's copy stream) while this step
+            # computes, then read this step's node charge back
+            if R.host_batches[lo] is not None:
+                sim.inject(R.host_batches[lo], on_device=False)
+            sim.phase_timing(bool(args.field))
+            sim.phase_times()
+            for s in range(lo, lo + ke):
+                R.field()
+                sim.step(cfg["dt"], 1.0, cfg["w"], stats=False, fill=True)
+                if s + 1 < lo + ke and R.host_batches[s + 1] is not None:
+                    sim.inject(R.host_batches[s + 1], on_device=False)
+                O.opp_get_node_charge(sim.ctx, sim.node_charge, q_host)
+            e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
         if args.field:
             ems -= sim.phase_times()["field"][0]
         sim.phase_timing(False)
         s1 = sim.last_stats()
-        epushed = s1["cum_pushed"] - s0["cum_pushed"]
-        if world > 1:
-            ems = D.max_over_ranks(ems)
-            epushed = D.sum_over_ranks(epushed)
-        line["e2e"] = {"value": epushed / (ems / 1e3), "unit": UNIT,
-                       "h2d_bytes_per_step": n_inj * 60, "d2h_bytes_per_step": nn * 8 * world,
-                       "steps": ke, "note": "injection arrays from pinned host memory (opp_inject "
+        out["e2e"] = dict(ms=group.max("e2e_ms", ems), pushed=group.sum("e2e_p", s1["cum_pushed"] - s0["cum_pushed"]),
+                          steps=ke, h2d=group.sum("e2e_h2d", R.n_inj * 60),
+                          d2h=group.sum("e2e_d2h", R.mesh["n_nodes"] * 8))
+    out["dm"] = R.dm
+    sim.close()
+    res[rank] = out
+
+
+def nccl_info(group, world):
+    """NCCL version, ranks and devices of the job (printed to stderr and
+    recorded in the JSON line so a run's rank count can be checked)."""
+    import torch
+    dev = torch.cuda.current_device()
+    p = torch.cuda.get_device_properties(dev)
+    me = {"rank": int(os.environ.get("RANK", 0)), "device": dev, "name": p.name,
+          "pci_bus_id": f"{p.pci_bus_id:02x}" if hasattr(p, "pci_bus_id") else None,
+          "uuid": str(getattr(p, "uuid", ""))}
+    if group.mode == "dist":
+        import torch.distributed as dist
+        allv = [None] * world
+        dist.all_gather_object(allv, me)
+    else:
+        allv = [me]
+    info = {"nccl_version": ".".join(map(str, torch.cuda.nccl.version())), "ranks": world,
+            "backend": group.mode, "devices": allv}
+    return info
+
+
+def run_ours(args, rank, world, mode):
+    """mode: "single" (N = 1), "dist" (this process is one of N torchrun
+    ranks, NCCL) or "loopback" (N ranks as threads of this process on one GPU)."""
+    import torch
+    from paper_conf_icpp_lantra0m24_b200 import dist as D
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    cfg, gmesh, gef, qm, dt, cluster, name = workload(args, world)
+    group = Group(world, mode)
+    uid = None
+    if mode == "dist":
+        uid = D.broadcast_bytes(O.opp_get_nccl_unique_id() if rank == 0 else None)
+        info = nccl_info(group, world)
+        if rank == 0:
+            print("[bench] NCCL", json.dumps(info), file=sys.stderr, flush=True)
+    elif mode == "loopback":
+        uid = os.urandom(128)
+        info = {"backend": "loopback", "ranks": world, "devices": [0]}
+    else:
+        info = None
+    res = [None] * world
+    if mode == "loopback":
+        errs = []
+
+        def worker(r):
+            try:
+                es_rank_main(args, r, world, group, cfg, gmesh, gef, cluster, uid, 1, res)
+            except BaseException as e:   # noqa: BLE001
+                errs.append((r, repr(e)))
+                group._bar.abort()
+                raise
+
+        th = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        if errs:
+            raise SystemExit(f"loopback ranks failed: {errs}")
+    else:
+        es_rank_main(args, rank, world, group, cfg, gmesh, gef, cluster, uid, 0, res)
+    if rank != 0:
+        return
+    out = res[0]
+    reps = out["reps"]
+    order = sorted(range(len(reps)), key=lambda k: reps[k]["value"])
+    med = reps[order[len(order) // 2]]
+    value = med["value"]
+    mesh = out["mesh"]
+    nc, nn = mesh["n_cells"], mesh["n_nodes"]
+    n_avg = med["pushed"] / args.steps / world       # per rank
+    n_inj = cfg["n_inj"]
+    # ---- roofline of the dominant kernel (k_push_move_deposit, pass 1):
+    # algorithmic bytes per launch (DESIGN.md §6) / the pass-1 kernel's mean
+    # CUDA-event duration (events recorded by the library on its stream)
+    peak, peak_src = load_peaks()
+    pmd_ms, pmd_cnt = med["phases"]["push_move_deposit"]
+    n_local = med["pushed_local"] / args.steps
+    bytes_per_launch = 104.0 * n_local + 160.0 * nc + 16.0 * nn
+    achieved = bytes_per_launch / (pmd_ms / max(pmd_cnt, 1) / 1e3) / 1e9
+    tb, tsrc = traffic_for(f"{args.config}_dep{args.deposit}_dh{int(args.dh)}")
+    # whole-step model bytes (SURVEY.md §8(d) B_ps)
+    f_inj = n_inj / max(n_avg * world, 1)
+    b_ps = 104.0 + (160.0 * nc + 16.0 * nn) / max(n_avg, 1) + 60.0 * f_inj
+    nranks_txt = f"{world} GPU" + ("s" if world > 1 else "")
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT,
+        "n_gpus": 1 if mode == "loopback" else world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": med["ms"] / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": name, "mesh_cells_per_rank": nc, "mesh_nodes_per_rank": nn,
+                   "particles_seeded_per_rank": cfg["n0"], "inject_per_step": n_inj,
+                   "avg_particles_per_step_per_rank": n_avg, "deposit": DEP_NAMES[args.deposit],
+                   "walk": (f"DH{args.dh}(overlay {args.ov} h)+MH" if args.dh else "MH"),
+                   "hop_budget_per_pass": args.hpass,
+                   "sort_every": args.sort, "shuffle_every": args.shuffle,
+                   "pipeline": "direct" if args.direct else "tma",
+                   "sort_key": "axis z" if args.axis else "cell id",
+                   "l2": "inputs larger than L2 (particle state %.1f GB per rank > 126 MB L2)" % (n_avg * 60 / 1e9),
+                   "parallelism": f"slab{world}" + (" (loopback: all ranks on one GPU)" if mode == "loopback" else ""),
+                   "mesh_global": f"{cfg['dims'][0]}x{cfg['dims'][1]}x{cfg['dims'][2] * world} hex",
+                   "ranks": world},
+        "reps": {"values": [r["value"] for r in reps], "median": value,
+                 "min": min(r["value"] for r in reps), "ms_per_step": [r["ms"] / args.steps for r in reps]},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": tb, "traffic_source": tsrc,
+                     "kernel": "k_push_move_deposit_tiled (pass 1)",
+                     "bytes_model": "104 B/particle + 160 B/cell + 16 B/node per launch",
+                     "peak_source": peak_src,
+                     "step_frac": b_ps * (value / world) / (peak * 1e9), "step_bytes_per_particle": b_ps},
+        "gpu_launches": med["launches"],
+        "phases_ms_per_step": {k: v[0] / args.steps for k, v in med["phases"].items() if v[1]},
+        "walk": {"hops_per_particle_last_step": med["st"]["total_hops"] / max(med["st"]["n_before"], 1),
+                 "max_hops_last_step": med["st"]["max_hops"], "hop_capped": med["st"]["n_hop_capped"],
+                 "deferred_last_step": med["st"]["n_deferred"],
+                 "migrated_out_last_step_rank0": med["st"]["n_migrated_out"]},
+        "clocks": out["clocks"],
+        "env": opp_env(),
+    }
+    if info is not None:
+        line["config"]["comm"] = info
+    if args.field and args.field_model == "boltzmann":
+        line["field"] = {"ms_per_step": med["field_ms"] / args.steps, "model": "boltzmann",
+                         "last_solve": out["bz"], "newton_tol": args.cg_tol, "inner_cg_tol": args.newton_cg_tol,
+                         "ne_coef": args.ne, "te": args.te, "rhs_scale": args.rhs,
+                         "wall_potential": args.wall,
+                         "note": "value excludes the field solve (timed separately, SURVEY.md "
+                                 "§8(d)); value_incl_field counts it"}
+        line["value_incl_field"] = med["pushed"] / (med["ms"] / 1e3)
+    elif args.field:
+        fst = out["fst"]
+        line["field"] = {"ms_per_step": med["field_ms"] / args.steps, "cg_iterations_last": fst["iterations"],
+                         "rel_residual_last": fst["rel_residual"], "tol": args.cg_tol,
+                         "rhs_scale": args.rhs, "wall_potential": args.wall,
+                         "solver": "Jacobi-PCG, one persistent cooperative kernel, warm start " +
+                                   ("extrapolated from the last two solutions" if args.cg_warm == 2
+                                    else "from the last solution"),
+                         "note": "value excludes the field solve (timed separately, SURVEY.md "
+                                 "§8(d)); value_incl_field counts it"}
+        line["value_incl_field"] = med["pushed"] / (med["ms"] / 1e3)
+    if "e2e" in out:
+        e = out["e2e"]
+        line["e2e"] = {"value": e["pushed"] / (e["ms"] / 1e3), "unit": UNIT,
+                       "h2d_bytes_per_step": e["h2d"], "d2h_bytes_per_step": e["d2h"],
+                       "steps": e["steps"], "note": "injection arrays from pinned host memory (opp_inject "
                        "on_device=0, H2D overlapped with the previous step on the library's copy "
                        "stream) + node charge read back every step (opp_get_node_charge)"}
-
-    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1)
-    if not args.no_cpu and world == 1 and rank == 0:
+    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1), one pinned core
+    if not args.no_cpu and world == 1:
         n_sample = 4_000_000 if args.config != "c1" else cfg["n0"]
-        pushed_c, secs, ninj_c = oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, 3, cluster, dm=dm)
+        pushed_c, secs, ninj_c, core = oracle_sample(gmesh, gef, qm, dt, cfg["w"], cfg, n_sample, 3, cluster,
+                                                     dm=out["dm"])
         line["cpu_baseline"] = {"value": pushed_c / secs, "unit": UNIT, "cores": 1,
                                 "kind": "oracle",
                                 "sample": f"{n_sample:,} particles of the same workload "
                                           f"(+{ninj_c:,} injected/step), 3 steps, 1 thread, "
-                                          f"{secs:.1f} s"}
-    sim.close()
-    if rank == 0:
-        print(json.dumps(line), flush=True)
+                                          f"{secs:.1f} s", **cpu_meta(core)}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- launch
+def free_port() -> int:
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
 
 
 def main():
     args = parse()
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is None and args.gpus > 1 and not args.loopback and args.impl == "ours":
+        # outside torchrun: start the N ranks (one process per GPU) ourselves
+        import torch
+        ndev = torch.cuda.device_count()
+        if ndev < args.gpus:
+            print(json.dumps({"error": f"--gpus {args.gpus} needs {args.gpus} GPUs, found {ndev} "
+                                       "(--loopback runs the N slabs on one GPU as a protocol check)"}),
+                  flush=True)
+            sys.exit(2)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+               f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+               "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+        sys.exit(subprocess.call(cmd))
+    world = int(world_env or 1)
     rank = int(os.environ.get("RANK", "0"))
+    if world_env is not None and world != args.gpus:
+        print(json.dumps({"error": f"WORLD_SIZE={world} but --gpus {args.gpus}"}), flush=True)
+        sys.exit(2)
     if world > 1:
         import torch
         import torch.distributed as dist
@@ -716,8 +987,10 @@ def main():
         (run_reference_c3 if args.impl == "reference" else run_ours_c3)(args, rank, world)
     elif args.impl == "reference":
         run_reference(args, rank, world)
+    elif args.loopback and args.gpus > 1:
+        run_ours(args, 0, args.gpus, "loopback")
     else:
-        run_ours(args, rank, world)
+        run_ours(args, rank, world, "dist" if world > 1 else "single")
     if world > 1:
         import torch.distributed as dist
         dist.destroy_process_group()

@@ -172,14 +172,16 @@ def _inlet_faces(c2n, c2c, xyz, zin) -> np.ndarray:
 # ----------------------------------------------------------------------------
 
 def seed_particles(mesh: dict, n: int, seed: int, drift: float = 0.25,
-                   spread: float = 0.05, id_base: int = 0, cluster=None) -> dict:
+                   spread: float = 0.05, id_base: int = 0, cluster=None, first: int = 0) -> dict:
     """n particles: cell uniform over tets (or clustered), point uniform in the
     tet (gaps of 3 sorted uniforms), v = drift*z + U(-spread, spread)^3.
 
     cluster = (frac, cell_ids): that fraction of particles is drawn uniformly
     from cell_ids instead (config C5).
+    first: generate particles [first, first + n) of the population (chunks
+    of a large population equal generating it at once).
     """
-    idx = np.arange(n, dtype=np.uint64)
+    idx = np.arange(first, first + n, dtype=np.uint64)
     nc = mesh["n_cells"]
     u = u01(seed, STREAM_CELL, idx * np.uint64(2))
     cell = np.minimum((u * nc).astype(np.int64), nc - 1)
@@ -202,7 +204,7 @@ def seed_particles(mesh: dict, n: int, seed: int, drift: float = 0.25,
     return {
         "pos": np.ascontiguousarray(pos), "vel": np.ascontiguousarray(vel),
         "cell": np.ascontiguousarray(cell.astype(np.int32)),
-        "id": np.arange(id_base, id_base + n, dtype=np.int64),
+        "id": np.arange(id_base + first, id_base + first + n, dtype=np.int64),
     }
 
 
@@ -274,6 +276,12 @@ CONFIGS = {
                c1E=(0.0, 0.0, 1e-3), dt=1.0, w=1.0),
     # C2: 48x48x72 hex = 995,328 tets, pre-seeded 50M steady state + 250k/step
     "c2": dict(dims=(48, 48, 72), n0=50_000_000, n_inj=250_000, steps=200, seed=20240813,
+               c1E=(0.0, 0.0, 1e-3), dt=1.0, w=1.0),
+    # C4: weak scaling, per GPU a 40x40x72-hex slab (691,200 tets) holding 1e9
+    # particles (~1,447 per cell, the paper's ~70M per 48k cells,
+    # PAPER.md:1885-1903); the global duct is 40x40x(72 N); injection on
+    # rank 0 balances the outflow at 0.25 h/step over 72 layers (1e9 / 288)
+    "c4": dict(dims=(40, 40, 72), n0=1_000_000_000, n_inj=3_500_000, steps=20, seed=20240815,
                c1E=(0.0, 0.0, 1e-3), dt=1.0, w=1.0),
     # C5: C2 mesh, 90% of 50M particles in the 12^3-hex block, no injection
     "c5": dict(dims=(48, 48, 72), n0=50_000_000, n_inj=0, steps=10, seed=20240816,

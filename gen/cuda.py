@@ -30,7 +30,7 @@ def lib():
     if _lib is None:
         _lib = C.CDLL(build())
         P, L, U, D = C.c_void_p, C.c_longlong, C.c_ulonglong, C.c_double
-        _lib.gen_seed_particles.argtypes = [P, P, L, L, U, D, D, L, P, L, D, P, P, P, P, P]
+        _lib.gen_seed_particles.argtypes = [P, P, L, L, L, U, D, D, L, P, L, D, P, P, P, P, P]
         _lib.gen_inject_batch.argtypes = [P, P, L, L, L, U, D, L, P, P, P, P, P]
         I = C.c_int
         _lib.gen_em_two_stream.argtypes = [I, I, I, I, U, D, D, D, P, P, P, P, P, P]
@@ -59,7 +59,9 @@ def _out(n, device):
 
 
 def seed_particles(dm: DeviceMesh, n: int, seed: int, drift=0.25, spread=0.05, id_base=0,
-                   cluster=None, stream=None):
+                   cluster=None, stream=None, first=0):
+    """Particles [first, first + n) of the seeded population (chunks of a
+    large population are bit-identical to generating it at once)."""
     import torch
     o = _out(n, dm.device)
     hot_t, nhot, frac = None, 0, 0.0
@@ -68,7 +70,7 @@ def seed_particles(dm: DeviceMesh, n: int, seed: int, drift=0.25, spread=0.05, i
         hot_t = torch.from_numpy(np.asarray(hot, dtype=np.int64)).to(dm.device)
         nhot = hot_t.numel()
     s = stream if stream is not None else torch.cuda.current_stream().cuda_stream
-    rc = lib().gen_seed_particles(dm.xyz.data_ptr(), dm.c2n.data_ptr(), dm.nc, n, seed, drift, spread,
+    rc = lib().gen_seed_particles(dm.xyz.data_ptr(), dm.c2n.data_ptr(), dm.nc, first, n, seed, drift, spread,
                                   id_base, hot_t.data_ptr() if hot_t is not None else None, nhot,
                                   float(frac), o["pos"].data_ptr(), o["vel"].data_ptr(),
                                   o["cell"].data_ptr(), o["id"].data_ptr(), s)

@@ -46,12 +46,13 @@ struct Keys {
 };
 
 __global__ void k_seed(const double *__restrict__ xyz, const int *__restrict__ c2n, long long nc,
-                       long long n, Keys k, double drift, double spread, long long id_base,
+                       long long first, long long n, Keys k, double drift, double spread, long long id_base,
                        const long long *__restrict__ hot, long long nhot, double frac,
                        double *pos, double *vel, int *cell, long long *id) {
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
          i += (long long)gridDim.x * blockDim.x) {
-        const unsigned long long ui = (unsigned long long)i;
+        // particle first + i of the seeded population (chunked generation)
+        const unsigned long long ui = (unsigned long long)(first + i);
         double u = u01(k.cell, ui * 2ull);
         long long c = (long long)dm(u, (double)nc);
         if (c > nc - 1) c = nc - 1;
@@ -81,7 +82,7 @@ __global__ void k_seed(const double *__restrict__ xyz, const int *__restrict__ c
             vel[3 * i + d] = v;
         }
         cell[i] = (int)c;
-        id[i] = id_base + i;
+        id[i] = id_base + first + i;
     }
 }
 
@@ -140,7 +141,8 @@ __global__ void k_em_two_stream(long long n, int ppc, long long nxy, unsigned lo
 
 }  // namespace
 
-extern "C" int gen_seed_particles(const double *xyz, const int *c2n, long long nc, long long n,
+extern "C" int gen_seed_particles(const double *xyz, const int *c2n, long long nc, long long first,
+                                  long long n,
                                   unsigned long long seed, double drift, double spread,
                                   long long id_base, const long long *hot, long long nhot,
                                   double frac, double *pos, double *vel, int *cell, long long *id,
@@ -148,7 +150,7 @@ extern "C" int gen_seed_particles(const double *xyz, const int *c2n, long long n
     if (n <= 0) return 0;
     long long g = (n + 255) / 256;
     if (g > 148 * 16) g = 148 * 16;
-    k_seed<<<(int)g, 256, 0, (cudaStream_t)stream>>>(xyz, c2n, nc, n, keys(seed), drift, spread,
+    k_seed<<<(int)g, 256, 0, (cudaStream_t)stream>>>(xyz, c2n, nc, first, n, keys(seed), drift, spread,
                                                      id_base, hot, nhot, frac, pos, vel, cell, id);
     return (int)cudaGetLastError();
 }

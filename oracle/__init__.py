@@ -27,12 +27,24 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 ORC_DONE, ORC_REMOVE = 0, 2
 
 
+CC = "gcc"
+CFLAGS = ["-O2", "-ffp-contract=off", "-std=c99", "-Wall"]
+
+
 def build(force: bool = False) -> str:
     """Compile liboracle.so (gcc, -O2 -ffp-contract=off: no FMA, S11)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-std=c99", "-Wall",
-                               "-shared", "-fPIC", _SRC, "-o", _LIB, "-lm"])
+        subprocess.check_call([CC, *CFLAGS, "-shared", "-fPIC", _SRC, "-o", _LIB, "-lm"])
     return _LIB
+
+
+def build_info() -> dict:
+    """Compiler and flags of the oracle build (reported with cpu_baseline)."""
+    try:
+        ver = subprocess.run([CC, "--version"], capture_output=True, text=True).stdout.split("\n")[0]
+    except Exception:   # noqa: BLE001
+        ver = CC
+    return {"compiler": ver, "flags": " ".join(CFLAGS)}
 
 
 class _Params(C.Structure):

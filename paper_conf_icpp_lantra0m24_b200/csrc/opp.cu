@@ -82,10 +82,16 @@ struct PSet {
     cudaEvent_t stg_free[2] = {nullptr, nullptr}, stg_ready[2] = {nullptr, nullptr};
     int stg_next = 0;
     std::vector<int> cols;
-    std::vector<char *> alt;     // sort double buffers (one per column, lazily allocated)
-    long long alt_cap = 0;
+    // sort spares: one buffer per distinct column size (bytes per particle),
+    // capacity `cap`; a sort gathers a column into the spare of its size and
+    // swaps the two (no second copy of the whole set)
+    struct Spare {
+        size_t bpp;
+        char *ptr;
+    };
+    std::vector<Spare> spares;
+    long long spare_cap = 0;
     long long steps = 0;         // pushes so far (drives sort_every)
-    bool fused_sort = false;     // this step's move already wrote the particles sorted
 };
 
 struct Set {
@@ -158,15 +164,6 @@ struct opp_ctx_s {
     cudaStream_t cs = nullptr;     // copy stream (host injection staging)
     int nsm = 148;
     int bps = 0;                   // resident blocks / SM of the fused kernel
-    int tile_group = 16;           // OPP_TILE_GROUP: tiles per block visit (TileMap)
-    int dbg = 0;                   // OPP_PMD_DEBUG (diagnostic kernels; results invalid)
-    int refill = 0;                // OPP_REFILL: per-lane refill consumer in the tiled kernel
-    int minb = 3;                  // OPP_MINB: register cap for 3 resident blocks / SM
-    int sort_hgrid = 8;            // OPP_SORT_HGRID / OPP_SORT_RGRID: blocks per SM of the
-    int sort_rgrid = 8;            //   sort histogram / rank kernels
-    int prefetch = 0;              // OPP_PREFETCH: producer-warp L1 warming
-    int fuse_sort = 0;             // OPP_FUSE_SORT=1: sort steps write the move's output sorted
-                                   //   (C2: slower -- 2.71 vs 2.42 ms/step: scattered writes)
     std::vector<Set> sets;
     std::vector<Col> cols;
     std::vector<PSet> psets;
@@ -239,6 +236,10 @@ static int col_check(opp_ctx c, int h) {
     return OPP_OK;
 }
 
+// Consecutive 256-particle tiles a block of the fused kernel visits in a row
+// (TileMap): runs of adjacent cells per SM for L1 reuse of the walk lines.
+constexpr int kTileGroup = 16;
+
 static int grid_for(opp_ctx c, long long n, int cap_mult = 8) {
     long long g = (n + 255) / 256;
     long long cap = (long long)c->nsm * cap_mult;
@@ -303,14 +304,6 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
         return fail(OPP_ERR_CUDA, "copy stream");
     }
     cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, params->device);
-    if (const char *tg = getenv("OPP_TILE_GROUP")) c->tile_group = std::max(1, atoi(tg));
-    if (const char *db = getenv("OPP_PMD_DEBUG")) c->dbg = atoi(db);
-    if (const char *rf = getenv("OPP_REFILL")) c->refill = atoi(rf);
-    if (const char *mb = getenv("OPP_MINB")) c->minb = atoi(mb);
-    if (const char *e = getenv("OPP_SORT_HGRID")) c->sort_hgrid = atoi(e);
-    if (const char *e = getenv("OPP_SORT_RGRID")) c->sort_rgrid = atoi(e);
-    if (const char *pf = getenv("OPP_PREFETCH")) c->prefetch = atoi(pf);
-    if (const char *fs = getenv("OPP_FUSE_SORT")) c->fuse_sort = atoi(fs);
     if (cudaMallocHost(&c->hcnt, sizeof(DevCounters)) != cudaSuccess) {
         cudaStreamDestroy(c->cs);
         delete c;
@@ -328,6 +321,12 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
     }
     *out = c;
     return OPP_OK;
+}
+
+static void free_spares(opp_ctx c, PSet &ps) {
+    for (auto &sp : ps.spares) c->dfree(sp.ptr, sp.bpp * (size_t)ps.spare_cap);
+    ps.spares.clear();
+    ps.spare_cap = 0;
 }
 
 static void free_pset(opp_ctx c, PSet &ps) {
@@ -369,9 +368,7 @@ extern "C" int opp_finalize(opp_ctx c) {
     if (!c) return OPP_OK;
     cudaSetDevice(c->p.device);
     cudaStreamSynchronize(c->s);
-    for (auto &ps : c->psets)
-        for (size_t j = 0; j < ps.alt.size(); j++)
-            c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
+    for (auto &ps : c->psets) free_spares(c, ps);
     for (auto &col : c->cols) c->dfree(col.d, col.bytes);
     for (auto &ps : c->psets) free_pset(c, ps);
     MeshCache &m = c->mc;
@@ -708,10 +705,7 @@ static int grow(opp_ctx c, PSet &ps, long long extra) {
     ps.holes = tmp.holes; ps.work = tmp.work; ps.head = tmp.head; ps.tail = tmp.tail;
     ps.work_hops = tmp.work_hops; ps.sr_cell = tmp.sr_cell; ps.sr_val = tmp.sr_val;
     ps.mig = tmp.mig; ps.mig_cell = tmp.mig_cell; ps.mig_hops = tmp.mig_hops;
-    for (size_t j = 0; j < ps.alt.size(); j++)
-        c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
-    ps.alt.clear();
-    ps.alt_cap = 0;
+    free_spares(c, ps);
     ps.cap = ncap;
     return OPP_OK;
 }
@@ -976,8 +970,7 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         m.ov_off = nullptr;
         m.ov_base = nullptr;
         ov.compact = 0;
-        const char *ce = getenv("OPP_OV_COMPACT");
-        if (!ce || atoi(ce)) {
+        {
             long long nbt = 1;
             for (int k = 0; k < 3; k++) {
                 ov.nbc[k] = (ov.n[k] + 3) / 4;
@@ -1045,57 +1038,67 @@ static int check_col(opp_ctx c, int h, bool want_map, int set, int dim, int type
     return OPP_OK;
 }
 
-// Counting sort by cell into the double buffers, then swap (drops holes).
-static int ensure_alt(opp_ctx c, PSet &ps) {
-    if (ps.alt_cap != ps.cap) {
-        for (size_t j = 0; j < ps.alt.size(); j++)
-            c->dfree(ps.alt[j], (size_t)ps.alt_cap * c->cols[ps.cols[j]].dim * c->cols[ps.cols[j]].eb);
-        ps.alt.assign(ps.cols.size(), nullptr);
-        for (size_t j = 0; j < ps.cols.size(); j++) {
-            Col &col = c->cols[ps.cols[j]];
-            ps.alt[j] = (char *)c->dalloc((size_t)ps.cap * col.dim * col.eb);
-            if (!ps.alt[j]) {
-                for (size_t k = 0; k < j; k++)
-                    c->dfree(ps.alt[k], (size_t)ps.cap * c->cols[ps.cols[k]].dim * c->cols[ps.cols[k]].eb);
-                ps.alt.clear();
-                ps.alt_cap = 0;
-                return fail(OPP_ERR_NOMEM, "sort buffers");
-            }
+// Spares for the sort: one buffer per distinct column size, allocated up
+// front so a failed allocation leaves the set unchanged.
+static int ensure_spares(opp_ctx c, PSet &ps) {
+    if (ps.spare_cap != ps.cap) free_spares(c, ps);
+    for (int h : ps.cols) {
+        const size_t bpp = (size_t)c->cols[h].dim * c->cols[h].eb;
+        bool have = false;
+        for (auto &sp : ps.spares) have = have || sp.bpp == bpp;
+        if (have) continue;
+        char *p = (char *)c->dalloc(bpp * (size_t)ps.cap);
+        if (!p) {
+            free_spares(c, ps);
+            return fail(OPP_ERR_NOMEM, "sort spare (%zu B per particle)", bpp);
         }
-        ps.alt_cap = ps.cap;
+        ps.spares.push_back(PSet::Spare{bpp, p});
+        ps.spare_cap = ps.cap;
     }
     return OPP_OK;
 }
 
-static int do_sort(opp_ctx c, PSet &ps, int p2c) {
+// Counting sort of the set by `keys` (the p2c map, or shuffle keys): count,
+// scan, rank (inverse permutation in ps.tail), then one gather per column
+// into the spare of its size, which becomes the column.  Drops holes.
+static int sort_by_keys(opp_ctx c, PSet &ps, const int32_t *keys, const uint32_t *skey) {
     MeshCache &m = c->mc;
-    if (!m.cell_hist) return fail(OPP_ERR_STATE, "sort needs the mesh: run a step first");
-    TRY(ensure_alt(c, ps));
-    ColSet src = make_colset(c, ps), dst = src;
-    for (int j = 0; j < dst.n; j++) dst.c[j].ptr = ps.alt[j];
-    const int32_t *pc = (const int32_t *)c->cols[p2c].d;
+    TRY(ensure_spares(c, ps));
     {
         PhaseScope ph(c, OPP_PH_SORT_COUNT);
-        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_hist,
-                             m.cell_start, m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
+        CK(launch_sort_count(keys, ps.dcnt, c->cell_base, m.nc, skey, m.cell_hist, m.cell_start,
+                             m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
+        CK(launch_sort_rank(keys, ps.dcnt, c->cell_base, skey, m.cell_start, ps.tail,
+                            grid_for(c, ps.n_ub, 8), c->s));
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        CK(launch_sort_move(src, dst, pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_start,
-                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), grid_for(c, ps.n_ub, c->sort_rgrid),
-                            c->s));
+        for (int h : ps.cols) {
+            Col &col = c->cols[h];
+            const size_t bpp = (size_t)col.dim * col.eb;
+            for (auto &sp : ps.spares) {
+                if (sp.bpp != bpp) continue;
+                CK(launch_sort_gather(ColDesc{col.d, ps.cap, col.eb, col.dim}, sp.ptr, ps.tail,
+                                      m.cell_start + m.nc, c->nsm * 4, c->s));
+                std::swap(col.d, sp.ptr);
+                break;
+            }
+        }
+        CK(launch_sort_commit(ps.dcnt, m.cell_start + m.nc, c->s));
     }
-    c->launches += 7;
-    for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
+    c->launches += 6 + (long long)ps.cols.size();
     ps.holes_pending = false;
     return OPP_OK;
 }
 
+static int do_sort(opp_ctx c, PSet &ps, int p2c) {
+    if (!c->mc.cell_hist) return fail(OPP_ERR_STATE, "sort needs the mesh: run a step first");
+    return sort_by_keys(c, ps, (const int32_t *)c->cols[p2c].d, c->mc.sort_key);
+}
+
 static int do_fill(opp_ctx c, PSet &ps, int p2c) {
     PhaseScope ph(c, OPP_PH_FILL);
-    if (c->p.sort_every > 0 && ps.steps % c->p.sort_every == 0 && !ps.fused_sort)
-        return do_sort(c, ps, p2c);
-    ps.fused_sort = false;
+    if (c->p.sort_every > 0 && ps.steps % c->p.sort_every == 0) return do_sort(c, ps, p2c);
     ColSet cs = make_colset(c, ps);
     CK(launch_fill(cs, ps.dcnt, ps.holes, (const int32_t *)c->cols[p2c].d, ps.head, ps.tail,
                    grid_for(c, ps.n_ub, 4), c->s));
@@ -1135,28 +1138,12 @@ extern "C" int opp_shuffle(opp_ctx c, opp_set parts, uint64_t seed) {
     if (p2c < 0) return fail(OPP_ERR_STATE, "particle set has no p2c map");
     MeshCache &m = c->mc;
     if (!m.cell_hist) return fail(OPP_ERR_STATE, "shuffle needs the mesh: run a step first");
-    TRY(ensure_alt(c, ps));
     PhaseScope ph(c, OPP_PH_FILL);
-    ColSet src = make_colset(c, ps), dst = src;
-    for (int j = 0; j < dst.n; j++) dst.c[j].ptr = ps.alt[j];
     int32_t *keys = (int32_t *)ps.work;   // the continuation worklist is free between steps
     CK(opp::launch_shuffle_keys((const int32_t *)c->cols[p2c].d, ps.dcnt, (unsigned long long)seed,
                                 m.nc, c->cell_base, keys, grid_for(c, ps.n_ub, 8), c->s));
-    {
-        PhaseScope ph2(c, OPP_PH_SORT_COUNT);
-        CK(launch_sort_count(keys, ps.dcnt, c->cell_base, m.nc, nullptr, m.cell_hist, m.cell_start,
-                             m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
-    }
-    {
-        PhaseScope ph2(c, OPP_PH_SORT_MOVE);
-        CK(launch_sort_move(src, dst, keys, ps.dcnt, c->cell_base, m.nc, nullptr, m.cell_start,
-                            ps.head, ps.tail, grid_for(c, ps.n_ub, 8), grid_for(c, ps.n_ub, c->sort_rgrid),
-                            c->s));
-    }
-    c->launches += 8;
-    for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
-    ps.holes_pending = false;
-    return OPP_OK;
+    c->launches++;
+    return sort_by_keys(c, ps, keys, nullptr);
 }
 
 // Refresh the particle-side pointers of the step arguments (after growth).
@@ -1164,10 +1151,6 @@ static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int
     a.pos = (double *)c->cols[pos].d;
     a.vel = (double *)c->cols[vel].d;
     a.p2c = (int32_t *)c->cols[p2c].d;
-    a.pos_out = a.pos;
-    a.vel_out = a.vel;
-    a.p2c_out = a.p2c;
-    a.dest = nullptr;
     a.cap = ps.cap;
     a.holes = ps.holes;
     a.work = ps.work;
@@ -1288,51 +1271,6 @@ static int read_stats(opp_ctx c, PSet &ps, opp_step_stats *stats) {
     return OPP_OK;
 }
 
-// Sort fused into the move (a sort step, opp_init_params.sort_every): the
-// counting sort's rank pass runs on the START cells before the move, and the
-// move writes every particle straight to its sorted position in the second
-// buffers (the columns it does not touch, e.g. ids, are scattered here); the
-// buffers are swapped after the move.  Saves the sort's separate read +
-// write of every particle (the auxiliary sort).
-static int fused_sort_prepass(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int p2c) {
-    MeshCache &m = c->mc;
-    TRY(ensure_alt(c, ps));
-    int jp = -1, jv = -1, jc = -1;
-    ColSet src{}, dst{};
-    for (size_t j = 0; j < ps.cols.size(); j++) {
-        const int h = ps.cols[j];
-        if (h == pos) jp = (int)j;
-        else if (h == vel) jv = (int)j;
-        else if (h == p2c) jc = (int)j;
-        else {
-            const Col &col = c->cols[h];
-            src.c[src.n] = ColDesc{col.d, ps.cap, col.eb, col.dim};
-            dst.c[dst.n] = ColDesc{ps.alt[j], ps.cap, col.eb, col.dim};
-            src.n++;
-            dst.n++;
-        }
-    }
-    if (jp < 0 || jv < 0 || jc < 0) return fail(OPP_ERR_STATE, "fused sort: columns not found");
-    const int32_t *pc = (const int32_t *)c->cols[p2c].d;
-    {
-        PhaseScope ph(c, OPP_PH_SORT_COUNT);
-        CK(launch_sort_count(pc, ps.dcnt, c->cell_base, m.nc, m.sort_key, m.cell_hist, m.cell_start,
-                             m.tile_sums, grid_for(c, ps.n_ub, c->sort_hgrid), c->s));
-        CK(launch_sort_rank(pc, ps.dcnt, c->cell_base, m.sort_key, m.cell_start, ps.head, ps.tail,
-                            grid_for(c, ps.n_ub, c->sort_rgrid), c->s));
-    }
-    {
-        PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        CK(launch_scatter_cols(src, dst, ps.head, ps.dcnt, grid_for(c, ps.n_ub, 8), c->s));
-    }
-    c->launches += 6;
-    a.pos_out = (double *)ps.alt[jp];
-    a.vel_out = (double *)ps.alt[jv];
-    a.p2c_out = (int32_t *)ps.alt[jc];
-    a.dest = ps.head;
-    return OPP_OK;
-}
-
 extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_dat vel,
                                      opp_map p2c, opp_map c2c, opp_map c2n, opp_dat node_pos,
                                      opp_dat cell_ef, opp_dat node_charge,
@@ -1363,10 +1301,6 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.pos = (double *)c->cols[pos].d;
     a.vel = (double *)c->cols[vel].d;
     a.p2c = (int32_t *)c->cols[p2c].d;
-    a.pos_out = a.pos;
-    a.vel_out = a.vel;
-    a.p2c_out = a.p2c;
-    a.dest = nullptr;
     a.cap = ps.cap;
     a.lines = m.lines;
     a.ef = m.efp;
@@ -1387,11 +1321,7 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.n_cells = (int)m.nc;
     a.hpass = c->p.hop_budget_per_pass;
     a.hcap = c->p.hop_cap;
-    a.tile_group = c->tile_group;
-    a.dbg = c->dbg;
-    a.refill = c->refill;
-    a.minb = c->minb;
-    a.prefetch = c->prefetch;
+    a.tile_group = kTileGroup;
     a.ov = m.ov;
     const int dep = c->p.deposit_mode;
     const int dh = c->p.direct_hop;
@@ -1404,22 +1334,14 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     }
     c->launches++;
     const bool tiled = c->p.tma_pipeline != 0;
-    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled, c->minb);
+    if (!c->bps) c->bps = opp::pmd_blocks_per_sm(tiled);
     const int bps = c->bps;
     const int pgrid = (int)std::max<long long>(1, std::min<long long>((ps.n_ub + 255) / 256,
                                                                        (long long)c->nsm * bps));
-    const bool fuse = c->fuse_sort && c->p.sort_every > 0 && (ps.steps + 1) % c->p.sort_every == 0 &&
-                      m.cell_hist && !c->refill && !c->dbg;
-    if (fuse) TRY(fused_sort_prepass(c, ps, a, pos, vel, p2c));
     {
         PhaseScope ph(c, OPP_PH_PUSH_MOVE_DEPOSIT);
         const int g1 = tiled ? c->nsm * bps : pgrid;
         CK(launch_push_move_deposit(dep, dh, multi, false, tiled, a, g1, c->s));
-    }
-    if (fuse) {   // the sorted copies become the particle set
-        for (size_t j = 0; j < ps.cols.size(); j++) std::swap(c->cols[ps.cols[j]].d, ps.alt[j]);
-        refresh_args(c, ps, a, pos, vel, p2c);
-        ps.fused_sort = true;
     }
     {
         PhaseScope ph(c, OPP_PH_CONTINUE);
@@ -1910,26 +1832,30 @@ extern "C" int opp_em_sort_by_cell(opp_ctx c, int64_t n, int64_t stride, const d
     }
     es.n_host = (unsigned long long)n;
     CK(cudaMemcpyAsync(&es.dc->n, &es.n_host, sizeof(unsigned long long), cudaMemcpyHostToDevice, c->s));
-    ColSet src{}, dst{};
+    // every cell id must lie in [0, n_cells): out-of-range ids would index the
+    // histogram out of bounds (checked on the device, one flag read back)
+    CK(cudaMemsetAsync(&es.dc->err_flags, 0, sizeof(unsigned), c->s));
+    CK(opp::launch_check_cells(cell, n, n_cells, &es.dc->err_flags, grid_for(c, n, 4), c->s));
+    unsigned bad = 0;
+    CK(cudaMemcpyAsync(&bad, &es.dc->err_flags, sizeof bad, cudaMemcpyDeviceToHost, c->s));
+    CK(cudaStreamSynchronize(c->s));
+    if (bad) return fail(OPP_ERR_ARG, "opp_em_sort_by_cell: a cell id lies outside [0, n_cells)");
     const void *in[4] = {off, u, w, cell};
-    void *out[4] = {off_out, u_out, w_out, cell_out};
+    char *out[4] = {(char *)off_out, (char *)u_out, (char *)w_out, (char *)cell_out};
     const int dims[4] = {3, 3, 1, 1}, ebs[4] = {8, 8, 8, 4};
-    for (int j = 0; j < 4; j++) {
-        src.c[j] = ColDesc{(char *)in[j], stride, ebs[j], dims[j]};
-        dst.c[j] = ColDesc{(char *)out[j], stride, ebs[j], dims[j]};
-    }
-    src.n = dst.n = 4;
     {
         PhaseScope ph(c, OPP_PH_SORT_COUNT);
         CK(launch_sort_count(cell, es.dc, 0, n_cells, nullptr, es.hist, es.start, es.tile_sums,
-                             grid_for(c, n, c->sort_hgrid), c->s));
+                             grid_for(c, n, 8), c->s));
+        CK(launch_sort_rank(cell, es.dc, 0, nullptr, es.start, es.src_of, grid_for(c, n, 8), c->s));
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        CK(launch_sort_move(src, dst, cell, es.dc, 0, n_cells, nullptr, es.start, nullptr, es.src_of,
-                            grid_for(c, n, 8), grid_for(c, n, c->sort_rgrid), c->s));
+        for (int j = 0; j < 4; j++)
+            CK(launch_sort_gather(ColDesc{(char *)in[j], stride, ebs[j], dims[j]}, out[j], es.src_of,
+                                  es.start + n_cells, c->nsm * 4, c->s));
     }
-    c->launches += 7;
+    c->launches += 10;
     return OPP_OK;
 }
 
@@ -1967,7 +1893,6 @@ extern "C" int opp_em_move_deposit(opp_ctx c, int64_t n, int64_t stride, double 
     a.kcap = prm->kcap;
     a.dep = prm->deposit_mode == OPP_DEP_ATOMIC_WARPAGG ? 1 : 0;
     a.cnt = c->em_cnt;
-    if (const char *ed = getenv("OPP_EM_DEFER")) c->em_defer = atoi(ed);
     if (c->em_defer && n > c->em_work_cap) {
         c->dfree(c->em_work, 0);
         c->em_work = (uint32_t *)c->dalloc(4 * (size_t)n);
@@ -2012,7 +1937,6 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     a.z = f.vec + 7 * nn;
     a.q = f.vec + 8 * nn;
     a.pipelined = 1;
-    if (const char *e = getenv("OPP_CG_PIPE")) a.pipelined = atoi(e);
     a.part = f.part;
     a.st = f.st;
     a.rhs_scale = prm->rhs_scale;
@@ -2032,7 +1956,6 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
         c->launches++;
         f.xprev_dat = node_potential;
     }
-    if (const char *e = getenv("OPP_CG_DBG")) a.dbg = atoi(e);
     {
         PhaseScope ph(c, OPP_PH_FIELD);
         int grid = 0;
@@ -2041,8 +1964,7 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
         if (nn > 0 && (c->p.nranks > 1 || (hl && atoi(hl)))) {
             TRY(field_solve_hostloop(c, a));
         } else if (nn > 0) {
-            int bps = 2;
-            if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
+            int bps = 2;   // blocks per SM: 2 (1.50 ms per C2 solve) beat 1 (1.91 ms)
             bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
             CK(launch_cg(a, c->nsm, bps, c->s, &grid));
             c->launches++;
@@ -2204,8 +2126,7 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
             a.max_iter = prm->cg_max_iter;
             a.warm = 0;
             a.precond = prm->precond != 0;
-            int bps = 2;
-            if (const char *e = getenv("OPP_CG_BPS")) bps = std::max(1, atoi(e));
+            int bps = 2;   // blocks per SM: 2 (1.50 ms per C2 solve) beat 1 (1.91 ms)
             bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
             double thr = 0.0;
             bool pending_it = false;   // single rank: CG iterations still on the device

@@ -656,12 +656,9 @@ cudaError_t launch_field_assemble(const double *xyz, const int32_t *c2n, const i
 cudaError_t launch_cg(const CgArgs &a, int nsm, int max_bps, cudaStream_t s, int *grid_out) {
     int occ = 0;
     const void *fn = a.pipelined ? (const void *)k_pcg : (const void *)k_cg;
-    // OPP_CG_REG (default 1): k_pcg_reg<R>, the smallest R (<= 6) for which
-    // every thread's rows fit its R shared-memory slots at the grid it gets
-    static const int use_reg = [] {
-        const char *e = getenv("OPP_CG_REG");
-        return e ? atoi(e) : 1;
-    }();
+    // k_pcg_reg<R>: the smallest R (<= 6) for which every thread's rows fit
+    // its R shared-memory slots at the grid it gets (else k_pcg)
+    constexpr int use_reg = 1;
     size_t dsm = 0;
     if (a.pipelined && use_reg) {
         const void *regk[6] = {(const void *)k_pcg_reg<1>, (const void *)k_pcg_reg<2>,

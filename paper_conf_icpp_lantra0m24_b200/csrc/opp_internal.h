@@ -99,22 +99,10 @@ struct StepArgs {
     uint32_t *mig;             // migrants: particle index, target global cell, hops
     int32_t *mig_cell;
     int32_t *mig_hops;
-    // sort fused into the move (sort steps, opp_init_params.sort_every): the
-    // particle with index i is written to position dest[i] of the *_out
-    // columns (the sort's second buffers, counting-sorted by start cell) and
-    // recorded (holes, deferred walks, migrants) under that position.
-    // Otherwise dest == NULL and the *_out columns are the inputs (in place).
-    double *pos_out, *vel_out;
-    int32_t *p2c_out;
-    const uint32_t *dest;
     double c1, dt, w;
     int cell_base, n_cells;    // global id of local cell 0, local cell count
     int hpass, hcap;
     int tile_group;            // consecutive 256-particle tiles per block visit (>= 1)
-    int refill;                // tiled kernel: per-lane refill consumer (OPP_REFILL)
-    int minb;                  // tiled kernel: min resident blocks per SM (OPP_MINB: 1 or 3)
-    int prefetch;              // tiled kernel: producer-warp L1 warming (OPP_PREFETCH, default 1)
-    int dbg;                   // diagnostics only (OPP_PMD_DEBUG): 1 stream, 2 +E, 3 +line, 4 no deposit
     Overlay ov;
 };
 

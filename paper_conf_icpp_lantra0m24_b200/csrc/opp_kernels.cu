@@ -29,22 +29,15 @@ __device__ __forceinline__ double sub(double a, double b) { return __dsub_rn(a, 
 
 struct Line {
     double g0, g1, g2, g3, g4, g5, g6, g7, g8, px, py, pz;
-    int4 cc, cn;
 };
 
-#ifndef OPP_LAZY_LINE
-// 1: a visit loads only the 96 B lambda needs (gradients, p0: three 256-bit
-// loads); the neighbour ids (c2c) are loaded by the lanes that hop and the
-// node ids (c2n) by the lanes that issue the deposit reductions.  An L1 load
-// costs ~8 SM cycles per 256-bit warp instruction and distinct line even for
-// one active lane (scripts/micro/wf_cost.cu), so the fourth sector of every
-// visit was a quarter of the walk's L1 data-pipe time.
-#define OPP_LAZY_LINE 1
-#endif
-constexpr bool kLazyLine = OPP_LAZY_LINE != 0;
-
-// One 128-B walk line: four 256-bit read-only loads (LDG.E.256), or the first
-// three (lazy: the c2c / c2n sector is read on demand, below).
+// The 96 B of a walk line that lambda needs (gradients, p0): three 256-bit
+// read-only loads (LDG.E.256).  The neighbour ids (c2c, bytes 96..111) are
+// loaded only by the lanes that hop and the node ids (c2n, 112..127) only by
+// the lanes that issue the deposit reductions: an L1 load costs ~8 SM cycles
+// per 256-bit warp instruction and distinct line even for one active lane
+// (scripts/micro/wf_cost.cu), so a fourth sector per visit was a quarter of
+// the walk's L1 data-pipe time.
 __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, int c) {
     const double *L = reinterpret_cast<const double *>(lines + c);
     Line l;
@@ -54,11 +47,6 @@ __device__ __forceinline__ Line load_line(const WalkLine *__restrict__ lines, in
         : "=d"(l.g4), "=d"(l.g5), "=d"(l.g6), "=d"(l.g7) : "l"(L + 4));
     asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
         : "=d"(l.g8), "=d"(l.px), "=d"(l.py), "=d"(l.pz) : "l"(L + 8));
-    if (!kLazyLine) {
-        asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-            : "=r"(l.cc.x), "=r"(l.cc.y), "=r"(l.cc.z), "=r"(l.cc.w),
-              "=r"(l.cn.x), "=r"(l.cn.y), "=r"(l.cn.z), "=r"(l.cn.w) : "l"(L + 12));
-    }
     return l;
 }
 
@@ -69,27 +57,10 @@ __device__ __forceinline__ int4 line_c2c(const WalkLine *__restrict__ lines, int
 __device__ __forceinline__ int4 line_c2n(const WalkLine *__restrict__ lines, int c) {
     return __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(lines + c) + 14));
 }
-__device__ __forceinline__ int line_node(const WalkLine *__restrict__ lines, int c, int q) {
-    return __ldg(reinterpret_cast<const int *>(reinterpret_cast<const double *>(lines + c) + 14) + q);
-}
-// the neighbours of the cell whose line L is (lc: its local index)
-__device__ __forceinline__ int4 cc_of(const WalkLine *__restrict__ lines, const Line &L, int lc) {
-    return kLazyLine ? line_c2c(lines, lc) : L.cc;
-}
 
-// Cell field E (double4, 32-B aligned): one 256-bit read-only load, or
-// (OPP_E_NARROW) a 128-bit + a 64-bit load of just the 24 B used.
-#ifndef OPP_E_NARROW
-#define OPP_E_NARROW 0
-#endif
+// Cell field E (double4, 32-B aligned): one 256-bit read-only load.
 __device__ __forceinline__ void load_E(const double4 *__restrict__ ef, int lc, double2 &exy,
                                        double &ez) {
-    if (OPP_E_NARROW) {
-        const double *p = reinterpret_cast<const double *>(ef + lc);
-        exy = __ldg(reinterpret_cast<const double2 *>(p));
-        ez = __ldg(p + 2);
-        return;
-    }
     double pad;
     asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
         : "=d"(exy.x), "=d"(exy.y), "=d"(ez), "=d"(pad) : "l"(ef + lc));
@@ -135,49 +106,38 @@ __device__ __forceinline__ void bary(const Line &l, double x, double y, double z
 
 __device__ __forceinline__ bool in01(double v) { return v >= 0.0 && v <= 1.0; }
 
+// Most-probable neighbour (reading S2): the face opposite
+// the most negative lambda, lowest local index on a tie.
+__device__ __forceinline__ int argmin_face(double l0, double l1, double l2, double l3) {
+    int f = 0;
+    double m = l0;
+    if (l1 < m) { m = l1; f = 1; }
+    if (l2 < m) { m = l2; f = 2; }
+    if (l3 < m) { f = 3; }
+    return f;
+}
+__device__ __forceinline__ int pick(int4 v, int f) {
+    return f == 0 ? v.x : f == 1 ? v.y : f == 2 ? v.z : v.w;
+}
 
 // Multi-hop walk (Fig. 6 template 1098-1124).  `cell` is a
 // global id in/out and L its already-loaded walk line; stops when inside
 // (DONE), at H_cap (DONE, capped), when hops reaches stop_at (NEED_MOVE:
 // deferred), across a boundary face (NEED_REMOVE) or into a cell another
 // rank owns (NEED_MIGRATE).
-// Position source for the walk: registers, or (TMA-pipelined kernel) the
-// warp's shared output buffer, re-read at every visit so the three doubles do
-// not occupy registers across the line-load latency.
-struct PosRegs {
-    double x, y, z;
-    __device__ __forceinline__ void get(double &a, double &b, double &c) const { a = x; b = y; c = z; }
-};
-struct PosSmem {
-    const double *p;   // p[0], p[32], p[64]
-    __device__ __forceinline__ void get(double &a, double &b, double &c) const {
-        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(a) : "r"((unsigned)__cvta_generic_to_shared(p)));
-        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(b) : "r"((unsigned)__cvta_generic_to_shared(p + 32)));
-        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(c) : "r"((unsigned)__cvta_generic_to_shared(p + 64)));
-    }
-};
-
-template <bool MULTI, typename PS>
-__device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, const PS &ps,
-                                         int &hops, int stop_at, double &l0, double &l1,
-                                         double &l2, double &l3, int &capped, int4 &cn) {
+template <bool MULTI>
+__device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, double x, double y,
+                                         double z, int &hops, int stop_at, double &l0, double &l1,
+                                         double &l2, double &l3, int &capped) {
     for (;;) {
-        double x, y, z;
-        ps.get(x, y, z);
         bary(L, x, y, z, l0, l1, l2, l3);
-        cn = L.cn;
         if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) return ST_DONE;
         if (hops >= a.hcap) {
             capped = 1;
             return ST_DONE;
         }
         if (hops >= stop_at) return ST_MOVE;
-        const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
-        int nb = cc.x;
-        double m = l0;
-        if (l1 < m) { m = l1; nb = cc.y; }
-        if (l2 < m) { m = l2; nb = cc.z; }
-        if (l3 < m) { nb = cc.w; }
+        const int nb = pick(line_c2c(a.lines, cell - a.cell_base), argmin_face(l0, l1, l2, l3));
         if (nb < 0) return ST_REMOVE;
         if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
             cell = nb;       // the hop into the other rank's cell counts here
@@ -207,39 +167,14 @@ __device__ __forceinline__ unsigned long long warp_append(bool pred, unsigned lo
 // DEP 0: one fp64 reduction per (particle, node).
 // DEP 1: lanes with the same cell (same 4 nodes) are aggregated inside the
 //        warp before one set of 4 reductions per cell -- "warp-level
-//        aggregation of same-cell deposits before global atomics".
-//
-// Lanes with the same key are found with __match_any_sync wherever they sit
-// in the warp.  A lane alone with its cell reduces straight to Q.  Each
-// group of >= 2 lanes (in cell-sorted storage: the one or two cells a warp's
-// slice covers, while the few particles that hopped are mostly alone) is
-// summed by a full-warp reduce-scatter -- xor 16 halves the 4 values, xor 8
-// halves them again, xor 4/2/1 finish -- 12 shuffles and 6 adds per group;
-// lanes 0, 8, 16, 24 then hold the group's 4 sums and issue one reduction
-// each.  With more than kMaxRsGroups groups a log-step tree over each group
-// (lowest lane issues the 4 reductions) is cheaper.
-#ifndef OPP_RS_GROUPS
-#define OPP_RS_GROUPS 0   // C2: 0 (always the tree) 1.894 ms, 3: 1.912, 8: 2.35
-#endif
-constexpr int kMaxRsGroups = OPP_RS_GROUPS;
-#ifndef OPP_DEP_MERGE
-#define OPP_DEP_MERGE 1   // singles through the tree too: C2 pass 1 1.901 -> 1.849 ms, C5 2.80 -> 2.71
-#endif
-
-// Node ids of the depositing cell: from the walk line already in registers,
-// or (lazy line) loaded by the lanes that issue the reductions only.
-struct CnSrc {
-    const WalkLine *lines;
-    int base;   // cell_base: key - base is the local cell
-    __device__ __forceinline__ int4 get(int key, int4 cn) const {
-        return kLazyLine ? line_c2n(lines, key - base) : cn;
-    }
-    __device__ __forceinline__ int node(int key, int4 cn, int q) const {
-        if (kLazyLine) return line_node(lines, key - base, q);
-        return q == 0 ? cn.x : q == 1 ? cn.y : q == 2 ? cn.z : cn.w;
-    }
-};
-
+//        aggregation of same-cell deposits before global atomics".  Lanes
+//        with the same key are found with __match_any_sync wherever they sit
+//        in the warp and summed by a log-step tree per group; cells with a
+//        single particle ride through the same tree as groups of one, so all
+//        cells' reductions leave in the same 4 instructions (a reduction
+//        instruction has a fixed L1 cost: C2 pass 1 1.901 -> 1.849 ms against
+//        reducing singles separately).  The group's lowest lane loads the
+//        cell's node ids while the tree runs.
 __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0, double v1,
                                      double v2, double v3) {
     atomicAdd(Q + cn.x, v0);
@@ -248,99 +183,44 @@ __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0,
     atomicAdd(Q + cn.w, v3);
 }
 
-// Log-step tree over every peer group of the lanes with `act` set.
-__device__ __forceinline__ void deposit_tree(double *__restrict__ Q, bool act, unsigned peers,
-                                             const CnSrc &cs, int key, int4 cn, double v0,
-                                             double v1, double v2, double v3) {
+__device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepArgs &a, bool act,
+                                            int key, double v0, double v1, double v2, double v3) {
+    const unsigned FULL = 0xffffffffu;
+    if (!__any_sync(FULL, act)) return;
     const unsigned lane = lane_id();
+    const unsigned peers = __match_any_sync(FULL, act ? key : -2 - (int)lane);
     const int first = __ffs(peers) - 1;
     int rel = __popc(peers & ((1u << lane) - 1u));       // my rank inside the group
     unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
     if (lane == 31) up = 0;
-    // the lowest lane of each group fetches the node ids while the tree runs
-    if (act && (int)lane == first) cn = cs.get(key, cn);
-    while (__any_sync(0xffffffffu, up != 0)) {
+    int4 cn = make_int4(0, 0, 0, 0);
+    if (act && (int)lane == first) cn = line_c2n(a.lines, key - a.cell_base);
+    while (__any_sync(FULL, up != 0)) {
         const int next = up ? __ffs(up) - 1 : (int)lane;
-        const double t0 = __shfl_sync(0xffffffffu, v0, next);
-        const double t1 = __shfl_sync(0xffffffffu, v1, next);
-        const double t2 = __shfl_sync(0xffffffffu, v2, next);
-        const double t3 = __shfl_sync(0xffffffffu, v3, next);
+        const double t0 = __shfl_sync(FULL, v0, next);
+        const double t1 = __shfl_sync(FULL, v1, next);
+        const double t2 = __shfl_sync(FULL, v2, next);
+        const double t3 = __shfl_sync(FULL, v3, next);
         if (up) {
             v0 = add(v0, t0); v1 = add(v1, t1); v2 = add(v2, t2); v3 = add(v3, t3);
         }
         // lanes at odd group rank have been absorbed by their lower neighbour
-        const unsigned gone = __ballot_sync(0xffffffffu, (rel & 1) != 0);
+        const unsigned gone = __ballot_sync(FULL, (rel & 1) != 0);
         up &= ~gone;
         rel >>= 1;
     }
     if (act && (int)lane == first) red4(Q, cn, v0, v1, v2, v3);
 }
 
-// Warp-aggregated deposit of (key, cn, v0..v3) for the lanes with `done`
-// (key: the cell; lanes with equal keys have equal cn).
-__device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const CnSrc &cs, bool done,
-                                            int key, int4 cn, double v0, double v1, double v2,
-                                            double v3) {
-    const unsigned FULL = 0xffffffffu;
-    const unsigned lane = lane_id();
-    const unsigned peers = __match_any_sync(FULL, done ? key : -2 - (int)lane);
-    const bool single = peers == (1u << lane);
-    if (OPP_DEP_MERGE && kMaxRsGroups == 0) {
-        // singles ride through the tree as groups of one, so every cell's
-        // four reductions leave in the same four instructions (the fixed
-        // cost of a reduction instruction is paid once, not twice)
-        if (__any_sync(FULL, done)) deposit_tree(Q, done, peers, cs, key, cn, v0, v1, v2, v3);
-        return;
-    }
-    if (done && single) red4(Q, cs.get(key, cn), v0, v1, v2, v3);
-    unsigned lead = __ballot_sync(FULL, done && !single && (int)lane == __ffs(peers) - 1);
-    if (!lead) return;
-    if (__popc(lead) > kMaxRsGroups) {
-        deposit_tree(Q, done && !single, peers, cs, key, cn, v0, v1, v2, v3);
-        return;
-    }
-    const bool h16 = (lane & 16u) != 0, h8 = (lane & 8u) != 0;
-    do {
-        const int L = __ffs(lead) - 1;
-        lead &= lead - 1u;
-        const unsigned gm = __shfl_sync(FULL, peers, L);
-        const bool in = done && ((gm >> lane) & 1u);
-        const double a0 = in ? v0 : 0.0, a1 = in ? v1 : 0.0, a2 = in ? v2 : 0.0, a3 = in ? v3 : 0.0;
-        double k0 = h16 ? a2 : a0, k1 = h16 ? a3 : a1;    // the pair this lane keeps
-        const double s0 = h16 ? a0 : a2, s1 = h16 ? a1 : a3;
-        k0 = add(k0, __shfl_xor_sync(FULL, s0, 16));
-        k1 = add(k1, __shfl_xor_sync(FULL, s1, 16));
-        double t = h8 ? k1 : k0;
-        t = add(t, __shfl_xor_sync(FULL, h8 ? k0 : k1, 8));
-        t = add(t, __shfl_xor_sync(FULL, t, 4));
-        t = add(t, __shfl_xor_sync(FULL, t, 2));
-        t = add(t, __shfl_xor_sync(FULL, t, 1));
-        // lane 8q holds the sum of value q = 2*h16 + h8
-        const int q = 2 * (int)h16 + (int)h8;
-        if (kLazyLine) {
-            const int kL = __shfl_sync(FULL, key, L);
-            if ((lane & 7u) == 0) atomicAdd(Q + cs.node(kL, cn, q), t);
-        } else {
-            const int n0 = __shfl_sync(FULL, cn.x, L), n1 = __shfl_sync(FULL, cn.y, L);
-            const int n2 = __shfl_sync(FULL, cn.z, L), n3 = __shfl_sync(FULL, cn.w, L);
-            if ((lane & 7u) == 0) {
-                const int node = h16 ? (h8 ? n3 : n2) : (h8 ? n1 : n0);
-                atomicAdd(Q + node, t);
-            }
-        }
-    } while (lead);
-}
-
 template <int DEP>
-__device__ __forceinline__ void deposit(double *__restrict__ Q, const CnSrc &cs, bool done,
-                                        int cell, int4 cn, double w, double l0, double l1,
-                                        double l2, double l3) {
+__device__ __forceinline__ void deposit(const StepArgs &a, bool done, int cell, double w,
+                                        double l0, double l1, double l2, double l3) {
     double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
     if (DEP == 0) {
-        if (done) red4(Q, cs.get(cell, cn), v0, v1, v2, v3);
+        if (done) red4(a.Q, line_c2n(a.lines, cell - a.cell_base), v0, v1, v2, v3);
         return;
     }
-    deposit_agg(Q, cs, done, cell, cn, v0, v1, v2, v3);
+    deposit_agg(a.Q, a, done, cell, v0, v1, v2, v3);
 }
 
 // SR deposit, phase 1: store (cell, w*lambda[4]) records.
@@ -354,6 +234,13 @@ __device__ __forceinline__ void sr_store(const StepArgs &a, bool done, int cell,
         a.sr_val[2 * a.cap + slot] = mul(w, l2);
         a.sr_val[3 * a.cap + slot] = mul(w, l3);
     }
+}
+
+template <int DEP>
+__device__ __forceinline__ void deposit_any(const StepArgs &a, bool done, int cell, double l0,
+                                            double l1, double l2, double l3) {
+    if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
+    else deposit<DEP>(a, done, cell, a.w, l0, l1, l2, l3);
 }
 
 // Per-warp flush of walk statistics.
@@ -394,28 +281,13 @@ __device__ __forceinline__ int dh_seed(const Overlay &ov, double x, double y, do
     return s >= 0 ? s : cell;
 }
 
-// DH mode 2 (reading S19''): a particle no longer inside its cell (L = its
-// line) takes the overlay seed; one still inside keeps cell and line.
-__device__ __forceinline__ void dh_if_left(const StepArgs &a, double x, double y, double z,
-                                           int &cell, Line &L) {
-    double l0, l1, l2, l3;
-    bary(L, x, y, z, l0, l1, l2, l3);
-    if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) return;
-    const int sc = dh_seed(a.ov, x, y, z, cell);
-    if (sc != cell) {
-        cell = sc;
-        L = load_line(a.lines, sc - a.cell_base);
-    }
-}
-
 }  // namespace
 
 // ---------------------------------------------------------------------------
 // Per-particle body shared by the fused kernel (both its TMA-tiled and its
-// direct paths) and the continuation pass.  Must be called by full warps
-// (the deposit / append collectives use all 32 lanes); `valid` masks lanes
-// without a particle.  On return x..vz and cell hold what is written back
-// (cell = -1 for a hole).
+// direct paths).  Must be called by full warps (the deposit / append
+// collectives use all 32 lanes); `valid` masks lanes without a particle.  On
+// return x..vz and cell hold what is written back (cell = -1 for a hole).
 // ---------------------------------------------------------------------------
 struct Tally {
     unsigned hops = 0, maxh = 0, capped = 0, removed = 0;
@@ -435,16 +307,15 @@ struct TileMap {
         if (b + (nb - 1) * G == ng - 1) c -= ng * K - ntiles;
         return c;
     }
-    __device__ __forceinline__ unsigned long long tile(unsigned long long it) const {
-        return ((it / K) * G + b) * K + it % K;
-    }
 };
 
 // Sequential walk over a block's tiles without 64-bit divisions.
 struct TileIter {
-    unsigned group_first, sub, K, step;   // step = G * K; tile ids < 2^32 / kTile
+    unsigned long long group_first;
+    unsigned sub, K;
+    unsigned long long step;   // G * K
     __device__ __forceinline__ TileIter(const TileMap &m)
-        : group_first((unsigned)(m.b * m.K)), sub(0), K((unsigned)m.K), step((unsigned)(m.G * m.K)) {}
+        : group_first(m.b * m.K), sub(0), K((unsigned)m.K), step(m.G * m.K) {}
     __device__ __forceinline__ unsigned long long tile() const { return group_first + sub; }
     __device__ __forceinline__ void next() {
         if (++sub == K) {
@@ -454,35 +325,19 @@ struct TileIter {
     }
 };
 
-// TMA-pipelined kernel geometry: tiles of kTile particles, kStages stages.
+// TMA-pipelined kernel geometry: tiles of kTile particles, kStages stages
+// (2 measured best on C2: more stages take L1 capacity from the walk lines,
+// pmd 1.91 -> 1.87 ms), 3 resident blocks per SM (68 registers, no spills).
 constexpr int kTile = 256;
 constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
-#ifndef OPP_STAGES
-#define OPP_STAGES 2   // measured on C2: 2 stages leave more of the L1/shared array to
-                       // L1 for the walk lines (pmd 1.91 -> 1.87 ms vs 4 stages)
-#endif
-#ifndef OPP_MINB_HI
-#define OPP_MINB_HI 3   // resident blocks per SM the register budget is cut for
-#endif
-constexpr int kStages = OPP_STAGES;
+constexpr int kStages = 2;
+constexpr int kMinBlocks = 3;
 constexpr int kStageBytes = kTile * (6 * 8 + 4);
-constexpr int kRingBytesPerWarp = 64 * 12 + 128;   // holes ring (4 B) + work ring (4 B + 4 B hops) + lane permutation (32 x 4 B)
-#ifndef OPP_SEED_PERM
-#define OPP_SEED_PERM 0   // 1: regroup a warp's lanes by seed cell before the first walk-line load
-                          // (C2: parity green, pass 1 1.844 -> 1.884 ms: the shuffles cost more than
-                          // the cheaper line loads save -- off)
-#endif
-#ifndef OPP_TMA_OUT
-// 0: results leave as coalesced per-lane stores (C2: pmd 1.99 vs 2.06 ms --
-// staging the stores in shared memory cost L1 data-pipe wavefronts twice,
-// the shared stores and the bulk copy's reads); 1: per-warp shared buffer +
-// cp.async.bulk shared -> global
-#define OPP_TMA_OUT 0
-#endif
-constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8 +
-                          (OPP_TMA_OUT ? (kTile / 32) * 32 * (6 * 8 + 4) : 0);
-constexpr int kTiledSmem = kRingBase + (kTile / 32) * kRingBytesPerWarp;
+constexpr int kRing = 64;
+constexpr int kRingBytesPerWarp = kRing * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
+constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8;
+constexpr int kTiledSmem = kRingBase + kConsumerWarps * kRingBytesPerWarp;
 
 struct StageView {
     double *c[6];   // x, y, z, vx, vy, vz
@@ -496,17 +351,10 @@ __device__ __forceinline__ StageView stage_view(char *smem, int s) {
     return v;
 }
 
-
-// Per-warp output buffers (TMA-out): 2 x [6 x 32 doubles | 32 ints] after the
-// stages and the barriers.
-constexpr int kOutBytes = 32 * (6 * 8 + 4);
-constexpr int kOutBase = kStages * kStageBytes + 2 * kStages * 8;
-
 // Per-warp staging ring for appends to a global list (holes, deferred
 // walks): items are buffered in shared memory and leave 32 at a time with one
 // global atomic, instead of one single-address atomic per warp-iteration
 // (those serialise in L2 when every warp appends).
-constexpr int kRing = 64;
 struct WarpRing {
     uint32_t *va;          // shared ring of values
     int32_t *vb;           // optional second value (hop counts), may be null
@@ -547,151 +395,75 @@ __device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *coun
     }
 }
 
-__device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b);
-__device__ __forceinline__ void fence_proxy_async_fwd();
-
-// Gathers of the NEXT slice issued one slice ahead by the TMA-pipelined
-// consumer (OPP_PREFETCH_NEXT): the cell field and the speculative overlay
-// entry only depend on the streamed state, so they leave the per-slice
-// dependent chain (their latency hides behind the current slice's walk).
-struct Pre {
-    long long slot;
-    int val;
-    double2 Exy;
-    double Ez;
-};
-
-// `release`: the stage mbarrier to arrive on once this warp no longer needs
-// the shared-memory copy of its particles (TMA-pipelined kernel; every lane
-// valid) -- after the push has consumed all seven loaded values, so no shared
-// load is still pending when the producer's next bulk copy overwrites it.
-template <int DEP, int DH, bool CONT, bool MULTI, bool SOUT = false>
+// LATE: the start cell's walk line is loaded after the push and the DH seed,
+// through an opaque dependency on the pushed position, so the 24 line
+// registers and the streamed particle state are never live at once (the
+// TMA-pipelined kernel: fewer registers, 3 blocks per SM); otherwise it is
+// issued together with E (one round trip; direct paths).
+template <int DEP, int DH, bool MULTI, bool LATE>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
-                                         int hops, double &x, double &y, double &z, double &vx,
+                                         double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
-                                         uint64_t *release = nullptr, double *sout = nullptr,
-                                         int sj = 0, Appends *ap = nullptr,
-                                         const Pre *pre = nullptr, int *perm = nullptr) {
+                                         Appends *ap = nullptr) {
     int status = ST_NONE;
-    int capped = 0;
+    int capped = 0, hops = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
-    int4 cn = make_int4(0, 0, 0, 0);
-    // output position: i (in place), or dest[i] on a sort-fused step
-    unsigned long long o = (!CONT && a.dest && valid) ? (unsigned long long)__ldg(a.dest + i) : i;
-    if (valid && a.dbg == 1) {   // diagnostic: stream only
-        vx = add(vx, a.c1); x = add(x, mul(vx, a.dt));
-        a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-        a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-        valid = false;
-    }
-    if (valid && a.dbg == 2) {   // diagnostic: stream + E gather
-        const double *Ep = reinterpret_cast<const double *>(a.ef + (cell - a.cell_base));
-        vx = add(vx, mul(a.c1, __ldg(Ep))); x = add(x, mul(vx, a.dt));
-        a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-        a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-        valid = false;
-    }
     if (valid) {
         const int lc = cell - a.cell_base;
-        // First visit.  Direct paths issue the walk line together with E (one
-        // round trip).  The TMA-out path issues it after the push (through an
-        // opaque dependency on the pushed x) so the 32 line registers and the
-        // particle state are never live at once: fewer registers, more warps.
         Line L;
-        if (!(SOUT && !CONT)) L = load_line(a.lines, lc);
-        if (!CONT) {
-            // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
-            // DH: the overlay entry of the drift-only position x + v dt is
-            // fetched together with E; it is used only when the pushed
-            // position lies in the same overlay cell (all but ~|c1 E dt| / dx
-            // of the particles), so the seed is exactly that of the pushed
-            // position and the lookup leaves the dependent chain.
-            long long spec_slot = -1;
-            int spec_val = -1;
-            double2 Exy;
-            double Ez;
-            if (pre) {
-                spec_slot = pre->slot;
-                spec_val = pre->val;
-                Exy = pre->Exy;
-                Ez = pre->Ez;
-            } else {
-                if (DH == 1) {
-                    spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
-                                        add(z, mul(vz, a.dt)));
-                    spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
-                }
-                load_E(a.ef, lc, Exy, Ez);
+        if (!LATE) L = load_line(a.lines, lc);
+        // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
+        // DH: the overlay entry of the drift-only position x + v dt is
+        // fetched together with E; it is used only when the pushed position
+        // lies in the same overlay cell (all but ~|c1 E dt| / dx of the
+        // particles), so the seed is exactly that of the pushed position and
+        // the lookup leaves the dependent chain.
+        long long spec_slot = -1;
+        int spec_val = -1;
+        if (DH == 1) {
+            spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
+                                add(z, mul(vz, a.dt)));
+            spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
+        }
+        double2 Exy;
+        double Ez;
+        load_E(a.ef, lc, Exy, Ez);
+        vx = add(vx, mul(a.c1, Exy.x));
+        vy = add(vy, mul(a.c1, Exy.y));
+        vz = add(vz, mul(a.c1, Ez));
+        x = add(x, mul(vx, a.dt));
+        y = add(y, mul(vy, a.dt));
+        z = add(z, mul(vz, a.dt));
+        // position and velocity are final now: store them before the walk
+        a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+        a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+        if (DH == 1) {   // seed every particle from the overlay (reading S19'' mode 1)
+            const long long g = dh_slot(a.ov, x, y, z);
+            int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
+            if (g < 0) v = -1;
+            const int sc = v >= 0 ? v : cell;
+            if (sc != cell) {
+                cell = sc;
+                if (!LATE) L = load_line(a.lines, sc - a.cell_base);
             }
-            vx = add(vx, mul(a.c1, Exy.x));
-            vy = add(vy, mul(a.c1, Exy.y));
-            vz = add(vz, mul(a.c1, Ez));
-            x = add(x, mul(vx, a.dt));
-            y = add(y, mul(vy, a.dt));
-            z = add(z, mul(vz, a.dt));
-            // position and velocity are final now: store them before the walk
-            // (TMA-out path: into the shared stage, bulk-stored by the warp)
-            if (SOUT && sout) {   // per-warp output buffer: 6 columns of 32 doubles
-                sout[sj] = x; sout[32 + sj] = y; sout[64 + sj] = z;
-                sout[96 + sj] = vx; sout[128 + sj] = vy; sout[160 + sj] = vz;
-            } else {
-                a.pos_out[o] = x; a.pos_out[a.cap + o] = y; a.pos_out[2 * a.cap + o] = z;
-                a.vel_out[o] = vx; a.vel_out[a.cap + o] = vy; a.vel_out[2 * a.cap + o] = vz;
-            }
-            if (release) {
-                fence_proxy_async_fwd();   // generic reads before the async-proxy refill
-                __syncwarp();
-                if ((threadIdx.x & 31u) == 0) mbar_arrive_fwd(release);
-            }
-            if (DH == 1) {   // seed every particle from the overlay
-                const long long g = dh_slot(a.ov, x, y, z);
-                int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
-                if (g < 0) v = -1;
-                int sc = v >= 0 ? v : cell;
+        }
+        if (LATE) {
+            int zero;
+            asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}"
+                         : "=r"(zero) : "d"(z));
+            L = load_line(a.lines, cell - a.cell_base + zero);
+        }
+        if (DH == 2) {   // mode 2: only a particle no longer inside its cell takes the seed
+            bary(L, x, y, z, l0, l1, l2, l3);
+            if (!(in01(l0) && in01(l1) && in01(l2) && in01(l3))) {
+                const int sc = dh_seed(a.ov, x, y, z, cell);
                 if (sc != cell) {
                     cell = sc;
-                    if (!SOUT) L = load_line(a.lines, sc - a.cell_base);
+                    L = load_line(a.lines, sc - a.cell_base);
                 }
             }
-            if (SOUT && DH == 1 && perm) {
-                // regroup the warp's particles by seed cell (contiguous lanes share
-                // a cell): a 256-bit load costs the L1 ~2 cycles per distinct line
-                // per 8-lane quarter, so interleaved seeds (~6 per warp) cost ~27
-                // cycles per walk-line load and grouped ones ~17.  Position, cell
-                // and output slot move; v is already stored.
-                const unsigned FULL = 0xffffffffu, ln = threadIdx.x & 31u;
-                const unsigned peers = __match_any_sync(FULL, cell);
-                const int leader = __ffs(peers) - 1;
-                const int sz = (int)ln == leader ? __popc(peers) : 0;
-                int incl = sz;
-#pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {
-                    const int tq = __shfl_up_sync(FULL, incl, d);
-                    if ((int)ln >= d) incl += tq;
-                }
-                const int dest = __shfl_sync(FULL, incl - sz, leader) + __popc(peers & ((1u << ln) - 1u));
-                perm[dest] = (int)ln;
-                __syncwarp();
-                const int src = perm[ln];
-                __syncwarp();
-                x = __shfl_sync(FULL, x, src);
-                y = __shfl_sync(FULL, y, src);
-                z = __shfl_sync(FULL, z, src);
-                cell = __shfl_sync(FULL, cell, src);
-                o = __shfl_sync(FULL, o, src);
-            }
-            if (SOUT) {
-                int zero;
-                asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}"
-                             : "=r"(zero) : "d"(z));
-                L = load_line(a.lines, cell - a.cell_base + zero);
-            }
-            if (DH == 2) dh_if_left(a, x, y, z, cell, L);
         }
-        const int stop_at = a.dbg == 3 ? 0 : (CONT ? INT_MAX : a.hpass);
-        status = walk_from<MULTI>(a, cell, L, PosRegs{x, y, z}, hops, stop_at, l0, l1, l2, l3,
-                                  capped, cn);
-        if (a.dbg == 3 && status == ST_MOVE) status = ST_DONE;
+        status = walk_from<MULTI>(a, cell, L, x, y, z, hops, a.hpass, l0, l1, l2, l3, capped);
         if (status != ST_MOVE && status != ST_MIGRATE) {   // counted where the walk ends
             t.hops += (unsigned)hops;
             t.maxh = max(t.maxh, (unsigned)hops);
@@ -699,135 +471,113 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         }
         t.removed += (status == ST_REMOVE);
     }
-    const bool done = status == ST_DONE && a.dbg == 0;
-    if (DEP == 2) {
-        sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-    } else {
-        deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
-    }
+    deposit_any<DEP>(a, status == ST_DONE, cell, l0, l1, l2, l3);
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
     if (ap) {
-        ring_push(ap->holes, rem, (uint32_t)o, 0);
+        ring_push(ap->holes, rem, (uint32_t)i, 0);
         ring_flush(ap->holes, &a.cnt->n_holes, a.holes, nullptr, false);
-        if (!CONT) {
-            ring_push(ap->work, status == ST_MOVE, (uint32_t)o, hops);
-            ring_flush(ap->work, &a.cnt->n_work, a.work, a.work_hops, false);
-        }
+        ring_push(ap->work, status == ST_MOVE, (uint32_t)i, hops);
+        ring_flush(ap->work, &a.cnt->n_work, a.work, a.work_hops, false);
     } else {
         unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
-        if (rem) a.holes[hs] = (uint32_t)o;
-        if (!CONT) {
-            const bool mv = status == ST_MOVE;
-            unsigned long long ws = warp_append(mv, &a.cnt->n_work);
-            if (mv) {
-                a.work[ws] = (uint32_t)o;
-                a.work_hops[ws] = hops;
-            }
+        if (rem) a.holes[hs] = (uint32_t)i;
+        const bool mv = status == ST_MOVE;
+        unsigned long long ws = warp_append(mv, &a.cnt->n_work);
+        if (mv) {
+            a.work[ws] = (uint32_t)i;
+            a.work_hops[ws] = hops;
         }
     }
     if (MULTI) {
         const bool mg = status == ST_MIGRATE;
         unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
         if (mg) {
-            a.mig[ms] = (uint32_t)o;
+            a.mig[ms] = (uint32_t)i;
             a.mig_cell[ms] = cell;
             a.mig_hops[ms] = hops;
         }
     }
     if (rem) cell = -1;
-    if (perm) a.p2c_out[o] = cell;   // regrouped lanes store their own particle's cell
 }
 
 // ---------------------------------------------------------------------------
 // Direct-load variant: warps stride over [lo, hi) one particle per lane; the
 // next particle's state is loaded before the current one walks (a register
 // double buffer), so the HBM stream stays in flight during the latency-bound
-// walk.  Used for the continuation pass, the ragged tail of the tiled
-// kernel, and as the non-TMA variant of pass 1.
+// walk.  Used for the ragged tail of the tiled kernel and as the non-TMA
+// variant of pass 1 (opp_init_params.tma_pipeline = 0).
 // ---------------------------------------------------------------------------
 struct PState {
     double x, y, z, vx, vy, vz;
-    int cell, hops;
+    int cell;
     unsigned long long i;
     bool valid;
 };
 
-template <bool CONT>
 __device__ __forceinline__ void load_pstate(const StepArgs &a, unsigned long long k,
                                             unsigned long long hi, PState &p) {
     p.valid = k < hi;
     p.i = k;
-    p.hops = 0;
     p.cell = 0;
     p.x = p.y = p.z = p.vx = p.vy = p.vz = 0.0;
     if (p.valid) {
-        if (CONT) {
-            p.i = a.work[k];
-            p.hops = a.work_hops[k];
-        }
-        p.x = a.pos[p.i]; p.y = a.pos[a.cap + p.i]; p.z = a.pos[2 * a.cap + p.i];
-        if (!CONT) { p.vx = a.vel[p.i]; p.vy = a.vel[a.cap + p.i]; p.vz = a.vel[2 * a.cap + p.i]; }
-        p.cell = a.p2c[p.i];
+        p.x = a.pos[k]; p.y = a.pos[a.cap + k]; p.z = a.pos[2 * a.cap + k];
+        p.vx = a.vel[k]; p.vy = a.vel[a.cap + k]; p.vz = a.vel[2 * a.cap + k];
+        p.cell = a.p2c[k];
     }
 }
 
-template <int DEP, int DH, bool CONT, bool MULTI>
+template <int DEP, int DH, bool MULTI>
 __device__ __forceinline__ void pmd_direct_range(const StepArgs &a, unsigned long long lo,
                                                  unsigned long long hi, unsigned long long first,
                                                  unsigned long long stride, Tally &t) {
     unsigned long long i0 = lo + first;
     if (i0 >= hi) return;
     PState cur;
-    load_pstate<CONT>(a, i0 + lane_id(), hi, cur);
+    load_pstate(a, i0 + lane_id(), hi, cur);
     for (; i0 < hi; i0 += stride) {
         PState nxt;
         const bool more = i0 + stride < hi;
-        if (more) load_pstate<CONT>(a, i0 + stride + lane_id(), hi, nxt);
-        pmd_body<DEP, DH, CONT, MULTI>(a, cur.valid, cur.i, cur.hops, cur.x, cur.y, cur.z, cur.vx,
-                                       cur.vy, cur.vz, cur.cell, t);
-        if (cur.valid) a.p2c_out[(!CONT && a.dest) ? (unsigned long long)__ldg(a.dest + cur.i) : cur.i] = cur.cell;
+        if (more) load_pstate(a, i0 + stride + lane_id(), hi, nxt);
+        pmd_body<DEP, DH, MULTI, false>(a, cur.valid, cur.i, cur.x, cur.y, cur.z, cur.vx, cur.vy,
+                                        cur.vz, cur.cell, t);
+        if (cur.valid) a.p2c[cur.i] = cur.cell;
         if (more) cur = nxt;
     }
 }
 
-// Pass 1 (direct variant): every block owns one contiguous chunk of the
-// particle array, so in cell-sorted storage the walk lines a block touches
-// stay hot in its SM's L1.  Continuation: grid-stride over the worklist.
-template <int DEP, int DH, bool CONT, bool MULTI>
+// Pass 1 (direct variant): blocks visit groups of consecutive 256-particle
+// tiles, so in cell-sorted storage the walk lines a block touches stay hot in
+// its SM's L1.
+template <int DEP, int DH, bool MULTI>
 __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
     Tally t;
-    if (CONT) {
-        const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n_work;
-        pmd_direct_range<DEP, DH, true, MULTI>(
-            a, 0, n, (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u),
-            (unsigned long long)gridDim.x * blockDim.x, t);
-    } else {
-        const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
-        const TileMap tm{(n + 255) / 256, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
-        const unsigned long long my = tm.count();
-        TileIter ti(tm);
-        for (unsigned long long it = 0; it < my; it++, ti.next()) {
-            const unsigned long long lo = ti.tile() * 256;
-            pmd_direct_range<DEP, DH, false, MULTI>(a, lo, lo + 256 < n ? lo + 256 : n,
-                                                    threadIdx.x & ~31u, 256, t);
-        }
+    const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
+    const TileMap tm{(n + 255) / 256, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
+    const unsigned long long my = tm.count();
+    TileIter ti(tm);
+    for (unsigned long long it = 0; it < my; it++, ti.next()) {
+        const unsigned long long lo = ti.tile() * 256;
+        pmd_direct_range<DEP, DH, MULTI>(a, lo, lo + 256 < n ? lo + 256 : n, threadIdx.x & ~31u, 256, t);
     }
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
 // ---------------------------------------------------------------------------
 // The fused push / move / deposit kernel, TMA-pipelined (CalcPosVel + Move +
-// DepositCharge of PAPER.md:1586-1604 in one pass).  Each block owns a
-// contiguous range of kTile-particle tiles (L1 locality of the walk lines in
-// cell-sorted storage).  A producer warp streams each tile's 7 SoA column
-// segments global -> shared with cp.async.bulk (complete_tx on the stage's
-// `full` mbarrier) up to kStages tiles ahead; each of the 8 consumer warps
-// copies its 32 particles out of the stage, releases it (`empty` mbarrier,
-// one arrival per warp) and then pushes / walks / deposits, storing results
-// with coalesced stores.  No block-wide barrier inside the loop: a warp whose
-// lanes walk far never stalls the others.  The ragged tail (< kTile) takes
-// the direct path.
+// DepositCharge of PAPER.md:1586-1604 in one pass).  Blocks visit groups of
+// a.tile_group consecutive kTile-particle tiles round-robin (L1 locality of
+// the walk lines in cell-sorted storage).  A producer warp streams each
+// tile's 7 SoA column segments global -> shared with cp.async.bulk
+// (complete_tx on the stage's `full` mbarrier) up to kStages tiles ahead;
+// each of the 8 consumer warps copies its 32 particles out of the stage,
+// releases it (`empty` mbarrier, one arrival per warp) and then pushes /
+// walks / deposits, storing results with coalesced per-lane stores (staging
+// the stores in shared memory cost the L1 data pipe twice: C2 pmd 1.99 vs
+// 2.06 ms).  No block-wide barrier inside the loop: a warp whose lanes walk
+// far never stalls the others.  The ragged tail (< kTile) is a separate
+// launch (k_push_move_deposit_tail).
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -855,21 +605,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
             : "=r"(done) : "r"(smem_u32(b)), "r"(parity), "r"(1000000u) : "memory");
     } while (!done);
 }
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t *b, uint32_t parity) { mbar_wait(b, parity); }
-__device__ __forceinline__ void mbar_arrive_fwd(uint64_t *b) { mbar_arrive(b); }
-__device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
-    uint32_t done;
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(done) : "r"(smem_u32(b)), "r"(parity) : "memory");
-    return done != 0;
-}
-__device__ __forceinline__ void prefetch_l1(const void *p) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
-}
-__device__ __forceinline__ void fence_proxy_async_fwd() {
+__device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
@@ -877,22 +613,6 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
         ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
-__device__ __forceinline__ void fence_proxy_async() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
-                 ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_read0() {
-    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait_read1() {
-    asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-
 
 // producer: load tile `tile` into stage s
 __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, uint64_t *full,
@@ -907,53 +627,14 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
-// Producer-warp L1 warming for tile p (already issued; waits until landed).
-__device__ __forceinline__ void warm_tile(const StepArgs &a, char *smem, uint64_t *full,
-                                          unsigned long long p, unsigned lane) {
-    const int sp = (int)(p % kStages);
-    mbar_wait(&full[sp], (uint32_t)((p / kStages) & 1ull));
-    const int *cells = stage_view(smem, sp).cell + lane * (kTile / 32);
-    int prev = INT_MIN;
-    int4 cc[kTile / 32];
-    int lcs[kTile / 32];
-    int nd = 0;
-#pragma unroll
-    for (int k = 0; k < kTile / 32; k++) {
-        const int lc = cells[k] - a.cell_base;
-        if (lc == prev || (unsigned)lc >= (unsigned)a.n_cells) continue;
-        prev = lc;
-        lcs[nd] = lc;
-        cc[nd] = __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(a.lines + lc) + 12));
-        prefetch_l1(a.ef + lc);
-        nd++;
-    }
-    for (int k = 0; k < nd; k++) {
-        const int nb[4] = {cc[k].x, cc[k].y, cc[k].z, cc[k].w};
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            const int ln = nb[q] - a.cell_base;
-            if (nb[q] >= 0 && (unsigned)ln < (unsigned)a.n_cells) prefetch_l1(a.lines + ln);
-        }
-        (void)lcs;
-    }
-}
-
-#ifndef OPP_PRE
-#define OPP_PRE 0   // 1: issue the next slice's E / overlay gathers one slice ahead
-                    // (C2: pmd 1.98 vs 1.94 ms -- the extra stage reads cost more L1
-                    // data-pipe wavefronts than the hidden latency saves)
-#endif
-template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
-__global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled(StepArgs a) {
-    constexpr bool PRE = OPP_PRE != 0;
-    constexpr bool TMA_OUT = OPP_TMA_OUT != 0;
+template <int DEP, int DH, bool MULTI>
+__global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
     uint64_t *empty = full + kStages;
     const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
     const unsigned long long ntiles = n / kTile;
-    const unsigned long long G = gridDim.x;
-    const TileMap tm{ntiles, G, (unsigned long long)a.tile_group, blockIdx.x};
+    const TileMap tm{ntiles, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
     const unsigned long long my = tm.count();
     const int warp = threadIdx.x >> 5;
     const unsigned lane = lane_id();
@@ -966,271 +647,56 @@ __global__ void __launch_bounds__(kTiledThreads, MINB) k_push_move_deposit_tiled
     }
     __syncthreads();
     if (warp == kConsumerWarps) {
-        // producer warp: lane 0 streams tiles kStages ahead of the slowest
-        // consumer; then the whole warp warms the SM's L1 for the tile that
-        // landed before: the walk lines and fields of its (few, cell-sorted)
-        // start cells and the lines of their four face neighbours -- the
-        // cells the consumers' first visit and first hop will touch.
-        TileIter ti(tm);
-        for (unsigned long long it = 0; it < my; it++, ti.next()) {
-            const int s = (int)(it % kStages);
-            if (lane == 0) {
-                if (it >= kStages) mbar_wait_sleep(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
+        // producer warp: lane 0 streams tiles kStages ahead of the slowest consumer
+        if (lane == 0) {
+            TileIter ti(tm);
+            for (unsigned long long it = 0; it < my; it++, ti.next()) {
+                const int s = (int)(it % kStages);
+                if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
                 issue_tile_load(a, smem, full, s, ti.tile());
             }
-            __syncwarp();
-            if (a.prefetch && it >= 1) warm_tile(a, smem, full, it - 1, lane);
         }
-        if (a.prefetch && my >= 1) warm_tile(a, smem, full, my - 1, lane);
         return;
     }
+    // Consumer warp, warp-synchronous: one 32-particle slice per tile.  The
+    // warp copies its slice to registers, forces the shared loads to land,
+    // fences the generic proxy against the producer's next bulk copy and
+    // releases the stage at once.
     Tally t;
-    if (!REFILL) {
-        // Consumer warp, warp-synchronous: one 32-particle slice per tile;
-        // the slice is copied to registers and the stage released at once.
-        // Input: the warp copies its slice to registers, forces the shared
-        // loads to complete, fences the generic proxy against the producer's
-        // next bulk copy and releases the stage at once.  Output: results go
-        // to a per-warp double buffer in shared memory and leave with
-        // cp.async.bulk shared -> global (256-B / 128-B segments per column),
-        // so the LSU pipe carries no particle stores.
-        Appends ap;
-        {
-            char *rb = smem + kRingBase + (size_t)warp * kRingBytesPerWarp;
-            ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
-            ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
-                               reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
-        }
-        TileIter ti(tm);
-        Pre cur{-1, -1, make_double2(0.0, 0.0), 0.0};
-        bool have_cur = false;
-        for (unsigned long long it = 0; it < my; it++, ti.next()) {
-            const int s = (int)(it % kStages);
-            const int ob_i = 0;   // one output buffer per warp (keeps 3 blocks / SM in smem)
-            mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
-            StageView v = stage_view(smem, s);
-            const int j = threadIdx.x;
-            double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
-            double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
-            int cell = v.cell[j];
-            Pre nxt;
-            bool have_nxt = false;
-            if (PRE && it + 1 < my) {
-                const int s1 = (int)((it + 1) % kStages);
-                const bool landed = __all_sync(0xffffffffu,
-                                               mbar_test(&full[s1], (uint32_t)(((it + 1) / kStages) & 1ull)));
-                if (landed) {
-                    StageView v1 = stage_view(smem, s1);
-                    const double x1 = v1.c[0][j], y1 = v1.c[1][j], z1 = v1.c[2][j];
-                    const double vx1 = v1.c[3][j], vy1 = v1.c[4][j], vz1 = v1.c[5][j];
-                    const int c1 = v1.cell[j];
-                    nxt.slot = -1;
-                    nxt.val = -1;
-                    if (DH == 1) {
-                        nxt.slot = dh_slot(a.ov, add(x1, mul(vx1, a.dt)), add(y1, mul(vy1, a.dt)),
-                                           add(z1, mul(vz1, a.dt)));
-                        nxt.val = ov_value(a.ov, nxt.slot >= 0 ? nxt.slot : 0);
-                    }
-                    load_E(a.ef, c1 - a.cell_base, nxt.Exy, nxt.Ez);
-                    have_nxt = true;
-                }
-            }
-            const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
-                                         (unsigned long long)__double_as_longlong(y) ^
-                                         (unsigned long long)__double_as_longlong(z) ^
-                                         (unsigned long long)__double_as_longlong(vx) ^
-                                         (unsigned long long)__double_as_longlong(vy) ^
-                                         (unsigned long long)__double_as_longlong(vz) ^
-                                         (unsigned long long)(unsigned)cell;
-            asm volatile("" ::"l"(h));   // the shared loads have landed
-            fence_proxy_async();
-            __syncwarp();
-            if (lane == 0) {
-                mbar_arrive(&empty[s]);
-                if (it >= 1) bulk_wait_read0();   // the previous stores have read the buffer
-            }
-            __syncwarp();
-            const unsigned long long tile = ti.tile();
-            const unsigned long long i = tile * kTile + j;
-            double *o = reinterpret_cast<double *>(smem + kOutBase +
-                                                   (size_t)(warp + ob_i) * kOutBytes);
-            // results leave through the shared buffer + bulk stores (TMA_OUT),
-            // or (sort-fused step / OPP_TMA_OUT=0) as coalesced per-lane stores
-            double *obuf = (TMA_OUT && !a.dest) ? o : nullptr;
-            int *perm = (OPP_SEED_PERM && DH == 1 && !obuf)
-                             ? reinterpret_cast<int *>(smem + kRingBase + (size_t)warp * kRingBytesPerWarp + 64 * 12)
-                             : nullptr;
-            pmd_body<DEP, DH, false, MULTI, true>(a, true, i, 0, x, y, z, vx, vy, vz, cell, t,
-                                                  nullptr, obuf, (int)lane, &ap,
-                                                  (PRE && have_cur) ? &cur : nullptr, perm);
-            if (PRE) {
-                cur = nxt;
-                have_cur = have_nxt;
-            }
-            if (!obuf) {
-                if (!perm) a.p2c_out[a.dest ? (unsigned long long)__ldg(a.dest + i) : i] = cell;
-                continue;
-            }
-            reinterpret_cast<int *>(o + 192)[lane] = cell;
-            fence_proxy_async();
-            __syncwarp();
-            if (lane == 0) {
-                const unsigned long long g0 = tile * kTile + warp * 32;
-                for (int k = 0; k < 3; k++) {
-                    bulk_s2g(a.pos + k * a.cap + g0, o + 32 * k, 256);
-                    bulk_s2g(a.vel + k * a.cap + g0, o + 32 * (3 + k), 256);
-                }
-                bulk_s2g(a.p2c + g0, o + 192, 128);
-                bulk_commit();
-            }
-        }
-        ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
-        ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
-        if (lane == 0) bulk_wait_all();
-        // the ragged tail (< kTile particles) is done by k_push_move_deposit_tail
-        flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
-        return;
+    Appends ap;
+    {
+        char *rb = smem + kRingBase + (size_t)warp * kRingBytesPerWarp;
+        ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
+        ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
+                           reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
     }
-    // Consumer warp with per-lane refill: its particle stream is its 32-slot slice of every tile.
-    // Lanes are refilled independently: whenever a lane's particle finishes
-    // (DONE / REMOVE / deferred / migrating) it takes the next stream entry,
-    // so every iteration advances 32 walks by one cell visit instead of
-    // waiting for the warp's longest walk.
-    const unsigned long long total = 32ull * my;
-    unsigned long long pos = 0;
-    long long waited = -1;
-    bool active = false;
-    double x = 0, y = 0, z = 0;
-    int cell = 0, hops = 0;
-    unsigned long long i = 0;
-    Line L;
-    const unsigned lt_mask = (1u << lane) - 1u;
-    for (;;) {
-        // ---- refill idle lanes from the stream
-        const unsigned need = __ballot_sync(0xffffffffu, !active);
-        if (need && pos < total) {
-            const unsigned long long avail = total - pos;
-            const int k = (int)min((unsigned long long)__popc(need), avail);
-            const int r = __popc(need & lt_mask);
-            const bool take = !active && r < k;
-            const long long last_tile = (long long)((pos + k - 1) / 32);
-            if (last_tile > waited) {
-                mbar_wait(&full[last_tile % kStages], (uint32_t)((last_tile / kStages) & 1));
-                waited = last_tile;
-            }
-            double vx = 0, vy = 0, vz = 0;
-            if (take) {
-                const unsigned long long p = pos + r, it = p / 32;
-                const int j = warp * 32 + (int)(p % 32);
-                StageView v = stage_view(smem, (int)(it % kStages));
-                x = v.c[0][j]; y = v.c[1][j]; z = v.c[2][j];
-                vx = v.c[3][j]; vy = v.c[4][j]; vz = v.c[5][j];
-                cell = v.cell[j];
-                i = tm.tile(it) * kTile + j;
-                hops = 0;
-            }
-            const unsigned long long pos0 = pos, npos = pos + k;
-            pos = npos;
-            if (take) {
-                const int lc = cell - a.cell_base;
-                L = load_line(a.lines, lc);
-                double2 Exy;
-                double Ez;
-                load_E(a.ef, lc, Exy, Ez);
-                vx = add(vx, mul(a.c1, Exy.x));
-                vy = add(vy, mul(a.c1, Exy.y));
-                vz = add(vz, mul(a.c1, Ez));
-                x = add(x, mul(vx, a.dt));
-                y = add(y, mul(vy, a.dt));
-                z = add(z, mul(vz, a.dt));
-                a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-                a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-                if (DH == 1) {
-                    const int sc = dh_seed(a.ov, x, y, z, cell);
-                    if (sc != cell) {
-                        cell = sc;
-                        L = load_line(a.lines, sc - a.cell_base);
-                    }
-                }
-                if (DH == 2) dh_if_left(a, x, y, z, cell, L);
-                active = true;
-            }
-            // the push has consumed the shared copies: release fully read slices
-            fence_proxy_async();
-            __syncwarp();
-            if (lane == 0)
-                for (unsigned long long tt = pos0 / 32; tt < npos / 32; tt++)
-                    mbar_arrive(&empty[tt % kStages]);
-        }
-        if (!__any_sync(0xffffffffu, active)) break;
-        // ---- one cell visit per active lane
-        int status = ST_NONE;
-        int capped = 0;
-        double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
-        int4 cn = make_int4(0, 0, 0, 0);
-        if (active) {
-            bary(L, x, y, z, l0, l1, l2, l3);
-            cn = L.cn;
-            if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
-                status = ST_DONE;
-            } else if (hops >= a.hcap) {
-                status = ST_DONE;
-                capped = 1;
-            } else if (hops >= a.hpass) {
-                status = ST_MOVE;
-            } else {
-                const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
-                int nb = cc.x;
-                double m = l0;
-                if (l1 < m) { m = l1; nb = cc.y; }
-                if (l2 < m) { m = l2; nb = cc.z; }
-                if (l3 < m) { nb = cc.w; }
-                if (nb < 0) {
-                    status = ST_REMOVE;
-                } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
-                    cell = nb;
-                    hops++;
-                    status = ST_MIGRATE;
-                } else {
-                    cell = nb;
-                    hops++;
-                    L = load_line(a.lines, nb - a.cell_base);
-                }
-            }
-        }
-        const bool fin = status != ST_NONE;
-        if (fin && status != ST_MOVE && status != ST_MIGRATE) {
-            t.hops += (unsigned)hops;
-            t.maxh = max(t.maxh, (unsigned)hops);
-            t.capped += (unsigned)capped;
-        }
-        t.removed += (status == ST_REMOVE);
-        const bool done = status == ST_DONE;
-        if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-        else deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
-        const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
-        unsigned long long hs = warp_append(rem, &a.cnt->n_holes);
-        if (rem) a.holes[hs] = (uint32_t)i;
-        const bool mv = status == ST_MOVE;
-        unsigned long long ws = warp_append(mv, &a.cnt->n_work);
-        if (mv) {
-            a.work[ws] = (uint32_t)i;
-            a.work_hops[ws] = hops;
-        }
-        if (MULTI) {
-            const bool mg = status == ST_MIGRATE;
-            unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
-            if (mg) {
-                a.mig[ms] = (uint32_t)i;
-                a.mig_cell[ms] = cell;
-                a.mig_hops[ms] = hops;
-            }
-        }
-        if (fin) {
-            a.p2c[i] = rem ? -1 : cell;
-            active = false;
-        }
+    TileIter ti(tm);
+    for (unsigned long long it = 0; it < my; it++, ti.next()) {
+        const int s = (int)(it % kStages);
+        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
+        StageView v = stage_view(smem, s);
+        const int j = threadIdx.x;
+        double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
+        double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
+        int cell = v.cell[j];
+        const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
+                                     (unsigned long long)__double_as_longlong(y) ^
+                                     (unsigned long long)__double_as_longlong(z) ^
+                                     (unsigned long long)__double_as_longlong(vx) ^
+                                     (unsigned long long)__double_as_longlong(vy) ^
+                                     (unsigned long long)__double_as_longlong(vz) ^
+                                     (unsigned long long)(unsigned)cell;
+        asm volatile("" ::"l"(h));   // the shared loads have landed
+        fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[s]);
+        __syncwarp();
+        const unsigned long long i = ti.tile() * kTile + j;
+        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap);
+        a.p2c[i] = cell;
     }
+    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
+    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
@@ -1242,18 +708,17 @@ __global__ void __launch_bounds__(256) k_push_move_deposit_tail(StepArgs a) {
     const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
     const unsigned long long lo = n / kTile * kTile;
     Tally t;
-    pmd_direct_range<DEP, DH, false, MULTI>(a, lo, n, threadIdx.x & ~31u, 256, t);
+    pmd_direct_range<DEP, DH, MULTI>(a, lo, n, threadIdx.x & ~31u, 256, t);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
 // ---------------------------------------------------------------------------
 // Continuation walk with per-lane refill: finishes the deferred walks (and
 // received migrants).  Each lane carries one particle and advances it by one
-// cell visit per iteration; a lane whose particle finished claims the next
-// worklist entry (the warp leader claims a batch with one atomic), so every
-// iteration keeps ~32 walks in flight instead of waiting for the longest walk
-// of the warp.  Small register footprint -> many resident warps to hide the
-// L2 latency of the line gathers.
+// cell visit per iteration; a lane whose particle finished takes the next
+// worklist entry, so every iteration keeps ~32 walks in flight instead of
+// waiting for the longest walk of the warp.  Small register footprint -> many
+// resident warps to hide the L2 latency of the line gathers.
 // ---------------------------------------------------------------------------
 template <int DEP, bool MULTI>
 __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
@@ -1317,22 +782,15 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
         if (!__any_sync(0xffffffffu, active)) break;
         int status = ST_NONE, capped = 0;
         double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
-        int4 cn = make_int4(0, 0, 0, 0);
         if (active) {
             bary(L, x, y, z, l0, l1, l2, l3);
-            cn = L.cn;
             if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
                 status = ST_DONE;
             } else if (hops >= a.hcap) {
                 status = ST_DONE;
                 capped = 1;
             } else {
-                const int4 cc = cc_of(a.lines, L, cell - a.cell_base);
-                int nb = cc.x;
-                double m = l0;
-                if (l1 < m) { m = l1; nb = cc.y; }
-                if (l2 < m) { m = l2; nb = cc.z; }
-                if (l3 < m) { nb = cc.w; }
+                const int nb = pick(line_c2c(a.lines, cell - a.cell_base), argmin_face(l0, l1, l2, l3));
                 if (nb < 0) {
                     status = ST_REMOVE;
                 } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
@@ -1353,9 +811,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
             t.capped += (unsigned)capped;
         }
         t.removed += (status == ST_REMOVE);
-        const bool done = status == ST_DONE;
-        if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
-        else deposit<DEP>(a.Q, CnSrc{a.lines, a.cell_base}, done, cell, cn, a.w, l0, l1, l2, l3);
+        deposit_any<DEP>(a, status == ST_DONE, cell, l0, l1, l2, l3);
         const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
         ring_push(hr, rem, (uint32_t)i, 0);
         ring_flush(hr, &a.cnt->n_holes, a.holes, nullptr, false);
@@ -1770,10 +1226,9 @@ __global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *
 }
 
 // Phase 1: destination slot of every particle (run heads take one atomic
-// per run of equal cells); holes get 0xffffffff.
+// per run of equal cells), recorded as the inverse permutation src_of.
 __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
-                            const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *dest,
-                            uint32_t *src_of) {
+                            const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *src_of) {
     const unsigned long long n = c->n;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
@@ -1789,22 +1244,23 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
         if (head && cell >= 0)
             base = atomicAdd(cursor + bucket_of(skey, cell - cell_base), (unsigned)rl);
         base = __shfl_sync(0xffffffffu, base, rs);
-        if (cell >= 0) {
-            src_of[base + (lane_id() - rs)] = (uint32_t)i;   // inverse permutation
-            if (dest) dest[i] = base + (lane_id() - rs);      // forward (sort fused into the move)
-        }
+        if (cell >= 0) src_of[base + (lane_id() - rs)] = (uint32_t)i;
     }
 }
 
-// Phase 2: gather move dst[d] = src[src_of[d]] for d in [0, total): the
-// writes stream in order (full sectors, no read-modify-write of partially
-// written sectors), the reads of nearly sorted data hit sectors that their
-// neighbours in d fetched a moment ago.
+// Phase 2, one column per launch: gather move dst[d] = src[src_of[d]] for d
+// in [0, total): the writes stream in order (full sectors, no
+// read-modify-write of partially written sectors), the reads of nearly
+// sorted data hit sectors that their neighbours in d fetched a moment ago.
+// dst is a spare buffer of the column's size that then becomes the column
+// (its old storage becomes the spare), so a sort needs one spare per column
+// size, not a second copy of every column.
 constexpr int kSortUnroll = 4;
-__global__ void __launch_bounds__(256) k_sort_gather(ColSet src, ColSet dst,
+template <typename T>
+__global__ void __launch_bounds__(256) k_sort_gather(const T *__restrict__ src, T *__restrict__ dst,
+                                                     int dim, long long cap,
                                                      const uint32_t *__restrict__ src_of,
-                                                     const unsigned *__restrict__ total_p,
-                                                     int u0, int u1) {
+                                                     const unsigned *__restrict__ total_p) {
     const unsigned long long n = *total_p;
     const unsigned long long span = (unsigned long long)blockDim.x * kSortUnroll;
     for (unsigned long long b = (unsigned long long)blockIdx.x * span; b < n;
@@ -1816,52 +1272,14 @@ __global__ void __launch_bounds__(256) k_sort_gather(ColSet src, ColSet dst,
             dd[u] = b + (unsigned long long)u * blockDim.x + threadIdx.x;
             ss[u] = dd[u] < n ? __ldg(src_of + dd[u]) : 0u;
         }
-        int u = 0;   // flattened (column, component) index; this launch moves [u0, u1)
-        for (int j = 0; j < src.n; j++) {
-            const ColDesc cs = src.c[j], cd = dst.c[j];
-            for (int e = 0; e < cs.dim; e++, u++) {
-                if (u < u0 || u >= u1) continue;
-                if (cs.elem_bytes == 8) {
-                    const long long *sp = reinterpret_cast<const long long *>(cs.ptr) + e * cs.cap;
-                    long long *dp = reinterpret_cast<long long *>(cd.ptr) + e * cd.cap;
-                    long long v[kSortUnroll];
+        for (int e = 0; e < dim; e++) {
+            const T *sp = src + e * cap;
+            T *dp = dst + e * cap;
+            T v[kSortUnroll];
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : 0;
+            for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : T(0);
 #pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
-                } else {
-                    const int *sp = reinterpret_cast<const int *>(cs.ptr) + e * cs.cap;
-                    int *dp = reinterpret_cast<int *>(cd.ptr) + e * cd.cap;
-                    int v[kSortUnroll];
-#pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : 0;
-#pragma unroll
-                    for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
-                }
-            }
-        }
-    }
-}
-
-// Sort-fused step: the columns the move does not write (ids, user dats)
-// follow their particles, dst[dest[i]] = src[i] for i < n.
-__global__ void __launch_bounds__(256) k_scatter_cols(ColSet src, ColSet dst,
-                                                      const uint32_t *__restrict__ dest,
-                                                      const DevCounters *c) {
-    const unsigned long long n = c->n;
-    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-         i += (unsigned long long)gridDim.x * blockDim.x) {
-        const unsigned long long d = __ldg(dest + i);
-        for (int j = 0; j < src.n; j++) {
-            const ColDesc cs = src.c[j], cd = dst.c[j];
-            for (int e = 0; e < cs.dim; e++) {
-                if (cs.elem_bytes == 8)
-                    reinterpret_cast<long long *>(cd.ptr)[e * cd.cap + d] =
-                        __ldg(reinterpret_cast<const long long *>(cs.ptr) + e * cs.cap + i);
-                else
-                    reinterpret_cast<int *>(cd.ptr)[e * cd.cap + d] =
-                        __ldg(reinterpret_cast<const int *>(cs.ptr) + e * cs.cap + i);
-            }
+            for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
         }
     }
 }
@@ -2040,91 +1458,54 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
 }
 
 cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
-                             unsigned *start, uint32_t *dest, uint32_t *src_of, int rank_grid,
-                             cudaStream_t s) {
-    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, dest, src_of);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_scatter_cols(const ColSet &src, const ColSet &dst, const uint32_t *dest,
-                                const DevCounters *c, int grid, cudaStream_t s) {
-    if (src.n == 0) return cudaSuccess;
-    k_scatter_cols<<<grid, 256, 0, s>>>(src, dst, dest, c);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
-                             DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
-                             unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
-                             int rank_grid, cudaStream_t s) {
+                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s) {
     // the scan left the total in start[nc]; the rank pass consumes start[] as
     // cursors but never touches start[nc].  One thread per particle: every
     // warp waits on its cursor atomics once, so the round trips overlap.
-    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, nullptr, src_of);
-    // column passes: each pass moves a group of components so that the
-    // source window it re-reads stays resident in L2 (OPP_SORT_PASSES)
-    int nu = 0;
-    for (int j = 0; j < src.n; j++) nu += src.c[j].dim;
-    // defaults measured on C2 (sort_move 0.36 -> 0.315 ms/step at sort_every 5):
-    // two passes, 4 blocks per SM
-    static const int passes = [] {
-        const char *e = getenv("OPP_SORT_PASSES");
-        return e ? atoi(e) : 2;
-    }();
-    static const int gmul = [] {
-        const char *e = getenv("OPP_SORT_GRID");
-        return e ? atoi(e) : 4;
-    }();
-    if (gmul > 0) {
-        int dev = 0, nsm = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-        grid = nsm * gmul;
-    }
-    const int np = passes < 1 ? 1 : (passes > nu ? nu : passes);
-    for (int q = 0; q < np; q++)
-        k_sort_gather<<<grid, 256, 0, s>>>(src, dst, src_of, start + nc, q * nu / np,
-                                           (q + 1) * nu / np);
-    k_sort_commit<<<1, 1, 0, s>>>(c, start + nc);
+    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, src_of);
     return cudaGetLastError();
 }
 
-template <int DEP, int DH, bool MULTI, bool REFILL, int MINB>
-static cudaError_t launch_tiled_b(const StepArgs &a, int grid, cudaStream_t s) {
+cudaError_t launch_sort_gather(const ColDesc &src, char *dst, const uint32_t *src_of,
+                               const unsigned *total_p, int grid, cudaStream_t s) {
+    if (src.elem_bytes == 8)
+        k_sort_gather<long long><<<grid, 256, 0, s>>>(reinterpret_cast<const long long *>(src.ptr),
+                                                      reinterpret_cast<long long *>(dst), src.dim,
+                                                      src.cap, src_of, total_p);
+    else
+        k_sort_gather<int><<<grid, 256, 0, s>>>(reinterpret_cast<const int *>(src.ptr),
+                                                reinterpret_cast<int *>(dst), src.dim, src.cap,
+                                                src_of, total_p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sort_commit(DevCounters *c, const unsigned *start_total, cudaStream_t s) {
+    k_sort_commit<<<1, 1, 0, s>>>(c, start_total);
+    return cudaGetLastError();
+}
+
+template <int DEP, int DH, bool MULTI>
+static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB>,
+        cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
         if (e != cudaSuccess) return e;
-        // shared-memory carveout (percent of the unified L1/shared array);
-        // what the stages do not take is L1 for the walk lines (OPP_CARVEOUT)
-        if (const char *cv = getenv("OPP_CARVEOUT")) {
-            e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB>,
-                                     cudaFuncAttributePreferredSharedMemoryCarveout, atoi(cv));
-            if (e != cudaSuccess) return e;
-        }
         attr = true;
     }
-    k_push_move_deposit_tiled<DEP, DH, MULTI, REFILL, MINB><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+    k_push_move_deposit_tiled<DEP, DH, MULTI><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
     k_push_move_deposit_tail<DEP, DH, MULTI><<<1, 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 
-template <int DEP, int DH, bool MULTI, bool REFILL>
-static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
-    return a.minb >= 3 ? launch_tiled_b<DEP, DH, MULTI, REFILL, OPP_MINB_HI>(a, grid, s)
-                       : launch_tiled_b<DEP, DH, MULTI, REFILL, 1>(a, grid, s);
-}
-
 template <int DEP, int DH, bool CONT, bool MULTI>
 static cudaError_t launch_pmd_t(const StepArgs &a, int grid, bool tiled, cudaStream_t s) {
-    if (!CONT && tiled) {
-        return a.refill ? launch_tiled<DEP, DH, MULTI, true>(a, grid, s)
-                        : launch_tiled<DEP, DH, MULTI, false>(a, grid, s);
-    } else if (CONT) {
+    if (CONT) {
         k_walk_refill<DEP, MULTI><<<grid, 256, 0, s>>>(a);
+    } else if (tiled) {
+        return launch_tiled<DEP, DH, MULTI>(a, grid, s);
     } else {
-        k_push_move_deposit<DEP, DH, CONT, MULTI><<<grid, 256, 0, s>>>(a);
+        k_push_move_deposit<DEP, DH, MULTI><<<grid, 256, 0, s>>>(a);
     }
     return cudaGetLastError();
 }
@@ -2154,24 +1535,16 @@ cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, boo
                 : launch_pmd_c<false>(dep, dh, multi, a, grid, tiled, s);
 }
 
-int pmd_blocks_per_sm(bool tiled, int minb) {
+int pmd_blocks_per_sm(bool tiled) {
     int nb = 0;
     cudaError_t e;
     if (tiled) {
-        if (minb >= 3) {
-            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &nb, k_push_move_deposit_tiled<0, 0, false, false, OPP_MINB_HI>, kTiledThreads, kTiledSmem);
-        } else {
-            cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false, false, 1>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &nb, k_push_move_deposit_tiled<0, 0, false, false, 1>, kTiledThreads, kTiledSmem);
-        }
-    } else {
+        cudaFuncSetAttribute(k_push_move_deposit_tiled<0, 0, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &nb, k_push_move_deposit<0, 0, false, false>, 256, 0);
+            &nb, k_push_move_deposit_tiled<0, 0, false>, kTiledThreads, kTiledSmem);
+    } else {
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_push_move_deposit<0, 0, false>, 256, 0);
     }
     return (e == cudaSuccess && nb > 0) ? nb : 1;
 }
@@ -2313,6 +1686,22 @@ cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *h
     int gc = (int)((nc + 255) / 256), gn = (int)((nn + 255) / 256);
     k_sr_cell_reduce<<<gc > 0 ? gc : 1, 256, 0, s>>>(start, sorted, nc, cellsum);
     k_sr_node_gather<<<gn > 0 ? gn : 1, 256, 0, s>>>(n2cs_ptr, n2cs, cellsum, nn, a.Q);
+    return cudaGetLastError();
+}
+
+// Range check of externally supplied cell ids (opp_em_sort_by_cell).
+__global__ void k_check_cells(const int32_t *__restrict__ cell, long long n, long long nc,
+                              unsigned *flag) {
+    bool bad = false;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x)
+        bad = bad || (unsigned)cell[i] >= (unsigned long long)nc;
+    if (__any_sync(0xffffffffu, bad) && lane_id() == 0) atomicOr(flag, 1u);
+}
+
+cudaError_t launch_check_cells(const int32_t *cell, long long n, long long nc, unsigned *flag,
+                               int grid, cudaStream_t s) {
+    k_check_cells<<<grid, 256, 0, s>>>(cell, n, nc, flag);
     return cudaGetLastError();
 }
 

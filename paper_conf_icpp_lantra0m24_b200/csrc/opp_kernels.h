@@ -6,7 +6,7 @@ namespace opp {
 
 cudaError_t launch_push_move_deposit(int dep, int dh, bool multi, bool cont, bool tiled,
                                      const StepArgs &a, int grid, cudaStream_t s);
-int pmd_blocks_per_sm(bool tiled, int minb);
+int pmd_blocks_per_sm(bool tiled);
 cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero, int grid,
                               cudaStream_t s);
 cudaError_t launch_fill(const ColSet &cols, DevCounters *c, const uint32_t *holes,
@@ -35,14 +35,10 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
                               unsigned long long *tile_sums, int grid, cudaStream_t s);
 cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
-                             unsigned *start, uint32_t *dest, uint32_t *src_of, int rank_grid,
-                             cudaStream_t s);
-cudaError_t launch_scatter_cols(const ColSet &src, const ColSet &dst, const uint32_t *dest,
-                                const DevCounters *c, int grid, cudaStream_t s);
-cudaError_t launch_sort_move(const ColSet &src, const ColSet &dst, const int32_t *p2c,
-                             DevCounters *c, int cell_base, long long nc, const uint32_t *skey,
-                             unsigned *start, uint32_t *dest, uint32_t *src_of, int grid,
-                             int rank_grid, cudaStream_t s);
+                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s);
+cudaError_t launch_sort_gather(const ColDesc &src, char *dst, const uint32_t *src_of,
+                               const unsigned *total_p, int grid, cudaStream_t s);
+cudaError_t launch_sort_commit(DevCounters *c, const unsigned *start_total, cudaStream_t s);
 
 cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
                              unsigned long long *counts, int grid, cudaStream_t s);
@@ -57,5 +53,8 @@ cudaError_t launch_halo_pack(const double *Q, const int32_t *idx, long long m, d
                              cudaStream_t s);
 cudaError_t launch_halo_add(double *Q, const int32_t *idx, long long m, const double *in,
                             cudaStream_t s);
+
+cudaError_t launch_check_cells(const int32_t *cell, long long n, long long nc, unsigned *flag,
+                               int grid, cudaStream_t s);
 
 }  // namespace opp

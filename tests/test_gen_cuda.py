@@ -16,6 +16,12 @@ def test_seed_and_inject_bit_identical():
         b = gc.seed_particles(dm, 100_003, 77, cluster=cluster, id_base=5)
         for k in ("pos", "vel", "cell", "id"):
             np.testing.assert_array_equal(a[k], b[k].cpu().numpy())
+    # chunked generation (C4 seeds 1e9 particles in chunks) = generating at once
+    whole = gen.seed_particles(mesh, 50_000, 78, id_base=7)
+    for first, n in ((0, 20_000), (20_000, 30_000)):
+        b = gc.seed_particles(dm, n, 78, id_base=7, first=first)
+        for k in ("pos", "vel", "cell", "id"):
+            np.testing.assert_array_equal(whole[k][first:first + n], b[k].cpu().numpy())
     for s in (0, 3):
         a = gen.inject_batch(mesh, s, 5001, 77, id_base=9)
         b = gc.inject_batch(dm, s, 5001, 77, id_base=9)

@@ -175,15 +175,12 @@ def test_conservation_and_bookkeeping_gpu_only():
     sim.close()
 
 
-@pytest.mark.parametrize("fused", ["1", "0"])
 @pytest.mark.parametrize("dep,sort_every,axis", [(0, 1, 0), (1, 3, 0), (2, 2, 0), (1, 1, 1), (0, 2, 1)])
-def test_c1_parity_with_periodic_sort(dep, sort_every, axis, fused, monkeypatch):
+def test_c1_parity_with_periodic_sort(dep, sort_every, axis):
     """The periodic counting sort by cell (which also compacts) changes the
     storage order only: results keyed by id are identical (plain cell-id key
-    and the locality key along the duct axis).  fused 1: the sort step's move
-    writes every particle to its sorted position (the default); 0: a separate
-    counting-sort pass after the move."""
-    monkeypatch.setenv("OPP_FUSE_SORT", fused)
+    and the locality key along the duct axis).  The sort gathers one column
+    at a time into the spare of its size (column rotation)."""
     mesh, ef, init, inject, steps = c1_case()
     _check(mesh, ef, init, inject, steps, deposit_mode=dep, sort_every=sort_every,
            sort_axis=(0.0, 0.0, 1.0) if axis else (0.0, 0.0, 0.0))

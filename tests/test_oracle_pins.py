@@ -381,3 +381,15 @@ def test_walk_tie_takes_lowest_index():
     assert lam[1] == lam[2] < 0
     st, fc, hops, lam2, cap = om.walk(0, x, hcap=1)
     assert cap == 1 and hops == 1 and fc == mesh["c2c"][0, 1]
+
+
+def test_seed_generator_chunks_equal_whole():
+    """gen.seed_particles(first=...) chunks reproduce the whole population
+    (C4's 1e9 particles are generated in chunks on the device)."""
+    import gen
+    mesh = gen.kuhn_duct(3, 3, 4)
+    whole = gen.seed_particles(mesh, 1000, 11, id_base=3)
+    a = gen.seed_particles(mesh, 400, 11, id_base=3)
+    b = gen.seed_particles(mesh, 600, 11, id_base=3, first=400)
+    for k in ("pos", "vel", "cell", "id"):
+        np.testing.assert_array_equal(whole[k], np.concatenate([a[k], b[k]]))
