@@ -70,6 +70,8 @@ def parse(argv=None):
     ap.add_argument("--ov", type=float, default=0.125, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=10, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--sort-init", type=int, default=-1,
+                    help="sort the seeded population once before the run (default: iff --sort > 0)")
     ap.add_argument("--shuffle", type=int, default=0,
                     help="randomly shuffle the particles every K steps (the paper's GPU policy; use with --sort 0)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
@@ -655,7 +657,7 @@ class EsRank:
                 sim.inject(init, on_device=True)
                 stream.synchronize()
                 del init
-            if args.sort:
+            if args.sort_init > 0 or (args.sort_init < 0 and args.sort):
                 # the population is born in random cell order; a sorted steady
                 # state is what periodic sorting maintains (setup, untimed)
                 sim.step(0.0, 1.0, w, stats=False, fill=True)   # builds mesh data; dt = 0: no motion

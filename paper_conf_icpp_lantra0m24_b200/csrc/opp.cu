@@ -1228,8 +1228,8 @@ static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p
 }
 
 // Node-charge halo: exchange the interface nodes'
-// partial sums with each neighbour and add them (a + b = b + a: both copies
-// of a node end bit-identical when two ranks share it).
+// partial sums with every peer sharing them and combine all holders' values
+// in global rank order (k_halo_combine: every copy ends bit-identical).
 static int halo_sum(opp_ctx c, double *Q) {
     opp::Comm *cm = c->comm;
     const int R = cm->nranks;
@@ -1241,7 +1241,7 @@ static int halo_sum(opp_ctx c, double *Q) {
     }
     TRY(cm->t->exchange((const char *)cm->d_halo_send, off, bytes, (char *)cm->d_halo_recv, off, bytes,
                         c->s, g_err));
-    CK(launch_halo_add(Q, cm->d_halo_idx, cm->halo_n, cm->d_halo_recv, c->s));
+    CK(launch_halo_combine(Q, cm->d_hc_node, cm->d_hc_ptr, cm->d_hc_ent, cm->hc_n, cm->d_halo_recv, c->s));
     c->launches += 2;
     return OPP_OK;
 }

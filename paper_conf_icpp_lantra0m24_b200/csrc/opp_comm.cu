@@ -263,6 +263,9 @@ void comm_free(Comm *c) {
     if (c->d_halo_idx) cudaFree(c->d_halo_idx);
     if (c->d_halo_send) cudaFree(c->d_halo_send);
     if (c->d_halo_recv) cudaFree(c->d_halo_recv);
+    if (c->d_hc_node) cudaFree(c->d_hc_node);
+    if (c->d_hc_ptr) cudaFree(c->d_hc_ptr);
+    if (c->d_hc_ent) cudaFree(c->d_hc_ent);
     if (c->sendbuf) cudaFree(c->sendbuf);
     if (c->recvbuf) cudaFree(c->recvbuf);
     delete c;
@@ -380,6 +383,36 @@ int comm_set_partition(Comm *c, long long n_global_cells, const int32_t *rank_of
     }
     if (!idx.empty())
         cudaMemcpyAsync(c->d_halo_idx, idx.data(), 4 * idx.size(), cudaMemcpyHostToDevice, s);
+    // combine plan: for each distinct shared local node, (rank, entry) pairs
+    // of every holder sorted by rank (entry -1 = this rank's own value)
+    std::map<int32_t, std::vector<std::pair<int, int32_t>>> holders;
+    for (int p = 0; p < R; p++)
+        for (int64_t k = c->halo_off[p]; k < c->halo_off[p] + c->halo_cnt[p]; k++)
+            holders[idx[k]].push_back({p, (int32_t)k});
+    std::vector<int32_t> hnode, hptr(1, 0), hent;
+    for (auto &kv : holders) {
+        kv.second.push_back({c->rank, -1});
+        std::sort(kv.second.begin(), kv.second.end());
+        hnode.push_back(kv.first);
+        for (auto &pe : kv.second) hent.push_back(pe.second);
+        hptr.push_back((int32_t)hent.size());
+    }
+    c->hc_n = (int64_t)hnode.size();
+    if (c->d_hc_node) cudaFree(c->d_hc_node);
+    if (c->d_hc_ptr) cudaFree(c->d_hc_ptr);
+    if (c->d_hc_ent) cudaFree(c->d_hc_ent);
+    c->d_hc_node = c->d_hc_ptr = c->d_hc_ent = nullptr;
+    if (cudaMalloc(&c->d_hc_node, 4 * std::max<size_t>(hnode.size(), 1)) != cudaSuccess ||
+        cudaMalloc(&c->d_hc_ptr, 4 * hptr.size()) != cudaSuccess ||
+        cudaMalloc(&c->d_hc_ent, 4 * std::max<size_t>(hent.size(), 1)) != cudaSuccess) {
+        err = "halo combine plan";
+        return OPP_ERR_NOMEM;
+    }
+    if (!hnode.empty()) {
+        cudaMemcpyAsync(c->d_hc_node, hnode.data(), 4 * hnode.size(), cudaMemcpyHostToDevice, s);
+        cudaMemcpyAsync(c->d_hc_ent, hent.data(), 4 * hent.size(), cudaMemcpyHostToDevice, s);
+    }
+    cudaMemcpyAsync(c->d_hc_ptr, hptr.data(), 4 * hptr.size(), cudaMemcpyHostToDevice, s);
     e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return cuda_fail(e, "halo plan upload", err);
     c->partitioned = true;

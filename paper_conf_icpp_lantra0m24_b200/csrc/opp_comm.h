@@ -40,6 +40,12 @@ struct Comm {
     int32_t *d_halo_idx = nullptr;
     double *d_halo_send = nullptr, *d_halo_recv = nullptr;
     int64_t halo_n = 0;
+    // combine plan: per distinct shared local node, its holders' values in
+    // global rank order (own value: entry -1, a peer's: its recv slot), so
+    // every rank sums a node's copies in the same order (bit-identical copies
+    // for any number of ranks sharing a node)
+    int32_t *d_hc_node = nullptr, *d_hc_ptr = nullptr, *d_hc_ent = nullptr;
+    int64_t hc_n = 0;
     // migration
     unsigned long long *d_counts = nullptr;    // nranks
     unsigned long long *d_cursor = nullptr;    // nranks

@@ -58,6 +58,11 @@ __device__ __forceinline__ int4 line_c2n(const WalkLine *__restrict__ lines, int
     return __ldg(reinterpret_cast<const int4 *>(reinterpret_cast<const double *>(lines + c) + 14));
 }
 
+// One neighbour id: c2c[c][f] (4 B per lane instead of the 16-B sector).
+__device__ __forceinline__ int line_c2c_face(const WalkLine *__restrict__ lines, int c, int f) {
+    return __ldg(reinterpret_cast<const int *>(reinterpret_cast<const double *>(lines + c) + 12) + f);
+}
+
 // Cell field E (double4, 32-B aligned): one 256-bit read-only load.
 __device__ __forceinline__ void load_E(const double4 *__restrict__ ef, int lc, double2 &exy,
                                        double &ez) {
@@ -223,23 +228,31 @@ __device__ __forceinline__ void deposit(const StepArgs &a, bool done, int cell, 
     deposit_agg(a.Q, a, done, cell, v0, v1, v2, v3);
 }
 
-// SR deposit, phase 1: store (cell, w*lambda[4]) records.
-__device__ __forceinline__ void sr_store(const StepArgs &a, bool done, int cell, double w,
-                                         double l0, double l1, double l2, double l3) {
-    unsigned long long slot = warp_append(done, &a.cnt->n_sr);
+// SR deposit, phase 1 (Fig. 3 "store values and keys"):
+// the record of particle i sits at index i -- key = its local cell, or -1
+// when it deposits nothing here (removed, migrating, deferred: a deferred or
+// received particle's record is written where its walk ends) -- so records
+// follow the storage order (coalesced stores; nearly sorted by cell in
+// cell-sorted storage, which the run-aggregated passes below exploit).
+__device__ __forceinline__ void sr_store(const StepArgs &a, bool write, bool done, unsigned long long i,
+                                         int cell, double w, double l0, double l1, double l2,
+                                         double l3) {
+    if (!write) return;
+    a.sr_cell[i] = done ? cell - a.cell_base : -1;
     if (done) {
-        a.sr_cell[slot] = cell - a.cell_base;
-        a.sr_val[slot] = mul(w, l0);
-        a.sr_val[a.cap + slot] = mul(w, l1);
-        a.sr_val[2 * a.cap + slot] = mul(w, l2);
-        a.sr_val[3 * a.cap + slot] = mul(w, l3);
+        a.sr_val[i] = mul(w, l0);
+        a.sr_val[a.cap + i] = mul(w, l1);
+        a.sr_val[2 * a.cap + i] = mul(w, l2);
+        a.sr_val[3 * a.cap + i] = mul(w, l3);
     }
 }
 
+// `write`: this lane's particle ends its visit sequence here (SR writes its
+// record, done or not); `done`: it deposits.
 template <int DEP>
-__device__ __forceinline__ void deposit_any(const StepArgs &a, bool done, int cell, double l0,
-                                            double l1, double l2, double l3) {
-    if (DEP == 2) sr_store(a, done, cell, a.w, l0, l1, l2, l3);
+__device__ __forceinline__ void deposit_any(const StepArgs &a, bool write, bool done, unsigned long long i,
+                                            int cell, double l0, double l1, double l2, double l3) {
+    if (DEP == 2) sr_store(a, write, done, i, cell, a.w, l0, l1, l2, l3);
     else deposit<DEP>(a, done, cell, a.w, l0, l1, l2, l3);
 }
 
@@ -333,21 +346,36 @@ constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
 constexpr int kStages = 2;
 constexpr int kMinBlocks = 3;
-constexpr int kStageBytes = kTile * (6 * 8 + 4);
+constexpr int kStageBytes = kTile * (6 * 8 + 4);          // the bulk-copied particle columns
+// per-particle gathers the producer warp adds to a landed stage (OPP_AUX):
+// E of the start cell (3 doubles), the DH seed of the drift-only position and
+// its overlay slot
+#ifndef OPP_AUX
+#define OPP_AUX 0
+#endif
+constexpr int kAuxBytes = OPP_AUX ? kTile * (3 * 8 + 4 + 4) : 0;
+constexpr int kStageStride = kStageBytes + kAuxBytes;
 constexpr int kRing = 64;
 constexpr int kRingBytesPerWarp = kRing * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
-constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8;
-constexpr int kTiledSmem = kRingBase + kConsumerWarps * kRingBytesPerWarp;
+constexpr int kRingBase = kStages * kStageStride + 3 * kStages * 8;
+constexpr int kQBase = kRingBase + kConsumerWarps * kRingBytesPerWarp;
 
 struct StageView {
     double *c[6];   // x, y, z, vx, vy, vz
     int *cell;
+    double *e[3];   // aux: E of the start cell
+    int *seed;      // aux: DH seed of the drift-only position (DH 1), else the start cell
+    int *slot;      // aux: its overlay slot (-1 outside the overlay)
 };
 __device__ __forceinline__ StageView stage_view(char *smem, int s) {
     StageView v;
-    char *b = smem + (size_t)s * kStageBytes;
+    char *b = smem + (size_t)s * kStageStride;
     for (int k = 0; k < 6; k++) v.c[k] = reinterpret_cast<double *>(b + k * kTile * 8);
     v.cell = reinterpret_cast<int *>(b + 6 * kTile * 8);
+    char *x = b + kStageBytes;
+    for (int k = 0; k < 3; k++) v.e[k] = reinterpret_cast<double *>(x + k * kTile * 8);
+    v.seed = reinterpret_cast<int *>(x + 3 * kTile * 8);
+    v.slot = v.seed + kTile;
     return v;
 }
 
@@ -395,22 +423,39 @@ __device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *coun
     }
 }
 
+// What the producer warp gathered for a particle (OPP_AUX): E of its start
+// cell, the raw overlay value of its drift-only position (DH 1; -1 = none)
+// and that position's overlay slot (-1 = outside the overlay).
+struct Aux {
+    double ex, ey, ez;
+    int seed, slot;
+};
+
 // LATE: the start cell's walk line is loaded after the push and the DH seed,
 // through an opaque dependency on the pushed position, so the 24 line
 // registers and the streamed particle state are never live at once (the
 // TMA-pipelined kernel: fewer registers, 3 blocks per SM); otherwise it is
 // issued together with E (one round trip; direct paths).
+// OPP_LADDER (measurement builds only, scripts/build_variant.sh; 0 = the
+// method): 1 stream the particle state, 2 + E gather and push, 3 + DH seed
+// and first walk-line visit, 4 + the whole walk; deposits and hole records
+// are skipped at levels 1-4, so results are invalid there.
+#ifndef OPP_LADDER
+#define OPP_LADDER 0
+#endif
 template <int DEP, int DH, bool MULTI, bool LATE>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
-                                         Appends *ap = nullptr) {
+                                         Appends *ap = nullptr, const Aux *aux = nullptr) {
     int status = ST_NONE;
     int capped = 0, hops = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
+    Line L;
+    long long spec_slot = -1;
+    int spec_val = -1;
     if (valid) {
         const int lc = cell - a.cell_base;
-        Line L;
         if (!LATE) L = load_line(a.lines, lc);
         // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
         // DH: the overlay entry of the drift-only position x + v dt is
@@ -418,16 +463,24 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         // lies in the same overlay cell (all but ~|c1 E dt| / dx of the
         // particles), so the seed is exactly that of the pushed position and
         // the lookup leaves the dependent chain.
-        long long spec_slot = -1;
-        int spec_val = -1;
-        if (DH == 1) {
-            spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
-                                add(z, mul(vz, a.dt)));
-            spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
-        }
         double2 Exy;
         double Ez;
-        load_E(a.ef, lc, Exy, Ez);
+        if (OPP_LADDER == 1) {
+            Exy = make_double2(0.0, 0.0);
+            Ez = 0.0;
+        } else if (aux) {
+            spec_slot = aux->slot;
+            spec_val = aux->seed;
+            Exy = make_double2(aux->ex, aux->ey);
+            Ez = aux->ez;
+        } else {
+            if (DH == 1 && OPP_LADDER != 2) {
+                spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
+                                    add(z, mul(vz, a.dt)));
+                spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
+            }
+            load_E(a.ef, lc, Exy, Ez);
+        }
         vx = add(vx, mul(a.c1, Exy.x));
         vy = add(vy, mul(a.c1, Exy.y));
         vz = add(vz, mul(a.c1, Ez));
@@ -437,6 +490,9 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         // position and velocity are final now: store them before the walk
         a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
         a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+        if (OPP_LADDER == 1 || OPP_LADDER == 2) valid = false;
+    }
+    if (valid) {
         if (DH == 1) {   // seed every particle from the overlay (reading S19'' mode 1)
             const long long g = dh_slot(a.ov, x, y, z);
             int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
@@ -463,7 +519,9 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
                 }
             }
         }
-        status = walk_from<MULTI>(a, cell, L, x, y, z, hops, a.hpass, l0, l1, l2, l3, capped);
+        status = walk_from<MULTI>(a, cell, L, x, y, z, hops, OPP_LADDER == 3 ? 0 : a.hpass, l0, l1, l2,
+                                  l3, capped);
+        if (OPP_LADDER) status = ST_DONE;
         if (status != ST_MOVE && status != ST_MIGRATE) {   // counted where the walk ends
             t.hops += (unsigned)hops;
             t.maxh = max(t.maxh, (unsigned)hops);
@@ -471,7 +529,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         }
         t.removed += (status == ST_REMOVE);
     }
-    deposit_any<DEP>(a, status == ST_DONE, cell, l0, l1, l2, l3);
+    if (!OPP_LADDER) deposit_any<DEP>(a, valid, status == ST_DONE, i, cell, l0, l1, l2, l3);
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
     if (ap) {
@@ -565,6 +623,200 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
 }
 
 // ---------------------------------------------------------------------------
+// Hop queue (TMA-pipelined kernel): a particle that is not inside the cell of
+// its first visit does not keep its warp in the walk loop.  Its position,
+// cell, the face to cross and its hop count go to a per-warp queue in shared
+// memory; whenever 32 are queued the warp advances them all by one cell visit
+// together and requeues those still outside.  A warp instruction costs the L1
+// data pipe the same whether 1 or 32 lanes are active (scripts/micro/wf_cost.cu:
+// a 256-bit load costs 8 cycles even for one lane), and ~19% of the particles
+// hop (DH seeding, 0.25 h/step drift), so a hop iteration of a whole warp used
+// to cost a full walk-line load for a few lanes.  Semantics are the walk's
+// (walk_from): the same visits in the same order per particle, H_cap and
+// H_pass tested at the same points.
+// ---------------------------------------------------------------------------
+#ifndef OPP_HOPQ
+#define OPP_HOPQ 0
+#endif
+constexpr int kQ = 64;                                   // ring entries per warp
+constexpr int kQBytesPerWarp = kQ * (3 * 8 + 4 * 4);     // x, y, z | cell, face, hops, index
+constexpr int kTiledSmem = kQBase + (OPP_HOPQ ? kConsumerWarps * kQBytesPerWarp : 0);
+struct HopQueue {
+    double *x, *y, *z;
+    int *cell, *face, *hops;
+    uint32_t *idx;
+    unsigned head, count;   // warp-uniform
+};
+__device__ __forceinline__ HopQueue hop_queue(char *base) {
+    HopQueue q;
+    q.x = reinterpret_cast<double *>(base);
+    q.y = q.x + kQ;
+    q.z = q.y + kQ;
+    q.cell = reinterpret_cast<int *>(q.z + kQ);
+    q.face = q.cell + kQ;
+    q.hops = q.face + kQ;
+    q.idx = reinterpret_cast<uint32_t *>(q.hops + kQ);
+    q.head = 0;
+    q.count = 0;
+    return q;
+}
+__device__ __forceinline__ void q_push(HopQueue &q, bool pred, double x, double y, double z, int cell,
+                                       int face, int hops, uint32_t i) {
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    if (!m) return;
+    if (pred) {
+        const unsigned sl = (q.head + q.count + __popc(m & ((1u << lane_id()) - 1u))) & (kQ - 1);
+        q.x[sl] = x; q.y[sl] = y; q.z[sl] = z;
+        q.cell[sl] = cell; q.face[sl] = face; q.hops[sl] = hops; q.idx[sl] = i;
+    }
+    q.count += __popc(m);
+    __syncwarp();
+}
+
+// Appends of a finished walk (holes, deferred walks, migrants) and its stats.
+template <bool MULTI>
+__device__ __forceinline__ void finish_appends(const StepArgs &a, Appends &ap, int status, uint32_t i,
+                                               int cell, int hops, int capped, Tally &t) {
+    if (status != ST_NONE && status != ST_MOVE && status != ST_MIGRATE) {
+        t.hops += (unsigned)hops;
+        t.maxh = max(t.maxh, (unsigned)hops);
+        t.capped += (unsigned)capped;
+    }
+    t.removed += (status == ST_REMOVE);
+    const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
+    ring_push(ap.holes, rem, i, 0);
+    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
+    ring_push(ap.work, status == ST_MOVE, i, hops);
+    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
+    if (MULTI) {
+        const bool mg = status == ST_MIGRATE;
+        unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
+        if (mg) {
+            a.mig[ms] = i;
+            a.mig_cell[ms] = cell;
+            a.mig_hops[ms] = hops;
+        }
+    }
+}
+
+// First visit of one 32-particle slice: push, DH seed, the seed cell's walk
+// line; a particle inside is done (deposited here), one outside is queued with
+// the face to cross (or, at H_cap / H_pass = 0, accepted / deferred as the walk
+// would).  On return `cell` is what p2c holds after this slice (-1 = hole;
+// queued particles hold their current cell until their walk ends).
+template <int DEP, int DH, bool MULTI>
+__device__ __forceinline__ void pmd_first(const StepArgs &a, uint32_t i, double x, double y, double z,
+                                          double vx, double vy, double vz, int &cell, Tally &t,
+                                          Appends &ap, HopQueue &q, const Aux *aux) {
+    const int lc = cell - a.cell_base;
+    long long spec_slot = -1;
+    int spec_val = -1;
+    double2 Exy;
+    double Ez;
+    if (aux) {
+        spec_slot = aux->slot;
+        spec_val = aux->seed;
+        Exy = make_double2(aux->ex, aux->ey);
+        Ez = aux->ez;
+    } else {
+        if (DH == 1) {   // the overlay entry of the drift-only position (see pmd_body)
+            spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)), add(z, mul(vz, a.dt)));
+            spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
+        }
+        load_E(a.ef, lc, Exy, Ez);
+    }
+    vx = add(vx, mul(a.c1, Exy.x));
+    vy = add(vy, mul(a.c1, Exy.y));
+    vz = add(vz, mul(a.c1, Ez));
+    x = add(x, mul(vx, a.dt));
+    y = add(y, mul(vy, a.dt));
+    z = add(z, mul(vz, a.dt));
+    a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
+    a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+    if (DH == 1) {
+        const long long g = dh_slot(a.ov, x, y, z);
+        int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
+        if (g < 0) v = -1;
+        if (v >= 0) cell = v;
+    }
+    int zero;   // the line load after the push (see pmd_body, LATE)
+    asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}" : "=r"(zero) : "d"(z));
+    Line L = load_line(a.lines, cell - a.cell_base + zero);
+    double l0, l1, l2, l3;
+    bary(L, x, y, z, l0, l1, l2, l3);
+    bool inside = in01(l0) && in01(l1) && in01(l2) && in01(l3);
+    if (DH == 2 && !inside) {
+        const int sc = dh_seed(a.ov, x, y, z, cell);
+        if (sc != cell) {
+            cell = sc;
+            L = load_line(a.lines, sc - a.cell_base);
+            bary(L, x, y, z, l0, l1, l2, l3);
+            inside = in01(l0) && in01(l1) && in01(l2) && in01(l3);
+        }
+    }
+    int status = ST_DONE, capped = 0;
+    if (!inside) {
+        if (0 >= a.hcap) capped = 1;              // accepted as it stands (S4)
+        else if (0 >= a.hpass) status = ST_MOVE;  // deferred to the continuation
+        else status = ST_NONE;                    // queued
+    }
+    deposit_any<DEP>(a, true, status == ST_DONE, i, cell, l0, l1, l2, l3);
+    finish_appends<MULTI>(a, ap, status, i, cell, 0, capped, t);
+    q_push(q, status == ST_NONE, x, y, z, cell, argmin_face(l0, l1, l2, l3), 0, i);
+}
+
+// One cell visit for k <= 32 queued particles (lane l takes entry head + l).
+template <int DEP, bool MULTI>
+__device__ __forceinline__ void hop_round(const StepArgs &a, HopQueue &q, unsigned k, Tally &t,
+                                          Appends &ap) {
+    const unsigned lane = lane_id();
+    const bool act = lane < k;
+    double x = 0, y = 0, z = 0;
+    int cell = 0, f = 0, hops = 0;
+    uint32_t i = 0;
+    if (act) {
+        const unsigned sl = (q.head + lane) & (kQ - 1);
+        x = q.x[sl]; y = q.y[sl]; z = q.z[sl];
+        cell = q.cell[sl]; f = q.face[sl]; hops = q.hops[sl]; i = q.idx[sl];
+    }
+    __syncwarp();
+    q.head = (q.head + k) & (kQ - 1);
+    q.count -= k;
+    int status = ST_NONE, capped = 0;
+    double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
+    if (act) {
+        const int nb = line_c2c_face(a.lines, cell - a.cell_base, f);
+        if (nb < 0) {
+            status = ST_REMOVE;
+        } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
+            cell = nb;   // the hop into the other rank's cell counts here
+            hops++;
+            status = ST_MIGRATE;
+        } else {
+            cell = nb;
+            hops++;
+            const Line L = load_line(a.lines, nb - a.cell_base);
+            bary(L, x, y, z, l0, l1, l2, l3);
+            if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
+                status = ST_DONE;
+            } else if (hops >= a.hcap) {
+                status = ST_DONE;
+                capped = 1;
+            } else if (hops >= a.hpass) {
+                status = ST_MOVE;
+            } else {
+                f = argmin_face(l0, l1, l2, l3);
+            }
+        }
+    }
+    deposit_any<DEP>(a, act && status != ST_NONE, status == ST_DONE, i, cell, l0, l1, l2, l3);
+    finish_appends<MULTI>(a, ap, status, i, cell, hops, capped, t);
+    if (act && status != ST_NONE)
+        a.p2c[i] = (status == ST_REMOVE || status == ST_MIGRATE) ? -1 : cell;
+    q_push(q, act && status == ST_NONE, x, y, z, cell, f, hops, i);
+}
+
+// ---------------------------------------------------------------------------
 // The fused push / move / deposit kernel, TMA-pipelined (CalcPosVel + Move +
 // DepositCharge of PAPER.md:1586-1604 in one pass).  Blocks visit groups of
 // a.tile_group consecutive kTile-particle tiles round-robin (L1 locality of
@@ -614,6 +866,10 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
 
+__device__ __forceinline__ void prefetch_l1(const void *p) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+}
+
 // producer: load tile `tile` into stage s
 __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, uint64_t *full,
                                                 int s, unsigned long long tile) {
@@ -627,11 +883,62 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
+// Producer warp, tile t (landed in stage t % kStages): per particle E of the
+// start cell and (DH 1) the overlay entry of the drift-only position x + v dt
+// into the stage's aux columns, and an L1 prefetch of the walk line the
+// consumer will load first (the seed cell, else the start cell).  Lane l
+// takes particles l, l + 32, ... (coalesced shared accesses), four at a time
+// so their loads are in flight together.
+template <int DH>
+__device__ __forceinline__ void producer_aux(const StepArgs &a, char *smem, uint64_t *full,
+                                             uint64_t *ready, unsigned long long t, unsigned lane) {
+    const int s = (int)(t % kStages);
+    mbar_wait(&full[s], (uint32_t)((t / kStages) & 1ull));
+    const StageView v = stage_view(smem, s);
+#pragma unroll
+    for (int half = 0; half < kTile / 128; half++) {
+        double ex[4], ey[4], ez[4];
+        int cl[4], sl[4], sv[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const int j = (int)lane + 32 * (4 * half + q);
+            cl[q] = v.cell[j];
+            double2 exy;
+            load_E(a.ef, cl[q] - a.cell_base, exy, ez[q]);
+            ex[q] = exy.x;
+            ey[q] = exy.y;
+            sl[q] = -1;
+            sv[q] = -1;
+            if (DH == 1) {
+                const long long g = dh_slot(a.ov, add(v.c[0][j], mul(v.c[3][j], a.dt)),
+                                            add(v.c[1][j], mul(v.c[4][j], a.dt)),
+                                            add(v.c[2][j], mul(v.c[5][j], a.dt)));
+                sl[q] = (int)g;
+                sv[q] = ov_value(a.ov, g >= 0 ? g : 0);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const int j = (int)lane + 32 * (4 * half + q);
+            v.e[0][j] = ex[q];
+            v.e[1][j] = ey[q];
+            v.e[2][j] = ez[q];
+            v.seed[j] = sv[q];
+            v.slot[j] = sl[q];
+            const int sc = (DH == 1 && sl[q] >= 0 && sv[q] >= 0) ? sv[q] : cl[q];
+            prefetch_l1(a.lines + (sc - a.cell_base));
+        }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&ready[s]);
+}
+
 template <int DEP, int DH, bool MULTI>
 __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageStride);
     uint64_t *empty = full + kStages;
+    uint64_t *ready = empty + kStages;   // OPP_AUX: the producer's gathers have landed
     const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
     const unsigned long long ntiles = n / kTile;
     const TileMap tm{ntiles, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
@@ -642,20 +949,29 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
         for (int s = 0; s < kStages; s++) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], kConsumerWarps);
+            mbar_init(&ready[s], 1);
         }
         fence_proxy_async();
     }
     __syncthreads();
     if (warp == kConsumerWarps) {
-        // producer warp: lane 0 streams tiles kStages ahead of the slowest consumer
-        if (lane == 0) {
-            TileIter ti(tm);
-            for (unsigned long long it = 0; it < my; it++, ti.next()) {
-                const int s = (int)(it % kStages);
+        // producer warp: lane 0 streams tiles kStages ahead of the slowest
+        // consumer; then (OPP_AUX) the whole warp does the gathers that only
+        // depend on the streamed state for the tile that landed before -- E
+        // of the start cell, the DH seed of the drift-only position -- and
+        // prefetches the seed cell's walk line into L1, so the consumers'
+        // dependent chain starts from shared memory and an L1 hit.
+        TileIter ti(tm);
+        for (unsigned long long it = 0; it < my; it++, ti.next()) {
+            const int s = (int)(it % kStages);
+            if (lane == 0) {
                 if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
                 issue_tile_load(a, smem, full, s, ti.tile());
             }
+            __syncwarp();
+            if (OPP_AUX && it >= 1) producer_aux<DH>(a, smem, full, ready, it - 1, lane);
         }
+        if (OPP_AUX && my >= 1) producer_aux<DH>(a, smem, full, ready, my - 1, lane);
         return;
     }
     // Consumer warp, warp-synchronous: one 32-particle slice per tile.  The
@@ -670,31 +986,54 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
         ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
                            reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
     }
+#if OPP_HOPQ
+    HopQueue q = hop_queue(smem + kQBase + (size_t)warp * kQBytesPerWarp);
+#endif
     TileIter ti(tm);
     for (unsigned long long it = 0; it < my; it++, ti.next()) {
         const int s = (int)(it % kStages);
-        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
+        const uint32_t par = (uint32_t)((it / kStages) & 1ull);
+        mbar_wait(&full[s], par);
+        if (OPP_AUX) mbar_wait(&ready[s], par);
         StageView v = stage_view(smem, s);
         const int j = threadIdx.x;
         double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
         double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
         int cell = v.cell[j];
-        const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
-                                     (unsigned long long)__double_as_longlong(y) ^
-                                     (unsigned long long)__double_as_longlong(z) ^
-                                     (unsigned long long)__double_as_longlong(vx) ^
-                                     (unsigned long long)__double_as_longlong(vy) ^
-                                     (unsigned long long)__double_as_longlong(vz) ^
-                                     (unsigned long long)(unsigned)cell;
+        Aux ax;
+        if (OPP_AUX) {
+            ax.ex = v.e[0][j]; ax.ey = v.e[1][j]; ax.ez = v.e[2][j];
+            ax.seed = v.seed[j]; ax.slot = v.slot[j];
+        }
+        unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
+                               (unsigned long long)__double_as_longlong(y) ^
+                               (unsigned long long)__double_as_longlong(z) ^
+                               (unsigned long long)__double_as_longlong(vx) ^
+                               (unsigned long long)__double_as_longlong(vy) ^
+                               (unsigned long long)__double_as_longlong(vz) ^
+                               (unsigned long long)(unsigned)cell;
+        if (OPP_AUX)
+            h ^= (unsigned long long)__double_as_longlong(ax.ex) ^ (unsigned long long)__double_as_longlong(ax.ey) ^
+                 (unsigned long long)__double_as_longlong(ax.ez) ^ (unsigned long long)(unsigned)ax.seed ^
+                 ((unsigned long long)(unsigned)ax.slot << 32);
         asm volatile("" ::"l"(h));   // the shared loads have landed
         fence_proxy_async();
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[s]);
         __syncwarp();
         const unsigned long long i = ti.tile() * kTile + j;
-        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap);
+#if OPP_HOPQ
+        pmd_first<DEP, DH, MULTI>(a, (uint32_t)i, x, y, z, vx, vy, vz, cell, t, ap, q, OPP_AUX ? &ax : nullptr);
         a.p2c[i] = cell;
+        while (q.count >= 32u) hop_round<DEP, MULTI>(a, q, 32u, t, ap);
+#else
+        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap, OPP_AUX ? &ax : nullptr);
+        a.p2c[i] = cell;
+#endif
     }
+#if OPP_HOPQ
+    while (q.count) hop_round<DEP, MULTI>(a, q, min(q.count, 32u), t, ap);
+#endif
     ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
     ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
@@ -811,7 +1150,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
             t.capped += (unsigned)capped;
         }
         t.removed += (status == ST_REMOVE);
-        deposit_any<DEP>(a, status == ST_DONE, cell, l0, l1, l2, l3);
+        deposit_any<DEP>(a, fin, status == ST_DONE, i, cell, l0, l1, l2, l3);
         const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
         ring_push(hr, rem, (uint32_t)i, 0);
         ring_flush(hr, &a.cnt->n_holes, a.holes, nullptr, false);
@@ -1052,42 +1391,88 @@ __global__ void k_overlay_finish(int32_t *map, long long n) {
 // sort is a counting sort: histogram -> exclusive scan -> scatter; the
 // per-cell reduction then sums each cell's contiguous segment and the
 // per-node pass gathers the 4 sums of every incident cell through a
-// node->(cell,slot) CSR -- no floating-point atomics at all.
+// node->(cell,slot) CSR -- no floating-point atomics at all.  The records sit
+// in storage order (sr_store), so in cell-sorted storage a warp's 32 records
+// are a few runs of equal keys: the histogram and the scatter take one
+// atomic per run (run_info), not one per record.
 // ---------------------------------------------------------------------------
-__global__ void k_sr_hist(const int32_t *__restrict__ sr_cell, const DevCounters *c,
-                          unsigned *hist) {
-    const unsigned long long m = c->n_sr;
-    for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
-         k += (unsigned long long)gridDim.x * blockDim.x)
-        atomicAdd(hist + sr_cell[k], 1u);
+// Runs of equal keys in a warp: the run head, start lane and length of each lane's run.
+__device__ __forceinline__ void run_info(int key, unsigned &heads, int &run_start, int &run_len,
+                                         bool &head) {
+    const unsigned lane = lane_id();
+    int prev = __shfl_up_sync(0xffffffffu, key, 1);
+    head = (lane == 0) || (prev != key);
+    heads = __ballot_sync(0xffffffffu, head);
+    unsigned below = heads & ((2u << lane) - 1u);      // heads at or below this lane
+    if (lane == 31) below = heads;
+    run_start = 31 - __clz(below);
+    unsigned above = heads & ~((2u << lane) - 1u);
+    if (lane == 31) above = 0;
+    int run_end = above ? (__ffs(above) - 2) : 31;
+    run_len = run_end - run_start + 1;
 }
 
-__global__ void k_sr_scatter(const int32_t *__restrict__ sr_cell, const double *__restrict__ sr_val,
-                             long long cap, const DevCounters *c, unsigned *cursor,
-                             double *sorted) {
-    const unsigned long long m = c->n_sr;
-    for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
-         k += (unsigned long long)gridDim.x * blockDim.x) {
-        unsigned pos = atomicAdd(cursor + sr_cell[k], 1u);
-        sorted[4ull * pos + 0] = sr_val[k];
-        sorted[4ull * pos + 1] = sr_val[cap + k];
-        sorted[4ull * pos + 2] = sr_val[2 * cap + k];
-        sorted[4ull * pos + 3] = sr_val[3 * cap + k];
+__global__ void k_sr_hist(const int32_t *__restrict__ sr_cell, const DevCounters *c, unsigned *hist) {
+    const unsigned long long m = c->n;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+         i0 < m; i0 += stride) {
+        const unsigned long long i = i0 + lane_id();
+        const int key = i < m ? sr_cell[i] : -1;
+        unsigned heads;
+        int rs, rl;
+        bool head;
+        run_info(key >= 0 ? key : -2 - (int)lane_id(), heads, rs, rl, head);
+        if (head && key >= 0) atomicAdd(hist + key, (unsigned)rl);
     }
 }
 
-// per-cell reduce: cellsum[c][i] = sum over the cell's segment
+__global__ void k_sr_scatter(const int32_t *__restrict__ sr_cell, const double *__restrict__ sr_val,
+                             long long cap, const DevCounters *c, unsigned *cursor, double *sorted) {
+    const unsigned long long m = c->n;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+         i0 < m; i0 += stride) {
+        const unsigned long long i = i0 + lane_id();
+        const int key = i < m ? sr_cell[i] : -1;
+        unsigned heads;
+        int rs, rl;
+        bool head;
+        run_info(key >= 0 ? key : -2 - (int)lane_id(), heads, rs, rl, head);
+        unsigned base = 0;
+        if (head && key >= 0) base = atomicAdd(cursor + key, (unsigned)rl);
+        base = __shfl_sync(0xffffffffu, base, rs);
+        if (key >= 0) {
+            const unsigned long long d = base + (lane_id() - rs);
+            *reinterpret_cast<double4 *>(sorted + 4 * d) =
+                make_double4(sr_val[i], sr_val[cap + i], sr_val[2 * cap + i], sr_val[3 * cap + i]);
+        }
+    }
+}
+
+// per-cell reduce, one warp per cell: cellsum[c][i] = sum over the cell's
+// segment (lanes stride the segment, then a shuffle tree) -- a hot cell of
+// thousands of records (config C5) costs segment / 32 steps, not segment
 __global__ void k_sr_cell_reduce(const unsigned *__restrict__ start, const double *__restrict__ sorted,
                                  long long nc, double *cellsum) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
-         c += (long long)gridDim.x * blockDim.x) {
-        unsigned b = start[c], e = start[c + 1];
+    const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
+    for (long long c = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < nc; c += nw) {
+        const unsigned b = start[c], e = start[c + 1];
         double s0 = 0, s1 = 0, s2 = 0, s3 = 0;
-        for (unsigned k = b; k < e; k++) {
+        for (unsigned k = b + lane_id(); k < e; k += 32) {
             const double4 v = *reinterpret_cast<const double4 *>(sorted + 4ull * k);
             s0 = add(s0, v.x); s1 = add(s1, v.y); s2 = add(s2, v.z); s3 = add(s3, v.w);
         }
-        *reinterpret_cast<double4 *>(cellsum + 4 * c) = make_double4(s0, s1, s2, s3);
+        if (e - b > 1) {
+#pragma unroll
+            for (int d = 16; d >= 1; d >>= 1) {
+                s0 = add(s0, __shfl_xor_sync(0xffffffffu, s0, d));
+                s1 = add(s1, __shfl_xor_sync(0xffffffffu, s1, d));
+                s2 = add(s2, __shfl_xor_sync(0xffffffffu, s2, d));
+                s3 = add(s3, __shfl_xor_sync(0xffffffffu, s3, d));
+            }
+        }
+        if (lane_id() == 0) *reinterpret_cast<double4 *>(cellsum + 4 * c) = make_double4(s0, s1, s2, s3);
     }
 }
 
@@ -1187,20 +1572,6 @@ __global__ void __launch_bounds__(1024) k_scan_apply(const unsigned *__restrict_
 // Holes (p2c = -1) are dropped, so the sorted set is also hole-free.  Runs of
 // equal cells inside a warp are aggregated into one atomic.
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ void run_info(int key, unsigned &heads, int &run_start, int &run_len,
-                                         bool &head) {
-    const unsigned lane = lane_id();
-    int prev = __shfl_up_sync(0xffffffffu, key, 1);
-    head = (lane == 0) || (prev != key);
-    heads = __ballot_sync(0xffffffffu, head);
-    unsigned below = heads & ((2u << lane) - 1u);      // heads at or below this lane
-    if (lane == 31) below = heads;
-    run_start = 31 - __clz(below);
-    unsigned above = heads & ~((2u << lane) - 1u);
-    if (lane == 31) above = 0;
-    int run_end = above ? (__ffs(above) - 2) : 31;
-    run_len = run_end - run_start + 1;
-}
 
 // Sort bucket of a cell: its locality key (see opp_init_params.sort_axis) or
 // the local cell index.
@@ -1402,11 +1773,22 @@ __global__ void k_halo_pack(const double *__restrict__ Q, const int32_t *__restr
         out[k] = Q[idx[k]];
 }
 
-__global__ void k_halo_add(double *Q, const int32_t *__restrict__ idx, long long m,
-                           const double *__restrict__ in) {
-    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
-         k += (long long)gridDim.x * blockDim.x)
-        atomicAdd(Q + idx[k], in[k]);
+// Combine: every holder's partial sum of a shared node added in global rank
+// order (the own value where the entry is -1), identically on every rank, so
+// all copies of a node end bit-identical however many ranks share it.
+__global__ void k_halo_combine(double *Q, const int32_t *__restrict__ node, const int32_t *__restrict__ ptr,
+                               const int32_t *__restrict__ ent, long long m, const double *__restrict__ in) {
+    for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < m;
+         u += (long long)gridDim.x * blockDim.x) {
+        const int n = node[u];
+        const double own = Q[n];
+        double s = 0.0;
+        for (int e = ptr[u]; e < ptr[u + 1]; e++) {
+            const double v = ent[e] < 0 ? own : in[ent[e]];
+            s = e == ptr[u] ? v : add(s, v);
+        }
+        Q[n] = s;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -1580,10 +1962,10 @@ cudaError_t launch_halo_pack(const double *Q, const int32_t *idx, long long m, d
     return cudaGetLastError();
 }
 
-cudaError_t launch_halo_add(double *Q, const int32_t *idx, long long m, const double *in,
-                            cudaStream_t s) {
+cudaError_t launch_halo_combine(double *Q, const int32_t *node, const int32_t *ptr, const int32_t *ent,
+                                long long m, const double *in, cudaStream_t s) {
     int g = (int)std::min<long long>(1184, (m + 255) / 256);
-    k_halo_add<<<g > 0 ? g : 1, 256, 0, s>>>(Q, idx, m, in);
+    k_halo_combine<<<g > 0 ? g : 1, 256, 0, s>>>(Q, node, ptr, ent, m, in);
     return cudaGetLastError();
 }
 
@@ -1683,7 +2065,7 @@ cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *h
     if (e != cudaSuccess) return e;
     cudaMemcpyAsync(hist, start, sizeof(unsigned) * (nc + 1), cudaMemcpyDeviceToDevice, s);
     k_sr_scatter<<<grid, 256, 0, s>>>(a.sr_cell, a.sr_val, a.cap, a.cnt, hist, sorted);
-    int gc = (int)((nc + 255) / 256), gn = (int)((nn + 255) / 256);
+    int gc = (int)std::min<long long>((nc + 7) / 8, 148 * 16), gn = (int)((nn + 255) / 256);
     k_sr_cell_reduce<<<gc > 0 ? gc : 1, 256, 0, s>>>(start, sorted, nc, cellsum);
     k_sr_node_gather<<<gn > 0 ? gn : 1, 256, 0, s>>>(n2cs_ptr, n2cs, cellsum, nn, a.Q);
     return cudaGetLastError();

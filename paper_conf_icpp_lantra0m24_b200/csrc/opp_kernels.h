@@ -51,8 +51,8 @@ cudaError_t launch_mig_unpack(const ColSet &cols, const char *recvbuf, long long
                               cudaStream_t s);
 cudaError_t launch_halo_pack(const double *Q, const int32_t *idx, long long m, double *out,
                              cudaStream_t s);
-cudaError_t launch_halo_add(double *Q, const int32_t *idx, long long m, const double *in,
-                            cudaStream_t s);
+cudaError_t launch_halo_combine(double *Q, const int32_t *node, const int32_t *ptr, const int32_t *ent,
+                                long long m, const double *in, cudaStream_t s);
 
 cudaError_t launch_check_cells(const int32_t *cell, long long n, long long nc, unsigned *flag,
                                int grid, cudaStream_t s);

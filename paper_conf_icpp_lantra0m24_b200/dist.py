@@ -31,16 +31,26 @@ def rank_of_cell(mesh: dict, nranks: int) -> np.ndarray:
     return out
 
 
-def slab(mesh: dict, nranks: int, rank: int) -> dict:
+def slab(mesh: dict, nranks: int, rank: int, rank_of_cell_: np.ndarray | None = None) -> dict:
     """Rank `rank`'s slab of a global gen.kuhn_duct mesh.
 
     Local cells are the global range [cell_base, cell_base + n_cells) in
     order; c2c keeps GLOBAL cell ids (neighbours on other ranks included);
     c2n is renumbered to the slab's own nodes, whose global ids are in
-    node_gid (interface-plane nodes appear on both neighbouring ranks)."""
+    node_gid (interface-plane nodes appear on both neighbouring ranks).
+    rank_of_cell_: any partition into contiguous cell ranges (default: whole
+    hex layers, rank_of_cell); ranges that cut layers make some nodes shared
+    by more than two ranks."""
     cpl = 6 * mesh["nx"] * mesh["ny"]
-    k0, k1 = layer_bounds(mesh["nz"], nranks)[rank]
-    lo, hi = k0 * cpl, k1 * cpl
+    if rank_of_cell_ is None:
+        k0, k1 = layer_bounds(mesh["nz"], nranks)[rank]
+        lo, hi = k0 * cpl, k1 * cpl
+        roc = rank_of_cell(mesh, nranks)
+    else:
+        roc = np.ascontiguousarray(rank_of_cell_, dtype=np.int32)
+        mine = np.nonzero(roc == rank)[0]
+        lo, hi = int(mine[0]), int(mine[-1]) + 1
+        k0, k1 = lo // cpl, -(-hi // cpl)
     c2n_g = mesh["c2n"][lo:hi]
     gid = np.unique(c2n_g)
     c2n_l = np.searchsorted(gid, c2n_g).astype(np.int32)
@@ -56,7 +66,7 @@ def slab(mesh: dict, nranks: int, rank: int) -> dict:
         "c2c": np.ascontiguousarray(mesh["c2c"][lo:hi]),
         "n_cells": hi - lo, "n_nodes": int(gid.size),
         "node_gid": gid.astype(np.int64), "cell_base": lo,
-        "n_cells_global": mesh["n_cells"], "rank_of_cell": rank_of_cell(mesh, nranks),
+        "n_cells_global": mesh["n_cells"], "rank_of_cell": roc,
         "inlet": inl, "inlet_local": np.ascontiguousarray(inl_local), "box": mesh["box"],
         "rank": rank, "nranks": nranks,
         "layers": (k0, k1),

@@ -10,7 +10,9 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libopp.so")
+# OPP_LIB: an alternative build of the same library (measurement A/B runs;
+# bench.py records every OPP_* variable in its JSON line)
+LIB_PATH = os.environ.get("OPP_LIB") or os.path.join(_HERE, "libopp.so")
 
 OPP_OK, OPP_ERR_ARG, OPP_ERR_STATE, OPP_ERR_NOMEM, OPP_ERR_CAPACITY = 0, -1, -2, -3, -4
 OPP_ERR_CUDA, OPP_ERR_NCCL, OPP_ERR_MESH = -5, -6, -7

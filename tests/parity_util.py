@@ -47,10 +47,13 @@ def run_oracle(mesh, ef, init, inject, steps, c1, dt, w, hcap=1024, use_dh=False
     return om, out, Q, stats, removed
 
 
-def compare(om, c2n, orc, Q_orc, removed_margin, gpu, Q_gpu, w, h=1.0, v_ref=0.25):
-    """Returns a report dict; raises AssertionError on a parity failure."""
-    excl = set(orc["id"][orc["margin"] < NEAR].tolist())
-    excl |= {i for i, m in removed_margin.items() if m < NEAR}
+def compare(om, c2n, orc, Q_orc, removed_margin, gpu, Q_gpu, w, h=1.0, v_ref=0.25, near=NEAR):
+    """Returns a report dict; raises AssertionError on a parity failure.
+    near=None: no near-face exclusion (every particle compared bit-exactly)."""
+    excl = set()
+    if near is not None:
+        excl = set(orc["id"][orc["margin"] < near].tolist())
+        excl |= {i for i, m in removed_margin.items() if m < near}
     o_ids, g_ids = orc["id"], gpu["id"]
     so, sg = set(o_ids.tolist()), set(g_ids.tolist())
     assert len(sg) == len(g_ids), "duplicate ids on the GPU side"

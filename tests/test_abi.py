@@ -29,11 +29,25 @@ def test_library_builds_and_exports_every_declared_symbol():
 
 
 def test_sass_is_sm100a_and_has_no_fp64_fma_in_push():
+    """S11: the push and the barycentric coordinates are evaluated without FMA
+    contraction, as the oracle (-ffp-contract=off) evaluates them.  Every
+    instance of the particle-loop kernels (pass 1 tiled / direct / tail, the
+    continuation) must contain fp64 multiplies and adds but no DFMA."""
     from paper_conf_icpp_lantra0m24_b200 import build
     lib_path = build.build()
     out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", lib_path],
                          capture_output=True, text=True).stdout
     assert "sm_100a" in out
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", lib_path],
+                          capture_output=True, text=True).stdout
+    secs = re.split(r"\n\s*Function : ", sass)[1:]
+    hot = [sec for sec in secs if any(k in sec.split("\n", 1)[0]
+                                      for k in ("k_push_move_deposit", "k_walk_refill"))]
+    assert len(hot) >= 40   # 3 deposit modes x 3 DH modes x (1, N ranks) x (tiled, direct, tail) + refill
+    for sec in hot:
+        name = sec.split("\n", 1)[0].strip()
+        assert "DMUL" in sec and "DADD" in sec, name
+        assert not re.search(r"\bDFMA\b", sec), f"fp64 FMA in {name}"
 
 
 def test_defaults_and_errors_without_gpu():

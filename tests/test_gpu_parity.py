@@ -289,3 +289,59 @@ def test_c5_style_clustered_parity(dep, sort_every):
     init = gen.seed_particles(mesh, 100_000, 20240816, cluster=(0.9, hot))
     rep, ost, gst = _check(mesh, ef, init, None, 4, deposit_mode=dep, sort_every=sort_every)
     assert rep["n_compared"] > 95_000
+
+
+def exact_geometry_case():
+    """Particles whose positions are exact dyadic numbers on an unjittered
+    Kuhn duct (h = 1, E = 0): after every step they sit exactly on nodes,
+    edges, shared faces (box faces and the Kuhn faces x = y, y = z, x = z of a
+    hex), at argmin ties (lambda_i = lambda_j < 0: moves across an edge),
+    outside the box beyond faces, edges and corners (removal through them),
+    or at rest (v = 0).  Both sides evaluate lambda in the same order, so even
+    these decisions (inclusive inside test S1, lowest-index tie S2, removal)
+    must agree exactly: compared with NO near-face exclusion."""
+    import oracle
+    mesh = gen.kuhn_duct(3, 3, 4)
+    om = oracle.Mesh.from_gen(mesh)
+    ax = [np.arange(-0.25, 3.26, 0.25)] * 2 + [np.arange(-0.25, 4.26, 0.25)]
+    T = np.stack(np.meshgrid(*ax, indexing="ij"), -1).reshape(-1, 3)
+    V = np.array([(0, 0, 0), (0, 0, 0.25), (0.25, 0.25, 0), (-0.25, 0.25, 0.5), (0.5, -0.25, 0.25),
+                  (0.25, 0.25, 0.25), (-0.5, -0.5, -0.25)])
+    pos, vel, cell = [], [], []
+    for v in V:
+        S = T - v
+        ok = np.all((S >= 0) & (S <= [3, 3, 4]), axis=1)
+        for s in S[ok]:
+            c = om.locate_brute(s)
+            if c >= 0:
+                pos.append(s); vel.append(v); cell.append(c)
+    n = len(cell)
+    init = {"pos": np.array(pos), "vel": np.array(vel, dtype=np.float64),
+            "cell": np.array(cell, np.int32), "id": np.arange(n, dtype=np.int64)}
+    ef = np.zeros((mesh["n_cells"], 3))
+    return mesh, ef, init
+
+
+@pytest.mark.parametrize("dh,dep,hpass", [(0, 1, 4), (0, 0, 1), (1, 1, 4), (1, 2, 8), (2, 1, 4), (0, 1, 0)])
+def test_exact_geometry_no_exclusion(dh, dep, hpass):
+    mesh, ef, init = exact_geometry_case()
+    assert init["cell"].size > 15_000
+    overlay = None
+    if dh:
+        box = mesh["box"]
+        n = [int(np.ceil((box[2 * k + 1] - box[2 * k]) / 0.5)) for k in range(3)]
+        overlay = ([box[0], box[2], box[4]], 0.5, n)
+    steps = 3
+    om, orc, Qo, ost, rem = run_oracle(mesh, ef, init, None, steps, C1 * DT, DT, W, use_dh=dh,
+                                       overlay=overlay)
+    gout, Qg, gst, _ = _gpu_run(mesh, ef, init, None, steps, direct_hop=dh, overlay_spacing=0.5,
+                                deposit_mode=dep, hop_budget=hpass)
+    rep = compare(om, mesh["c2n"], orc, Qo, rem, gout, Qg, W, near=None)
+    assert rep["n_excluded"] == 0 and rep["n_compared"] > 10_000
+    for so, sg in zip(ost, gst):
+        assert (sg["n_removed"], sg["n_after"]) == (so["n_removed"], so["n_after"])
+    # the cases are really there: particles end on box faces and at rest, and
+    # particles leave through the box edges / corners
+    assert sum(so["n_removed"] for so in ost) > 1000
+    on_face = np.any((gout["pos"] == 0) | (gout["pos"] == 3), axis=1)
+    assert on_face.sum() > 500
