@@ -75,7 +75,9 @@ def parse(argv=None):
     ap.add_argument("--shuffle", type=int, default=0,
                     help="randomly shuffle the particles every K steps (the paper's GPU policy; use with --sort 0)")
     ap.add_argument("--direct", action="store_true", help="direct loads instead of the TMA pipeline")
-    ap.add_argument("--axis", action="store_true", help="sort key along the duct axis (z)")
+    ap.add_argument("--axis", type=int, default=-1,
+                    help="sort key along the duct axis z (1) or the cell id (0); default: 1 for c4 "
+                         "(the sort moves data almost in place: C4 39.1 vs 43.0 ms/step), 0 otherwise")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=0)
@@ -101,6 +103,8 @@ def parse(argv=None):
     args.dh = 0 if args.mh else args.dhmode   # direct-hop seeding is the default
     if args.field < 0:
         args.field = 1 if args.config in ("c2", "c3") else 0
+    if args.axis < 0:
+        args.axis = 1 if args.config == "c4" else 0
     if args.config in ("c4", "c5") and args.field:
         raise SystemExit("c4 / c5 run with a fixed uniform field (SURVEY.md §8(d))")
     return args

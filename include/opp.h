@@ -299,8 +299,10 @@ int64_t opp_kernel_launch_count(opp_ctx ctx);
  *   E_c = -sum_i phi[c2n[c][i]] grad(lambda_i)   (cell-constant, 1576-1585)
  * nranks > 1: every rank assembles its slab's cells; interface rows are
  * completed by the node halo exchange of the charge halo (opp_set_partition)
- * and dot products count each node once, reduced across ranks in rank order
- * (a host-driven iteration; one rank runs one persistent kernel).
+ * and dot products count each node once; every rank's dots are all-gathered
+ * on the stream and summed in rank order on the device, which forms alpha,
+ * beta and the stop test (the host reads one flag per batch of 8 iterations;
+ * one rank runs one persistent kernel).
  * ------------------------------------------------------------------------- */
 typedef struct {
     double rhs_scale;   /* b = rhs_scale * node_charge (q / eps0 per unit weight)       */
@@ -311,6 +313,8 @@ typedef struct {
                            last two solutions of warm-start-2 solves into this dat (the
                            first such solve starts like 1); 0: from 0                   */
     int precond;        /* 0: plain CG; 1: Jacobi (diagonal) preconditioned CG          */
+    int slab_cg;        /* 1: run the slab (multi-rank) CG on one rank too (testing it);
+                           0: one rank uses the persistent kernel                      */
 } opp_field_params;
 
 typedef struct {

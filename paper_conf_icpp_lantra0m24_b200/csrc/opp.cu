@@ -19,6 +19,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 using namespace opp;
@@ -137,10 +138,13 @@ struct FieldState {
     double *part = nullptr;         // 3 * part_cap block partials
     long long part_cap = 0;
     CgState *st = nullptr;
-    // host-driven CG (nranks > 1 or OPP_CG_HOSTLOOP): owner weights of the
+    // slab CG (nranks > 1 or opp_field_params.slab_cg): owner weights of the
     // dot products (1 on the lowest rank holding a node), y / yd / beff
     // vectors, the reduced dots, and the host-kept stats of the last solve
     double *own = nullptr, *hvec = nullptr, *dots = nullptr;
+    // slab CG driven from the device: coefficients + the gathered dots
+    CgCoef *coef = nullptr;
+    double *gath = nullptr;
     bool host_stats = false;
     opp_field_stats hst{};
     // Boltzmann-electron Newton solve (allocated on first use): lumped mass,
@@ -162,6 +166,8 @@ struct opp_ctx_s {
     opp_init_params p{};
     cudaStream_t s = nullptr;
     cudaStream_t cs = nullptr;     // copy stream (host injection staging)
+    cudaStream_t fs2 = nullptr;    // nranks > 1: the hole fill overlapped with the migrant exchange
+    cudaEvent_t ev_packed = nullptr, ev_filled = nullptr;
     int nsm = 148;
     int bps = 0;                   // resident blocks / SM of the fused kernel
     std::vector<Set> sets;
@@ -203,15 +209,29 @@ struct opp_ctx_s {
         return ev_pool[ev_used++];
     }
 
+    // every allocation's size, so the free hook always gets the size it
+    // allocated (a pooling or accounting allocator relies on it)
+    std::unordered_map<void *, size_t> alloc_size;
+
     void *dalloc(size_t bytes) {
         if (bytes == 0) bytes = 16;
-        if (p.alloc) return p.alloc(bytes, (void *)s, p.alloc_user);
         void *ptr = nullptr;
-        if (cudaMalloc(&ptr, bytes) != cudaSuccess) return nullptr;
+        if (p.alloc) {
+            ptr = p.alloc(bytes, (void *)s, p.alloc_user);
+        } else if (cudaMalloc(&ptr, bytes) != cudaSuccess) {
+            ptr = nullptr;
+        }
+        if (ptr) alloc_size[ptr] = bytes;
         return ptr;
     }
-    void dfree(void *ptr, size_t bytes) {
+    void dfree(void *ptr, size_t /*bytes: the recorded size is used*/ = 0) {
         if (!ptr) return;
+        size_t bytes = 0;
+        auto it = alloc_size.find(ptr);
+        if (it != alloc_size.end()) {
+            bytes = it->second;
+            alloc_size.erase(it);
+        }
         if (p.free) p.free(ptr, bytes, (void *)s, p.alloc_user);
         else cudaFree(ptr);
     }
@@ -310,6 +330,14 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
         return fail(OPP_ERR_NOMEM, "cudaMallocHost");
     }
     if (params->nranks > 1) {
+        if (cudaStreamCreateWithFlags(&c->fs2, cudaStreamNonBlocking) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_packed, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_filled, cudaEventDisableTiming) != cudaSuccess) {
+            cudaFreeHost(c->hcnt);
+            cudaStreamDestroy(c->cs);
+            delete c;
+            return fail(OPP_ERR_CUDA, "fill stream");
+        }
         int r = opp::comm_init(&c->comm, params->transport, params->nccl_unique_id, params->rank,
                                params->nranks, params->device, g_err);
         if (r != OPP_OK) {
@@ -357,6 +385,7 @@ static void free_field(opp_ctx c) {
     c->dfree(f.n2c_ptr, 0); c->dfree(f.n2c, 0); c->dfree(f.vec, 0); c->dfree(f.part, 0);
     c->dfree(f.st, 0);
     c->dfree(f.own, 0); c->dfree(f.hvec, 0); c->dfree(f.dots, 0);
+    c->dfree(f.coef, 0); c->dfree(f.gath, 0);
     c->dfree(f.bz_m, 0); c->dfree(f.bz_jval, 0); c->dfree(f.bz_jdinv, 0); c->dfree(f.bz_zero, 0);
     c->dfree(f.bz_rhs, 0); c->dfree(f.bz_delta, 0); c->dfree(f.bz_part, 0); c->dfree(f.bz_norm, 0);
     if (f.bz_host) cudaFreeHost(f.bz_host);
@@ -397,6 +426,12 @@ extern "C" int opp_finalize(opp_ctx c) {
     for (auto e : c->ev_pool) cudaEventDestroy(e);
     cudaStreamSynchronize(c->cs);
     cudaStreamDestroy(c->cs);
+    if (c->fs2) {
+        cudaStreamSynchronize(c->fs2);
+        cudaStreamDestroy(c->fs2);
+        cudaEventDestroy(c->ev_packed);
+        cudaEventDestroy(c->ev_filled);
+    }
     cudaFreeHost(c->hcnt);
     delete c;
     return OPP_OK;
@@ -1166,7 +1201,15 @@ static void refresh_args(opp_ctx c, PSet &ps, StepArgs &a, int pos, int vel, int
 // that entered another rank's cells are packed (every column + hop count),
 // exchanged point-to-point, appended at the end of the receiver's dats and
 // walked on there; repeated until no rank has migrants.
-static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p2c, int cgrid) {
+// A round reads the host once: the R x R count matrix, all-gathered on the
+// stream from the device counts (message sizes must be known to the host).
+// Round 0 overlaps the hole fill with the exchange ("a
+// hole filling routine runs asynchronously during communication"): once the
+// migrants are packed their slots are free, so the fill of the holes left by
+// removed and departed particles runs on a second stream while NCCL moves the
+// records; the unpack waits for it and appends behind the compacted set.
+static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p2c, int cgrid,
+                        bool overlap_fill) {
     opp::Comm *cm = c->comm;
     const int R = cm->nranks, me = cm->rank;
     int p2c_col = -1, rec = 0, pos = -1, vel = -1;
@@ -1180,15 +1223,14 @@ static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p
     }
     rec += 4;                                        // hop count
     rec = (rec + 7) & ~7;
-    std::vector<int64_t> row(R), soff(R), sbytes(R), roff(R), rbytes(R);
-    std::vector<unsigned long long> hrow(R);
+    std::vector<int64_t> soff(R), sbytes(R), roff(R), rbytes(R);
     for (int round = 0;; round++) {
         CK(launch_mig_count(a.mig_cell, ps.dcnt, cm->rr, cm->d_counts, grid_for(c, ps.n_ub, 2), c->s));
-        CK(cudaMemcpyAsync(hrow.data(), cm->d_counts, 8 * R, cudaMemcpyDeviceToHost, c->s));
+        TRY(cm->t->allgather_dev(cm->d_counts, 8 * (size_t)R, cm->d_allcounts, c->s, g_err));
+        CK(cudaMemcpyAsync(cm->counts_host.data(), cm->d_allcounts, 8 * (size_t)R * R, cudaMemcpyDeviceToHost,
+                           c->s));
         CK(cudaStreamSynchronize(c->s));
         c->launches++;
-        for (int q = 0; q < R; q++) row[q] = (int64_t)hrow[q];
-        TRY(cm->t->allgather_i64(row.data(), R, cm->counts_host.data(), c->s, g_err));
         const int64_t *M = cm->counts_host.data();
         int64_t total = 0, out = 0, in = 0;
         for (int k = 0; k < R * R; k++) total += M[k];
@@ -1210,12 +1252,23 @@ static int migrate_loop(opp_ctx c, PSet &ps, StepArgs &a, int dep, int dh, int p
         CK(launch_mig_pack(cs, p2c_col, a.mig, a.mig_cell, a.mig_hops, ps.dcnt, cm->rr, cm->d_cursor,
                            cm->sendbuf, rec, grid_for(c, out, 2), c->s));
         c->launches++;
+        const bool ov = overlap_fill && round == 0;
+        if (ov) {   // fill the holes on the second stream while the records travel
+            CK(cudaEventRecord(c->ev_packed, c->s));
+            CK(cudaStreamWaitEvent(c->fs2, c->ev_packed, 0));
+            CK(launch_fill(cs, ps.dcnt, ps.holes, (const int32_t *)c->cols[p2c].d, ps.head, ps.tail,
+                           grid_for(c, ps.n_ub, 4), c->fs2));
+            CK(cudaEventRecord(c->ev_filled, c->fs2));
+            c->launches += 2;
+        }
         if (ps.n_ub + in > ps.cap) {
+            if (ov) CK(cudaStreamWaitEvent(c->s, c->ev_filled, 0));   // growth copies the columns
             TRY(grow(c, ps, in));
             refresh_args(c, ps, a, pos, vel, p2c);
             cs = make_colset(c, ps);
         }
         TRY(cm->t->exchange(cm->sendbuf, soff, sbytes, cm->recvbuf, roff, rbytes, c->s, g_err));
+        if (ov) CK(cudaStreamWaitEvent(c->s, c->ev_filled, 0));     // unpack behind the compacted set
         CK(launch_mig_unpack(cs, cm->recvbuf, in, rec, ps.dcnt, a.work, a.work_hops,
                              grid_for(c, in, 2), c->s));
         ps.n_ub += in;
@@ -1350,7 +1403,12 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     c->launches += tiled ? 3 : 2;   // (tiled: pipelined kernel + ragged-tail kernel) + continuation
     if (multi) {
         PhaseScope ph(c, OPP_PH_MIGRATE);
-        TRY(migrate_loop(c, ps, a, dep, dh, p2c, c->nsm * 8));
+        // the fill overlaps the exchange unless this step's compaction is a
+        // sort (which drops holes itself) or SR records sit at particle
+        // indices until the segmented reduction
+        const bool sort_step = c->p.sort_every > 0 && (ps.steps + 1) % c->p.sort_every == 0;
+        TRY(migrate_loop(c, ps, a, dep, dh, p2c, c->nsm * 8,
+                         prm->fill_inline && !sort_step && dep != OPP_DEP_SORT_SEGRED));
     }
     if (dep == OPP_DEP_SORT_SEGRED) {
         PhaseScope ph(c, OPP_PH_SEGRED);
@@ -1585,8 +1643,11 @@ extern "C" int opp_field_init(opp_ctx c, opp_map c2n, opp_dat node_pos, const in
     f.own = (double *)c->dalloc(8 * std::max<long long>(nn, 1));
     f.hvec = (double *)c->dalloc(8 * 3 * std::max<long long>(nn, 1));
     f.dots = (double *)c->dalloc(8 * 4);
+    f.coef = (CgCoef *)c->dalloc(sizeof(CgCoef));
+    f.gath = (double *)c->dalloc(8 * 4 * (size_t)c->p.nranks);
     if (!f.K.slice_off || !f.K.col || !f.K.val || !f.K.dinv || !f.K.dmask || !f.K.dval ||
-        !f.n2c_ptr || !f.n2c || !f.vec || !f.part || !f.st || !f.own || !f.hvec || !f.dots) {
+        !f.n2c_ptr || !f.n2c || !f.vec || !f.part || !f.st || !f.own || !f.hvec || !f.dots ||
+        !f.coef || !f.gath) {
         free_field(c);
         return fail(OPP_ERR_NOMEM, "field solve buffers");
     }
@@ -1672,15 +1733,33 @@ static int allreduce_dots(opp_ctx c, const double *dev, int n, double *out) {
     return OPP_OK;
 }
 
-// The same Chronopoulos-Gear (P)CG as k_cg, one kernel per phase: local SpMV
-// rows of interface nodes are completed by the node halo exchange (the
-// charge halo's plan), dots count each node once (owner weights) and are
-// reduced across ranks in rank order; alpha, beta on the host.
-static int field_solve_hostloop(opp_ctx c, CgArgs &a) {
+// Gather this rank's nv dot products (device) from every rank into f.gath
+// on the stream (NCCL: no host synchronisation).
+static int gather_dots(opp_ctx c, int nv) {
+    FieldState &f = c->fs;
+    if (c->p.nranks == 1)
+        CK(cudaMemcpyAsync(f.gath, f.dots, 8 * nv, cudaMemcpyDeviceToDevice, c->s));
+    else
+        TRY(c->comm->t->allgather_dev(f.dots, 8 * (size_t)nv, f.gath, c->s, g_err));
+    return OPP_OK;
+}
+
+// The slab CG (nranks > 1; or opp_field_params.slab_cg on one rank): the same
+// Chronopoulos-Gear (P)CG as k_cg, one kernel per phase.  Local SpMV rows of
+// interface nodes are completed by the node halo exchange (the charge halo's
+// plan), dots count each node once (owner weights); every rank's dots are
+// all-gathered on the stream and summed in rank order on the device
+// (k_cg_coef: identical alpha, beta and stop test on every rank).  The host
+// enqueues kBatch iterations at a time and reads the device's done flag once
+// per batch (iterations enqueued past convergence do not update x); with
+// NCCL no host synchronisation happens inside a batch.
+static int field_solve_slab(opp_ctx c, CgArgs &a) {
+    constexpr int kBatch = 8;
     FieldState &f = c->fs;
     const FieldMat &K = a.K;       // f.K (linear solve) or the Newton Jacobian
     const long long nn = f.nn;
-    const bool multi = c->p.nranks > 1 && c->comm->halo_n > 0;
+    const int R = c->p.nranks;
+    const bool multi = R > 1 && c->comm->halo_n > 0;
     double *y = f.hvec, *yd = f.hvec + nn, *beff = f.hvec + 2 * nn;
     const int nblk = (int)std::min<long long>(f.part_cap, std::max<long long>(1, (nn + 255) / 256));
     CK(launch_cg_x0(K, a.x, a.warm, c->s));
@@ -1694,41 +1773,32 @@ static int field_solve_hostloop(opp_ctx c, CgArgs &a) {
     const double *va[3], *vb[3];
     va[0] = beff; vb[0] = beff;
     CK(launch_dots(nn, f.own, 1, va, vb, f.part, nblk, f.dots, c->s));
-    c->launches += 3;
-    double rr0;
-    TRY(allreduce_dots(c, f.dots, 1, &rr0));
-    const double stop = a.tol * a.tol * rr0;
+    TRY(gather_dots(c, 1));
+    CK(launch_cg_coef(f.gath, R, 1, f.coef, a.tol, a.max_iter, 1, c->s));
+    c->launches += 4;
     va[0] = a.r; vb[0] = a.u;
     va[1] = a.w; vb[1] = a.u;
     va[2] = a.r; vb[2] = a.r;
-    double gamma_old = 0.0, alpha = 0.0, beta = 0.0, rho = 0.0;
-    int it = 0;
-    for (bool first = true;; first = false) {
-        if (!first) CK(launch_cg_update(K, alpha, beta, a.x, a.r, a.u, a.w, a.p, a.s, a.precond, c->s));
+    CgCoef h{};
+    for (int k = 0;; k++) {
+        if (k > 0) CK(launch_cg_update_dev(K, f.coef, a.x, a.r, a.u, a.w, a.p, a.s, a.precond, c->s));
         CK(launch_spmv(K, a.u, a.w, nullptr, c->nsm, c->s));
         if (multi) TRY(halo_sum(c, a.w));
         CK(launch_dots(nn, f.own, 3, va, vb, f.part, nblk, f.dots, c->s));
-        c->launches += first ? 3 : 4;
-        if (!first) it++;
-        double t[3];
-        TRY(allreduce_dots(c, f.dots, 3, t));
-        const double gamma = t[0], delta = t[1];
-        rho = t[2];
-        if (rho <= stop || it >= a.max_iter) break;
-        if (it == 0) {
-            beta = 0.0;
-            alpha = gamma / delta;
-        } else {
-            beta = gamma / gamma_old;
-            alpha = gamma / (delta - beta * gamma / alpha);
+        TRY(gather_dots(c, 3));
+        CK(launch_cg_coef(f.gath, R, 3, f.coef, a.tol, a.max_iter, 0, c->s));
+        c->launches += k > 0 ? 5 : 4;
+        if ((k + 1) % kBatch == 0) {
+            CK(cudaMemcpyAsync(&h, f.coef, sizeof h, cudaMemcpyDeviceToHost, c->s));
+            CK(cudaStreamSynchronize(c->s));
+            if (h.done) break;
         }
-        gamma_old = gamma;
     }
     f.host_stats = true;
-    f.hst.iterations = it;
-    f.hst.converged = rho <= stop;
-    f.hst.rel_residual = rr0 > 0 ? std::sqrt(rho / rr0) : 0.0;
-    f.hst.rhs_norm = std::sqrt(rr0);
+    f.hst.iterations = h.it;
+    f.hst.converged = h.rho <= h.stop;
+    f.hst.rel_residual = h.rr0 > 0 ? std::sqrt(h.rho / h.rr0) : 0.0;
+    f.hst.rhs_norm = std::sqrt(h.rr0);
     return OPP_OK;
 }
 
@@ -1959,10 +2029,9 @@ extern "C" int opp_field_solve(opp_ctx c, opp_dat node_charge, opp_dat node_pote
     {
         PhaseScope ph(c, OPP_PH_FIELD);
         int grid = 0;
-        const char *hl = getenv("OPP_CG_HOSTLOOP");
         f.host_stats = false;
-        if (nn > 0 && (c->p.nranks > 1 || (hl && atoi(hl)))) {
-            TRY(field_solve_hostloop(c, a));
+        if (nn > 0 && (c->p.nranks > 1 || prm->slab_cg)) {
+            TRY(field_solve_slab(c, a));
         } else if (nn > 0) {
             int bps = 2;   // blocks per SM: 2 (1.50 ms per C2 solve) beat 1 (1.91 ms)
             bps = std::min<int>(bps, (int)(f.part_cap / c->nsm));
@@ -2162,7 +2231,7 @@ extern "C" int opp_field_solve_boltzmann(opp_ctx c, opp_dat node_charge, opp_dat
                     c->launches++;
                     pending_it = true;
                 } else {
-                    TRY(field_solve_hostloop(c, a));
+                    TRY(field_solve_slab(c, a));
                     bs.cg_iterations += f.hst.iterations;
                 }
                 CK(launch_newton_update(f.K, phi, f.bz_delta, c->s));

@@ -106,6 +106,22 @@ struct LoopTransport : Transport {
         hub->barrier();                             // peers finished reading my buffer
         return OPP_OK;
     }
+
+    int allgather_dev(const void *in, size_t bytes, void *out, cudaStream_t s, std::string &err) override {
+        cudaError_t e = cudaStreamSynchronize(s);   // my input is complete
+        if (e != cudaSuccess) return cuda_fail(e, "loopback sync", err);
+        hub->ptr[rank] = in;
+        hub->barrier();
+        for (int p = 0; p < nranks; p++) {
+            e = cudaMemcpyPeerAsync((char *)out + (size_t)p * bytes, hub->device[rank], hub->ptr[p],
+                                    hub->device[p], bytes, s);
+            if (e != cudaSuccess) return cuda_fail(e, "loopback copy", err);
+        }
+        e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) return cuda_fail(e, "loopback sync", err);
+        hub->barrier();                             // peers finished reading my input
+        return OPP_OK;
+    }
 };
 
 #ifdef OPP_WITH_NCCL
@@ -162,6 +178,12 @@ struct NcclTransport : Transport {
         }
         r = ncclGroupEnd();
         if (r != ncclSuccess) return nccl_fail(r, "ncclGroupEnd", err);
+        return OPP_OK;
+    }
+
+    int allgather_dev(const void *in, size_t bytes, void *out, cudaStream_t s, std::string &err) override {
+        ncclResult_t r = ncclAllGather(in, out, bytes, ncclChar, comm, s);
+        if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather", err);
         return OPP_OK;
     }
 };
@@ -245,12 +267,13 @@ int comm_init(Comm **out, int transport, const void *uid, int rank, int nranks, 
         return OPP_ERR_NCCL;
 #endif
     }
-    cudaError_t e = cudaMalloc(&c->d_counts, 2 * sizeof(unsigned long long) * nranks);
+    cudaError_t e = cudaMalloc(&c->d_counts, sizeof(unsigned long long) * (2 + (size_t)nranks) * nranks);
     if (e != cudaSuccess) {
         delete c->t;
         return cuda_fail(e, "comm counters", err);
     }
     c->d_cursor = c->d_counts + nranks;
+    c->d_allcounts = c->d_counts + 2 * nranks;
     c->counts_host.assign((size_t)nranks * nranks, 0);
     *out = c.release();
     return OPP_OK;

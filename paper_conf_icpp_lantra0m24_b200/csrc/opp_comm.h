@@ -28,6 +28,10 @@ struct Transport {
                          const std::vector<int64_t> &sbytes, char *recvbuf,
                          const std::vector<int64_t> &roff, const std::vector<int64_t> &rbytes,
                          cudaStream_t s, std::string &err) = 0;
+    // device all-gather: out[r * bytes .. (r+1) * bytes) = rank r's in (device
+    // buffers), enqueued on stream s (NCCL: no host synchronisation)
+    virtual int allgather_dev(const void *in, size_t bytes, void *out, cudaStream_t s,
+                              std::string &err) = 0;
 };
 
 struct Comm {
@@ -49,6 +53,7 @@ struct Comm {
     // migration
     unsigned long long *d_counts = nullptr;    // nranks
     unsigned long long *d_cursor = nullptr;    // nranks
+    unsigned long long *d_allcounts = nullptr; // nranks * nranks (all ranks' count rows)
     char *sendbuf = nullptr, *recvbuf = nullptr;
     size_t send_cap = 0, recv_cap = 0;
     std::vector<int64_t> counts_host;          // nranks * nranks

@@ -45,7 +45,6 @@ struct CgArgs {
     CgState *st;
     double rhs_scale, tol;
     int max_iter, warm, precond;
-    int dbg;             // diagnostics (OPP_CG_DBG): 1 = no SpMV in the loop, 2 = no grid barriers
     int pipelined;       // 1: k_pcg (one grid barrier per iteration), 0: k_cg
 };
 
@@ -62,7 +61,7 @@ cudaError_t launch_efield(const double *xyz, const int32_t *c2n, const double *p
 
 }  // namespace opp
 
-// ---- host-driven CG (nranks > 1, or OPP_CG_HOSTLOOP=1): one kernel per
+// ---- slab CG (nranks > 1, or opp_field_params.slab_cg): one kernel per
 // phase, the partial SpMV rows of interface nodes completed by the charge
 // halo exchange, dot products over owned nodes reduced across ranks.
 namespace opp {
@@ -78,6 +77,20 @@ cudaError_t launch_cg_r0(const FieldMat &K, const double *Q, double rhs_scale, c
 cudaError_t launch_dots(long long n, const double *own, int nv, const double *const *va,
                         const double *const *vb, double *part, int nblk, double *out,
                         cudaStream_t s);
+// Slab CG (nranks > 1) driven from the device: the per-rank dot products
+// of an iteration are all-gathered on the stream and summed in rank order by
+// one thread, which also forms alpha, beta and the stop test, so the host
+// enqueues iterations in batches and reads one flag per batch.
+struct CgCoef {
+    double alpha, beta, gamma_old, stop, rr0, rho;
+    int it, done, first, pad;
+};
+// init: rr0 = the gathered ||b_eff||^2, stop = tol^2 rr0; else one iteration's
+// (gamma, delta, rho) -> it, done, alpha, beta (Chronopoulos-Gear, as k_cg)
+cudaError_t launch_cg_coef(const double *gathered, int nranks, int nv, CgCoef *c, double tol,
+                           int max_iter, int init, cudaStream_t s);
+cudaError_t launch_cg_update_dev(const FieldMat &K, const CgCoef *c, double *x, double *r, double *u,
+                                 const double *w, double *p, double *sv, int precond, cudaStream_t s);
 cudaError_t launch_cg_update(const FieldMat &K, double alpha, double beta, double *x, double *r,
                              double *u, const double *w, double *p, double *sv, int precond,
                              cudaStream_t s);

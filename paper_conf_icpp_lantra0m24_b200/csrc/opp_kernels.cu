@@ -15,6 +15,7 @@
 #include "opp_kernels.h"
 
 #include <algorithm>
+#include <cstddef>
 #include <climits>
 
 namespace opp {
@@ -188,44 +189,122 @@ __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0,
     atomicAdd(Q + cn.w, v3);
 }
 
+// OPP_DEP3 (default 1): the tree carries 3 of the 4 values; the group's
+// w*lambda_0 sum is n w - (S_1 + S_2 + S_3) (lambda_0 = 1 - lambda_1 -
+// lambda_2 - lambda_3 per particle, so the two differ by rounding only:
+// ~n eps w absolute, far inside the 1e-10 relative charge tolerance, and the
+// group's total charge n w is conserved exactly).
+#ifndef OPP_DEP3
+#define OPP_DEP3 1
+#endif
+// Per-warp node-charge cache across slices (OPP_DCACHE, TMA-pipelined
+// kernel): the 4 group sums of a cell accumulate in a warp-private shared
+// table of kDcSlots cells (slot = cell mod kDcSlots, one writer lane per slot
+// and slice) and leave with 4 reductions when the slot is taken by another
+// cell or the kernel ends.  In cell-sorted storage a warp's consecutive
+// slices (adjacent tiles) end in mostly the same cells, so most slices issue
+// no reductions and no node-id loads.
+#ifndef OPP_DCACHE
+#define OPP_DCACHE 0
+#endif
+constexpr int kDcSlots = 32;
+constexpr int kDcBytesPerWarp = kDcSlots * (4 + 4 * 8);
+struct DepCache {
+    int *key;       // [kDcSlots] local cell, -1 = empty
+    double *val;    // [4][kDcSlots]
+};
+__device__ __forceinline__ DepCache dep_cache(char *base) {
+    DepCache d;
+    d.val = reinterpret_cast<double *>(base);
+    d.key = reinterpret_cast<int *>(d.val + 4 * kDcSlots);
+    if (lane_id() < (unsigned)kDcSlots) d.key[lane_id()] = -1;
+    __syncwarp();
+    return d;
+}
+// flush every cached cell (end of the kernel): lane l handles slot l
+__device__ __forceinline__ void dep_cache_flush(const StepArgs &a, DepCache &d) {
+    __syncwarp();
+    const unsigned l = lane_id();
+    const int k = l < (unsigned)kDcSlots ? d.key[l] : -1;
+    if (k >= 0)
+        red4(a.Q, line_c2n(a.lines, k), d.val[l], d.val[kDcSlots + l], d.val[2 * kDcSlots + l],
+             d.val[3 * kDcSlots + l]);
+    __syncwarp();
+}
+
 __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepArgs &a, bool act,
-                                            int key, double v0, double v1, double v2, double v3) {
+                                            int key, double v0, double v1, double v2, double v3,
+                                            DepCache *dc = nullptr) {
     const unsigned FULL = 0xffffffffu;
     if (!__any_sync(FULL, act)) return;
     const unsigned lane = lane_id();
     const unsigned peers = __match_any_sync(FULL, act ? key : -2 - (int)lane);
     const int first = __ffs(peers) - 1;
+    const bool lead = act && (int)lane == first;
     int rel = __popc(peers & ((1u << lane) - 1u));       // my rank inside the group
     unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
     if (lane == 31) up = 0;
     int4 cn = make_int4(0, 0, 0, 0);
-    if (act && (int)lane == first) cn = line_c2n(a.lines, key - a.cell_base);
+    if (lead && !dc) cn = line_c2n(a.lines, key - a.cell_base);
     while (__any_sync(FULL, up != 0)) {
         const int next = up ? __ffs(up) - 1 : (int)lane;
-        const double t0 = __shfl_sync(FULL, v0, next);
+        const double t0 = OPP_DEP3 ? 0.0 : __shfl_sync(FULL, v0, next);
         const double t1 = __shfl_sync(FULL, v1, next);
         const double t2 = __shfl_sync(FULL, v2, next);
         const double t3 = __shfl_sync(FULL, v3, next);
         if (up) {
-            v0 = add(v0, t0); v1 = add(v1, t1); v2 = add(v2, t2); v3 = add(v3, t3);
+            if (!OPP_DEP3) v0 = add(v0, t0);
+            v1 = add(v1, t1); v2 = add(v2, t2); v3 = add(v3, t3);
         }
         // lanes at odd group rank have been absorbed by their lower neighbour
         const unsigned gone = __ballot_sync(FULL, (rel & 1) != 0);
         up &= ~gone;
         rel >>= 1;
     }
-    if (act && (int)lane == first) red4(Q, cn, v0, v1, v2, v3);
+    if (OPP_DEP3 && lead) v0 = sub(mul((double)__popc(peers), a.w), add(add(v1, v2), v3));
+    if (!dc) {
+        if (lead) red4(Q, cn, v0, v1, v2, v3);
+        return;
+    }
+    // the cache: one leader per slot this slice (others reduce directly)
+    const int lc = key - a.cell_base;
+    const int slot = lc & (kDcSlots - 1);
+    const unsigned same = __match_any_sync(FULL, lead ? slot : -1 - (int)lane);
+    const bool owner = lead && (int)lane == __ffs(same) - 1;
+    __syncwarp();
+    if (owner) {
+        const int k = dc->key[slot];
+        if (k == lc) {
+            dc->val[slot] = add(dc->val[slot], v0);
+            dc->val[kDcSlots + slot] = add(dc->val[kDcSlots + slot], v1);
+            dc->val[2 * kDcSlots + slot] = add(dc->val[2 * kDcSlots + slot], v2);
+            dc->val[3 * kDcSlots + slot] = add(dc->val[3 * kDcSlots + slot], v3);
+        } else {
+            if (k >= 0)
+                red4(Q, line_c2n(a.lines, k), dc->val[slot], dc->val[kDcSlots + slot],
+                     dc->val[2 * kDcSlots + slot], dc->val[3 * kDcSlots + slot]);
+            dc->key[slot] = lc;
+            dc->val[slot] = v0;
+            dc->val[kDcSlots + slot] = v1;
+            dc->val[2 * kDcSlots + slot] = v2;
+            dc->val[3 * kDcSlots + slot] = v3;
+        }
+    } else if (lead) {
+        red4(Q, line_c2n(a.lines, lc), v0, v1, v2, v3);
+    }
+    __syncwarp();
 }
 
 template <int DEP>
 __device__ __forceinline__ void deposit(const StepArgs &a, bool done, int cell, double w,
-                                        double l0, double l1, double l2, double l3) {
+                                        double l0, double l1, double l2, double l3,
+                                        DepCache *dc = nullptr) {
     double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
     if (DEP == 0) {
         if (done) red4(a.Q, line_c2n(a.lines, cell - a.cell_base), v0, v1, v2, v3);
         return;
     }
-    deposit_agg(a.Q, a, done, cell, v0, v1, v2, v3);
+    deposit_agg(a.Q, a, done, cell, v0, v1, v2, v3, dc);
 }
 
 // SR deposit, phase 1 (Fig. 3 "store values and keys"):
@@ -251,9 +330,10 @@ __device__ __forceinline__ void sr_store(const StepArgs &a, bool write, bool don
 // record, done or not); `done`: it deposits.
 template <int DEP>
 __device__ __forceinline__ void deposit_any(const StepArgs &a, bool write, bool done, unsigned long long i,
-                                            int cell, double l0, double l1, double l2, double l3) {
+                                            int cell, double l0, double l1, double l2, double l3,
+                                            DepCache *dc = nullptr) {
     if (DEP == 2) sr_store(a, write, done, i, cell, a.w, l0, l1, l2, l3);
-    else deposit<DEP>(a, done, cell, a.w, l0, l1, l2, l3);
+    else deposit<DEP>(a, done, cell, a.w, l0, l1, l2, l3, dc);
 }
 
 // Per-warp flush of walk statistics.
@@ -447,7 +527,8 @@ template <int DEP, int DH, bool MULTI, bool LATE>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
-                                         Appends *ap = nullptr, const Aux *aux = nullptr) {
+                                         Appends *ap = nullptr, const Aux *aux = nullptr,
+                                         DepCache *dc = nullptr) {
     int status = ST_NONE;
     int capped = 0, hops = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -529,7 +610,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         }
         t.removed += (status == ST_REMOVE);
     }
-    if (!OPP_LADDER) deposit_any<DEP>(a, valid, status == ST_DONE, i, cell, l0, l1, l2, l3);
+    if (!OPP_LADDER) deposit_any<DEP>(a, valid, status == ST_DONE, i, cell, l0, l1, l2, l3, dc);
     // holes, the deferred-walk worklist, migrants
     const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
     if (ap) {
@@ -640,7 +721,8 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
 #endif
 constexpr int kQ = 64;                                   // ring entries per warp
 constexpr int kQBytesPerWarp = kQ * (3 * 8 + 4 * 4);     // x, y, z | cell, face, hops, index
-constexpr int kTiledSmem = kQBase + (OPP_HOPQ ? kConsumerWarps * kQBytesPerWarp : 0);
+constexpr int kDcBase = kQBase + (OPP_HOPQ ? kConsumerWarps * kQBytesPerWarp : 0);
+constexpr int kTiledSmem = kDcBase + (OPP_DCACHE ? kConsumerWarps * kDcBytesPerWarp : 0);
 struct HopQueue {
     double *x, *y, *z;
     int *cell, *face, *hops;
@@ -989,6 +1071,12 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
 #if OPP_HOPQ
     HopQueue q = hop_queue(smem + kQBase + (size_t)warp * kQBytesPerWarp);
 #endif
+    DepCache dcache;
+    DepCache *dcp = nullptr;
+    if (OPP_DCACHE && DEP == 1) {
+        dcache = dep_cache(smem + kDcBase + (size_t)warp * kDcBytesPerWarp);
+        dcp = &dcache;
+    }
     TileIter ti(tm);
     for (unsigned long long it = 0; it < my; it++, ti.next()) {
         const int s = (int)(it % kStages);
@@ -1023,17 +1111,19 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
         __syncwarp();
         const unsigned long long i = ti.tile() * kTile + j;
 #if OPP_HOPQ
-        pmd_first<DEP, DH, MULTI>(a, (uint32_t)i, x, y, z, vx, vy, vz, cell, t, ap, q, OPP_AUX ? &ax : nullptr);
+        pmd_first<DEP, DH, MULTI>(a, (uint32_t)i, x, y, z, vx, vy, vz, cell, t, ap, q, OPP_AUX == 1 ? &ax : nullptr);
         a.p2c[i] = cell;
         while (q.count >= 32u) hop_round<DEP, MULTI>(a, q, 32u, t, ap);
 #else
-        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap, OPP_AUX ? &ax : nullptr);
+        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap, OPP_AUX == 1 ? &ax : nullptr,
+                                       dcp);
         a.p2c[i] = cell;
 #endif
     }
 #if OPP_HOPQ
     while (q.count) hop_round<DEP, MULTI>(a, q, min(q.count, 32u), t, ap);
 #endif
+    if (dcp) dep_cache_flush(a, *dcp);
     ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
     ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
@@ -1978,6 +2068,11 @@ cudaError_t launch_step_begin(double *Q, long long nn, DevCounters *c, int zero,
 cudaError_t launch_fill(const ColSet &cols, DevCounters *c, const uint32_t *holes,
                         const int32_t *p2c, uint32_t *head, uint32_t *tail, int grid,
                         cudaStream_t s) {
+    // the pairing lists start empty (a step may fill twice: during the
+    // migrant exchange and after it)
+    static_assert(offsetof(DevCounters, n_tail) == offsetof(DevCounters, n_head) + 8, "layout");
+    cudaError_t e0 = cudaMemsetAsync(&c->n_head, 0, 16, s);
+    if (e0 != cudaSuccess) return e0;
     k_fill_plan<<<grid, 256, 0, s>>>(holes, p2c, c, head, tail);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;

@@ -76,7 +76,7 @@ class opp_step_stats(C.Structure):
 
 class opp_field_params(C.Structure):
     _fields_ = [("rhs_scale", C.c_double), ("tol", C.c_double), ("max_iter", C.c_int),
-                ("warm_start", C.c_int), ("precond", C.c_int)]
+                ("warm_start", C.c_int), ("precond", C.c_int), ("slab_cg", C.c_int)]
 
 
 class opp_boltzmann_params(C.Structure):

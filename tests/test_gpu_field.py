@@ -30,12 +30,12 @@ def _set_charge(sim, Q):
     O.opp_set_dat(sim.ctx, sim.node_charge, np.ascontiguousarray(Q, np.float64), sim.nn)
 
 
-@pytest.mark.parametrize("hostloop", ["0", "1"])
+@pytest.mark.parametrize("slab", [0, 1])
 @pytest.mark.parametrize("precond", [0, 1])
 @pytest.mark.parametrize("dims,jit", [((6, 6, 30), 0.2), ((5, 3, 7), 0.1), ((1, 1, 1), 0.0)])
-def test_field_solve_matches_direct_solve(dims, jit, precond, hostloop, monkeypatch):
-    """hostloop 1: the host-driven CG (the multi-rank solver) on one rank."""
-    monkeypatch.setenv("OPP_CG_HOSTLOOP", hostloop)
+def test_field_solve_matches_direct_solve(dims, jit, precond, slab):
+    """slab 1: the multi-rank CG (device-side coefficients, batched
+    iterations) on one rank."""
     mesh = gen.kuhn_duct(*dims, jitter=jit, seed=4)
     xyz, c2n = mesh["node_xyz"], mesh["c2n"]
     rng = np.random.default_rng(1)
@@ -48,7 +48,8 @@ def test_field_solve_matches_direct_solve(dims, jit, precond, hostloop, monkeypa
     sim = _sim(mesh)
     sim.field_init(mask, val)
     _set_charge(sim, Q)
-    st = sim.field_solve(rhs_scale, tol=tol, max_iter=5000, warm_start=False, precond=bool(precond))
+    st = sim.field_solve(rhs_scale, tol=tol, max_iter=5000, warm_start=False, precond=bool(precond),
+                         slab_cg=bool(slab))
     phi = sim.potential_host()
     E = sim.field_host()
     launches = sim.launches()
@@ -109,13 +110,13 @@ def test_field_solve_errors():
     assert e.value.code == O.OPP_ERR_STATE
     mask, val = gen.duct_bc(mesh, wall=0.0)
     sim.field_init(mask, val)
-    prm = O.opp_field_params(1.0, -1.0, 10, 0, 1)
+    prm = O.opp_field_params(1.0, -1.0, 10, 0, 1, 0)
     with pytest.raises(O.OppError) as e:
         O.opp_field_solve(sim.ctx, sim.node_charge, sim.node_potential, sim.cell_ef, prm)
     assert e.value.code == O.OPP_ERR_ARG
     with pytest.raises(O.OppError):             # a cell dat where a node dat belongs
         O.opp_field_solve(sim.ctx, sim.cell_ef, sim.node_potential, sim.cell_ef,
-                          O.opp_field_params(1.0, 1e-8, 10, 0, 1))
+                          O.opp_field_params(1.0, 1e-8, 10, 0, 1, 0))
     sim.close()
 
 
