@@ -64,6 +64,8 @@ def parse(argv=None):
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count (per rank)")
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
+    ap.add_argument("--deposit-cache", type=int, default=0,
+                    help="warp-aggregated deposit through the per-warp node-charge cache (1)")
     ap.add_argument("--mh", action="store_true", help="multi-hop only (no direct-hop seeding)")
     ap.add_argument("--dhmode", type=int, default=1,
                     help="1: overlay seed for every particle; 2: only for particles that left their cell")
@@ -642,6 +644,7 @@ class EsRank:
                               direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
                               sort_every=args.sort, tma_pipeline=not args.direct,
                               sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0),
+                              deposit_cache=bool(args.deposit_cache),
                               torch_alloc=transport == 0, device=stream.device.index, **kw)
         sim = self.sim
         if args.field:
@@ -883,7 +886,8 @@ def run_ours(args, rank, world, mode):
         "data": "synthetic",
         "config": {"workload": name, "mesh_cells_per_rank": nc, "mesh_nodes_per_rank": nn,
                    "particles_seeded_per_rank": cfg["n0"], "inject_per_step": n_inj,
-                   "avg_particles_per_step_per_rank": n_avg, "deposit": DEP_NAMES[args.deposit],
+                   "avg_particles_per_step_per_rank": n_avg,
+                   "deposit": DEP_NAMES[args.deposit] + (" + per-warp cache" if args.deposit_cache else ""),
                    "walk": (f"DH{args.dh}(overlay {args.ov} h)+MH" if args.dh else "MH"),
                    "hop_budget_per_pass": args.hpass,
                    "sort_every": args.sort, "shuffle_every": args.shuffle,

@@ -71,7 +71,8 @@ enum opp_move_status { OPP_MOVE_DONE = 0, OPP_NEED_MOVE = 1, OPP_NEED_REMOVE = 2
  *                before one atomic per distinct node
  * SORT_SEGRED   store (cell, w*lambda[4]) per particle, counting-sort by
  *                cell, reduce per cell, then per node               ("SR")
- * AUTO          library choice (currently ATOMIC)      */
+ * AUTO          library choice by measurement: ATOMIC_WARPAGG (fastest on
+ *               C2, C4 and the clustered C5)                */
 enum opp_deposit_mode { OPP_DEP_ATOMIC = 0, OPP_DEP_ATOMIC_WARPAGG = 1,
                         OPP_DEP_SORT_SEGRED = 2, OPP_DEP_AUTO = 3 };
 
@@ -110,6 +111,12 @@ typedef struct {
                                    used as the sort-by-cell locality key: cells are
                                    ordered by transverse bin, then along the axis;
                                    (0,0,0) = plain cell-id order                    */
+    int deposit_cache;          /* ATOMIC_WARPAGG in the TMA pipeline: 1 = cell sums
+                                   accumulate in a per-warp shared-memory cache
+                                   across slices and leave with 4 reductions when
+                                   evicted -- pays under deposit contention
+                                   (clustered particles, config C5), costs
+                                   otherwise; 0 = off (default)     */
 } opp_init_params;
 
 /* Per-step arguments of opp_push_move_deposit. */

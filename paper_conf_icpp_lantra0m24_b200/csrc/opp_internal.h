@@ -103,6 +103,7 @@ struct StepArgs {
     int cell_base, n_cells;    // global id of local cell 0, local cell count
     int hpass, hcap;
     int tile_group;            // consecutive 256-particle tiles per block visit (>= 1)
+    int dcache;                // per-warp node-charge cache (opp_init_params.deposit_cache)
     Overlay ov;
 };
 

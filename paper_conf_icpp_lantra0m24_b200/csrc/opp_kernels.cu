@@ -189,25 +189,15 @@ __device__ __forceinline__ void red4(double *__restrict__ Q, int4 cn, double v0,
     atomicAdd(Q + cn.w, v3);
 }
 
-// OPP_DEP3 (default 1): the tree carries 3 of the 4 values; the group's
-// w*lambda_0 sum is n w - (S_1 + S_2 + S_3) (lambda_0 = 1 - lambda_1 -
-// lambda_2 - lambda_3 per particle, so the two differ by rounding only:
-// ~n eps w absolute, far inside the 1e-10 relative charge tolerance, and the
-// group's total charge n w is conserved exactly).
-#ifndef OPP_DEP3
-#define OPP_DEP3 1
-#endif
-// Per-warp node-charge cache across slices (OPP_DCACHE, TMA-pipelined
-// kernel): the 4 group sums of a cell accumulate in a warp-private shared
-// table of kDcSlots cells (slot = cell mod kDcSlots, one writer lane per slot
-// and slice) and leave with 4 reductions when the slot is taken by another
-// cell or the kernel ends.  In cell-sorted storage a warp's consecutive
-// slices (adjacent tiles) end in mostly the same cells, so most slices issue
-// no reductions and no node-id loads.
-#ifndef OPP_DCACHE
-#define OPP_DCACHE 0
-#endif
-constexpr int kDcSlots = 32;
+// Per-warp node-charge cache across slices (opp_init_params.deposit_cache,
+// TMA-pipelined kernel): the group sums of a cell accumulate in a
+// warp-private shared table of kDcSlots cells (multiplicative hash of the
+// cell, one writer lane per slot and slice) and leave with 4 reductions when
+// the slot is taken by another cell or the kernel ends.  Pays when many
+// particles per warp share cells across slices under contention (C5: pass 1
+// 2.58 -> 1.94 ms), costs otherwise (C4 30.8 -> 32.9 ms): off by default.
+constexpr int kDcLog2 = 5;
+constexpr int kDcSlots = 1 << kDcLog2;
 constexpr int kDcBytesPerWarp = kDcSlots * (4 + 4 * 8);
 struct DepCache {
     int *key;       // [kDcSlots] local cell, -1 = empty
@@ -248,12 +238,10 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepAr
     if (lead && !dc) cn = line_c2n(a.lines, key - a.cell_base);
     while (__any_sync(FULL, up != 0)) {
         const int next = up ? __ffs(up) - 1 : (int)lane;
-        const double t0 = OPP_DEP3 ? 0.0 : __shfl_sync(FULL, v0, next);
         const double t1 = __shfl_sync(FULL, v1, next);
         const double t2 = __shfl_sync(FULL, v2, next);
         const double t3 = __shfl_sync(FULL, v3, next);
         if (up) {
-            if (!OPP_DEP3) v0 = add(v0, t0);
             v1 = add(v1, t1); v2 = add(v2, t2); v3 = add(v3, t3);
         }
         // lanes at odd group rank have been absorbed by their lower neighbour
@@ -261,14 +249,21 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepAr
         up &= ~gone;
         rel >>= 1;
     }
-    if (OPP_DEP3 && lead) v0 = sub(mul((double)__popc(peers), a.w), add(add(v1, v2), v3));
+    // the tree carries lambda_1..3; the group's w lambda_0 sum is n w - (S_1 +
+    // S_2 + S_3) (lambda_0 = 1 - lambda_1 - lambda_2 - lambda_3 per particle,
+    // so the two differ by rounding only: ~n eps w absolute, far inside the
+    // 1e-10 relative charge tolerance; the group's charge n w is conserved
+    // exactly; C4 pass 1 30.95 -> 30.74 ms)
+    if (lead) v0 = sub(mul((double)__popc(peers), a.w), add(add(v1, v2), v3));
     if (!dc) {
         if (lead) red4(Q, cn, v0, v1, v2, v3);
         return;
     }
     // the cache: one leader per slot this slice (others reduce directly)
     const int lc = key - a.cell_base;
-    const int slot = lc & (kDcSlots - 1);
+    // multiplicative hash: cell ids of a Kuhn duct differ by 6, 6 nx, 6 nx ny
+    // between neighbours, which a plain "id mod 32" maps onto the same slot
+    const int slot = (int)(((unsigned)lc * 0x9E3779B1u) >> (32 - kDcLog2));
     const unsigned same = __match_any_sync(FULL, lead ? slot : -1 - (int)lane);
     const bool owner = lead && (int)lane == __ffs(same) - 1;
     __syncwarp();
@@ -426,36 +421,21 @@ constexpr int kConsumerWarps = kTile / 32;
 constexpr int kTiledThreads = kTile + 32;
 constexpr int kStages = 2;
 constexpr int kMinBlocks = 3;
-constexpr int kStageBytes = kTile * (6 * 8 + 4);          // the bulk-copied particle columns
-// per-particle gathers the producer warp adds to a landed stage (OPP_AUX):
-// E of the start cell (3 doubles), the DH seed of the drift-only position and
-// its overlay slot
-#ifndef OPP_AUX
-#define OPP_AUX 0
-#endif
-constexpr int kAuxBytes = OPP_AUX ? kTile * (3 * 8 + 4 + 4) : 0;
-constexpr int kStageStride = kStageBytes + kAuxBytes;
+constexpr int kStageBytes = kTile * (6 * 8 + 4);   // the bulk-copied particle columns
 constexpr int kRing = 64;
 constexpr int kRingBytesPerWarp = kRing * 12;   // holes ring (4 B) + work ring (4 B + 4 B hops)
-constexpr int kRingBase = kStages * kStageStride + 3 * kStages * 8;
-constexpr int kQBase = kRingBase + kConsumerWarps * kRingBytesPerWarp;
+constexpr int kRingBase = kStages * kStageBytes + 2 * kStages * 8;
+constexpr int kDcBase = kRingBase + kConsumerWarps * kRingBytesPerWarp;
 
 struct StageView {
     double *c[6];   // x, y, z, vx, vy, vz
     int *cell;
-    double *e[3];   // aux: E of the start cell
-    int *seed;      // aux: DH seed of the drift-only position (DH 1), else the start cell
-    int *slot;      // aux: its overlay slot (-1 outside the overlay)
 };
 __device__ __forceinline__ StageView stage_view(char *smem, int s) {
     StageView v;
-    char *b = smem + (size_t)s * kStageStride;
+    char *b = smem + (size_t)s * kStageBytes;
     for (int k = 0; k < 6; k++) v.c[k] = reinterpret_cast<double *>(b + k * kTile * 8);
     v.cell = reinterpret_cast<int *>(b + 6 * kTile * 8);
-    char *x = b + kStageBytes;
-    for (int k = 0; k < 3; k++) v.e[k] = reinterpret_cast<double *>(x + k * kTile * 8);
-    v.seed = reinterpret_cast<int *>(x + 3 * kTile * 8);
-    v.slot = v.seed + kTile;
     return v;
 }
 
@@ -503,19 +483,6 @@ __device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *coun
     }
 }
 
-// What the producer warp gathered for a particle (OPP_AUX): E of its start
-// cell, the raw overlay value of its drift-only position (DH 1; -1 = none)
-// and that position's overlay slot (-1 = outside the overlay).
-struct Aux {
-    double ex, ey, ez;
-    int seed, slot;
-};
-
-// LATE: the start cell's walk line is loaded after the push and the DH seed,
-// through an opaque dependency on the pushed position, so the 24 line
-// registers and the streamed particle state are never live at once (the
-// TMA-pipelined kernel: fewer registers, 3 blocks per SM); otherwise it is
-// issued together with E (one round trip; direct paths).
 // OPP_LADDER (measurement builds only, scripts/build_variant.sh; 0 = the
 // method): 1 stream the particle state, 2 + E gather and push, 3 + DH seed
 // and first walk-line visit, 4 + the whole walk; deposits and hole records
@@ -527,8 +494,7 @@ template <int DEP, int DH, bool MULTI, bool LATE>
 __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned long long i,
                                          double &x, double &y, double &z, double &vx,
                                          double &vy, double &vz, int &cell, Tally &t,
-                                         Appends *ap = nullptr, const Aux *aux = nullptr,
-                                         DepCache *dc = nullptr) {
+                                         Appends *ap = nullptr, DepCache *dc = nullptr) {
     int status = ST_NONE;
     int capped = 0, hops = 0;
     double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
@@ -549,11 +515,6 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         if (OPP_LADDER == 1) {
             Exy = make_double2(0.0, 0.0);
             Ez = 0.0;
-        } else if (aux) {
-            spec_slot = aux->slot;
-            spec_val = aux->seed;
-            Exy = make_double2(aux->ex, aux->ey);
-            Ez = aux->ez;
         } else {
             if (DH == 1 && OPP_LADDER != 2) {
                 spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)),
@@ -703,200 +664,8 @@ __global__ void __launch_bounds__(256) k_push_move_deposit(StepArgs a) {
     flush_stats(a.cnt, t.hops, t.maxh, t.capped, t.removed);
 }
 
-// ---------------------------------------------------------------------------
-// Hop queue (TMA-pipelined kernel): a particle that is not inside the cell of
-// its first visit does not keep its warp in the walk loop.  Its position,
-// cell, the face to cross and its hop count go to a per-warp queue in shared
-// memory; whenever 32 are queued the warp advances them all by one cell visit
-// together and requeues those still outside.  A warp instruction costs the L1
-// data pipe the same whether 1 or 32 lanes are active (scripts/micro/wf_cost.cu:
-// a 256-bit load costs 8 cycles even for one lane), and ~19% of the particles
-// hop (DH seeding, 0.25 h/step drift), so a hop iteration of a whole warp used
-// to cost a full walk-line load for a few lanes.  Semantics are the walk's
-// (walk_from): the same visits in the same order per particle, H_cap and
-// H_pass tested at the same points.
-// ---------------------------------------------------------------------------
-#ifndef OPP_HOPQ
-#define OPP_HOPQ 0
-#endif
-constexpr int kQ = 64;                                   // ring entries per warp
-constexpr int kQBytesPerWarp = kQ * (3 * 8 + 4 * 4);     // x, y, z | cell, face, hops, index
-constexpr int kDcBase = kQBase + (OPP_HOPQ ? kConsumerWarps * kQBytesPerWarp : 0);
-constexpr int kTiledSmem = kDcBase + (OPP_DCACHE ? kConsumerWarps * kDcBytesPerWarp : 0);
-struct HopQueue {
-    double *x, *y, *z;
-    int *cell, *face, *hops;
-    uint32_t *idx;
-    unsigned head, count;   // warp-uniform
-};
-__device__ __forceinline__ HopQueue hop_queue(char *base) {
-    HopQueue q;
-    q.x = reinterpret_cast<double *>(base);
-    q.y = q.x + kQ;
-    q.z = q.y + kQ;
-    q.cell = reinterpret_cast<int *>(q.z + kQ);
-    q.face = q.cell + kQ;
-    q.hops = q.face + kQ;
-    q.idx = reinterpret_cast<uint32_t *>(q.hops + kQ);
-    q.head = 0;
-    q.count = 0;
-    return q;
-}
-__device__ __forceinline__ void q_push(HopQueue &q, bool pred, double x, double y, double z, int cell,
-                                       int face, int hops, uint32_t i) {
-    const unsigned m = __ballot_sync(0xffffffffu, pred);
-    if (!m) return;
-    if (pred) {
-        const unsigned sl = (q.head + q.count + __popc(m & ((1u << lane_id()) - 1u))) & (kQ - 1);
-        q.x[sl] = x; q.y[sl] = y; q.z[sl] = z;
-        q.cell[sl] = cell; q.face[sl] = face; q.hops[sl] = hops; q.idx[sl] = i;
-    }
-    q.count += __popc(m);
-    __syncwarp();
-}
-
-// Appends of a finished walk (holes, deferred walks, migrants) and its stats.
-template <bool MULTI>
-__device__ __forceinline__ void finish_appends(const StepArgs &a, Appends &ap, int status, uint32_t i,
-                                               int cell, int hops, int capped, Tally &t) {
-    if (status != ST_NONE && status != ST_MOVE && status != ST_MIGRATE) {
-        t.hops += (unsigned)hops;
-        t.maxh = max(t.maxh, (unsigned)hops);
-        t.capped += (unsigned)capped;
-    }
-    t.removed += (status == ST_REMOVE);
-    const bool rem = status == ST_REMOVE || status == ST_MIGRATE;
-    ring_push(ap.holes, rem, i, 0);
-    ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, false);
-    ring_push(ap.work, status == ST_MOVE, i, hops);
-    ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, false);
-    if (MULTI) {
-        const bool mg = status == ST_MIGRATE;
-        unsigned long long ms = warp_append(mg, &a.cnt->n_mig);
-        if (mg) {
-            a.mig[ms] = i;
-            a.mig_cell[ms] = cell;
-            a.mig_hops[ms] = hops;
-        }
-    }
-}
-
-// First visit of one 32-particle slice: push, DH seed, the seed cell's walk
-// line; a particle inside is done (deposited here), one outside is queued with
-// the face to cross (or, at H_cap / H_pass = 0, accepted / deferred as the walk
-// would).  On return `cell` is what p2c holds after this slice (-1 = hole;
-// queued particles hold their current cell until their walk ends).
-template <int DEP, int DH, bool MULTI>
-__device__ __forceinline__ void pmd_first(const StepArgs &a, uint32_t i, double x, double y, double z,
-                                          double vx, double vy, double vz, int &cell, Tally &t,
-                                          Appends &ap, HopQueue &q, const Aux *aux) {
-    const int lc = cell - a.cell_base;
-    long long spec_slot = -1;
-    int spec_val = -1;
-    double2 Exy;
-    double Ez;
-    if (aux) {
-        spec_slot = aux->slot;
-        spec_val = aux->seed;
-        Exy = make_double2(aux->ex, aux->ey);
-        Ez = aux->ez;
-    } else {
-        if (DH == 1) {   // the overlay entry of the drift-only position (see pmd_body)
-            spec_slot = dh_slot(a.ov, add(x, mul(vx, a.dt)), add(y, mul(vy, a.dt)), add(z, mul(vz, a.dt)));
-            spec_val = ov_value(a.ov, spec_slot >= 0 ? spec_slot : 0);
-        }
-        load_E(a.ef, lc, Exy, Ez);
-    }
-    vx = add(vx, mul(a.c1, Exy.x));
-    vy = add(vy, mul(a.c1, Exy.y));
-    vz = add(vz, mul(a.c1, Ez));
-    x = add(x, mul(vx, a.dt));
-    y = add(y, mul(vy, a.dt));
-    z = add(z, mul(vz, a.dt));
-    a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
-    a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
-    if (DH == 1) {
-        const long long g = dh_slot(a.ov, x, y, z);
-        int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
-        if (g < 0) v = -1;
-        if (v >= 0) cell = v;
-    }
-    int zero;   // the line load after the push (see pmd_body, LATE)
-    asm volatile("{\n\t.reg .b64 t;\n\tmov.b64 t, %1;\n\tmov.b32 %0, 0;\n\t}" : "=r"(zero) : "d"(z));
-    Line L = load_line(a.lines, cell - a.cell_base + zero);
-    double l0, l1, l2, l3;
-    bary(L, x, y, z, l0, l1, l2, l3);
-    bool inside = in01(l0) && in01(l1) && in01(l2) && in01(l3);
-    if (DH == 2 && !inside) {
-        const int sc = dh_seed(a.ov, x, y, z, cell);
-        if (sc != cell) {
-            cell = sc;
-            L = load_line(a.lines, sc - a.cell_base);
-            bary(L, x, y, z, l0, l1, l2, l3);
-            inside = in01(l0) && in01(l1) && in01(l2) && in01(l3);
-        }
-    }
-    int status = ST_DONE, capped = 0;
-    if (!inside) {
-        if (0 >= a.hcap) capped = 1;              // accepted as it stands (S4)
-        else if (0 >= a.hpass) status = ST_MOVE;  // deferred to the continuation
-        else status = ST_NONE;                    // queued
-    }
-    deposit_any<DEP>(a, true, status == ST_DONE, i, cell, l0, l1, l2, l3);
-    finish_appends<MULTI>(a, ap, status, i, cell, 0, capped, t);
-    q_push(q, status == ST_NONE, x, y, z, cell, argmin_face(l0, l1, l2, l3), 0, i);
-}
-
-// One cell visit for k <= 32 queued particles (lane l takes entry head + l).
-template <int DEP, bool MULTI>
-__device__ __forceinline__ void hop_round(const StepArgs &a, HopQueue &q, unsigned k, Tally &t,
-                                          Appends &ap) {
-    const unsigned lane = lane_id();
-    const bool act = lane < k;
-    double x = 0, y = 0, z = 0;
-    int cell = 0, f = 0, hops = 0;
-    uint32_t i = 0;
-    if (act) {
-        const unsigned sl = (q.head + lane) & (kQ - 1);
-        x = q.x[sl]; y = q.y[sl]; z = q.z[sl];
-        cell = q.cell[sl]; f = q.face[sl]; hops = q.hops[sl]; i = q.idx[sl];
-    }
-    __syncwarp();
-    q.head = (q.head + k) & (kQ - 1);
-    q.count -= k;
-    int status = ST_NONE, capped = 0;
-    double l0 = 0, l1 = 0, l2 = 0, l3 = 0;
-    if (act) {
-        const int nb = line_c2c_face(a.lines, cell - a.cell_base, f);
-        if (nb < 0) {
-            status = ST_REMOVE;
-        } else if (MULTI && (unsigned)(nb - a.cell_base) >= (unsigned)a.n_cells) {
-            cell = nb;   // the hop into the other rank's cell counts here
-            hops++;
-            status = ST_MIGRATE;
-        } else {
-            cell = nb;
-            hops++;
-            const Line L = load_line(a.lines, nb - a.cell_base);
-            bary(L, x, y, z, l0, l1, l2, l3);
-            if (in01(l0) && in01(l1) && in01(l2) && in01(l3)) {
-                status = ST_DONE;
-            } else if (hops >= a.hcap) {
-                status = ST_DONE;
-                capped = 1;
-            } else if (hops >= a.hpass) {
-                status = ST_MOVE;
-            } else {
-                f = argmin_face(l0, l1, l2, l3);
-            }
-        }
-    }
-    deposit_any<DEP>(a, act && status != ST_NONE, status == ST_DONE, i, cell, l0, l1, l2, l3);
-    finish_appends<MULTI>(a, ap, status, i, cell, hops, capped, t);
-    if (act && status != ST_NONE)
-        a.p2c[i] = (status == ST_REMOVE || status == ST_MIGRATE) ? -1 : cell;
-    q_push(q, act && status == ST_NONE, x, y, z, cell, f, hops, i);
-}
+constexpr int kTiledSmem = kDcBase;                                        // without the cache
+constexpr int kTiledSmemDc = kDcBase + kConsumerWarps * kDcBytesPerWarp;   // with it
 
 // ---------------------------------------------------------------------------
 // The fused push / move / deposit kernel, TMA-pipelined (CalcPosVel + Move +
@@ -965,62 +734,11 @@ __device__ __forceinline__ void issue_tile_load(const StepArgs &a, char *smem, u
     bulk_g2s(v.cell, a.p2c + base, kTile * 4, &full[s]);
 }
 
-// Producer warp, tile t (landed in stage t % kStages): per particle E of the
-// start cell and (DH 1) the overlay entry of the drift-only position x + v dt
-// into the stage's aux columns, and an L1 prefetch of the walk line the
-// consumer will load first (the seed cell, else the start cell).  Lane l
-// takes particles l, l + 32, ... (coalesced shared accesses), four at a time
-// so their loads are in flight together.
-template <int DH>
-__device__ __forceinline__ void producer_aux(const StepArgs &a, char *smem, uint64_t *full,
-                                             uint64_t *ready, unsigned long long t, unsigned lane) {
-    const int s = (int)(t % kStages);
-    mbar_wait(&full[s], (uint32_t)((t / kStages) & 1ull));
-    const StageView v = stage_view(smem, s);
-#pragma unroll
-    for (int half = 0; half < kTile / 128; half++) {
-        double ex[4], ey[4], ez[4];
-        int cl[4], sl[4], sv[4];
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            const int j = (int)lane + 32 * (4 * half + q);
-            cl[q] = v.cell[j];
-            double2 exy;
-            load_E(a.ef, cl[q] - a.cell_base, exy, ez[q]);
-            ex[q] = exy.x;
-            ey[q] = exy.y;
-            sl[q] = -1;
-            sv[q] = -1;
-            if (DH == 1) {
-                const long long g = dh_slot(a.ov, add(v.c[0][j], mul(v.c[3][j], a.dt)),
-                                            add(v.c[1][j], mul(v.c[4][j], a.dt)),
-                                            add(v.c[2][j], mul(v.c[5][j], a.dt)));
-                sl[q] = (int)g;
-                sv[q] = ov_value(a.ov, g >= 0 ? g : 0);
-            }
-        }
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-            const int j = (int)lane + 32 * (4 * half + q);
-            v.e[0][j] = ex[q];
-            v.e[1][j] = ey[q];
-            v.e[2][j] = ez[q];
-            v.seed[j] = sv[q];
-            v.slot[j] = sl[q];
-            const int sc = (DH == 1 && sl[q] >= 0 && sv[q] >= 0) ? sv[q] : cl[q];
-            prefetch_l1(a.lines + (sc - a.cell_base));
-        }
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&ready[s]);
-}
-
 template <int DEP, int DH, bool MULTI>
 __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit_tiled(StepArgs a) {
     extern __shared__ __align__(128) char smem[];
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageStride);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + kStages * kStageBytes);
     uint64_t *empty = full + kStages;
-    uint64_t *ready = empty + kStages;   // OPP_AUX: the producer's gathers have landed
     const unsigned long long n = *(volatile unsigned long long *)&a.cnt->n;
     const unsigned long long ntiles = n / kTile;
     const TileMap tm{ntiles, gridDim.x, (unsigned long long)a.tile_group, blockIdx.x};
@@ -1031,29 +749,20 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
         for (int s = 0; s < kStages; s++) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], kConsumerWarps);
-            mbar_init(&ready[s], 1);
         }
         fence_proxy_async();
     }
     __syncthreads();
     if (warp == kConsumerWarps) {
-        // producer warp: lane 0 streams tiles kStages ahead of the slowest
-        // consumer; then (OPP_AUX) the whole warp does the gathers that only
-        // depend on the streamed state for the tile that landed before -- E
-        // of the start cell, the DH seed of the drift-only position -- and
-        // prefetches the seed cell's walk line into L1, so the consumers'
-        // dependent chain starts from shared memory and an L1 hit.
-        TileIter ti(tm);
-        for (unsigned long long it = 0; it < my; it++, ti.next()) {
-            const int s = (int)(it % kStages);
-            if (lane == 0) {
+        // producer warp: lane 0 streams tiles kStages ahead of the slowest consumer
+        if (lane == 0) {
+            TileIter ti(tm);
+            for (unsigned long long it = 0; it < my; it++, ti.next()) {
+                const int s = (int)(it % kStages);
                 if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1ull));
                 issue_tile_load(a, smem, full, s, ti.tile());
             }
-            __syncwarp();
-            if (OPP_AUX && it >= 1) producer_aux<DH>(a, smem, full, ready, it - 1, lane);
         }
-        if (OPP_AUX && my >= 1) producer_aux<DH>(a, smem, full, ready, my - 1, lane);
         return;
     }
     // Consumer warp, warp-synchronous: one 32-particle slice per tile.  The
@@ -1068,61 +777,37 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
         ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
                            reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
     }
-#if OPP_HOPQ
-    HopQueue q = hop_queue(smem + kQBase + (size_t)warp * kQBytesPerWarp);
-#endif
     DepCache dcache;
     DepCache *dcp = nullptr;
-    if (OPP_DCACHE && DEP == 1) {
+    if (DEP == 1 && a.dcache) {
         dcache = dep_cache(smem + kDcBase + (size_t)warp * kDcBytesPerWarp);
         dcp = &dcache;
     }
     TileIter ti(tm);
     for (unsigned long long it = 0; it < my; it++, ti.next()) {
         const int s = (int)(it % kStages);
-        const uint32_t par = (uint32_t)((it / kStages) & 1ull);
-        mbar_wait(&full[s], par);
-        if (OPP_AUX) mbar_wait(&ready[s], par);
+        mbar_wait(&full[s], (uint32_t)((it / kStages) & 1ull));
         StageView v = stage_view(smem, s);
         const int j = threadIdx.x;
         double x = v.c[0][j], y = v.c[1][j], z = v.c[2][j];
         double vx = v.c[3][j], vy = v.c[4][j], vz = v.c[5][j];
         int cell = v.cell[j];
-        Aux ax;
-        if (OPP_AUX) {
-            ax.ex = v.e[0][j]; ax.ey = v.e[1][j]; ax.ez = v.e[2][j];
-            ax.seed = v.seed[j]; ax.slot = v.slot[j];
-        }
-        unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
-                               (unsigned long long)__double_as_longlong(y) ^
-                               (unsigned long long)__double_as_longlong(z) ^
-                               (unsigned long long)__double_as_longlong(vx) ^
-                               (unsigned long long)__double_as_longlong(vy) ^
-                               (unsigned long long)__double_as_longlong(vz) ^
-                               (unsigned long long)(unsigned)cell;
-        if (OPP_AUX)
-            h ^= (unsigned long long)__double_as_longlong(ax.ex) ^ (unsigned long long)__double_as_longlong(ax.ey) ^
-                 (unsigned long long)__double_as_longlong(ax.ez) ^ (unsigned long long)(unsigned)ax.seed ^
-                 ((unsigned long long)(unsigned)ax.slot << 32);
+        const unsigned long long h = (unsigned long long)__double_as_longlong(x) ^
+                                     (unsigned long long)__double_as_longlong(y) ^
+                                     (unsigned long long)__double_as_longlong(z) ^
+                                     (unsigned long long)__double_as_longlong(vx) ^
+                                     (unsigned long long)__double_as_longlong(vy) ^
+                                     (unsigned long long)__double_as_longlong(vz) ^
+                                     (unsigned long long)(unsigned)cell;
         asm volatile("" ::"l"(h));   // the shared loads have landed
         fence_proxy_async();
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[s]);
         __syncwarp();
         const unsigned long long i = ti.tile() * kTile + j;
-#if OPP_HOPQ
-        pmd_first<DEP, DH, MULTI>(a, (uint32_t)i, x, y, z, vx, vy, vz, cell, t, ap, q, OPP_AUX == 1 ? &ax : nullptr);
+        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap, dcp);
         a.p2c[i] = cell;
-        while (q.count >= 32u) hop_round<DEP, MULTI>(a, q, 32u, t, ap);
-#else
-        pmd_body<DEP, DH, MULTI, true>(a, true, i, x, y, z, vx, vy, vz, cell, t, &ap, OPP_AUX == 1 ? &ax : nullptr,
-                                       dcp);
-        a.p2c[i] = cell;
-#endif
     }
-#if OPP_HOPQ
-    while (q.count) hop_round<DEP, MULTI>(a, q, min(q.count, 32u), t, ap);
-#endif
     if (dcp) dep_cache_flush(a, *dcp);
     ring_flush(ap.holes, &a.cnt->n_holes, a.holes, nullptr, true);
     ring_flush(ap.work, &a.cnt->n_work, a.work, a.work_hops, true);
@@ -1961,11 +1646,12 @@ static cudaError_t launch_tiled(const StepArgs &a, int grid, cudaStream_t s) {
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(k_push_move_deposit_tiled<DEP, DH, MULTI>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmem);
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTiledSmemDc);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    k_push_move_deposit_tiled<DEP, DH, MULTI><<<grid, kTiledThreads, kTiledSmem, s>>>(a);
+    const int smem = (DEP == 1 && a.dcache) ? kTiledSmemDc : kTiledSmem;
+    k_push_move_deposit_tiled<DEP, DH, MULTI><<<grid, kTiledThreads, smem, s>>>(a);
     k_push_move_deposit_tail<DEP, DH, MULTI><<<1, 256, 0, s>>>(a);
     return cudaGetLastError();
 }

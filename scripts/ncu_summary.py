@@ -3,12 +3,20 @@
 
   scripts/ncu_summary.py launches <launches.csv>      per-kernel share of device time
   scripts/ncu_summary.py full <prof.ncu-rep>          key counters of a --set full capture
+  scripts/ncu_summary.py traffic <prof.ncu-rep> <key> <capture-name>
+        record dram read + write bytes of the capture's (single) kernel launch in
+        profiles/ncu_traffic.json under <key>, tagged with the library source
+        hash (bench.py reports it only while the sources are unchanged)
 """
 import csv
 import io
+import json
+import os
 import subprocess
 import sys
 from collections import defaultdict
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 KEYS = [
     "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
@@ -16,6 +24,8 @@ KEYS = [
     "l1tex__throughput.avg.pct_of_peak_sustained_active",
     "lts__throughput.avg.pct_of_peak_sustained_elapsed",
     "l1tex__t_sector_hit_rate.pct", "lts__t_sector_hit_rate.pct",
+    "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "smsp__issue_active.avg.pct_of_peak_sustained_active",
     "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
     "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum",
     "l1tex__t_output_wavefronts_pipe_lsu_mem_global_op_ld.sum",
@@ -65,5 +75,32 @@ def full(path):
                 print(f"  {k:70s} {d[k]:>20s} {units[hdr.index(k)]}")
 
 
+def traffic(path, key, name):
+    sys.path.insert(0, ROOT)
+    import bench
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
+                         text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr, units = rows[0], rows[1]
+    d = dict(zip(hdr, rows[2]))
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+    tot = 0.0
+    for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+        tot += float(d[k].replace(",", "")) * scale[units[hdr.index(k)]]
+    tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        tj = json.load(open(tf))
+    except Exception:   # noqa: BLE001
+        tj = {}
+    tj[key] = {"bytes": tot, "src_hash": bench.src_hash(), "capture": name,
+               "kernel": d.get("Kernel Name", "?")[:80]}
+    json.dump(tj, open(tf, "w"), indent=1, sort_keys=True)
+    print(key, tot)
+
+
 if __name__ == "__main__":
-    {"launches": launches, "full": full}[sys.argv[1]](sys.argv[2])
+    cmd = sys.argv[1]
+    if cmd == "traffic":
+        traffic(sys.argv[2], sys.argv[3], sys.argv[4])
+    else:
+        {"launches": launches, "full": full}[cmd](sys.argv[2])

@@ -276,18 +276,21 @@ def test_shuffle_permutes_and_preserves():
     sim.close()
 
 
-@pytest.mark.parametrize("dep,sort_every", [(0, 0), (1, 0), (1, 2), (2, 0)])
-def test_c5_style_clustered_parity(dep, sort_every):
+@pytest.mark.parametrize("dep,sort_every,cache", [(0, 0, 0), (1, 0, 0), (1, 2, 0), (2, 0, 0), (1, 2, 1),
+                                                 (1, 0, 1)])
+def test_c5_style_clustered_parity(dep, sort_every, cache):
     """C5's shape at C1 size: 90% of 100k particles in a 2x2x3-hex block
     (72 tets, ~1,250 particles per hot tet): the deposit under heavy
-    same-cell contention (plain fp64 atomics, warp-aggregated, sort +
-    segmented reduction), sorted and unsorted storage."""
+    same-cell contention (plain fp64 atomics, warp-aggregated with and
+    without the per-warp node-charge cache, sort + segmented reduction),
+    sorted and unsorted storage."""
     mesh = gen.kuhn_duct(6, 6, 30, jitter=0.2, seed=20240816)
     rng = np.random.default_rng(16)
     ef = rng.uniform(-2e-3, 2e-3, (mesh["n_cells"], 3))
     hot = gen.hot_block_cells(mesh, lo=(2, 2, 10), size=(2, 2, 3))
     init = gen.seed_particles(mesh, 100_000, 20240816, cluster=(0.9, hot))
-    rep, ost, gst = _check(mesh, ef, init, None, 4, deposit_mode=dep, sort_every=sort_every)
+    rep, ost, gst = _check(mesh, ef, init, None, 4, deposit_mode=dep, sort_every=sort_every,
+                           deposit_cache=bool(cache))
     assert rep["n_compared"] > 95_000
 
 
@@ -322,8 +325,9 @@ def exact_geometry_case():
     return mesh, ef, init
 
 
-@pytest.mark.parametrize("dh,dep,hpass", [(0, 1, 4), (0, 0, 1), (1, 1, 4), (1, 2, 8), (2, 1, 4), (0, 1, 0)])
-def test_exact_geometry_no_exclusion(dh, dep, hpass):
+@pytest.mark.parametrize("dh,dep,hpass,cache", [(0, 1, 4, 0), (0, 0, 1, 0), (1, 1, 4, 0), (1, 2, 8, 0),
+                                                (2, 1, 4, 0), (0, 1, 0, 0), (1, 1, 4, 1)])
+def test_exact_geometry_no_exclusion(dh, dep, hpass, cache):
     mesh, ef, init = exact_geometry_case()
     assert init["cell"].size > 15_000
     overlay = None
@@ -335,7 +339,7 @@ def test_exact_geometry_no_exclusion(dh, dep, hpass):
     om, orc, Qo, ost, rem = run_oracle(mesh, ef, init, None, steps, C1 * DT, DT, W, use_dh=dh,
                                        overlay=overlay)
     gout, Qg, gst, _ = _gpu_run(mesh, ef, init, None, steps, direct_hop=dh, overlay_spacing=0.5,
-                                deposit_mode=dep, hop_budget=hpass)
+                                deposit_mode=dep, hop_budget=hpass, deposit_cache=bool(cache))
     rep = compare(om, mesh["c2n"], orc, Qo, rem, gout, Qg, W, near=None)
     assert rep["n_excluded"] == 0 and rep["n_compared"] > 10_000
     for so, sg in zip(ost, gst):
