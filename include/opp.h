@@ -512,6 +512,41 @@ int opp_em_advance_e(opp_ctx ctx, double *e, const double *b, const double *J, c
 /* Statistics of the last opp_em_move_deposit; synchronises. */
 int opp_em_get_stats(opp_ctx ctx, opp_em_stats *stats);
 
+/* ---- CabanaPIC over slabs (config C3 on several GPUs; PAPER.md:1794-1800:
+ * Update_Ghosts is the halo exchange of the CabanaPIC field side).  Each rank
+ * (opp_init nranks / rank / transport) owns the z-layers [k0, k1) of the
+ * periodic nx x ny x nz grid, i.e. cells [k0 nx ny, k1 nx ny); the ranks'
+ * ranges must tile [0, nz) in rank order, so the neighbours are rank -+ 1
+ * (mod nranks).  Collective.  Field arrays stay global-sized (nc cells) on
+ * every rank: a rank computes its own cells and keeps the ghost layers it
+ * reads current.  Errors: OPP_ERR_ARG (ranges do not tile). */
+int opp_em_set_partition(opp_ctx ctx, int nx, int ny, int nz, int k0, int k1);
+
+/* Move_Deposit over slabs: opp_em_move_deposit for this rank's particles
+ * [0, *n) (columns of stride cap; id[cap] int64, may be NULL, travels with
+ * its particle).  A particle whose path enters another rank's cell stops on
+ * that face -- its deposits so far are this rank's -- and migrates with the
+ * rest of its streak (96-B records over the transport, appended behind the
+ * receiver's particles, which walks and deposits the rest); rounds repeat
+ * until no rank has migrants; the departed particles' slots are filled from
+ * the end.  On return *n = this rank's new count.
+ * Collective.  Requires kcap >= 1.  Errors: OPP_ERR_STATE (no partition),
+ * OPP_ERR_CAPACITY (arrivals beyond cap), OPP_ERR_ARG.  Synchronises once per
+ * migration round (the message sizes). */
+int opp_em_move_deposit_slab(opp_ctx ctx, int64_t *n, int64_t cap, double *off, double *u, double *w,
+                             int32_t *cell, int64_t *id, const double *interp, const int32_t *c2c,
+                             int64_t n_cells, double *acc, const opp_em_params *params,
+                             opp_em_stats *stats);
+
+/* The field side over slabs, one leap-frog step on this rank's cells:
+ * AccumulateCurrent, AdvanceB(dt/2), AdvanceE(dt), AdvanceB(dt/2),
+ * Interpolate, then acc := 0 on this rank's cells -- with Update_Ghosts
+ * before each kernel that reads a neighbour's layer: acc and B of layer
+ * k0 - 1 from rank - 1, E and B of layer k1 from rank + 1.  Collective;
+ * global-sized arrays as above.  Errors as opp_em_accumulate_current. */
+int opp_em_field_step_slab(opp_ctx ctx, double *e, double *b, double *J, double *acc, double *interp,
+                           const int32_t *c2c, int64_t n_cells, const double *h, double dt);
+
 /* Synchronise the context's stream; reports sticky asynchronous errors. */
 int opp_sync(opp_ctx ctx);
 

@@ -176,10 +176,22 @@ struct opp_ctx_s {
     MeshCache mc;
     FieldState fs;
     opp::EmCounters *em_cnt = nullptr;   // opp_em_move_deposit statistics (device)
-    uint32_t *em_work = nullptr;         // deferred face crossers (continuation worklist)
-    long long em_work_cap = 0;
-    int em_defer = 0;                    // OPP_EM_DEFER=1: face crossers finish in a continuation pass
-                                         // (C3: 4.16 -> 5.17 ms, parity green: off)
+    struct {                             // EM slab partition (opp_em_set_partition)
+        bool on = false;
+        int nx = 0, ny = 0, nz = 0, k0 = 0, k1 = 0;
+        opp::EmRanges rr{};
+        long long cap = 0;               // particle capacity the migrant lists are sized for
+        unsigned long long *mig_n = nullptr;
+        uint32_t *mig_i = nullptr, *holes = nullptr;
+        double *mig_p = nullptr, *mig_d = nullptr;
+        int32_t *mig_c = nullptr, *mig_k = nullptr;
+        double *dbuf = nullptr;          // received particles' rest of streak [3][cap]
+        int32_t *kbuf = nullptr;
+        unsigned long long *counts = nullptr;   // [R] + cursor [R] + all [R * R]
+        char *send = nullptr, *recv = nullptr, *gsend = nullptr, *grecv = nullptr;
+        size_t send_cap = 0, recv_cap = 0, gcap = 0, gcap2 = 0;
+        DevCounters *dc = nullptr;       // the compaction's counters
+    } em_slab;
     struct {                             // opp_em_sort_by_cell scratch
         unsigned *hist = nullptr, *start = nullptr;
         unsigned long long *tile_sums = nullptr;
@@ -422,7 +434,16 @@ extern "C" int opp_finalize(opp_ctx c) {
     c->dfree(m.n2cs, 0);
     free_field(c);
     c->dfree(c->em_cnt, sizeof(opp::EmCounters));
-    c->dfree(c->em_work, 0);
+    {
+        auto &es = c->em_slab;
+        c->dfree(es.mig_n); c->dfree(es.mig_i); c->dfree(es.holes); c->dfree(es.mig_p); c->dfree(es.mig_d);
+        c->dfree(es.mig_c); c->dfree(es.mig_k); c->dfree(es.dbuf); c->dfree(es.kbuf); c->dfree(es.counts);
+        c->dfree(es.dc);
+        if (es.send) cudaFree(es.send);
+        if (es.recv) cudaFree(es.recv);
+        if (es.gsend) cudaFree(es.gsend);
+        if (es.grecv) cudaFree(es.grecv);
+    }
     c->dfree(c->em_sort.hist, 0);
     c->dfree(c->em_sort.start, 0);
     c->dfree(c->em_sort.tile_sums, 0);
@@ -1970,20 +1991,247 @@ extern "C" int opp_em_move_deposit(opp_ctx c, int64_t n, int64_t stride, double 
     a.kcap = prm->kcap;
     a.dep = prm->deposit_mode == OPP_DEP_ATOMIC_WARPAGG ? 1 : 0;
     a.cnt = c->em_cnt;
-    if (c->em_defer && n > c->em_work_cap) {
-        c->dfree(c->em_work, 0);
-        c->em_work = (uint32_t *)c->dalloc(4 * (size_t)n);
-        if (!c->em_work) return fail(OPP_ERR_NOMEM, "em worklist");
-        c->em_work_cap = n;
-    }
-    a.work = c->em_defer ? c->em_work : nullptr;
-    if (n > (long long)UINT32_MAX) a.work = nullptr;
+    a.c0 = 0;
+    a.c1 = n_cells;
     if (n > 0) {
         PhaseScope ph(c, OPP_PH_EM_MOVE_DEPOSIT);
         CK(opp::launch_em_move_deposit(a, c->nsm, c->s));
-        c->launches += (a.work && a.kcap > 0) ? 2 : 1;
+        c->launches += 1;
     }
     if (stats) return opp_em_get_stats(c, stats);
+    return OPP_OK;
+}
+
+// ---------------------------------------------------------------------------
+// CabanaPIC over slabs (config C3 on several GPUs): each
+// rank owns consecutive z-layers of the periodic grid; Move_Deposit
+// migrates the particles whose path leaves the slab (with the rest of their
+// streak) and Update_Ghosts exchanges the boundary layers the field kernels
+// read from the neighbours.
+// ---------------------------------------------------------------------------
+extern "C" int opp_em_set_partition(opp_ctx c, int nx, int ny, int nz, int k0, int k1) {
+    TRY(ctx_check(c));
+    if (nx < 1 || ny < 1 || nz < 1 || k0 < 0 || k1 <= k0 || k1 > nz)
+        return fail(OPP_ERR_ARG, "0 <= k0 < k1 <= nz, sizes >= 1");
+    const int R = c->p.nranks;
+    if (R > opp::kEmMaxRanks) return fail(OPP_ERR_ARG, "too many ranks");
+    auto &es = c->em_slab;
+    std::vector<int64_t> mine = {k0, k1}, all(2 * (size_t)R);
+    if (R > 1) TRY(c->comm->t->allgather_i64(mine.data(), 2, all.data(), c->s, g_err));
+    else all = mine;
+    const long long L = (long long)nx * ny;
+    int expect = 0;
+    for (int r = 0; r < R; r++) {
+        if (all[2 * r] != expect || all[2 * r + 1] <= all[2 * r])
+            return fail(OPP_ERR_ARG, "ranks' z-layer ranges must tile [0, nz) in rank order");
+        es.rr.lo[r] = all[2 * r] * L;
+        expect = (int)all[2 * r + 1];
+    }
+    if (expect != nz) return fail(OPP_ERR_ARG, "ranks' z-layer ranges must tile [0, nz)");
+    es.rr.lo[R] = (long long)nz * L;
+    es.rr.n = R;
+    es.nx = nx; es.ny = ny; es.nz = nz; es.k0 = k0; es.k1 = k1;
+    if (!es.counts) {
+        es.counts = (unsigned long long *)c->dalloc(8 * (size_t)(2 + R) * R);
+        es.mig_n = (unsigned long long *)c->dalloc(8);
+        es.dc = (DevCounters *)c->dalloc(sizeof(DevCounters));
+        if (!es.counts || !es.mig_n || !es.dc) return fail(OPP_ERR_NOMEM, "em slab counters");
+    }
+    es.on = true;
+    return OPP_OK;
+}
+
+static int em_slab_reserve(opp_ctx c, long long cap) {
+    auto &es = c->em_slab;
+    if (es.cap >= cap) return OPP_OK;
+    c->dfree(es.mig_i); c->dfree(es.holes); c->dfree(es.mig_p); c->dfree(es.mig_d);
+    c->dfree(es.mig_c); c->dfree(es.mig_k); c->dfree(es.dbuf); c->dfree(es.kbuf);
+    const size_t n = (size_t)cap;
+    es.mig_i = (uint32_t *)c->dalloc(4 * n);
+    es.holes = (uint32_t *)c->dalloc(4 * n);
+    es.mig_p = (double *)c->dalloc(24 * n);
+    es.mig_d = (double *)c->dalloc(24 * n);
+    es.mig_c = (int32_t *)c->dalloc(4 * n);
+    es.mig_k = (int32_t *)c->dalloc(4 * n);
+    es.dbuf = (double *)c->dalloc(24 * n);
+    es.kbuf = (int32_t *)c->dalloc(4 * n);
+    if (!es.mig_i || !es.holes || !es.mig_p || !es.mig_d || !es.mig_c || !es.mig_k || !es.dbuf || !es.kbuf) {
+        es.cap = 0;
+        return fail(OPP_ERR_NOMEM, "em slab migrant lists");
+    }
+    es.cap = cap;
+    return OPP_OK;
+}
+
+extern "C" int opp_em_move_deposit_slab(opp_ctx c, int64_t *n_io, int64_t cap, double *off, double *u,
+                                        double *w, int32_t *cell, int64_t *id, const double *interp,
+                                        const int32_t *c2c, int64_t n_cells, double *acc,
+                                        const opp_em_params *prm, opp_em_stats *stats) {
+    TRY(ctx_check(c));
+    auto &es = c->em_slab;
+    if (!es.on) return fail(OPP_ERR_STATE, "opp_em_set_partition first");
+    if (!prm || !n_io) return fail(OPP_ERR_ARG, "null params / n");
+    const long long n = *n_io;
+    if (n < 0 || cap < n || cap > (int64_t)UINT32_MAX) return fail(OPP_ERR_ARG, "0 <= n <= cap < 2^32");
+    if (n_cells != es.rr.lo[es.rr.n]) return fail(OPP_ERR_ARG, "n_cells differs from the partition's grid");
+    if (cap > 0 && (!off || !u || !w || !cell)) return fail(OPP_ERR_ARG, "null particle column");
+    if (!interp || !c2c || !acc) return fail(OPP_ERR_ARG, "null mesh array");
+    if (prm->kcap < 1) return fail(OPP_ERR_ARG, "slabs: kcap >= 1");
+    if (prm->deposit_mode != OPP_DEP_ATOMIC && prm->deposit_mode != OPP_DEP_ATOMIC_WARPAGG)
+        return fail(OPP_ERR_ARG, "deposit_mode: OPP_DEP_ATOMIC or OPP_DEP_ATOMIC_WARPAGG");
+    TRY(em_slab_reserve(c, std::max<long long>(cap, 1)));
+    if (!c->em_cnt) {
+        c->em_cnt = (opp::EmCounters *)c->dalloc(sizeof(opp::EmCounters));
+        if (!c->em_cnt) return fail(OPP_ERR_NOMEM, "em counters");
+    }
+    const int R = es.rr.n, me = c->p.rank;
+    CK(cudaMemsetAsync(c->em_cnt, 0, sizeof(opp::EmCounters), c->s));
+    CK(cudaMemsetAsync(es.mig_n, 0, 8, c->s));
+    opp::EmArgs a{};
+    a.n = n;
+    a.cap = cap;
+    a.off = off;
+    a.u = u;
+    a.w = w;
+    a.cell = cell;
+    a.interp = interp;
+    a.c2c = c2c;
+    a.nc = n_cells;
+    a.acc = acc;
+    a.qdt_2mc = prm->qdt_2mc;
+    for (int k = 0; k < 3; k++) a.cdt[k] = prm->cdt_2h[k];
+    a.qsp = prm->qsp;
+    a.kcap = prm->kcap;
+    a.dep = prm->deposit_mode == OPP_DEP_ATOMIC_WARPAGG ? 1 : 0;
+    a.cnt = c->em_cnt;
+    a.c0 = es.rr.lo[me];
+    a.c1 = es.rr.lo[me + 1];
+    a.mig_n = es.mig_n;
+    a.mig_i = es.mig_i;
+    a.mig_p = es.mig_p;
+    a.mig_d = es.mig_d;
+    a.mig_c = es.mig_c;
+    a.mig_k = es.mig_k;
+    a.mig_cap = cap;
+    PhaseScope ph(c, OPP_PH_EM_MOVE_DEPOSIT);
+    if (n > 0) CK(opp::launch_em_move_deposit(a, c->nsm, c->s));
+    c->launches++;
+    long long cur = n, nholes = 0;
+    unsigned long long *counts = es.counts, *cursor = es.counts + R, *all = es.counts + 2 * R;
+    std::vector<unsigned long long> M((size_t)R * R);
+    std::vector<int64_t> soff(R), sbytes(R), roff(R), rbytes(R);
+    const int rec = (int)sizeof(opp::EmRecord);
+    for (int round = 0;; round++) {
+        // migrants of this round per destination, all ranks' rows gathered
+        CK(opp::launch_em_mig_count(a, es.rr, counts, c->s));
+        if (R > 1) TRY(c->comm->t->allgather_dev(counts, 8 * (size_t)R, all, c->s, g_err));
+        else CK(cudaMemcpyAsync(all, counts, 8, cudaMemcpyDeviceToDevice, c->s));
+        unsigned long long nmig = 0;
+        CK(cudaMemcpyAsync(M.data(), all, 8 * (size_t)R * R, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaMemcpyAsync(&nmig, es.mig_n, 8, cudaMemcpyDeviceToHost, c->s));
+        CK(cudaStreamSynchronize(c->s));
+        c->launches++;
+        unsigned long long total = 0;
+        for (auto v : M) total += v;
+        if (total == 0) break;
+        long long out = 0, in = 0;
+        for (int q = 0; q < R; q++) {
+            soff[q] = out * rec;
+            sbytes[q] = (int64_t)M[(size_t)me * R + q] * rec;
+            out += (long long)M[(size_t)me * R + q];
+            roff[q] = in * rec;
+            rbytes[q] = (int64_t)M[(size_t)q * R + me] * rec;
+            in += (long long)M[(size_t)q * R + me];
+        }
+        if (cur + in > cap) return fail(OPP_ERR_CAPACITY, "em slab: capacity %lld < %lld", (long long)cap, cur + in);
+        TRY(opp::comm_reserve(&es.send, &es.send_cap, (size_t)std::max<long long>(out, 1) * rec, g_err));
+        TRY(opp::comm_reserve(&es.recv, &es.recv_cap, (size_t)std::max<long long>(in, 1) * rec, g_err));
+        std::vector<unsigned long long> cu(R);
+        for (int q = 0; q < R; q++) cu[q] = (unsigned long long)(soff[q] / rec);
+        CK(cudaMemcpyAsync(cursor, cu.data(), 8 * R, cudaMemcpyHostToDevice, c->s));
+        // the departed particles' slots join the hole list
+        CK(opp::launch_em_mig_pack(a, es.rr, cursor, (const long long *)id, (opp::EmRecord *)es.send,
+                                   es.holes + nholes, c->s));
+        nholes += (long long)nmig;
+        if (R > 1) TRY(c->comm->t->exchange(es.send, soff, sbytes, es.recv, roff, rbytes, c->s, g_err));
+        else CK(cudaMemcpyAsync(es.recv, es.send, (size_t)in * rec, cudaMemcpyDeviceToDevice, c->s));
+        CK(cudaMemsetAsync(es.mig_n, 0, 8, c->s));
+        CK(opp::launch_em_mig_unpack(a, (long long *)id, (const opp::EmRecord *)es.recv, cur, in, es.dbuf,
+                                     es.kbuf, c->s));
+        CK(opp::launch_em_continue(a, cur, in, es.dbuf, es.kbuf, c->nsm, c->s));
+        c->launches += 4;
+        cur += in;
+        if (round > 64 * R) return fail(OPP_ERR_STATE, "em migration did not terminate");
+    }
+    if (nholes > 0) {   // fill the departed particles' slots from the end
+        DevCounters h{};
+        h.n = (unsigned long long)cur;
+        h.n_holes = (unsigned long long)nholes;
+        CK(cudaMemcpyAsync(es.dc, &h, sizeof h, cudaMemcpyHostToDevice, c->s));
+        ColSet cs{};
+        cs.c[0] = ColDesc{(char *)off, cap, 8, 3};
+        cs.c[1] = ColDesc{(char *)u, cap, 8, 3};
+        cs.c[2] = ColDesc{(char *)w, cap, 8, 1};
+        cs.c[3] = ColDesc{(char *)cell, cap, 4, 1};
+        cs.n = 4;
+        if (id) cs.c[cs.n++] = ColDesc{(char *)id, cap, 8, 1};
+        CK(launch_fill(cs, es.dc, es.holes, cell, es.mig_i, es.kbuf ? (uint32_t *)es.kbuf : nullptr,
+                       grid_for(c, cur, 4), c->s));
+        c->launches += 2;
+    }
+    *n_io = cur - nholes;
+    if (stats) return opp_em_get_stats(c, stats);
+    return OPP_OK;
+}
+
+// Update_Ghosts: one z-layer of a global-sized field (ncomp components
+// `stride` apart, `per` doubles per cell) from a neighbour: up = 1: my top
+// layer k1 - 1 -> rank + 1, into my layer k0 - 1 from rank - 1; up = 0: my
+// bottom layer k0 -> rank - 1, into my layer k1 from rank + 1 (periodic).
+static int em_ghost(opp_ctx c, double *f, int ncomp, long long stride, int per, int up) {
+    auto &es = c->em_slab;
+    const int R = es.rr.n, me = c->p.rank;
+    if (R == 1) return OPP_OK;
+    const long long L = (long long)es.nx * es.ny * per;                // doubles per layer and component
+    const int sl = up ? es.k1 - 1 : es.k0;
+    const int rl = up ? (es.k0 - 1 + es.nz) % es.nz : es.k1 % es.nz;
+    const int to = up ? (me + 1) % R : (me - 1 + R) % R, from = up ? (me - 1 + R) % R : (me + 1) % R;
+    const size_t bytes = (size_t)ncomp * L * 8;
+    TRY(opp::comm_reserve(&es.gsend, &es.gcap, bytes, g_err));
+    TRY(opp::comm_reserve(&es.grecv, &es.gcap2, bytes, g_err));
+    CK(cudaMemcpy2DAsync(es.gsend, L * 8, f + (long long)sl * L, stride * 8, L * 8, ncomp,
+                         cudaMemcpyDeviceToDevice, c->s));
+    std::vector<int64_t> off(R, 0), sb(R, 0), rb(R, 0);
+    sb[to] = (int64_t)bytes;
+    rb[from] = (int64_t)bytes;
+    TRY(c->comm->t->exchange(es.gsend, off, sb, es.grecv, off, rb, c->s, g_err));
+    CK(cudaMemcpy2DAsync(f + (long long)rl * L, stride * 8, es.grecv, L * 8, L * 8, ncomp,
+                         cudaMemcpyDeviceToDevice, c->s));
+    return OPP_OK;
+}
+
+extern "C" int opp_em_field_step_slab(opp_ctx c, double *e, double *b, double *J, double *acc, double *interp,
+                                      const int32_t *c2c, int64_t n_cells, const double *h, double dt) {
+    TRY(ctx_check(c));
+    auto &es = c->em_slab;
+    if (!es.on) return fail(OPP_ERR_STATE, "opp_em_set_partition first");
+    TRY(em_field_check(e, b, c2c, n_cells, h, dt));
+    if (!J || !acc || !interp) return fail(OPP_ERR_ARG, "null J / acc / interp");
+    if (n_cells != es.rr.lo[es.rr.n]) return fail(OPP_ERR_ARG, "n_cells differs from the partition's grid");
+    const int me = c->p.rank;
+    const long long c0 = es.rr.lo[me], c1 = es.rr.lo[me + 1];
+    PhaseScope ph(c, OPP_PH_FIELD);
+    TRY(em_ghost(c, acc, 1, n_cells * opp::kEmNA, opp::kEmNA, 1));   // AccumulateCurrent reads k0 - 1
+    CK(opp::launch_em_accumulate_current(acc, c2c, n_cells, h, dt, J, c->s, c0, c1));
+    CK(opp::launch_em_advance_b(e, b, c2c, n_cells, h, dt / 2, c->s, c0, c1));   // reads E at k1
+    TRY(em_ghost(c, b, 3, n_cells, 1, 1));                            // AdvanceE reads B at k0 - 1
+    CK(opp::launch_em_advance_e(e, b, J, c2c, n_cells, h, dt, c->s, c0, c1));
+    TRY(em_ghost(c, e, 3, n_cells, 1, 0));                            // AdvanceB, Interpolate: E at k1
+    CK(opp::launch_em_advance_b(e, b, c2c, n_cells, h, dt / 2, c->s, c0, c1));
+    TRY(em_ghost(c, b, 3, n_cells, 1, 0));                            // Interpolate: B at k1
+    CK(opp::launch_em_interpolate(es.nx, es.ny, es.nz, e, b, interp, c->s, c0, c1));
+    CK(cudaMemsetAsync(acc + c0 * opp::kEmNA, 0, 8 * (size_t)(c1 - c0) * opp::kEmNA, c->s));
+    c->launches += 6;
     return OPP_OK;
 }
 

@@ -39,9 +39,10 @@ __device__ __forceinline__ double dvd(double a, double b) { return __ddiv_rn(a, 
 // B_a).  Same layouts and evaluation order as the oracle's em_interpolate.
 // ---------------------------------------------------------------------------
 __global__ void k_em_interpolate(int nx, int ny, int nz, const double *__restrict__ e,
-                                 const double *__restrict__ b, double *__restrict__ interp) {
+                                 const double *__restrict__ b, double *__restrict__ interp, long long c0,
+                                 long long c1) {
     const long long nc = (long long)nx * ny * nz;
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+    for (long long c = c0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; c < c1;
          c += (long long)gridDim.x * blockDim.x) {
         const int i = (int)(c % nx), j = (int)((c / nx) % ny), k = (int)(c / ((long long)nx * ny));
         const int ip = (i + 1) % nx, jp = (j + 1) % ny, kp = (k + 1) % nz;
@@ -323,6 +324,34 @@ __device__ __forceinline__ void em_streak(const EmArgs &a, const double uu[3], d
     d[2] = mul(a.cdt[2], mul(uu[2], rg));
 }
 
+// Slabs: a cell of another rank (cells outside [c0, c1))
+__device__ __forceinline__ bool em_foreign(const EmArgs &a, int c) {
+    return a.mig_n && ((long long)c < a.c0 || (long long)c >= a.c1);
+}
+// Record migrants (warp-aggregated append): index, face point, rest of the
+// streak, new cell, crossings so far; the particle's slot becomes a hole.
+__device__ __forceinline__ void em_mig_push(const EmArgs &a, bool pred, long long i, const double p[3],
+                                            const double d[3], int c, int k) {
+    const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
+    const unsigned m = __ballot_sync(FULL, pred);
+    if (!m) return;
+    unsigned long long base = 0;
+    const int leader = __ffs(m) - 1;
+    if ((int)lane == leader) base = atomicAdd(a.mig_n, (unsigned long long)__popc(m));
+    base = __shfl_sync(FULL, base, leader);
+    if (pred) {
+        const unsigned long long sl = base + __popc(m & ((1u << lane) - 1u));
+        a.mig_i[sl] = (uint32_t)i;
+        for (int ax = 0; ax < 3; ax++) {
+            a.mig_p[ax * a.mig_cap + sl] = p[ax];
+            a.mig_d[ax * a.mig_cap + sl] = d[ax];
+        }
+        a.mig_c[sl] = c;
+        a.mig_k[sl] = k;
+        a.cell[i] = -1;
+    }
+}
+
 // Per-warp queue of particles still crossing faces (OPP_EM_QUEUE): their later
 // move rounds run in batches of 32, so a round never runs for a handful of
 // lanes (a round costs the warp the same ~250 instructions for 2 lanes as
@@ -390,12 +419,13 @@ __device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, dou
     }
     // queued particles sit in scattered cells: direct reductions (OPP_EM_QDEP=1: warp-aggregated)
     em_deposit<OPP_EM_QDEP ? DEP : 0>(a.acc, has, c, v, wbuf);
-    bool again = false, capped = false;
+    bool again = false, capped = false, migr = false;
     if (has) {
         if (face >= 0 && k < a.kcap) {
             em_cross(p, d, q, face, c, a.c2c);
             k++;
-            again = true;
+            if (em_foreign(a, c)) migr = true;
+            else again = true;
         } else {
             capped = face >= 0;
             a.off[i] = q[0]; a.off[a.cap + i] = q[1]; a.off[2 * a.cap + i] = q[2];
@@ -405,10 +435,11 @@ __device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, dou
             maxk = max(maxk, (unsigned)k);
         }
     }
+    em_mig_push(a, migr, i, p, d, c, k);
     qs.push(again, p, d, c, k, i);
 }
 
-template <int DEP, bool DEFER, bool QUEUE>
+template <int DEP, bool QUEUE>
 __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
     extern __shared__ __align__(16) char em_dyn[];   // per warp: transpose buffer, then the queue
@@ -481,14 +512,11 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
             a.u[i] = uu[0]; a.u[a.cap + i] = uu[1]; a.u[2 * a.cap + i] = uu[2];
         }
         // 4. move through the faces crossed; one segment per lane per round,
-        //    deposited warp-aggregated (rounds continue while any lane moves).
-        //    DEFER: only the first round runs here; particles that cross a face
-        //    (~10% per step on C3) go to a worklist that k_em_move_continue
-        //    finishes in full warps (a later round with a few active lanes
-        //    costs a whole warp pass of the move)
+        //    deposited warp-aggregated (rounds continue while any lane moves);
+        //    QUEUE: a particle that crosses a face continues in the warp's queue
         bool moving = valid;
         int k = 0;
-        bool capped = false, deferred = false, queued = false;
+        bool capped = false, queued = false, migr = false;
         while (__any_sync(FULL, moving)) {
             double v[kEmNA];
             int face = -1;
@@ -509,30 +537,21 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                     p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
                     capped = true;
                     moving = false;
-                } else if (DEFER) {
-                    deferred = true;
-                    moving = false;
-                } else if (QUEUE) {
-                    em_cross(p, d, q, face, c, a.c2c);
-                    k++;
-                    queued = true;
-                    moving = false;
                 } else {
                     em_cross(p, d, q, face, c, a.c2c);
                     k++;
+                    if (em_foreign(a, c)) {   // slab: the rest of the walk is another rank's
+                        migr = true;
+                        moving = false;
+                    } else if (QUEUE) {
+                        queued = true;
+                        moving = false;
+                    }
                 }
             }
         }
-        if (DEFER) {
-            const unsigned m = __ballot_sync(FULL, deferred);
-            if (m) {
-                unsigned long long base = 0;
-                if (lane == (unsigned)(__ffs(m) - 1)) base = atomicAdd(&a.cnt->n_work, (unsigned long long)__popc(m));
-                base = __shfl_sync(FULL, base, __ffs(m) - 1);
-                if (deferred) a.work[base + __popc(m & ((1u << lane) - 1u))] = (uint32_t)i;
-            }
-        }
-        if (valid && !deferred && !queued) {
+        em_mig_push(a, migr, i, p, d, c, k);
+        if (valid && !queued && !migr) {
             a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
             a.cell[i] = c;
             ncross += (unsigned)k;
@@ -556,54 +575,62 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
     }
 }
 
-// Continuation of the deferred particles: one particle per lane, lanes fully
-// independent (the deposit reduces directly: the particles are few and in
-// scattered cells).  The first round is recomputed bit for bit from the
-// stored state (offsets not yet written, u already pushed) and not deposited
-// again; the later rounds are deposited.
-__global__ void __launch_bounds__(256) k_em_move_continue(EmArgs a) {
+// Slabs: particles received from another rank resume their walk -- from the
+// face point (off) in their new cell with the rest of the streak d and the
+// crossings k -- one per lane, depositing every segment directly (they are
+// few and in scattered cells); one that enters yet another rank's cell
+// migrates again.  The segment sequence is the one the single-domain kernel
+// walks, so deposits and final states are those of one domain.
+__global__ void __launch_bounds__(256) k_em_continue(EmArgs a, long long first, long long m,
+                                                     const double *__restrict__ dbuf,
+                                                     const int32_t *__restrict__ kbuf) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
-    const unsigned long long nw = *(volatile unsigned long long *)&a.cnt->n_work;
     unsigned long long ncross = 0, ncap = 0;
     unsigned maxk = 0;
-    for (unsigned long long w = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; w < nw;
-         w += (unsigned long long)gridDim.x * blockDim.x) {
-        const long long i = a.work[w];
-        int c = a.cell[i];
-        double p[3] = {a.off[i], a.off[a.cap + i], a.off[2 * a.cap + i]};
-        const double uu[3] = {a.u[i], a.u[a.cap + i], a.u[2 * a.cap + i]};
-        const double Q = mul(a.qsp, a.w[i]);
-        double d[3];
-        em_streak(a, uu, d);
-        double q[3];
-        int face = em_face(p, d, q);   // round 1 (deposited by the first pass): crosses
-        em_cross(p, d, q, face, c, a.c2c);
-        int k = 1;
-        bool capped = false;
-        for (;;) {
-            double v[kEmNA];
-            face = em_face(p, d, q);
+    const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
+    for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; base < m;
+         base += nw * 32) {
+        const long long t = base + lane;
+        const bool valid = t < m;
+        const long long i = first + t;
+        int c = 0, k = 0;
+        double p[3] = {0, 0, 0}, d[3] = {0, 0, 0}, Q = 0;
+        if (valid) {
+            c = a.cell[i];
+            p[0] = a.off[i]; p[1] = a.off[a.cap + i]; p[2] = a.off[2 * a.cap + i];
+            d[0] = dbuf[t]; d[1] = dbuf[m + t]; d[2] = dbuf[2 * m + t];
+            k = kbuf[t];
+            Q = mul(a.qsp, a.w[i]);
+        }
+        bool moving = valid, capped = false, migr = false;
+        while (moving) {
+            double v[kEmNA], q[3];
+            const int face = em_face(p, d, q);
             seg_current(p, q, Q, v);
             double *acc = a.acc + (long long)kEmNA * c;
 #pragma unroll
-            for (int s = 0; s < kEmNA; s++) atomicAdd(acc + s, v[s]);
-            if (face < 0) {
+            for (int s_ = 0; s_ < kEmNA; s_++) atomicAdd(acc + s_, v[s_]);
+            if (face < 0 || k >= a.kcap) {
                 p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
-                break;
+                capped = face >= 0;
+                moving = false;
+            } else {
+                em_cross(p, d, q, face, c, a.c2c);
+                k++;
+                if (em_foreign(a, c)) {
+                    migr = true;
+                    moving = false;
+                }
             }
-            if (k >= a.kcap) {
-                p[0] = q[0]; p[1] = q[1]; p[2] = q[2];
-                capped = true;
-                break;
-            }
-            em_cross(p, d, q, face, c, a.c2c);
-            k++;
         }
-        a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
-        a.cell[i] = c;
-        ncross += (unsigned)k;
-        ncap += capped;
-        maxk = max(maxk, (unsigned)k);
+        em_mig_push(a, migr, i, p, d, c, k);
+        if (valid && !migr) {
+            a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
+            a.cell[i] = c;
+            ncross += (unsigned)k;
+            ncap += capped;
+            maxk = max(maxk, (unsigned)k);
+        }
     }
     const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
     const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
@@ -612,6 +639,68 @@ __global__ void __launch_bounds__(256) k_em_move_continue(EmArgs a) {
         if (sc) atomicAdd(&a.cnt->n_crossings, (unsigned long long)sc);
         if (scap) atomicAdd(&a.cnt->n_capped, (unsigned long long)scap);
         if (mk) atomicMax(&a.cnt->max_crossings, mk);
+    }
+}
+
+__device__ __forceinline__ int em_owner(const EmRanges &rr, long long c) {
+    for (int r = 0; r < rr.n; r++)
+        if (c >= rr.lo[r] && c < rr.lo[r + 1]) return r;
+    return -1;
+}
+
+__global__ void k_em_mig_count(EmArgs a, EmRanges rr, unsigned long long *counts) {
+    __shared__ unsigned long long sc[kEmMaxRanks];
+    for (int r = threadIdx.x; r < rr.n; r += blockDim.x) sc[r] = 0;
+    __syncthreads();
+    const unsigned long long m = *a.mig_n;
+    for (unsigned long long j = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; j < m;
+         j += (unsigned long long)gridDim.x * blockDim.x) {
+        const int o = em_owner(rr, a.mig_c[j]);
+        if (o >= 0) atomicAdd(&sc[o], 1ull);
+    }
+    __syncthreads();
+    for (int r = threadIdx.x; r < rr.n; r += blockDim.x)
+        if (sc[r]) atomicAdd(&counts[r], sc[r]);
+}
+
+__global__ void k_em_mig_pack(EmArgs a, EmRanges rr, unsigned long long *cursor,
+                              const long long *__restrict__ id, EmRecord *out, uint32_t *holes) {
+    const unsigned long long m = *a.mig_n;
+    for (unsigned long long j = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; j < m;
+         j += (unsigned long long)gridDim.x * blockDim.x) {
+        const int o = em_owner(rr, a.mig_c[j]);
+        const long long i = a.mig_i[j];
+        holes[j] = (uint32_t)i;
+        if (o < 0) continue;
+        EmRecord r;
+        for (int ax = 0; ax < 3; ax++) {
+            r.p[ax] = a.mig_p[ax * a.mig_cap + j];
+            r.d[ax] = a.mig_d[ax * a.mig_cap + j];
+            r.u[ax] = a.u[ax * a.cap + i];
+        }
+        r.w = a.w[i];
+        r.id = id ? id[i] : i;
+        r.cell = a.mig_c[j];
+        r.k = a.mig_k[j];
+        out[atomicAdd(&cursor[o], 1ull)] = r;
+    }
+}
+
+__global__ void k_em_mig_unpack(EmArgs a, long long *id, const EmRecord *__restrict__ in, long long first,
+                                long long m, double *dbuf, int32_t *kbuf) {
+    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < m;
+         t += (long long)gridDim.x * blockDim.x) {
+        const EmRecord r = in[t];
+        const long long i = first + t;
+        for (int ax = 0; ax < 3; ax++) {
+            a.off[ax * a.cap + i] = r.p[ax];
+            a.u[ax * a.cap + i] = r.u[ax];
+            dbuf[ax * m + t] = r.d[ax];
+        }
+        const_cast<double *>(a.w)[i] = r.w;
+        if (id) id[i] = r.id;
+        a.cell[i] = r.cell;
+        kbuf[t] = r.k;
     }
 }
 
@@ -624,8 +713,9 @@ __global__ void __launch_bounds__(256) k_em_move_continue(EmArgs a) {
 // ---------------------------------------------------------------------------
 __global__ void k_em_accumulate_current(const double *__restrict__ acc,
                                         const int32_t *__restrict__ c2c, long long nc, double sx,
-                                        double sy, double sz, double *__restrict__ J) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+                                        double sy, double sz, double *__restrict__ J, long long c0,
+                                        long long c1) {
+    for (long long c = c0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; c < c1;
          c += (long long)gridDim.x * blockDim.x) {
         const int *nb = c2c + 6 * c;
         const int xm = nb[0], ym = nb[2], zm = nb[4];
@@ -650,8 +740,8 @@ __global__ void k_em_accumulate_current(const double *__restrict__ acc,
 
 __global__ void k_em_advance_b(const double *__restrict__ e, double *__restrict__ b,
                                const int32_t *__restrict__ c2c, long long nc, double hx, double hy,
-                               double hz, double fdt) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+                               double hz, double fdt, long long c0, long long c1) {
+    for (long long c = c0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; c < c1;
          c += (long long)gridDim.x * blockDim.x) {
         const int *nb = c2c + 6 * c;
         const long long xp = nb[1], yp = nb[3], zp = nb[5];
@@ -667,8 +757,9 @@ __global__ void k_em_advance_b(const double *__restrict__ e, double *__restrict_
 
 __global__ void k_em_advance_e(double *__restrict__ e, const double *__restrict__ b,
                                const double *__restrict__ J, const int32_t *__restrict__ c2c,
-                               long long nc, double hx, double hy, double hz, double dt) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nc;
+                               long long nc, double hx, double hy, double hz, double dt, long long c0,
+                               long long c1) {
+    for (long long c = c0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; c < c1;
          c += (long long)gridDim.x * blockDim.x) {
         const int *nb = c2c + 6 * c;
         const long long xm = nb[0], ym = nb[2], zm = nb[4];
@@ -684,70 +775,91 @@ __global__ void k_em_advance_e(double *__restrict__ e, const double *__restrict_
 
 }  // namespace
 
+static int em_grid(long long n) { return (int)std::max(1LL, std::min<long long>((n + 255) / 256, 4096)); }
+
 cudaError_t launch_em_accumulate_current(const double *acc, const int32_t *c2c, long long nc,
-                                         const double h[3], double dt, double *J, cudaStream_t s) {
-    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
+                                         const double h[3], double dt, double *J, cudaStream_t s,
+                                         long long c0, long long c1) {
+    if (c1 < 0) c1 = nc;
     // scale 2 dt h_b h_c, formed as the oracle forms it: (2.0 * dt) * h_b * h_c
     const double sx = 2.0 * dt * h[1] * h[2], sy = 2.0 * dt * h[2] * h[0], sz = 2.0 * dt * h[0] * h[1];
-    k_em_accumulate_current<<<grid, 256, 0, s>>>(acc, c2c, nc, sx, sy, sz, J);
+    k_em_accumulate_current<<<em_grid(c1 - c0), 256, 0, s>>>(acc, c2c, nc, sx, sy, sz, J, c0, c1);
     return cudaGetLastError();
 }
 
 cudaError_t launch_em_advance_b(const double *e, double *b, const int32_t *c2c, long long nc,
-                                const double h[3], double fdt, cudaStream_t s) {
-    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
-    k_em_advance_b<<<grid, 256, 0, s>>>(e, b, c2c, nc, h[0], h[1], h[2], fdt);
+                                const double h[3], double fdt, cudaStream_t s, long long c0, long long c1) {
+    if (c1 < 0) c1 = nc;
+    k_em_advance_b<<<em_grid(c1 - c0), 256, 0, s>>>(e, b, c2c, nc, h[0], h[1], h[2], fdt, c0, c1);
     return cudaGetLastError();
 }
 
 cudaError_t launch_em_advance_e(double *e, const double *b, const double *J, const int32_t *c2c,
-                                long long nc, const double h[3], double dt, cudaStream_t s) {
-    const int grid = (int)std::max(1LL, std::min<long long>((nc + 255) / 256, 4096));
-    k_em_advance_e<<<grid, 256, 0, s>>>(e, b, J, c2c, nc, h[0], h[1], h[2], dt);
+                                long long nc, const double h[3], double dt, cudaStream_t s, long long c0,
+                                long long c1) {
+    if (c1 < 0) c1 = nc;
+    k_em_advance_e<<<em_grid(c1 - c0), 256, 0, s>>>(e, b, J, c2c, nc, h[0], h[1], h[2], dt, c0, c1);
     return cudaGetLastError();
 }
-
 
 cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
-                                  double *interp, cudaStream_t s) {
+                                  double *interp, cudaStream_t s, long long c0, long long c1) {
     const long long nc = (long long)nx * ny * nz;
-    const int grid = (int)std::min<long long>((nc + 255) / 256, 4096);
-    k_em_interpolate<<<grid > 0 ? grid : 1, 256, 0, s>>>(nx, ny, nz, e, b, interp);
+    if (c1 < 0) c1 = nc;
+    k_em_interpolate<<<em_grid(c1 - c0), 256, 0, s>>>(nx, ny, nz, e, b, interp, c0, c1);
     return cudaGetLastError();
 }
 
-template <int DEP, bool DEFER, bool QUEUE>
-static cudaError_t em_launch(const EmArgs &a, int nsm, cudaStream_t s, long long *grid_out) {
+template <int DEP, bool QUEUE>
+static cudaError_t em_launch(const EmArgs &a, int nsm, cudaStream_t s) {
     const int smem = 8 * (kEmBufBytes + (QUEUE ? kEmQBytes : 0));
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_em_move_deposit<DEP, DEFER, QUEUE>,
+        cudaError_t e = cudaFuncSetAttribute(k_em_move_deposit<DEP, QUEUE>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
     int per = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<DEP, DEFER, QUEUE>, 256, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<DEP, QUEUE>, 256, smem);
     const long long need = (a.n + 255) / 256;
     const long long grid = std::max(1LL, std::min<long long>(need, (long long)nsm * std::max(per, 1)));
-    k_em_move_deposit<DEP, DEFER, QUEUE><<<(int)grid, 256, smem, s>>>(a);
-    *grid_out = grid;
+    k_em_move_deposit<DEP, QUEUE><<<(int)grid, 256, smem, s>>>(a);
     return cudaGetLastError();
 }
 
 cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
-    const bool defer = a.work != nullptr && a.kcap > 0;
-    const bool queue = !defer && OPP_EM_QUEUE && a.kcap > 0 && a.n < (1LL << 31);
-    long long grid = 1;
-    cudaError_t e;
-    if (a.dep == 1)
-        e = defer ? em_launch<1, true, false>(a, nsm, s, &grid)
-                  : queue ? em_launch<1, false, true>(a, nsm, s, &grid) : em_launch<1, false, false>(a, nsm, s, &grid);
-    else
-        e = defer ? em_launch<0, true, false>(a, nsm, s, &grid)
-                  : queue ? em_launch<0, false, true>(a, nsm, s, &grid) : em_launch<0, false, false>(a, nsm, s, &grid);
+    const bool queue = OPP_EM_QUEUE && a.kcap > 0 && a.n < (1LL << 31);
+    if (a.dep == 1) return queue ? em_launch<1, true>(a, nsm, s) : em_launch<1, false>(a, nsm, s);
+    return queue ? em_launch<0, true>(a, nsm, s) : em_launch<0, false>(a, nsm, s);
+}
+
+cudaError_t launch_em_continue(const EmArgs &a, long long first, long long m, const double *d,
+                               const int32_t *k, int nsm, cudaStream_t s) {
+    if (m <= 0) return cudaSuccess;
+    const long long g = std::max(1LL, std::min<long long>((m + 255) / 256, (long long)nsm * 8));
+    k_em_continue<<<(int)g, 256, 0, s>>>(a, first, m, d, k);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_mig_count(const EmArgs &a, const EmRanges &rr, unsigned long long *counts,
+                                cudaStream_t s) {
+    cudaError_t e = cudaMemsetAsync(counts, 0, sizeof(unsigned long long) * rr.n, s);
     if (e != cudaSuccess) return e;
-    if (defer) k_em_move_continue<<<(int)std::min<long long>(grid, (long long)nsm * 8), 256, 0, s>>>(a);
+    k_em_mig_count<<<em_grid(a.mig_cap), 256, 0, s>>>(a, rr, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_mig_pack(const EmArgs &a, const EmRanges &rr, unsigned long long *cursor,
+                               const long long *id, EmRecord *out, uint32_t *holes, cudaStream_t s) {
+    k_em_mig_pack<<<em_grid(a.mig_cap), 256, 0, s>>>(a, rr, cursor, id, out, holes);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_em_mig_unpack(const EmArgs &a, long long *id, const EmRecord *in, long long first,
+                                 long long m, double *dbuf, int32_t *kbuf, cudaStream_t s) {
+    if (m <= 0) return cudaSuccess;
+    k_em_mig_unpack<<<em_grid(m), 256, 0, s>>>(a, id, in, first, m, dbuf, kbuf);
     return cudaGetLastError();
 }
 

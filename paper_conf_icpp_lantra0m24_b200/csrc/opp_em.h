@@ -29,17 +29,60 @@ struct EmArgs {
     int kcap;
     int dep;                   // 0: 12 reductions per segment and lane; 1: warp-aggregated
     EmCounters *cnt;
-    uint32_t *work;            // deferred particles (face crossers), capacity >= n; null: no deferral
+    // slab partition (opp_em_set_partition): cells [c0, c1) are this rank's
+    // (single domain: [0, nc)); a particle whose path enters another rank's
+    // cell stops on the face and is recorded as a migrant: its index, the face
+    // point in the new cell's offsets, the rest of its streak, the crossings
+    // so far and the new cell (mig_n == null: single domain, never happens)
+    long long c0, c1;
+    unsigned long long *mig_n;
+    uint32_t *mig_i;
+    double *mig_p, *mig_d;     // [3][mig_cap]
+    int32_t *mig_c, *mig_k;
+    long long mig_cap;
+};
+
+// One migrating particle on the wire (opp_em_move_deposit_slab): face point,
+// rest of the streak, momentum, weight, id, new cell, crossings so far.
+struct EmRecord {
+    double p[3], d[3], u[3], w;
+    long long id;
+    int32_t cell, k;
+};
+static_assert(sizeof(EmRecord) == 96, "EmRecord is 96 bytes");
+
+// Slab ranges: rank r owns cells [lo[r], lo[r + 1]).
+constexpr int kEmMaxRanks = 64;
+struct EmRanges {
+    long long lo[kEmMaxRanks + 1];
+    int n;
 };
 
 cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const double *b,
-                                  double *interp, cudaStream_t s);
+                                  double *interp, cudaStream_t s, long long c0 = 0, long long c1 = -1);
 cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s);
+// Slabs: the received particles [first, first + m) resume their walk from
+// (off, cell) with the rest of their streak d[3][m] and crossings k[m].
+cudaError_t launch_em_continue(const EmArgs &a, long long first, long long m, const double *d,
+                               const int32_t *k, int nsm, cudaStream_t s);
+// migrants -> records, grouped by destination rank (cursor[r] = first slot);
+// dest rank of a cell: the rank whose cell range [lo, hi) holds it
+cudaError_t launch_em_mig_count(const EmArgs &a, const EmRanges &rr, unsigned long long *counts,
+                                cudaStream_t s);
+cudaError_t launch_em_mig_pack(const EmArgs &a, const EmRanges &rr, unsigned long long *cursor,
+                               const long long *id, EmRecord *out, uint32_t *holes, cudaStream_t s);
+// records -> particles [first, first + m) (d, k of each into dbuf / kbuf)
+cudaError_t launch_em_mig_unpack(const EmArgs &a, long long *id, const EmRecord *in, long long first,
+                                 long long m, double *dbuf, int32_t *kbuf, cudaStream_t s);
+// (field kernels: cells [c0, c1) of the nc; c1 < 0: all)
 cudaError_t launch_em_accumulate_current(const double *acc, const int32_t *c2c, long long nc,
-                                         const double h[3], double dt, double *J, cudaStream_t s);
+                                         const double h[3], double dt, double *J, cudaStream_t s,
+                                         long long c0 = 0, long long c1 = -1);
 cudaError_t launch_em_advance_b(const double *e, double *b, const int32_t *c2c, long long nc,
-                                const double h[3], double fdt, cudaStream_t s);
+                                const double h[3], double fdt, cudaStream_t s, long long c0 = 0,
+                                long long c1 = -1);
 cudaError_t launch_em_advance_e(double *e, const double *b, const double *J, const int32_t *c2c,
-                                long long nc, const double h[3], double dt, cudaStream_t s);
+                                long long nc, const double h[3], double dt, cudaStream_t s,
+                                long long c0 = 0, long long c1 = -1);
 
 }  // namespace opp

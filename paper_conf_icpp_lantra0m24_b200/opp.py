@@ -34,6 +34,7 @@ EXPORTS = (
     "opp_field_init", "opp_field_solve", "opp_get_field_stats", "opp_field_solve_boltzmann",
     "opp_em_interpolate", "opp_em_move_deposit", "opp_em_get_stats", "opp_em_sort_by_cell",
     "opp_shuffle", "opp_em_accumulate_current", "opp_em_advance_b", "opp_em_advance_e",
+    "opp_em_set_partition", "opp_em_move_deposit_slab", "opp_em_field_step_slab",
 )
 PHASES = ("inject", "begin", "push_move_deposit", "continue", "segred", "fill", "migrate", "halo",
           "sort_count", "sort_move", "field", "em_move_deposit")
@@ -163,6 +164,10 @@ def _load():
         "opp_em_accumulate_current": (I, [P, P, P, I64, P, C.c_double, P]),
         "opp_em_advance_b": (I, [P, P, P, P, I64, P, C.c_double]),
         "opp_em_advance_e": (I, [P, P, P, P, P, I64, P, C.c_double]),
+        "opp_em_set_partition": (I, [P, I, I, I, I, I]),
+        "opp_em_move_deposit_slab": (I, [P, C.POINTER(C.c_int64), I64, P, P, P, P, P, P, P, I64, P,
+                                         C.POINTER(opp_em_params), C.POINTER(opp_em_stats)]),
+        "opp_em_field_step_slab": (I, [P, P, P, P, P, P, P, I64, P, C.c_double]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -408,3 +413,23 @@ def opp_em_advance_b(ctx, e, b, c2c, n_cells: int, h, frac_dt: float) -> None:
 
 def opp_em_advance_e(ctx, e, b, J, c2c, n_cells: int, h, dt: float) -> None:
     _ck(lib.opp_em_advance_e(ctx, _ptr(e), _ptr(b), _ptr(J), _ptr(c2c), int(n_cells), _h3(h), float(dt)))
+
+
+def opp_em_set_partition(ctx, nx: int, ny: int, nz: int, k0: int, k1: int) -> None:
+    _ck(lib.opp_em_set_partition(ctx, int(nx), int(ny), int(nz), int(k0), int(k1)))
+
+
+def opp_em_move_deposit_slab(ctx, n: int, cap: int, off, u, w, cell, pid, interp, c2c, n_cells: int, acc,
+                             params: opp_em_params, want_stats: bool = True):
+    """Device tensors (SoA columns of row stride `cap`); returns (new n, stats or None)."""
+    st = opp_em_stats() if want_stats else None
+    nn = C.c_int64(int(n))
+    _ck(lib.opp_em_move_deposit_slab(ctx, C.byref(nn), int(cap), _ptr(off), _ptr(u), _ptr(w), _ptr(cell),
+                                     _ptr(pid) if pid is not None else None, _ptr(interp), _ptr(c2c),
+                                     int(n_cells), _ptr(acc), C.byref(params), C.byref(st) if st else None))
+    return nn.value, st
+
+
+def opp_em_field_step_slab(ctx, e, b, J, acc, interp, c2c, n_cells: int, h, dt: float) -> None:
+    _ck(lib.opp_em_field_step_slab(ctx, _ptr(e), _ptr(b), _ptr(J), _ptr(acc), _ptr(interp), _ptr(c2c),
+                                   int(n_cells), _h3(h), float(dt)))
