@@ -31,6 +31,7 @@ workload.
 from __future__ import annotations
 
 import argparse
+import contextlib
 import hashlib
 import json
 import os
@@ -417,28 +418,42 @@ def run_reference_c3(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def run_ours_c3(args, rank, world):
-    """C3: one step = Move_Deposit over the whole resident population (the
-    accumulator is zeroed between steps outside the timed kernel's model).
-    N > 1: independent replicas (the periodic two-stream box is not
-    partitioned: DESIGN.md §10)."""
+def c3_rank_main(args, rank, world, group, uid, transport, stream, res):
+    """One rank of C3.  N = 1: the 40x40x60 box.  N > 1: weak scaling along z --
+    the periodic box is 40x40x(60 N), rank r owns layers [60 r, 60 (r + 1))
+    with its own seeded 750 ppc population (the two-stream perturbation
+    repeats per slab); Move_Deposit migrates the particles whose streak leaves
+    the slab and the field side exchanges ghost layers (opp_em_*_slab)."""
     import torch
     import gen.cuda as gc
+    import gen.em as ge
     from paper_conf_icpp_lantra0m24_b200.em_app import CabanaPicEM
-    from paper_conf_icpp_lantra0m24_b200 import dist as D
     from paper_conf_icpp_lantra0m24_b200 import opp as O
-    dev = int(os.environ.get("LOCAL_RANK", 0))
-    torch.cuda.set_device(dev)
-    nx, ny, nz, c2c, e, b = c3_inputs(args)
+    dev = torch.cuda.current_device()
+    nx, ny, nzl = C3["dims"]
+    nz = nzl * world
+    e, b = ge.em_fields(nx, ny, nz, C3["seed"], e_amp=C3["e_amp"], b0=C3["b0"], b_amp=C3["b_amp"])
+    c2c = ge.periodic_hex(nx, ny, nz)
     nc = nx * ny * nz
+    L = nx * ny
+    k0, k1 = rank * nzl, (rank + 1) * nzl
+    c0, c1 = k0 * L, k1 * L
+    slab = (k0, k1) if world > 1 else None
     sim = CabanaPicEM(nx, ny, nz, c2c, e, b, C3["qdt_2mc"], C3["cdt_2h"], C3["qsp"], C3["kcap"],
-                      deposit_mode=1 if args.deposit != 0 else 0, device=dev)
-    d = gc.em_two_stream(nx, ny, nz, args.ppc, C3["seed"] + rank, v0=C3["v0"], pert=C3["pert"],
+                      deposit_mode=1 if args.deposit != 0 else 0, device=dev, nranks=world, rank=rank,
+                      uid=uid, transport=transport, slab=slab, stream=stream.cuda_stream,
+                      torch_alloc=transport == 0)
+    d = gc.em_two_stream(nx, ny, nzl, args.ppc, C3["seed"] + rank, v0=C3["v0"], pert=C3["pert"],
                          vth=C3["vth"])
-    sim.set_particles(d["off"], d["u"], d["w"], d["cell"])
+    n0 = d["n"]
+    if slab is None:
+        sim.set_particles(d["off"], d["u"], d["w"], d["cell"])
+    else:
+        ids = torch.arange(n0, dtype=torch.int64, device=d["cell"].device) + rank * n0
+        sim.set_particles(d["off"], d["u"], d["w"], d["cell"] + c0, ids=ids,
+                          capacity=int(n0 * 1.05) + (1 << 16))
+        del ids
     del d
-    n = sim.n
-    stream = torch.cuda.current_stream()
     nstep = [0]
     em_field = args.field != 0      # c3 default: the field side runs every step
 
@@ -457,15 +472,15 @@ def run_ours_c3(args, rank, world):
         em_step()
     reps = []
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(dev) as clk:
-        for _ in range(max(args.reps, 1)):
+    with ClockSampler(dev) if rank == 0 else contextlib.nullcontext() as clk:
+        for rep in range(max(args.reps, 1)):
             torch.cuda.synchronize()
-            if world > 1:
-                torch.distributed.barrier()
+            group.barrier()
             torch.cuda.synchronize()
             l0 = sim.launches()
             O.opp_phase_timing(sim.ctx, True)
             O.opp_get_phase_times(sim.ctx)
+            n_start = sim.n
             e0.record(stream)
             for _ in range(args.steps):
                 em_step()
@@ -475,39 +490,147 @@ def run_ours_c3(args, rank, world):
             launches = sim.launches() - l0
             ph = O.opp_get_phase_times(sim.ctx)
             O.opp_phase_timing(sim.ctx, False)
-            pushed = n * args.steps
+            pushed = n_start * args.steps
             field_ms = ph["field"][0] if em_field else 0.0
-            if world > 1:
-                ms = D.max_over_ranks(ms)
-                field_ms = D.max_over_ranks(field_ms)
-                pushed = D.sum_over_ranks(pushed)
-                launches = D.sum_over_ranks(launches)
+            ms = group.max(f"c3ms{rep}", ms)
+            field_ms = group.max(f"c3f{rep}", field_ms)
+            pushed = group.sum(f"c3p{rep}", pushed)
+            launches = group.sum(f"c3l{rep}", launches)
             reps.append(dict(ms=ms, field_ms=field_ms, pushed=pushed, launches=launches, ph=ph,
-                             value=pushed / ((ms - field_ms) / 1e3)))
-    st = em_step(stats=True)
+                             n_local=n_start, value=pushed / ((ms - field_ms) / 1e3)))
+    out = {"reps": reps, "st": em_step(stats=True), "n": sim.n, "nc": nc,
+           "clocks": clk.summary() if rank == 0 else None}
+    if not args.no_e2e:
+        # e2e through the public API: the step's fields (this rank's layers) arrive
+        # from pinned host memory (H2D), Interpolate + Move_Deposit (+ the field
+        # side) run, this rank's accumulator is read back
+        ke = args.e2e_steps or min(args.steps, 10)
+        eh = torch.from_numpy(np.ascontiguousarray(e[:, c0:c1])).pin_memory()
+        bh = torch.from_numpy(np.ascontiguousarray(b[:, c0:c1])).pin_memory()
+        acc_h = torch.empty((c1 - c0, 12), dtype=torch.float64).pin_memory()
+        # copies on a side stream, overlapped with the previous step's compute:
+        # step s's fields are staged H2D while step s-1 runs, the accumulator
+        # is snapshotted on the device and read back while step s+1 runs
+        cs = torch.cuda.Stream()
+        e_st, b_st = torch.empty_like(eh, device=sim.dev), torch.empty_like(bh, device=sim.dev)
+        acc_snap = torch.empty((c1 - c0, 12), dtype=torch.float64, device=sim.dev)
+        staged, consumed, snapped = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
+        ev, bv = sim.e.view(3, -1)[:, c0:c1], sim.b.view(3, -1)[:, c0:c1]
+        torch.cuda.synchronize()
+        group.barrier()
+        n_e2e = sim.n
+        e0.record(stream)
+        with torch.cuda.stream(cs):
+            cs.wait_event(e0)                       # every copy inside the timed region
+            e_st.copy_(eh, non_blocking=True)
+            b_st.copy_(bh, non_blocking=True)
+            staged.record(cs)
+        for s_ in range(ke):
+            stream.wait_event(staged)
+            ev.copy_(e_st, non_blocking=True)
+            bv.copy_(b_st, non_blocking=True)
+            consumed.record(stream)
+            if s_ + 1 < ke:
+                with torch.cuda.stream(cs):
+                    cs.wait_event(consumed)
+                    e_st.copy_(eh, non_blocking=True)     # the next step's fields
+                    b_st.copy_(bh, non_blocking=True)
+                    staged.record(cs)
+            sim.interpolate()
+            em_step()
+            if s_ > 0:
+                stream.wait_event(snapped)          # the previous read-back left acc_snap
+            acc_snap.copy_(sim.acc[c0:c1], non_blocking=True)
+            done = torch.cuda.Event()
+            done.record(stream)
+            with torch.cuda.stream(cs):
+                cs.wait_event(done)
+                acc_h.copy_(acc_snap, non_blocking=True)
+                snapped.record(cs)
+        stream.wait_event(snapped)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        out["e2e"] = {"ms": group.max("c3e2e", e0.elapsed_time(e1)), "pushed": group.sum("c3e2ep", n_e2e * ke),
+                      "steps": ke, "h2d": int(eh.nbytes + bh.nbytes), "d2h": int(acc_h.nbytes)}
+    sim.close()
+    res[rank] = out
+
+
+def run_ours_c3(args, rank, world, mode):
+    """C3: one step = Move_Deposit over the whole resident population + the
+    field side (timed apart).  mode as run_ours: "single", "dist" (torchrun
+    ranks over NCCL), "loopback" (N ranks as threads on one GPU)."""
+    import torch
+    from paper_conf_icpp_lantra0m24_b200 import dist as D
+    from paper_conf_icpp_lantra0m24_b200 import opp as O
+    group = Group(world, mode)
+    uid, info = None, None
+    if mode == "dist":
+        uid = D.broadcast_bytes(O.opp_get_nccl_unique_id() if rank == 0 else None)
+        info = nccl_info(group, world)
+    elif mode == "loopback":
+        uid = os.urandom(128)
+        info = {"backend": "loopback", "ranks": world, "devices": [0]}
+    res = [None] * world
+    if mode == "loopback":
+        errs = []
+        streams = [torch.cuda.Stream() for _ in range(world)]
+
+        def worker(r):
+            try:
+                with torch.cuda.stream(streams[r]):
+                    c3_rank_main(args, r, world, group, uid, 1, streams[r], res)
+            except BaseException as ex:   # noqa: BLE001
+                errs.append((r, repr(ex)))
+                group._bar.abort()
+                raise
+
+        th = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        if errs:
+            raise SystemExit(f"loopback ranks failed: {errs}")
+    else:
+        c3_rank_main(args, rank, world, group, uid, 0, torch.cuda.current_stream(), res)
+    if rank != 0:
+        return
+    out = res[0]
+    reps = out["reps"]
+    em_field = args.field != 0
     order = sorted(range(len(reps)), key=lambda k: reps[k]["value"])
     med = reps[order[len(order) // 2]]
     ms, field_ms, pushed, launches, ph = med["ms"], med["field_ms"], med["pushed"], med["launches"], med["ph"]
     value = med["value"]          # the particle loop; the field side apart (as C2)
+    n, nc, st = med["n_local"], out["nc"], out["st"]
+    ncl = nc // world             # this rank's cells (the kernel's per-cell traffic)
     peak, peak_src = load_peaks()
     k_ms, k_cnt = ph["em_move_deposit"]
     # algorithmic bytes per launch: particle state in (off, u, w, cell = 60 B) and
     # out (off, u, cell = 52 B); per cell the interpolator (144 B), c2c (24 B)
     # and the accumulator read-modify-write (2 x 96 B)
-    bpl = 112.0 * n + (144.0 + 24.0 + 192.0) * nc
+    bpl = 112.0 * n + (144.0 + 24.0 + 192.0) * ncl
     achieved = bpl / (k_ms / max(k_cnt, 1) / 1e3) / 1e9
     tb, tsrc = traffic_for(f"c3_dep{1 if args.deposit != 0 else 0}")
+    fields = (", field side every step (AccumulateCurrent + Yee AdvanceB/E/B + Interpolate, timed apart)"
+              if em_field else ", fixed fields")
+    workload_name = C3_NAME.format(ppc=args.ppc, fields=fields)
+    if world > 1:
+        workload_name += (f"; weak scaling: global box 40x40x{60 * world}, one 60-layer z-slab per rank, "
+                          "migration + Update_Ghosts")
     line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1 if mode == "loopback" else world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": C3_NAME.format(ppc=args.ppc, fields=(
-                       ", field side every step (AccumulateCurrent + Yee AdvanceB/E/B + Interpolate, "
-                       "timed apart)" if em_field else ", fixed fields")), "mesh_cells": nc, "particles": n,
-                   "ppc": args.ppc, "deposit": "atomic_warpagg" if args.deposit != 0 else "atomic",
+        "config": {"workload": workload_name, "mesh_cells": nc, "mesh_cells_per_rank": ncl,
+                   "particles_per_rank": n, "ppc": args.ppc,
+                   "deposit": "atomic_warpagg" if args.deposit != 0 else "atomic",
                    "sort_every": args.em_sort,
-                   "l2": "inputs larger than L2 (particle state %.1f GB > 126 MB L2)" % (n * 60 / 1e9),
-                   "parallelism": f"replicas{world}" if world > 1 else "single"},
+                   "l2": "inputs larger than L2 (particle state %.1f GB per rank > 126 MB L2)" % (n * 60 / 1e9),
+                   "parallelism": (f"slab{world}" + (" (loopback: all ranks on one GPU)" if mode == "loopback"
+                                                     else "")) if world > 1 else "single",
+                   "ranks": world},
         "reps": {"values": [r["value"] for r in reps], "median": value,
                  "min": min(r["value"] for r in reps)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -522,68 +645,23 @@ def run_ours_c3(args, rank, world):
         "value_incl_field": pushed / (ms / 1e3),
         "move": {"crossings_per_particle": st["n_crossings"] / max(n, 1),
                  "max_crossings": st["max_crossings"], "capped": st["n_capped"]},
-        "clocks": clk.summary(),
+        "clocks": out["clocks"],
         "env": opp_env(),
     }
-    if not args.no_e2e:
-        # e2e through the public API: the step's fields arrive from pinned host
-        # memory (H2D), Interpolate + Move_Deposit run, the accumulator is read back
-        ke = args.e2e_steps or min(args.steps, 10)
-        eh = torch.from_numpy(e).pin_memory()
-        bh = torch.from_numpy(b).pin_memory()
-        acc_h = torch.empty((nc, 12), dtype=torch.float64).pin_memory()
-        # copies on a side stream, overlapped with the previous step's compute:
-        # step s's fields are staged H2D while step s-1 runs, the accumulator
-        # is snapshotted on the device and read back while step s+1 runs
-        cs = torch.cuda.Stream()
-        e_st, b_st = torch.empty_like(sim.e), torch.empty_like(sim.b)
-        acc_snap = torch.empty_like(sim.acc)
-        staged, consumed, snapped = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
-        torch.cuda.synchronize()
-        e0.record(stream)
-        with torch.cuda.stream(cs):
-            cs.wait_event(e0)                       # every copy inside the timed region
-            e_st.copy_(eh, non_blocking=True)
-            b_st.copy_(bh, non_blocking=True)
-            staged.record(cs)
-        for s_ in range(ke):
-            stream.wait_event(staged)
-            sim.e.copy_(e_st, non_blocking=True)
-            sim.b.copy_(b_st, non_blocking=True)
-            consumed.record(stream)
-            if s_ + 1 < ke:
-                with torch.cuda.stream(cs):
-                    cs.wait_event(consumed)
-                    e_st.copy_(eh, non_blocking=True)     # the next step's fields
-                    b_st.copy_(bh, non_blocking=True)
-                    staged.record(cs)
-            sim.interpolate()
-            em_step()
-            if s_ > 0:
-                stream.wait_event(snapped)          # the previous read-back left acc_snap
-            acc_snap.copy_(sim.acc, non_blocking=True)
-            done = torch.cuda.Event()
-            done.record(stream)
-            with torch.cuda.stream(cs):
-                cs.wait_event(done)
-                acc_h.copy_(acc_snap, non_blocking=True)
-                snapped.record(cs)
-        stream.wait_event(snapped)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        ems = e0.elapsed_time(e1)
-        ep = n * ke
-        if world > 1:
-            ems = D.max_over_ranks(ems)
-            ep = D.sum_over_ranks(ep)
-        line["e2e"] = {"value": ep / (ems / 1e3), "unit": UNIT,
-                       "h2d_bytes_per_step": int(e.nbytes + b.nbytes), "d2h_bytes_per_step": nc * 96,
-                       "steps": ke, "note": "edge E and face B from pinned host memory every step, "
-                       "opp_em_interpolate + opp_em_move_deposit, accumulator read back; copies on a "
-                       "side stream overlapped with the neighbouring steps' compute"}
-    if not args.no_cpu and world == 1 and rank == 0:
+    if info is not None:
+        line["config"]["comm"] = info
+    if "e2e" in out:
+        e2 = out["e2e"]
+        line["e2e"] = {"value": e2["pushed"] / (e2["ms"] / 1e3), "unit": UNIT,
+                       "h2d_bytes_per_step": e2["h2d"], "d2h_bytes_per_step": e2["d2h"],
+                       "steps": e2["steps"], "note": "edge E and face B of the rank's cells from pinned host "
+                       "memory every step, opp_em_interpolate + opp_em_move_deposit (+ field side), the "
+                       "rank's accumulator read back; copies on a side stream overlapped with the "
+                       "neighbouring steps' compute"}
+    if not args.no_cpu and world == 1:
         import gen.em as ge
         import oracle.em as OE
+        nx, ny, nz, c2c, e, b = c3_inputs(args)
         interp = OE.interpolate(nx, ny, nz, e, b)
         p = ge.two_stream(nx, ny, nz, 16, C3["seed"], v0=C3["v0"], pert=C3["pert"], vth=C3["vth"])
         acc = np.zeros((nc, 12))
@@ -596,9 +674,7 @@ def run_ours_c3(args, rank, world):
         line["cpu_baseline"] = {"value": 2 * p["n"] / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"{p['n']:,} particles (16/cell) of the C3 workload, 2 steps, "
                                           f"1 thread, {secs:.1f} s", **cpu_meta(pc.core)}
-    sim.close()
-    if rank == 0:
-        print(json.dumps(line), flush=True)
+    print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------- our arm (electrostatic)
@@ -993,8 +1069,13 @@ def main():
             dist.init_process_group("nccl")
         else:
             dist.init_process_group("gloo")
-    if args.config == "c3":
-        (run_reference_c3 if args.impl == "reference" else run_ours_c3)(args, rank, world)
+    if args.config == "c3" and args.impl == "reference":
+        run_reference_c3(args, rank, world)
+    elif args.config == "c3":
+        if args.loopback and args.gpus > 1:
+            run_ours_c3(args, 0, args.gpus, "loopback")
+        else:
+            run_ours_c3(args, rank, world, "dist" if world > 1 else "single")
     elif args.impl == "reference":
         run_reference(args, rank, world)
     elif args.loopback and args.gpus > 1:

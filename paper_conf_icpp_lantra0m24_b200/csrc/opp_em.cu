@@ -326,7 +326,7 @@ __device__ __forceinline__ void em_streak(const EmArgs &a, const double uu[3], d
 
 // Slabs: a cell of another rank (cells outside [c0, c1))
 __device__ __forceinline__ bool em_foreign(const EmArgs &a, int c) {
-    return a.mig_n && ((long long)c < a.c0 || (long long)c >= a.c1);
+    return (long long)c < a.c0 || (long long)c >= a.c1;
 }
 // Record migrants (warp-aggregated append): index, face point, rest of the
 // streak, new cell, crossings so far; the particle's slot becomes a hole.
@@ -391,7 +391,7 @@ constexpr int kEmBufBytes = kEmNA * kEmBufLd * 8;                   // per warp
 #define OPP_EM_MINB 3   // resident blocks per SM (80 registers); 4 spills and measured slower
 #endif
 // One move round for up to 32 queued particles (lane j takes entry head + j).
-template <int DEP>
+template <int DEP, bool SLAB>
 __device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, double *wbuf,
                                                unsigned long long &ncross, unsigned long long &ncap,
                                                unsigned &maxk) {
@@ -424,7 +424,7 @@ __device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, dou
         if (face >= 0 && k < a.kcap) {
             em_cross(p, d, q, face, c, a.c2c);
             k++;
-            if (em_foreign(a, c)) migr = true;
+            if (SLAB && em_foreign(a, c)) migr = true;
             else again = true;
         } else {
             capped = face >= 0;
@@ -435,11 +435,13 @@ __device__ __forceinline__ void em_queue_round(const EmArgs &a, EmQueue &qs, dou
             maxk = max(maxk, (unsigned)k);
         }
     }
-    em_mig_push(a, migr, i, p, d, c, k);
+    if (SLAB) em_mig_push(a, migr, i, p, d, c, k);
     qs.push(again, p, d, c, k, i);
 }
 
-template <int DEP, bool QUEUE>
+// SLAB: this rank owns cells [c0, c1); a walk entering another rank's cell
+// stops there and migrates (the single-domain instance has none of it).
+template <int DEP, bool QUEUE, bool SLAB>
 __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) {
     const unsigned FULL = 0xffffffffu, lane = threadIdx.x & 31u;
     extern __shared__ __align__(16) char em_dyn[];   // per warp: transpose buffer, then the queue
@@ -540,7 +542,7 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                 } else {
                     em_cross(p, d, q, face, c, a.c2c);
                     k++;
-                    if (em_foreign(a, c)) {   // slab: the rest of the walk is another rank's
+                    if (SLAB && em_foreign(a, c)) {   // slab: the rest of the walk is another rank's
                         migr = true;
                         moving = false;
                     } else if (QUEUE) {
@@ -550,7 +552,7 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
                 }
             }
         }
-        em_mig_push(a, migr, i, p, d, c, k);
+        if (SLAB) em_mig_push(a, migr, i, p, d, c, k);
         if (valid && !queued && !migr) {
             a.off[i] = p[0]; a.off[a.cap + i] = p[1]; a.off[2 * a.cap + i] = p[2];
             a.cell[i] = c;
@@ -560,11 +562,11 @@ __global__ void __launch_bounds__(256, OPP_EM_MINB) k_em_move_deposit(EmArgs a) 
         }
         if (QUEUE) {
             qs.push(queued, p, d, c, k, (int)i);
-            while (qs.count() >= 32) em_queue_round<DEP>(a, qs, wbuf, ncross, ncap, maxk);
+            while (qs.count() >= 32) em_queue_round<DEP, SLAB>(a, qs, wbuf, ncross, ncap, maxk);
         }
     }
     if (QUEUE)
-        while (qs.count() > 0) em_queue_round<DEP>(a, qs, wbuf, ncross, ncap, maxk);
+        while (qs.count() > 0) em_queue_round<DEP, SLAB>(a, qs, wbuf, ncross, ncap, maxk);
     const unsigned sc = __reduce_add_sync(FULL, (unsigned)ncross);
     const unsigned scap = __reduce_add_sync(FULL, (unsigned)ncap);
     const unsigned mk = __reduce_max_sync(FULL, maxk);
@@ -810,28 +812,32 @@ cudaError_t launch_em_interpolate(int nx, int ny, int nz, const double *e, const
     return cudaGetLastError();
 }
 
-template <int DEP, bool QUEUE>
+template <int DEP, bool QUEUE, bool SLAB>
 static cudaError_t em_launch(const EmArgs &a, int nsm, cudaStream_t s) {
     const int smem = 8 * (kEmBufBytes + (QUEUE ? kEmQBytes : 0));
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_em_move_deposit<DEP, QUEUE>,
+        cudaError_t e = cudaFuncSetAttribute(k_em_move_deposit<DEP, QUEUE, SLAB>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
         attr = true;
     }
     int per = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<DEP, QUEUE>, 256, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_em_move_deposit<DEP, QUEUE, SLAB>, 256, smem);
     const long long need = (a.n + 255) / 256;
     const long long grid = std::max(1LL, std::min<long long>(need, (long long)nsm * std::max(per, 1)));
-    k_em_move_deposit<DEP, QUEUE><<<(int)grid, 256, smem, s>>>(a);
+    k_em_move_deposit<DEP, QUEUE, SLAB><<<(int)grid, 256, smem, s>>>(a);
     return cudaGetLastError();
 }
 
 cudaError_t launch_em_move_deposit(const EmArgs &a, int nsm, cudaStream_t s) {
     const bool queue = OPP_EM_QUEUE && a.kcap > 0 && a.n < (1LL << 31);
-    if (a.dep == 1) return queue ? em_launch<1, true>(a, nsm, s) : em_launch<1, false>(a, nsm, s);
-    return queue ? em_launch<0, true>(a, nsm, s) : em_launch<0, false>(a, nsm, s);
+    if (a.mig_n) {   // slabs
+        if (a.dep == 1) return queue ? em_launch<1, true, true>(a, nsm, s) : em_launch<1, false, true>(a, nsm, s);
+        return queue ? em_launch<0, true, true>(a, nsm, s) : em_launch<0, false, true>(a, nsm, s);
+    }
+    if (a.dep == 1) return queue ? em_launch<1, true, false>(a, nsm, s) : em_launch<1, false, false>(a, nsm, s);
+    return queue ? em_launch<0, true, false>(a, nsm, s) : em_launch<0, false, false>(a, nsm, s);
 }
 
 cudaError_t launch_em_continue(const EmArgs &a, long long first, long long m, const double *d,

@@ -103,6 +103,8 @@ class CabanaPicEM:
 
     def sort_by_cell(self) -> None:
         """Group the particles by cell (opp_em_sort_by_cell into spare columns, then swap)."""
+        if self.slab is not None:
+            raise NotImplementedError("sort_by_cell: single domain only (the sort does not carry ids)")
         t = self.torch
         if getattr(self, "_alt", None) is None or self._alt[3].shape[0] != self.n:
             self._alt = (t.empty_like(self.off), t.empty_like(self.u), t.empty_like(self.w),
