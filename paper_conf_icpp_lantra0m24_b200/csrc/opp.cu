@@ -923,14 +923,30 @@ static int build_sort_key(opp_ctx c, const Col &cn, const Col &np, long long nc)
         bv[e] = ctr[0] * v[0] + ctr[1] * v[1] + ctr[2] * v[2];
     }
     const double h = std::cbrt(6.0 * vol / nc);   // ~ hex edge of a Kuhn-split mesh
-    std::vector<long long> ku(nc), kv(nc);
+    // Order: (tile of kSortTile x kSortTile transverse bins, layer along d,
+    // transverse bin, position along d).  A particle that drifts along d or
+    // across a bin inside its tile lands within one tile layer (~16 columns
+    // of one layer) of its old place in the sorted order, so the next sort's
+    // gathers re-read source lines still in L2; only tile-boundary crossings
+    // move far.  Plain column order (bin, then position along d) sends every
+    // transverse crossing 1 or 40 columns away: on C4 the sort 10 steps after
+    // the last costs 99 ms with column order, 56 ms with tiles of 4 (8: 99 ms;
+    // 2: 62 ms), pass 1 unchanged (scripts/probe/sort_probe.py).
+    constexpr long long kSortTile = 4;
+    std::vector<long long> ku(nc), kv(nc), kz(nc);
     for (long long e = 0; e < nc; e++) {
         ku[e] = (long long)std::floor(bu[e] / h);
         kv[e] = (long long)std::floor(bv[e] / h);
+        kz[e] = (long long)std::floor(ax[e] / h);
     }
+    auto tile = [&](long long k) { return k >= 0 ? k / kSortTile : -((-k + kSortTile - 1) / kSortTile); };
     std::vector<int32_t> order(nc);
     for (long long e = 0; e < nc; e++) order[e] = (int32_t)e;
     std::sort(order.begin(), order.end(), [&](int32_t p, int32_t q) {
+        const long long tvp = tile(kv[p]), tvq = tile(kv[q]), tup = tile(ku[p]), tuq = tile(ku[q]);
+        if (tvp != tvq) return tvp < tvq;
+        if (tup != tuq) return tup < tuq;
+        if (kz[p] != kz[q]) return kz[p] < kz[q];
         if (kv[p] != kv[q]) return kv[p] < kv[q];
         if (ku[p] != ku[q]) return ku[p] < ku[q];
         if (ax[p] != ax[q]) return ax[p] < ax[q];
@@ -1135,20 +1151,44 @@ static int sort_by_keys(opp_ctx c, PSet &ps, const int32_t *keys, const uint32_t
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        for (int h : ps.cols) {
-            Col &col = c->cols[h];
-            const size_t bpp = (size_t)col.dim * col.eb;
-            for (auto &sp : ps.spares) {
-                if (sp.bpp != bpp) continue;
-                CK(launch_sort_gather(ColDesc{col.d, ps.cap, col.eb, col.dim}, sp.ptr, ps.tail,
-                                      m.cell_start + m.nc, c->nsm * 4, c->s));
-                std::swap(col.d, sp.ptr);
-                break;
+        // one launch per column, each into its size's spare (the spare of a
+        // size used twice -- vel after pos -- is the buffer the first left)
+        std::vector<int> pending(ps.cols.begin(), ps.cols.end());
+        int groups = 0;
+        while (!pending.empty()) {
+            GatherCols g{};
+            g.cap = ps.cap;
+            std::vector<std::pair<int, size_t>> used;   // column, spare index
+            std::vector<int> rest;
+            for (int h : pending) {
+                Col &col = c->cols[h];
+                const size_t bpp = (size_t)col.dim * col.eb;
+                size_t k = ps.spares.size();
+                for (size_t q = 0; q < ps.spares.size(); q++)
+                    if (ps.spares[q].bpp == bpp) k = q;
+                bool taken = false;
+                for (auto &u : used) taken = taken || u.second == k;
+                if (k == ps.spares.size()) return fail(OPP_ERR_STATE, "sort: no spare for a column");
+                if (taken || g.n == 1) {   // one column per launch (k_sort_gather)
+                    rest.push_back(h);
+                    continue;
+                }
+                g.src[g.n] = col.d;
+                g.dst[g.n] = ps.spares[k].ptr;
+                g.dim[g.n] = col.dim;
+                g.eb[g.n] = col.eb;
+                g.n++;
+                used.push_back({h, k});
             }
+            CK(launch_sort_gather(g, ps.tail, m.cell_start + m.nc, c->nsm, c->s));
+            for (auto &u : used) std::swap(c->cols[u.first].d, ps.spares[u.second].ptr);
+            pending.swap(rest);
+            groups++;
         }
         CK(launch_sort_commit(ps.dcnt, m.cell_start + m.nc, c->s));
+        c->launches += groups;
     }
-    c->launches += 6 + (long long)ps.cols.size();
+    c->launches += 6;
     ps.holes_pending = false;
     return OPP_OK;
 }
@@ -1949,9 +1989,16 @@ extern "C" int opp_em_sort_by_cell(opp_ctx c, int64_t n, int64_t stride, const d
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
-        for (int j = 0; j < 4; j++)
-            CK(launch_sort_gather(ColDesc{(char *)in[j], stride, ebs[j], dims[j]}, out[j], es.src_of,
-                                  es.start + n_cells, c->nsm * 4, c->s));
+        for (int j = 0; j < 4; j++) {
+            GatherCols g{};
+            g.cap = stride;
+            g.src[0] = (const char *)in[j];
+            g.dst[0] = out[j];
+            g.dim[0] = dims[j];
+            g.eb[0] = ebs[j];
+            g.n = 1;
+            CK(launch_sort_gather(g, es.src_of, es.start + n_cells, c->nsm, c->s));
+        }
     }
     c->launches += 10;
     return OPP_OK;

@@ -63,6 +63,17 @@ struct ColSet {
     int n;
 };
 
+// One launch of the sort's gather: columns of equal capacity, each gathered
+// from src into its spare dst.
+struct GatherCols {
+    const char *src[kMaxCols];
+    char *dst[kMaxCols];
+    int dim[kMaxCols];
+    int eb[kMaxCols];
+    int n;
+    long long cap;
+};
+
 // Direct-hop overlay.
 struct Overlay {
     double x0[3];

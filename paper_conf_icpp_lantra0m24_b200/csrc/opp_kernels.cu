@@ -1354,25 +1354,86 @@ __device__ __forceinline__ unsigned bucket_of(const uint32_t *__restrict__ skey,
     return skey ? __ldg(skey + lc) : (unsigned)lc;
 }
 
-__global__ void k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
-                            const uint32_t *__restrict__ skey, unsigned *hist) {
+// Block-level aggregation: a block takes chunks of kSortChunk consecutive
+// particles; lanes of a warp with the same bucket form one group
+// (__match_any_sync), whose leader adds the group to a shared-memory table
+// keyed by bucket; the table leaves with ONE global atomic per (chunk,
+// bucket).  Nearly sorted storage puts a chunk in a handful of buckets, so the
+// global atomics drop from ~1 per particle (runs of equal cells are short
+// once particles have moved) to ~1 per hundred.  A group that finds no slot
+// within kSortProbe probes (random order: the shuffle, the first sort of a
+// seeded population) takes its global atomic directly.
+constexpr int kSortChunk = 2048;            // 256 threads x 8
+constexpr int kSortPer = kSortChunk / 256;
+constexpr int kSortSlots = 1024;
+constexpr int kSortProbe = 8;
+
+__device__ __forceinline__ int sort_tab_insert(int *tkey, unsigned *tcnt, int key, unsigned m,
+                                               unsigned &old) {
+    const unsigned h = ((unsigned)key * 0x9E3779B1u) >> (32 - 10);
+#pragma unroll 1
+    for (int p = 0; p < kSortProbe; p++) {
+        const int sl = (int)((h + (unsigned)p) & (kSortSlots - 1));
+        const int prev = atomicCAS(tkey + sl, -1, key);
+        if (prev == -1 || prev == key) {
+            old = atomicAdd(tcnt + sl, m);
+            return sl;
+        }
+    }
+    return -1;
+}
+
+__device__ __forceinline__ void sort_tab_clear(int *tkey, unsigned *tcnt) {
+    for (int sl = threadIdx.x; sl < kSortSlots; sl += blockDim.x) {
+        tkey[sl] = -1;
+        tcnt[sl] = 0;
+    }
+}
+
+__global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *c,
+                                                   int cell_base, const uint32_t *__restrict__ skey,
+                                                   unsigned *hist) {
+    __shared__ int tkey[kSortSlots];
+    __shared__ unsigned tcnt[kSortSlots];
     const unsigned long long n = c->n;
-    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-         i0 < n; i0 += stride) {
-        const unsigned long long i = i0 + lane_id();
-        int cell = i < n ? p2c[i] : -1;
-        int key = cell >= 0 ? cell : -2 - (int)lane_id();
-        unsigned heads;
-        int rs, rl;
-        bool head;
-        run_info(key, heads, rs, rl, head);
-        if (head && cell >= 0) atomicAdd(hist + bucket_of(skey, cell - cell_base), (unsigned)rl);
+    const unsigned lane = lane_id();
+    sort_tab_clear(tkey, tcnt);
+    __syncthreads();
+    for (unsigned long long base = (unsigned long long)blockIdx.x * kSortChunk; base < n;
+         base += (unsigned long long)gridDim.x * kSortChunk) {
+        int cell[kSortPer];
+#pragma unroll
+        for (int r = 0; r < kSortPer; r++) {
+            const unsigned long long i = base + r * 256 + threadIdx.x;
+            cell[r] = i < n ? __ldcs(p2c + i) : -1;
+        }
+#pragma unroll
+        for (int r = 0; r < kSortPer; r++) {
+            const int key = cell[r] >= 0 ? (int)bucket_of(skey, cell[r] - cell_base) : -1;
+            const unsigned m = __match_any_sync(0xffffffffu, key);
+            if (key >= 0 && (int)lane == __ffs(m) - 1) {
+                unsigned old;
+                if (sort_tab_insert(tkey, tcnt, key, __popc(m), old) < 0) atomicAdd(hist + key, (unsigned)__popc(m));
+            }
+        }
+        __syncthreads();
+        for (int sl = threadIdx.x; sl < kSortSlots; sl += blockDim.x)
+            if (tkey[sl] >= 0) {
+                atomicAdd(hist + tkey[sl], tcnt[sl]);
+                tkey[sl] = -1;
+                tcnt[sl] = 0;
+            }
+        __syncthreads();
     }
 }
 
 // Phase 1: destination slot of every particle (run heads take one atomic
-// per run of equal cells), recorded as the inverse permutation src_of.
+// per run of equal cells), recorded as the inverse permutation src_of.  The
+// cursor atomics arrive roughly in storage order, so each bucket's particles
+// keep their storage order: the gathers then read every source line in a
+// short window (a block-aggregated rank that places (chunk, bucket) groups
+// contiguously measured 1.3-1.7x slower gathers after a few steps of motion,
+// scripts/probe/sort_probe.py).
 __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
                             const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *src_of) {
     const unsigned long long n = c->n;
@@ -1395,37 +1456,55 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
 }
 
 // Phase 2, one column per launch: gather move dst[d] = src[src_of[d]] for d
-// in [0, total): the writes stream in order (full sectors, no
-// read-modify-write of partially written sectors), the reads of nearly
-// sorted data hit sectors that their neighbours in d fetched a moment ago.
-// dst is a spare buffer of the column's size that then becomes the column
-// (its old storage becomes the spare), so a sort needs one spare per column
-// size, not a second copy of every column.
+// in [0, total).  The writes stream in order with evict-first stores, so L2
+// keeps the source lines that neighbouring destinations re-read (particles
+// that moved to a nearby cell since the last sort).  The number of loads in
+// flight is kept at ~600k (4 blocks of 256 threads per SM, 4 per thread, one
+// column): a wider front (8 per thread, 8 blocks per SM, or all columns in
+// one launch) is 1.2x faster on freshly sorted data but 1.5-2x slower after
+// 5-10 steps of motion -- the source lines leave L2 before their neighbours
+// read them (scripts/probe/sort_probe.py, profiles/r02/README.md).  dst is
+// a spare buffer of the column's size that then becomes the column.
 constexpr int kSortUnroll = 4;
-template <typename T>
-__global__ void __launch_bounds__(256) k_sort_gather(const T *__restrict__ src, T *__restrict__ dst,
-                                                     int dim, long long cap,
-                                                     const uint32_t *__restrict__ src_of,
+__global__ void __launch_bounds__(256) k_sort_gather(GatherCols g, const uint32_t *__restrict__ src_of,
                                                      const unsigned *__restrict__ total_p) {
     const unsigned long long n = *total_p;
     const unsigned long long span = (unsigned long long)blockDim.x * kSortUnroll;
     for (unsigned long long b = (unsigned long long)blockIdx.x * span; b < n;
          b += (unsigned long long)gridDim.x * span) {
-        unsigned long long dd[kSortUnroll];
+        const unsigned long long d0 = b + threadIdx.x;
+        // components u with d0 + 256 u < n
+        const unsigned all = (1u << kSortUnroll) - 1u;
+        const unsigned live = d0 >= n ? 0u
+                              : (n - d0 >= span ? all : (unsigned)((1ull << ((n - d0 + 255) / 256)) - 1));
         uint32_t ss[kSortUnroll];
 #pragma unroll
-        for (int u = 0; u < kSortUnroll; u++) {
-            dd[u] = b + (unsigned long long)u * blockDim.x + threadIdx.x;
-            ss[u] = dd[u] < n ? __ldg(src_of + dd[u]) : 0u;
-        }
-        for (int e = 0; e < dim; e++) {
-            const T *sp = src + e * cap;
-            T *dp = dst + e * cap;
-            T v[kSortUnroll];
+        for (int u = 0; u < kSortUnroll; u++) ss[u] = (live >> u) & 1u ? __ldcs(src_of + d0 + u * 256) : 0u;
+#pragma unroll 1
+        for (int k = 0; k < g.n; k++) {
+            const int dim = g.dim[k], eb = g.eb[k];
+            const char *sbase = g.src[k];
+            char *dbase = g.dst[k];
+#pragma unroll 1
+            for (int e = 0; e < dim; e++) {
+                if (eb == 8) {
+                    const long long *sp = reinterpret_cast<const long long *>(sbase) + e * g.cap;
+                    long long *dp = reinterpret_cast<long long *>(dbase) + e * g.cap + d0;
+                    long long v[kSortUnroll];
 #pragma unroll
-            for (int u = 0; u < kSortUnroll; u++) v[u] = dd[u] < n ? __ldg(sp + ss[u]) : T(0);
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = (live >> u) & 1u ? __ldg(sp + ss[u]) : 0;
 #pragma unroll
-            for (int u = 0; u < kSortUnroll; u++) if (dd[u] < n) dp[dd[u]] = v[u];
+                    for (int u = 0; u < kSortUnroll; u++) if ((live >> u) & 1u) __stcs(dp + u * 256, v[u]);
+                } else {
+                    const int *sp = reinterpret_cast<const int *>(sbase) + e * g.cap;
+                    int *dp = reinterpret_cast<int *>(dbase) + e * g.cap + d0;
+                    int v[kSortUnroll];
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) v[u] = (live >> u) & 1u ? __ldg(sp + ss[u]) : 0;
+#pragma unroll
+                    for (int u = 0; u < kSortUnroll; u++) if ((live >> u) & 1u) __stcs(dp + u * 256, v[u]);
+                }
+            }
         }
     }
 }
@@ -1623,16 +1702,9 @@ cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, 
     return cudaGetLastError();
 }
 
-cudaError_t launch_sort_gather(const ColDesc &src, char *dst, const uint32_t *src_of,
-                               const unsigned *total_p, int grid, cudaStream_t s) {
-    if (src.elem_bytes == 8)
-        k_sort_gather<long long><<<grid, 256, 0, s>>>(reinterpret_cast<const long long *>(src.ptr),
-                                                      reinterpret_cast<long long *>(dst), src.dim,
-                                                      src.cap, src_of, total_p);
-    else
-        k_sort_gather<int><<<grid, 256, 0, s>>>(reinterpret_cast<const int *>(src.ptr),
-                                                reinterpret_cast<int *>(dst), src.dim, src.cap,
-                                                src_of, total_p);
+cudaError_t launch_sort_gather(const GatherCols &g, const uint32_t *src_of, const unsigned *total_p,
+                               int nsm, cudaStream_t s) {
+    k_sort_gather<<<nsm * 4, 256, 0, s>>>(g, src_of, total_p);
     return cudaGetLastError();
 }
 

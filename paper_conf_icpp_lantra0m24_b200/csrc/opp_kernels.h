@@ -36,8 +36,8 @@ cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base,
                               unsigned long long *tile_sums, int grid, cudaStream_t s);
 cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
                              unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s);
-cudaError_t launch_sort_gather(const ColDesc &src, char *dst, const uint32_t *src_of,
-                               const unsigned *total_p, int grid, cudaStream_t s);
+cudaError_t launch_sort_gather(const GatherCols &g, const uint32_t *src_of, const unsigned *total_p,
+                               int nsm, cudaStream_t s);
 cudaError_t launch_sort_commit(DevCounters *c, const unsigned *start_total, cudaStream_t s);
 
 cudaError_t launch_mig_count(const int32_t *mig_cell, const DevCounters *c, const RankRanges &rr,
