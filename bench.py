@@ -63,6 +63,9 @@ def parse(argv=None):
     ap.add_argument("--loopback", action="store_true",
                     help="with --gpus N: N slabs as N contexts on one GPU (in-process transport)")
     ap.add_argument("--n0", type=int, default=0, help="override the seeded particle count (per rank)")
+    ap.add_argument("--empty", action="store_true",
+                    help="start from an empty domain (no seeded population): with --config c2 --steps 200 "
+                         "the literal Mini-FEM-PIC protocol of PAPER.md:1502-1510 (250k injected/step)")
     ap.add_argument("--deposit", type=int, default=1, choices=[0, 1, 2],
                     help="0 atomic, 1 warp-aggregated atomic (default), 2 sort + segmented reduction")
     ap.add_argument("--deposit-cache", type=int, default=0,
@@ -73,6 +76,8 @@ def parse(argv=None):
     ap.add_argument("--ov", type=float, default=0.125, help="DH overlay spacing (mesh units)")
     ap.add_argument("--hpass", type=int, default=4)
     ap.add_argument("--sort", type=int, default=10, help="sort by cell every K steps (0 = never)")
+    ap.add_argument("--sort-lead", type=float, default=-1.0,
+                    help="sort key at x + L dt v (opp_init_params.sort_lead); default: --sort / 2 with DH, else 0")
     ap.add_argument("--sort-init", type=int, default=-1,
                     help="sort the seeded population once before the run (default: iff --sort > 0)")
     ap.add_argument("--shuffle", type=int, default=0,
@@ -108,6 +113,8 @@ def parse(argv=None):
         args.field = 1 if args.config in ("c2", "c3") else 0
     if args.axis < 0:
         args.axis = 1 if args.config == "c4" else 0
+    if args.sort_lead < 0:   # C4 pass 1 33.4 -> 32.2 ms with the key at mid-interval (lead 3 or 5)
+        args.sort_lead = args.sort / 2.0 if (args.dh and args.sort > 0 and args.config != "c3") else 0.0
     if args.config in ("c4", "c5") and args.field:
         raise SystemExit("c4 / c5 run with a fixed uniform field (SURVEY.md §8(d))")
     return args
@@ -286,6 +293,9 @@ def workload(args, world=1):
     cfg = dict(gen.CONFIGS[args.config])
     if args.n0:
         cfg["n0"] = args.n0
+    if args.empty:
+        cfg["n0_ref"] = cfg["n0"]   # the oracle sample keeps the steady state's injection ratio
+        cfg["n0"] = 0
     nx, ny, nz = cfg["dims"]
     mesh = gen.kuhn_duct(nx, ny, nz * world)
     c1E = np.array(cfg["c1E"])
@@ -299,8 +309,9 @@ def workload(args, world=1):
     name = {"c4": f"C4 Mini-FEM-PIC weak scaling: per GPU a 40x40x72-hex Kuhn slab (691,200 tets) "
                   f"with {cfg['n0']:,} particles, global duct 40x40x{72 * world}, "
                   f"{cfg['n_inj']:,} injected/step on rank 0, {field}",
-            "c2": "C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), pre-seeded steady state "
-                  "+ 250k injected/step, " + field,
+            "c2": ("C2 Mini-FEM-PIC duct 48x48x72 hex (995,328 tets), " +
+                   ("starting empty (the literal protocol, PAPER.md:1502-1510)" if args.empty
+                    else "pre-seeded steady state") + " + 250k injected/step, " + field),
             "c5": "C5 clustered deposit stress: C2 mesh, 90% of particles in 1.04% of cells",
             "c1": "C1 Mini-FEM-PIC duct 6x6x30 hex (6,480 tets)"}[args.config]
     return cfg, mesh, ef, qm, dt, cluster, name
@@ -325,7 +336,7 @@ def oracle_sample(mesh, ef, qm, dt, w, cfg, n_sample, steps, cluster, dm=None):
         init = gen.seed_particles(mesh, n_sample, cfg["seed"], cluster=cluster)
     P.append(init["pos"], init["vel"], init["cell"], init["id"])
     Q = np.zeros(mesh["n_nodes"])
-    scale = n_sample / max(cfg["n0"], 1)
+    scale = n_sample / max(cfg["n0"], cfg.get("n0_ref", 1))
     n_inj = int(round(cfg["n_inj"] * scale))
     pushed, secs = 0, 0.0
     with pinned_core() as pc:
@@ -716,11 +727,13 @@ class EsRank:
         # capacity: the seeded population + a 4% margin for the flow imbalance
         # between ranks + two steps of injection (injection precedes the push)
         cap = int(n0 * 1.04) + 2 * self.n_inj + 4096
+        if args.empty:   # the population grows by n_inj per step (no outflow before z = 72 h)
+            cap = (total + 2) * self.n_inj + 4096
         self.sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
                               direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
                               sort_every=args.sort, tma_pipeline=not args.direct,
                               sort_axis=(0.0, 0.0, 1.0) if args.axis else (0.0, 0.0, 0.0),
-                              deposit_cache=bool(args.deposit_cache),
+                              deposit_cache=bool(args.deposit_cache), sort_lead=args.sort_lead,
                               torch_alloc=transport == 0, device=stream.device.index, **kw)
         sim = self.sim
         if args.field:
@@ -968,8 +981,12 @@ def run_ours(args, rank, world, mode):
                    "hop_budget_per_pass": args.hpass,
                    "sort_every": args.sort, "shuffle_every": args.shuffle,
                    "pipeline": "direct" if args.direct else "tma",
-                   "sort_key": "axis z" if args.axis else "cell id",
-                   "l2": "inputs larger than L2 (particle state %.1f GB per rank > 126 MB L2)" % (n_avg * 60 / 1e9),
+                   "sort_key": ("axis z" if args.axis else "cell id") +
+                               (f" at x + {args.sort_lead:g} dt v" if args.sort_lead > 0 else ""),
+                   "l2": ("inputs larger than L2 (particle state %.1f GB per rank > 126 MB L2)" % (n_avg * 60 / 1e9))
+                         if not args.empty else
+                         ("particle state grows from empty (average %.2f GB per rank; > 126 MB L2 after the first "
+                          "~9 steps); the mesh data (walk lines, field, DH overlay) exceeds L2 throughout" % (n_avg * 60 / 1e9)),
                    "parallelism": f"slab{world}" + (" (loopback: all ranks on one GPU)" if mode == "loopback" else ""),
                    "mesh_global": f"{cfg['dims'][0]}x{cfg['dims'][1]}x{cfg['dims'][2] * world} hex",
                    "ranks": world},

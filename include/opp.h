@@ -117,6 +117,17 @@ typedef struct {
                                    evicted -- pays under deposit contention
                                    (clustered particles, config C5), costs
                                    otherwise; 0 = off (default)     */
+    double sort_lead;           /* periodic sort (sort_every > 0) keyed at the
+                                   ballistic extrapolation x + sort_lead*dt*v of each
+                                   particle (the DH overlay's tet of that point, else
+                                   the particle's cell) instead of its cell: the
+                                   order is then best sort_lead steps after the sort
+                                   (sort_every/2 centres it on the interval) rather
+                                   than right after it.  The order of the set is
+                                   implementation-defined (an
+                                   auxiliary sort; reading S10), so results
+                                   do not depend on it.  Needs direct_hop != 0;
+                                   0 = key at the current cell (default)            */
 } opp_init_params;
 
 /* Per-step arguments of opp_push_move_deposit. */

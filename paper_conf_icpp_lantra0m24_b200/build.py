@@ -48,7 +48,10 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
     objs = []
-    os.makedirs(os.path.join(ROOT, "build"), exist_ok=True)
+    # objects of an alternative build (OPP_LIB_OUT) live apart from the in-tree library's
+    odir = os.path.join(ROOT, "build") if "OPP_LIB_OUT" not in os.environ else \
+        os.path.join(ROOT, "build", os.path.splitext(os.path.basename(LIB))[0])
+    os.makedirs(odir, exist_ok=True)
     nccl = _nccl_dir()
     extra, link = [], []
     if nccl:
@@ -56,7 +59,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         link = ["-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
                 "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     for src in SOURCES:
-        obj = os.path.join(ROOT, "build", src.replace(".cu", ".o"))
+        obj = os.path.join(odir, src.replace(".cu", ".o"))
         cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:

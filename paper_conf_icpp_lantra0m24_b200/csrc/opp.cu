@@ -93,6 +93,7 @@ struct PSet {
     std::vector<Spare> spares;
     long long spare_cap = 0;
     long long steps = 0;         // pushes so far (drives sort_every)
+    bool pcell_valid = false;    // ps.head holds the predicted sort cells of the last pass
 };
 
 struct Set {
@@ -270,7 +271,10 @@ static int col_check(opp_ctx c, int h) {
 
 // Consecutive 256-particle tiles a block of the fused kernel visits in a row
 // (TileMap): runs of adjacent cells per SM for L1 reuse of the walk lines.
-constexpr int kTileGroup = 16;
+#ifndef OPP_TILE_GROUP
+#define OPP_TILE_GROUP 16
+#endif
+constexpr int kTileGroup = OPP_TILE_GROUP;
 
 static int grid_for(opp_ctx c, long long n, int cap_mult = 8) {
     long long g = (n + 255) / 256;
@@ -322,6 +326,8 @@ extern "C" int opp_init(const opp_init_params *params, opp_ctx *out) {
         return fail(OPP_ERR_ARG, "hop_budget_per_pass and hop_cap must be >= 0");
     if (params->deposit_mode < 0 || params->deposit_mode > OPP_DEP_AUTO)
         return fail(OPP_ERR_ARG, "bad deposit_mode %d", params->deposit_mode);
+    if (!(params->sort_lead >= 0.0))
+        return fail(OPP_ERR_ARG, "sort_lead must be >= 0");
     if (params->direct_hop < 0 || params->direct_hop > 2)
         return fail(OPP_ERR_ARG, "bad direct_hop %d (0, 1 or 2)", params->direct_hop);
     if ((params->alloc == nullptr) != (params->free == nullptr))
@@ -767,6 +773,7 @@ static int grow(opp_ctx c, PSet &ps, long long extra) {
     ps.holes = tmp.holes; ps.work = tmp.work; ps.head = tmp.head; ps.tail = tmp.tail;
     ps.work_hops = tmp.work_hops; ps.sr_cell = tmp.sr_cell; ps.sr_val = tmp.sr_val;
     ps.mig = tmp.mig; ps.mig_cell = tmp.mig_cell; ps.mig_hops = tmp.mig_hops;
+    ps.pcell_valid = false;   // the fill lists are not carried over
     free_spares(c, ps);
     ps.cap = ncap;
     return OPP_OK;
@@ -1136,6 +1143,8 @@ static int ensure_spares(opp_ctx c, PSet &ps) {
     return OPP_OK;
 }
 
+static int p2c_of(opp_ctx c, PSet &ps);
+
 // Counting sort of the set by `keys` (the p2c map, or shuffle keys): count,
 // scan, rank (inverse permutation in ps.tail), then one gather per column
 // into the spare of its size, which becomes the column.  Drops holes.
@@ -1144,10 +1153,15 @@ static int sort_by_keys(opp_ctx c, PSet &ps, const int32_t *keys, const uint32_t
     TRY(ensure_spares(c, ps));
     {
         PhaseScope ph(c, OPP_PH_SORT_COUNT);
+        // the predicted sort cells of the last pass (opp_init_params.sort_lead),
+        // only for the periodic sort by cell right after that pass
+        const int32_t *pcell = (ps.pcell_valid && keys == (const int32_t *)c->cols[p2c_of(c, ps)].d)
+                                   ? (const int32_t *)ps.head : nullptr;
+        ps.pcell_valid = false;
         CK(launch_sort_count(keys, ps.dcnt, c->cell_base, m.nc, skey, m.cell_hist, m.cell_start,
-                             m.tile_sums, grid_for(c, ps.n_ub, 8), c->s));
+                             m.tile_sums, grid_for(c, ps.n_ub, 8), c->s, pcell));
         CK(launch_sort_rank(keys, ps.dcnt, c->cell_base, skey, m.cell_start, ps.tail,
-                            grid_for(c, ps.n_ub, 8), c->s));
+                            grid_for(c, ps.n_ub, 8), c->s, pcell, m.nc));
     }
     {
         PhaseScope ph(c, OPP_PH_SORT_MOVE);
@@ -1439,11 +1453,22 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.w = prm->weight;
     a.cell_base = c->cell_base;
     a.n_cells = (int)m.nc;
+    a.n_nodes = (int)nn;
     a.hpass = c->p.hop_budget_per_pass;
     a.hcap = c->p.hop_cap;
     a.tile_group = kTileGroup;
     a.dcache = c->p.deposit_cache != 0;
     a.ov = m.ov;
+    // the step before a periodic sort records each particle's predicted sort
+    // cell in the fill's head list (free until the next fill; the sort
+    // replaces that fill)
+    const bool sort_next = c->p.sort_every > 0 && (ps.steps + 1) % c->p.sort_every == 0;
+    ps.pcell_valid = false;
+    if (sort_next && c->p.sort_lead > 0 && c->p.direct_hop != 0 && prm->fill_inline) {
+        a.pcell = (int32_t *)ps.head;
+        a.lead_dt = c->p.sort_lead * prm->dt;
+        ps.pcell_valid = true;
+    }
     const int dep = c->p.deposit_mode;
     const int dh = c->p.direct_hop;
     const bool multi = c->p.nranks > 1;

@@ -116,6 +116,10 @@ struct StepArgs {
     int tile_group;            // consecutive 256-particle tiles per block visit (>= 1)
     int dcache;                // per-warp node-charge cache (opp_init_params.deposit_cache)
     Overlay ov;
+    int n_nodes;               // local nodes (bounds of Q; checked builds)
+    int32_t *pcell;            // non-null on the step before a sort: the sort-key cell of
+                               // every pushed particle (overlay tet of x + lead_dt v, -1 none)
+    double lead_dt;
 };
 
 // Slab partition: rank r owns global cells [lo[r], hi[r]).

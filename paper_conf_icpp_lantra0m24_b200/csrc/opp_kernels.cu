@@ -15,8 +15,22 @@
 #include "opp_kernels.h"
 
 #include <algorithm>
+#include <cassert>
 #include <cstddef>
 #include <climits>
+
+// OPP_CHECKED=1 (a verification build, tests/test_gpu_bounds.py): device
+// asserts on every index the particle loop, the sort and the fill compute
+// (cells, nodes, overlay slots, particle and list indices).  compute-sanitizer
+// is closed on the GPU pool; this build stands in for its memcheck.
+#ifndef OPP_CHECKED
+#define OPP_CHECKED 0
+#endif
+#if OPP_CHECKED
+#define OPP_CHECK(c) assert(c)
+#else
+#define OPP_CHECK(c) ((void)0)
+#endif
 
 namespace opp {
 
@@ -92,6 +106,8 @@ __device__ __forceinline__ long long ov_slot(const Overlay &ov, int ix, int iy, 
     return ov.compact ? ov_slot16(ov, ix, iy, iz) : ov_slot32(ov, ix, iy, iz);
 }
 __device__ __forceinline__ int ov_value(const Overlay &ov, long long slot) {
+    OPP_CHECK(slot >= 0 && slot < (ov.compact ? 64ll * ov.nbc[0] * ov.nbc[1] * ov.nbc[2]
+                                              : 32ll * ov.nb[0] * ov.nb[1] * ov.nb[2]));
     if (ov.compact) {   // the two loads are independent: one round trip
         const int o = __ldg(ov.off + slot);
         const int b = __ldg(ov.base + (slot >> 6));
@@ -152,6 +168,7 @@ __device__ __forceinline__ int walk_from(const StepArgs &a, int &cell, Line L, d
         }
         cell = nb;
         hops++;
+        OPP_CHECK((unsigned)(cell - a.cell_base) < (unsigned)a.n_cells);
         L = load_line(a.lines, cell - a.cell_base);
     }
 }
@@ -255,6 +272,9 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepAr
     // 1e-10 relative charge tolerance; the group's charge n w is conserved
     // exactly; C4 pass 1 30.95 -> 30.74 ms)
     if (lead) v0 = sub(mul((double)__popc(peers), a.w), add(add(v1, v2), v3));
+    OPP_CHECK(!lead || (unsigned)(key - a.cell_base) < (unsigned)a.n_cells);
+    OPP_CHECK(!lead || dc || ((unsigned)cn.x < (unsigned)a.n_nodes && (unsigned)cn.y < (unsigned)a.n_nodes &&
+                              (unsigned)cn.z < (unsigned)a.n_nodes && (unsigned)cn.w < (unsigned)a.n_nodes));
     if (!dc) {
         if (lead) red4(Q, cn, v0, v1, v2, v3);
         return;
@@ -296,6 +316,7 @@ __device__ __forceinline__ void deposit(const StepArgs &a, bool done, int cell, 
                                         DepCache *dc = nullptr) {
     double v0 = mul(w, l0), v1 = mul(w, l1), v2 = mul(w, l2), v3 = mul(w, l3);
     if (DEP == 0) {
+        OPP_CHECK(!done || (unsigned)(cell - a.cell_base) < (unsigned)a.n_cells);
         if (done) red4(a.Q, line_c2n(a.lines, cell - a.cell_base), v0, v1, v2, v3);
         return;
     }
@@ -312,6 +333,7 @@ __device__ __forceinline__ void sr_store(const StepArgs &a, bool write, bool don
                                          int cell, double w, double l0, double l1, double l2,
                                          double l3) {
     if (!write) return;
+    OPP_CHECK(i < (unsigned long long)a.cap && (!done || (unsigned)(cell - a.cell_base) < (unsigned)a.n_cells));
     a.sr_cell[i] = done ? cell - a.cell_base : -1;
     if (done) {
         a.sr_val[i] = mul(w, l0);
@@ -447,6 +469,7 @@ struct WarpRing {
     uint32_t *va;          // shared ring of values
     int32_t *vb;           // optional second value (hop counts), may be null
     unsigned head, tail;   // warp-uniform
+    long long cap;         // length of the global list (checked builds)
 };
 struct Appends {
     WarpRing holes, work;
@@ -475,6 +498,7 @@ __device__ __forceinline__ void ring_flush(WarpRing &r, unsigned long long *coun
         base = __shfl_sync(0xffffffffu, base, 0);
         if (lane < k) {
             const unsigned sl = (r.head + lane) & (kRing - 1);
+            OPP_CHECK(base + lane < (unsigned long long)r.cap);
             ga[base + lane] = r.va[sl];
             if (gb) gb[base + lane] = r.vb[sl];
         }
@@ -503,6 +527,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     int spec_val = -1;
     if (valid) {
         const int lc = cell - a.cell_base;
+        OPP_CHECK((unsigned)lc < (unsigned)a.n_cells && i < (unsigned long long)a.cap);
         if (!LATE) L = load_line(a.lines, lc);
         // gather the cell-constant field, leap-frog push (569-583, 1576-1590)
         // DH: the overlay entry of the drift-only position x + v dt is
@@ -532,6 +557,14 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
         // position and velocity are final now: store them before the walk
         a.pos[i] = x; a.pos[a.cap + i] = y; a.pos[2 * a.cap + i] = z;
         a.vel[i] = vx; a.vel[a.cap + i] = vy; a.vel[2 * a.cap + i] = vz;
+        // the next sort's key (opp_init_params.sort_lead; only on the step
+        // before a sort): the overlay tet of the ballistic extrapolation
+        // x + lead_dt v (-1 outside the overlay or its mesh)
+        if (DH != 0 && a.pcell) {
+            const long long g = dh_slot(a.ov, add(x, mul(vx, a.lead_dt)), add(y, mul(vy, a.lead_dt)),
+                                        add(z, mul(vz, a.lead_dt)));
+            a.pcell[i] = g >= 0 ? ov_value(a.ov, g) : -1;
+        }
         if (OPP_LADDER == 1 || OPP_LADDER == 2) valid = false;
     }
     if (valid) {
@@ -540,6 +573,7 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
             int v = g == spec_slot ? spec_val : (g >= 0 ? ov_value(a.ov, g) : -1);
             if (g < 0) v = -1;
             const int sc = v >= 0 ? v : cell;
+            OPP_CHECK((unsigned)(sc - a.cell_base) < (unsigned)a.n_cells);
             if (sc != cell) {
                 cell = sc;
                 if (!LATE) L = load_line(a.lines, sc - a.cell_base);
@@ -773,9 +807,9 @@ __global__ void __launch_bounds__(kTiledThreads, kMinBlocks) k_push_move_deposit
     Appends ap;
     {
         char *rb = smem + kRingBase + (size_t)warp * kRingBytesPerWarp;
-        ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u};
+        ap.holes = WarpRing{reinterpret_cast<uint32_t *>(rb), nullptr, 0u, 0u, a.cap};
         ap.work = WarpRing{reinterpret_cast<uint32_t *>(rb + 4 * kRing),
-                           reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u};
+                           reinterpret_cast<int32_t *>(rb + 8 * kRing), 0u, 0u, a.cap};
     }
     DepCache dcache;
     DepCache *dcp = nullptr;
@@ -850,7 +884,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
     unsigned long long cur = gstart;                              // next unclaimed entry
     unsigned long long gend = gstart + 32 < nw ? gstart + 32 : nw;
     __shared__ uint32_t hring[8][kRing];
-    WarpRing hr{hring[threadIdx.x >> 5], nullptr, 0u, 0u};
+    WarpRing hr{hring[threadIdx.x >> 5], nullptr, 0u, 0u, a.cap};
     Tally t;
     bool active = false, more = gstart < nw;
     unsigned long long i = 0;
@@ -885,8 +919,10 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
                 }
             }
             if (!active && q != ~0ull) {
+                OPP_CHECK(q < (unsigned long long)a.cap);
                 i = a.work[q];
                 hops = a.work_hops[q];
+                OPP_CHECK(i < (unsigned long long)a.cap);
                 x = a.pos[i]; y = a.pos[a.cap + i]; z = a.pos[2 * a.cap + i];
                 cell = a.p2c[i];
                 L = load_line(a.lines, cell - a.cell_base);
@@ -914,6 +950,7 @@ __global__ void __launch_bounds__(256, 4) k_walk_refill(StepArgs a) {
                 } else {
                     cell = nb;
                     hops++;
+                    OPP_CHECK((unsigned)(nb - a.cell_base) < (unsigned)a.n_cells);
                     L = load_line(a.lines, nb - a.cell_base);
                 }
             }
@@ -1011,6 +1048,7 @@ __global__ void k_fill_move(ColSet cols, DevCounters *c, const uint32_t *__restr
     for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
          k += (unsigned long long)gridDim.x * blockDim.x) {
         const unsigned long long d = head[k], s = tail[k];
+        OPP_CHECK(d < (unsigned long long)cols.c[0].cap && s < (unsigned long long)cols.c[0].cap);
         for (int j = 0; j < cols.n; j++) {
             const ColDesc cd = cols.c[j];
             for (int e = 0; e < cd.dim; e++) {
@@ -1351,6 +1389,7 @@ __global__ void __launch_bounds__(1024) k_scan_apply(const unsigned *__restrict_
 // Sort bucket of a cell: its locality key (see opp_init_params.sort_axis) or
 // the local cell index.
 __device__ __forceinline__ unsigned bucket_of(const uint32_t *__restrict__ skey, int lc) {
+    OPP_CHECK(lc >= 0);
     return skey ? __ldg(skey + lc) : (unsigned)lc;
 }
 
@@ -1390,7 +1429,21 @@ __device__ __forceinline__ void sort_tab_clear(int *tkey, unsigned *tcnt) {
     }
 }
 
-__global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p2c, const DevCounters *c,
+// Sort cell of particle i: its cell, or the predicted cell the last pass
+// recorded (opp_init_params.sort_lead) when that is a local cell; holes stay
+// holes.  Both sort passes use the same rule, so the key is consistent.
+__device__ __forceinline__ int sort_cell(const int32_t *__restrict__ p2c, const int32_t *__restrict__ pcell,
+                                         unsigned long long i, int cell_base, long long nc) {
+    int cell = __ldcs(p2c + i);
+    if (pcell && cell >= 0) {
+        const int q = __ldcs(pcell + i);
+        if ((unsigned long long)(unsigned)(q - cell_base) < (unsigned long long)nc) cell = q;
+    }
+    return cell;
+}
+
+__global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p2c, const int32_t *__restrict__ pcell,
+                                                   long long nc, const DevCounters *c,
                                                    int cell_base, const uint32_t *__restrict__ skey,
                                                    unsigned *hist) {
     __shared__ int tkey[kSortSlots];
@@ -1405,11 +1458,12 @@ __global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p
 #pragma unroll
         for (int r = 0; r < kSortPer; r++) {
             const unsigned long long i = base + r * 256 + threadIdx.x;
-            cell[r] = i < n ? __ldcs(p2c + i) : -1;
+            cell[r] = i < n ? sort_cell(p2c, pcell, i, cell_base, nc) : -1;
         }
 #pragma unroll
         for (int r = 0; r < kSortPer; r++) {
             const int key = cell[r] >= 0 ? (int)bucket_of(skey, cell[r] - cell_base) : -1;
+            OPP_CHECK(key < 0 || (nc == 0 || key < nc));
             const unsigned m = __match_any_sync(0xffffffffu, key);
             if (key >= 0 && (int)lane == __ffs(m) - 1) {
                 unsigned old;
@@ -1434,14 +1488,15 @@ __global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p
 // short window (a block-aggregated rank that places (chunk, bucket) groups
 // contiguously measured 1.3-1.7x slower gathers after a few steps of motion,
 // scripts/probe/sort_probe.py).
-__global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *c, int cell_base,
+__global__ void k_sort_rank(const int32_t *__restrict__ p2c, const int32_t *__restrict__ pcell, long long nc,
+                            const DevCounters *c, int cell_base,
                             const uint32_t *__restrict__ skey, unsigned *cursor, uint32_t *src_of) {
     const unsigned long long n = c->n;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
          i0 < n; i0 += stride) {
         const unsigned long long i = i0 + lane_id();
-        int cell = i < n ? p2c[i] : -1;
+        int cell = i < n ? sort_cell(p2c, pcell, i, cell_base, nc) : -1;
         int key = cell >= 0 ? cell : -2 - (int)lane_id();
         unsigned heads;
         int rs, rl;
@@ -1451,6 +1506,7 @@ __global__ void k_sort_rank(const int32_t *__restrict__ p2c, const DevCounters *
         if (head && cell >= 0)
             base = atomicAdd(cursor + bucket_of(skey, cell - cell_base), (unsigned)rl);
         base = __shfl_sync(0xffffffffu, base, rs);
+        OPP_CHECK(cell < 0 || base + (lane_id() - rs) < n);
         if (cell >= 0) src_of[base + (lane_id() - rs)] = (uint32_t)i;
     }
 }
@@ -1480,6 +1536,8 @@ __global__ void __launch_bounds__(256) k_sort_gather(GatherCols g, const uint32_
         uint32_t ss[kSortUnroll];
 #pragma unroll
         for (int u = 0; u < kSortUnroll; u++) ss[u] = (live >> u) & 1u ? __ldcs(src_of + d0 + u * 256) : 0u;
+#pragma unroll
+        for (int u = 0; u < kSortUnroll; u++) OPP_CHECK(ss[u] < (unsigned long long)g.cap);
 #pragma unroll 1
         for (int k = 0; k < g.n; k++) {
             const int dim = g.dim[k], eb = g.eb[k];
@@ -1686,19 +1744,21 @@ cudaError_t launch_shuffle_keys(const int32_t *p2c, const DevCounters *c, unsign
 
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
-                              unsigned long long *tile_sums, int grid, cudaStream_t s) {
+                              unsigned long long *tile_sums, int grid, cudaStream_t s,
+                              const int32_t *pcell) {
     cudaError_t e = cudaMemsetAsync(hist, 0, sizeof(unsigned) * (nc + 1), s);
     if (e != cudaSuccess) return e;
-    k_cell_hist<<<grid, 256, 0, s>>>(p2c, c, cell_base, skey, hist);
+    k_cell_hist<<<grid, 256, 0, s>>>(p2c, pcell, nc, c, cell_base, skey, hist);
     return scan_exclusive(hist, start, nc + 1, tile_sums, s);
 }
 
 cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
-                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s) {
+                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s,
+                             const int32_t *pcell, long long nc) {
     // the scan left the total in start[nc]; the rank pass consumes start[] as
     // cursors but never touches start[nc].  One thread per particle: every
     // warp waits on its cursor atomics once, so the round trips overlap.
-    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, c, cell_base, skey, start, src_of);
+    k_sort_rank<<<rank_grid, 256, 0, s>>>(p2c, pcell, nc, c, cell_base, skey, start, src_of);
     return cudaGetLastError();
 }
 

@@ -33,9 +33,12 @@ cudaError_t launch_shuffle_keys(const int32_t *p2c, const DevCounters *c, unsign
                                 long long nb, int cell_base, int32_t *keys, int grid, cudaStream_t s);
 cudaError_t launch_sort_count(const int32_t *p2c, DevCounters *c, int cell_base, long long nc,
                               const uint32_t *skey, unsigned *hist, unsigned *start,
-                              unsigned long long *tile_sums, int grid, cudaStream_t s);
+                              unsigned long long *tile_sums, int grid, cudaStream_t s,
+                              const int32_t *pcell = nullptr);
+// pcell: optional predicted sort cell per particle (StepArgs::pcell); nc: local cells
 cudaError_t launch_sort_rank(const int32_t *p2c, DevCounters *c, int cell_base, const uint32_t *skey,
-                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s);
+                             unsigned *start, uint32_t *src_of, int rank_grid, cudaStream_t s,
+                             const int32_t *pcell = nullptr, long long nc = 0);
 cudaError_t launch_sort_gather(const GatherCols &g, const uint32_t *src_of, const unsigned *total_p,
                                int nsm, cudaStream_t s);
 cudaError_t launch_sort_commit(DevCounters *c, const unsigned *start_total, cudaStream_t s);

@@ -55,7 +55,8 @@ class opp_init_params(C.Structure):
                 ("hop_budget_per_pass", C.c_int), ("hop_cap", C.c_int),
                 ("allow_growth", C.c_int), ("sort_every", C.c_int),
                 ("tma_pipeline", C.c_int), ("transport", C.c_int),
-                ("sort_axis", C.c_double * 3), ("deposit_cache", C.c_int)]
+                ("sort_axis", C.c_double * 3), ("deposit_cache", C.c_int),
+                ("sort_lead", C.c_double)]
 
 
 class opp_step_params(C.Structure):

@@ -16,12 +16,12 @@ import gen  # noqa: E402
 from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic  # noqa: E402
 
 
-def main(dep: int, dh: int):
+def main(dep: int, dh: int, lead: float = 0.0):
     mesh = gen.kuhn_duct(4, 4, 12, jitter=0.2, seed=3)
     ef = np.random.default_rng(3).uniform(-2e-3, 2e-3, (mesh["n_cells"], 3))
     init = gen.seed_particles(mesh, 20_000, 3, drift=0.4, spread=0.1)
     sim = MiniFemPic(mesh, ef, torch_alloc=False, deposit_mode=dep, direct_hop=dh, overlay_spacing=0.25,
-                     sort_every=2, hop_budget=2)
+                     sort_every=2, hop_budget=2, sort_lead=lead if dh else 0.0)
     sim.inject(init)
     for s in range(3):
         sim.inject(gen.inject_batch(mesh, s, 300, 3, id_base=20_000))
@@ -33,4 +33,5 @@ def main(dep: int, dh: int):
 
 
 if __name__ == "__main__":
-    main(int(sys.argv[1]) if len(sys.argv) > 1 else 1, int(sys.argv[2]) if len(sys.argv) > 2 else 1)
+    main(int(sys.argv[1]) if len(sys.argv) > 1 else 1, int(sys.argv[2]) if len(sys.argv) > 2 else 1,
+         float(sys.argv[3]) if len(sys.argv) > 3 else 0.0)

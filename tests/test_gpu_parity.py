@@ -186,6 +186,48 @@ def test_c1_parity_with_periodic_sort(dep, sort_every, axis):
            sort_axis=(0.0, 0.0, 1.0) if axis else (0.0, 0.0, 0.0))
 
 
+@pytest.mark.parametrize("dep,sort_every,lead,axis", [(1, 2, 1.0, 1), (0, 3, 1.5, 0), (2, 2, 4.0, 1), (1, 1, 2.0, 0)])
+def test_c1_parity_with_predicted_sort_key(dep, sort_every, lead, axis):
+    """opp_init_params.sort_lead: the periodic sort keys each particle by the
+    overlay tet of its ballistic extrapolation x + lead dt v (recorded by the
+    pass before the sort).  Only the storage order changes, so every result
+    keyed by id equals the oracle's (DH both sides; the key never reaches the
+    walk)."""
+    mesh, ef, init, inject, steps = c1_case()
+    rep, ost, gst = _check(mesh, ef, init, inject, steps, deposit_mode=dep, dh=1, overlay_spacing=0.25,
+                           sort_every=sort_every, sort_lead=lead,
+                           sort_axis=(0.0, 0.0, 1.0) if axis else (0.0, 0.0, 0.0))
+    assert [s["total_hops"] for s in gst] == [s["total_hops"] for s in ost]
+
+
+def test_predicted_sort_key_orders_by_extrapolated_cell():
+    """After a sort step with sort_lead > 0 the storage order is the order of
+    the cells of x + lead dt v (by the overlay), not of the current cells."""
+    import oracle
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    mesh, ef, init, inject, steps = c1_case(n0=50_000, n_inj=0, steps=1)
+    sim = MiniFemPic(mesh, ef, direct_hop=1, overlay_spacing=0.25, sort_every=2, sort_lead=3.0)
+    sim.inject(init)
+    for _ in range(2):   # the second step records the key and sorts
+        sim.step(DT, C1, W)
+    raw = sim.particles(sort_by_id=False)
+    box = mesh["box"]
+    n = [int(np.ceil((box[2 * k + 1] - box[2 * k]) / 0.25)) for k in range(3)]
+    x0 = np.array([box[0], box[2], box[4]])
+    omap = oracle.Mesh.from_gen(mesh).build_overlay(x0, 0.25, n)   # [gx + n0 (gy + n1 gz)]
+    xp = raw["pos"] + raw["vel"] * (3.0 * DT)
+    t = (xp - x0) * (1.0 / 0.25)
+    inside = np.all(t >= 0.0, axis=1)
+    g = np.floor(np.where(inside[:, None], t, 0.0)).astype(np.int64)
+    inside &= np.all(g < np.array(n), axis=1)
+    g = np.where(inside[:, None], g, 0)
+    key = np.where(inside, omap[g[:, 0] + n[0] * (g[:, 1] + n[1] * g[:, 2])], -1)
+    key = np.where(key >= 0, key, raw["cell"])
+    assert np.all(np.diff(key) >= 0)
+    assert np.any(key != raw["cell"])
+    sim.close()
+
+
 def test_sort_by_cell_orders_and_preserves():
     from paper_conf_icpp_lantra0m24_b200 import opp as O
     from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
