@@ -233,7 +233,11 @@ int opp_inject(opp_ctx ctx, opp_set parts, int64_t n, int ncols, const int32_t *
  * cell_ef: cell dat dim 3 OPP_REAL; node_charge: node dat dim 1 OPP_REAL.
  * Between this call and opp_fill_holes the particle dats contain holes
  * (opp_get_dat returns OPP_ERR_STATE) unless params->fill_inline.
- * stats may be NULL (no host synchronisation). */
+ * stats may be NULL (no host synchronisation).
+ * A particle whose p2c entry is not one of this rank's cells (bad input to
+ * opp_inject / opp_set_dat) is dropped as a hole without any memory access
+ * through it; the next call that reads the step statistics (this one with
+ * stats != NULL, or opp_get_step_stats) returns OPP_ERR_ARG once. */
 int opp_push_move_deposit(opp_ctx ctx, opp_set parts, opp_dat pos, opp_dat vel, opp_map p2c,
                           opp_map c2c, opp_map c2n, opp_dat node_pos, opp_dat cell_ef,
                           opp_dat node_charge, const opp_step_params *params,

@@ -1402,6 +1402,10 @@ static int read_stats(opp_ctx c, PSet &ps, opp_step_stats *stats) {
         ps.n_ub = (long long)h.n;
         ps.n_exact = true;
     }
+    if (h.err_flags & 4u) {
+        CK(cudaMemsetAsync(&ps.dcnt->err_flags, 0, sizeof(unsigned), c->s));
+        return fail(OPP_ERR_ARG, "particles whose cell is not a cell of this rank were dropped at the push");
+    }
     return OPP_OK;
 }
 

@@ -525,6 +525,13 @@ __device__ __forceinline__ void pmd_body(const StepArgs &a, bool valid, unsigned
     Line L;
     long long spec_slot = -1;
     int spec_val = -1;
+    if (valid && (unsigned)(cell - a.cell_base) >= (unsigned)a.n_cells) {
+        // not one of this rank's cells (bad input): the particle is dropped
+        // as a hole and the step reports OPP_ERR_ARG (include/opp.h)
+        valid = false;
+        status = ST_REMOVE;
+        atomicOr(&a.cnt->err_flags, 4u);
+    }
     if (valid) {
         const int lc = cell - a.cell_base;
         OPP_CHECK((unsigned)lc < (unsigned)a.n_cells && i < (unsigned long long)a.cap);
