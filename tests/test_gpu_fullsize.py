@@ -94,3 +94,96 @@ def test_c2_full_size_sampled():
     assert ex.max() <= 1e-12 and ev.max() <= 1e-12
     assert common.size > 19_000 and len(excl) <= 5
     assert ost["n_removed"] >= 0
+
+
+def test_c4_full_size_sampled():
+    """BASELINE.json configs[3] per GPU at full size in bench.py's default
+    launch configuration (40x40x72 Kuhn slab = 691,200 tets, 1e9 seeded
+    particles generated on the device in 50M chunks, sorted by the duct-axis
+    locality key, 3.5M injected per step, DH h/8, H_pass 4, warp-aggregated
+    deposit, TMA pipeline, sort every 10 steps keyed at x + 5 dt v): ten
+    steps -- the tenth ends with the periodic sort on the predicted key --
+    then a 20k-particle sample (seeded ids and ids of the first injected
+    batch) against the oracle stepped ten times particle by particle (the
+    steps are independent per particle given the fixed random field), with
+    exact per-step bookkeeping and charge conservation over the whole
+    population.  Particles are selected on the device (the population does
+    not fit a host download)."""
+    torch = pytest.importorskip("torch")
+    if torch.cuda.get_device_properties(0).total_memory < 150e9:
+        pytest.skip("needs a 180 GB B200")
+    import gen.cuda as gc
+    from paper_conf_icpp_lantra0m24_b200.app import MiniFemPic
+    cfg = gen.CONFIGS["c4"]
+    nx, ny, nz = cfg["dims"]
+    n0, n_inj, seed, dt, w, qm = cfg["n0"], cfg["n_inj"], cfg["seed"], 1.0, 1.0, 1.0
+    steps = 10
+    mesh = gen.kuhn_duct(nx, ny, nz)
+    rng = np.random.default_rng(7)
+    ef = rng.uniform(-2e-3, 2e-3, (mesh["n_cells"], 3)) + np.array([0.0, 0.0, 1e-3])
+    dm = gc.DeviceMesh(mesh)
+    sim = MiniFemPic(mesh, ef, capacity=int(n0 * 1.04) + 2 * n_inj + 4096,
+                     stream=torch.cuda.current_stream().cuda_stream, deposit_mode=1,
+                     direct_hop=1, overlay_spacing=0.125, hop_budget=4, sort_every=10,
+                     sort_axis=(0.0, 0.0, 1.0), sort_lead=5.0)
+    chunk = 50_000_000
+    for first in range(0, n0, chunk):
+        init = gc.seed_particles(dm, min(chunk, n0 - first), seed, first=first)
+        sim.inject(init, on_device=True)
+        del init
+    sim.step(0.0, qm, w, stats=False, fill=True)      # builds the mesh data; dt = 0: no motion
+    sim.sort_by_cell()
+    sid = np.union1d(rng.choice(n0, 18_000, replace=False), n0 + rng.choice(n_inj, 2_000, replace=False))
+    before = sim.particles_with_ids(sid)
+    assert before["id"].shape[0] == 18_000
+    b0 = None
+    sts = []
+    for s in range(steps):
+        batch = gc.inject_batch(dm, s, n_inj, seed, id_base=n0)   # ids n0 + s n_inj + k (S21)
+        if s == 0:
+            b0 = {k: batch[k].cpu().numpy() for k in ("pos", "vel", "cell", "id")}
+        sim.inject(batch, on_device=True)
+        del batch
+        sts.append(sim.step(dt, qm, w, stats=True, fill=True))
+    after = sim.particles_with_ids(sid)
+    Q = sim.node_charge_host()
+    n_final = sim.count()
+    sim.close()
+
+    # whole population: bookkeeping per step and charge conservation
+    n = n0
+    for st in sts:
+        assert st["n_before"] == n + n_inj
+        n = st["n_before"] - st["n_removed"]
+        assert st["n_after"] == n
+    assert n_final == n
+    assert abs(Q.sum() - w * n) <= 1e-9 * w * n
+
+    # the sample through the oracle, one particle at a time (multi-hop walk:
+    # the final cell is the containing tet, pin P7)
+    om = oracle.Mesh.from_gen(mesh)
+    om.set_field(ef)
+    P = oracle.Particles()
+    P.append(before["pos"], before["vel"], before["cell"], before["id"])
+    mi = np.isin(b0["id"], sid)
+    Qs = np.zeros(mesh["n_nodes"])
+    excl = set()
+    for s in range(steps):
+        if s == 0:
+            P.append(b0["pos"][mi], b0["vel"][mi], b0["cell"][mi], b0["id"][mi])
+        oracle.step(om, P, qm * dt, dt, w, Qs, use_dh=0)
+        rid, rmg = P.removed()
+        excl |= {i for i, m in zip(rid.tolist(), rmg.tolist()) if m < NEAR}
+    orc = P.get()
+    excl |= set(orc["id"][orc["margin"] < NEAR].tolist())
+    so, sg = set(orc["id"].tolist()), set(after["id"].tolist())
+    assert not ((so ^ sg) - excl), "survivor sets differ"
+    common = np.array(sorted((so & sg) - excl), dtype=np.int64)
+    oo = np.argsort(orc["id"])
+    io = oo[np.searchsorted(orc["id"][oo], common)]
+    ig = np.searchsorted(after["id"], common)
+    assert np.array_equal(orc["cell"][io], after["cell"][ig])
+    ex = np.abs(orc["pos"][io] - after["pos"][ig]) / np.maximum(np.abs(orc["pos"][io]), 1.0)
+    ev = np.abs(orc["vel"][io] - after["vel"][ig]) / np.maximum(np.abs(orc["vel"][io]), 0.25)
+    assert ex.max() <= 1e-12 and ev.max() <= 1e-12
+    assert common.size > 15_000 and len(excl) <= 10
