@@ -67,8 +67,12 @@ enum opp_move_status { OPP_MOVE_DONE = 0, OPP_NEED_MOVE = 1, OPP_NEED_REMOVE = 2
 
 /* Deposit race handling (§3.3 and Fig. 3):
  * ATOMIC        one fp64 atomic add per (particle, node)              ("AT")
- * ATOMIC_WARPAGG same-node contributions of a warp summed by shuffles
- *                before one atomic per distinct node
+ * ATOMIC_WARPAGG same-cell contributions of a warp summed by shuffles
+ *                before one set of 4 atomics per distinct cell, into the
+ *                cell's 4 node slots (32 contiguous bytes); after the
+ *                step's walks every node adds its slots in a fixed order
+ *                (Eq. 10 unchanged: the same w*lambda_i, summed per cell
+ *                first)
  * SORT_SEGRED   store (cell, w*lambda[4]) per particle, counting-sort by
  *                cell, reduce per cell, then per node               ("SR")
  * AUTO          library choice by measurement: ATOMIC_WARPAGG (fastest on
@@ -113,10 +117,11 @@ typedef struct {
                                    (0,0,0) = plain cell-id order                    */
     int deposit_cache;          /* ATOMIC_WARPAGG in the TMA pipeline: 1 = cell sums
                                    accumulate in a per-warp shared-memory cache
-                                   across slices and leave with 4 reductions when
-                                   evicted -- pays under deposit contention
-                                   (clustered particles, config C5), costs
-                                   otherwise; 0 = off (default)     */
+                                   across slices and leave with 4 node reductions
+                                   when evicted (instead of the per-cell node
+                                   slots); measured slower than the default on C2,
+                                   C4 and the clustered C5; 0 = off
+                                   (default)                                        */
     double sort_lead;           /* periodic sort (sort_every > 0) keyed at the
                                    ballistic extrapolation x + sort_lead*dt*v of each
                                    particle (the DH overlay's tet of that point, else

@@ -1087,7 +1087,11 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
         m.ov = ov;
         m.ov_built = true;
     }
-    if (c->p.deposit_mode == OPP_DEP_SORT_SEGRED && !m.sr_cellsum) {
+    // per-cell node-slot sums + the node -> (cell, slot) CSR: the SR deposit,
+    // and the warp-aggregated one (without the deposit cache: StepArgs::cacc)
+    const bool cellsum_mode = c->p.deposit_mode == OPP_DEP_SORT_SEGRED ||
+                              (c->p.deposit_mode == OPP_DEP_ATOMIC_WARPAGG && !c->p.deposit_cache);
+    if (cellsum_mode && !m.sr_cellsum) {
         long long nn = c->sets[c->cols[c2n].to].size;
         const int32_t *h = (const int32_t *)cn.host.data();
         std::vector<int32_t> ptr(nn + 1, 0), idx((size_t)4 * nc);
@@ -1102,6 +1106,7 @@ static int prepare_mesh(opp_ctx c, PSet &ps, int c2c, int c2n, int node_pos, int
             return fail(OPP_ERR_NOMEM, "SR mesh buffers");
         CK(cudaMemcpyAsync(m.n2cs_ptr, ptr.data(), 4 * (nn + 1), cudaMemcpyHostToDevice, c->s));
         CK(cudaMemcpyAsync(m.n2cs, idx.data(), 4 * 4 * nc, cudaMemcpyHostToDevice, c->s));
+        CK(cudaMemsetAsync(m.sr_cellsum, 0, 32 * std::max<long long>(nc, 1), c->s));
         CK(cudaStreamSynchronize(c->s));
     }
     if (c->p.deposit_mode == OPP_DEP_SORT_SEGRED && m.sr_cap < ps.cap) {
@@ -1458,6 +1463,8 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
     a.cell_base = c->cell_base;
     a.n_cells = (int)m.nc;
     a.n_nodes = (int)nn;
+    // warp-aggregated deposit into per-cell node slots, gathered into Q below
+    a.cacc = (c->p.deposit_mode == OPP_DEP_ATOMIC_WARPAGG && !c->p.deposit_cache) ? m.sr_cellsum : nullptr;
     a.hpass = c->p.hop_budget_per_pass;
     a.hcap = c->p.hop_cap;
     a.tile_group = kTileGroup;
@@ -1519,6 +1526,15 @@ extern "C" int opp_push_move_deposit(opp_ctx c, opp_set parts, opp_dat pos, opp_
         CK(launch_sr(a, m.nc, nn, m.cell_hist, m.cell_start, m.tile_sums, m.sr_sorted,
                      m.sr_cellsum, m.n2cs_ptr, m.n2cs, grid_for(c, ps.n_ub, 8), c->s));
         c->launches += 5;
+    }
+    if (a.cacc) {
+        // every walk of the step has deposited: node charge += its slots, then
+        // the slots are cleared for the next step (timed as the deposit's
+        // node-reduction phase, like the SR deposit's last stage)
+        PhaseScope ph(c, OPP_PH_SEGRED);
+        CK(launch_cell_to_nodes(m.n2cs_ptr, m.n2cs, a.cacc, nn, a.Q, c->s));
+        CK(cudaMemsetAsync(a.cacc, 0, 32 * (size_t)m.nc, c->s));
+        c->launches++;
     }
     if (multi && c->comm->halo_n > 0) {
         PhaseScope ph(c, OPP_PH_HALO);

@@ -117,6 +117,8 @@ struct StepArgs {
     int dcache;                // per-warp node-charge cache (opp_init_params.deposit_cache)
     Overlay ov;
     int n_nodes;               // local nodes (bounds of Q; checked builds)
+    double *cacc;              // ATOMIC_WARPAGG: per-cell node-slot sums [4 * n_cells] (zeroed per
+                               // step, gathered into Q after the move); null = reduce into Q
     int32_t *pcell;            // non-null on the step before a sort: the sort-key cell of
                                // every pushed particle (overlay tet of x + lead_dt v, -1 none)
     double lead_dt;

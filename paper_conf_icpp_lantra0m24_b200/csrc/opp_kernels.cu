@@ -252,7 +252,7 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepAr
     unsigned up = peers & ~((2u << lane) - 1u);           // group lanes above me
     if (lane == 31) up = 0;
     int4 cn = make_int4(0, 0, 0, 0);
-    if (lead && !dc) cn = line_c2n(a.lines, key - a.cell_base);
+    if (lead && !dc && !a.cacc) cn = line_c2n(a.lines, key - a.cell_base);
     while (__any_sync(FULL, up != 0)) {
         const int next = up ? __ffs(up) - 1 : (int)lane;
         const double t1 = __shfl_sync(FULL, v1, next);
@@ -273,6 +273,16 @@ __device__ __forceinline__ void deposit_agg(double *__restrict__ Q, const StepAr
     // exactly; C4 pass 1 30.95 -> 30.74 ms)
     if (lead) v0 = sub(mul((double)__popc(peers), a.w), add(add(v1, v2), v3));
     OPP_CHECK(!lead || (unsigned)(key - a.cell_base) < (unsigned)a.n_cells);
+    if (a.cacc && !dc) {
+        // the group's sums go to the cell's 4 node slots (one 32-B sector,
+        // no node-id load); k_sr_node_gather adds each node's slots once the
+        // step's walks are done
+        if (lead) {
+            double *cs = a.cacc + 4ll * (key - a.cell_base);
+            atomicAdd(cs, v0); atomicAdd(cs + 1, v1); atomicAdd(cs + 2, v2); atomicAdd(cs + 3, v3);
+        }
+        return;
+    }
     OPP_CHECK(!lead || dc || ((unsigned)cn.x < (unsigned)a.n_nodes && (unsigned)cn.y < (unsigned)a.n_nodes &&
                               (unsigned)cn.z < (unsigned)a.n_nodes && (unsigned)cn.w < (unsigned)a.n_nodes));
     if (!dc) {
@@ -1972,6 +1982,13 @@ cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long n
     k_overlay_init<<<g1 > 0 ? g1 : 1, 256, 0, s>>>(map, tot);
     k_overlay_build<<<g2 > 0 ? g2 : 1, 256, 0, s>>>(lines, xyz, nc, cell_base, ov, map);
     k_overlay_finish<<<g1 > 0 ? g1 : 1, 256, 0, s>>>(map, tot);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_cell_to_nodes(const int32_t *n2cs_ptr, const int32_t *n2cs, const double *cellsum,
+                                 long long nn, double *Q, cudaStream_t s) {
+    const int gn = (int)((nn + 255) / 256);
+    k_sr_node_gather<<<gn > 0 ? gn : 1, 256, 0, s>>>(n2cs_ptr, n2cs, cellsum, nn, Q);
     return cudaGetLastError();
 }
 

@@ -21,6 +21,9 @@ cudaError_t launch_overlay(const WalkLine *lines, const double *xyz, long long n
                            const Overlay &ov, int32_t *map, cudaStream_t s);
 cudaError_t launch_overlay_compact(const int32_t *map, const Overlay &ov, int16_t *off, int32_t *base,
                                    unsigned *overflow, cudaStream_t s);
+// Q[v] += sum of cellsum[n2cs[k]] over node v's (cell, slot) entries (fixed order)
+cudaError_t launch_cell_to_nodes(const int32_t *n2cs_ptr, const int32_t *n2cs, const double *cellsum,
+                                 long long nn, double *Q, cudaStream_t s);
 cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *hist,
                       unsigned *start, unsigned long long *tile_sums, double *sorted,
                       double *cellsum, const int32_t *n2cs_ptr, const int32_t *n2cs, int grid,
