@@ -727,8 +727,10 @@ class EsRank:
         # capacity: the seeded population + a 4% margin for the flow imbalance
         # between ranks + two steps of injection (injection precedes the push)
         cap = int(n0 * 1.04) + 2 * self.n_inj + 4096
-        if args.empty:   # the population grows by n_inj per step (no outflow before z = 72 h)
-            cap = (total + 2) * self.n_inj + 4096
+        if args.empty:   # the population grows by n_inj per step (no outflow before z = 72 h),
+            # through the timed steps and the e2e leg's
+            ke = 0 if args.no_e2e else (args.e2e_steps or min(args.steps, 10))
+            cap = (total + ke + 2) * self.n_inj + 4096
         self.sim = MiniFemPic(mesh, ef, capacity=cap, stream=stream.cuda_stream, deposit_mode=args.deposit,
                               direct_hop=args.dh, overlay_spacing=args.ov, hop_budget=args.hpass,
                               sort_every=args.sort, tma_pipeline=not args.direct,
