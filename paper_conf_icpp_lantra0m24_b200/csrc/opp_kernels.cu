@@ -1036,24 +1036,52 @@ __global__ void k_step_begin(double *Q, long long nn, DevCounters *c, int zero) 
 // head list; tail slots [N', N) still holding a particle (p2c >= 0) form the
 // tail list; both have the same length.  Move: tail[k] -> head[k].
 // ---------------------------------------------------------------------------
-__global__ void k_fill_plan(const uint32_t *__restrict__ holes, const int32_t *__restrict__ p2c,
-                            DevCounters *c, uint32_t *head, uint32_t *tail) {
+// Block-aggregated append: the block's lanes with `pred` get consecutive
+// slots from ONE global atomic per block (the lists' single counters would
+// otherwise take an atomic per warp); slots follow the lanes' order.
+__device__ __forceinline__ unsigned long long block_append(bool pred, unsigned long long *counter,
+                                                           unsigned *wcnt, unsigned long long *bbase) {
+    const unsigned lane = lane_id(), warp = threadIdx.x >> 5;
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    if (lane == 0) wcnt[warp] = __popc(m);
+    __syncthreads();
+    unsigned before = 0, total = 0;
+    for (unsigned w = 0; w < (blockDim.x >> 5); w++) {
+        const unsigned c = wcnt[w];
+        before += w < warp ? c : 0u;
+        total += c;
+    }
+    if (threadIdx.x == 0) *bbase = total ? atomicAdd(counter, (unsigned long long)total) : 0ull;
+    __syncthreads();
+    const unsigned long long slot = *bbase + before + __popc(m & ((1u << lane) - 1u));
+    __syncthreads();   // wcnt / bbase are reused by the next call
+    return slot;
+}
+
+__global__ void __launch_bounds__(256) k_fill_plan(const uint32_t *__restrict__ holes, const int32_t *__restrict__ p2c,
+                                                   DevCounters *c, uint32_t *head, uint32_t *tail) {
+    __shared__ unsigned wcnt[8];
+    __shared__ unsigned long long bbase;
     const unsigned long long R = c->n_holes, N = c->n, Np = N - R;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    for (unsigned long long k0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-         k0 < R; k0 += stride) {
-        unsigned long long k = k0 + lane_id();
-        bool v = k < R;
-        uint32_t h = v ? holes[k] : 0;
-        bool is_head = v && h < Np;
-        unsigned long long s = warp_append(is_head, &c->n_head);
-        if (is_head) head[s] = h;
-        bool is_tail = v && p2c[Np + k] >= 0;
-        unsigned long long t = warp_append(is_tail, &c->n_tail);
-        if (is_tail) tail[t] = (uint32_t)(Np + k);
+    // block-uniform trip count: every thread of a block takes part in each append
+    for (unsigned long long k0 = (unsigned long long)blockIdx.x * blockDim.x; k0 < R; k0 += stride) {
+        const unsigned long long k = k0 + threadIdx.x;
+        const bool v = k < R;
+        const uint32_t h = v ? holes[k] : 0;
+        const bool is_head = v && h < Np;
+        const bool is_tail = v && p2c[Np + k] >= 0;
+        const unsigned long long hs = block_append(is_head, &c->n_head, wcnt, &bbase);
+        if (is_head) head[hs] = h;
+        const unsigned long long ts = block_append(is_tail, &c->n_tail, wcnt, &bbase);
+        if (is_tail) tail[ts] = (uint32_t)(Np + k);
     }
 }
 
+// Column moves tail[k] -> head[k]: each thread moves kFillU pairs at a time,
+// one component after the other, all loads of a component before its stores
+// (independent requests in flight instead of one load-store chain per value).
+constexpr int kFillU = 4;
 __global__ void k_fill_move(ColSet cols, DevCounters *c, const uint32_t *__restrict__ head,
                             const uint32_t *__restrict__ tail) {
     const unsigned long long m = c->n_head;
@@ -1062,20 +1090,36 @@ __global__ void k_fill_move(ColSet cols, DevCounters *c, const uint32_t *__restr
         c->n = c->n - c->n_holes;
         c->n_holes = 0;
     }
-    for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k < m;
-         k += (unsigned long long)gridDim.x * blockDim.x) {
-        const unsigned long long d = head[k], s = tail[k];
-        OPP_CHECK(d < (unsigned long long)cols.c[0].cap && s < (unsigned long long)cols.c[0].cap);
+    const unsigned long long T = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long k0 = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k0 < m;
+         k0 += T * kFillU) {
+        unsigned long long d[kFillU], s[kFillU];
+#pragma unroll
+        for (int u = 0; u < kFillU; u++) {
+            const unsigned long long k = k0 + (unsigned long long)u * T;
+            d[u] = k < m ? head[k] : ~0ull;
+            s[u] = k < m ? tail[k] : 0ull;
+            OPP_CHECK(d[u] == ~0ull || (d[u] < (unsigned long long)cols.c[0].cap &&
+                                        s[u] < (unsigned long long)cols.c[0].cap));
+        }
         for (int j = 0; j < cols.n; j++) {
             const ColDesc cd = cols.c[j];
             for (int e = 0; e < cd.dim; e++) {
                 const long long off = (long long)e * cd.cap;
                 if (cd.elem_bytes == 8) {
-                    long long *p = reinterpret_cast<long long *>(cd.ptr);
-                    p[off + d] = p[off + s];
+                    long long *p = reinterpret_cast<long long *>(cd.ptr) + off;
+                    long long t[kFillU];
+#pragma unroll
+                    for (int u = 0; u < kFillU; u++) t[u] = d[u] != ~0ull ? p[s[u]] : 0;
+#pragma unroll
+                    for (int u = 0; u < kFillU; u++) if (d[u] != ~0ull) p[d[u]] = t[u];
                 } else {
-                    int *p = reinterpret_cast<int *>(cd.ptr);
-                    p[off + d] = p[off + s];
+                    int *p = reinterpret_cast<int *>(cd.ptr) + off;
+                    int t[kFillU];
+#pragma unroll
+                    for (int u = 0; u < kFillU; u++) t[u] = d[u] != ~0ull ? p[s[u]] : 0;
+#pragma unroll
+                    for (int u = 0; u < kFillU; u++) if (d[u] != ~0ull) p[d[u]] = t[u];
                 }
             }
         }
