@@ -1001,6 +1001,11 @@ def run_ours(args, rank, world, mode):
                      "peak_source": peak_src,
                      "step_frac": b_ps * (value / world) / (peak * 1e9), "step_bytes_per_particle": b_ps},
         "gpu_launches": med["launches"],
+        # the fused kernel's own rate (the slowest rank's pass-1 time, all
+        # ranks' particles; the continuation, fill, sort and comm excluded)
+        "fused_kernel_only": {"value": med["pushed"] / (med["pmd_ms"] / 1e3) if med["pmd_ms"] > 0 else None,
+                              "unit": UNIT, "kernel": "k_push_move_deposit_tiled (pass 1)",
+                              "ms_per_step": med["pmd_ms"] / args.steps},
         "phases_ms_per_step": {k: v[0] / args.steps for k, v in med["phases"].items() if v[1]},
         "walk": {"hops_per_particle_last_step": med["st"]["total_hops"] / max(med["st"]["n_before"], 1),
                  "max_hops_last_step": med["st"]["max_hops"], "hop_capped": med["st"]["n_hop_capped"],
