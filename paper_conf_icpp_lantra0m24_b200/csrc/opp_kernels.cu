@@ -1286,44 +1286,6 @@ __device__ __forceinline__ void run_info(int key, unsigned &heads, int &run_star
     run_len = run_end - run_start + 1;
 }
 
-__global__ void k_sr_hist(const int32_t *__restrict__ sr_cell, const DevCounters *c, unsigned *hist) {
-    const unsigned long long m = c->n;
-    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-         i0 < m; i0 += stride) {
-        const unsigned long long i = i0 + lane_id();
-        const int key = i < m ? sr_cell[i] : -1;
-        unsigned heads;
-        int rs, rl;
-        bool head;
-        run_info(key >= 0 ? key : -2 - (int)lane_id(), heads, rs, rl, head);
-        if (head && key >= 0) atomicAdd(hist + key, (unsigned)rl);
-    }
-}
-
-__global__ void k_sr_scatter(const int32_t *__restrict__ sr_cell, const double *__restrict__ sr_val,
-                             long long cap, const DevCounters *c, unsigned *cursor, double *sorted) {
-    const unsigned long long m = c->n;
-    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
-    for (unsigned long long i0 = (unsigned long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-         i0 < m; i0 += stride) {
-        const unsigned long long i = i0 + lane_id();
-        const int key = i < m ? sr_cell[i] : -1;
-        unsigned heads;
-        int rs, rl;
-        bool head;
-        run_info(key >= 0 ? key : -2 - (int)lane_id(), heads, rs, rl, head);
-        unsigned base = 0;
-        if (head && key >= 0) base = atomicAdd(cursor + key, (unsigned)rl);
-        base = __shfl_sync(0xffffffffu, base, rs);
-        if (key >= 0) {
-            const unsigned long long d = base + (lane_id() - rs);
-            *reinterpret_cast<double4 *>(sorted + 4 * d) =
-                make_double4(sr_val[i], sr_val[cap + i], sr_val[2 * cap + i], sr_val[3 * cap + i]);
-        }
-    }
-}
-
 // per-cell reduce, one warp per cell: cellsum[c][i] = sum over the cell's
 // segment (lanes stride the segment, then a shuffle tree) -- a hot cell of
 // thousands of records (config C5) costs segment / 32 steps, not segment
@@ -1548,6 +1510,66 @@ __global__ void __launch_bounds__(256) k_cell_hist(const int32_t *__restrict__ p
                 tkey[sl] = -1;
                 tcnt[sl] = 0;
             }
+        __syncthreads();
+    }
+}
+
+// SR deposit, scatter (Fig. 3): the records of a chunk
+// of kSortChunk particles are placed per (chunk, cell) group with ONE global
+// cursor atomic per group (runs of equal cells add to the block's shared
+// table; a cell's records keep no particular order -- the per-cell reduce
+// sums them), instead of one atomic per run: hot cells (config C5) no longer
+// serialise every warp on their cursor.
+__global__ void __launch_bounds__(256) k_sr_scatter_blk(const int32_t *__restrict__ sr_cell,
+                                                        const double *__restrict__ sr_val, long long cap,
+                                                        const DevCounters *c, unsigned *cursor, double *sorted) {
+    __shared__ int tkey[kSortSlots];
+    __shared__ unsigned tcnt[kSortSlots];
+    __shared__ unsigned tbase[kSortSlots];
+    const unsigned long long n = c->n;
+    const unsigned lane = lane_id();
+    sort_tab_clear(tkey, tcnt);
+    __syncthreads();
+    for (unsigned long long base = (unsigned long long)blockIdx.x * kSortChunk; base < n;
+         base += (unsigned long long)gridDim.x * kSortChunk) {
+        int key[kSortPer], slot[kSortPer];
+        unsigned off[kSortPer];
+#pragma unroll
+        for (int r = 0; r < kSortPer; r++) {
+            const unsigned long long i = base + r * 256 + threadIdx.x;
+            key[r] = i < n ? __ldcs(sr_cell + i) : -1;
+        }
+#pragma unroll
+        for (int r = 0; r < kSortPer; r++) {
+            unsigned heads;
+            int rs, rl;
+            bool head;
+            run_info(key[r] >= 0 ? key[r] : -2 - (int)lane, heads, rs, rl, head);
+            int sl = -1;
+            unsigned old = 0;
+            if (head && key[r] >= 0) {
+                sl = sort_tab_insert(tkey, tcnt, key[r], (unsigned)rl, old);
+                if (sl < 0) old = atomicAdd(cursor + key[r], (unsigned)rl);   // table full: direct
+            }
+            sl = __shfl_sync(0xffffffffu, sl, rs);
+            old = __shfl_sync(0xffffffffu, old, rs);
+            slot[r] = sl;
+            off[r] = old + (lane - (unsigned)rs);
+        }
+        __syncthreads();
+        for (int sl = threadIdx.x; sl < kSortSlots; sl += blockDim.x)
+            if (tkey[sl] >= 0) tbase[sl] = atomicAdd(cursor + tkey[sl], tcnt[sl]);
+        __syncthreads();
+#pragma unroll
+        for (int r = 0; r < kSortPer; r++) {
+            if (key[r] < 0) continue;
+            const unsigned long long i = base + r * 256 + threadIdx.x;
+            const unsigned long long d = slot[r] >= 0 ? (unsigned long long)tbase[slot[r]] + off[r] : off[r];
+            *reinterpret_cast<double4 *>(sorted + 4 * d) =
+                make_double4(sr_val[i], sr_val[cap + i], sr_val[2 * cap + i], sr_val[3 * cap + i]);
+        }
+        __syncthreads();
+        sort_tab_clear(tkey, tcnt);
         __syncthreads();
     }
 }
@@ -2051,11 +2073,13 @@ cudaError_t launch_sr(const StepArgs &a, long long nc, long long nn, unsigned *h
                       double *cellsum, const int32_t *n2cs_ptr, const int32_t *n2cs, int grid,
                       cudaStream_t s) {
     cudaMemsetAsync(hist, 0, sizeof(unsigned) * (nc + 1), s);
-    k_sr_hist<<<grid, 256, 0, s>>>(a.sr_cell, a.cnt, hist);
+    // records hold local cells (-1: none): the block-aggregated histogram of
+    // the sort by cell, keyed by the record's cell
+    k_cell_hist<<<grid, 256, 0, s>>>(a.sr_cell, nullptr, nc, a.cnt, 0, nullptr, hist);
     cudaError_t e = scan_exclusive(hist, start, nc + 1, tile_sums, s);
     if (e != cudaSuccess) return e;
     cudaMemcpyAsync(hist, start, sizeof(unsigned) * (nc + 1), cudaMemcpyDeviceToDevice, s);
-    k_sr_scatter<<<grid, 256, 0, s>>>(a.sr_cell, a.sr_val, a.cap, a.cnt, hist, sorted);
+    k_sr_scatter_blk<<<grid, 256, 0, s>>>(a.sr_cell, a.sr_val, a.cap, a.cnt, hist, sorted);
     int gc = (int)std::min<long long>((nc + 7) / 8, 148 * 16), gn = (int)((nn + 255) / 256);
     k_sr_cell_reduce<<<gc > 0 ? gc : 1, 256, 0, s>>>(start, sorted, nc, cellsum);
     k_sr_node_gather<<<gn > 0 ? gn : 1, 256, 0, s>>>(n2cs_ptr, n2cs, cellsum, nn, a.Q);
