@@ -1041,7 +1041,9 @@ def run_ours(args, rank, world, mode):
                        "h2d_bytes_per_step": e["h2d"], "d2h_bytes_per_step": e["d2h"],
                        "steps": e["steps"], "note": "injection arrays from pinned host memory (opp_inject "
                        "on_device=0, H2D overlapped with the previous step on the library's copy "
-                       "stream) + node charge read back every step (opp_get_node_charge)"}
+                       "stream) + node charge read back every step (opp_get_node_charge); the same run "
+                       "continued after the timed repetitions (its later steps: a population thinned by "
+                       "the side walls, C4 ~0.1% per step), its own sort steps included"}
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1), one pinned core
     if not args.no_cpu and world == 1:
         n_sample = 4_000_000 if args.config != "c1" else cfg["n0"]
