@@ -80,6 +80,26 @@ def test_loopback_multi_slab_crossing_and_sort():
 
 
 @pytest.mark.parametrize("R", [2, 3])
+def test_loopback_dh_cell_slots_predicted_sort(R):
+    """Slabs with DH seeding (each rank's overlay over its own slab), the
+    warp-aggregated deposit into per-cell node slots gathered before the
+    halo, and the periodic sort keyed at the predicted cell (sort_lead; the
+    recorded keys of migrants fall back to their cell): the merged result
+    equals the single-domain oracle (multi-hop walk there: same final cells,
+    pin P7; near-face particles excluded as everywhere)."""
+    mesh, ef, init, inject, steps = c1_case(drift=0.4, spread=0.1)
+    om, orc, Qo, ost, rem = run_oracle(mesh, ef, init, inject, steps, QM * DT, DT, W)
+    parts, Qg, stats = _run_ranks(mesh, ef, init, inject, steps, R, deposit_mode=1, direct_hop=1,
+                                  overlay_spacing=0.25, sort_every=2, sort_lead=1.5,
+                                  sort_axis=(0.0, 0.0, 1.0))
+    compare(om, mesh["c2n"], orc, Qo, rem, parts, Qg, W)
+    for s in range(steps):
+        assert sum(st[s]["n_after"] for st in stats) == ost[s]["n_after"]
+        assert sum(st[s]["n_removed"] for st in stats) == ost[s]["n_removed"]
+    assert sum(st[s]["n_migrated_out"] for st in stats for s in range(steps)) > 1000
+
+
+@pytest.mark.parametrize("R", [2, 3])
 def test_loopback_field_solve_equals_single_domain(R):
     """Slab-partitioned CG (host-driven, node halo + cross-rank dots) on R
     contexts: the merged potential equals the single-domain direct solve
