@@ -11,10 +11,11 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-@pytest.mark.parametrize("config", ["c4", "c2", "c3"])
+@pytest.mark.parametrize("config", ["c4", "c2", "c3", "c2-empty"])
 def test_reference_arm_json_line(config):
-    out = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--config", config,
-                          "--steps", "1", "--warmup", "0"], cwd=ROOT, capture_output=True,
+    extra = ["--empty"] if config.endswith("-empty") else []
+    out = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--config", config.split("-")[0],
+                          "--steps", "1", "--warmup", "0"] + extra, cwd=ROOT, capture_output=True,
                          text=True, timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]
     lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
